@@ -1,0 +1,149 @@
+"""ctypes harness of the CPU oracle (liboracle.so).
+
+TEST INFRASTRUCTURE ONLY: imported by tests/, __graft_entry__.smoke() and
+bench.py's cpu_baseline / --impl reference legs -- never by the product
+package.  See oracle/ve_oracle.h for what the oracle computes and where each
+definition comes from.
+"""
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB = None
+
+MAX_TOPK = 64
+LINE_EMPTY, LINE_POINT, LINE_LINE, LINE_FAIL = 0, 1, 2, 3
+DIFF_WRITTEN, DIFF_ALL, DIFF_MASK = 0, 1, 2
+TYPE_NAMES = ["u8", "u16", "u32", "u64", "i8", "i16", "i32", "i64", "f16", "f32", "f64", "bf16"]
+
+SUM_FIELDS = ["n_ld", "n_st", "n_zero", "n_ld_eq_pre", "n_st_eq_pre", "n_nosnap"]
+FLAG_SUM_FIELDS = ["n_nan", "n_nonint", "n_not_f16", "n_not_bf16", "n_not_f32"]
+MINMAX_FIELDS = ["raw_min", "raw_max", "ord_min", "ord_max", "trunc_min", "trunc_max"]
+DERIVED_FIELDS = ["single_value", "single_zero", "frequent", "structured", "approx", "dict8", "heavy",
+                  "single_type"]
+
+KEY_DTYPE = np.dtype(
+    [(f, "<u8") for f in SUM_FIELDS] + [("n_type", "<u8", (12,))] + [(f, "<u8") for f in FLAG_SUM_FIELDS]
+    + [(f, "<u8") for f in MINMAX_FIELDS]
+    + [("line_state", "<u8"), ("p_x", "<u8"), ("p_ylo", "<u8"), ("p_yhi", "<i8"), ("q_x", "<u8"),
+       ("q_ylo", "<u8"), ("q_yhi", "<i8")]
+    + [("n_distinct", "<u8"), ("n_top", "<u8"), ("top_bits", "<u8", (MAX_TOPK,)),
+       ("top_count", "<u8", (MAX_TOPK,))]
+    + [(f, "<u4") for f in DERIVED_FIELDS])
+GLOB_DTYPE = np.dtype([("n_records", "<u8"), ("n_invalid", "<u8"), ("n_unmapped", "<u8"), ("u_touched", "<u8")])
+OBJSTAT_DTYPE = np.dtype([("n_elems", "<u8"), ("n_written", "<u8"), ("n_loaded_eq", "<u8"),
+                          ("n_ld_reload", "<u8"), ("n_touched", "<u8")])
+DIFF_DTYPE = np.dtype([("n_elems", "<u8"), ("n_masked", "<u8"), ("n_unchanged", "<u8"), ("n_changed", "<u8"),
+                       ("n_untouched", "<u8"), ("redundant", "<u4"), ("pad", "<u4")])
+
+
+class VoObject(ctypes.Structure):
+    _fields_ = [("base", ctypes.c_uint64), ("size", ctypes.c_uint64), ("pre", ctypes.c_void_p),
+                ("post", ctypes.c_void_p), ("id", ctypes.c_uint32), ("elem_width", ctypes.c_uint32)]
+
+
+class VoConfig(ctypes.Structure):
+    _fields_ = [("n_pcs", ctypes.c_uint32), ("topk", ctypes.c_uint32), ("mant_bits", ctypes.c_uint32),
+                ("t_redundant_pct", ctypes.c_uint32), ("t_frequent_pct", ctypes.c_uint32),
+                ("pad", ctypes.c_uint32)]
+
+
+def lib():
+    global _LIB
+    if _LIB is None:
+        path = os.path.join(_HERE, "liboracle.so")
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} missing: run __graft_entry__.build()")
+        L = ctypes.CDLL(path)
+        vp, u32, u64 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64
+        L.vo_analyze.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
+        L.vo_snapshot_diff.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, u32, u32, vp, vp]
+        L.vo_object_dedup.argtypes = [vp, u32, vp]
+        L.vo_ord.argtypes = [u64, u32, u32]
+        L.vo_ord.restype = u64
+        L.vo_float_flags.argtypes = [u64, u32, u32]
+        L.vo_float_flags.restype = u32
+        L.vo_trunc.argtypes = [u64, u32, u32, u32]
+        L.vo_trunc.restype = u64
+        L.vo_sizeof.argtypes = [ctypes.c_int]
+        L.vo_sizeof.restype = u64
+        for which, dt in enumerate([KEY_DTYPE, GLOB_DTYPE, OBJSTAT_DTYPE, DIFF_DTYPE]):
+            assert L.vo_sizeof(which) == dt.itemsize, (which, L.vo_sizeof(which), dt.itemsize)
+        assert L.vo_sizeof(4) == ctypes.sizeof(VoObject)
+        _LIB = L
+    return _LIB
+
+
+def make_config(n_pcs, topk=8, mant_bits=7, t_redundant_pct=33, t_frequent_pct=33):
+    return VoConfig(n_pcs, topk, mant_bits, t_redundant_pct, t_frequent_pct, 0)
+
+
+def _objects(objs):
+    """objs: list of dicts {base, size, id, elem_width, pre (np.uint8 or None), post}."""
+    arr = (VoObject * max(len(objs), 1))()
+    keep = []
+    for i, o in enumerate(objs):
+        pre, post = o.get("pre"), o.get("post")
+        for a in (pre, post):
+            if a is not None:
+                assert a.dtype == np.uint8 and a.flags.c_contiguous and len(a) >= o["size"]
+                keep.append(a)
+        arr[i] = VoObject(o["base"], o["size"], pre.ctypes.data if pre is not None else None,
+                          post.ctypes.data if post is not None else None, o["id"], o["elem_width"])
+    return arr, keep
+
+
+def analyze(cfg, objs, recs):
+    """Returns (keys[n_pcs + n_obj + 1], globals, objstat[n_obj]) as numpy structured arrays."""
+    recs = np.ascontiguousarray(recs)
+    assert recs.dtype.itemsize == 24
+    arr, _keep = _objects(objs)
+    n_keys = cfg.n_pcs + len(objs) + 1
+    keys = np.zeros(n_keys, dtype=KEY_DTYPE)
+    glob = np.zeros(1, dtype=GLOB_DTYPE)
+    objstat = np.zeros(max(len(objs), 1), dtype=OBJSTAT_DTYPE)
+    rc = lib().vo_analyze(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), keys.ctypes.data,
+                          glob.ctypes.data, objstat.ctypes.data)
+    if rc != 0:
+        raise ValueError("vo_analyze rejected its arguments")
+    return keys, glob[0], objstat[:len(objs)]
+
+
+def snapshot_diff(cfg, objs, recs, obj_id, mode=DIFF_WRITTEN, mask=None):
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    out = np.zeros(1, dtype=DIFF_DTYPE)
+    m = None
+    if mask is not None:
+        m = np.ascontiguousarray(mask, dtype=np.uint32)
+    rc = lib().vo_snapshot_diff(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), obj_id, mode,
+                                m.ctypes.data if m is not None else None, out.ctypes.data)
+    if rc != 0:
+        raise ValueError("vo_snapshot_diff rejected its arguments")
+    return out[0]
+
+
+def object_dedup(objs):
+    arr, _keep = _objects(objs)
+    g = np.zeros(max(len(objs), 1), dtype=np.uint32)
+    lib().vo_object_dedup(arr, len(objs), g.ctypes.data)
+    return g[:len(objs)]
+
+
+def y_of(lo, hi):
+    """signed 128-bit y of a line endpoint from its (lo, hi) halves"""
+    return (int(hi) << 64) | int(lo)
+
+
+def ord_key(b, kind, w):
+    return lib().vo_ord(b, kind, w)
+
+
+def float_flags(b, kind, w):
+    return lib().vo_float_flags(b, kind, w)
+
+
+def trunc(b, kind, w, K):
+    return lib().vo_trunc(b, kind, w, K)

@@ -1,0 +1,590 @@
+/*
+ * ve_oracle.c -- CPU ORACLE (test infrastructure only; see ve_oracle.h).
+ *
+ * Plain C11 + gcc extensions (__int128, _Float16, __bf16).  Single-threaded.
+ * Each function cites the passage it follows.  P:L<n> = PAPER.md line n;
+ * "C<k>" / "Q<k>" = the definition / reading in SURVEY.md 8(c), restated in
+ * DESIGN.md section 3.
+ *
+ * Nothing here is blocked, fused or reordered: records are visited in array
+ * order, histograms are "sort + run-length", the line fit visits every point
+ * against the extreme-x pair, snapshots are compared with memcmp.
+ */
+#include "ve_oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+typedef __int128 i128;
+
+/* ---- record decoding (SURVEY 8(b) ve_record.meta) --------- */
+
+static uint32_t rec_w(uint32_t meta) { return 1u << (meta & 3u); }
+static uint32_t rec_kind(uint32_t meta) { return (meta >> 2) & 3u; }
+static int rec_store(uint32_t meta) { return (meta >> 4) & 1u; }
+static int rec_shared(uint32_t meta) { return (meta >> 5) & 1u; }
+
+/* Validity rules of SURVEY 8(b) "Invalid records are data, not errors". */
+static int rec_valid(const vo_record* r, uint32_t n_pcs) {
+  uint32_t w = rec_w(r->meta), kind = rec_kind(r->meta);
+  if (r->meta >> 6) return 0;
+  if (kind == 2 && w == 1) return 0;
+  if (kind == 3 && w != 2) return 0;
+  if (r->pc >= n_pcs) return 0;
+  if (w < 8 && (r->value >> (8 * w)) != 0) return 0;
+  if (r->addr >= (1ull << 48)) return 0;
+  return 1;
+}
+
+/* Type code order u8 u16 u32 u64 i8 i16 i32 i64 f16 f32 f64 bf16 (C1). */
+static uint32_t type_code(uint32_t kind, uint32_t w) {
+  uint32_t lg = (w == 1) ? 0 : (w == 2) ? 1 : (w == 4) ? 2 : 3;
+  if (kind == 0) return lg;
+  if (kind == 1) return 4 + lg;
+  if (kind == 3) return 11;
+  return (w == 2) ? 8 : (w == 4) ? 9 : 10;
+}
+
+static uint32_t tc_width(uint32_t tc) {
+  static const uint32_t wid[12] = {1, 2, 4, 8, 1, 2, 4, 8, 2, 4, 8, 2};
+  return wid[tc];
+}
+
+/* Exact value of a float record, through the compiler's own conversions
+ * (an independent path from the GPU's bit manipulation). */
+static double float_value(uint64_t b, uint32_t kind, uint32_t w) {
+  if (kind == 3) {                     /* bfloat16 = top half of a binary32 */
+    uint32_t u = (uint32_t)b << 16;
+    float f;
+    memcpy(&f, &u, 4);
+    return (double)f;
+  }
+  if (w == 2) {
+    uint16_t u = (uint16_t)b;
+    _Float16 h;
+    memcpy(&h, &u, 2);
+    return (double)h;
+  }
+  if (w == 4) {
+    uint32_t u = (uint32_t)b;
+    float f;
+    memcpy(&f, &u, 4);
+    return (double)f;
+  }
+  double d;
+  memcpy(&d, &b, 8);
+  return d;
+}
+
+static int64_t sext(uint64_t b, uint32_t w) {
+  if (w == 8) return (int64_t)b;
+  uint32_t sh = 64 - 8 * w;
+  return (int64_t)(b << sh) >> sh;
+}
+
+/* C5: orderable key.  uint -> b; sint -> sext(b) XOR 2^63;
+ * float -> sign set ? ~b & mask_w : b | signbit_w. */
+uint64_t vo_ord(uint64_t b, uint32_t kind, uint32_t w) {
+  if (kind == 0) return b;
+  if (kind == 1) return (uint64_t)sext(b, w) ^ (1ull << 63);
+  uint64_t mask = (w == 8) ? ~0ull : ((1ull << (8 * w)) - 1);
+  uint64_t sign = 1ull << (8 * w - 1);
+  return (b & sign) ? (~b & mask) : (b | sign);
+}
+
+/* C5 float flags: bit0 NaN, bit1 nonint, bit2 not_f16, bit3 not_bf16,
+ * bit4 not_f32 (f64 sources only).  "not_X" = the round trip through X
+ * (round-to-nearest-even) is not the identity; NaNs fail all of them. */
+uint32_t vo_float_flags(uint64_t b, uint32_t kind, uint32_t w) {
+  if (kind < 2) return 0;
+  double v = float_value(b, kind, w);
+  int is_f64 = (kind == 2 && w == 8);
+  if (isnan(v)) return 1u | 2u | 4u | 8u | (is_f64 ? 16u : 0u);
+  uint32_t f = 0;
+  /* nonint: +-Inf, non-integral, -0.0, or |v| >= 2^63 (C5; Q11) */
+  if (isinf(v) || v != trunc(v) || (v == 0.0 && signbit(v)) || fabs(v) >= 9223372036854775808.0)
+    f |= 2u;
+  if ((double)(_Float16)v != v) f |= 4u;
+  if ((double)(__bf16)v != v) f |= 8u;
+  if (is_f64 && (double)(float)v != v) f |= 16u;
+  return f;
+}
+
+/* C7: clear the low (m-K) mantissa bits; m = 10/7/23/52 (Def 3.8; Q6). */
+uint64_t vo_trunc(uint64_t b, uint32_t kind, uint32_t w, uint32_t K) {
+  uint32_t m = (kind == 3) ? 7 : (w == 2) ? 10 : (w == 4) ? 23 : 52;
+  if (K >= m) return b;
+  return b & ~((1ull << (m - K)) - 1);
+}
+
+/* ---- object table (start address + size per object) ------------ */
+
+typedef struct {
+  const vo_object** by_base;
+  uint32_t n;
+} objtab;
+
+static int cmp_obj_base(const void* a, const void* b) {
+  const vo_object* x = *(const vo_object* const*)a;
+  const vo_object* y = *(const vo_object* const*)b;
+  return (x->base > y->base) - (x->base < y->base);
+}
+
+static int objtab_build(objtab* t, const vo_object* objs, uint32_t n) {
+  t->n = n;
+  t->by_base = (const vo_object**)malloc(sizeof(*t->by_base) * (n ? n : 1));
+  char* seen = (char*)calloc(n ? n : 1, 1);
+  for (uint32_t i = 0; i < n; ++i) {
+    const vo_object* o = &objs[i];
+    uint32_t ew = o->elem_width;
+    if (o->size == 0 || o->id >= n || seen[o->id] || !(ew == 1 || ew == 2 || ew == 4 || ew == 8) ||
+        o->base >= (1ull << 48) || o->size > (1ull << 48) - o->base) {
+      free(seen);
+      free(t->by_base);
+      return -1;
+    }
+    seen[o->id] = 1;
+    t->by_base[i] = o;
+  }
+  free(seen);
+  qsort(t->by_base, n, sizeof(*t->by_base), cmp_obj_base);
+  for (uint32_t i = 1; i < n; ++i)
+    if (t->by_base[i - 1]->base + t->by_base[i - 1]->size > t->by_base[i]->base) {
+      free(t->by_base);
+      return -1;
+    }
+  return 0;
+}
+
+/* The object containing addr (first byte), or NULL. */
+static const vo_object* objtab_find(const objtab* t, uint64_t addr) {
+  uint32_t lo = 0, hi = t->n;          /* first object with base > addr */
+  while (lo < hi) {
+    uint32_t mid = lo + (hi - lo) / 2;
+    if (t->by_base[mid]->base <= addr) lo = mid + 1; else hi = mid;
+  }
+  if (lo == 0) return NULL;
+  const vo_object* o = t->by_base[lo - 1];
+  return (addr - o->base < o->size) ? o : NULL;
+}
+
+static uint64_t n_elems_of(const vo_object* o) {
+  return (o->size + o->elem_width - 1) / o->elem_width;
+}
+
+/* ---- one decoded record ------------------------------------------------- */
+
+typedef struct {
+  int valid, store, shared;
+  uint32_t w, kind, tc, fflags;
+  const vo_object* obj;     /* mapped object (global space) */
+  int inside;               /* [addr, addr+w) inside obj */
+  int eq_defined, eq_pre;   /* C2 */
+} dec_t;
+
+static void decode(const vo_config* cfg, const objtab* t, const vo_record* r, dec_t* d) {
+  memset(d, 0, sizeof(*d));
+  d->valid = rec_valid(r, cfg->n_pcs);
+  if (!d->valid) return;
+  d->w = rec_w(r->meta);
+  d->kind = rec_kind(r->meta);
+  d->store = rec_store(r->meta);
+  d->shared = rec_shared(r->meta);
+  d->tc = type_code(d->kind, d->w);
+  d->fflags = vo_float_flags(r->value, d->kind, d->w);
+  if (d->shared) return;                                  /* Q20: no snapshot */
+  d->obj = objtab_find(t, r->addr);
+  if (!d->obj) return;
+  uint64_t off = r->addr - d->obj->base;
+  d->inside = (off + d->w <= d->obj->size);               /* Q21 */
+  if (d->inside && d->obj->pre) {
+    d->eq_defined = 1;
+    int eq = 1;                                           /* C2: little-endian bytes */
+    for (uint32_t i = 0; i < d->w; ++i)
+      if (d->obj->pre[off + i] != (uint8_t)(r->value >> (8 * i))) eq = 0;
+    d->eq_pre = eq;
+  }
+}
+
+/* ---- histogram entries for C9 ------------------------------------------ */
+
+typedef struct { uint64_t key, bits, count; } hent;
+
+static int cmp_key_bits(const void* a, const void* b) {
+  const hent* x = (const hent*)a;
+  const hent* y = (const hent*)b;
+  if (x->key != y->key) return x->key < y->key ? -1 : 1;
+  if (x->bits != y->bits) return x->bits < y->bits ? -1 : 1;
+  return 0;
+}
+
+/* (key asc, count desc, bits asc): the top-k order of C9 / Q18 */
+static int cmp_key_count_bits(const void* a, const void* b) {
+  const hent* x = (const hent*)a;
+  const hent* y = (const hent*)b;
+  if (x->key != y->key) return x->key < y->key ? -1 : 1;
+  if (x->count != y->count) return x->count > y->count ? -1 : 1;
+  if (x->bits != y->bits) return x->bits < y->bits ? -1 : 1;
+  return 0;
+}
+
+/* ---- line fit (C8, Def 3.7) ---------------------------------- */
+
+typedef struct {
+  int have, fail;
+  uint64_t px, qx;
+  i128 py, qy;
+} line_acc;
+
+/* y of a record for the structured check; returns 0 if the record FAILs it */
+static int point_y(uint64_t b, uint32_t kind, uint32_t w, uint32_t fflags, i128* y) {
+  if (kind == 0) { *y = (i128)b; return 1; }
+  if (kind == 1) { *y = (i128)sext(b, w); return 1; }
+  if (fflags & 2u) return 0;                               /* nonint float => FAIL */
+  *y = (i128)(int64_t)float_value(b, kind, w);
+  return 1;
+}
+
+static int collinear(i128 px, i128 py, i128 qx, i128 qy, i128 x, i128 y) {
+  return (y - py) * (qx - px) == (qy - py) * (x - px);
+}
+
+/* ---- C6 heavy type (report-time) --------------------------------------- */
+
+static double ord_to_double(uint64_t ord, uint32_t kind, uint32_t w) {
+  uint64_t mask = (w == 8) ? ~0ull : ((1ull << (8 * w)) - 1);
+  uint64_t sign = 1ull << (8 * w - 1);
+  uint64_t b = (ord & sign) ? (ord & ~sign) : (~ord & mask);
+  return float_value(b, kind, w);
+}
+
+static uint32_t heavy_type(const vo_key* k, uint32_t tc) {
+  uint32_t w = tc_width(tc);
+  static const uint32_t cand_w[3] = {1, 2, 4};
+  if (tc <= 3) {                                           /* uint source */
+    for (int i = 0; i < 3; ++i) {
+      uint32_t v = cand_w[i];
+      if (v >= w) break;
+      if (k->ord_max <= ((1ull << (8 * v)) - 1)) return (v == 1) ? 0 : (v == 2) ? 1 : 2;
+    }
+    return 255;
+  }
+  if (tc <= 7) {                                           /* sint source */
+    int64_t mn = (int64_t)(k->ord_min ^ (1ull << 63));
+    int64_t mx = (int64_t)(k->ord_max ^ (1ull << 63));
+    for (int i = 0; i < 3; ++i) {
+      uint32_t v = cand_w[i];
+      if (v >= w) break;
+      int64_t lo = -(1ll << (8 * v - 1)), hi = (1ll << (8 * v - 1)) - 1;
+      if (mn >= lo && mx <= hi) return (v == 1) ? 4 : (v == 2) ? 5 : 6;
+    }
+    return 255;
+  }
+  /* float source: integer candidates by exact range when every value is
+   * integral, then the float formats by exact round trip (C6, Q10) */
+  uint32_t kind = (tc == 11) ? 3 : 2;
+  double mn = ord_to_double(k->ord_min, kind, w), mx = ord_to_double(k->ord_max, kind, w);
+  for (int i = 0; i < 3; ++i) {
+    uint32_t v = cand_w[i];
+    if (v >= w) break;
+    if (k->n_nonint == 0) {
+      if (mn >= 0) {
+        if (mx <= (double)((1ull << (8 * v)) - 1)) return (v == 1) ? 0 : (v == 2) ? 1 : 2;
+      } else {
+        double lo = -(double)(1ull << (8 * v - 1)), hi = (double)(1ull << (8 * v - 1)) - 1;
+        if (mn >= lo && mx <= hi) return (v == 1) ? 4 : (v == 2) ? 5 : 6;
+      }
+    }
+    if (v == 2 && k->n_not_f16 == 0) return 8;
+    if (v == 2 && k->n_not_bf16 == 0) return 11;
+    if (v == 4 && k->n_not_f32 == 0) return 9;
+  }
+  return 255;
+}
+
+static void derive_flags(const vo_config* cfg, vo_key* k) {
+  uint64_t n = k->n_ld + k->n_st;
+  uint32_t nt = 0, tc = 0;
+  for (uint32_t t = 0; t < 12; ++t)
+    if (k->n_type[t]) { ++nt; tc = t; }
+  k->single_type = (nt == 1);
+  k->single_value = (n > 0 && k->raw_min == k->raw_max);                  /* Def 3.4 */
+  k->single_zero = (n > 0 && k->n_zero == n);                             /* Def 3.5 */
+  k->frequent = (k->n_top > 0 &&                                          /* Def 3.3 */
+                 (unsigned __int128)100 * k->top_count[0] > (unsigned __int128)cfg->t_frequent_pct * n);
+  k->structured = 0; k->approx = 0; k->dict8 = 0; k->heavy = 255;
+  if (!k->single_type) return;                                            /* Q15 */
+  int is_float = (tc >= 8);
+  i128 py = (i128)(((unsigned __int128)(uint64_t)k->p_yhi << 64) | k->p_ylo);
+  i128 qy = (i128)(((unsigned __int128)(uint64_t)k->q_yhi << 64) | k->q_ylo);
+  k->structured = (k->line_state == VO_LINE_LINE && py != qy);            /* Def 3.7 */
+  k->approx = (is_float && k->n_nan == 0 && n > 0 && k->trunc_min == k->trunc_max &&
+               !k->single_value);                                          /* Def 3.8 */
+  k->dict8 = (k->n_distinct <= 256 && tc_width(tc) > 1);
+  k->heavy = heavy_type(k, tc);                                            /* Def 3.6 */
+}
+
+/* ---- vo_analyze: C1-C9 per key, C3 per object --------------------------- */
+
+int vo_analyze(const vo_config* cfg, const vo_object* objs, uint32_t n_obj,
+               const vo_record* recs, uint64_t n,
+               vo_key* keys, vo_globals* glob, vo_objstat* objstat) {
+  if (!cfg || cfg->topk > VO_MAX_TOPK || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t n_keys = (uint64_t)cfg->n_pcs + n_obj + 1;
+  const uint64_t key_shared = (uint64_t)cfg->n_pcs + n_obj;
+
+  memset(keys, 0, sizeof(vo_key) * n_keys);
+  for (uint64_t k = 0; k < n_keys; ++k) {
+    keys[k].raw_min = keys[k].ord_min = keys[k].trunc_min = ~0ull;
+  }
+  memset(glob, 0, sizeof(*glob));
+
+  /* per-object element marks: W (written), L (eq_pre loads), U (eq-defined refs) */
+  unsigned char** Wm = (unsigned char**)calloc(n_obj ? n_obj : 1, sizeof(*Wm));
+  unsigned char** Lm = (unsigned char**)calloc(n_obj ? n_obj : 1, sizeof(*Lm));
+  unsigned char** Um = (unsigned char**)calloc(n_obj ? n_obj : 1, sizeof(*Um));
+  for (uint32_t i = 0; i < n_obj; ++i) {
+    uint64_t ne = n_elems_of(&objs[i]);
+    Wm[objs[i].id] = (unsigned char*)calloc(ne, 1);
+    Lm[objs[i].id] = (unsigned char*)calloc(ne, 1);
+    Um[objs[i].id] = (unsigned char*)calloc(ne, 1);
+  }
+
+  hent* pairs = (hent*)malloc(sizeof(hent) * (2 * n + 1));
+  uint64_t n_pairs = 0;
+  line_acc* la = (line_acc*)calloc(n_keys, sizeof(line_acc));
+
+  glob->n_records = n;
+  /* pass 1: sums, min/max, histogram pairs, extreme-x points */
+  for (uint64_t i = 0; i < n; ++i) {
+    const vo_record* r = &recs[i];
+    dec_t d;
+    decode(cfg, &t, r, &d);
+    if (!d.valid) { glob->n_invalid++; continue; }
+    if (!d.shared && !d.obj) glob->n_unmapped++;
+
+    uint64_t kset[2];
+    int nk = 0;
+    kset[nk++] = r->pc;                                    /* PC key */
+    if (d.shared) kset[nk++] = key_shared;                 /* Q20 */
+    else if (d.obj) kset[nk++] = (uint64_t)cfg->n_pcs + d.obj->id;
+
+    uint64_t ord = vo_ord(r->value, d.kind, d.w);
+    int is_nan = (d.fflags & 1u) != 0;
+    for (int j = 0; j < nk; ++j) {
+      vo_key* k = &keys[kset[j]];
+      if (d.store) k->n_st++; else k->n_ld++;
+      if (r->value == 0) k->n_zero++;                      /* Q8: bitwise zero */
+      if (d.eq_defined) {
+        if (d.eq_pre) { if (d.store) k->n_st_eq_pre++; else k->n_ld_eq_pre++; }
+      } else {
+        k->n_nosnap++;
+      }
+      k->n_type[d.tc]++;
+      if (d.kind >= 2) {
+        if (d.fflags & 1u) k->n_nan++;
+        if (d.fflags & 2u) k->n_nonint++;
+        if (d.fflags & 4u) k->n_not_f16++;
+        if (d.fflags & 8u) k->n_not_bf16++;
+        if (d.fflags & 16u) k->n_not_f32++;
+      }
+      if (r->value < k->raw_min) k->raw_min = r->value;
+      if (r->value > k->raw_max) k->raw_max = r->value;
+      if (!is_nan) {
+        if (ord < k->ord_min) k->ord_min = ord;
+        if (ord > k->ord_max) k->ord_max = ord;
+      }
+      if (d.kind >= 2 && !is_nan) {
+        uint64_t tb = vo_trunc(r->value, d.kind, d.w, cfg->mant_bits);
+        if (tb < k->trunc_min) k->trunc_min = tb;
+        if (tb > k->trunc_max) k->trunc_max = tb;
+      }
+      pairs[n_pairs].key = kset[j];
+      pairs[n_pairs].bits = r->value;
+      pairs[n_pairs].count = 1;
+      n_pairs++;
+
+      line_acc* L = &la[kset[j]];
+      i128 y;
+      if (!point_y(r->value, d.kind, d.w, d.fflags, &y)) { L->fail = 1; continue; }
+      if (!L->have) {
+        L->have = 1; L->px = L->qx = r->addr; L->py = L->qy = y;
+      } else {
+        if (r->addr < L->px) { L->px = r->addr; L->py = y; }
+        if (r->addr > L->qx) { L->qx = r->addr; L->qy = y; }
+      }
+    }
+
+    /* per-object marks (C3, C10) */
+    if (d.obj && d.inside) {
+      const vo_object* o = d.obj;
+      uint64_t off = r->addr - o->base;
+      uint64_t e0 = off / o->elem_width, e1 = (off + d.w - 1) / o->elem_width;
+      if (d.store)
+        for (uint64_t e = e0; e <= e1; ++e) Wm[o->id][e] = 1;
+      if (!d.store && d.eq_pre) Lm[o->id][e0] = 1;
+      if (d.eq_defined)
+        for (uint64_t e = e0; e <= e1; ++e) Um[o->id][e] = 1;
+    }
+  }
+
+  /* pass 2: every point against the extreme-x pair (C8) */
+  for (uint64_t i = 0; i < n; ++i) {
+    const vo_record* r = &recs[i];
+    dec_t d;
+    decode(cfg, &t, r, &d);
+    if (!d.valid) continue;
+    uint64_t kset[2];
+    int nk = 0;
+    kset[nk++] = r->pc;
+    if (d.shared) kset[nk++] = key_shared;
+    else if (d.obj) kset[nk++] = (uint64_t)cfg->n_pcs + d.obj->id;
+    for (int j = 0; j < nk; ++j) {
+      line_acc* L = &la[kset[j]];
+      if (L->fail) continue;
+      i128 y;
+      if (!point_y(r->value, d.kind, d.w, d.fflags, &y)) { L->fail = 1; continue; }
+      if (L->px == L->qx) {
+        if (y != L->py) L->fail = 1;               /* same x, different y */
+      } else if (!collinear((i128)L->px, L->py, (i128)L->qx, L->qy, (i128)r->addr, y)) {
+        L->fail = 1;
+      }
+    }
+  }
+  for (uint64_t k = 0; k < n_keys; ++k) {
+    line_acc* L = &la[k];
+    vo_key* K = &keys[k];
+    if (L->fail) K->line_state = VO_LINE_FAIL;
+    else if (!L->have) K->line_state = VO_LINE_EMPTY;
+    else {
+      K->line_state = (L->px == L->qx) ? VO_LINE_POINT : VO_LINE_LINE;
+      K->p_x = L->px; K->q_x = L->qx;
+      K->p_ylo = (uint64_t)L->py; K->p_yhi = (int64_t)(L->py >> 64);
+      K->q_ylo = (uint64_t)L->qy; K->q_yhi = (int64_t)(L->qy >> 64);
+    }
+  }
+  free(la);
+
+  /* C9: exact histogram = sort (key, bits) + run-length, then top-k by
+   * (count desc, bits asc) */
+  qsort(pairs, n_pairs, sizeof(hent), cmp_key_bits);
+  uint64_t n_runs = 0;
+  for (uint64_t i = 0; i < n_pairs;) {
+    uint64_t j = i;
+    while (j < n_pairs && pairs[j].key == pairs[i].key && pairs[j].bits == pairs[i].bits) ++j;
+    pairs[n_runs].key = pairs[i].key;
+    pairs[n_runs].bits = pairs[i].bits;
+    pairs[n_runs].count = j - i;
+    ++n_runs;
+    i = j;
+  }
+  qsort(pairs, n_runs, sizeof(hent), cmp_key_count_bits);
+  for (uint64_t i = 0; i < n_runs; ++i) {
+    vo_key* K = &keys[pairs[i].key];
+    if (K->n_distinct < cfg->topk) {
+      K->top_bits[K->n_distinct] = pairs[i].bits;
+      K->top_count[K->n_distinct] = pairs[i].count;
+      K->n_top = K->n_distinct + 1;
+    }
+    K->n_distinct++;
+  }
+  free(pairs);
+
+  for (uint64_t k = 0; k < n_keys; ++k) derive_flags(cfg, &keys[k]);
+
+  /* C3 per object, and U */
+  for (uint32_t i = 0; i < n_obj; ++i) {
+    uint32_t id = objs[i].id;
+    uint64_t ne = n_elems_of(&objs[i]);
+    vo_objstat* s = &objstat[id];
+    memset(s, 0, sizeof(*s));
+    s->n_elems = ne;
+    for (uint64_t e = 0; e < ne; ++e) {
+      s->n_written += Wm[id][e];
+      s->n_loaded_eq += Lm[id][e];
+      s->n_touched += (Wm[id][e] | Lm[id][e]);
+      glob->u_touched += Um[id][e];
+    }
+    s->n_ld_reload = keys[(uint64_t)cfg->n_pcs + id].n_ld_eq_pre - s->n_loaded_eq;
+    free(Wm[id]); free(Lm[id]); free(Um[id]);
+  }
+  free(Wm); free(Lm); free(Um);
+  free(t.by_base);
+  return 0;
+}
+
+/* ---- C10: snapshot diff (Def 3.1; footnote P:L267) */
+
+int vo_snapshot_diff(const vo_config* cfg, const vo_object* objs, uint32_t n_obj,
+                     const vo_record* recs, uint64_t n, uint32_t obj_id,
+                     uint32_t mode, const uint32_t* mask, vo_diff* out) {
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const vo_object* o = NULL;
+  for (uint32_t i = 0; i < n_obj; ++i) if (objs[i].id == obj_id) o = &objs[i];
+  if (!o || !o->pre || !o->post || mode > VO_DIFF_MASK || (mode == VO_DIFF_MASK && !mask)) {
+    free(t.by_base);
+    return -1;
+  }
+  uint64_t ne = n_elems_of(o);
+  unsigned char* W = (unsigned char*)calloc(ne, 1);
+  unsigned char* L = (unsigned char*)calloc(ne, 1);
+  for (uint64_t i = 0; i < n; ++i) {
+    dec_t d;
+    decode(cfg, &t, &recs[i], &d);
+    if (!d.valid || d.obj != o || !d.inside) continue;
+    uint64_t off = recs[i].addr - o->base;
+    uint64_t e0 = off / o->elem_width, e1 = (off + d.w - 1) / o->elem_width;
+    if (d.store) for (uint64_t e = e0; e <= e1; ++e) W[e] = 1;
+    if (!d.store && d.eq_pre) L[e0] = 1;
+  }
+  memset(out, 0, sizeof(*out));
+  out->n_elems = ne;
+  uint64_t touched = 0;
+  for (uint64_t e = 0; e < ne; ++e) {
+    int m = (mode == VO_DIFF_ALL) ? 1 : (mode == VO_DIFF_WRITTEN) ? W[e] : (int)((mask[e / 32] >> (e % 32)) & 1u);
+    touched += (W[e] | L[e]);
+    if (!m) continue;
+    out->n_masked++;
+    uint64_t b0 = e * o->elem_width;
+    uint64_t len = (b0 + o->elem_width <= o->size) ? o->elem_width : o->size - b0;
+    if (memcmp(o->pre + b0, o->post + b0, len) == 0) out->n_unchanged++;
+  }
+  out->n_changed = out->n_masked - out->n_unchanged;
+  out->n_untouched = ne - touched;
+  out->redundant = (out->n_masked > 0 &&
+                    (unsigned __int128)100 * out->n_unchanged >
+                        (unsigned __int128)cfg->t_redundant_pct * out->n_masked);
+  free(W); free(L); free(t.by_base);
+  return 0;
+}
+
+/* ---- C11: duplicate objects (Def 3.2; Q17) --------------- */
+
+int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of) {
+  for (uint32_t i = 0; i < n; ++i) {
+    group_of[i] = objs[i].id;
+    if (objs[i].size == 0 || !objs[i].post) continue;
+    for (uint32_t j = 0; j < n; ++j) {
+      if (objs[j].size != objs[i].size || !objs[j].post) continue;
+      if (objs[j].id < group_of[i] && memcmp(objs[i].post, objs[j].post, objs[i].size) == 0)
+        group_of[i] = objs[j].id;
+    }
+  }
+  return 0;
+}
+
+/* struct sizes, for the ctypes harness to check its mirrors */
+uint64_t vo_sizeof(int which) {
+  switch (which) {
+    case 0: return sizeof(vo_key);
+    case 1: return sizeof(vo_globals);
+    case 2: return sizeof(vo_objstat);
+    case 3: return sizeof(vo_diff);
+    case 4: return sizeof(vo_object);
+    default: return sizeof(vo_record);
+  }
+}

@@ -1,0 +1,128 @@
+/*
+ * ve_oracle.h -- CPU ORACLE for the ValueExpert value-trace analysis.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load liboracle.so.
+ * The product library (libve.so) never includes, links or calls this code,
+ * and this code includes nothing from the product tree.
+ *
+ * A plain, slow, single-threaded implementation of the definitions of
+ * SURVEY.md 8(c) C1-C12, which restate PAPER.md Defs 3.1-3.8
+ * (section 3) and section 5.1.
+ * Every statistic is an order-free function of the record multiset plus the
+ * snapshots, so the oracle computes each definition directly (sort +
+ * run-length for histograms, two passes over the points for the exact line
+ * fit, bytewise memcmp for snapshots).  Readings of ambiguous passages are
+ * listed in DESIGN.md section 3 (Q1-Q23).
+ *
+ * Parity pins: see tests/test_oracle_pins.py (paper worked examples
+ * P1-P14, closed forms of cfg1, brute force B1-B5, invariants I1-I10).
+ * Every function below is pinned; none is "parity unpinned".
+ *
+ * The record / object byte layouts are the only thing shared with the product
+ * ABI (include/ve.h); they are re-declared here, not included.
+ */
+#ifndef VE_ORACLE_H
+#define VE_ORACLE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct vo_record {       /* 24 bytes: same byte layout as ve_record */
+  uint64_t addr;
+  uint64_t value;
+  uint32_t pc;
+  uint32_t meta;
+} vo_record;
+
+typedef struct vo_object {       /* host-memory snapshots */
+  uint64_t base, size;
+  const uint8_t* pre;            /* NULL = no pre snapshot  */
+  const uint8_t* post;           /* NULL = no post snapshot */
+  uint32_t id;                   /* dense 0..n-1 */
+  uint32_t elem_width;           /* 1,2,4,8 */
+} vo_object;
+
+typedef struct vo_config {
+  uint32_t n_pcs;
+  uint32_t topk;                 /* <= 64 */
+  uint32_t mant_bits;            /* K */
+  uint32_t t_redundant_pct;
+  uint32_t t_frequent_pct;
+  uint32_t pad;
+} vo_config;
+
+#define VO_MAX_TOPK 64
+
+/* line states (C8) */
+enum { VO_LINE_EMPTY = 0, VO_LINE_POINT = 1, VO_LINE_LINE = 2, VO_LINE_FAIL = 3 };
+
+/* per-key statistics; key index: PCs [0,n_pcs), objects n_pcs+id, SHARED n_pcs+n_obj */
+typedef struct vo_key {
+  /* C1, C2, C5 sums */
+  uint64_t n_ld, n_st, n_zero, n_ld_eq_pre, n_st_eq_pre, n_nosnap;
+  uint64_t n_type[12];
+  uint64_t n_nan, n_nonint, n_not_f16, n_not_bf16, n_not_f32;
+  /* C4, C5, C7 min/max (identity values when no contributor: min=~0, max=0) */
+  uint64_t raw_min, raw_max, ord_min, ord_max, trunc_min, trunc_max;
+  /* C8 line state; y is a signed 128-bit integer split in (lo, hi) */
+  uint64_t line_state;
+  uint64_t p_x, p_ylo; int64_t p_yhi;
+  uint64_t q_x, q_ylo; int64_t q_yhi;
+  /* C9 */
+  uint64_t n_distinct;
+  uint64_t n_top;
+  uint64_t top_bits[VO_MAX_TOPK];
+  uint64_t top_count[VO_MAX_TOPK];
+  /* derived flags (report-time, from the fields above) */
+  uint32_t single_value, single_zero, frequent, structured, approx, dict8;
+  uint32_t heavy;                /* type code 0..11 of the narrowest type, 255 = none */
+  uint32_t single_type;          /* 1 iff exactly one n_type bin is non-zero */
+} vo_key;
+
+typedef struct vo_globals {
+  uint64_t n_records, n_invalid, n_unmapped;
+  uint64_t u_touched;            /* U of SURVEY 8(d): distinct pre elements referenced with eq_pre defined */
+} vo_globals;
+
+typedef struct vo_objstat {
+  uint64_t n_elems;
+  uint64_t n_written;            /* |W| */
+  uint64_t n_loaded_eq;          /* |L| */
+  uint64_t n_ld_reload;          /* C3 */
+  uint64_t n_touched;            /* |W u L| */
+} vo_objstat;
+
+typedef struct vo_diff {
+  uint64_t n_elems, n_masked, n_unchanged, n_changed, n_untouched;
+  uint32_t redundant, pad;
+} vo_diff;
+
+enum { VO_DIFF_WRITTEN = 0, VO_DIFF_ALL = 1, VO_DIFF_MASK = 2 };
+
+/* Analyze records (C1-C9, C3); keys has n_pcs + n_obj + 1 entries, objstat n_obj.
+ * Returns 0 on success, -1 on invalid arguments. */
+int vo_analyze(const vo_config* cfg, const vo_object* objs, uint32_t n_obj,
+               const vo_record* recs, uint64_t n,
+               vo_key* keys, vo_globals* glob, vo_objstat* objstat);
+
+/* C10: snapshot diff of object obj_id (mask bit e in word e/32, LSB first). */
+int vo_snapshot_diff(const vo_config* cfg, const vo_object* objs, uint32_t n_obj,
+                     const vo_record* recs, uint64_t n, uint32_t obj_id,
+                     uint32_t mode, const uint32_t* mask, vo_diff* out);
+
+/* C11: duplicate objects; group_of[i] = min id of i's class. */
+int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of);
+
+/* helpers exposed for pinning */
+uint64_t vo_ord(uint64_t b, uint32_t kind, uint32_t w);
+uint32_t vo_float_flags(uint64_t b, uint32_t kind, uint32_t w);   /* bit0 nan, 1 nonint, 2 not_f16, 3 not_bf16, 4 not_f32 */
+uint64_t vo_trunc(uint64_t b, uint32_t kind, uint32_t w, uint32_t K);
+uint64_t vo_sizeof(int which);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
