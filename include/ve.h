@@ -1,0 +1,182 @@
+/*
+ * ve.h -- C ABI of libve.so: B200-native ValueExpert value-trace analysis.
+ *
+ * The boundary of the hot path of Zhou et al., "ValueExpert: Exploring Value
+ * Patterns in GPU-Accelerated Applications", ASPLOS '22.  Citations
+ * P:L<n> are PAPER.md line numbers; C<k>/Q<k> are the definitions / readings
+ * restated in DESIGN.md section 3.
+ *
+ * Conventions for every call:
+ *   - All integers little-endian.  No C++ types cross the ABI.
+ *   - Pointers named d_* are DEVICE pointers (caller-owned, on the ctx's
+ *     device, valid until the work queued on the stream completes; the library
+ *     never writes or frees them).  Pointers named h_* or plain arrays are HOST
+ *     memory, copied before the call returns unless stated otherwise.
+ *   - Every call returns ve_status; nothing throws or aborts across the ABI.
+ *     ve_last_error(ctx) describes the last failure (cudaGetErrorString for
+ *     CUDA errors).  Asynchronous kernel faults surface at the next
+ *     synchronising call (ve_snapshot_diff, ve_object_dedup, ve_report).
+ *   - A ctx is bound to one CUDA device and is not thread-safe.
+ */
+#ifndef VE_H
+#define VE_H
+#include <stdint.h>
+#include <cuda_runtime_api.h>   /* cudaStream_t only */
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* One value-trace record: the (PC, address, size, raw value) the paper's
+ * collector emits per thread per memory instruction, plus the access
+ * type its offline analyzer derives.  24 bytes, alignment 8,
+ * arrays are AoS.  Vector accesses (STG.64 = 2 x f32) are split by the
+ * producer into one record per value at consecutive addresses (Q16). */
+typedef struct ve_record {
+  uint64_t addr;   /* effective byte address; >= 2^48 => invalid record            */
+  uint64_t value;  /* raw bits of ONE value, zero-extended from w bytes; bits >= 8w */
+                   /* must be 0 (else invalid)                                      */
+  uint32_t pc;     /* dense PC id; >= cfg.n_pcs => invalid                          */
+  uint32_t meta;   /* [1:0] log2 w (w in 1,2,4,8)                                   */
+                   /* [3:2] kind: 0 uint, 1 sint, 2 IEEE float (w 2/4/8), 3 bf16 (w 2) */
+                   /* [4] store   [5] shared space   [31:6] must be 0               */
+} ve_record;
+
+/* A data object: address range + pre/post snapshots of one GPU API. */
+typedef struct ve_object {
+  uint64_t base, size;     /* [base, base+size), size > 0, base+size <= 2^48, no overlaps */
+  const void* pre;         /* device ptr: snapshot before the API (size bytes) or NULL     */
+  const void* post;        /* device ptr: snapshot after the API (size bytes) or NULL      */
+  uint32_t id;             /* dense: the n objects of one call carry ids 0..n-1            */
+  uint32_t elem_width;     /* 1,2,4,8: granularity of bitmaps and of the diff (Q4)         */
+} ve_object;
+
+typedef struct ve_config {
+  uint32_t n_pcs;           /* 1..65535                                                   */
+  uint32_t max_objects;     /* <= 65534; SHARED pseudo-object key = n_pcs + n_objects     */
+  uint32_t topk;            /* 1..64, default 8 (Q18)                                     */
+  uint32_t mant_bits;       /* K of Def 3.8, default 7 (Q6)                               */
+  uint32_t t_redundant_pct; /* default 33 (footnote P:L267)                               */
+  uint32_t t_frequent_pct;  /* default 33 (Q2)                                            */
+  uint64_t hist_capacity;   /* exact value-histogram slots (rounded up to 2^k); overflow  */
+                            /* => VE_ERR_CAPACITY, never silently wrong stats              */
+} ve_config;
+
+typedef enum {
+  VE_OK = 0, VE_ERR_INVALID = 1, VE_ERR_CUDA = 2, VE_ERR_NOMEM = 3,
+  VE_ERR_CAPACITY = 4, VE_ERR_NCCL = 5, VE_ERR_STATE = 6
+} ve_status;
+
+enum { VE_DIFF_WRITTEN = 0, VE_DIFF_ALL = 1, VE_DIFF_MASK = 2 };
+enum { VE_LINE_EMPTY = 0, VE_LINE_POINT = 1, VE_LINE_LINE = 2, VE_LINE_FAIL = 3 };
+
+typedef struct ve_ctx ve_ctx;
+typedef struct ve_rep ve_rep;         /* host report, library-owned */
+
+/* C10 result of ve_snapshot_diff. */
+typedef struct ve_diff {
+  uint64_t n_elems, n_masked, n_unchanged, n_changed, n_untouched;
+  uint32_t redundant;      /* n_masked > 0 && 100*n_unchanged > t_redundant_pct*n_masked */
+  uint32_t pad;
+} ve_diff;
+
+/* Per-key statistics (key index: PCs [0,n_pcs), object id -> n_pcs+id, SHARED
+ * n_pcs+n_objects).  Raw fields are the parity target; derived flags are
+ * recomputed from them. */
+typedef struct ve_key_stats {
+  uint64_t n_ld, n_st, n_zero, n_ld_eq_pre, n_st_eq_pre, n_nosnap;     /* C1, C2 */
+  uint64_t n_type[12];          /* u8 u16 u32 u64 i8 i16 i32 i64 f16 f32 f64 bf16  */
+  uint64_t n_nan, n_nonint, n_not_f16, n_not_bf16, n_not_f32;          /* C5 */
+  uint64_t raw_min, raw_max, ord_min, ord_max, trunc_min, trunc_max;   /* C4 C5 C7 */
+  uint64_t line_state;          /* VE_LINE_*                                  C8 */
+  uint64_t p_x, p_ylo; int64_t p_yhi;   /* min-x end point, y as signed 128 bit */
+  uint64_t q_x, q_ylo; int64_t q_yhi;   /* max-x end point                      */
+  uint64_t n_distinct, n_top;   /* C9 */
+  uint32_t single_value, single_zero, frequent, structured, approx, dict8;
+  uint32_t heavy;               /* type code of the narrowest type, 255 = none (C6) */
+  uint32_t single_type;
+} ve_key_stats;
+
+typedef struct ve_topk_entry { uint64_t bits, count; } ve_topk_entry;
+
+typedef struct ve_obj_stats {
+  uint64_t n_elems, n_written, n_loaded_eq, n_ld_reload, n_touched;    /* C3, C10 */
+} ve_obj_stats;
+
+typedef struct ve_globals {
+  uint64_t n_records, n_invalid, n_unmapped;
+  uint64_t hist_entries;        /* occupied (pc, object, value) histogram slots */
+} ve_globals;
+
+/* ---- lifecycle ----------------------------------------------------------- */
+ve_status   ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out);
+ve_status   ve_destroy(ve_ctx* ctx);
+const char* ve_last_error(const ve_ctx* ctx);   /* valid until the next call on ctx */
+/* Host array of n objects (device snapshot pointers) is copied, sorted and
+ * validated (VE_ERR_INVALID on overlap, bad id/size/width); resets all stats. */
+ve_status   ve_set_objects(ve_ctx* ctx, const ve_object* objs, uint32_t n);
+ve_status   ve_reset(ve_ctx* ctx);              /* zero all statistics, clear poison */
+
+/* ---- the five hot-path calls --------------------------------------------- */
+
+/* S1-S9: analyze n device records (C1-C9, C3 bitmaps), accumulating into the
+ * ctx; may be called repeatedly on chunks of one trace (the paper's buffer
+ * flushes).  d_records must be 8-byte aligned.  Asynchronous
+ * on s.  VE_ERR_STATE if the ctx is poisoned (histogram overflow). */
+ve_status ve_analyze_records(ve_ctx* ctx, const ve_record* d_records, uint64_t n, cudaStream_t s);
+
+/* End-to-end variant: records in HOST memory (pinned or pageable), streamed to
+ * the device in chunks through a double-buffered staging area and analyzed
+ * (the paper's collector->analyzer buffer path).  Returns after the
+ * last chunk is queued; h_records must stay valid until s completes. */
+ve_status ve_analyze_records_host(ve_ctx* ctx, const ve_record* h_records, uint64_t n, cudaStream_t s);
+
+/* S10 / C10 (Def 3.1): compare pre and post of object
+ * obj_id element-wise over the mask: W (written elements, VE_DIFF_WRITTEN),
+ * all elements (VE_DIFF_ALL) or the caller's device bitmap d_mask (bit e in
+ * word e/32, LSB first, VE_DIFF_MASK).  Needs both snapshots.  Synchronizes s;
+ * writes *h_out. */
+ve_status ve_snapshot_diff(ve_ctx* ctx, uint32_t obj_id, uint32_t mode, const uint32_t* d_mask,
+                           ve_diff* h_out, cudaStream_t s);
+
+/* S11 / C11 (Def 3.2): duplicate objects among the n given
+ * objects (their post snapshots; ids need not be dense here).  Content hash
+ * as a filter, byte verification for every grouping.  h_group_of[i] = min id
+ * of object i's class (its own id if size 0 or post NULL).  Synchronizes s. */
+ve_status ve_object_dedup(ve_ctx* ctx, const ve_object* objs, uint32_t n, uint32_t* h_group_of,
+                          cudaStream_t s);
+
+/* S12 / C12: merge statistics.  src != NULL: dst <- dst (+) src on one device
+ * (same config and object table).  nccl_comm != NULL (an ncclComm_t over all
+ * ranks, each holding a ctx with the same config/objects): every rank ends
+ * with the merged statistics of all ranks (sum/min/max allreduce, line-state
+ * allgather + monoid merge, bitmap allgather + OR, exact histogram by hash
+ * partition all-to-all + top-k re-rank).  Synchronizes s. */
+ve_status ve_merge_stats(ve_ctx* dst, const ve_ctx* src_or_null, void* nccl_comm_or_null, cudaStream_t s);
+
+/* S13: finalize (top-k, distinct counts, bitmap popcounts, derived flags) and
+ * copy to a library-owned host report.  Synchronizes the ctx's streams.
+ * VE_ERR_STATE if poisoned. */
+ve_status ve_report(ve_ctx* ctx, ve_rep** h_out);
+void      ve_report_free(ve_rep* r);
+
+/* report accessors (host memory, caller-allocated arrays) */
+uint32_t  ve_report_n_keys(const ve_rep* r);
+uint32_t  ve_report_n_objects(const ve_rep* r);
+uint32_t  ve_report_topk(const ve_rep* r);
+ve_status ve_report_keys(const ve_rep* r, ve_key_stats* out);          /* n_keys entries         */
+ve_status ve_report_topk_entries(const ve_rep* r, ve_topk_entry* out); /* n_keys * topk entries  */
+ve_status ve_report_objects(const ve_rep* r, ve_obj_stats* out);       /* n_objects entries      */
+ve_status ve_report_globals(const ve_rep* r, ve_globals* out);
+/* format 0: binary (magic "VERP", header, then the arrays above); 1: JSON */
+ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
+
+/* NCCL helpers (NCCL is loaded at run time; only ve_merge_stats with a comm needs it) */
+ve_status ve_nccl_get_unique_id(void* out128);                          /* 128-byte ncclUniqueId */
+ve_status ve_nccl_comm_init(void** comm_out, int nranks, const void* id128, int rank);
+ve_status ve_nccl_comm_destroy(void* comm);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* VE_H */

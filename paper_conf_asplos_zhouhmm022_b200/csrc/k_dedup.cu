@@ -1,0 +1,175 @@
+// k_dedup.cu -- K7 / K8: duplicate objects (C11).
+//
+// Def 3.2: objects D1, D2 with the same values.  The paper groups
+// SHA256 digests of the post snapshots; here a chunk-parallel,
+// order-free 64-bit content hash (sum over 8-byte words of a position-keyed
+// mix, so any reduction order gives the same value) only FILTERS candidates:
+// every class is then byte-verified against its representative (K8), so a hash
+// collision can never produce a false duplicate ("no false positives").
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <map>
+#include <vector>
+
+#include "ve_internal.cuh"
+
+namespace ve {
+
+__device__ __forceinline__ uint64_t word_mix(uint64_t w, uint64_t j) {
+  return mix64(w ^ (j * 0x9E3779B97F4A7C15ull) ^ 0x5851F42D4C957F2Dull) + j;
+}
+
+struct HashJob {
+  const uint8_t* p;
+  uint64_t size;
+};
+
+// K7: blockIdx.y = object, grid-stride over its 16-byte words; +tail bytes
+__global__ void __launch_bounds__(256) k_hash(const HashJob* jobs, unsigned long long* hash) {
+  const HashJob jb = jobs[blockIdx.y];
+  unsigned long long acc = 0;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  if (((uintptr_t)jb.p & 15) == 0) {
+    const uint64_t nv = jb.size / 16;
+    const uint4* v = (const uint4*)jb.p;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nv; i += stride) {
+      const uint4 x = __ldcs(v + i);
+      acc += word_mix(((uint64_t)x.y << 32) | x.x, 2 * i) + word_mix(((uint64_t)x.w << 32) | x.z, 2 * i + 1);
+    }
+    // tail: remaining words (incl. a zero-padded partial word)
+    const uint64_t done = nv * 16;
+    for (uint64_t j = done / 8 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j * 8 < jb.size; j += stride) {
+      uint64_t w = 0;
+      for (uint64_t b = 0; b < 8 && j * 8 + b < jb.size; ++b) w |= (uint64_t)jb.p[j * 8 + b] << (8 * b);
+      acc += word_mix(w, j);
+    }
+  } else {
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j * 8 < jb.size; j += stride) {
+      uint64_t w = 0;
+      for (uint64_t b = 0; b < 8 && j * 8 + b < jb.size; ++b) w |= (uint64_t)jb.p[j * 8 + b] << (8 * b);
+      acc += word_mix(w, j);
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xFFFFFFFFu, acc, o);
+  if ((threadIdx.x & 31) == 0) atomicAdd(&hash[blockIdx.y], acc);
+}
+
+struct CmpJob {
+  const uint8_t* a;
+  const uint8_t* b;
+  uint64_t off, len;   // byte range of this chunk
+  uint32_t pair;
+  uint32_t pad;
+};
+
+// K8: bytewise verification of (member, representative) pairs, 64 KiB per CTA
+__global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned int* differs) {
+  const CmpJob jb = jobs[blockIdx.x];
+  if (*(volatile unsigned int*)&differs[jb.pair]) return;
+  bool diff = false;
+  const uint8_t* a = jb.a + jb.off;
+  const uint8_t* b = jb.b + jb.off;
+  if ((((uintptr_t)a | (uintptr_t)b) & 15) == 0) {
+    const uint64_t nv = jb.len / 16;
+    for (uint64_t i = threadIdx.x; i < nv; i += blockDim.x) {
+      const uint4 x = __ldcs((const uint4*)a + i), y = __ldcs((const uint4*)b + i);
+      diff |= (x.x != y.x) | (x.y != y.y) | (x.z != y.z) | (x.w != y.w);
+    }
+    for (uint64_t k = nv * 16 + threadIdx.x; k < jb.len; k += blockDim.x) diff |= a[k] != b[k];
+  } else {
+    for (uint64_t k = threadIdx.x; k < jb.len; k += blockDim.x) diff |= a[k] != b[k];
+  }
+  if (__syncthreads_or(diff) && threadIdx.x == 0) atomicOr(&differs[jb.pair], 1u);
+}
+
+ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* group_of, cudaStream_t s) {
+  for (uint32_t i = 0; i < n; ++i) group_of[i] = objs[i].id;
+  std::vector<uint32_t> elig;
+  for (uint32_t i = 0; i < n; ++i)
+    if (objs[i].size > 0 && objs[i].post) elig.push_back(i);
+  if (elig.size() < 2) return VE_OK;
+  // K7: content hash of every eligible object
+  std::vector<HashJob> hj(elig.size());
+  uint64_t maxsz = 0;
+  for (size_t k = 0; k < elig.size(); ++k) {
+    hj[k] = HashJob{(const uint8_t*)objs[elig[k]].post, objs[elig[k]].size};
+    maxsz = std::max<uint64_t>(maxsz, objs[elig[k]].size);
+  }
+  void* d = nullptr;
+  const size_t nb = hj.size() * (sizeof(HashJob) + 8);
+  cudaError_t e = cudaMallocAsync(&d, nb, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dedup alloc");
+  HashJob* d_jobs = (HashJob*)d;
+  unsigned long long* d_hash = (unsigned long long*)((uint8_t*)d + hj.size() * sizeof(HashJob));
+  cudaMemcpyAsync(d_jobs, hj.data(), hj.size() * sizeof(HashJob), cudaMemcpyHostToDevice, s);
+  cudaMemsetAsync(d_hash, 0, hj.size() * 8, s);
+  // grid.x sized so the largest object gets ~8 KiB per CTA-iteration, capped
+  uint64_t gx = (maxsz / 16 + 255) / 256;
+  gx = std::min<uint64_t>(std::max<uint64_t>(gx / 4, 1), 1024);
+  for (size_t y0 = 0; y0 < hj.size(); y0 += 65535) {
+    const unsigned gy = (unsigned)std::min<size_t>(65535, hj.size() - y0);
+    k_hash<<<dim3((unsigned)gx, gy), 256, 0, s>>>(d_jobs + y0, d_hash + y0);
+  }
+  std::vector<unsigned long long> h(hj.size());
+  cudaMemcpyAsync(h.data(), d_hash, hj.size() * 8, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dedup hash");
+
+  // candidate groups: equal (size, hash); members ordered by id
+  std::map<std::pair<uint64_t, uint64_t>, std::vector<uint32_t>> groups;
+  for (size_t k = 0; k < elig.size(); ++k) groups[{objs[elig[k]].size, h[k]}].push_back(elig[k]);
+  std::vector<std::vector<uint32_t>> pending;
+  for (auto& g : groups) {
+    if (g.second.size() < 2) continue;
+    std::sort(g.second.begin(), g.second.end(), [&](uint32_t a, uint32_t b) { return objs[a].id < objs[b].id; });
+    pending.push_back(g.second);
+  }
+  // K8: verify against the representative (lowest id); mismatches form a new pending group
+  const uint64_t CH = 1 << 16;
+  while (!pending.empty()) {
+    std::vector<CmpJob> jobs;
+    std::vector<std::pair<uint32_t, uint32_t>> pairs;  // (group index, member index)
+    for (uint32_t gi = 0; gi < pending.size(); ++gi) {
+      const auto& g = pending[gi];
+      const ve_object& rep = objs[g[0]];
+      for (uint32_t mi = 1; mi < g.size(); ++mi) {
+        const ve_object& m = objs[g[mi]];
+        const uint32_t pid = (uint32_t)pairs.size();
+        pairs.push_back({gi, mi});
+        for (uint64_t off = 0; off < m.size; off += CH)
+          jobs.push_back(CmpJob{(const uint8_t*)m.post, (const uint8_t*)rep.post, off, std::min(CH, m.size - off), pid, 0});
+      }
+    }
+    void* dd = nullptr;
+    e = cudaMallocAsync(&dd, jobs.size() * sizeof(CmpJob) + pairs.size() * 4, s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "dedup verify alloc");
+    CmpJob* d_cj = (CmpJob*)dd;
+    unsigned int* d_diff = (unsigned int*)((uint8_t*)dd + jobs.size() * sizeof(CmpJob));
+    cudaMemcpyAsync(d_cj, jobs.data(), jobs.size() * sizeof(CmpJob), cudaMemcpyHostToDevice, s);
+    cudaMemsetAsync(d_diff, 0, pairs.size() * 4, s);
+    for (size_t j0 = 0; j0 < jobs.size(); j0 += (1u << 30)) {
+      const unsigned gxx = (unsigned)std::min<size_t>(jobs.size() - j0, 1u << 30);
+      k_compare<<<gxx, 256, 0, s>>>(d_cj + j0, d_diff);
+    }
+    std::vector<unsigned int> diff(pairs.size());
+    cudaMemcpyAsync(diff.data(), d_diff, pairs.size() * 4, cudaMemcpyDeviceToHost, s);
+    cudaFreeAsync(dd, s);
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "dedup verify");
+    std::vector<std::vector<uint32_t>> next(pending.size());
+    for (size_t p = 0; p < pairs.size(); ++p) {
+      const auto& g = pending[pairs[p].first];
+      const uint32_t mem = g[pairs[p].second];
+      if (!diff[p]) group_of[mem] = objs[g[0]].id;
+      else next[pairs[p].first].push_back(mem);
+    }
+    pending.clear();
+    for (auto& g : next)
+      if (g.size() >= 2) pending.push_back(g);
+  }
+  return VE_OK;
+}
+
+}  // namespace ve

@@ -1,0 +1,162 @@
+// k_diff.cu -- K5: snapshot diff (C10).
+//
+// Def 3.1 and section 5.1: compare the pre and post value
+// snapshots of an object element by element, restricted to the addresses the
+// API wrote (the written-element bitmap W) or to all elements or a
+// caller mask.  HBM-bound: each warp streams 512 contiguous bytes of pre and
+// of post per instruction (128-bit coalesced loads, 4 in flight per thread),
+// compares per element, and counts masked / unchanged elements with popcounts.
+#include <cuda_runtime.h>
+
+#include <vector>
+
+#include "ve_internal.cuh"
+
+namespace ve {
+
+// per-16-byte equality bits of its 16/ew elements, LSB = first element
+__device__ __forceinline__ uint32_t eq_bits16(const uint4& a, const uint4& b, uint32_t ew_lg) {
+  const uint32_t x[4] = {a.x ^ b.x, a.y ^ b.y, a.z ^ b.z, a.w ^ b.w};
+  uint32_t r = 0;
+  if (ew_lg == 3) {
+    r = ((x[0] | x[1]) == 0) | (((x[2] | x[3]) == 0) << 1);
+  } else if (ew_lg == 2) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) r |= (uint32_t)(x[i] == 0) << i;
+  } else if (ew_lg == 1) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+      r |= ((uint32_t)((x[i] & 0xFFFFu) == 0) | ((uint32_t)((x[i] >> 16) == 0) << 1)) << (2 * i);
+  } else {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const uint32_t z = __vcmpeq4(x[i], 0u);  // 0xFF per equal byte
+      r |= (((z >> 0) & 1u) | ((z >> 7) & 2u) | ((z >> 14) & 4u) | ((z >> 21) & 8u)) << (4 * i);
+    }
+  }
+  return r;
+}
+
+// vector part: bytes [0, nvec*16) of 16-byte aligned pre/post
+__global__ void __launch_bounds__(256) k_diff_vec(const uint4* __restrict__ pre, const uint4* __restrict__ post,
+                                                  uint64_t nvec, uint32_t ew_lg, const uint32_t* __restrict__ mask,
+                                                  unsigned long long* out /* [2] masked, unchanged */) {
+  const uint32_t per = 16u >> ew_lg;  // elements per 16 bytes
+  unsigned long long cm = 0, cu = 0;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  constexpr int U = 4;
+  for (; i + (U - 1) * stride < nvec; i += U * stride) {
+    uint4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) { a[u] = __ldcs(pre + i + u * stride); b[u] = __ldcs(post + i + u * stride); }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t v = i + u * stride;
+      const uint64_t e0 = v * per;
+      uint32_t m = (per == 32u) ? 0xFFFFFFFFu : ((1u << per) - 1u);
+      if (mask) m &= __ldg(mask + (e0 >> 5)) >> (e0 & 31);
+      const uint32_t q = eq_bits16(a[u], b[u], ew_lg);
+      cm += __popc(m);
+      cu += __popc(m & q);
+    }
+  }
+  for (; i < nvec; i += stride) {
+    const uint4 a = __ldcs(pre + i), b = __ldcs(post + i);
+    const uint64_t e0 = i * per;
+    uint32_t m = (per == 32u) ? 0xFFFFFFFFu : ((1u << per) - 1u);
+    if (mask) m &= __ldg(mask + (e0 >> 5)) >> (e0 & 31);
+    const uint32_t q = eq_bits16(a, b, ew_lg);
+    cm += __popc(m);
+    cu += __popc(m & q);
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    cm += __shfl_xor_sync(0xFFFFFFFFu, cm, o);
+    cu += __shfl_xor_sync(0xFFFFFFFFu, cu, o);
+  }
+  __shared__ unsigned long long sm[8], su[8];
+  if ((threadIdx.x & 31) == 0) { sm[threadIdx.x >> 5] = cm; su[threadIdx.x >> 5] = cu; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long a = 0, b = 0;
+    for (int w = 0; w < 8; ++w) { a += sm[w]; b += su[w]; }
+    if (a) atomicAdd(&out[0], a);
+    if (b) atomicAdd(&out[1], b);
+  }
+}
+
+// scalar part: elements [e_begin, n_elems) byte by byte (tail, or unaligned snapshots)
+__global__ void k_diff_scalar(const uint8_t* pre, const uint8_t* post, uint64_t size, uint32_t ew,
+                              uint64_t e_begin, uint64_t n_elems, const uint32_t* mask,
+                              unsigned long long* out) {
+  unsigned long long cm = 0, cu = 0;
+  for (uint64_t e = e_begin + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < n_elems;
+       e += (uint64_t)gridDim.x * blockDim.x) {
+    if (mask && !((mask[e >> 5] >> (e & 31)) & 1u)) continue;
+    const uint64_t b0 = e * ew;
+    const uint64_t b1 = (b0 + ew <= size) ? b0 + ew : size;
+    bool same = true;
+    for (uint64_t b = b0; b < b1; ++b) same &= (pre[b] == post[b]);
+    cm += 1;
+    cu += same;
+  }
+  if (cm) atomicAdd(&out[0], cm);
+  if (cu) atomicAdd(&out[1], cu);
+}
+
+ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask, ve_diff* out, cudaStream_t s) {
+  const HostObject& o = c->objs[oi];
+  if (!o.pre || !o.post) return fail(c, VE_ERR_INVALID, "ve_snapshot_diff: object needs pre and post snapshots");
+  const uint32_t* mask = nullptr;
+  if (mode == VE_DIFF_WRITTEN) mask = c->t.W + o.bmoff;
+  else if (mode == VE_DIFF_MASK) {
+    if (!d_mask) return fail(c, VE_ERR_INVALID, "ve_snapshot_diff: VE_DIFF_MASK needs d_mask");
+    mask = d_mask;
+  } else if (mode != VE_DIFF_ALL) {
+    return fail(c, VE_ERR_INVALID, "ve_snapshot_diff: bad mode");
+  }
+  const uint32_t ew_lg = o.ew == 1 ? 0 : o.ew == 2 ? 1 : o.ew == 4 ? 2 : 3;
+  unsigned long long* d_out = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&d_out, 16, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "diff alloc");
+  cudaMemsetAsync(d_out, 0, 16, s);
+  const bool aligned = (o.pre % 16 == 0) && (o.post % 16 == 0);
+  uint64_t e_begin = 0;
+  if (aligned) {
+    const uint64_t nvec = o.size / 16;
+    if (nvec) {
+      uint64_t blocks = (nvec + 255) / 256;
+      const uint64_t cap = (uint64_t)c->num_sms * 8;
+      if (blocks > cap) blocks = cap;
+      k_diff_vec<<<(unsigned)blocks, 256, 0, s>>>((const uint4*)o.pre, (const uint4*)o.post, nvec, ew_lg, mask,
+                                                 d_out);
+    }
+    e_begin = nvec * 16 / o.ew;
+  }
+  if (e_begin < o.n_elems) {
+    const uint64_t rem = o.n_elems - e_begin;
+    uint64_t blocks = (rem + 255) / 256;
+    if (blocks > (uint64_t)c->num_sms * 8) blocks = (uint64_t)c->num_sms * 8;
+    k_diff_scalar<<<(unsigned)blocks, 256, 0, s>>>((const uint8_t*)o.pre, (const uint8_t*)o.post, o.size, o.ew,
+                                                  e_begin, o.n_elems, mask, d_out);
+  }
+  unsigned long long h[2];
+  cudaMemcpyAsync(h, d_out, 16, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d_out, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_snapshot_diff");
+  // n_untouched = n_elems - |W u L|
+  std::vector<ve_obj_stats> bc;
+  ve_status st = bitmap_counts(c, s, bc);
+  if (st != VE_OK) return st;
+  out->n_elems = o.n_elems;
+  out->n_masked = h[0];
+  out->n_unchanged = h[1];
+  out->n_changed = h[0] - h[1];
+  out->n_untouched = o.n_elems - bc[o.id].n_touched;
+  out->redundant = (h[0] > 0 && (unsigned __int128)100 * h[1] > (unsigned __int128)c->cfg.t_redundant_pct * h[0]);
+  out->pad = 0;
+  return VE_OK;
+}
+
+}  // namespace ve

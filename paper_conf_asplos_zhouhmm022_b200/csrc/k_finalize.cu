@@ -1,0 +1,341 @@
+// k_finalize.cu -- report-time reductions (SURVEY 8(a) S8 top-k, S9 popcounts).
+//
+// K4: the exact (pc, object, value) histogram is compacted, re-aggregated into
+// the per-PC and per-object views (Def 3.3 counts accesses per key),
+// grouped by key, and reduced to n_distinct + top-k by (count desc, bits asc)
+// with a chunked block-wide selection (levels until one chunk per key).
+// K6: popcounts of the written / loaded element bitmaps per object (C3, C10).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "ve_internal.cuh"
+
+namespace ve {
+
+// ---- scratch management ------------------------------------------------------
+static cudaError_t scratch_need(ve_ctx* c, size_t bytes) {
+  if (c->scratch_bytes >= bytes) return cudaSuccess;
+  if (c->scratch) cudaFree(c->scratch);
+  c->scratch = nullptr;
+  c->scratch_bytes = 0;
+  cudaError_t e = cudaMalloc(&c->scratch, bytes);
+  if (e == cudaSuccess) c->scratch_bytes = bytes;
+  return e;
+}
+
+__device__ __forceinline__ bool vinsert(HSlot* slots, unsigned long long* counts, uint64_t mask,
+                                        unsigned long long* overflow, uint32_t tag, uint64_t bits,
+                                        unsigned long long cnt) {
+  uint64_t h = hist_hash(tag, bits) & mask;
+  for (uint64_t probe = 0; probe <= mask; ++probe) {
+    HSlot* s = &slots[h];
+    uint64_t lo, hi;
+    ld128_volatile(s, lo, hi);
+    if ((uint32_t)hi == EMPTY_TAG) {
+      uint64_t olo, ohi;
+      cas128_global(s, lo, hi, bits, (uint64_t)tag, olo, ohi);
+      if (((uint32_t)ohi == EMPTY_TAG && olo == lo) || ((uint32_t)ohi == tag && olo == bits)) {
+        atomicAdd(&counts[h], cnt);
+        return true;
+      }
+    } else if ((uint32_t)hi == tag && lo == bits) {
+      atomicAdd(&counts[h], cnt);
+      return true;
+    }
+    h = (h + 1) & mask;
+  }
+  atomicExch(overflow, 1ull);
+  return false;
+}
+
+// occupied main-table slots -> per-PC and per-object view table
+__global__ void k_views(const HSlot* hs, const unsigned long long* hc, uint64_t hcap, uint32_t n_pcs,
+                        HSlot* vs, unsigned long long* vc, uint64_t vmask, unsigned long long* overflow,
+                        unsigned long long* n_entries) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < hcap; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t tag = hs[i].tag;
+    if (tag == EMPTY_TAG) continue;
+    const uint64_t bits = hs[i].bits;
+    const unsigned long long cnt = hc[i];
+    atomicAdd(n_entries, 1ull);
+    const uint32_t pc = tag >> 16, koi = tag & 0xFFFFu;
+    vinsert(vs, vc, vmask, overflow, pc, bits, cnt);
+    if (koi != KO_NONE) vinsert(vs, vc, vmask, overflow, n_pcs + koi, bits, cnt);
+  }
+}
+
+__global__ void k_view_count(const HSlot* vs, uint64_t vcap, unsigned long long* ndist) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < vcap; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t tag = vs[i].tag;
+    if (tag != EMPTY_TAG) atomicAdd(&ndist[tag], 1ull);
+  }
+}
+
+__global__ void k_view_scatter(const HSlot* vs, const unsigned long long* vc, uint64_t vcap,
+                               const unsigned long long* off, unsigned long long* cursor, uint64_t* gbits,
+                               uint64_t* gcnt) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < vcap; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t tag = vs[i].tag;
+    if (tag == EMPTY_TAG) continue;
+    const unsigned long long p = off[tag] + atomicAdd(&cursor[tag], 1ull);
+    gbits[p] = vs[i].bits;
+    gcnt[p] = vc[i];
+  }
+}
+
+struct Chunk {
+  uint64_t start, out;
+  uint32_t len, nout;
+};
+
+constexpr int TK_THREADS = 256;
+constexpr int TK_PER = 16;
+constexpr int TK_CHUNK = TK_THREADS * TK_PER;
+
+// "a before b" in the top-k order: count desc, then bits asc
+__device__ __forceinline__ bool before(uint64_t ca, uint64_t ba, uint64_t cb, uint64_t bb) {
+  return ca > cb || (ca == cb && ba < bb);
+}
+
+__global__ void __launch_bounds__(TK_THREADS) k_topk_chunk(const Chunk* chunks, const uint64_t* ib,
+                                                            const uint64_t* ic, uint64_t* ob, uint64_t* oc) {
+  const Chunk ch = chunks[blockIdx.x];
+  uint64_t b[TK_PER], c[TK_PER];
+#pragma unroll
+  for (int j = 0; j < TK_PER; ++j) {
+    const uint32_t idx = threadIdx.x + j * TK_THREADS;
+    if (idx < ch.len) { b[j] = ib[ch.start + idx]; c[j] = ic[ch.start + idx]; }
+    else { b[j] = 0; c[j] = 0; }
+  }
+  __shared__ uint64_t sb[TK_THREADS / 32], sc[TK_THREADS / 32];
+  __shared__ uint64_t pb_s, pc_s;
+  // previous pick; "after prev" = before(prev, e).  Start with a sentinel above everything.
+  uint64_t pb = 0, pcnt = ~0ull;
+  bool first = true;
+  for (uint32_t r = 0; r < ch.nout; ++r) {
+    uint64_t bb = ~0ull, bc = 0;
+    bool have = false;
+#pragma unroll
+    for (int j = 0; j < TK_PER; ++j) {
+      const uint32_t idx = threadIdx.x + j * TK_THREADS;
+      if (idx >= ch.len) continue;
+      const bool after = first || before(pcnt, pb, c[j], b[j]);
+      if (after && (!have || before(c[j], b[j], bc, bb))) { bb = b[j]; bc = c[j]; have = true; }
+    }
+    // warp reduce (no candidate = count 0, bits ~0: loses to every real entry since counts >= 1)
+    for (int o = 16; o > 0; o >>= 1) {
+      const uint64_t ob2 = __shfl_xor_sync(0xFFFFFFFFu, bb, o);
+      const uint64_t oc2 = __shfl_xor_sync(0xFFFFFFFFu, bc, o);
+      if (before(oc2, ob2, bc, bb)) { bb = ob2; bc = oc2; }
+    }
+    if ((threadIdx.x & 31) == 0) { sb[threadIdx.x >> 5] = bb; sc[threadIdx.x >> 5] = bc; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint64_t xb = sb[0], xc = sc[0];
+      for (int wdx = 1; wdx < TK_THREADS / 32; ++wdx)
+        if (before(sc[wdx], sb[wdx], xc, xb)) { xb = sb[wdx]; xc = sc[wdx]; }
+      ob[ch.out + r] = xb;
+      oc[ch.out + r] = xc;
+      pb_s = xb;
+      pc_s = xc;
+    }
+    __syncthreads();
+    pb = pb_s;
+    pcnt = pc_s;
+    first = false;
+  }
+}
+
+__global__ void k_occupancy(const HSlot* hs, uint64_t cap, unsigned long long* cnt) {
+  unsigned long long local = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < cap; i += (uint64_t)gridDim.x * blockDim.x)
+    local += (hs[i].tag != EMPTY_TAG);
+  for (int o = 16; o > 0; o >>= 1) local += __shfl_xor_sync(0xFFFFFFFFu, local, o);
+  if ((threadIdx.x & 31) == 0 && local) atomicAdd(cnt, local);
+}
+
+// Exact n_distinct and top-k of every key (PC keys, then object keys).
+ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
+                        std::vector<ve_topk_entry>& top) {
+  const uint32_t nk = c->n_keys, K = c->cfg.topk;
+  ndistinct.assign(nk, 0);
+  top.assign((size_t)nk * K, ve_topk_entry{0, 0});
+  cudaError_t e;
+  // 1. count occupied slots (upper bound on view entries = 2x)
+  unsigned long long* d_small = nullptr;  // [0] overflow, [1] n_entries
+  e = cudaMallocAsync((void**)&d_small, 16, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "finalize alloc");
+  cudaMemsetAsync(d_small, 0, 16, s);
+  // occupancy of the main table sizes the view table (<= 2 view entries per slot, load <= 1/2)
+  uint64_t occ = 0;
+  {
+    unsigned long long* d_cnt = d_small + 1;
+    k_occupancy<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->hcap, d_cnt);
+    unsigned long long h_cnt = 0;
+    e = cudaMemcpyAsync(&h_cnt, d_cnt, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize occupancy"); }
+    occ = h_cnt;
+    cudaMemsetAsync(d_small, 0, 16, s);
+  }
+  uint64_t vcap = 1024;
+  while (vcap < 4 * occ) vcap <<= 1;
+  const uint64_t vmask = vcap - 1;
+  // scratch: view slots + counts, ndist, off, cursor, grouped bits/counts (x2 for levels)
+  const uint64_t nent = 2 * occ + 1;
+  size_t need = vcap * sizeof(HSlot) + vcap * 8 + 3 * (size_t)nk * 8 + 4 * nent * 8 + 64;
+  e = scratch_need(c, need);
+  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize scratch"); }
+  uint8_t* p = (uint8_t*)c->scratch;
+  HSlot* vs = (HSlot*)p; p += vcap * sizeof(HSlot);
+  unsigned long long* vc = (unsigned long long*)p; p += vcap * 8;
+  unsigned long long* d_nd = (unsigned long long*)p; p += (size_t)nk * 8;
+  unsigned long long* d_off = (unsigned long long*)p; p += (size_t)nk * 8;
+  unsigned long long* d_cur = (unsigned long long*)p; p += (size_t)nk * 8;
+  uint64_t* gb[2]; uint64_t* gc[2];
+  gb[0] = (uint64_t*)p; p += nent * 8;
+  gc[0] = (uint64_t*)p; p += nent * 8;
+  gb[1] = (uint64_t*)p; p += nent * 8;
+  gc[1] = (uint64_t*)p; p += nent * 8;
+  cudaMemsetAsync(vs, 0xFF, vcap * sizeof(HSlot), s);
+  cudaMemsetAsync(vc, 0, vcap * 8, s);
+  cudaMemsetAsync(d_nd, 0, (size_t)nk * 8 * 3, s);
+  const int grid = c->num_sms * 4;
+  k_views<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, c->cfg.n_pcs, vs, vc, vmask, d_small,
+                               d_small + 1);
+  k_view_count<<<grid, 256, 0, s>>>(vs, vcap, d_nd);
+  e = cudaMemcpyAsync(ndistinct.data(), d_nd, (size_t)nk * 8, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize ndistinct"); }
+  std::vector<unsigned long long> off(nk);
+  uint64_t acc = 0;
+  for (uint32_t k = 0; k < nk; ++k) { off[k] = acc; acc += ndistinct[k]; }
+  cudaMemcpyAsync(d_off, off.data(), (size_t)nk * 8, cudaMemcpyHostToDevice, s);
+  k_view_scatter<<<grid, 256, 0, s>>>(vs, vc, vcap, d_off, d_cur, gb[0], gc[0]);
+
+  // selection levels
+  std::vector<uint64_t> len(ndistinct.begin(), ndistinct.end()), start(off.begin(), off.end());
+  int cur = 0;
+  Chunk* d_chunks = nullptr;
+  size_t chunk_cap = 0;
+  for (int level = 0;; ++level) {
+    std::vector<Chunk> chunks;
+    std::vector<uint64_t> nlen(nk, 0), nstart(nk, 0);
+    uint64_t outp = 0;
+    bool single = true;
+    for (uint32_t k = 0; k < nk; ++k) {
+      if (len[k] == 0) continue;
+      const uint64_t nch = (len[k] + TK_CHUNK - 1) / TK_CHUNK;
+      if (nch > 1) single = false;
+      nstart[k] = outp;
+      for (uint64_t j = 0; j < nch; ++j) {
+        Chunk ch;
+        ch.start = start[k] + j * TK_CHUNK;
+        ch.len = (uint32_t)std::min<uint64_t>(TK_CHUNK, len[k] - j * TK_CHUNK);
+        ch.nout = std::min<uint32_t>(K, ch.len);
+        ch.out = outp;
+        outp += ch.nout;
+        chunks.push_back(ch);
+      }
+      nlen[k] = outp - nstart[k];
+    }
+    if (chunks.empty()) break;
+    if (chunks.size() > chunk_cap) {
+      if (d_chunks) cudaFreeAsync(d_chunks, s);
+      chunk_cap = chunks.size() * 2;
+      e = cudaMallocAsync((void**)&d_chunks, chunk_cap * sizeof(Chunk), s);
+      if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize chunks"); }
+    }
+    cudaMemcpyAsync(d_chunks, chunks.data(), chunks.size() * sizeof(Chunk), cudaMemcpyHostToDevice, s);
+    k_topk_chunk<<<(unsigned)chunks.size(), TK_THREADS, 0, s>>>(d_chunks, gb[cur], gc[cur], gb[1 - cur],
+                                                                gc[1 - cur]);
+    cur = 1 - cur;
+    len.swap(nlen);
+    start.swap(nstart);
+    if (single) {
+      std::vector<uint64_t> hb(outp), hc(outp);
+      cudaMemcpyAsync(hb.data(), gb[cur], outp * 8, cudaMemcpyDeviceToHost, s);
+      cudaMemcpyAsync(hc.data(), gc[cur], outp * 8, cudaMemcpyDeviceToHost, s);
+      e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) break;
+      for (uint32_t k = 0; k < nk; ++k)
+        for (uint64_t j = 0; j < len[k]; ++j) top[(size_t)k * K + j] = ve_topk_entry{hb[start[k] + j], hc[start[k] + j]};
+      break;
+    }
+  }
+  unsigned long long h_small[2] = {0, 0};
+  cudaMemcpyAsync(h_small, d_small, 16, cudaMemcpyDeviceToHost, s);
+  if (d_chunks) cudaFreeAsync(d_chunks, s);
+  cudaFreeAsync(d_small, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "finalize top-k");
+  if (h_small[0]) return fail(c, VE_ERR_CAPACITY, "finalize: view table overflow");
+  return VE_OK;
+}
+
+// ---- K6: bitmap popcounts -------------------------------------------------
+__global__ void k_bitmap_counts(const uint32_t* W, const uint32_t* L, const uint64_t* bmoff, const uint64_t* nwords,
+                                unsigned long long* out /* [n][3] */) {
+  const uint32_t o = blockIdx.y;
+  const uint64_t base = bmoff[o], nw = nwords[o];
+  unsigned long long cw = 0, cl = 0, cu = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t w = W[base + i], l = L[base + i];
+    cw += __popc(w);
+    cl += __popc(l);
+    cu += __popc(w | l);
+  }
+  for (int s = 16; s > 0; s >>= 1) {
+    cw += __shfl_xor_sync(0xFFFFFFFFu, cw, s);
+    cl += __shfl_xor_sync(0xFFFFFFFFu, cl, s);
+    cu += __shfl_xor_sync(0xFFFFFFFFu, cu, s);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (cw) atomicAdd(&out[3 * o + 0], cw);
+    if (cl) atomicAdd(&out[3 * o + 1], cl);
+    if (cu) atomicAdd(&out[3 * o + 2], cu);
+  }
+}
+
+ve_status bitmap_counts(ve_ctx* c, cudaStream_t s, std::vector<ve_obj_stats>& out) {
+  const uint32_t n = c->n_obj;
+  out.assign(n, ve_obj_stats{0, 0, 0, 0, 0});
+  if (n == 0) return VE_OK;
+  std::vector<uint64_t> host(2 * n);
+  uint64_t maxw = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    host[i] = c->objs[i].bmoff;
+    host[n + i] = c->objs[i].bmwords;
+    maxw = std::max<uint64_t>(maxw, c->objs[i].bmwords);
+  }
+  void* d = nullptr;
+  cudaError_t e = cudaMallocAsync(&d, 2 * n * 8 + 3 * n * 8, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "bitmap_counts alloc");
+  uint64_t* d_off = (uint64_t*)d;
+  unsigned long long* d_out = (unsigned long long*)((uint8_t*)d + 2 * n * 8);
+  cudaMemcpyAsync(d_off, host.data(), 2 * n * 8, cudaMemcpyHostToDevice, s);
+  cudaMemsetAsync(d_out, 0, 3 * n * 8, s);
+  uint64_t gx = (maxw + 255) / 256;
+  if (gx > 64) gx = 64;
+  if (gx == 0) gx = 1;
+  k_bitmap_counts<<<dim3((unsigned)gx, n), 256, 0, s>>>(c->t.W, c->t.L, d_off, d_off + n, d_out);
+  std::vector<unsigned long long> h(3 * n);
+  cudaMemcpyAsync(h.data(), d_out, 3 * n * 8, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "bitmap_counts");
+  // out is indexed by object id
+  for (uint32_t i = 0; i < n; ++i) {
+    const HostObject& ho = c->objs[i];
+    ve_obj_stats& st = out[ho.id];
+    st.n_elems = ho.n_elems;
+    st.n_written = h[3 * i + 0];
+    st.n_loaded_eq = h[3 * i + 1];
+    st.n_touched = h[3 * i + 2];
+  }
+  return VE_OK;
+}
+
+}  // namespace ve

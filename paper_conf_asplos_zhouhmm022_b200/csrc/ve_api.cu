@@ -1,0 +1,499 @@
+// ve_api.cu -- the C ABI of include/ve.h: context lifecycle, argument
+// validation, the host side of the five hot-path calls, and the report (R1:
+// integer threshold tests and the heavy-type lattice).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "ve_internal.cuh"
+
+namespace ve {
+
+ve_status fail(ve_ctx* c, ve_status s, const std::string& msg) {
+  if (c) c->err = msg;
+  return s;
+}
+ve_status cuda_fail(ve_ctx* c, cudaError_t e, const char* where) {
+  if (c) c->err = std::string(where) + ": " + cudaGetErrorString(e);
+  return VE_ERR_CUDA;
+}
+
+static void free_dev(ve_ctx* c) {
+  cudaFree(c->t.sum);
+  cudaFree(c->t.mn);
+  cudaFree(c->t.mx);
+  cudaFree(c->t.line);
+  cudaFree(c->t.glob);
+  cudaFree(c->t.W);
+  cudaFree(c->t.L);
+  cudaFree(c->t.hslot);
+  cudaFree(c->t.hcount);
+  cudaFree(c->obj_block);
+  cudaFree(c->scratch);
+  for (int i = 0; i < 2; ++i) {
+    if (c->stage[i]) cudaFree(c->stage[i]);
+    if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);
+  }
+}
+
+ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
+  const uint64_t nk_max = (uint64_t)c->cfg.n_pcs + c->cfg.max_objects + 1;
+  cudaMemsetAsync(c->t.sum, 0, nk_max * NSUM * 8, s);
+  cudaMemsetAsync(c->t.mn, 0xFF, nk_max * NMM * 8, s);
+  cudaMemsetAsync(c->t.mx, 0, nk_max * NMM * 8, s);
+  cudaMemsetAsync(c->t.line, 0, nk_max * sizeof(LineState), s);
+  cudaMemsetAsync(c->t.glob, 0, 8 * 8, s);
+  if (c->bm_words) {
+    cudaMemsetAsync(c->t.W, 0, c->bm_words * 4, s);
+    cudaMemsetAsync(c->t.L, 0, c->bm_words * 4, s);
+  }
+  cudaMemsetAsync(c->t.hslot, 0xFF, c->hcap * sizeof(HSlot), s);
+  cudaError_t e = cudaMemsetAsync(c->t.hcount, 0, c->hcap * 8, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "reset");
+  c->poisoned = false;
+  c->hist_merged = false;
+  c->merged_ndistinct.clear();
+  c->merged_topk.clear();
+  return VE_OK;
+}
+
+// ---- R1: heavy type from the raw fields (C6) --------------------------------
+static int64_t float_int_of_ord(uint64_t ord, uint32_t tc) {
+  // invert the orderable key, then decode the (integral) float exactly
+  const uint32_t w = (tc == 8 || tc == 11) ? 2 : (tc == 9) ? 4 : 8;
+  const uint32_t nb = 8 * w;
+  const uint64_t mask = nb == 64 ? ~0ull : ((1ull << nb) - 1);
+  const uint64_t sign = 1ull << (nb - 1);
+  const uint64_t b = (ord & sign) ? (ord & ~sign) : (~ord & mask);
+  int eb, mb;
+  if (tc == 11) { eb = 8; mb = 7; } else if (w == 2) { eb = 5; mb = 10; } else if (w == 4) { eb = 8; mb = 23; }
+  else { eb = 11; mb = 52; }
+  const bool neg = (b >> (nb - 1)) & 1;
+  const uint64_t E = (b >> mb) & ((1ull << eb) - 1), M = b & ((1ull << mb) - 1);
+  const uint64_t sig = E ? (M | (1ull << mb)) : M;
+  const int ex = (E ? (int)E : 1) - ((1 << (eb - 1)) - 1) - mb;
+  uint64_t mag;
+  if (sig == 0) mag = 0;
+  else if (ex >= 0) mag = sig << ex;
+  else mag = (-ex >= 64) ? 0 : (sig >> -ex);
+  return neg ? -(int64_t)mag : (int64_t)mag;
+}
+
+static uint32_t heavy_of(const ve_key_stats& k, uint32_t tc) {
+  static const uint32_t wid[12] = {1, 2, 4, 8, 1, 2, 4, 8, 2, 4, 8, 2};
+  const uint32_t w = wid[tc];
+  const uint32_t cand[3] = {1, 2, 4};
+  if (tc <= 3) {
+    for (uint32_t v : cand) {
+      if (v >= w) break;
+      if (k.ord_max <= ((1ull << (8 * v)) - 1)) return v == 1 ? 0 : v == 2 ? 1 : 2;
+    }
+    return 255;
+  }
+  if (tc <= 7) {
+    const int64_t mn = (int64_t)(k.ord_min ^ (1ull << 63)), mx = (int64_t)(k.ord_max ^ (1ull << 63));
+    for (uint32_t v : cand) {
+      if (v >= w) break;
+      const int64_t lo = -(1ll << (8 * v - 1)), hi = (1ll << (8 * v - 1)) - 1;
+      if (mn >= lo && mx <= hi) return v == 1 ? 4 : v == 2 ? 5 : 6;
+    }
+    return 255;
+  }
+  for (uint32_t v : cand) {
+    if (v >= w) break;
+    if (k.n_nonint == 0) {
+      const int64_t mn = float_int_of_ord(k.ord_min, tc), mx = float_int_of_ord(k.ord_max, tc);
+      if (mn >= 0) {
+        if ((uint64_t)mx <= ((1ull << (8 * v)) - 1)) return v == 1 ? 0 : v == 2 ? 1 : 2;
+      } else {
+        const int64_t lo = -(1ll << (8 * v - 1)), hi = (1ll << (8 * v - 1)) - 1;
+        if (mn >= lo && mx <= hi) return v == 1 ? 4 : v == 2 ? 5 : 6;
+      }
+    }
+    if (v == 2 && k.n_not_f16 == 0) return 8;
+    if (v == 2 && k.n_not_bf16 == 0) return 11;
+    if (v == 4 && k.n_not_f32 == 0) return 9;
+  }
+  return 255;
+}
+
+static void derive(const ve_config& cfg, ve_key_stats& k, const ve_topk_entry* top) {
+  static const uint32_t wid[12] = {1, 2, 4, 8, 1, 2, 4, 8, 2, 4, 8, 2};
+  const uint64_t n = k.n_ld + k.n_st;
+  uint32_t nt = 0, tc = 0;
+  for (uint32_t t = 0; t < 12; ++t)
+    if (k.n_type[t]) { ++nt; tc = t; }
+  k.single_type = nt == 1;
+  k.single_value = n > 0 && k.raw_min == k.raw_max;
+  k.single_zero = n > 0 && k.n_zero == n;
+  k.frequent = k.n_top > 0 && (unsigned __int128)100 * top[0].count > (unsigned __int128)cfg.t_frequent_pct * n;
+  k.structured = k.approx = k.dict8 = 0;
+  k.heavy = 255;
+  if (!k.single_type) return;
+  const __int128 py = (__int128)(((unsigned __int128)(uint64_t)k.p_yhi << 64) | k.p_ylo);
+  const __int128 qy = (__int128)(((unsigned __int128)(uint64_t)k.q_yhi << 64) | k.q_ylo);
+  k.structured = k.line_state == VE_LINE_LINE && py != qy;
+  k.approx = tc >= 8 && k.n_nan == 0 && n > 0 && k.trunc_min == k.trunc_max && !k.single_value;
+  k.dict8 = k.n_distinct <= 256 && wid[tc] > 1;
+  k.heavy = heavy_of(k, tc);
+}
+
+static bool ctx_ok(const ve_ctx* c) { return c != nullptr; }
+
+}  // namespace ve
+
+using namespace ve;
+
+extern "C" {
+
+ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
+  if (!cfg || !out) return VE_ERR_INVALID;
+  *out = nullptr;
+  if (cfg->n_pcs == 0 || cfg->n_pcs > 65535 || cfg->max_objects > 65534 || cfg->topk == 0 || cfg->topk > 64 ||
+      cfg->hist_capacity == 0)
+    return VE_ERR_INVALID;
+  ve_ctx* c = new (std::nothrow) ve_ctx();
+  if (!c) return VE_ERR_NOMEM;
+  c->cfg = *cfg;
+  c->device = cuda_device;
+  cudaError_t e = cudaSetDevice(cuda_device);
+  if (e != cudaSuccess) { delete c; return VE_ERR_CUDA; }
+  cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  uint64_t hcap = 1024;
+  while (hcap < cfg->hist_capacity) hcap <<= 1;
+  c->hcap = hcap;
+  c->t.hmask = hcap - 1;
+  const uint64_t nk_max = (uint64_t)cfg->n_pcs + cfg->max_objects + 1;
+  bool ok = cudaMalloc(&c->t.sum, nk_max * NSUM * 8) == cudaSuccess &&
+            cudaMalloc(&c->t.mn, nk_max * NMM * 8) == cudaSuccess &&
+            cudaMalloc(&c->t.mx, nk_max * NMM * 8) == cudaSuccess &&
+            cudaMalloc(&c->t.line, nk_max * sizeof(LineState)) == cudaSuccess &&
+            cudaMalloc(&c->t.glob, 8 * 8) == cudaSuccess &&
+            cudaMalloc(&c->t.hslot, hcap * sizeof(HSlot)) == cudaSuccess &&
+            cudaMalloc(&c->t.hcount, hcap * 8) == cudaSuccess;
+  if (!ok) {
+    cudaGetLastError();
+    free_dev(c);
+    delete c;
+    return VE_ERR_NOMEM;
+  }
+  c->n_obj = 0;
+  c->n_keys = cfg->n_pcs + 1;
+  if (launch_reset(c, 0) != VE_OK || cudaDeviceSynchronize() != cudaSuccess) {
+    free_dev(c);
+    delete c;
+    return VE_ERR_CUDA;
+  }
+  *out = c;
+  return VE_OK;
+}
+
+ve_status ve_destroy(ve_ctx* c) {
+  if (!c) return VE_ERR_INVALID;
+  cudaSetDevice(c->device);
+  cudaDeviceSynchronize();
+  free_dev(c);
+  delete c;
+  return VE_OK;
+}
+
+const char* ve_last_error(const ve_ctx* c) { return c ? c->err.c_str() : "null context"; }
+
+ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
+  if (!ctx_ok(c)) return VE_ERR_INVALID;
+  if (n > c->cfg.max_objects) return fail(c, VE_ERR_INVALID, "ve_set_objects: n > max_objects");
+  if (n && !objs) return fail(c, VE_ERR_INVALID, "ve_set_objects: null objects");
+  std::vector<HostObject> v(n);
+  std::vector<char> seen(n, 0);
+  for (uint32_t i = 0; i < n; ++i) {
+    const ve_object& o = objs[i];
+    const uint32_t ew = o.elem_width;
+    if (o.size == 0 || o.id >= n || seen[o.id] || !(ew == 1 || ew == 2 || ew == 4 || ew == 8) ||
+        o.base >= (1ull << 48) || o.size > (1ull << 48) - o.base)
+      return fail(c, VE_ERR_INVALID, "ve_set_objects: bad object " + std::to_string(i));
+    seen[o.id] = 1;
+    v[i] = HostObject{o.base, o.size, (uint64_t)(uintptr_t)o.pre, (uint64_t)(uintptr_t)o.post, o.id, ew,
+                      (o.size + ew - 1) / ew, 0, 0};
+  }
+  std::sort(v.begin(), v.end(), [](const HostObject& a, const HostObject& b) { return a.base < b.base; });
+  for (uint32_t i = 1; i < n; ++i)
+    if (v[i - 1].base + v[i - 1].size > v[i].base) return fail(c, VE_ERR_INVALID, "ve_set_objects: overlap");
+  uint64_t words = 0;
+  for (auto& o : v) {
+    o.bmoff = words;
+    o.bmwords = (o.n_elems + 31) / 32;
+    words += o.bmwords;
+  }
+  cudaSetDevice(c->device);
+  cudaDeviceSynchronize();
+  if (words > c->bm_words || !c->t.W) {
+    cudaFree(c->t.W);
+    cudaFree(c->t.L);
+    c->t.W = c->t.L = nullptr;
+    const uint64_t alloc = words ? words : 1;
+    if (cudaMalloc(&c->t.W, alloc * 4) != cudaSuccess || cudaMalloc(&c->t.L, alloc * 4) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(c, VE_ERR_NOMEM, "ve_set_objects: bitmaps");
+    }
+  }
+  c->bm_words = words;
+  // device object table (SoA, sorted by base)
+  cudaFree(c->obj_block);
+  c->obj_block = nullptr;
+  const size_t nb = (size_t)(n ? n : 1) * (8 * 4 + 4 * 2) + 64;
+  if (cudaMalloc(&c->obj_block, nb) != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "objects"); }
+  std::vector<uint8_t> host(nb, 0);
+  uint64_t* hb = (uint64_t*)host.data();
+  uint64_t* he = hb + n;
+  uint64_t* hp = he + n;
+  uint64_t* hm = hp + n;
+  uint32_t* hid = (uint32_t*)(hm + n);
+  uint32_t* hew = hid + n;
+  c->sorted_of_id.assign(n, 0);
+  for (uint32_t i = 0; i < n; ++i) {
+    hb[i] = v[i].base; he[i] = v[i].base + v[i].size; hp[i] = v[i].pre; hm[i] = v[i].bmoff;
+    hid[i] = v[i].id; hew[i] = v[i].ew;
+    c->sorted_of_id[v[i].id] = i;
+  }
+  cudaMemcpy(c->obj_block, host.data(), nb, cudaMemcpyHostToDevice);
+  uint64_t* db = (uint64_t*)c->obj_block;
+  c->o.base = db;
+  c->o.end = db + n;
+  c->o.pre = db + 2 * n;
+  c->o.bmoff = db + 3 * n;
+  c->o.id = (const uint32_t*)(db + 4 * n);
+  c->o.ew = c->o.id + n;
+  c->o.n = n;
+  c->objs = v;
+  c->n_obj = n;
+  c->n_keys = c->cfg.n_pcs + n + 1;
+  ve_status st = launch_reset(c, 0);
+  if (st != VE_OK) return st;
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_set_objects");
+  return VE_OK;
+}
+
+ve_status ve_reset(ve_ctx* c) {
+  if (!ctx_ok(c)) return VE_ERR_INVALID;
+  cudaSetDevice(c->device);
+  ve_status st = launch_reset(c, 0);
+  if (st != VE_OK) return st;
+  cudaError_t e = cudaDeviceSynchronize();
+  return e == cudaSuccess ? VE_OK : cuda_fail(c, e, "ve_reset");
+}
+
+ve_status ve_analyze_records(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
+  if (!ctx_ok(c)) return VE_ERR_INVALID;
+  if (c->poisoned || c->hist_merged) return fail(c, VE_ERR_STATE, "ve_analyze_records: ctx poisoned or merged; ve_reset first");
+  if (n == 0) return VE_OK;
+  if (!d || ((uintptr_t)d & 7)) return fail(c, VE_ERR_INVALID, "ve_analyze_records: d_records null or not 8-byte aligned");
+  // per-CTA shared counters are 32-bit: keep each launch well below 2^32 records per CTA
+  const uint64_t CH = 1ull << 36;
+  for (uint64_t off = 0; off < n; off += CH) {
+    ve_status st = launch_analyze(c, d + off, std::min(CH, n - off), s);
+    if (st != VE_OK) return st;
+  }
+  return VE_OK;
+}
+
+ve_status ve_analyze_records_host(ve_ctx* c, const ve_record* h, uint64_t n, cudaStream_t s) {
+  if (!ctx_ok(c)) return VE_ERR_INVALID;
+  if (c->poisoned || c->hist_merged) return fail(c, VE_ERR_STATE, "ve_analyze_records_host: ctx poisoned or merged");
+  if (n == 0) return VE_OK;
+  if (!h) return fail(c, VE_ERR_INVALID, "ve_analyze_records_host: null records");
+  const uint64_t CH = 1ull << 21;  // 2 Mi records = 48 MiB per staging buffer
+  if (!c->stage[0]) {
+    for (int i = 0; i < 2; ++i) {
+      if (cudaMalloc(&c->stage[i], CH * sizeof(ve_record)) != cudaSuccess ||
+          cudaEventCreateWithFlags(&c->stage_ev[i], cudaEventDisableTiming) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, VE_ERR_NOMEM, "staging buffers");
+      }
+    }
+    c->stage_bytes = CH * sizeof(ve_record);
+  }
+  // chunk i: copy into stage[i%2] (after that buffer's previous analysis), then analyze it
+  for (uint64_t off = 0, i = 0; off < n; off += CH, ++i) {
+    const int b = (int)(i & 1);
+    const uint64_t m = std::min(CH, n - off);
+    cudaError_t e = cudaStreamWaitEvent(s, c->stage_ev[b], 0);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(c->stage[b], h + off, m * sizeof(ve_record), cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "ve_analyze_records_host copy");
+    ve_status st = launch_analyze(c, (const ve_record*)c->stage[b], m, s);
+    if (st != VE_OK) return st;
+    cudaEventRecord(c->stage_ev[b], s);
+  }
+  return VE_OK;
+}
+
+ve_status ve_snapshot_diff(ve_ctx* c, uint32_t obj_id, uint32_t mode, const uint32_t* d_mask, ve_diff* h_out,
+                           cudaStream_t s) {
+  if (!ctx_ok(c) || !h_out) return VE_ERR_INVALID;
+  if (obj_id >= c->n_obj) return fail(c, VE_ERR_INVALID, "ve_snapshot_diff: bad object id");
+  return run_diff(c, c->sorted_of_id[obj_id], mode, d_mask, h_out, s);
+}
+
+ve_status ve_object_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* h_group_of, cudaStream_t s) {
+  if (!ctx_ok(c) || (n && (!objs || !h_group_of))) return VE_ERR_INVALID;
+  return run_dedup(c, objs, n, h_group_of, s);
+}
+
+ve_status ve_merge_stats(ve_ctx* dst, const ve_ctx* src, void* comm, cudaStream_t s) {
+  if (!ctx_ok(dst) || (!src && !comm) || (src && comm)) return VE_ERR_INVALID;
+  if (dst->hist_merged) return fail(dst, VE_ERR_STATE, "ve_merge_stats: ctx already merged over ranks");
+  cudaSetDevice(dst->device);
+  if (src) return merge_local(dst, src, s);
+  return merge_nccl(dst, comm, s);
+}
+
+ve_status ve_report(ve_ctx* c, ve_rep** out) {
+  if (!ctx_ok(c) || !out) return VE_ERR_INVALID;
+  *out = nullptr;
+  cudaSetDevice(c->device);
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_report (pending work)");
+  if (c->poisoned) return fail(c, VE_ERR_STATE, "ve_report: ctx poisoned by histogram overflow; ve_reset");
+  unsigned long long glob[8];
+  cudaMemcpy(glob, c->t.glob, sizeof(glob), cudaMemcpyDeviceToHost);
+  if (glob[G_OVERFLOW]) {
+    c->poisoned = true;
+    return fail(c, VE_ERR_CAPACITY, "value histogram capacity exceeded (hist_capacity)");
+  }
+  const uint32_t nk = c->n_keys, K = c->cfg.topk;
+  std::vector<uint64_t> sum((size_t)nk * NSUM), mn((size_t)nk * NMM), mx((size_t)nk * NMM);
+  std::vector<LineState> line(nk);
+  cudaMemcpy(sum.data(), c->t.sum, sum.size() * 8, cudaMemcpyDeviceToHost);
+  cudaMemcpy(mn.data(), c->t.mn, mn.size() * 8, cudaMemcpyDeviceToHost);
+  cudaMemcpy(mx.data(), c->t.mx, mx.size() * 8, cudaMemcpyDeviceToHost);
+  e = cudaMemcpy(line.data(), c->t.line, nk * sizeof(LineState), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_report copy");
+  ve_rep* r = new (std::nothrow) ve_rep();
+  if (!r) return VE_ERR_NOMEM;
+  r->n_keys = nk;
+  r->n_obj = c->n_obj;
+  r->topk = K;
+  std::vector<uint64_t> nd;
+  ve_status st;
+  if (c->hist_merged) {
+    nd = c->merged_ndistinct;
+    r->top = c->merged_topk;
+  } else {
+    st = finalize_hist(c, 0, nd, r->top);
+    if (st != VE_OK) { delete r; return st; }
+  }
+  st = bitmap_counts(c, 0, r->objs);
+  if (st != VE_OK) { delete r; return st; }
+  r->keys.assign(nk, ve_key_stats{});
+  for (uint32_t k = 0; k < nk; ++k) {
+    ve_key_stats& ks = r->keys[k];
+    memset(&ks, 0, sizeof(ks));
+    const uint64_t* sv = &sum[(size_t)k * NSUM];
+    ks.n_ld = sv[F_LD]; ks.n_st = sv[F_ST]; ks.n_zero = sv[F_ZERO];
+    ks.n_ld_eq_pre = sv[F_LDEQ]; ks.n_st_eq_pre = sv[F_STEQ]; ks.n_nosnap = sv[F_NOSNAP];
+    for (int t = 0; t < 12; ++t) ks.n_type[t] = sv[F_TYPE0 + t];
+    ks.n_nan = sv[F_NAN]; ks.n_nonint = sv[F_NONINT]; ks.n_not_f16 = sv[F_NF16];
+    ks.n_not_bf16 = sv[F_NBF16]; ks.n_not_f32 = sv[F_NF32];
+    ks.raw_min = mn[(size_t)k * NMM + M_RAW]; ks.ord_min = mn[(size_t)k * NMM + M_ORD];
+    ks.trunc_min = mn[(size_t)k * NMM + M_TRUNC];
+    ks.raw_max = mx[(size_t)k * NMM + M_RAW]; ks.ord_max = mx[(size_t)k * NMM + M_ORD];
+    ks.trunc_max = mx[(size_t)k * NMM + M_TRUNC];
+    const LineState& L = line[k];
+    ks.line_state = L.state;
+    if (L.state == VE_LINE_POINT || L.state == VE_LINE_LINE) {
+      ks.p_x = L.px; ks.p_ylo = L.pylo; ks.p_yhi = L.pyhi;
+      ks.q_x = L.qx; ks.q_ylo = L.qylo; ks.q_yhi = L.qyhi;
+    }
+    ks.n_distinct = nd[k];
+    ks.n_top = std::min<uint64_t>(nd[k], K);
+    derive(c->cfg, ks, &r->top[(size_t)k * K]);
+  }
+  for (uint32_t i = 0; i < c->n_obj; ++i) {
+    ve_obj_stats& os = r->objs[i];
+    const uint64_t eq = r->keys[c->cfg.n_pcs + i].n_ld_eq_pre;
+    os.n_ld_reload = eq - os.n_loaded_eq;
+  }
+  r->glob.n_records = glob[G_RECORDS];
+  r->glob.n_invalid = glob[G_INVALID];
+  r->glob.n_unmapped = glob[G_UNMAPPED];
+  r->glob.hist_entries = 0;
+  *out = r;
+  return VE_OK;
+}
+
+void ve_report_free(ve_rep* r) { delete r; }
+uint32_t ve_report_n_keys(const ve_rep* r) { return r ? r->n_keys : 0; }
+uint32_t ve_report_n_objects(const ve_rep* r) { return r ? r->n_obj : 0; }
+uint32_t ve_report_topk(const ve_rep* r) { return r ? r->topk : 0; }
+
+ve_status ve_report_keys(const ve_rep* r, ve_key_stats* out) {
+  if (!r || !out) return VE_ERR_INVALID;
+  memcpy(out, r->keys.data(), r->keys.size() * sizeof(ve_key_stats));
+  return VE_OK;
+}
+ve_status ve_report_topk_entries(const ve_rep* r, ve_topk_entry* out) {
+  if (!r || !out) return VE_ERR_INVALID;
+  memcpy(out, r->top.data(), r->top.size() * sizeof(ve_topk_entry));
+  return VE_OK;
+}
+ve_status ve_report_objects(const ve_rep* r, ve_obj_stats* out) {
+  if (!r || !out) return VE_ERR_INVALID;
+  memcpy(out, r->objs.data(), r->objs.size() * sizeof(ve_obj_stats));
+  return VE_OK;
+}
+ve_status ve_report_globals(const ve_rep* r, ve_globals* out) {
+  if (!r || !out) return VE_ERR_INVALID;
+  *out = r->glob;
+  return VE_OK;
+}
+
+ve_status ve_report_dump(const ve_rep* r, const char* path, int format) {
+  if (!r || !path || (format != 0 && format != 1)) return VE_ERR_INVALID;
+  FILE* f = fopen(path, format == 0 ? "wb" : "w");
+  if (!f) return VE_ERR_INVALID;
+  if (format == 0) {
+    const uint32_t hdr[4] = {0x50524556u /* "VERP" */, 1u, r->n_keys, r->n_obj};
+    fwrite(hdr, 4, 4, f);
+    fwrite(&r->topk, 4, 1, f);
+    fwrite(&r->glob, sizeof(r->glob), 1, f);
+    fwrite(r->keys.data(), sizeof(ve_key_stats), r->keys.size(), f);
+    fwrite(r->top.data(), sizeof(ve_topk_entry), r->top.size(), f);
+    fwrite(r->objs.data(), sizeof(ve_obj_stats), r->objs.size(), f);
+  } else {
+    static const char* tn[12] = {"u8", "u16", "u32", "u64", "i8", "i16", "i32", "i64", "f16", "f32", "f64", "bf16"};
+    fprintf(f, "{\"n_records\": %llu, \"n_invalid\": %llu, \"n_unmapped\": %llu, \"keys\": [\n",
+            (unsigned long long)r->glob.n_records, (unsigned long long)r->glob.n_invalid,
+            (unsigned long long)r->glob.n_unmapped);
+    for (uint32_t k = 0; k < r->n_keys; ++k) {
+      const ve_key_stats& s = r->keys[k];
+      fprintf(f,
+              "  {\"key\": %u, \"n_ld\": %llu, \"n_st\": %llu, \"n_zero\": %llu, \"n_ld_eq_pre\": %llu, "
+              "\"n_st_eq_pre\": %llu, \"n_distinct\": %llu, \"single_value\": %u, \"single_zero\": %u, "
+              "\"frequent\": %u, \"structured\": %u, \"approx\": %u, \"dict8\": %u, \"heavy\": \"%s\", \"top\": [",
+              k, (unsigned long long)s.n_ld, (unsigned long long)s.n_st, (unsigned long long)s.n_zero,
+              (unsigned long long)s.n_ld_eq_pre, (unsigned long long)s.n_st_eq_pre,
+              (unsigned long long)s.n_distinct, s.single_value, s.single_zero, s.frequent, s.structured, s.approx,
+              s.dict8, s.heavy < 12 ? tn[s.heavy] : "none");
+      for (uint64_t j = 0; j < s.n_top; ++j)
+        fprintf(f, "%s[%llu, %llu]", j ? ", " : "", (unsigned long long)r->top[(size_t)k * r->topk + j].bits,
+                (unsigned long long)r->top[(size_t)k * r->topk + j].count);
+      fprintf(f, "]}%s\n", k + 1 < r->n_keys ? "," : "");
+    }
+    fprintf(f, "], \"objects\": [\n");
+    for (uint32_t i = 0; i < r->n_obj; ++i) {
+      const ve_obj_stats& o = r->objs[i];
+      fprintf(f, "  {\"id\": %u, \"n_elems\": %llu, \"n_written\": %llu, \"n_ld_reload\": %llu, \"n_touched\": %llu}%s\n",
+              i, (unsigned long long)o.n_elems, (unsigned long long)o.n_written, (unsigned long long)o.n_ld_reload,
+              (unsigned long long)o.n_touched, i + 1 < r->n_obj ? "," : "");
+    }
+    fprintf(f, "]}\n");
+  }
+  fclose(f);
+  return VE_OK;
+}
+
+}  // extern "C"

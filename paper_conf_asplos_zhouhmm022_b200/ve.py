@@ -1,0 +1,252 @@
+"""Thin ctypes binding of libve.so (include/ve.h): argument marshalling only.
+
+Every step of the analysis runs in libve.so's CUDA kernels; there is no CPU
+fallback -- importing this module on a box without the built library, or
+calling it without a CUDA device, fails loudly.  torch is used only for device
+memory and streams.
+"""
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB = None
+
+OK, ERR_INVALID, ERR_CUDA, ERR_NOMEM, ERR_CAPACITY, ERR_NCCL, ERR_STATE = range(7)
+DIFF_WRITTEN, DIFF_ALL, DIFF_MASK = 0, 1, 2
+LINE_EMPTY, LINE_POINT, LINE_LINE, LINE_FAIL = 0, 1, 2, 3
+STATUS_NAMES = ["VE_OK", "VE_ERR_INVALID", "VE_ERR_CUDA", "VE_ERR_NOMEM", "VE_ERR_CAPACITY", "VE_ERR_NCCL",
+                "VE_ERR_STATE"]
+
+RECORD_DTYPE = np.dtype([("addr", "<u8"), ("value", "<u8"), ("pc", "<u4"), ("meta", "<u4")])
+
+# mirror of ve_key_stats
+KEY_DTYPE = np.dtype(
+    [(f, "<u8") for f in ("n_ld", "n_st", "n_zero", "n_ld_eq_pre", "n_st_eq_pre", "n_nosnap")]
+    + [("n_type", "<u8", (12,))]
+    + [(f, "<u8") for f in ("n_nan", "n_nonint", "n_not_f16", "n_not_bf16", "n_not_f32")]
+    + [(f, "<u8") for f in ("raw_min", "raw_max", "ord_min", "ord_max", "trunc_min", "trunc_max")]
+    + [("line_state", "<u8"), ("p_x", "<u8"), ("p_ylo", "<u8"), ("p_yhi", "<i8"), ("q_x", "<u8"),
+       ("q_ylo", "<u8"), ("q_yhi", "<i8"), ("n_distinct", "<u8"), ("n_top", "<u8")]
+    + [(f, "<u4") for f in ("single_value", "single_zero", "frequent", "structured", "approx", "dict8", "heavy",
+                            "single_type")])
+TOPK_DTYPE = np.dtype([("bits", "<u8"), ("count", "<u8")])
+OBJ_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_written", "n_loaded_eq", "n_ld_reload", "n_touched")])
+GLOB_DTYPE = np.dtype([(f, "<u8") for f in ("n_records", "n_invalid", "n_unmapped", "hist_entries")])
+DIFF_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_masked", "n_unchanged", "n_changed", "n_untouched")]
+                      + [("redundant", "<u4"), ("pad", "<u4")])
+
+
+class VeError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS_NAMES[status] if 0 <= status < 7 else status}: {msg}")
+        self.status = status
+
+
+class _Config(ctypes.Structure):
+    _fields_ = [("n_pcs", ctypes.c_uint32), ("max_objects", ctypes.c_uint32), ("topk", ctypes.c_uint32),
+                ("mant_bits", ctypes.c_uint32), ("t_redundant_pct", ctypes.c_uint32),
+                ("t_frequent_pct", ctypes.c_uint32), ("hist_capacity", ctypes.c_uint64)]
+
+
+class _Object(ctypes.Structure):
+    _fields_ = [("base", ctypes.c_uint64), ("size", ctypes.c_uint64), ("pre", ctypes.c_void_p),
+                ("post", ctypes.c_void_p), ("id", ctypes.c_uint32), ("elem_width", ctypes.c_uint32)]
+
+
+def lib():
+    global _LIB
+    if _LIB is None:
+        path = os.path.join(_HERE, "libve.so")
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} missing: run __graft_entry__.build() (no CPU fallback exists)")
+        L = ctypes.CDLL(path)
+        vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+        st = ctypes.c_int
+        sig = {
+            "ve_create": ([ctypes.POINTER(_Config), i32, ctypes.POINTER(vp)], st),
+            "ve_destroy": ([vp], st),
+            "ve_last_error": ([vp], ctypes.c_char_p),
+            "ve_set_objects": ([vp, vp, u32], st),
+            "ve_reset": ([vp], st),
+            "ve_analyze_records": ([vp, vp, u64, vp], st),
+            "ve_analyze_records_host": ([vp, vp, u64, vp], st),
+            "ve_snapshot_diff": ([vp, u32, u32, vp, vp, vp], st),
+            "ve_object_dedup": ([vp, vp, u32, vp, vp], st),
+            "ve_merge_stats": ([vp, vp, vp, vp], st),
+            "ve_report": ([vp, ctypes.POINTER(vp)], st),
+            "ve_report_free": ([vp], None),
+            "ve_report_n_keys": ([vp], u32),
+            "ve_report_n_objects": ([vp], u32),
+            "ve_report_topk": ([vp], u32),
+            "ve_report_keys": ([vp, vp], st),
+            "ve_report_topk_entries": ([vp, vp], st),
+            "ve_report_objects": ([vp, vp], st),
+            "ve_report_globals": ([vp, vp], st),
+            "ve_report_dump": ([vp, ctypes.c_char_p, i32], st),
+            "ve_nccl_get_unique_id": ([vp], st),
+            "ve_nccl_comm_init": ([ctypes.POINTER(vp), i32, vp, i32], st),
+            "ve_nccl_comm_destroy": ([vp], st),
+        }
+        for name, (args, res) in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _LIB = L
+    return _LIB
+
+
+def _ptr(x):
+    """device/host pointer of a torch tensor, numpy array or int"""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    raise TypeError(type(x))
+
+
+def _stream(stream):
+    if stream is None:
+        try:
+            import torch
+            if torch.cuda.is_available():
+                return torch.cuda.current_stream().cuda_stream
+        except ImportError:
+            pass
+        return 0
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+class Report:
+    """Host copy of a ve_report: keys (KEY_DTYPE), topk[n_keys, k] (TOPK_DTYPE), objects, globals."""
+
+    def __init__(self, handle):
+        L = lib()
+        self.n_keys = L.ve_report_n_keys(handle)
+        self.n_objects = L.ve_report_n_objects(handle)
+        self.k = L.ve_report_topk(handle)
+        self.keys = np.zeros(self.n_keys, dtype=KEY_DTYPE)
+        self.topk = np.zeros((self.n_keys, self.k), dtype=TOPK_DTYPE)
+        self.objects = np.zeros(max(self.n_objects, 1), dtype=OBJ_DTYPE)
+        g = np.zeros(1, dtype=GLOB_DTYPE)
+        L.ve_report_keys(handle, self.keys.ctypes.data)
+        L.ve_report_topk_entries(handle, self.topk.ctypes.data)
+        L.ve_report_objects(handle, self.objects.ctypes.data)
+        L.ve_report_globals(handle, g.ctypes.data)
+        self.objects = self.objects[:self.n_objects]
+        self.globals = g[0]
+        self._handle = handle
+
+    def dump(self, path, fmt=1):
+        rc = lib().ve_report_dump(self._handle, path.encode(), fmt)
+        if rc != OK:
+            raise VeError(rc, "ve_report_dump")
+
+    def close(self):
+        if self._handle:
+            lib().ve_report_free(self._handle)
+            self._handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Context:
+    """A ve_ctx bound to one CUDA device."""
+
+    def __init__(self, n_pcs, max_objects=64, topk=8, mant_bits=7, t_redundant_pct=33, t_frequent_pct=33,
+                 hist_capacity=1 << 22, device=None):
+        L = lib()
+        if device is None:
+            import torch
+            device = torch.cuda.current_device()
+        self.device = device
+        cfg = _Config(n_pcs, max_objects, topk, mant_bits, t_redundant_pct, t_frequent_pct, hist_capacity)
+        h = ctypes.c_void_p()
+        rc = L.ve_create(ctypes.byref(cfg), device, ctypes.byref(h))
+        if rc != OK:
+            raise VeError(rc, "ve_create")
+        self._h = h
+        self.n_pcs = n_pcs
+        self._keep = []
+
+    def _check(self, rc, what):
+        if rc != OK:
+            raise VeError(rc, f"{what}: {lib().ve_last_error(self._h).decode()}")
+
+    @property
+    def handle(self):
+        return self._h
+
+    def set_objects(self, objs):
+        """objs: dicts {base, size, id, elem_width, pre, post} (pre/post: device tensors/pointers or None)."""
+        arr = (_Object * max(len(objs), 1))()
+        keep = []
+        for i, o in enumerate(objs):
+            arr[i] = _Object(o["base"], o["size"], _ptr(o.get("pre")), _ptr(o.get("post")), o["id"],
+                             o["elem_width"])
+            keep += [o.get("pre"), o.get("post")]
+        self._keep = keep
+        self._check(lib().ve_set_objects(self._h, arr, len(objs)), "ve_set_objects")
+        self.n_objects = len(objs)
+
+    def reset(self):
+        self._check(lib().ve_reset(self._h), "ve_reset")
+
+    def analyze_records(self, d_records, n=None, stream=None):
+        if n is None:
+            n = d_records.numel() // 24 if hasattr(d_records, "numel") else len(d_records)
+        self._check(lib().ve_analyze_records(self._h, _ptr(d_records), n, _stream(stream)), "ve_analyze_records")
+
+    def analyze_records_host(self, h_records, n=None, stream=None):
+        if n is None:
+            n = len(h_records) if isinstance(h_records, np.ndarray) and h_records.dtype.itemsize == 24 else \
+                h_records.numel() // 24
+        self._check(lib().ve_analyze_records_host(self._h, _ptr(h_records), n, _stream(stream)),
+                    "ve_analyze_records_host")
+
+    def snapshot_diff(self, obj_id, mode=DIFF_WRITTEN, d_mask=None, stream=None):
+        out = np.zeros(1, dtype=DIFF_DTYPE)
+        self._check(lib().ve_snapshot_diff(self._h, obj_id, mode, _ptr(d_mask), out.ctypes.data, _stream(stream)),
+                    "ve_snapshot_diff")
+        return out[0]
+
+    def object_dedup(self, objs, stream=None):
+        arr = (_Object * max(len(objs), 1))()
+        for i, o in enumerate(objs):
+            arr[i] = _Object(o["base"], o["size"], _ptr(o.get("pre")), _ptr(o.get("post")), o["id"],
+                             o.get("elem_width", 8))
+        g = np.zeros(max(len(objs), 1), dtype=np.uint32)
+        self._check(lib().ve_object_dedup(self._h, arr, len(objs), g.ctypes.data, _stream(stream)),
+                    "ve_object_dedup")
+        return g[:len(objs)]
+
+    def merge(self, other=None, comm=None, stream=None):
+        self._check(lib().ve_merge_stats(self._h, other._h if other is not None else None, comm, _stream(stream)),
+                    "ve_merge_stats")
+
+    def report(self):
+        h = ctypes.c_void_p()
+        self._check(lib().ve_report(self._h, ctypes.byref(h)), "ve_report")
+        return Report(h)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().ve_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

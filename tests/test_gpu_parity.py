@@ -1,0 +1,168 @@
+"""GPU parity: libve.so (sm_100a) against the CPU oracle, bit-exact, through
+the C ABI.  Sizes span many CTAs/windows and ragged tails; adversarial fuzz
+traces exercise every slow path."""
+import numpy as np
+import pytest
+
+from gen import vegen as G
+from oracle import oracle as O
+from tests import parity, workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def _ve():
+    from paper_conf_asplos_zhouhmm022_b200 import ve
+    return ve
+
+
+def _run_gpu(torch_cuda, n_pcs, hobjs, recs, chunks=None, topk=8, hist_capacity=1 << 20, diff_modes=()):
+    ve = _ve()
+    dobjs = W.device_objects(hobjs)
+    ctx = ve.Context(n_pcs=n_pcs, max_objects=max(len(hobjs), 1), topk=topk, hist_capacity=hist_capacity)
+    ctx.set_objects(dobjs)
+    drec = W.device_records(recs)
+    n = len(recs)
+    if chunks is None:
+        ctx.analyze_records(drec, n)
+    else:
+        bounds = [0] + list(chunks) + [n]
+        for a, b in zip(bounds[:-1], bounds[1:]):
+            if b > a:
+                ctx.analyze_records(drec[a * 24:b * 24], b - a)
+    rep = ctx.report()
+    diffs = {}
+    for oid, mode, mask in diff_modes:
+        dm = torch_cuda.from_numpy(mask).cuda() if mask is not None else None
+        diffs[(oid, mode)] = ctx.snapshot_diff(oid, mode, dm)
+    ctx.close()
+    return rep, diffs
+
+
+def _check(torch_cuda, n_pcs, hobjs, recs, **kw):
+    cfg = O.make_config(n_pcs, topk=kw.get("topk", 8))
+    okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
+    modes = []
+    for o in hobjs:
+        if o.get("pre") is not None and o.get("post") is not None:
+            ne = (o["size"] + o["elem_width"] - 1) // o["elem_width"]
+            mask = np.random.default_rng(o["id"]).integers(0, 1 << 32, (ne + 31) // 32, dtype=np.uint64).astype(np.uint32)
+            modes += [(o["id"], O.DIFF_WRITTEN, None), (o["id"], O.DIFF_ALL, None), (o["id"], O.DIFF_MASK, mask)]
+    rep, diffs = _run_gpu(torch_cuda, n_pcs, hobjs, recs, diff_modes=modes, **kw)
+    bad = parity.compare_with_oracle(rep, okeys, oglob, oobj)
+    for (oid, mode), gd in diffs.items():
+        mask = [m for (i, md, m) in modes if i == oid and md == mode][0]
+        od = O.snapshot_diff(cfg, hobjs, recs, oid, mode, mask)
+        bad += [f"obj {oid} mode {mode} " + s for s in parity.compare_diff(gd, od)]
+    assert not bad, "\n".join(bad[:40])
+    return rep, okeys
+
+
+def test_cfg1_parity(torch_cuda):
+    hobjs = W.host_objects(G.CFG1, 0, 1)
+    recs = G.records_host(G.CFG1, 0, 1, 0, 1 << 20)
+    rep, okeys = _check(torch_cuda, 16, hobjs, recs)
+    assert rep.keys["structured"][2] == 1 and rep.keys["approx"][5] == 1      # the cfg1 closed forms hold on GPU too
+
+
+@pytest.mark.parametrize("seed,n", [(1, 4096), (2, 65536), (3, 100003), (4, 300001)])
+def test_fuzz_parity(torch_cuda, seed, n):
+    hobjs = W.host_objects(G.FUZZ, 0, seed)
+    recs = G.records_host(G.FUZZ, 0, seed, 0, n)
+    _check(torch_cuda, 64, hobjs, recs)
+
+
+def test_fuzz_parity_topk_variants(torch_cuda):
+    hobjs = W.host_objects(G.FUZZ, 0, 9)
+    recs = G.records_host(G.FUZZ, 0, 9, 0, 50000)
+    for k in (1, 3, 64):
+        _check(torch_cuda, 64, hobjs, recs, topk=k)
+
+
+def test_chunk_and_permutation_invariance(torch_cuda):
+    """I10 / C12: chunked calls and shuffled records give the same report."""
+    seed, n = 5, 120007
+    hobjs = W.host_objects(G.FUZZ, 0, seed)
+    recs = G.records_host(G.FUZZ, 0, seed, 0, n)
+    cfg = O.make_config(64)
+    okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
+    rep, _ = _run_gpu(torch_cuda, 64, hobjs, recs, chunks=[1, 33, 1000, 1001, 50000, 99999])
+    assert not parity.compare_with_oracle(rep, okeys, oglob, oobj)
+    perm = np.random.default_rng(1).permutation(n)
+    rep, _ = _run_gpu(torch_cuda, 64, hobjs, recs[perm])
+    assert not parity.compare_with_oracle(rep, okeys, oglob, oobj)
+
+
+def test_local_merge(torch_cuda):
+    """ve_merge_stats(dst, src): merge(A, B) == analyze(A u B)."""
+    ve = _ve()
+    seed, n = 6, 80000
+    hobjs = W.host_objects(G.FUZZ, 0, seed)
+    recs = G.records_host(G.FUZZ, 0, seed, 0, n)
+    cfg = O.make_config(64)
+    okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
+    dobjs = W.device_objects(hobjs)
+    drec = W.device_records(recs)
+    a = ve.Context(n_pcs=64, max_objects=8, hist_capacity=1 << 20)
+    b = ve.Context(n_pcs=64, max_objects=8, hist_capacity=1 << 20)
+    a.set_objects(dobjs)
+    b.set_objects(dobjs)
+    a.analyze_records(drec[:30011 * 24], 30011)
+    b.analyze_records(drec[30011 * 24:], n - 30011)
+    a.merge(b)
+    bad = parity.compare_with_oracle(a.report(), okeys, oglob, oobj)
+    assert not bad, "\n".join(bad[:20])
+
+
+def test_dedup_parity(torch_cuda):
+    ve = _ve()
+    seed, unit = 3, 4096
+    n = 60
+    objs, hpost = [], []
+    for i in range(n):
+        o = G.dedup_object(seed, i, unit)
+        host = G.dedup_host(seed, i, unit)
+        hpost.append(host)
+        objs.append(o)
+    # adversaries: an all-zero object and its copy, a one-byte flip of a random one, a NULL post
+    hobjs = [dict(o, pre=None, post=hpost[i]) for i, o in enumerate(objs)]
+    hobjs[7] = dict(hobjs[7], post=None)
+    oracle_groups = O.object_dedup(hobjs)
+    import torch
+    dposts = [torch.from_numpy(h).cuda() if h is not None else None for h in [o["post"] for o in hobjs]]
+    dobjs = [dict(o, post=dposts[i], pre=None) for i, o in enumerate(hobjs)]
+    ctx = ve.Context(n_pcs=1, max_objects=1)
+    g = ctx.object_dedup(dobjs)
+    assert list(g) == list(oracle_groups)
+    assert len(set(g)) < n                                      # duplicates exist in the set
+
+
+def test_capacity_overflow_is_an_error(torch_cuda):
+    ve = _ve()
+    hobjs = W.host_objects(G.FUZZ, 0, 8)
+    recs = G.records_host(G.FUZZ, 0, 8, 0, 200000)
+    ctx = ve.Context(n_pcs=64, max_objects=8, hist_capacity=1024)
+    ctx.set_objects(W.device_objects(hobjs))
+    ctx.analyze_records(W.device_records(recs), len(recs))
+    with pytest.raises(ve.VeError) as ei:
+        ctx.report()
+    assert ei.value.status == ve.ERR_CAPACITY
+    with pytest.raises(ve.VeError) as ei:
+        ctx.analyze_records(W.device_records(recs[:10]), 10)
+    assert ei.value.status == ve.ERR_STATE
+    ctx.reset()                                                 # clears the poison
+
+
+def test_empty_and_tiny(torch_cuda):
+    hobjs = W.host_objects(G.FUZZ, 0, 12)
+    for n in (1, 2, 31, 32, 33):
+        recs = G.records_host(G.FUZZ, 0, 12, 7, n)
+        _check(torch_cuda, 64, hobjs, recs)
