@@ -168,7 +168,9 @@ __device__ __forceinline__ void apply_group(const AnalyzeParams& P, const Smem& 
 
   // C8 structured: group line state, merged into the key's state unless it already FAILed
   LineState* ls = (slot >= 0) ? &S.sline[slot] : &P.t.line[key];
-  if (*(volatile uint32_t*)&ls->state == VE_LINE_FAIL) return;
+  // the state may change under us (other warps merge concurrently): decide group-uniformly
+  const uint32_t cur = __shfl_sync(gm, *(volatile uint32_t*)&ls->state, __ffs(gm) - 1);
+  if (cur == VE_LINE_FAIL) return;
   LinePts g;
   if (__any_sync(gm, f.pfail)) {
     g.state = VE_LINE_FAIL;
