@@ -171,6 +171,9 @@ ve_status ve_report_globals(const ve_rep* r, ve_globals* out);
 /* format 0: binary (magic "VERP", header, then the arrays above); 1: JSON */
 ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
 
+/* Number of libve kernels launched by this process so far (all contexts). */
+uint64_t  ve_kernel_launches(void);
+
 /* NCCL helpers (NCCL is loaded at run time; only ve_merge_stats with a comm needs it) */
 ve_status ve_nccl_get_unique_id(void* out128);                          /* 128-byte ncclUniqueId */
 ve_status ve_nccl_comm_init(void** comm_out, int nranks, const void* id128, int rank);

@@ -1,22 +1,33 @@
 // k_analyze.cu -- K1: the fused record-analysis pass.
 //
-// One persistent CTA per SM streams 24-byte records (PC, address,
-// size, raw value per access) in warp windows of 32 consecutive records.
-// Per window each lane decodes one record, maps it to its data object
-// (P:L230), gathers and compares the pre-snapshot bytes (Def 3.1),
-// and derives the bit-level value tests of Defs 3.3-3.8.  Lanes
-// are then grouped by key (PC, object) with __match_any_sync and every group
-// is reduced with warp REDUX into per-CTA shared-memory stat rows, an
-// open-addressing shared-memory value histogram (overflow to the exact HBM
-// table), per-key line states (the (+) monoid) and the written / loaded
-// element bitmaps.  At the end each CTA folds its shared state into the
-// global tables.  All results are integer and order-free, hence identical for
-// any grid, chunking or rank split (C12).
+// One persistent CTA per SM (16 warps).  Every warp streams its own
+// CONTIGUOUS range of 24-byte records (PC, address, size, raw value per
+// access) in windows of 32, with the next two windows' loads in flight.  Per
+// window each lane decodes one record, maps it to its data object,
+// gathers and compares the pre-snapshot bytes (Def 3.1) and derives
+// the bit-level value tests of Defs 3.3-3.8.
+//
+//  * Fast path -- the valid lanes share (pc, access type, object), as a warp's
+//    memory instruction does: one set of warp REDUX reductions serves both the
+//    PC key and the object key, and is folded into lane-distributed register
+//    accumulators (2 key slots per warp, 16 fields each); rows in shared memory
+//    are only touched when a slot is evicted.
+//  * Slow path -- mixed windows: lanes grouped per key with __match_any_sync,
+//    each group reduced and folded into the shared rows directly.
+//  * Both paths: exact (pc, object, value) histogram (shared open addressing,
+//    overflow to HBM), per-key line states through a warp-private cache of the
+//    (+) monoid, written / loaded element bitmaps.
+// At exit each CTA folds its shared state into the global tables.  All results
+// are integer and order-free, so any grid, chunking or rank split gives the
+// same bits (C12).
 #include <cuda_runtime.h>
 
 #include "ve_internal.cuh"
 
 namespace ve {
+
+constexpr int K1_THREADS = 512;
+constexpr int K1_WARPS = K1_THREADS / 32;
 
 struct AnalyzeParams {
   const ve_record* recs;
@@ -103,7 +114,7 @@ __device__ __forceinline__ void atomic_max_u64(unsigned long long* p, unsigned l
 __device__ __forceinline__ uint64_t load_pre(uint64_t p, uint32_t lg) {
   uint32_t w = 1u << lg;
   if ((p & (w - 1)) == 0) {
-    if (lg == 0) return *(const uint8_t*)p;
+    if (lg == 0) return __ldg((const unsigned char*)p);
     if (lg == 1) return __ldg((const unsigned short*)p);
     if (lg == 2) return __ldg((const unsigned int*)p);
     return __ldg((const unsigned long long*)p);
@@ -113,7 +124,7 @@ __device__ __forceinline__ uint64_t load_pre(uint64_t p, uint32_t lg) {
   return v;
 }
 
-// per-lane record facts shared by the PC-key and object-key groups
+// per-lane record facts shared by the key groups
 struct Facts {
   uint64_t addr, val, ordv, truncv;
   __int128 y;
@@ -122,10 +133,49 @@ struct Facts {
   bool nan, isf, pfail;
 };
 
-// Reduce one key group (all lanes in gm share the key) and fold it into the
-// key's row: shared memory when slot >= 0, else the global table.
+// line state of the points of the lanes in gm (all valid, none pfail)
+__device__ __forceinline__ void group_line(unsigned gm, const Facts& f, LinePts& g) {
+  if (__any_sync(gm, f.pfail)) {
+    g.state = VE_LINE_FAIL;
+    g.px = g.qx = 0; g.py = g.qy = 0;
+    return;
+  }
+  const uint64_t minx = redmin64(gm, f.addr), maxx = redmax64(gm, f.addr);
+  const int pl = __ffs(__ballot_sync(gm, f.addr == minx)) - 1;
+  const int ql = __ffs(__ballot_sync(gm, f.addr == maxx)) - 1;
+  const uint64_t ylo = (uint64_t)f.y, yhi = (uint64_t)(f.y >> 64);
+  // |y| < 2^62 for every point: exact 64x64->128 products, else the generic 128-bit path
+  const bool fits = (yhi == (uint64_t)((int64_t)ylo >> 63)) && (ylo + (1ull << 62)) < (1ull << 63);
+  const bool small = __all_sync(gm, fits);
+  bool ok;
+  __int128 py, qy;
+  if (small) {
+    const int64_t py64 = (int64_t)__shfl_sync(gm, (unsigned long long)ylo, pl);
+    const int64_t qy64 = (int64_t)__shfl_sync(gm, (unsigned long long)ylo, ql);
+    py = (__int128)py64;
+    qy = (__int128)qy64;
+    if (minx == maxx) {
+      ok = (int64_t)ylo == py64;
+    } else {
+      const int64_t dxq = (int64_t)(maxx - minx), dx = (int64_t)(f.addr - minx);
+      const int64_t dy = (int64_t)ylo - py64, dq = qy64 - py64;
+      ok = (dy * dxq == dq * dx) && (__mul64hi(dy, dxq) == __mul64hi(dq, dx));
+    }
+  } else {
+    py = mk128(shfl64(gm, ylo, pl), (int64_t)shfl64(gm, yhi, pl));
+    qy = mk128(shfl64(gm, ylo, ql), (int64_t)shfl64(gm, yhi, ql));
+    if (minx == maxx) ok = (f.y == py);
+    else ok = collinear(minx, py, maxx, qy, f.addr, f.y);
+  }
+  ok = __all_sync(gm, ok);
+  g.state = !ok ? VE_LINE_FAIL : (minx == maxx ? VE_LINE_POINT : VE_LINE_LINE);
+  g.px = minx; g.py = py; g.qx = maxx; g.qy = qy;
+}
+
+// Slow path: reduce one key group (all lanes in gm share the key) and fold it into
+// the key's row: shared memory when slot >= 0, else the global table.
 __device__ __forceinline__ void apply_group(const AnalyzeParams& P, const Smem& S, unsigned gm, int slot,
-                                            uint32_t key, const Facts& f) {
+                                            uint32_t key, const Facts& f, LinePts& g) {
   const int lane = threadIdx.x & 31;
   const unsigned gsize = __popc(gm);
   const int rank = __popc(gm & lanemask_lt());
@@ -165,31 +215,77 @@ __device__ __forceinline__ void apply_group(const AnalyzeParams& P, const Smem& 
     if (slot >= 0) atomicAdd(&S.ssum[slot * NSUM + F_TYPE0 + f.tc], c);
     else atomicAdd(&P.t.sum[(uint64_t)key * NSUM + F_TYPE0 + f.tc], (unsigned long long)c);
   }
-
-  // C8 structured: group line state, merged into the key's state unless it already FAILed
+  // C8: the group's line state unless the key's CTA state already FAILed
+  g.state = VE_LINE_EMPTY;
   LineState* ls = (slot >= 0) ? &S.sline[slot] : &P.t.line[key];
   // the state may change under us (other warps merge concurrently): decide group-uniformly
   const uint32_t cur = __shfl_sync(gm, *(volatile uint32_t*)&ls->state, __ffs(gm) - 1);
   if (cur == VE_LINE_FAIL) return;
-  LinePts g;
-  if (__any_sync(gm, f.pfail)) {
-    g.state = VE_LINE_FAIL;
-    g.px = g.qx = 0; g.py = g.qy = 0;
-  } else {
-    const uint64_t minx = redmin64(gm, f.addr), maxx = redmax64(gm, f.addr);
-    const int pl = __ffs(__ballot_sync(gm, f.addr == minx)) - 1;
-    const int ql = __ffs(__ballot_sync(gm, f.addr == maxx)) - 1;
-    const uint64_t ylo = (uint64_t)f.y, yhi = (uint64_t)(f.y >> 64);
-    const __int128 py = mk128(shfl64(gm, ylo, pl), (int64_t)shfl64(gm, yhi, pl));
-    const __int128 qy = mk128(shfl64(gm, ylo, ql), (int64_t)shfl64(gm, yhi, ql));
-    bool ok;
-    if (minx == maxx) ok = (f.y == py);
-    else ok = collinear(minx, py, maxx, qy, f.addr, f.y);
-    ok = __all_sync(gm, ok);
-    g.state = !ok ? VE_LINE_FAIL : (minx == maxx ? VE_LINE_POINT : VE_LINE_LINE);
-    g.px = minx; g.py = py; g.qx = maxx; g.qy = qy;
+  group_line(gm, f, g);
+}
+
+// ---- warp-private line-state cache -------------------------------------------
+// Line merges are the only read-modify-write of a wide state; doing them under a
+// lock per window serialises warps on keys that stay collinear.  Each warp keeps
+// the last WC keys' states privately and folds them into the CTA state only on
+// eviction, on the first FAIL (so other warps skip the key early) and at exit.
+constexpr int WC = 4;
+struct WarpCache {
+  uint32_t key1[WC];   // key + 1, 0 = empty
+  int32_t slot[WC];
+  uint32_t next, pad;
+  LineState st[WC];
+};
+
+__device__ __forceinline__ LineState* line_target(const AnalyzeParams& P, const Smem& S, int slot, uint32_t key) {
+  return (slot >= 0) ? &S.sline[slot] : &P.t.line[key];
+}
+
+// returns the key's merged (warp-local) state
+__device__ __forceinline__ uint32_t wcache_merge(const AnalyzeParams& P, const Smem& S, WarpCache& C, uint32_t key,
+                                                 int slot, const LinePts& g) {
+  for (int i = 0; i < WC; ++i) {
+    if (C.key1[i] == key + 1) {
+      const LinePts a = line_load(C.st[i]);
+      const LinePts r = line_merge(a, g);
+      line_store(C.st[i], r);
+      if (r.state == VE_LINE_FAIL && a.state != VE_LINE_FAIL) line_merge_locked(line_target(P, S, slot, key), r);
+      return r.state;
+    }
   }
-  if (rank == 0) line_merge_locked(ls, g);
+  int v = -1;
+  for (int i = 0; i < WC; ++i)
+    if (C.key1[i] == 0) { v = i; break; }
+  if (v < 0) {
+    v = (int)(C.next++ % WC);
+    line_merge_locked(line_target(P, S, C.slot[v], C.key1[v] - 1), line_load(C.st[v]));
+  }
+  C.key1[v] = key + 1;
+  C.slot[v] = slot;
+  line_store(C.st[v], g);
+  if (g.state == VE_LINE_FAIL) line_merge_locked(line_target(P, S, slot, key), g);
+  return g.state;
+}
+
+__device__ __forceinline__ void wcache_flush(const AnalyzeParams& P, const Smem& S, WarpCache& C) {
+  for (int i = 0; i < WC; ++i) {
+    if (C.key1[i]) {
+      if (C.st[i].state != VE_LINE_FAIL) line_merge_locked(line_target(P, S, C.slot[i], C.key1[i] - 1), line_load(C.st[i]));
+      C.key1[i] = 0;
+    }
+  }
+}
+
+// serialise the merges of this window's group leaders through the warp cache
+__device__ __forceinline__ void merge_lines(const AnalyzeParams& P, const Smem& S, WarpCache& C, bool lead,
+                                            uint32_t key, int slot, const LinePts& g) {
+  unsigned L = __ballot_sync(0xFFFFFFFFu, lead && g.state != VE_LINE_EMPTY);
+  while (L) {
+    const int l = __ffs(L) - 1;
+    L &= L - 1;
+    if ((int)(threadIdx.x & 31) == l) wcache_merge(P, S, C, key, slot, g);
+    __syncwarp();
+  }
 }
 
 // Insert a group of equal (tag, bits) with count c: shared table first, HBM table on miss/full.
@@ -240,11 +336,84 @@ __device__ __forceinline__ void bitmap_or(uint32_t* bm, bool part, uint64_t word
   }
 }
 
-__global__ void __launch_bounds__(512, 1) k_analyze(AnalyzeParams P) {
+// ---- fast path: lane-distributed register accumulators -----------------------
+// Two key slots per warp; lane l holds field (l & 15) of slot (l >> 4):
+//  0 n   1 n_zero   2 n_eq_pre   3 n_nosnap   4 nan   5 nonint   6 not_f16   7 not_bf16
+//  8 not_f32   9 raw_min 10 raw_max 11 ord_min 12 ord_max 13 trunc_min 14 trunc_max
+// For w <= 4 the ord fields of signed types hold sext32(b)^2^31 (order-isomorphic),
+// converted to the 64-bit key at flush.
+struct FastSlots {
+  uint32_t pc[2], koi[2], meta[2];
+  uint32_t used, mru;
+  uint32_t lfail[2];     // bit0: PC key line FAIL, bit1: object key line FAIL (known to this warp)
+};
+
+__device__ __forceinline__ uint64_t fast_identity(int f) {
+  return (f >= 9 && (f & 1)) ? ~0ull : 0ull;
+}
+
+__device__ __forceinline__ void fold_row(const AnalyzeParams& P, const Smem& S, int slot, uint32_t key, int f,
+                                         uint32_t field, uint64_t v) {
+  if (f <= 8 || f == 15) {
+    if (slot >= 0) atomicAdd(&S.ssum[slot * NSUM + field], (uint32_t)v);
+    else atomicAdd(&P.t.sum[(uint64_t)key * NSUM + field], (unsigned long long)v);
+  } else {
+    const int m = (f - 9) >> 1;
+    if (f & 1) atomic_min_u64(slot >= 0 ? &S.smin[slot * NMM + m] : &P.t.mn[(uint64_t)key * NMM + m], v);
+    else atomic_max_u64(slot >= 0 ? &S.smax[slot * NMM + m] : &P.t.mx[(uint64_t)key * NMM + m], v);
+  }
+}
+
+// fold slot s's accumulators into the PC-key row and the object-key row (lanes of half s)
+__device__ __forceinline__ void fast_flush(const AnalyzeParams& P, const Smem& S, const FastSlots& F, int s,
+                                           uint64_t acc) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t nrec = __shfl_sync(0xFFFFFFFFu, acc, s * 16);   // field 0 of slot s
+  if ((lane >> 4) != s) return;
+  const int f = lane & 15;
+  const uint32_t meta = F.meta[s], lg = meta & 3u, kind = (meta >> 2) & 3u;
+  const bool st = meta_store(meta);
+  uint64_t v = (f == 15) ? nrec : acc;
+  if (v == fast_identity(f) && f != 15) return;
+  if (f == 15 && v == 0) return;
+  uint32_t field;
+  if (f == 0) field = st ? F_ST : F_LD;
+  else if (f == 1) field = F_ZERO;
+  else if (f == 2) field = st ? F_STEQ : F_LDEQ;
+  else if (f == 3) field = F_NOSNAP;
+  else if (f <= 8) field = F_NAN + (uint32_t)(f - 4);
+  else if (f == 15) field = F_TYPE0 + type_code(kind, lg);
+  else field = 0;
+  if ((f == 11 || f == 12) && kind == 1u && lg < 3u) {
+    const int32_t sv = (int32_t)((uint32_t)v ^ 0x80000000u);
+    v = (uint64_t)(int64_t)sv ^ (1ull << 63);
+  }
+  const uint32_t pc = F.pc[s], koi = F.koi[s];
+  fold_row(P, S, pc < P.sp ? (int)pc : -1, pc, f, field, v);
+  if (koi != KO_NONE) fold_row(P, S, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
+}
+
+struct Rec {
+  uint64_t addr, val, pm;
+};
+
+__device__ __forceinline__ Rec load_rec(const AnalyzeParams& P, uint64_t w, uint64_t wend, int lane) {
+  Rec r{0, 0, 0};
+  const uint64_t i = w * 32 + lane;
+  if (w < wend && i < P.n) {
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&P.recs[i]);
+    r.addr = __ldcs(q);
+    r.val = __ldcs(q + 1);
+    r.pm = __ldcs(q + 2);
+  }
+  return r;
+}
+
+__global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   const uint32_t nsk = P.sp + P.so;
   Smem S = carve(smem_raw, nsk, P.hs, P.objc);
-  const int tid = threadIdx.x, lane = tid & 31;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
   for (uint32_t i = tid; i < nsk * NSUM; i += blockDim.x) S.ssum[i] = 0;
   for (uint32_t i = tid; i < nsk * NMM; i += blockDim.x) { S.smin[i] = ~0ull; S.smax[i] = 0; }
@@ -254,26 +423,32 @@ __global__ void __launch_bounds__(512, 1) k_analyze(AnalyzeParams P) {
   }
   for (uint32_t i = tid; i < P.objc; i += blockDim.x) { S.sob[i] = P.o.base[i]; S.soe[i] = P.o.end[i]; }
   if (tid < 4) S.sctr[tid] = 0;
+  __shared__ WarpCache s_wc[K1_WARPS];
+  WarpCache& wc = s_wc[warp];
+  if (lane < WC) wc.key1[lane] = 0;
+  if (lane == 0) wc.next = 0;
   __syncthreads();
 
+  // this warp's contiguous range of windows
   const uint64_t nwin = (P.n + 31) / 32;
-  const uint64_t wstride = (uint64_t)gridDim.x * (blockDim.x / 32);
+  const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + warp;
+  const uint64_t wbeg = gw * nwin / tw, wend = (gw + 1) * nwin / tw;
   int ocache = -1;  // warp-uniform last object
   uint32_t n_invalid = 0, n_unmapped = 0;
+  FastSlots F;
+  F.used = 0;
+  F.mru = 0;
+  uint64_t acc = 0;
 
-  for (uint64_t w = (uint64_t)blockIdx.x * (blockDim.x / 32) + (tid >> 5); w < nwin; w += wstride) {
-    const uint64_t r = w * 32 + lane;
-    const bool inrange = r < P.n;
-    uint64_t addr = 0, val = 0;
-    uint32_t pc = 0, meta = 0;
-    if (inrange) {
-      const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&P.recs[r]);
-      addr = __ldcs(q);
-      val = __ldcs(q + 1);
-      const unsigned long long pm = __ldcs(q + 2);
-      pc = (uint32_t)pm;
-      meta = (uint32_t)(pm >> 32);
-    }
+  Rec ra = load_rec(P, wbeg, wend, lane), rb = load_rec(P, wbeg + 1, wend, lane);
+  for (uint64_t w = wbeg; w < wend; ++w) {
+    const Rec cur = ra;
+    ra = rb;
+    rb = load_rec(P, w + 2, wend, lane);
+    const uint64_t addr = cur.addr, val = cur.val;
+    const uint32_t pc = (uint32_t)cur.pm, meta = (uint32_t)(cur.pm >> 32);
+    const bool inrange = w * 32 + lane < P.n;
+
     // S1 decode + validate
     const bool valid = inrange && rec_valid(addr, val, pc, meta, P.n_pcs);
     const unsigned vmask = __ballot_sync(0xFFFFFFFFu, valid);
@@ -334,11 +509,12 @@ __global__ void __launch_bounds__(512, 1) k_analyze(AnalyzeParams P) {
           else b1 |= 1u << (e & 31);
         }
       }
-      bitmap_or(P.t.W, wpart, w0, b0);
+      const unsigned wany = __ballot_sync(0xFFFFFFFFu, wpart);
+      if (wany) bitmap_or(P.t.W, wpart, w0, b0);
       const bool spill = wpart && w1 != w0;
       if (__any_sync(0xFFFFFFFFu, spill)) bitmap_or(P.t.W, spill, w1, b1);
       const bool lpart = inside && !st && eq;
-      bitmap_or(P.t.L, lpart, w0, 1u << (e0 & 31));
+      if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, w0, 1u << (e0 & 31));
     }
 
     // per-record value tests (S4-S7)
@@ -358,40 +534,160 @@ __global__ void __launch_bounds__(512, 1) k_analyze(AnalyzeParams P) {
       const uint32_t sh64 = 64u - (8u << lg);
       f.y = (__int128)((int64_t)(val << sh64) >> sh64);
     } else f.y = (__int128)ival;
-    f.packA = (uint32_t)st | ((uint32_t)(val == 0) << 6) | ((uint32_t)(eq && !st) << 12) |
-              ((uint32_t)(eq && st) << 18) | ((uint32_t)(!eqdef) << 24);
-    f.packB = (ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) | (((ff >> 3) & 1u) << 18) |
-              (((ff >> 4) & 1u) << 24);
-
-    // PC-key groups
-    if (valid) {
-      const unsigned gm = __match_any_sync(vmask, pc);
-      apply_group(P, S, gm, pc < P.sp ? (int)pc : -1, pc, f);
-    }
-    // object-key groups (mapped global records, or the SHARED pseudo-object)
     const uint32_t koi = sh ? P.n_obj : (mapped ? oid : KO_NONE);
-    const bool opart = valid && koi != KO_NONE;
-    const unsigned omask = __ballot_sync(0xFFFFFFFFu, opart);
-    if (opart) {
-      const unsigned gm = __match_any_sync(omask, koi);
-      apply_group(P, S, gm, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f);
-    }
-    // S8 exact histogram on the composite (pc, object key) tag
-    if (valid) {
-      const uint32_t tag = (pc << 16) | (koi & 0xFFFFu);
-      const unsigned tg = __match_any_sync(vmask, tag);
-      const unsigned vg = __match_any_sync(tg, val);
-      if (lane == __ffs(vg) - 1) hist_insert(P, S, tag, val, __popc(vg));
+
+    // uniform window? (pc, access type and object shared by every valid lane)
+    const int l0 = __ffs(vmask) - 1;
+    const uint32_t pc0 = __shfl_sync(0xFFFFFFFFu, pc, l0);
+    const uint32_t meta0 = __shfl_sync(0xFFFFFFFFu, meta, l0);
+    const uint32_t koi0 = __shfl_sync(0xFFFFFFFFu, koi, l0);
+    const bool uniform = __all_sync(0xFFFFFFFFu, !valid || (pc == pc0 && meta == meta0 && koi == koi0));
+
+    if (uniform) {
+      // ---------------- fast path ----------------
+      // select / install the register slot for (pc, object key, access type)
+      int s;
+      if ((F.used & 1u) && F.pc[0] == pc0 && F.koi[0] == koi0 && F.meta[0] == meta0) s = 0;
+      else if ((F.used & 2u) && F.pc[1] == pc0 && F.koi[1] == koi0 && F.meta[1] == meta0) s = 1;
+      else {
+        s = !(F.used & 1u) ? 0 : !(F.used & 2u) ? 1 : (int)(F.mru ^ 1u);
+        if (F.used & (1u << s)) fast_flush(P, S, F, s, acc);
+        F.used |= 1u << s;
+        F.pc[s] = pc0; F.koi[s] = koi0; F.meta[s] = meta0;
+        if ((lane >> 4) == s) acc = fast_identity(lane & 15);
+        // line states this warp can skip (already FAIL in the CTA state)
+        const int ps = pc0 < P.sp ? (int)pc0 : -1;
+        uint32_t lf = (line_target(P, S, ps, pc0)->state == VE_LINE_FAIL) ? 1u : 0u;
+        if (koi0 == KO_NONE) lf |= 2u;
+        else {
+          const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
+          if (line_target(P, S, os, P.n_pcs + koi0)->state == VE_LINE_FAIL) lf |= 2u;
+        }
+        F.lfail[s] = __shfl_sync(0xFFFFFFFFu, lf, 0);
+      }
+      F.mru = (uint32_t)s;
+      const uint32_t nv = __popc(vmask);
+      const uint32_t pA = valid ? ((uint32_t)(val == 0) | ((uint32_t)eq << 6) | ((uint32_t)!eqdef << 12)) : 0u;
+      const uint32_t A = __reduce_add_sync(0xFFFFFFFFu, pA);
+      uint32_t B = 0;
+      uint64_t rmin, rmax, omin, omax, tmin = ~0ull, tmax = 0;
+      const bool okv = valid && !f.nan;            // contributes to ord / trunc
+      // branch only on the WINDOW's access type (invalid lanes may carry any meta)
+      const uint32_t lg0 = meta0 & 3u, kind0 = (meta0 >> 2) & 3u;
+      const bool isf0 = kind0 >= 2u;
+      if (isf0) {
+        const uint32_t pB = valid ? ((ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) |
+                                     (((ff >> 3) & 1u) << 18) | (((ff >> 4) & 1u) << 24)) : 0u;
+        B = __reduce_add_sync(0xFFFFFFFFu, pB);
+      }
+      if (lg0 < 3u) {
+        // w <= 4 bytes: every key fits 32 bits -> one REDUX per min / max
+        const uint32_t r32 = (uint32_t)val;
+        rmin = __reduce_min_sync(0xFFFFFFFFu, valid ? r32 : 0xFFFFFFFFu);
+        rmax = __reduce_max_sync(0xFFFFFFFFu, valid ? r32 : 0u);
+        if (kind0 == 0u) {
+          omin = rmin; omax = rmax;
+        } else {
+          const uint32_t k32 = (kind0 == 1u) ? ((uint32_t)f.y ^ 0x80000000u) : (uint32_t)f.ordv;
+          const unsigned okm = __ballot_sync(0xFFFFFFFFu, okv);
+          omin = __reduce_min_sync(0xFFFFFFFFu, okv ? k32 : 0xFFFFFFFFu);
+          omax = __reduce_max_sync(0xFFFFFFFFu, okv ? k32 : 0u);
+          if (isf0) {
+            tmin = __reduce_min_sync(0xFFFFFFFFu, okv ? (uint32_t)f.truncv : 0xFFFFFFFFu);
+            tmax = __reduce_max_sync(0xFFFFFFFFu, okv ? (uint32_t)f.truncv : 0u);
+          }
+          if (okm == 0) { omin = ~0ull; omax = 0; tmin = ~0ull; tmax = 0; }
+        }
+      } else {
+        rmin = redmin64(0xFFFFFFFFu, valid ? val : ~0ull);
+        rmax = redmax64(0xFFFFFFFFu, valid ? val : 0ull);
+        omin = redmin64(0xFFFFFFFFu, okv ? f.ordv : ~0ull);
+        omax = redmax64(0xFFFFFFFFu, okv ? f.ordv : 0ull);
+        if (isf0) {
+          tmin = redmin64(0xFFFFFFFFu, okv ? f.truncv : ~0ull);
+          tmax = redmax64(0xFFFFFFFFu, okv ? f.truncv : 0ull);
+        }
+      }
+      if ((lane >> 4) == s) {
+        const int fl = lane & 15;
+        if (fl == 0) acc += nv;
+        else if (fl <= 3) acc += (A >> (6 * (fl - 1))) & 63u;
+        else if (fl <= 8) acc += (B >> (6 * (fl - 4))) & 63u;
+        else if (fl <= 14) {
+          const int m = (fl - 9) >> 1;
+          if (fl & 1) {
+            const uint64_t v = m == 0 ? rmin : m == 1 ? omin : tmin;
+            acc = v < acc ? v : acc;
+          } else {
+            const uint64_t v = m == 0 ? rmax : m == 1 ? omax : tmax;
+            acc = v > acc ? v : acc;
+          }
+        }
+      }
+      // C8: one line state for the window, merged into each key not yet FAIL
+      if (F.lfail[s] != 3u) {
+        LinePts g;
+        g.state = VE_LINE_EMPTY;
+        if (valid) group_line(vmask, f, g);
+        const int ps = pc0 < P.sp ? (int)pc0 : -1;
+        const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
+        uint32_t lf = F.lfail[s];
+        if (lane == l0) {
+          if (!(lf & 1u) && wcache_merge(P, S, wc, pc0, ps, g) == VE_LINE_FAIL) lf |= 1u;
+          if (!(lf & 2u) && wcache_merge(P, S, wc, P.n_pcs + koi0, os, g) == VE_LINE_FAIL) lf |= 2u;
+        }
+        __syncwarp();
+        F.lfail[s] = __shfl_sync(0xFFFFFFFFu, lf, l0);
+      }
+      // S8: exact histogram, one insert per distinct value
+      if (valid) {
+        const unsigned vg = (lg0 < 3u) ? __match_any_sync(vmask, (uint32_t)val) : __match_any_sync(vmask, val);
+        if (lane == __ffs(vg) - 1) hist_insert(P, S, (pc0 << 16) | (koi0 & 0xFFFFu), val, __popc(vg));
+      }
+    } else {
+      // ---------------- slow path: per-key groups ----------------
+      f.packA = (uint32_t)st | ((uint32_t)(val == 0) << 6) | ((uint32_t)(eq && !st) << 12) |
+                ((uint32_t)(eq && st) << 18) | ((uint32_t)(!eqdef) << 24);
+      f.packB = (ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) | (((ff >> 3) & 1u) << 18) |
+                (((ff >> 4) & 1u) << 24);
+      LinePts gp, go;
+      gp.state = go.state = VE_LINE_EMPTY;
+      bool leadp = false, leado = false;
+      const int pslot = pc < P.sp ? (int)pc : -1;
+      if (valid) {
+        const unsigned gm = __match_any_sync(vmask, pc);
+        apply_group(P, S, gm, pslot, pc, f, gp);
+        leadp = lane == __ffs(gm) - 1;
+      }
+      const bool opart = valid && koi != KO_NONE;
+      const unsigned omask = __ballot_sync(0xFFFFFFFFu, opart);
+      const int oslot = koi < P.so ? (int)(P.sp + koi) : -1;
+      if (opart) {
+        const unsigned gm = __match_any_sync(omask, koi);
+        apply_group(P, S, gm, oslot, P.n_pcs + koi, f, go);
+        leado = lane == __ffs(gm) - 1;
+      }
+      merge_lines(P, S, wc, leadp, pc, pslot, gp);
+      merge_lines(P, S, wc, leado, P.n_pcs + koi, oslot, go);
+      if (valid) {
+        const uint32_t tag = (pc << 16) | (koi & 0xFFFFu);
+        const unsigned tg = __match_any_sync(vmask, tag);
+        const unsigned vg = __match_any_sync(tg, val);
+        if (lane == __ffs(vg) - 1) hist_insert(P, S, tag, val, __popc(vg));
+      }
     }
   }
 
+  // fold the warp's register slots and line cache, then the CTA's shared state
+  if (F.used & 1u) fast_flush(P, S, F, 0, acc);
+  if (F.used & 2u) fast_flush(P, S, F, 1, acc);
   if (lane == 0) {
     if (n_invalid) atomicAdd(&S.sctr[0], n_invalid);
     if (n_unmapped) atomicAdd(&S.sctr[1], n_unmapped);
+    wcache_flush(P, S, wc);
   }
   __syncthreads();
 
-  // fold the CTA's shared state into the global tables
   for (uint32_t i = tid; i < nsk * NSUM; i += blockDim.x) {
     const uint32_t v = S.ssum[i];
     if (v) {
@@ -442,16 +738,17 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   int dev_smem = 0;
   cudaDeviceGetAttribute(&dev_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device);
   uint32_t hs = 8192;
-  while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > (size_t)dev_smem - 1024) hs >>= 1;
+  while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > (size_t)dev_smem - 8192) hs >>= 1;
   P.hs = hs;
   const size_t sb = smem_bytes(sp + so, hs, P.objc);
   cudaError_t e = cudaFuncSetAttribute(k_analyze, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
   if (e != cudaSuccess) return cuda_fail(c, e, "cudaFuncSetAttribute(k_analyze)");
   if (n == 0) return VE_OK;
   uint64_t windows = (n + 31) / 32;
-  uint64_t blocks = (windows + 15) / 16;
+  uint64_t blocks = (windows + K1_WARPS - 1) / K1_WARPS;
   if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
-  k_analyze<<<(unsigned)blocks, 512, sb, s>>>(P);
+  count_launch();
+  k_analyze<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze launch");
   return VE_OK;

@@ -109,6 +109,7 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
   gx = std::min<uint64_t>(std::max<uint64_t>(gx / 4, 1), 1024);
   for (size_t y0 = 0; y0 < hj.size(); y0 += 65535) {
     const unsigned gy = (unsigned)std::min<size_t>(65535, hj.size() - y0);
+    count_launch();
     k_hash<<<dim3((unsigned)gx, gy), 256, 0, s>>>(d_jobs + y0, d_hash + y0);
   }
   std::vector<unsigned long long> h(hj.size());
@@ -151,6 +152,7 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
     cudaMemsetAsync(d_diff, 0, pairs.size() * 4, s);
     for (size_t j0 = 0; j0 < jobs.size(); j0 += (1u << 30)) {
       const unsigned gxx = (unsigned)std::min<size_t>(jobs.size() - j0, 1u << 30);
+      count_launch();
       k_compare<<<gxx, 256, 0, s>>>(d_cj + j0, d_diff);
     }
     std::vector<unsigned int> diff(pairs.size());

@@ -128,6 +128,7 @@ ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask
       uint64_t blocks = (nvec + 255) / 256;
       const uint64_t cap = (uint64_t)c->num_sms * 8;
       if (blocks > cap) blocks = cap;
+      count_launch();
       k_diff_vec<<<(unsigned)blocks, 256, 0, s>>>((const uint4*)o.pre, (const uint4*)o.post, nvec, ew_lg, mask,
                                                  d_out);
     }
@@ -137,6 +138,7 @@ ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask
     const uint64_t rem = o.n_elems - e_begin;
     uint64_t blocks = (rem + 255) / 256;
     if (blocks > (uint64_t)c->num_sms * 8) blocks = (uint64_t)c->num_sms * 8;
+    count_launch();
     k_diff_scalar<<<(unsigned)blocks, 256, 0, s>>>((const uint8_t*)o.pre, (const uint8_t*)o.post, o.size, o.ew,
                                                   e_begin, o.n_elems, mask, d_out);
   }

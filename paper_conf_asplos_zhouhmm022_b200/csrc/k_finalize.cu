@@ -172,6 +172,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   uint64_t occ = 0;
   {
     unsigned long long* d_cnt = d_small + 1;
+    count_launch();
     k_occupancy<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->hcap, d_cnt);
     unsigned long long h_cnt = 0;
     e = cudaMemcpyAsync(&h_cnt, d_cnt, 8, cudaMemcpyDeviceToHost, s);
@@ -203,8 +204,10 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   cudaMemsetAsync(vc, 0, vcap * 8, s);
   cudaMemsetAsync(d_nd, 0, (size_t)nk * 8 * 3, s);
   const int grid = c->num_sms * 4;
+  count_launch();
   k_views<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, c->cfg.n_pcs, vs, vc, vmask, d_small,
                                d_small + 1);
+  count_launch();
   k_view_count<<<grid, 256, 0, s>>>(vs, vcap, d_nd);
   e = cudaMemcpyAsync(ndistinct.data(), d_nd, (size_t)nk * 8, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
@@ -213,6 +216,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   uint64_t acc = 0;
   for (uint32_t k = 0; k < nk; ++k) { off[k] = acc; acc += ndistinct[k]; }
   cudaMemcpyAsync(d_off, off.data(), (size_t)nk * 8, cudaMemcpyHostToDevice, s);
+  count_launch();
   k_view_scatter<<<grid, 256, 0, s>>>(vs, vc, vcap, d_off, d_cur, gb[0], gc[0]);
 
   // selection levels
@@ -249,6 +253,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
       if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize chunks"); }
     }
     cudaMemcpyAsync(d_chunks, chunks.data(), chunks.size() * sizeof(Chunk), cudaMemcpyHostToDevice, s);
+    count_launch();
     k_topk_chunk<<<(unsigned)chunks.size(), TK_THREADS, 0, s>>>(d_chunks, gb[cur], gc[cur], gb[1 - cur],
                                                                 gc[1 - cur]);
     cur = 1 - cur;
@@ -320,6 +325,7 @@ ve_status bitmap_counts(ve_ctx* c, cudaStream_t s, std::vector<ve_obj_stats>& ou
   uint64_t gx = (maxw + 255) / 256;
   if (gx > 64) gx = 64;
   if (gx == 0) gx = 1;
+  count_launch();
   k_bitmap_counts<<<dim3((unsigned)gx, n), 256, 0, s>>>(c->t.W, c->t.L, d_off, d_off + n, d_out);
   std::vector<unsigned long long> h(3 * n);
   cudaMemcpyAsync(h.data(), d_out, 3 * n * 8, cudaMemcpyDeviceToHost, s);

@@ -46,7 +46,9 @@ ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s) {
         dst->objs[i].ew != src->objs[i].ew || dst->objs[i].id != src->objs[i].id)
       return fail(dst, VE_ERR_INVALID, "ve_merge_stats: object tables differ");
   const int grid = dst->num_sms * 4;
+  count_launch();
   k_merge_tables<<<grid, 256, 0, s>>>(dst->t, src->t, dst->n_keys, dst->bm_words);
+  count_launch();
   k_merge_hist<<<grid, 256, 0, s>>>(dst->t, src->t.hslot, src->t.hcount, src->hcap);
   cudaError_t e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(dst, e, "ve_merge_stats (local)");

@@ -11,7 +11,12 @@
 
 #include "ve_internal.cuh"
 
+#include <atomic>
+
 namespace ve {
+
+static std::atomic<unsigned long long> g_launches{0};
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 
 ve_status fail(ve_ctx* c, ve_status s, const std::string& msg) {
   if (c) c->err = msg;
@@ -163,6 +168,14 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
   cudaError_t e = cudaSetDevice(cuda_device);
   if (e != cudaSuccess) { delete c; return VE_ERR_CUDA; }
   cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  {
+    // keep stream-ordered scratch allocations cached in the pool across synchronizations
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, cuda_device) == cudaSuccess) {
+      uint64_t thr = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
   uint64_t hcap = 1024;
   while (hcap < cfg->hist_capacity) hcap <<= 1;
   c->hcap = hcap;
@@ -426,6 +439,7 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
 }
 
 void ve_report_free(ve_rep* r) { delete r; }
+uint64_t ve_kernel_launches(void) { return g_launches.load(std::memory_order_relaxed); }
 uint32_t ve_report_n_keys(const ve_rep* r) { return r ? r->n_keys : 0; }
 uint32_t ve_report_n_objects(const ve_rep* r) { return r ? r->n_obj : 0; }
 uint32_t ve_report_topk(const ve_rep* r) { return r ? r->topk : 0; }

@@ -6,6 +6,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <cstdio>
 
 #include <string>
 #include <vector>
@@ -133,6 +134,7 @@ ve_status run_diff(ve_ctx* c, uint32_t obj_index, uint32_t mode, const uint32_t*
 ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* group_of, cudaStream_t s);
 ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s);
 ve_status merge_nccl(ve_ctx* c, void* comm, cudaStream_t s);
+void count_launch();  // process-wide kernel launch counter (ve_kernel_launches)
 }  // namespace ve
 
 // ============================================================================
@@ -380,7 +382,15 @@ __device__ __forceinline__ LinePts line_merge(LinePts a, const LinePts& b) {
 // merge b into *s under the state's spin lock (global or shared)
 __device__ __forceinline__ void line_merge_locked(LineState* s, const LinePts& b) {
   if (b.state == VE_LINE_EMPTY) return;
-  while (atomicCAS(&s->lock, 0u, 1u) != 0u) { __nanosleep(20); }
+  uint32_t spins = 0;
+  while (atomicCAS(&s->lock, 0u, 1u) != 0u) {
+    __nanosleep(20);
+    if (++spins == (1u << 26)) {  // a lost lock is a bug: fail loudly instead of hanging
+      printf("libve: line-state lock %p stuck (state %u lock %u) block %d thread %d\n", (void*)s, s->state, s->lock,
+             blockIdx.x, threadIdx.x);
+      __trap();
+    }
+  }
   __threadfence();
   volatile LineState* vs = s;
   LinePts a;

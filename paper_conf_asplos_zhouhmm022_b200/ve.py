@@ -85,6 +85,7 @@ def lib():
             "ve_report_objects": ([vp, vp], st),
             "ve_report_globals": ([vp, vp], st),
             "ve_report_dump": ([vp, ctypes.c_char_p, i32], st),
+            "ve_kernel_launches": ([], u64),
             "ve_nccl_get_unique_id": ([vp], st),
             "ve_nccl_comm_init": ([ctypes.POINTER(vp), i32, vp, i32], st),
             "ve_nccl_comm_destroy": ([vp], st),
@@ -122,6 +123,11 @@ def _stream(stream):
     if isinstance(stream, int):
         return stream
     return stream.cuda_stream
+
+
+def kernel_launches():
+    """libve kernels launched by this process so far (ve_kernel_launches)."""
+    return lib().ve_kernel_launches()
 
 
 class Report:
