@@ -26,7 +26,7 @@
 
 namespace ve {
 
-constexpr int K1_THREADS = 512;
+constexpr int K1_THREADS = 384;  // 12 warps x <=168 registers: the fast path runs spill-free
 constexpr int K1_WARPS = K1_THREADS / 32;
 
 struct AnalyzeParams {
@@ -37,6 +37,7 @@ struct AnalyzeParams {
   uint32_t mant_bits;
   uint32_t hs;              // shared histogram slots (power of 2)
   uint32_t objc;            // objects cached in shared memory (0 = use global table)
+  uint32_t dense_ok;        // dense per-element counting enabled for this launch
   DevObjects o;
   DevTables t;
 };
@@ -346,7 +347,29 @@ struct FastSlots {
   uint32_t pc[2], koi[2], meta[2];
   uint32_t used, mru;
   uint32_t lfail[2];     // bit0: PC key line FAIL, bit1: object key line FAIL (known to this warp)
+  unsigned long long dense[2];  // per-element counters of this (pc, object), or 0
 };
+
+// claim (or find) a dense counter array of sorted object oi for pc (lane 0), broadcast
+__device__ __forceinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t pc) {
+  unsigned long long dp = 0;
+  if ((threadIdx.x & 31) == 0) {
+    for (int j = 0; j < DENSE_PER_OBJ; ++j) {
+      uint32_t* slot = &P.o.dense_pc[DENSE_PER_OBJ * oi + j];
+      uint32_t d = *(volatile uint32_t*)slot;
+      if (d == DENSE_OFF) break;
+      if (d == DENSE_FREE) {
+        d = atomicCAS(slot, DENSE_FREE, pc);
+        if (d == DENSE_FREE) d = pc;
+      }
+      if (d == pc) {
+        dp = (unsigned long long)(P.o.dense_pool + P.o.dense_off[DENSE_PER_OBJ * oi + j]);
+        break;
+      }
+    }
+  }
+  return __shfl_sync(0xFFFFFFFFu, dp, 0);
+}
 
 __device__ __forceinline__ uint64_t fast_identity(int f) {
   return (f >= 9 && (f & 1)) ? ~0ull : 0ull;
@@ -564,6 +587,9 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
           if (line_target(P, S, os, P.n_pcs + koi0)->state == VE_LINE_FAIL) lf |= 2u;
         }
         F.lfail[s] = __shfl_sync(0xFFFFFFFFu, lf, 0);
+        // dense per-element counting for loads of a real object that read the pre value
+        const int oi0 = __shfl_sync(0xFFFFFFFFu, oi, l0);
+        F.dense[s] = (P.dense_ok && oi0 >= 0 && !meta_store(meta0)) ? dense_lookup(P, oi0, pc0) : 0ull;
       }
       F.mru = (uint32_t)s;
       const uint32_t nv = __popc(vmask);
@@ -639,9 +665,15 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
         __syncwarp();
         F.lfail[s] = __shfl_sync(0xFFFFFFFFu, lf, l0);
       }
-      // S8: exact histogram, one insert per distinct value
-      if (valid) {
-        const unsigned vg = (lg0 < 3u) ? __match_any_sync(vmask, (uint32_t)val) : __match_any_sync(vmask, val);
+      // S8: exact histogram.  A load that reads an unchanged whole element carries the
+      // pre-snapshot value of that element, so it is counted per element (a coalesced
+      // counter increment) and mapped to its value at report time; every other record
+      // is inserted per distinct value.
+      const bool dl = F.dense[s] != 0ull && eq && lg == ew_lg && (off & ((1ull << ew_lg) - 1)) == 0;
+      if (dl) atomicAdd(reinterpret_cast<uint32_t*>(F.dense[s]) + (off >> ew_lg), 1u);
+      const unsigned hmask = __ballot_sync(0xFFFFFFFFu, valid && !dl);
+      if (valid && !dl) {
+        const unsigned vg = (lg0 < 3u) ? __match_any_sync(hmask, (uint32_t)val) : __match_any_sync(hmask, val);
         if (lane == __ffs(vg) - 1) hist_insert(P, S, (pc0 << 16) | (koi0 & 0xFFFFu), val, __popc(vg));
       }
     } else {
@@ -725,6 +757,9 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.n_pcs = c->cfg.n_pcs;
   P.n_obj = c->n_obj;
   P.mant_bits = c->cfg.mant_bits;
+  // u32 per-element counters cannot overflow while the ctx has seen < 2^32 records
+  P.dense_ok = (c->dense_used > 0 && c->records_analyzed + n < (1ull << 32)) ? 1u : 0u;
+  c->records_analyzed += n;
   // shared stat rows: up to 256 keys, PCs first then object keys (incl. SHARED)
   const uint32_t NSK_MAX = 256;
   uint32_t so = c->n_obj + 1 < 128 ? c->n_obj + 1 : 128;

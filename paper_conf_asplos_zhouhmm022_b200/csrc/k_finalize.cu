@@ -280,6 +280,59 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   return VE_OK;
 }
 
+// ---- dense per-element counts -> exact histogram ------------------------------
+// A dense counter cnt[e] of (pc, object) counts loads that read element e's unchanged
+// pre-snapshot value, so it contributes cnt[e] occurrences of that value (C9).
+__global__ void k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre, uint32_t ew, uint32_t tag,
+                              DevTables t) {
+  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < n_elems;
+       e += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t k = cnt[e];
+    if (!k) continue;
+    cnt[e] = 0;
+    const uint8_t* p = pre + e * ew;
+    uint64_t bits = 0;
+    if (((uintptr_t)p & (ew - 1)) == 0) {
+      bits = ew == 1 ? *p : ew == 2 ? *(const uint16_t*)p : ew == 4 ? *(const uint32_t*)p : *(const uint64_t*)p;
+    } else {
+      for (uint32_t i = 0; i < ew; ++i) bits |= (uint64_t)p[i] << (8 * i);
+    }
+    hist_insert_global(t, tag, bits, k);
+  }
+}
+
+ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
+  if (!c->dense_used || !c->n_obj) return VE_OK;
+  std::vector<uint32_t> dpc((size_t)DENSE_PER_OBJ * c->n_obj);
+  cudaError_t e = cudaMemcpyAsync(dpc.data(), c->o.dense_pc, dpc.size() * 4, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush");
+  bool any = false;
+  for (uint32_t i = 0; i < c->n_obj; ++i) {
+    for (int j = 0; j < DENSE_PER_OBJ; ++j) {
+      const uint32_t pc = dpc[DENSE_PER_OBJ * i + j];
+      if (pc == DENSE_FREE || pc == DENSE_OFF) continue;
+      const HostObject& o = c->objs[i];
+      uint64_t blocks = (o.n_elems + 255) / 256;
+      if (blocks > (uint64_t)c->num_sms * 8) blocks = (uint64_t)c->num_sms * 8;
+      count_launch();
+      k_dense_flush<<<(unsigned)blocks, 256, 0, s>>>((uint32_t*)c->dense_pool + c->dense_off_h[DENSE_PER_OBJ * i + j],
+                                                    o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, c->t);
+      any = true;
+    }
+  }
+  if (!any) return VE_OK;
+  unsigned long long glob[8];
+  e = cudaMemcpyAsync(glob, c->t.glob, sizeof(glob), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush");
+  if (glob[G_OVERFLOW]) {
+    c->poisoned = true;
+    return fail(c, VE_ERR_CAPACITY, "value histogram capacity exceeded (hist_capacity)");
+  }
+  return VE_OK;
+}
+
 // ---- K6: bitmap popcounts -------------------------------------------------
 __global__ void k_bitmap_counts(const uint32_t* W, const uint32_t* L, const uint64_t* bmoff, const uint64_t* nwords,
                                 unsigned long long* out /* [n][3] */) {

@@ -45,6 +45,11 @@ ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s) {
     if (dst->objs[i].base != src->objs[i].base || dst->objs[i].size != src->objs[i].size ||
         dst->objs[i].ew != src->objs[i].ew || dst->objs[i].id != src->objs[i].id)
       return fail(dst, VE_ERR_INVALID, "ve_merge_stats: object tables differ");
+  // dense per-element counts move into each side's exact histogram first
+  ve_status st = dense_flush(dst, s);
+  if (st != VE_OK) return st;
+  st = dense_flush(const_cast<ve_ctx*>(src), s);
+  if (st != VE_OK) return fail(dst, st, "ve_merge_stats: src: " + src->err);
   const int grid = dst->num_sms * 4;
   count_launch();
   k_merge_tables<<<grid, 256, 0, s>>>(dst->t, src->t, dst->n_keys, dst->bm_words);

@@ -39,6 +39,7 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->t.hcount);
   cudaFree(c->obj_block);
   cudaFree(c->scratch);
+  cudaFree(c->dense_pool);
   for (int i = 0; i < 2; ++i) {
     if (c->stage[i]) cudaFree(c->stage[i]);
     if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);
@@ -57,6 +58,10 @@ ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
     cudaMemsetAsync(c->t.L, 0, c->bm_words * 4, s);
   }
   cudaMemsetAsync(c->t.hslot, 0xFF, c->hcap * sizeof(HSlot), s);
+  if (c->dense_used) cudaMemsetAsync(c->dense_pool, 0, c->dense_used * 4, s);
+  if (c->n_obj)
+    cudaMemcpyAsync(c->o.dense_pc, c->dense_pc_init.data(), 4ull * DENSE_PER_OBJ * c->n_obj, cudaMemcpyHostToDevice, s);
+  c->records_analyzed = 0;
   cudaError_t e = cudaMemsetAsync(c->t.hcount, 0, c->hcap * 8, s);
   if (e != cudaSuccess) return cuda_fail(c, e, "reset");
   c->poisoned = false;
@@ -254,32 +259,69 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     }
   }
   c->bm_words = words;
+  // dense per-element counters: DENSE_PER_OBJ arrays per object with a pre snapshot,
+  // smallest objects first, within a budget of 2^30 counters (4 GiB)
+  const uint64_t DENSE_BUDGET = 1ull << 30;
+  std::vector<uint32_t> order(n);
+  for (uint32_t i = 0; i < n; ++i) order[i] = i;
+  std::sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return v[a].n_elems < v[b].n_elems; });
+  c->dense_off_h.assign((size_t)DENSE_PER_OBJ * n, ~0ull);
+  c->dense_pc_init.assign((size_t)DENSE_PER_OBJ * n, DENSE_OFF);
+  uint64_t dense = 0;
+  for (uint32_t i : order) {
+    if (!v[i].pre || dense + DENSE_PER_OBJ * v[i].n_elems > DENSE_BUDGET) continue;
+    for (int j = 0; j < DENSE_PER_OBJ; ++j) {
+      c->dense_off_h[DENSE_PER_OBJ * i + j] = dense;
+      c->dense_pc_init[DENSE_PER_OBJ * i + j] = DENSE_FREE;
+      dense += v[i].n_elems;
+    }
+  }
+  if (dense > c->dense_cap) {
+    cudaFree(c->dense_pool);
+    c->dense_pool = nullptr;
+    c->dense_cap = 0;
+    if (cudaMalloc(&c->dense_pool, dense * 4) != cudaSuccess) {
+      cudaGetLastError();
+      dense = 0;                                       // no memory: everything goes to the hash path
+      std::fill(c->dense_pc_init.begin(), c->dense_pc_init.end(), DENSE_OFF);
+    } else {
+      c->dense_cap = dense;
+    }
+  }
+  c->dense_used = dense;
   // device object table (SoA, sorted by base)
   cudaFree(c->obj_block);
   c->obj_block = nullptr;
-  const size_t nb = (size_t)(n ? n : 1) * (8 * 4 + 4 * 2) + 64;
+  const size_t nn = n ? n : 1;
+  const size_t nb = nn * (8 * 4 + 8 * DENSE_PER_OBJ + 4 * 2 + 4 * DENSE_PER_OBJ) + 64;
   if (cudaMalloc(&c->obj_block, nb) != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "objects"); }
   std::vector<uint8_t> host(nb, 0);
   uint64_t* hb = (uint64_t*)host.data();
   uint64_t* he = hb + n;
   uint64_t* hp = he + n;
   uint64_t* hm = hp + n;
-  uint32_t* hid = (uint32_t*)(hm + n);
+  uint64_t* hdo = hm + n;
+  uint32_t* hid = (uint32_t*)(hdo + DENSE_PER_OBJ * n);
   uint32_t* hew = hid + n;
+  uint32_t* hdp = hew + n;
   c->sorted_of_id.assign(n, 0);
   for (uint32_t i = 0; i < n; ++i) {
     hb[i] = v[i].base; he[i] = v[i].base + v[i].size; hp[i] = v[i].pre; hm[i] = v[i].bmoff;
     hid[i] = v[i].id; hew[i] = v[i].ew;
     c->sorted_of_id[v[i].id] = i;
   }
+  for (size_t k = 0; k < (size_t)DENSE_PER_OBJ * n; ++k) { hdo[k] = c->dense_off_h[k]; hdp[k] = c->dense_pc_init[k]; }
   cudaMemcpy(c->obj_block, host.data(), nb, cudaMemcpyHostToDevice);
   uint64_t* db = (uint64_t*)c->obj_block;
   c->o.base = db;
   c->o.end = db + n;
   c->o.pre = db + 2 * n;
   c->o.bmoff = db + 3 * n;
-  c->o.id = (const uint32_t*)(db + 4 * n);
+  c->o.dense_off = db + 4 * n;
+  c->o.id = (const uint32_t*)(db + 4 * n + DENSE_PER_OBJ * n);
   c->o.ew = c->o.id + n;
+  c->o.dense_pc = const_cast<uint32_t*>(c->o.ew + n);
+  c->o.dense_pool = (uint32_t*)c->dense_pool;
   c->o.n = n;
   c->objs = v;
   c->n_obj = n;
@@ -396,6 +438,8 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
     nd = c->merged_ndistinct;
     r->top = c->merged_topk;
   } else {
+    st = dense_flush(c, 0);
+    if (st != VE_OK) { delete r; return st; }
     st = finalize_hist(c, 0, nd, r->top);
     if (st != VE_OK) { delete r; return st; }
   }

@@ -70,8 +70,17 @@ struct DevObjects {          // sorted by base
   const uint32_t* ew;
   const uint64_t* pre;       // device pointers as integers (0 = none)
   const uint64_t* bmoff;     // first bitmap word of the object
+  // dense per-element access counters for loads that read the pre value
+  // (2 arrays per object, each claimed by one PC): dense_pc[2*i+j] = claimed pc,
+  // DENSE_FREE or DENSE_OFF; dense_off[2*i+j] = first counter in dense_pool
+  uint32_t* dense_pc;
+  const uint64_t* dense_off;
+  uint32_t* dense_pool;
   uint32_t n;
 };
+constexpr uint32_t DENSE_FREE = 0xFFFFFFFFu;
+constexpr uint32_t DENSE_OFF = 0xFFFFFFFEu;
+constexpr int DENSE_PER_OBJ = 2;
 
 // ---- host-side context ------------------------------------------------------
 struct HostObject {
@@ -100,6 +109,13 @@ struct ve_ctx {
   void* obj_block = nullptr;                 // backing store of DevObjects arrays
   uint64_t bm_words = 0;
   uint64_t hcap = 0;
+  // dense counters (see DevObjects); disabled once 2^32 records could overflow a u32 counter
+  void* dense_pool = nullptr;
+  uint64_t dense_cap = 0;                    // counters allocated
+  uint64_t dense_used = 0;                   // counters in use by the current object table
+  std::vector<uint64_t> dense_off_h;         // [2*n_obj]
+  std::vector<uint32_t> dense_pc_init;       // [2*n_obj]: DENSE_FREE or DENSE_OFF
+  uint64_t records_analyzed = 0;
   // finalize scratch
   void* scratch = nullptr;
   size_t scratch_bytes = 0;
@@ -134,6 +150,7 @@ ve_status run_diff(ve_ctx* c, uint32_t obj_index, uint32_t mode, const uint32_t*
 ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* group_of, cudaStream_t s);
 ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s);
 ve_status merge_nccl(ve_ctx* c, void* comm, cudaStream_t s);
+ve_status dense_flush(ve_ctx* c, cudaStream_t s);  // move dense counts into the exact histogram
 void count_launch();  // process-wide kernel launch counter (ve_kernel_launches)
 }  // namespace ve
 
@@ -223,21 +240,21 @@ __device__ __forceinline__ uint32_t float_flags(uint64_t b, uint32_t kind, uint3
   uint64_t sig = (E == 0ull) ? M : (M | (1ull << mb));
   int ex = (E == 0ull ? 1 : (int)E) - ((1 << (eb - 1)) - 1) - mb;
   if (sig == 0ull) return sign ? 2u : 0u;                                // -0.0 is nonint
+  // value = sig * 2^ex; its set bits span exponents [low, top]
+  const int low = ex + __ffsll((long long)sig) - 1;
+  const int top = ex + 63 - __clzll((long long)sig);
   uint32_t f = 0;
-  int nbits = 64 - __clzll((long long)sig);
-  if (ex + nbits - 1 >= 63) {
-    f |= 2u;                                                             // |v| >= 2^63
-  } else if (ex < 0) {
-    int sh = -ex;
-    if (sh >= 64 || (sig & ((1ull << sh) - 1ull)) != 0ull) f |= 2u;      // fractional part
-    else ival = (int64_t)(sig >> sh);
+  if (top >= 63 || low < 0) {
+    f |= 2u;                                                             // |v| >= 2^63 or a fraction
   } else {
-    ival = (int64_t)(sig << ex);
+    const uint64_t mag = (ex >= 0) ? (sig << ex) : (sig >> -ex);
+    ival = sign ? -(int64_t)mag : (int64_t)mag;
   }
-  if (!(f & 2u) && sign) ival = -ival;
-  if (!representable(sig, ex, 5, 10)) f |= 4u;
-  if (!representable(sig, ex, 8, 7)) f |= 8u;
-  if (is_f64 && !representable(sig, ex, 8, 23)) f |= 16u;
+  // representable in a format with bias B and m mantissa bits <=> top <= B and
+  // low >= max(top - m, 1 - B - m)  (round trip through it is then the identity)
+  if (!(top <= 15 && low >= max(top - 10, -24))) f |= 4u;               // binary16
+  if (!(top <= 127 && low >= max(top - 7, -133))) f |= 8u;              // bfloat16
+  if (is_f64 && !(top <= 127 && low >= max(top - 23, -149))) f |= 16u;  // binary32
   return f;
 }
 
