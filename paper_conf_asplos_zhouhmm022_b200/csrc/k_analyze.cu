@@ -28,6 +28,8 @@ namespace ve {
 
 constexpr int K1_THREADS = 384;  // 12 warps x <=168 registers: the fast path runs spill-free
 constexpr int K1_WARPS = K1_THREADS / 32;
+constexpr int RING = 8;                      // record windows in flight per warp (TMA ring)
+constexpr uint32_t WIN_BYTES = 32 * sizeof(ve_record);
 
 struct AnalyzeParams {
   const ve_record* recs;
@@ -38,6 +40,7 @@ struct AnalyzeParams {
   uint32_t hs;              // shared histogram slots (power of 2)
   uint32_t objc;            // objects cached in shared memory (0 = use global table)
   uint32_t dense_ok;        // dense per-element counting enabled for this launch
+  uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
   DevObjects o;
   DevTables t;
 };
@@ -52,6 +55,8 @@ struct Smem {
   uint64_t* sob;            // [objc] base
   uint64_t* soe;            // [objc] end
   uint32_t* sctr;           // [4]: invalid, unmapped, hist fill
+  uint8_t* ring;            // [K1_WARPS][RING][WIN_BYTES] TMA ring
+  uint64_t* bars;           // [K1_WARPS][RING] mbarriers
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
@@ -65,6 +70,7 @@ __host__ __device__ inline size_t smem_bytes(uint32_t nsk, uint32_t hs, uint32_t
   b += align16(sizeof(uint32_t) * hs);
   b += align16(sizeof(uint64_t) * objc) * 2;
   b += 16;
+  b += (size_t)K1_WARPS * RING * (WIN_BYTES + 8);
   return b;
 }
 
@@ -79,7 +85,9 @@ __device__ inline Smem carve(uint8_t* base, uint32_t nsk, uint32_t hs, uint32_t 
   s.shc = (uint32_t*)(base + off); off += align16(sizeof(uint32_t) * hs);
   s.sob = (uint64_t*)(base + off); off += align16(sizeof(uint64_t) * objc);
   s.soe = (uint64_t*)(base + off); off += align16(sizeof(uint64_t) * objc);
-  s.sctr = (uint32_t*)(base + off);
+  s.sctr = (uint32_t*)(base + off); off += 16;
+  s.ring = base + off; off += (size_t)K1_WARPS * RING * WIN_BYTES;
+  s.bars = (uint64_t*)(base + off);
   return s;
 }
 
@@ -420,6 +428,32 @@ struct Rec {
   uint64_t addr, val, pm;
 };
 
+// ---- per-warp TMA ring: cp.async.bulk of whole 768-byte windows into shared memory
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void ring_issue(uint8_t* dst, const void* src, uint64_t* bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(WIN_BYTES) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(WIN_BYTES), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void ring_wait(uint64_t* bar, uint32_t phase) {
+  uint32_t ok = 0;
+  while (!ok) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(phase)
+        : "memory");
+  }
+}
+
 __device__ __forceinline__ Rec load_rec(const AnalyzeParams& P, uint64_t w, uint64_t wend, int lane) {
   Rec r{0, 0, 0};
   const uint64_t i = w * 32 + lane;
@@ -450,12 +484,22 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   WarpCache& wc = s_wc[warp];
   if (lane < WC) wc.key1[lane] = 0;
   if (lane == 0) wc.next = 0;
-  __syncthreads();
 
-  // this warp's contiguous range of windows
+  // this warp's contiguous range of windows; full windows stream through a TMA ring
   const uint64_t nwin = (P.n + 31) / 32;
   const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + warp;
   const uint64_t wbeg = gw * nwin / tw, wend = (gw + 1) * nwin / tw;
+  const uint64_t nfull = P.n / 32;
+  const uint64_t rend = P.ring ? (wend < nfull ? wend : nfull) : wbeg;   // ring covers [wbeg, rend)
+  uint8_t (*s_ring)[RING][WIN_BYTES] = reinterpret_cast<uint8_t (*)[RING][WIN_BYTES]>(S.ring);
+  uint64_t (*s_bar)[RING] = reinterpret_cast<uint64_t (*)[RING]>(S.bars);
+  if (lane == 0) {
+    for (int d = 0; d < RING; ++d) mbar_init(&s_bar[warp][d], 1);
+    fence_mbar_init();
+    for (int d = 0; d < RING && wbeg + d < rend; ++d)
+      ring_issue(s_ring[warp][d], P.recs + (wbeg + d) * 32, &s_bar[warp][d]);
+  }
+  __syncthreads();
   int ocache = -1;  // warp-uniform last object
   uint32_t n_invalid = 0, n_unmapped = 0;
   FastSlots F;
@@ -463,11 +507,24 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   F.mru = 0;
   uint64_t acc = 0;
 
-  Rec ra = load_rec(P, wbeg, wend, lane), rb = load_rec(P, wbeg + 1, wend, lane);
   for (uint64_t w = wbeg; w < wend; ++w) {
-    const Rec cur = ra;
-    ra = rb;
-    rb = load_rec(P, w + 2, wend, lane);
+    Rec cur;
+    if (w < rend) {
+      const uint64_t i = w - wbeg;
+      const int d = (int)(i % RING);
+      ring_wait(&s_bar[warp][d], (uint32_t)((i / RING) & 1));
+      const unsigned long long* q = reinterpret_cast<const unsigned long long*>(s_ring[warp][d] + lane * 24);
+      cur.addr = q[0];
+      cur.val = q[1];
+      cur.pm = q[2];
+      __syncwarp();
+      if (lane == 0 && w + RING < rend) {
+        fence_proxy_async();   // our generic reads of the stage precede the next async write
+        ring_issue(s_ring[warp][d], P.recs + (w + RING) * 32, &s_bar[warp][d]);
+      }
+    } else {
+      cur = load_rec(P, w, wend, lane);
+    }
     const uint64_t addr = cur.addr, val = cur.val;
     const uint32_t pc = (uint32_t)cur.pm, meta = (uint32_t)(cur.pm >> 32);
     const bool inrange = w * 32 + lane < P.n;
@@ -759,6 +816,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.mant_bits = c->cfg.mant_bits;
   // u32 per-element counters cannot overflow while the ctx has seen < 2^32 records
   P.dense_ok = (c->dense_used > 0 && c->records_analyzed + n < (1ull << 32)) ? 1u : 0u;
+  P.ring = ((uintptr_t)d % 16 == 0) ? 1u : 0u;
   c->records_analyzed += n;
   // shared stat rows: up to 256 keys, PCs first then object keys (incl. SHARED)
   const uint32_t NSK_MAX = 256;
@@ -772,8 +830,11 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.t = c->t;
   int dev_smem = 0;
   cudaDeviceGetAttribute(&dev_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device);
+  cudaFuncAttributes fa;
+  cudaFuncGetAttributes(&fa, k_analyze);
+  const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring
   uint32_t hs = 8192;
-  while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > (size_t)dev_smem - 8192) hs >>= 1;
+  while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > budget) hs >>= 1;
   P.hs = hs;
   const size_t sb = smem_bytes(sp + so, hs, P.objc);
   cudaError_t e = cudaFuncSetAttribute(k_analyze, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
