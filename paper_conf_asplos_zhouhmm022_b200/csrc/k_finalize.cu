@@ -283,22 +283,59 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
 // ---- dense per-element counts -> exact histogram ------------------------------
 // A dense counter cnt[e] of (pc, object) counts loads that read element e's unchanged
 // pre-snapshot value, so it contributes cnt[e] occurrences of that value (C9).
-__global__ void k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre, uint32_t ew, uint32_t tag,
-                              DevTables t) {
-  for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < n_elems;
-       e += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t k = cnt[e];
-    if (!k) continue;
-    cnt[e] = 0;
-    const uint8_t* p = pre + e * ew;
+// Each block aggregates its chunk of elements by value (warp match, then a small
+// shared table) so runs of equal values (zero-filled regions) cost one global insert.
+constexpr int DF_THREADS = 256;
+constexpr int DF_SLOTS = 1024;
+constexpr uint64_t DF_CHUNK = 16384;
+
+__global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
+                                                           uint32_t ew, uint32_t tag, DevTables t) {
+  __shared__ unsigned long long sbits[DF_SLOTS], scnt[DF_SLOTS];
+  for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS) { sbits[i] = ~0ull; scnt[i] = 0; }
+  __syncthreads();
+  const uint64_t lo = blockIdx.x * DF_CHUNK, hi = lo + DF_CHUNK < n_elems ? lo + DF_CHUNK : n_elems;
+  const int lane = threadIdx.x & 31;
+  for (uint64_t base = lo; base < hi; base += DF_THREADS) {
+    const uint64_t e = base + threadIdx.x;
+    uint32_t k = 0;
     uint64_t bits = 0;
-    if (((uintptr_t)p & (ew - 1)) == 0) {
-      bits = ew == 1 ? *p : ew == 2 ? *(const uint16_t*)p : ew == 4 ? *(const uint32_t*)p : *(const uint64_t*)p;
-    } else {
-      for (uint32_t i = 0; i < ew; ++i) bits |= (uint64_t)p[i] << (8 * i);
+    if (e < hi) {
+      k = cnt[e];
+      if (k) {
+        cnt[e] = 0;
+        const uint8_t* p = pre + e * ew;
+        if (((uintptr_t)p & (ew - 1)) == 0) {
+          bits = ew == 1 ? *p : ew == 2 ? *(const uint16_t*)p : ew == 4 ? *(const uint32_t*)p : *(const uint64_t*)p;
+        } else {
+          for (uint32_t i = 0; i < ew; ++i) bits |= (uint64_t)p[i] << (8 * i);
+        }
+      }
     }
-    hist_insert_global(t, tag, bits, k);
+    const unsigned km = __ballot_sync(0xFFFFFFFFu, k != 0);
+    if (k) {
+      const unsigned g = __match_any_sync(km, bits);
+      const unsigned long long sum = __reduce_add_sync(g, k);   // < 32 * 2^32? counts are < 2^32 each
+      if (lane == __ffs(g) - 1) {
+        // shared slots are claimed by a 64-bit CAS of the value itself (empty = ~0, which
+        // only an 8-byte element can hold: such values go straight to the global table)
+        uint32_t h = (uint32_t)hist_hash(tag, bits) & (DF_SLOTS - 1);
+        bool done = false;
+        for (int probe = 0; probe < 8 && !done && bits != ~0ull; ++probe) {
+          const unsigned long long old = atomicCAS(&sbits[h], ~0ull, bits);
+          if (old == ~0ull || old == bits) {
+            atomicAdd(&scnt[h], sum);
+            done = true;
+          }
+          h = (h + 1) & (DF_SLOTS - 1);
+        }
+        if (!done) hist_insert_global(t, tag, bits, sum);
+      }
+    }
   }
+  __syncthreads();
+  for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS)
+    if (sbits[i] != ~0ull && scnt[i]) hist_insert_global(t, tag, sbits[i], scnt[i]);
 }
 
 ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
@@ -313,10 +350,9 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
       const uint32_t pc = dpc[DENSE_PER_OBJ * i + j];
       if (pc == DENSE_FREE || pc == DENSE_OFF) continue;
       const HostObject& o = c->objs[i];
-      uint64_t blocks = (o.n_elems + 255) / 256;
-      if (blocks > (uint64_t)c->num_sms * 8) blocks = (uint64_t)c->num_sms * 8;
+      const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
       count_launch();
-      k_dense_flush<<<(unsigned)blocks, 256, 0, s>>>((uint32_t*)c->dense_pool + c->dense_off_h[DENSE_PER_OBJ * i + j],
+      k_dense_flush<<<(unsigned)blocks, DF_THREADS, 0, s>>>((uint32_t*)c->dense_pool + c->dense_off_h[DENSE_PER_OBJ * i + j],
                                                     o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, c->t);
       any = true;
     }

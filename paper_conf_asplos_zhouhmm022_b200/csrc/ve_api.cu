@@ -4,7 +4,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -438,9 +440,22 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
     nd = c->merged_ndistinct;
     r->top = c->merged_topk;
   } else {
+    const bool tm = getenv("VE_TIMING") != nullptr;
+    auto t0 = std::chrono::steady_clock::now();
     st = dense_flush(c, 0);
     if (st != VE_OK) { delete r; return st; }
+    if (tm) {
+      cudaDeviceSynchronize();
+      fprintf(stderr, "[ve] dense_flush %.3f ms\n",
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+      t0 = std::chrono::steady_clock::now();
+    }
     st = finalize_hist(c, 0, nd, r->top);
+    if (tm) {
+      cudaDeviceSynchronize();
+      fprintf(stderr, "[ve] finalize_hist %.3f ms\n",
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    }
     if (st != VE_OK) { delete r; return st; }
   }
   st = bitmap_counts(c, 0, r->objs);
