@@ -109,7 +109,7 @@ class Workload:
             inf = G.info(G.CFG2, ep)
             n = inf["n_records"]
             self.total_records += n
-            lo, hi = n * rank // world, n * (rank + 1) // world
+            lo, hi = n * rank // world, n * (rank + 1) // world   # = ve.rank_chunk
             recs = torch.empty((hi - lo) * REC_BYTES, dtype=torch.uint8, device=device)
             G.records_device(G.CFG2, ep, self.seed, lo, hi - lo, recs.data_ptr(), stream)
             objs = []
@@ -223,6 +223,15 @@ def workload_config(sample=None, world=1):
 
 
 # ----------------------------------------------------------------------------- GPU arm
+def max_over_ranks(ms, device="cuda"):
+    """The slowest rank's device time (the job's time under strong scaling)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(ms)], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -278,9 +287,7 @@ def main():
     launches = ve.kernel_launches() - launches0
     ms = start.elapsed_time(end)
     if world > 1:
-        t = torch.tensor([ms], device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = max_over_ranks(ms, device=dev)
     ms_step = ms / args.steps
     value = wl.total_records / (ms_step / 1e3)
 

@@ -154,6 +154,12 @@ ve_status ve_object_dedup(ve_ctx* ctx, const ve_object* objs, uint32_t n, uint32
  * partition all-to-all + top-k re-rank).  Synchronizes s. */
 ve_status ve_merge_stats(ve_ctx* dst, const ve_ctx* src_or_null, void* nccl_comm_or_null, cudaStream_t s);
 
+/* S12 on one device: merge n contexts (same config, objects and device) with the
+ * same rank-merge algorithm ve_merge_stats runs over NCCL (context i plays rank
+ * i: allreduce, allgather and hash-partitioned all-to-all done with device
+ * copies); afterwards every context holds the merged statistics.  Synchronizes s. */
+ve_status ve_merge_group(ve_ctx** ctxs, uint32_t n, cudaStream_t s);
+
 /* S13: finalize (top-k, distinct counts, bitmap popcounts, derived flags) and
  * copy to a library-owned host report.  Synchronizes the ctx's streams.
  * VE_ERR_STATE if poisoned. */

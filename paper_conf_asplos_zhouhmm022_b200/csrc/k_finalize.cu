@@ -156,59 +156,87 @@ __global__ void k_occupancy(const HSlot* hs, uint64_t cap, unsigned long long* c
   if ((threadIdx.x & 31) == 0 && local) atomicAdd(cnt, local);
 }
 
-// Exact n_distinct and top-k of every key (PC keys, then object keys).
-ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
-                        std::vector<ve_topk_entry>& top) {
+// The per-PC / per-object view table built from the main (pc, object, value) table:
+// every entry of tag (pc, o) contributes to view key pc and to view key n_pcs + o.
+ve_status build_views(ve_ctx* c, cudaStream_t s, ViewTable& V) {
+  cudaError_t e;
+  unsigned long long* d_small = nullptr;  // [0] overflow, [1] occupancy / entries
+  e = cudaMallocAsync((void**)&d_small, 16, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "views alloc");
+  cudaMemsetAsync(d_small, 0, 16, s);
+  count_launch();
+  k_occupancy<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->hcap, d_small + 1);
+  unsigned long long occ = 0;
+  e = cudaMemcpyAsync(&occ, d_small + 1, 8, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "views occupancy"); }
+  cudaMemsetAsync(d_small, 0, 16, s);
+  ve_status st = alloc_views(c, s, 2 * occ, V);
+  if (st != VE_OK) { cudaFreeAsync(d_small, s); return st; }
+  count_launch();
+  k_views<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, c->cfg.n_pcs, V.vs, V.vc, V.vcap - 1,
+                                         d_small, d_small + 1);
+  unsigned long long h_small[2];
+  e = cudaMemcpyAsync(h_small, d_small, 16, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d_small, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "views build");
+  if (h_small[0]) return fail(c, VE_ERR_CAPACITY, "finalize: view table overflow");
+  return VE_OK;
+}
+
+// an empty view table for up to n entries (load <= 1/2)
+ve_status alloc_views(ve_ctx* c, cudaStream_t s, uint64_t n, ViewTable& V) {
+  uint64_t vcap = 1024;
+  while (vcap < 2 * n) vcap <<= 1;
+  V.vcap = vcap;
+  cudaError_t e = cudaMallocAsync((void**)&V.vs, vcap * sizeof(HSlot), s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&V.vc, vcap * 8, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "view table alloc");
+  cudaMemsetAsync(V.vs, 0xFF, vcap * sizeof(HSlot), s);
+  cudaMemsetAsync(V.vc, 0, vcap * 8, s);
+  return VE_OK;
+}
+
+void free_views(ViewTable& V, cudaStream_t s) {
+  if (V.vs) cudaFreeAsync(V.vs, s);
+  if (V.vc) cudaFreeAsync(V.vc, s);
+  V.vs = nullptr;
+  V.vc = nullptr;
+}
+
+// Exact n_distinct and top-k (count desc, bits asc) of every key of a view table.
+ve_status view_topk(ve_ctx* c, const ViewTable& V, cudaStream_t s, std::vector<uint64_t>& ndistinct,
+                    std::vector<ve_topk_entry>& top) {
   const uint32_t nk = c->n_keys, K = c->cfg.topk;
   ndistinct.assign(nk, 0);
   top.assign((size_t)nk * K, ve_topk_entry{0, 0});
   cudaError_t e;
-  // 1. count occupied slots (upper bound on view entries = 2x)
-  unsigned long long* d_small = nullptr;  // [0] overflow, [1] n_entries
-  e = cudaMallocAsync((void**)&d_small, 16, s);
-  if (e != cudaSuccess) return cuda_fail(c, e, "finalize alloc");
-  cudaMemsetAsync(d_small, 0, 16, s);
-  // occupancy of the main table sizes the view table (<= 2 view entries per slot, load <= 1/2)
-  uint64_t occ = 0;
-  {
-    unsigned long long* d_cnt = d_small + 1;
-    count_launch();
-    k_occupancy<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->hcap, d_cnt);
-    unsigned long long h_cnt = 0;
-    e = cudaMemcpyAsync(&h_cnt, d_cnt, 8, cudaMemcpyDeviceToHost, s);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize occupancy"); }
-    occ = h_cnt;
-    cudaMemsetAsync(d_small, 0, 16, s);
-  }
-  uint64_t vcap = 1024;
-  while (vcap < 4 * occ) vcap <<= 1;
-  const uint64_t vmask = vcap - 1;
-  // scratch: view slots + counts, ndist, off, cursor, grouped bits/counts (x2 for levels)
-  const uint64_t nent = 2 * occ + 1;
-  size_t need = vcap * sizeof(HSlot) + vcap * 8 + 3 * (size_t)nk * 8 + 4 * nent * 8 + 64;
-  e = scratch_need(c, need);
-  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize scratch"); }
-  uint8_t* p = (uint8_t*)c->scratch;
-  HSlot* vs = (HSlot*)p; p += vcap * sizeof(HSlot);
-  unsigned long long* vc = (unsigned long long*)p; p += vcap * 8;
-  unsigned long long* d_nd = (unsigned long long*)p; p += (size_t)nk * 8;
-  unsigned long long* d_off = (unsigned long long*)p; p += (size_t)nk * 8;
-  unsigned long long* d_cur = (unsigned long long*)p; p += (size_t)nk * 8;
-  uint64_t* gb[2]; uint64_t* gc[2];
-  gb[0] = (uint64_t*)p; p += nent * 8;
-  gc[0] = (uint64_t*)p; p += nent * 8;
-  gb[1] = (uint64_t*)p; p += nent * 8;
-  gc[1] = (uint64_t*)p; p += nent * 8;
-  cudaMemsetAsync(vs, 0xFF, vcap * sizeof(HSlot), s);
-  cudaMemsetAsync(vc, 0, vcap * 8, s);
+  const uint64_t vcap = V.vcap;
+  HSlot* vs = V.vs;
+  unsigned long long* vc = V.vc;
+  unsigned long long* d_nd = nullptr;                  // ndist, off, cursor
+  e = cudaMallocAsync((void**)&d_nd, (size_t)nk * 8 * 3, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "top-k alloc");
+  unsigned long long* d_off = d_nd + nk;
+  unsigned long long* d_cur = d_off + nk;
   cudaMemsetAsync(d_nd, 0, (size_t)nk * 8 * 3, s);
   const int grid = c->num_sms * 4;
   count_launch();
-  k_views<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, c->cfg.n_pcs, vs, vc, vmask, d_small,
-                               d_small + 1);
-  count_launch();
   k_view_count<<<grid, 256, 0, s>>>(vs, vcap, d_nd);
+  e = cudaMemcpyAsync(ndistinct.data(), d_nd, (size_t)nk * 8, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_nd, s); return cuda_fail(c, e, "finalize ndistinct"); }
+  uint64_t nent = 1;
+  for (uint32_t k = 0; k < nk; ++k) nent += ndistinct[k];
+  uint64_t* gbuf = nullptr;
+  e = cudaMallocAsync((void**)&gbuf, 4 * nent * 8, s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_nd, s); return cuda_fail(c, e, "top-k alloc"); }
+  uint64_t* gb[2] = {gbuf, gbuf + 2 * nent};
+  uint64_t* gc[2] = {gbuf + nent, gbuf + 3 * nent};
+  unsigned long long* d_small = nullptr;
+  cudaMallocAsync((void**)&d_small, 16, s);
+  cudaMemsetAsync(d_small, 0, 16, s);
   e = cudaMemcpyAsync(ndistinct.data(), d_nd, (size_t)nk * 8, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize ndistinct"); }
@@ -270,14 +298,23 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
       break;
     }
   }
-  unsigned long long h_small[2] = {0, 0};
-  cudaMemcpyAsync(h_small, d_small, 16, cudaMemcpyDeviceToHost, s);
   if (d_chunks) cudaFreeAsync(d_chunks, s);
   cudaFreeAsync(d_small, s);
+  cudaFreeAsync(gbuf, s);
+  cudaFreeAsync(d_nd, s);
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "finalize top-k");
-  if (h_small[0]) return fail(c, VE_ERR_CAPACITY, "finalize: view table overflow");
   return VE_OK;
+}
+
+// Exact n_distinct and top-k of every key (PC keys, then object keys).
+ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
+                        std::vector<ve_topk_entry>& top) {
+  ViewTable V;
+  ve_status st = build_views(c, s, V);
+  if (st == VE_OK) st = view_topk(c, V, s, ndistinct, top);
+  free_views(V, s);
+  return st;
 }
 
 // ---- dense per-element counts -> exact histogram ------------------------------

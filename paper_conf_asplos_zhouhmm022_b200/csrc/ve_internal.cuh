@@ -151,6 +151,16 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
 ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s);
 ve_status merge_nccl(ve_ctx* c, void* comm, cudaStream_t s);
 ve_status dense_flush(ve_ctx* c, cudaStream_t s);  // move dense counts into the exact histogram
+struct ViewTable {                                 // per-key (PC view, object view) value counts
+  HSlot* vs = nullptr;
+  unsigned long long* vc = nullptr;
+  uint64_t vcap = 0;
+};
+ve_status build_views(ve_ctx* c, cudaStream_t s, ViewTable& V);
+ve_status alloc_views(ve_ctx* c, cudaStream_t s, uint64_t n, ViewTable& V);
+void free_views(ViewTable& V, cudaStream_t s);
+ve_status view_topk(ve_ctx* c, const ViewTable& V, cudaStream_t s, std::vector<uint64_t>& ndistinct,
+                    std::vector<ve_topk_entry>& top);
 void count_launch();  // process-wide kernel launch counter (ve_kernel_launches)
 }  // namespace ve
 

@@ -86,6 +86,7 @@ def lib():
             "ve_report_globals": ([vp, vp], st),
             "ve_report_dump": ([vp, ctypes.c_char_p, i32], st),
             "ve_kernel_launches": ([], u64),
+            "ve_merge_group": ([ctypes.POINTER(vp), u32, vp], st),
             "ve_nccl_get_unique_id": ([vp], st),
             "ve_nccl_comm_init": ([ctypes.POINTER(vp), i32, vp, i32], st),
             "ve_nccl_comm_destroy": ([vp], st),
@@ -128,6 +129,50 @@ def _stream(stream):
 def kernel_launches():
     """libve kernels launched by this process so far (ve_kernel_launches)."""
     return lib().ve_kernel_launches()
+
+
+def rank_chunk(n, rank, world):
+    """[lo, hi) of the contiguous share of n records analyzed by `rank` of `world` (strong scaling)."""
+    return n * rank // world, n * (rank + 1) // world
+
+
+def merge_group(contexts, stream=None):
+    """ve_merge_group: merge same-device contexts with the rank-merge algorithm (context i = rank i)."""
+    arr = (ctypes.c_void_p * len(contexts))(*[c.handle.value for c in contexts])
+    rc = lib().ve_merge_group(arr, len(contexts), _stream(stream))
+    if rc != OK:
+        raise VeError(rc, "ve_merge_group: " + lib().ve_last_error(contexts[0].handle).decode())
+
+
+def nccl_unique_id():
+    buf = (ctypes.c_uint8 * 128)()
+    rc = lib().ve_nccl_get_unique_id(buf)
+    if rc != OK:
+        raise VeError(rc, "ve_nccl_get_unique_id")
+    return bytes(buf)
+
+
+def nccl_comm_init(uid, rank, world):
+    comm = ctypes.c_void_p()
+    buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
+    rc = lib().ve_nccl_comm_init(ctypes.byref(comm), world, buf, rank)
+    if rc != OK:
+        raise VeError(rc, "ve_nccl_comm_init")
+    return comm.value
+
+
+def nccl_comm_from_torch(rank, world, group=None):
+    """One NCCL communicator over the torch.distributed ranks: rank 0 creates the unique id,
+    torch.distributed broadcasts it (any backend), every rank joins."""
+    import torch
+    import torch.distributed as dist
+    uid = torch.zeros(128, dtype=torch.uint8)
+    if rank == 0:
+        uid = torch.tensor(list(nccl_unique_id()), dtype=torch.uint8)
+    if dist.get_backend(group) == "nccl":
+        uid = uid.cuda()
+    dist.broadcast(uid, src=0, group=group)
+    return nccl_comm_init(bytes(uid.cpu().tolist()), rank, world)
 
 
 class Report:
@@ -238,7 +283,9 @@ class Context:
         return g[:len(objs)]
 
     def merge(self, other=None, comm=None, stream=None):
-        self._check(lib().ve_merge_stats(self._h, other._h if other is not None else None, comm, _stream(stream)),
+        """ve_merge_stats: with another same-device context, or over all ranks of an NCCL comm."""
+        self._check(lib().ve_merge_stats(self._h, other._h if other is not None else None,
+                                         ctypes.c_void_p(comm) if comm else None, _stream(stream)),
                     "ve_merge_stats")
 
     def report(self):

@@ -5,6 +5,7 @@ import numpy as np
 import pytest
 
 from gen import vegen as G
+from gen import vegen as gen
 from oracle import oracle as O
 from tests import parity, workloads as W
 
@@ -166,3 +167,48 @@ def test_empty_and_tiny(torch_cuda):
     for n in (1, 2, 31, 32, 33):
         recs = G.records_host(G.FUZZ, 0, 12, 7, n)
         _check(torch_cuda, 64, hobjs, recs)
+
+
+@pytest.mark.parametrize("G", [2, 3, 4])
+def test_rank_merge_simulated(torch_cuda, G):
+    """S12 across ranks, simulated on one GPU: G contexts analyze contiguous record chunks
+    (as bench ranks do), ve_merge_group runs the NCCL algorithm (allreduce / allgather /
+    hash-partitioned all-to-all of view entries + re-rank) with device copies; every
+    context must report exactly the oracle's result over all records."""
+    ve = _ve()
+    seed, n = 13, 150001
+    hobjs = W.host_objects(gen.FUZZ, 0, seed)
+    recs = gen.records_host(gen.FUZZ, 0, seed, 0, n)
+    cfg = O.make_config(64)
+    okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
+    dobjs = W.device_objects(hobjs)
+    drec = W.device_records(recs)
+    ctxs = []
+    for r in range(G):
+        lo, hi = ve.rank_chunk(n, r, G)
+        c = ve.Context(n_pcs=64, max_objects=8, hist_capacity=1 << 20)
+        c.set_objects(dobjs)
+        c.analyze_records(drec[lo * 24:hi * 24], hi - lo)
+        ctxs.append(c)
+    ve.merge_group(ctxs)
+    for c in ctxs:
+        bad = parity.compare_with_oracle(c.report(), okeys, oglob, oobj)
+        assert not bad, "\n".join(bad[:20])
+    with pytest.raises(ve.VeError):                           # merged contexts refuse more records
+        ctxs[0].analyze_records(drec[:24], 1)
+
+
+def test_nccl_merge_single_rank(torch_cuda):
+    """ve_merge_stats over a real (1-rank) NCCL communicator leaves the result exact."""
+    ve = _ve()
+    seed, n = 14, 90000
+    hobjs = W.host_objects(gen.FUZZ, 0, seed)
+    recs = gen.records_host(gen.FUZZ, 0, seed, 0, n)
+    okeys, oglob, oobj = O.analyze(O.make_config(64), hobjs, recs)
+    comm = ve.nccl_comm_init(ve.nccl_unique_id(), 0, 1)
+    c = ve.Context(n_pcs=64, max_objects=8, hist_capacity=1 << 20)
+    c.set_objects(W.device_objects(hobjs))
+    c.analyze_records(W.device_records(recs), n)
+    c.merge(comm=comm)
+    bad = parity.compare_with_oracle(c.report(), okeys, oglob, oobj)
+    assert not bad, "\n".join(bad[:20])
