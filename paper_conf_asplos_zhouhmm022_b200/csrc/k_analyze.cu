@@ -143,7 +143,7 @@ struct Facts {
 };
 
 // line state of the points of the lanes in gm (all valid, none pfail)
-__device__ __forceinline__ void group_line(unsigned gm, const Facts& f, LinePts& g) {
+__device__ __noinline__ void group_line(unsigned gm, const Facts& f, LinePts& g) {
   if (__any_sync(gm, f.pfail)) {
     g.state = VE_LINE_FAIL;
     g.px = g.qx = 0; g.py = g.qy = 0;
@@ -183,7 +183,7 @@ __device__ __forceinline__ void group_line(unsigned gm, const Facts& f, LinePts&
 
 // Slow path: reduce one key group (all lanes in gm share the key) and fold it into
 // the key's row: shared memory when slot >= 0, else the global table.
-__device__ __forceinline__ void apply_group(const AnalyzeParams& P, const Smem& S, unsigned gm, int slot,
+__device__ __noinline__ void apply_group(const AnalyzeParams& P, const Smem& S, unsigned gm, int slot,
                                             uint32_t key, const Facts& f, LinePts& g) {
   const int lane = threadIdx.x & 31;
   const unsigned gsize = __popc(gm);
@@ -251,7 +251,7 @@ __device__ __forceinline__ LineState* line_target(const AnalyzeParams& P, const 
 }
 
 // returns the key's merged (warp-local) state
-__device__ __forceinline__ uint32_t wcache_merge(const AnalyzeParams& P, const Smem& S, WarpCache& C, uint32_t key,
+__device__ __noinline__ uint32_t wcache_merge(const AnalyzeParams& P, const Smem& S, WarpCache& C, uint32_t key,
                                                  int slot, const LinePts& g) {
   for (int i = 0; i < WC; ++i) {
     if (C.key1[i] == key + 1) {
@@ -276,7 +276,7 @@ __device__ __forceinline__ uint32_t wcache_merge(const AnalyzeParams& P, const S
   return g.state;
 }
 
-__device__ __forceinline__ void wcache_flush(const AnalyzeParams& P, const Smem& S, WarpCache& C) {
+__device__ __noinline__ void wcache_flush(const AnalyzeParams& P, const Smem& S, WarpCache& C) {
   for (int i = 0; i < WC; ++i) {
     if (C.key1[i]) {
       if (C.st[i].state != VE_LINE_FAIL) line_merge_locked(line_target(P, S, C.slot[i], C.key1[i] - 1), line_load(C.st[i]));
@@ -286,7 +286,7 @@ __device__ __forceinline__ void wcache_flush(const AnalyzeParams& P, const Smem&
 }
 
 // serialise the merges of this window's group leaders through the warp cache
-__device__ __forceinline__ void merge_lines(const AnalyzeParams& P, const Smem& S, WarpCache& C, bool lead,
+__device__ __noinline__ void merge_lines(const AnalyzeParams& P, const Smem& S, WarpCache& C, bool lead,
                                             uint32_t key, int slot, const LinePts& g) {
   unsigned L = __ballot_sync(0xFFFFFFFFu, lead && g.state != VE_LINE_EMPTY);
   while (L) {
@@ -324,7 +324,7 @@ __device__ __forceinline__ void hist_insert(const AnalyzeParams& P, const Smem& 
   hist_insert_global(P.t, tag, bits, c);
 }
 
-__device__ __forceinline__ int find_object(const AnalyzeParams& P, const Smem& S, uint64_t addr) {
+__device__ __noinline__ int find_object(const AnalyzeParams& P, const Smem& S, uint64_t addr) {
   const uint64_t* base = P.objc ? S.sob : P.o.base;
   int lo = 0, hi = (int)P.o.n;  // first object with base > addr
   while (lo < hi) {
@@ -359,7 +359,7 @@ struct FastSlots {
 };
 
 // claim (or find) a dense counter array of sorted object oi for pc (lane 0), broadcast
-__device__ __forceinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t pc) {
+__device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t pc) {
   unsigned long long dp = 0;
   if ((threadIdx.x & 31) == 0) {
     for (int j = 0; j < DENSE_PER_OBJ; ++j) {
@@ -396,13 +396,13 @@ __device__ __forceinline__ void fold_row(const AnalyzeParams& P, const Smem& S, 
 }
 
 // fold slot s's accumulators into the PC-key row and the object-key row (lanes of half s)
-__device__ __forceinline__ void fast_flush(const AnalyzeParams& P, const Smem& S, const FastSlots& F, int s,
-                                           uint64_t acc) {
+__device__ __noinline__ void fast_flush(const AnalyzeParams& P, const Smem& S, uint32_t pc, uint32_t koi,
+                                        uint32_t meta, int s, uint64_t acc) {
   const int lane = threadIdx.x & 31;
   const uint64_t nrec = __shfl_sync(0xFFFFFFFFu, acc, s * 16);   // field 0 of slot s
   if ((lane >> 4) != s) return;
   const int f = lane & 15;
-  const uint32_t meta = F.meta[s], lg = meta & 3u, kind = (meta >> 2) & 3u;
+  const uint32_t lg = meta & 3u, kind = (meta >> 2) & 3u;
   const bool st = meta_store(meta);
   uint64_t v = (f == 15) ? nrec : acc;
   if (v == fast_identity(f) && f != 15) return;
@@ -419,9 +419,143 @@ __device__ __forceinline__ void fast_flush(const AnalyzeParams& P, const Smem& S
     const int32_t sv = (int32_t)((uint32_t)v ^ 0x80000000u);
     v = (uint64_t)(int64_t)sv ^ (1ull << 63);
   }
-  const uint32_t pc = F.pc[s], koi = F.koi[s];
   fold_row(P, S, pc < P.sp ? (int)pc : -1, pc, f, field, v);
   if (koi != KO_NONE) fold_row(P, S, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
+}
+
+// per-lane facts of a uniform window handed to its specialised fast path
+struct WinCtx {
+  uint64_t addr, val, off;
+  uint32_t ew_lg;
+  bool valid, eq, eqdef;
+  unsigned vmask;
+  int l0;
+  uint32_t pc0, koi0;
+};
+
+// warp-uniform cache of the last object a window mapped to
+struct ObjCache {
+  int oi;
+  uint64_t base, end, bmoff, pre;
+  uint32_t id, ewlg;
+};
+
+// Fast path of a uniform window whose access type (KIND, LG = log2 width) is a
+// compile-time constant: the bit tests of C5-C8 specialise to the type.
+template <int KIND, int LG>
+__device__ __forceinline__ void fast_window(const AnalyzeParams& P, const Smem& S, uint32_t& lfail_s,
+                                            unsigned long long dense_s, int s, uint64_t& acc, WarpCache& wc,
+                                            const WinCtx& x) {
+  constexpr bool ISF = KIND >= 2;
+  const int lane = threadIdx.x & 31;
+  const uint64_t val = x.val;
+  const bool valid = x.valid;
+  int64_t ival = 0;
+  const uint32_t ff = ISF ? float_flags(val, KIND, LG, ival) : 0u;
+  const bool okv = valid && !(ff & 1u);       // contributes to ord / trunc (NaNs excluded)
+  const uint32_t nv = __popc(x.vmask);
+  const uint32_t pA = valid ? ((uint32_t)(val == 0) | ((uint32_t)x.eq << 6) | ((uint32_t)!x.eqdef << 12)) : 0u;
+  const uint32_t A = __reduce_add_sync(0xFFFFFFFFu, pA);
+  uint32_t B = 0;
+  if (ISF) {
+    const uint32_t pB = valid ? ((ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) |
+                                 (((ff >> 3) & 1u) << 18) | (((ff >> 4) & 1u) << 24)) : 0u;
+    B = __reduce_add_sync(0xFFFFFFFFu, pB);
+  }
+  uint64_t rmin, rmax, omin, omax, tmin = ~0ull, tmax = 0;
+  if (LG < 3) {
+    // w <= 4 bytes: every key fits 32 bits -> one REDUX per min / max
+    const uint32_t r32 = (uint32_t)val;
+    rmin = __reduce_min_sync(0xFFFFFFFFu, valid ? r32 : 0xFFFFFFFFu);
+    rmax = __reduce_max_sync(0xFFFFFFFFu, valid ? r32 : 0u);
+    if (KIND == 0) {
+      omin = rmin; omax = rmax;
+    } else {
+      uint32_t k32;
+      if (KIND == 1) {                          // sext32(b) ^ 2^31: order-isomorphic to the 64-bit key
+        constexpr uint32_t sh = 32 - (8 << LG);
+        k32 = (uint32_t)(((int32_t)(r32 << sh)) >> sh) ^ 0x80000000u;
+      } else {
+        k32 = (uint32_t)ord_key(val, KIND, LG);
+      }
+      const unsigned okm = __ballot_sync(0xFFFFFFFFu, okv);
+      omin = __reduce_min_sync(0xFFFFFFFFu, okv ? k32 : 0xFFFFFFFFu);
+      omax = __reduce_max_sync(0xFFFFFFFFu, okv ? k32 : 0u);
+      if (ISF) {
+        const uint32_t t32 = (uint32_t)trunc_bits(val, KIND, LG, P.mant_bits);
+        tmin = __reduce_min_sync(0xFFFFFFFFu, okv ? t32 : 0xFFFFFFFFu);
+        tmax = __reduce_max_sync(0xFFFFFFFFu, okv ? t32 : 0u);
+      }
+      if (okm == 0) { omin = ~0ull; omax = 0; tmin = ~0ull; tmax = 0; }
+    }
+  } else {
+    rmin = redmin64(0xFFFFFFFFu, valid ? val : ~0ull);
+    rmax = redmax64(0xFFFFFFFFu, valid ? val : 0ull);
+    if (KIND == 0) {
+      omin = rmin; omax = rmax;
+    } else {
+      const uint64_t o = ord_key(val, KIND, LG);
+      omin = redmin64(0xFFFFFFFFu, okv ? o : ~0ull);
+      omax = redmax64(0xFFFFFFFFu, okv ? o : 0ull);
+      if (ISF) {
+        const uint64_t t = trunc_bits(val, KIND, LG, P.mant_bits);
+        tmin = redmin64(0xFFFFFFFFu, okv ? t : ~0ull);
+        tmax = redmax64(0xFFFFFFFFu, okv ? t : 0ull);
+      }
+    }
+  }
+  if ((lane >> 4) == s) {
+    const int fl = lane & 15;
+    if (fl == 0) acc += nv;
+    else if (fl <= 3) acc += (A >> (6 * (fl - 1))) & 63u;
+    else if (fl <= 8) acc += (B >> (6 * (fl - 4))) & 63u;
+    else if (fl <= 14) {
+      const int m = (fl - 9) >> 1;
+      if (fl & 1) {
+        const uint64_t v = m == 0 ? rmin : m == 1 ? omin : tmin;
+        acc = v < acc ? v : acc;
+      } else {
+        const uint64_t v = m == 0 ? rmax : m == 1 ? omax : tmax;
+        acc = v > acc ? v : acc;
+      }
+    }
+  }
+  // C8: one line state for the window, merged into each key not yet FAIL
+  if (lfail_s != 3u) {
+    Facts f;
+    f.addr = x.addr;
+    f.pfail = ISF && (ff & 2u);
+    if (KIND == 0) f.y = (__int128)val;
+    else if (KIND == 1) {
+      constexpr uint32_t sh64 = 64u - (8u << LG);
+      f.y = (__int128)((int64_t)(val << sh64) >> sh64);
+    } else {
+      f.y = (__int128)ival;
+    }
+    LinePts g;
+    g.state = VE_LINE_EMPTY;
+    if (valid) group_line(x.vmask, f, g);
+    const int ps = x.pc0 < P.sp ? (int)x.pc0 : -1;
+    const int os = x.koi0 < P.so ? (int)(P.sp + x.koi0) : -1;
+    uint32_t lf = lfail_s;
+    if (lane == x.l0) {
+      if (!(lf & 1u) && wcache_merge(P, S, wc, x.pc0, ps, g) == VE_LINE_FAIL) lf |= 1u;
+      if (!(lf & 2u) && wcache_merge(P, S, wc, P.n_pcs + x.koi0, os, g) == VE_LINE_FAIL) lf |= 2u;
+    }
+    __syncwarp();
+    lfail_s = __shfl_sync(0xFFFFFFFFu, lf, x.l0);
+  }
+  // S8: exact histogram.  A load that reads an unchanged whole element carries the
+  // pre-snapshot value of that element, so it is counted per element (a coalesced
+  // counter increment) and mapped to its value at report time; every other record
+  // is inserted per distinct value.
+  const bool dl = dense_s != 0ull && x.eq && (uint32_t)LG == x.ew_lg && (x.off & ((1ull << LG) - 1)) == 0;
+  if (dl) atomicAdd(reinterpret_cast<uint32_t*>(dense_s) + (x.off >> LG), 1u);
+  const unsigned hmask = __ballot_sync(0xFFFFFFFFu, valid && !dl);
+  if (valid && !dl) {
+    const unsigned vg = (LG < 3) ? __match_any_sync(hmask, (uint32_t)val) : __match_any_sync(hmask, val);
+    if (lane == __ffs(vg) - 1) hist_insert(P, S, (x.pc0 << 16) | (x.koi0 & 0xFFFFu), val, __popc(vg));
+  }
 }
 
 struct Rec {
@@ -500,7 +634,8 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
       ring_issue(s_ring[warp][d], P.recs + (wbeg + d) * 32, &s_bar[warp][d]);
   }
   __syncthreads();
-  int ocache = -1;  // warp-uniform last object
+  ObjCache oc;
+  oc.oi = -1; oc.base = oc.end = oc.bmoff = oc.pre = 0; oc.id = 0; oc.ewlg = 0;
   uint32_t n_invalid = 0, n_unmapped = 0;
   FastSlots F;
   F.used = 0;
@@ -527,94 +662,83 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
     }
     const uint64_t addr = cur.addr, val = cur.val;
     const uint32_t pc = (uint32_t)cur.pm, meta = (uint32_t)(cur.pm >> 32);
-    const bool inrange = w * 32 + lane < P.n;
+    const bool full = (w + 1) * 32 <= P.n;
+    const bool inrange = full || (w * 32 + lane < P.n);
 
     // S1 decode + validate
     const bool valid = inrange && rec_valid(addr, val, pc, meta, P.n_pcs);
     const unsigned vmask = __ballot_sync(0xFFFFFFFFu, valid);
-    const unsigned imask = __ballot_sync(0xFFFFFFFFu, inrange);
-    if (lane == 0) n_invalid += (uint32_t)(__popc(imask) - __popc(vmask));
+    if (lane == 0) n_invalid += (full ? 32u : (uint32_t)min((uint64_t)32, P.n - w * 32)) - (uint32_t)__popc(vmask);
     if (vmask == 0) continue;
     const uint32_t lg = meta & 3u, kind = (meta >> 2) & 3u;
     const bool st = meta_store(meta), sh = meta_shared(meta);
 
-    // S2 address -> object (warp-uniform cache, then binary search)
+    // S2 address -> object: warp-uniform cached object, binary search only on a miss
     const bool need = valid && !sh;
-    int oi = -1;
-    bool hit = false;
-    if (ocache >= 0 && need) {
-      const uint64_t b = P.objc ? S.sob[ocache] : P.o.base[ocache];
-      const uint64_t e = P.objc ? S.soe[ocache] : P.o.end[ocache];
-      hit = addr >= b && addr < e;
-      if (hit) oi = ocache;
-    }
-    if (need && !hit) oi = find_object(P, S, addr);
-    {
-      const unsigned mm = __ballot_sync(0xFFFFFFFFu, need && oi >= 0);
-      if (mm) ocache = __shfl_sync(0xFFFFFFFFu, oi, __ffs(mm) - 1);
+    const bool hit = need && oc.oi >= 0 && addr >= oc.base && addr < oc.end;
+    int oi = hit ? oc.oi : -1;
+    uint64_t ob = oc.base, oe = oc.end, obm = oc.bmoff, opre = oc.pre;
+    uint32_t oid = oc.id, oewlg = oc.ewlg;
+    const unsigned missm = __ballot_sync(0xFFFFFFFFu, need && !hit);
+    if (missm) {
+      if (need && !hit) {
+        oi = find_object(P, S, addr);
+        if (oi >= 0) {
+          ob = P.objc ? S.sob[oi] : P.o.base[oi];
+          oe = P.objc ? S.soe[oi] : P.o.end[oi];
+          obm = P.o.bmoff[oi];
+          opre = P.o.pre[oi];
+          oid = P.o.id[oi];
+          const uint32_t ew = P.o.ew[oi];
+          oewlg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
+        }
+      }
+      const unsigned mm = __ballot_sync(0xFFFFFFFFu, need && !hit && oi >= 0);
+      if (mm) {                                    // adopt the first newly found object
+        const int src = __ffs(mm) - 1;
+        oc.oi = __shfl_sync(0xFFFFFFFFu, oi, src);
+        oc.base = __shfl_sync(0xFFFFFFFFu, ob, src);
+        oc.end = __shfl_sync(0xFFFFFFFFu, oe, src);
+        oc.bmoff = __shfl_sync(0xFFFFFFFFu, obm, src);
+        oc.pre = __shfl_sync(0xFFFFFFFFu, opre, src);
+        oc.id = __shfl_sync(0xFFFFFFFFu, oid, src);
+        oc.ewlg = __shfl_sync(0xFFFFFFFFu, oewlg, src);
+      }
+      const unsigned um = __ballot_sync(0xFFFFFFFFu, need && oi < 0);
+      if (lane == 0) n_unmapped += __popc(um);
     }
     const bool mapped = oi >= 0;
-    const unsigned um = __ballot_sync(0xFFFFFFFFu, need && !mapped);
-    if (lane == 0) n_unmapped += __popc(um);
 
     // S3 snapshot gather + eq_pre
-    uint32_t ew_lg = 0, oid = 0;
-    uint64_t off = 0, bmoff = 0;
-    bool inside = false, eqdef = false, eq = false;
-    if (mapped) {
-      const uint64_t b = P.objc ? S.sob[oi] : P.o.base[oi];
-      const uint64_t e = P.objc ? S.soe[oi] : P.o.end[oi];
-      off = addr - b;
-      inside = addr + (1u << lg) <= e;
-      oid = P.o.id[oi];
-      const uint32_t ew = P.o.ew[oi];
-      ew_lg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
-      bmoff = P.o.bmoff[oi];
-      const uint64_t pre = P.o.pre[oi];
-      if (inside && pre) {
-        eqdef = true;
-        eq = load_pre(pre + off, lg) == val;
-      }
-    }
+    const uint32_t ew_lg = mapped ? oewlg : 0u;
+    const uint64_t off = mapped ? addr - ob : 0ull;
+    const uint64_t bmoff = mapped ? obm : 0ull;
+    const bool inside = mapped && addr + (1u << lg) <= oe;
+    const bool eqdef = inside && opre != 0ull;
+    const bool eq = eqdef && load_pre(opre + off, lg) == val;
+    const uint32_t koi = sh ? P.n_obj : (mapped ? oid : KO_NONE);
 
     // W / L element bitmaps (C3, C10)
     {
       const bool wpart = inside && st;
       const uint64_t e0 = off >> ew_lg, e1 = (off + (1u << lg) - 1) >> ew_lg;
       const uint64_t w0 = bmoff + (e0 >> 5), w1 = bmoff + (e1 >> 5);
-      uint32_t b0 = 0, b1 = 0;
-      if (wpart) {
-        for (uint64_t e = e0; e <= e1; ++e) {
-          if (bmoff + (e >> 5) == w0) b0 |= 1u << (e & 31);
-          else b1 |= 1u << (e & 31);
-        }
-      }
       const unsigned wany = __ballot_sync(0xFFFFFFFFu, wpart);
-      if (wany) bitmap_or(P.t.W, wpart, w0, b0);
-      const bool spill = wpart && w1 != w0;
-      if (__any_sync(0xFFFFFFFFu, spill)) bitmap_or(P.t.W, spill, w1, b1);
+      if (wany) {
+        uint32_t b0 = 0, b1 = 0;
+        if (wpart) {
+          for (uint64_t e = e0; e <= e1; ++e) {
+            if (bmoff + (e >> 5) == w0) b0 |= 1u << (e & 31);
+            else b1 |= 1u << (e & 31);
+          }
+        }
+        bitmap_or(P.t.W, wpart, w0, b0);
+        const bool spill = wpart && w1 != w0;
+        if (__any_sync(0xFFFFFFFFu, spill)) bitmap_or(P.t.W, spill, w1, b1);
+      }
       const bool lpart = inside && !st && eq;
       if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, w0, 1u << (e0 & 31));
     }
-
-    // per-record value tests (S4-S7)
-    Facts f;
-    f.addr = addr;
-    f.val = val;
-    f.tc = type_code(kind, lg);
-    f.isf = kind >= 2u;
-    int64_t ival = 0;
-    const uint32_t ff = f.isf ? float_flags(val, kind, lg, ival) : 0u;
-    f.nan = ff & 1u;
-    f.pfail = f.isf && (ff & 2u);
-    f.ordv = ord_key(val, kind, lg);
-    f.truncv = f.isf ? trunc_bits(val, kind, lg, P.mant_bits) : 0ull;
-    if (kind == 0u) f.y = (__int128)val;
-    else if (kind == 1u) {
-      const uint32_t sh64 = 64u - (8u << lg);
-      f.y = (__int128)((int64_t)(val << sh64) >> sh64);
-    } else f.y = (__int128)ival;
-    const uint32_t koi = sh ? P.n_obj : (mapped ? oid : KO_NONE);
 
     // uniform window? (pc, access type and object shared by every valid lane)
     const int l0 = __ffs(vmask) - 1;
@@ -631,9 +755,14 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
       else if ((F.used & 2u) && F.pc[1] == pc0 && F.koi[1] == koi0 && F.meta[1] == meta0) s = 1;
       else {
         s = !(F.used & 1u) ? 0 : !(F.used & 2u) ? 1 : (int)(F.mru ^ 1u);
-        if (F.used & (1u << s)) fast_flush(P, S, F, s, acc);
+        if (F.used & (1u << s)) {
+          if (s) fast_flush(P, S, F.pc[1], F.koi[1], F.meta[1], 1, acc);
+          else fast_flush(P, S, F.pc[0], F.koi[0], F.meta[0], 0, acc);
+        }
         F.used |= 1u << s;
-        F.pc[s] = pc0; F.koi[s] = koi0; F.meta[s] = meta0;
+        // constant indices only: the slot table stays in registers
+        if (s) { F.pc[1] = pc0; F.koi[1] = koi0; F.meta[1] = meta0; }
+        else { F.pc[0] = pc0; F.koi[0] = koi0; F.meta[0] = meta0; }
         if ((lane >> 4) == s) acc = fast_identity(lane & 15);
         // line states this warp can skip (already FAIL in the CTA state)
         const int ps = pc0 < P.sp ? (int)pc0 : -1;
@@ -643,98 +772,56 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
           const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
           if (line_target(P, S, os, P.n_pcs + koi0)->state == VE_LINE_FAIL) lf |= 2u;
         }
-        F.lfail[s] = __shfl_sync(0xFFFFFFFFu, lf, 0);
+        lf = __shfl_sync(0xFFFFFFFFu, lf, 0);
         // dense per-element counting for loads of a real object that read the pre value
         const int oi0 = __shfl_sync(0xFFFFFFFFu, oi, l0);
-        F.dense[s] = (P.dense_ok && oi0 >= 0 && !meta_store(meta0)) ? dense_lookup(P, oi0, pc0) : 0ull;
+        const unsigned long long dn =
+            (P.dense_ok && oi0 >= 0 && !meta_store(meta0)) ? dense_lookup(P, oi0, pc0) : 0ull;
+        if (s) { F.lfail[1] = lf; F.dense[1] = dn; }
+        else { F.lfail[0] = lf; F.dense[0] = dn; }
       }
       F.mru = (uint32_t)s;
-      const uint32_t nv = __popc(vmask);
-      const uint32_t pA = valid ? ((uint32_t)(val == 0) | ((uint32_t)eq << 6) | ((uint32_t)!eqdef << 12)) : 0u;
-      const uint32_t A = __reduce_add_sync(0xFFFFFFFFu, pA);
-      uint32_t B = 0;
-      uint64_t rmin, rmax, omin, omax, tmin = ~0ull, tmax = 0;
-      const bool okv = valid && !f.nan;            // contributes to ord / trunc
-      // branch only on the WINDOW's access type (invalid lanes may carry any meta)
-      const uint32_t lg0 = meta0 & 3u, kind0 = (meta0 >> 2) & 3u;
-      const bool isf0 = kind0 >= 2u;
-      if (isf0) {
-        const uint32_t pB = valid ? ((ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) |
-                                     (((ff >> 3) & 1u) << 18) | (((ff >> 4) & 1u) << 24)) : 0u;
-        B = __reduce_add_sync(0xFFFFFFFFu, pB);
+      uint32_t lf_s = s ? F.lfail[1] : F.lfail[0];
+      const unsigned long long dn_s = s ? F.dense[1] : F.dense[0];
+      WinCtx x;
+      x.addr = addr; x.val = val; x.off = off; x.ew_lg = ew_lg;
+      x.valid = valid; x.eq = eq; x.eqdef = eqdef;
+      x.vmask = vmask; x.l0 = l0; x.pc0 = pc0; x.koi0 = koi0;
+      // specialised on the window's access type (compile-time width / kind)
+      switch (meta0 & 15u) {
+        case 0: fast_window<0, 0>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 1: fast_window<0, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 2: fast_window<0, 2>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 3: fast_window<0, 3>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 4: fast_window<1, 0>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 5: fast_window<1, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 6: fast_window<1, 2>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 7: fast_window<1, 3>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 9: fast_window<2, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 10: fast_window<2, 2>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        case 11: fast_window<2, 3>(P, S, lf_s, dn_s, s, acc, wc, x); break;
+        default: fast_window<3, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;   // 13: bfloat16
       }
-      if (lg0 < 3u) {
-        // w <= 4 bytes: every key fits 32 bits -> one REDUX per min / max
-        const uint32_t r32 = (uint32_t)val;
-        rmin = __reduce_min_sync(0xFFFFFFFFu, valid ? r32 : 0xFFFFFFFFu);
-        rmax = __reduce_max_sync(0xFFFFFFFFu, valid ? r32 : 0u);
-        if (kind0 == 0u) {
-          omin = rmin; omax = rmax;
-        } else {
-          const uint32_t k32 = (kind0 == 1u) ? ((uint32_t)f.y ^ 0x80000000u) : (uint32_t)f.ordv;
-          const unsigned okm = __ballot_sync(0xFFFFFFFFu, okv);
-          omin = __reduce_min_sync(0xFFFFFFFFu, okv ? k32 : 0xFFFFFFFFu);
-          omax = __reduce_max_sync(0xFFFFFFFFu, okv ? k32 : 0u);
-          if (isf0) {
-            tmin = __reduce_min_sync(0xFFFFFFFFu, okv ? (uint32_t)f.truncv : 0xFFFFFFFFu);
-            tmax = __reduce_max_sync(0xFFFFFFFFu, okv ? (uint32_t)f.truncv : 0u);
-          }
-          if (okm == 0) { omin = ~0ull; omax = 0; tmin = ~0ull; tmax = 0; }
-        }
-      } else {
-        rmin = redmin64(0xFFFFFFFFu, valid ? val : ~0ull);
-        rmax = redmax64(0xFFFFFFFFu, valid ? val : 0ull);
-        omin = redmin64(0xFFFFFFFFu, okv ? f.ordv : ~0ull);
-        omax = redmax64(0xFFFFFFFFu, okv ? f.ordv : 0ull);
-        if (isf0) {
-          tmin = redmin64(0xFFFFFFFFu, okv ? f.truncv : ~0ull);
-          tmax = redmax64(0xFFFFFFFFu, okv ? f.truncv : 0ull);
-        }
-      }
-      if ((lane >> 4) == s) {
-        const int fl = lane & 15;
-        if (fl == 0) acc += nv;
-        else if (fl <= 3) acc += (A >> (6 * (fl - 1))) & 63u;
-        else if (fl <= 8) acc += (B >> (6 * (fl - 4))) & 63u;
-        else if (fl <= 14) {
-          const int m = (fl - 9) >> 1;
-          if (fl & 1) {
-            const uint64_t v = m == 0 ? rmin : m == 1 ? omin : tmin;
-            acc = v < acc ? v : acc;
-          } else {
-            const uint64_t v = m == 0 ? rmax : m == 1 ? omax : tmax;
-            acc = v > acc ? v : acc;
-          }
-        }
-      }
-      // C8: one line state for the window, merged into each key not yet FAIL
-      if (F.lfail[s] != 3u) {
-        LinePts g;
-        g.state = VE_LINE_EMPTY;
-        if (valid) group_line(vmask, f, g);
-        const int ps = pc0 < P.sp ? (int)pc0 : -1;
-        const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
-        uint32_t lf = F.lfail[s];
-        if (lane == l0) {
-          if (!(lf & 1u) && wcache_merge(P, S, wc, pc0, ps, g) == VE_LINE_FAIL) lf |= 1u;
-          if (!(lf & 2u) && wcache_merge(P, S, wc, P.n_pcs + koi0, os, g) == VE_LINE_FAIL) lf |= 2u;
-        }
-        __syncwarp();
-        F.lfail[s] = __shfl_sync(0xFFFFFFFFu, lf, l0);
-      }
-      // S8: exact histogram.  A load that reads an unchanged whole element carries the
-      // pre-snapshot value of that element, so it is counted per element (a coalesced
-      // counter increment) and mapped to its value at report time; every other record
-      // is inserted per distinct value.
-      const bool dl = F.dense[s] != 0ull && eq && lg == ew_lg && (off & ((1ull << ew_lg) - 1)) == 0;
-      if (dl) atomicAdd(reinterpret_cast<uint32_t*>(F.dense[s]) + (off >> ew_lg), 1u);
-      const unsigned hmask = __ballot_sync(0xFFFFFFFFu, valid && !dl);
-      if (valid && !dl) {
-        const unsigned vg = (lg0 < 3u) ? __match_any_sync(hmask, (uint32_t)val) : __match_any_sync(hmask, val);
-        if (lane == __ffs(vg) - 1) hist_insert(P, S, (pc0 << 16) | (koi0 & 0xFFFFu), val, __popc(vg));
-      }
+      if (s) F.lfail[1] = lf_s;
+      else F.lfail[0] = lf_s;
     } else {
       // ---------------- slow path: per-key groups ----------------
+      Facts f;
+      f.addr = addr;
+      f.val = val;
+      f.tc = type_code(kind, lg);
+      f.isf = kind >= 2u;
+      int64_t ival = 0;
+      const uint32_t ff = f.isf ? float_flags(val, kind, lg, ival) : 0u;
+      f.nan = ff & 1u;
+      f.pfail = f.isf && (ff & 2u);
+      f.ordv = ord_key(val, kind, lg);
+      f.truncv = f.isf ? trunc_bits(val, kind, lg, P.mant_bits) : 0ull;
+      if (kind == 0u) f.y = (__int128)val;
+      else if (kind == 1u) {
+        const uint32_t sh64 = 64u - (8u << lg);
+        f.y = (__int128)((int64_t)(val << sh64) >> sh64);
+      } else f.y = (__int128)ival;
       f.packA = (uint32_t)st | ((uint32_t)(val == 0) << 6) | ((uint32_t)(eq && !st) << 12) |
                 ((uint32_t)(eq && st) << 18) | ((uint32_t)(!eqdef) << 24);
       f.packB = (ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) | (((ff >> 3) & 1u) << 18) |
@@ -768,8 +855,8 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   }
 
   // fold the warp's register slots and line cache, then the CTA's shared state
-  if (F.used & 1u) fast_flush(P, S, F, 0, acc);
-  if (F.used & 2u) fast_flush(P, S, F, 1, acc);
+  if (F.used & 1u) fast_flush(P, S, F.pc[0], F.koi[0], F.meta[0], 0, acc);
+  if (F.used & 2u) fast_flush(P, S, F.pc[1], F.koi[1], F.meta[1], 1, acc);
   if (lane == 0) {
     if (n_invalid) atomicAdd(&S.sctr[0], n_invalid);
     if (n_unmapped) atomicAdd(&S.sctr[1], n_unmapped);
