@@ -12,7 +12,21 @@
 
 #include "ve_internal.cuh"
 
+#include <chrono>
+#include <cstdlib>
+
 namespace ve {
+
+// VE_TIMING=2: per-stage timings of the report path on stderr
+static void stage(const char* name, cudaStream_t s) {
+  static const bool on = getenv("VE_TIMING") && atoi(getenv("VE_TIMING")) >= 2;
+  static auto t0 = std::chrono::steady_clock::now();
+  if (!on) return;
+  cudaStreamSynchronize(s);
+  const auto t1 = std::chrono::steady_clock::now();
+  fprintf(stderr, "[ve]   %-18s %.3f ms\n", name, std::chrono::duration<double, std::milli>(t1 - t0).count());
+  t0 = t1;
+}
 
 // ---- scratch management ------------------------------------------------------
 static cudaError_t scratch_need(ve_ctx* c, size_t bytes) {
@@ -66,22 +80,46 @@ __global__ void k_views(const HSlot* hs, const unsigned long long* hc, uint64_t 
   }
 }
 
+// Warp-aggregated counter increment: lanes with equal keys share one atomic (the
+// per-key counters are few and hot, so plain per-entry atomics serialise).
+// Every lane of the warp must call it; returns this lane's slot (cursor value).
+__device__ __forceinline__ unsigned long long warp_count(unsigned long long* ctr, bool active, uint32_t key) {
+  const unsigned am = __ballot_sync(0xFFFFFFFFu, active);
+  unsigned long long base = 0;
+  if (active) {
+    const unsigned g = __match_any_sync(am, key);
+    const int lead = __ffs(g) - 1, lane = threadIdx.x & 31;
+    if (lane == lead) base = atomicAdd(ctr, (unsigned long long)__popc(g));
+    base = __shfl_sync(g, base, lead);
+    base += __popc(g & ((1u << lane) - 1u));
+  }
+  return base;
+}
+
+// warp-uniform grid-stride loop over [0, n): every lane runs the same iterations
+#define VE_WARP_LOOP(i, n)                                                                        \
+  for (uint64_t i##_b = ((uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u)); i##_b < (n);  \
+       i##_b += (uint64_t)gridDim.x * blockDim.x)                                                 \
+    for (uint64_t i = i##_b + (threadIdx.x & 31u), i##_once = 1; i##_once; i##_once = 0)
+
 __global__ void k_view_count(const HSlot* vs, uint64_t vcap, unsigned long long* ndist) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < vcap; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t tag = vs[i].tag;
-    if (tag != EMPTY_TAG) atomicAdd(&ndist[tag], 1ull);
+  VE_WARP_LOOP(i, vcap) {
+    const uint32_t tag = i < vcap ? vs[i].tag : EMPTY_TAG;
+    warp_count(&ndist[tag != EMPTY_TAG ? tag : 0], tag != EMPTY_TAG, tag);
   }
 }
 
 __global__ void k_view_scatter(const HSlot* vs, const unsigned long long* vc, uint64_t vcap,
                                const unsigned long long* off, unsigned long long* cursor, uint64_t* gbits,
                                uint64_t* gcnt) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < vcap; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t tag = vs[i].tag;
-    if (tag == EMPTY_TAG) continue;
-    const unsigned long long p = off[tag] + atomicAdd(&cursor[tag], 1ull);
-    gbits[p] = vs[i].bits;
-    gcnt[p] = vc[i];
+  VE_WARP_LOOP(i, vcap) {
+    const uint32_t tag = i < vcap ? vs[i].tag : EMPTY_TAG;
+    const bool act = tag != EMPTY_TAG;
+    const unsigned long long p = warp_count(&cursor[act ? tag : 0], act, tag);
+    if (act) {
+      gbits[off[tag] + p] = vs[i].bits;
+      gcnt[off[tag] + p] = vc[i];
+    }
   }
 }
 
@@ -89,6 +127,9 @@ struct Chunk {
   uint64_t start, out;
   uint32_t len, nout;
 };
+
+ve_status select_topk(ve_ctx* c, cudaStream_t s, uint64_t* gb[2], uint64_t* gc[2], std::vector<uint64_t> len,
+                      std::vector<uint64_t> start, std::vector<ve_topk_entry>& top);
 
 constexpr int TK_THREADS = 256;
 constexpr int TK_PER = 16;
@@ -246,9 +287,25 @@ ve_status view_topk(ve_ctx* c, const ViewTable& V, cudaStream_t s, std::vector<u
   cudaMemcpyAsync(d_off, off.data(), (size_t)nk * 8, cudaMemcpyHostToDevice, s);
   count_launch();
   k_view_scatter<<<grid, 256, 0, s>>>(vs, vc, vcap, d_off, d_cur, gb[0], gc[0]);
-
-  // selection levels
   std::vector<uint64_t> len(ndistinct.begin(), ndistinct.end()), start(off.begin(), off.end());
+  ve_status st = select_topk(c, s, gb, gc, len, start, top);
+  cudaFreeAsync(d_small, s);
+  cudaFreeAsync(gbuf, s);
+  cudaFreeAsync(d_nd, s);
+  if (st != VE_OK) return st;
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "finalize top-k");
+  return VE_OK;
+}
+
+// Top-k by (count desc, bits asc) of every key whose distinct entries lie in
+// gb/gc[0][start[k] .. start[k]+len[k]): chunked block-wide selection, repeated
+// on the chunk winners until every key fits one chunk.
+ve_status select_topk(ve_ctx* c, cudaStream_t s, uint64_t* gb[2], uint64_t* gc[2], std::vector<uint64_t> len,
+                      std::vector<uint64_t> start, std::vector<ve_topk_entry>& top) {
+  const uint32_t nk = c->n_keys, K = c->cfg.topk;
+  cudaError_t e;
+  unsigned long long* d_small = nullptr;
   int cur = 0;
   Chunk* d_chunks = nullptr;
   size_t chunk_cap = 0;
@@ -281,9 +338,11 @@ ve_status view_topk(ve_ctx* c, const ViewTable& V, cudaStream_t s, std::vector<u
       if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize chunks"); }
     }
     cudaMemcpyAsync(d_chunks, chunks.data(), chunks.size() * sizeof(Chunk), cudaMemcpyHostToDevice, s);
+    stage("chunk build", s);
     count_launch();
     k_topk_chunk<<<(unsigned)chunks.size(), TK_THREADS, 0, s>>>(d_chunks, gb[cur], gc[cur], gb[1 - cur],
                                                                 gc[1 - cur]);
+    stage("topk level", s);
     cur = 1 - cur;
     len.swap(nlen);
     start.swap(nstart);
@@ -299,17 +358,193 @@ ve_status view_topk(ve_ctx* c, const ViewTable& V, cudaStream_t s, std::vector<u
     }
   }
   if (d_chunks) cudaFreeAsync(d_chunks, s);
-  cudaFreeAsync(d_small, s);
-  cudaFreeAsync(gbuf, s);
-  cudaFreeAsync(d_nd, s);
+  (void)d_small;
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "finalize top-k");
   return VE_OK;
 }
 
+// ---- finalize with direct grouping ------------------------------------------------
+// A key whose entries all carry one tag (a PC that touched one object, an object
+// touched by one PC -- the common case) needs no re-aggregation: its main-table
+// entries ARE its distinct values.  Only keys fed by several tags go through the
+// view table.
+constexpr uint32_t TAG_CAP = 1u << 16;
+
+__global__ void k_tagscan(const HSlot* hs, uint64_t cap, uint32_t* tags, unsigned long long* tcnt,
+                          unsigned long long* ovf) {
+  VE_WARP_LOOP(i, cap) {
+    const uint32_t tag = i < cap ? hs[i].tag : EMPTY_TAG;
+    uint32_t h = (uint32_t)mix64(tag) & (TAG_CAP - 1);
+    bool done = tag == EMPTY_TAG;
+    for (int p = 0; p < 64 && !done; ++p) {
+      uint32_t old = *(volatile uint32_t*)&tags[h];            // read first: the hot tags are already in
+      if (old == EMPTY_TAG) old = atomicCAS(&tags[h], EMPTY_TAG, tag);
+      if (old == EMPTY_TAG || old == tag) done = true;
+      else h = (h + 1) & (TAG_CAP - 1);
+    }
+    if (!done) atomicExch(ovf, 1ull);
+    const bool act = tag != EMPTY_TAG && done;
+    warp_count(&tcnt[act ? h : 0], act, h);
+  }
+}
+
+__global__ void k_emit(const HSlot* hs, const unsigned long long* hc, uint64_t cap, uint32_t n_pcs,
+                       const uint8_t* direct, const unsigned long long* off, unsigned long long* cur, uint64_t* gb,
+                       uint64_t* gc, HSlot* vs, unsigned long long* vc, uint64_t vmask, unsigned long long* ovf) {
+  VE_WARP_LOOP(i, cap) {
+    const uint32_t tag = i < cap ? hs[i].tag : EMPTY_TAG;
+    const bool occ = tag != EMPTY_TAG;
+    const uint64_t bits = occ ? hs[i].bits : 0;
+    const unsigned long long cnt = occ ? hc[i] : 0;
+    const uint32_t koi = tag & 0xFFFFu;
+    for (int side = 0; side < 2; ++side) {
+      const bool act = occ && !(side == 1 && koi == KO_NONE);
+      const uint32_t key = act ? (side == 0 ? (tag >> 16) : n_pcs + koi) : 0;
+      const bool dir = act && direct[key];
+      const unsigned long long p = warp_count(&cur[key], dir, key);
+      if (dir) {
+        gb[off[key] + p] = bits;
+        gc[off[key] + p] = cnt;
+      } else if (act) {
+        vinsert(vs, vc, vmask, ovf, key, bits, cnt);
+      }
+    }
+  }
+}
+
 // Exact n_distinct and top-k of every key (PC keys, then object keys).
 ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
                         std::vector<ve_topk_entry>& top) {
+  const uint32_t nk = c->n_keys, K = c->cfg.topk, npc = c->cfg.n_pcs;
+  ndistinct.assign(nk, 0);
+  top.assign((size_t)nk * K, ve_topk_entry{0, 0});
+  cudaError_t e;
+  const int grid = c->num_sms * 4;
+  // 1. distinct tags and their entry counts
+  uint32_t* d_tags = nullptr;
+  unsigned long long* d_tcnt = nullptr;
+  unsigned long long* d_small = nullptr;     // [0] overflow
+  e = cudaMallocAsync((void**)&d_tags, TAG_CAP * 4, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_tcnt, TAG_CAP * 8, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_small, 16, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "finalize alloc");
+  cudaMemsetAsync(d_tags, 0xFF, TAG_CAP * 4, s);
+  cudaMemsetAsync(d_tcnt, 0, TAG_CAP * 8, s);
+  cudaMemsetAsync(d_small, 0, 16, s);
+  stage("start", s);
+  count_launch();
+  k_tagscan<<<grid, 256, 0, s>>>(c->t.hslot, c->hcap, d_tags, d_tcnt, d_small);
+  std::vector<uint32_t> tags(TAG_CAP);
+  std::vector<unsigned long long> tcnt(TAG_CAP);
+  unsigned long long ovf = 0;
+  cudaMemcpyAsync(tags.data(), d_tags, TAG_CAP * 4, cudaMemcpyDeviceToHost, s);
+  cudaMemcpyAsync(tcnt.data(), d_tcnt, TAG_CAP * 8, cudaMemcpyDeviceToHost, s);
+  cudaMemcpyAsync(&ovf, d_small, 8, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d_tags, s);
+  cudaFreeAsync(d_tcnt, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize tags"); }
+  stage("tagscan+d2h", s);
+  if (ovf) {                                  // too many distinct tags: aggregate every key
+    cudaFreeAsync(d_small, s);
+    ViewTable V;
+    ve_status st = build_views(c, s, V);
+    if (st == VE_OK) st = view_topk(c, V, s, ndistinct, top);
+    free_views(V, s);
+    return st;
+  }
+  // 2. classify keys: direct (one tag) or aggregated (several tags)
+  std::vector<uint32_t> ntag(nk, 0);
+  std::vector<uint64_t> ent(nk, 0);
+  for (uint32_t i = 0; i < TAG_CAP; ++i) {
+    if (tags[i] == EMPTY_TAG) continue;
+    const uint32_t pk = tags[i] >> 16, koi = tags[i] & 0xFFFFu;
+    ntag[pk]++;
+    ent[pk] += tcnt[i];
+    if (koi != KO_NONE) {
+      ntag[npc + koi]++;
+      ent[npc + koi] += tcnt[i];
+    }
+  }
+  std::vector<uint8_t> direct(nk, 0);
+  std::vector<unsigned long long> off(nk, 0);
+  uint64_t pos = 0, agg_in = 0;
+  for (uint32_t k = 0; k < nk; ++k) {
+    if (ntag[k] == 1) {
+      direct[k] = 1;
+      off[k] = pos;
+      ndistinct[k] = ent[k];
+      pos += ent[k];
+    } else if (ntag[k] > 1) {
+      agg_in += ent[k];
+    }
+  }
+  const uint64_t nent = pos + agg_in + 1;
+  uint64_t* gbuf = nullptr;
+  uint8_t* d_direct = nullptr;
+  unsigned long long* d_off = nullptr;      // off, cur
+  e = cudaMallocAsync((void**)&gbuf, 4 * nent * 8, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_direct, nk, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_off, 16ull * nk, s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize alloc"); }
+  uint64_t* gb[2] = {gbuf, gbuf + 2 * nent};
+  uint64_t* gc[2] = {gbuf + nent, gbuf + 3 * nent};
+  cudaMemcpyAsync(d_direct, direct.data(), nk, cudaMemcpyHostToDevice, s);
+  cudaMemcpyAsync(d_off, off.data(), 8ull * nk, cudaMemcpyHostToDevice, s);
+  cudaMemsetAsync(d_off + nk, 0, 8ull * nk, s);
+  ViewTable V;
+  ve_status st = VE_OK;
+  if (agg_in) st = alloc_views(c, s, agg_in, V);
+  if (st != VE_OK) { cudaFreeAsync(d_small, s); return st; }
+  stage("alloc", s);
+  // 3. emit direct keys' entries, aggregate the others in the view table
+  count_launch();
+  k_emit<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, npc, d_direct, d_off, d_off + nk, gb[0], gc[0],
+                              V.vs, V.vc, V.vcap ? V.vcap - 1 : 0, d_small);
+  if (agg_in) {
+    unsigned long long* d_nd = nullptr;
+    cudaMallocAsync((void**)&d_nd, 8ull * nk, s);
+    cudaMemsetAsync(d_nd, 0, 8ull * nk, s);
+    count_launch();
+    k_view_count<<<grid, 256, 0, s>>>(V.vs, V.vcap, d_nd);
+    std::vector<uint64_t> nd(nk);
+    cudaMemcpyAsync(nd.data(), d_nd, 8ull * nk, cudaMemcpyDeviceToHost, s);
+    cudaFreeAsync(d_nd, s);
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize views"); }
+    for (uint32_t k = 0; k < nk; ++k)
+      if (!direct[k] && nd[k]) {
+        off[k] = pos;
+        ndistinct[k] = nd[k];
+        pos += nd[k];
+      }
+    cudaMemcpyAsync(d_off, off.data(), 8ull * nk, cudaMemcpyHostToDevice, s);
+    count_launch();
+    k_view_scatter<<<grid, 256, 0, s>>>(V.vs, V.vc, V.vcap, d_off, d_off + nk, gb[0], gc[0]);
+  }
+  stage("emit+views", s);
+  // 4. top-k per key
+  std::vector<uint64_t> len(ndistinct.begin(), ndistinct.end()), start(off.begin(), off.end());
+  st = select_topk(c, s, gb, gc, len, start, top);
+  stage("select_topk", s);
+  unsigned long long h_ovf = 0;
+  cudaMemcpyAsync(&h_ovf, d_small, 8, cudaMemcpyDeviceToHost, s);
+  free_views(V, s);
+  cudaFreeAsync(gbuf, s);
+  cudaFreeAsync(d_direct, s);
+  cudaFreeAsync(d_off, s);
+  cudaFreeAsync(d_small, s);
+  e = cudaStreamSynchronize(s);
+  if (st != VE_OK) return st;
+  if (e != cudaSuccess) return cuda_fail(c, e, "finalize");
+  if (h_ovf) return fail(c, VE_ERR_CAPACITY, "finalize: view table overflow");
+  return VE_OK;
+}
+
+// (reference path: every key aggregated through the view table)
+ve_status finalize_hist_views(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
+                              std::vector<ve_topk_entry>& top) {
   ViewTable V;
   ve_status st = build_views(c, s, V);
   if (st == VE_OK) st = view_topk(c, V, s, ndistinct, top);

@@ -2,7 +2,7 @@
 # iteration loop on the GPU box: parity tests, step timing, bench, gemm-launch ncu capture
 cd "${GRAFT_REPO_ROOT:-.}"; mkdir -p gpurun_out
 timeout 900 python -m pytest tests/ -x -q -m gpu > gpurun_out/gpu_tests.log 2>&1; echo "exit $?" >> gpurun_out/gpu_tests.log
-VE_TIMING=1 timeout 300 python scripts/step_timing.py > gpurun_out/step_timing.log 2>&1
+VE_TIMING=2 timeout 300 python scripts/step_timing.py > gpurun_out/step_timing.log 2>&1
 timeout 900 python bench.py --steps 5 --warmup 3 ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench exit $?" >> gpurun_out/bench.err
 if [ "${NCU:-1}" = "1" ]; then
 timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_analyze -s 3 -c 1 -f \
