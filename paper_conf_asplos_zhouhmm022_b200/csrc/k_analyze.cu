@@ -26,9 +26,9 @@
 
 namespace ve {
 
-constexpr int K1_THREADS = 384;  // 12 warps x <=168 registers: the fast path runs spill-free
+constexpr int K1_THREADS = 512;  // 16 warps x 128 registers
 constexpr int K1_WARPS = K1_THREADS / 32;
-constexpr int RING = 8;                      // record windows in flight per warp (TMA ring)
+constexpr int RING = 6;                      // record windows in flight per warp (TMA ring)
 constexpr uint32_t WIN_BYTES = 32 * sizeof(ve_record);
 
 struct AnalyzeParams {
