@@ -426,8 +426,11 @@ __device__ __noinline__ void fast_flush(const AnalyzeParams& P, const Smem& S, u
 // per-lane facts of a uniform window handed to its specialised fast path
 struct WinCtx {
   uint64_t addr, val, off;
+  uint64_t pv;            // pre-snapshot bytes (load in flight), valid iff eqdef
+  uint64_t lw0;           // L bitmap word of the first element
+  uint32_t lbit;
   uint32_t ew_lg;
-  bool valid, eq, eqdef;
+  bool valid, eqdef, inside, st;
   unsigned vmask;
   int l0;
   uint32_t pc0, koi0;
@@ -454,8 +457,6 @@ __device__ __forceinline__ void fast_window(const AnalyzeParams& P, const Smem& 
   const uint32_t ff = ISF ? float_flags(val, KIND, LG, ival) : 0u;
   const bool okv = valid && !(ff & 1u);       // contributes to ord / trunc (NaNs excluded)
   const uint32_t nv = __popc(x.vmask);
-  const uint32_t pA = valid ? ((uint32_t)(val == 0) | ((uint32_t)x.eq << 6) | ((uint32_t)!x.eqdef << 12)) : 0u;
-  const uint32_t A = __reduce_add_sync(0xFFFFFFFFu, pA);
   uint32_t B = 0;
   if (ISF) {
     const uint32_t pB = valid ? ((ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) |
@@ -504,6 +505,12 @@ __device__ __forceinline__ void fast_window(const AnalyzeParams& P, const Smem& 
       }
     }
   }
+  // the pre-snapshot gather is consumed only now
+  const bool eq = x.eqdef && x.pv == val;
+  const uint32_t pA = valid ? ((uint32_t)(val == 0) | ((uint32_t)eq << 6) | ((uint32_t)!x.eqdef << 12)) : 0u;
+  const uint32_t A = __reduce_add_sync(0xFFFFFFFFu, pA);
+  const bool lpart = x.inside && !x.st && eq;
+  if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, x.lw0, x.lbit);   // C3 loaded elements
   if ((lane >> 4) == s) {
     const int fl = lane & 15;
     if (fl == 0) acc += nv;
@@ -549,7 +556,7 @@ __device__ __forceinline__ void fast_window(const AnalyzeParams& P, const Smem& 
   // pre-snapshot value of that element, so it is counted per element (a coalesced
   // counter increment) and mapped to its value at report time; every other record
   // is inserted per distinct value.
-  const bool dl = dense_s != 0ull && x.eq && (uint32_t)LG == x.ew_lg && (x.off & ((1ull << LG) - 1)) == 0;
+  const bool dl = dense_s != 0ull && eq && (uint32_t)LG == x.ew_lg && (x.off & ((1ull << LG) - 1)) == 0;
   if (dl) atomicAdd(reinterpret_cast<uint32_t*>(dense_s) + (x.off >> LG), 1u);
   const unsigned hmask = __ballot_sync(0xFFFFFFFFu, valid && !dl);
   if (valid && !dl) {
@@ -715,10 +722,13 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
     const uint64_t bmoff = mapped ? obm : 0ull;
     const bool inside = mapped && addr + (1u << lg) <= oe;
     const bool eqdef = inside && opre != 0ull;
-    const bool eq = eqdef && load_pre(opre + off, lg) == val;
+    // issue the pre-snapshot gather now, consume it as late as possible (latency hiding)
+    const uint64_t pv = eqdef ? load_pre(opre + off, lg) : 0ull;
     const uint32_t koi = sh ? P.n_obj : (mapped ? oid : KO_NONE);
+    const uint64_t lw0 = bmoff + ((off >> ew_lg) >> 5);        // L bitmap word / bit of the first element
+    const uint32_t lbit = 1u << ((off >> ew_lg) & 31);
 
-    // W / L element bitmaps (C3, C10)
+    // W element bitmap (C10); L is set once eq_pre is known
     {
       const bool wpart = inside && st;
       const uint64_t e0 = off >> ew_lg, e1 = (off + (1u << lg) - 1) >> ew_lg;
@@ -736,8 +746,6 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
         const bool spill = wpart && w1 != w0;
         if (__any_sync(0xFFFFFFFFu, spill)) bitmap_or(P.t.W, spill, w1, b1);
       }
-      const bool lpart = inside && !st && eq;
-      if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, w0, 1u << (e0 & 31));
     }
 
     // uniform window? (pc, access type and object shared by every valid lane)
@@ -785,7 +793,8 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
       const unsigned long long dn_s = s ? F.dense[1] : F.dense[0];
       WinCtx x;
       x.addr = addr; x.val = val; x.off = off; x.ew_lg = ew_lg;
-      x.valid = valid; x.eq = eq; x.eqdef = eqdef;
+      x.valid = valid; x.eqdef = eqdef; x.inside = inside; x.st = st;
+      x.pv = pv; x.lw0 = lw0; x.lbit = lbit;
       x.vmask = vmask; x.l0 = l0; x.pc0 = pc0; x.koi0 = koi0;
       // specialised on the window's access type (compile-time width / kind)
       switch (meta0 & 15u) {
@@ -806,6 +815,9 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
       else F.lfail[0] = lf_s;
     } else {
       // ---------------- slow path: per-key groups ----------------
+      const bool eq = eqdef && pv == val;
+      const bool lpart = inside && !st && eq;
+      if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, lw0, lbit);   // C3 loaded elements
       Facts f;
       f.addr = addr;
       f.val = val;
