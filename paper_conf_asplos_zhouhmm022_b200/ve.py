@@ -58,7 +58,7 @@ class _Object(ctypes.Structure):
 def lib():
     global _LIB
     if _LIB is None:
-        path = os.path.join(_HERE, "libve.so")
+        path = os.environ.get("VE_LIB_PATH") or os.path.join(_HERE, "libve.so")   # override: A/B of builds
         if not os.path.exists(path):
             raise RuntimeError(f"{path} missing: run __graft_entry__.build() (no CPU fallback exists)")
         L = ctypes.CDLL(path)
