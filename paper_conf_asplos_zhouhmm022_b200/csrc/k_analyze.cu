@@ -41,6 +41,8 @@ struct AnalyzeParams {
   uint32_t objc;            // objects cached in shared memory (0 = use global table)
   uint32_t dense_ok;        // dense per-element counting enabled for this launch
   uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
+  // byte offsets of the dynamic shared-memory regions (see carve_offsets)
+  uint32_t o_ssum, o_smin, o_smax, o_sline, o_shs, o_shc, o_sob, o_soe, o_sctr, o_ring, o_bars;
   DevObjects o;
   DevTables t;
 };
@@ -74,20 +76,38 @@ __host__ __device__ inline size_t smem_bytes(uint32_t nsk, uint32_t hs, uint32_t
   return b;
 }
 
-__device__ inline Smem carve(uint8_t* base, uint32_t nsk, uint32_t hs, uint32_t objc) {
-  Smem s;
+// region offsets, computed once on the host (kernel code reads them from the
+// constant bank, so no pointer table lives in registers or on the stack)
+inline void carve_offsets(AnalyzeParams& P, uint32_t nsk) {
   size_t off = 0;
-  s.ssum = (uint32_t*)(base + off); off += align16(sizeof(uint32_t) * nsk * NSUM);
-  s.smin = (unsigned long long*)(base + off); off += align16(sizeof(unsigned long long) * nsk * NMM);
-  s.smax = (unsigned long long*)(base + off); off += align16(sizeof(unsigned long long) * nsk * NMM);
-  s.sline = (LineState*)(base + off); off += align16(sizeof(LineState) * nsk);
-  s.shs = (HSlot*)(base + off); off += align16(sizeof(HSlot) * hs);
-  s.shc = (uint32_t*)(base + off); off += align16(sizeof(uint32_t) * hs);
-  s.sob = (uint64_t*)(base + off); off += align16(sizeof(uint64_t) * objc);
-  s.soe = (uint64_t*)(base + off); off += align16(sizeof(uint64_t) * objc);
-  s.sctr = (uint32_t*)(base + off); off += 16;
-  s.ring = base + off; off += (size_t)K1_WARPS * RING * WIN_BYTES;
-  s.bars = (uint64_t*)(base + off);
+  P.o_ssum = (uint32_t)off; off += align16(sizeof(uint32_t) * nsk * NSUM);
+  P.o_smin = (uint32_t)off; off += align16(sizeof(unsigned long long) * nsk * NMM);
+  P.o_smax = (uint32_t)off; off += align16(sizeof(unsigned long long) * nsk * NMM);
+  P.o_sline = (uint32_t)off; off += align16(sizeof(LineState) * nsk);
+  P.o_shs = (uint32_t)off; off += align16(sizeof(HSlot) * P.hs);
+  P.o_shc = (uint32_t)off; off += align16(sizeof(uint32_t) * P.hs);
+  P.o_sob = (uint32_t)off; off += align16(sizeof(uint64_t) * P.objc);
+  P.o_soe = (uint32_t)off; off += align16(sizeof(uint64_t) * P.objc);
+  P.o_sctr = (uint32_t)off; off += 16;
+  P.o_ring = (uint32_t)off; off += (size_t)K1_WARPS * RING * WIN_BYTES;
+  P.o_bars = (uint32_t)off;
+}
+
+extern __shared__ __align__(16) uint8_t ve_smem[];
+
+__device__ __forceinline__ Smem smem_of(const AnalyzeParams& P) {
+  Smem s;
+  s.ssum = (uint32_t*)(ve_smem + P.o_ssum);
+  s.smin = (unsigned long long*)(ve_smem + P.o_smin);
+  s.smax = (unsigned long long*)(ve_smem + P.o_smax);
+  s.sline = (LineState*)(ve_smem + P.o_sline);
+  s.shs = (HSlot*)(ve_smem + P.o_shs);
+  s.shc = (uint32_t*)(ve_smem + P.o_shc);
+  s.sob = (uint64_t*)(ve_smem + P.o_sob);
+  s.soe = (uint64_t*)(ve_smem + P.o_soe);
+  s.sctr = (uint32_t*)(ve_smem + P.o_sctr);
+  s.ring = ve_smem + P.o_ring;
+  s.bars = (uint64_t*)(ve_smem + P.o_bars);
   return s;
 }
 
@@ -183,8 +203,9 @@ __device__ __noinline__ void group_line(unsigned gm, const Facts& f, LinePts& g)
 
 // Slow path: reduce one key group (all lanes in gm share the key) and fold it into
 // the key's row: shared memory when slot >= 0, else the global table.
-__device__ __noinline__ void apply_group(const AnalyzeParams& P, const Smem& S, unsigned gm, int slot,
+__device__ __noinline__ void apply_group(const AnalyzeParams& P, unsigned gm, int slot,
                                             uint32_t key, const Facts& f, LinePts& g) {
+  const Smem S = smem_of(P);
   const int lane = threadIdx.x & 31;
   const unsigned gsize = __popc(gm);
   const int rank = __popc(gm & lanemask_lt());
@@ -246,19 +267,21 @@ struct WarpCache {
   LineState st[WC];
 };
 
-__device__ __forceinline__ LineState* line_target(const AnalyzeParams& P, const Smem& S, int slot, uint32_t key) {
+__device__ __forceinline__ LineState* line_target(const AnalyzeParams& P, int slot, uint32_t key) {
+  const Smem S = smem_of(P);
   return (slot >= 0) ? &S.sline[slot] : &P.t.line[key];
 }
 
 // returns the key's merged (warp-local) state
-__device__ __noinline__ uint32_t wcache_merge(const AnalyzeParams& P, const Smem& S, WarpCache& C, uint32_t key,
+__device__ __noinline__ uint32_t wcache_merge(const AnalyzeParams& P, WarpCache& C, uint32_t key,
                                                  int slot, const LinePts& g) {
+  const Smem S = smem_of(P);
   for (int i = 0; i < WC; ++i) {
     if (C.key1[i] == key + 1) {
       const LinePts a = line_load(C.st[i]);
       const LinePts r = line_merge(a, g);
       line_store(C.st[i], r);
-      if (r.state == VE_LINE_FAIL && a.state != VE_LINE_FAIL) line_merge_locked(line_target(P, S, slot, key), r);
+      if (r.state == VE_LINE_FAIL && a.state != VE_LINE_FAIL) line_merge_locked(line_target(P, slot, key), r);
       return r.state;
     }
   }
@@ -267,39 +290,42 @@ __device__ __noinline__ uint32_t wcache_merge(const AnalyzeParams& P, const Smem
     if (C.key1[i] == 0) { v = i; break; }
   if (v < 0) {
     v = (int)(C.next++ % WC);
-    line_merge_locked(line_target(P, S, C.slot[v], C.key1[v] - 1), line_load(C.st[v]));
+    line_merge_locked(line_target(P, C.slot[v], C.key1[v] - 1), line_load(C.st[v]));
   }
   C.key1[v] = key + 1;
   C.slot[v] = slot;
   line_store(C.st[v], g);
-  if (g.state == VE_LINE_FAIL) line_merge_locked(line_target(P, S, slot, key), g);
+  if (g.state == VE_LINE_FAIL) line_merge_locked(line_target(P, slot, key), g);
   return g.state;
 }
 
-__device__ __noinline__ void wcache_flush(const AnalyzeParams& P, const Smem& S, WarpCache& C) {
+__device__ __noinline__ void wcache_flush(const AnalyzeParams& P, WarpCache& C) {
+  const Smem S = smem_of(P);
   for (int i = 0; i < WC; ++i) {
     if (C.key1[i]) {
-      if (C.st[i].state != VE_LINE_FAIL) line_merge_locked(line_target(P, S, C.slot[i], C.key1[i] - 1), line_load(C.st[i]));
+      if (C.st[i].state != VE_LINE_FAIL) line_merge_locked(line_target(P, C.slot[i], C.key1[i] - 1), line_load(C.st[i]));
       C.key1[i] = 0;
     }
   }
 }
 
 // serialise the merges of this window's group leaders through the warp cache
-__device__ __noinline__ void merge_lines(const AnalyzeParams& P, const Smem& S, WarpCache& C, bool lead,
+__device__ __noinline__ void merge_lines(const AnalyzeParams& P, WarpCache& C, bool lead,
                                             uint32_t key, int slot, const LinePts& g) {
+  const Smem S = smem_of(P);
   unsigned L = __ballot_sync(0xFFFFFFFFu, lead && g.state != VE_LINE_EMPTY);
   while (L) {
     const int l = __ffs(L) - 1;
     L &= L - 1;
-    if ((int)(threadIdx.x & 31) == l) wcache_merge(P, S, C, key, slot, g);
+    if ((int)(threadIdx.x & 31) == l) wcache_merge(P, C, key, slot, g);
     __syncwarp();
   }
 }
 
 // Insert a group of equal (tag, bits) with count c: shared table first, HBM table on miss/full.
-__device__ __forceinline__ void hist_insert(const AnalyzeParams& P, const Smem& S, uint32_t tag, uint64_t bits,
+__device__ __forceinline__ void hist_insert(const AnalyzeParams& P, uint32_t tag, uint64_t bits,
                                             uint32_t c) {
+  const Smem S = smem_of(P);
   const uint32_t hmask = P.hs - 1;
   uint32_t h = (uint32_t)hist_hash(tag, bits) & hmask;
   for (int probe = 0; probe < 16; ++probe) {
@@ -324,7 +350,8 @@ __device__ __forceinline__ void hist_insert(const AnalyzeParams& P, const Smem& 
   hist_insert_global(P.t, tag, bits, c);
 }
 
-__device__ __noinline__ int find_object(const AnalyzeParams& P, const Smem& S, uint64_t addr) {
+__device__ __noinline__ int find_object(const AnalyzeParams& P, uint64_t addr) {
+  const Smem S = smem_of(P);
   const uint64_t* base = P.objc ? S.sob : P.o.base;
   int lo = 0, hi = (int)P.o.n;  // first object with base > addr
   while (lo < hi) {
@@ -350,11 +377,11 @@ __device__ __forceinline__ void bitmap_or(uint32_t* bm, bool part, uint64_t word
 //  0 n   1 n_zero   2 n_eq_pre   3 n_nosnap   4 nan   5 nonint   6 not_f16   7 not_bf16
 //  8 not_f32   9 raw_min 10 raw_max 11 ord_min 12 ord_max 13 trunc_min 14 trunc_max
 // For w <= 4 the ord fields of signed types hold sext32(b)^2^31 (order-isomorphic),
-// converted to the 64-bit key at flush.
+// converted to the 64-bit key at flush.  A slot is keyed by (meta, object id, pc).
 struct FastSlots {
-  uint32_t pc[2], koi[2], meta[2];
-  uint32_t used, mru;
-  uint32_t lfail[2];     // bit0: PC key line FAIL, bit1: object key line FAIL (known to this warp)
+  uint64_t key[2];              // meta << 32 | object id << 16 | pc; ~0 = unused
+  uint32_t mru;
+  uint32_t lfail[2];            // bit0: PC key line FAIL, bit1: object key line FAIL (known to this warp)
   unsigned long long dense[2];  // per-element counters of this (pc, object), or 0
 };
 
@@ -379,12 +406,23 @@ __device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, 
   return __shfl_sync(0xFFFFFFFFu, dp, 0);
 }
 
+// line states of (pc, object id) this warp can skip (already FAIL in the CTA state)
+__device__ __noinline__ uint32_t slot_lfail(const AnalyzeParams& P, uint32_t pc, uint32_t koi) {
+  const Smem S = smem_of(P);
+  const int ps = pc < P.sp ? (int)pc : -1;
+  const int os = koi < P.so ? (int)(P.sp + koi) : -1;
+  uint32_t lf = (line_target(P, ps, pc)->state == VE_LINE_FAIL) ? 1u : 0u;
+  if (line_target(P, os, P.n_pcs + koi)->state == VE_LINE_FAIL) lf |= 2u;
+  return __shfl_sync(0xFFFFFFFFu, lf, 0);
+}
+
 __device__ __forceinline__ uint64_t fast_identity(int f) {
   return (f >= 9 && (f & 1)) ? ~0ull : 0ull;
 }
 
-__device__ __forceinline__ void fold_row(const AnalyzeParams& P, const Smem& S, int slot, uint32_t key, int f,
+__device__ __forceinline__ void fold_row(const AnalyzeParams& P, int slot, uint32_t key, int f,
                                          uint32_t field, uint64_t v) {
+  const Smem S = smem_of(P);
   if (f <= 8 || f == 15) {
     if (slot >= 0) atomicAdd(&S.ssum[slot * NSUM + field], (uint32_t)v);
     else atomicAdd(&P.t.sum[(uint64_t)key * NSUM + field], (unsigned long long)v);
@@ -396,11 +434,13 @@ __device__ __forceinline__ void fold_row(const AnalyzeParams& P, const Smem& S, 
 }
 
 // fold slot s's accumulators into the PC-key row and the object-key row (lanes of half s)
-__device__ __noinline__ void fast_flush(const AnalyzeParams& P, const Smem& S, uint32_t pc, uint32_t koi,
-                                        uint32_t meta, int s, uint64_t acc) {
+__device__ __noinline__ void fast_flush(const AnalyzeParams& P, uint64_t skey, int s, uint64_t acc) {
+  const Smem S = smem_of(P);
   const int lane = threadIdx.x & 31;
   const uint64_t nrec = __shfl_sync(0xFFFFFFFFu, acc, s * 16);   // field 0 of slot s
   if ((lane >> 4) != s) return;
+  const uint32_t pc = (uint32_t)skey & 0xFFFFu, koi = (uint32_t)(skey >> 16) & 0xFFFFu;
+  const uint32_t meta = (uint32_t)(skey >> 32);
   const int f = lane & 15;
   const uint32_t lg = meta & 3u, kind = (meta >> 2) & 3u;
   const bool st = meta_store(meta);
@@ -419,179 +459,84 @@ __device__ __noinline__ void fast_flush(const AnalyzeParams& P, const Smem& S, u
     const int32_t sv = (int32_t)((uint32_t)v ^ 0x80000000u);
     v = (uint64_t)(int64_t)sv ^ (1ull << 63);
   }
-  fold_row(P, S, pc < P.sp ? (int)pc : -1, pc, f, field, v);
-  if (koi != KO_NONE) fold_row(P, S, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
-}
-
-// per-lane facts of a uniform window handed to its specialised fast path
-struct WinCtx {
-  uint64_t addr, val, off;
-  uint64_t pv;            // pre-snapshot bytes (load in flight), valid iff eqdef
-  uint64_t lw0;           // L bitmap word of the first element
-  uint32_t lbit;
-  uint32_t ew_lg;
-  bool valid, eqdef, inside, st;
-  unsigned vmask;
-  int l0;
-  uint32_t pc0, koi0;
-};
-
-// warp-uniform cache of the last object a window mapped to
-struct ObjCache {
-  int oi;
-  uint64_t base, end, bmoff, pre;
-  uint32_t id, ewlg;
-};
-
-// Fast path of a uniform window whose access type (KIND, LG = log2 width) is a
-// compile-time constant: the bit tests of C5-C8 specialise to the type.
-template <int KIND, int LG>
-__device__ __forceinline__ void fast_window(const AnalyzeParams& P, const Smem& S, uint32_t& lfail_s,
-                                            unsigned long long dense_s, int s, uint64_t& acc, WarpCache& wc,
-                                            const WinCtx& x) {
-  constexpr bool ISF = KIND >= 2;
-  const int lane = threadIdx.x & 31;
-  const uint64_t val = x.val;
-  const bool valid = x.valid;
-  int64_t ival = 0;
-  const uint32_t ff = ISF ? float_flags(val, KIND, LG, ival) : 0u;
-  const bool okv = valid && !(ff & 1u);       // contributes to ord / trunc (NaNs excluded)
-  const uint32_t nv = __popc(x.vmask);
-  uint32_t B = 0;
-  if (ISF) {
-    const uint32_t pB = valid ? ((ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) |
-                                 (((ff >> 3) & 1u) << 18) | (((ff >> 4) & 1u) << 24)) : 0u;
-    B = __reduce_add_sync(0xFFFFFFFFu, pB);
-  }
-  uint64_t rmin, rmax, omin, omax, tmin = ~0ull, tmax = 0;
-  if (LG < 3) {
-    // w <= 4 bytes: every key fits 32 bits -> one REDUX per min / max
-    const uint32_t r32 = (uint32_t)val;
-    rmin = __reduce_min_sync(0xFFFFFFFFu, valid ? r32 : 0xFFFFFFFFu);
-    rmax = __reduce_max_sync(0xFFFFFFFFu, valid ? r32 : 0u);
-    if (KIND == 0) {
-      omin = rmin; omax = rmax;
-    } else {
-      uint32_t k32;
-      if (KIND == 1) {                          // sext32(b) ^ 2^31: order-isomorphic to the 64-bit key
-        constexpr uint32_t sh = 32 - (8 << LG);
-        k32 = (uint32_t)(((int32_t)(r32 << sh)) >> sh) ^ 0x80000000u;
-      } else {
-        k32 = (uint32_t)ord_key(val, KIND, LG);
-      }
-      const unsigned okm = __ballot_sync(0xFFFFFFFFu, okv);
-      omin = __reduce_min_sync(0xFFFFFFFFu, okv ? k32 : 0xFFFFFFFFu);
-      omax = __reduce_max_sync(0xFFFFFFFFu, okv ? k32 : 0u);
-      if (ISF) {
-        const uint32_t t32 = (uint32_t)trunc_bits(val, KIND, LG, P.mant_bits);
-        tmin = __reduce_min_sync(0xFFFFFFFFu, okv ? t32 : 0xFFFFFFFFu);
-        tmax = __reduce_max_sync(0xFFFFFFFFu, okv ? t32 : 0u);
-      }
-      if (okm == 0) { omin = ~0ull; omax = 0; tmin = ~0ull; tmax = 0; }
-    }
-  } else {
-    rmin = redmin64(0xFFFFFFFFu, valid ? val : ~0ull);
-    rmax = redmax64(0xFFFFFFFFu, valid ? val : 0ull);
-    if (KIND == 0) {
-      omin = rmin; omax = rmax;
-    } else {
-      const uint64_t o = ord_key(val, KIND, LG);
-      omin = redmin64(0xFFFFFFFFu, okv ? o : ~0ull);
-      omax = redmax64(0xFFFFFFFFu, okv ? o : 0ull);
-      if (ISF) {
-        const uint64_t t = trunc_bits(val, KIND, LG, P.mant_bits);
-        tmin = redmin64(0xFFFFFFFFu, okv ? t : ~0ull);
-        tmax = redmax64(0xFFFFFFFFu, okv ? t : 0ull);
-      }
-    }
-  }
-  // the pre-snapshot gather is consumed only now
-  const bool eq = x.eqdef && x.pv == val;
-  const uint32_t pA = valid ? ((uint32_t)(val == 0) | ((uint32_t)eq << 6) | ((uint32_t)!x.eqdef << 12)) : 0u;
-  const uint32_t A = __reduce_add_sync(0xFFFFFFFFu, pA);
-  const bool lpart = x.inside && !x.st && eq;
-  if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, x.lw0, x.lbit);   // C3 loaded elements
-  if ((lane >> 4) == s) {
-    const int fl = lane & 15;
-    if (fl == 0) acc += nv;
-    else if (fl <= 3) acc += (A >> (6 * (fl - 1))) & 63u;
-    else if (fl <= 8) acc += (B >> (6 * (fl - 4))) & 63u;
-    else if (fl <= 14) {
-      const int m = (fl - 9) >> 1;
-      if (fl & 1) {
-        const uint64_t v = m == 0 ? rmin : m == 1 ? omin : tmin;
-        acc = v < acc ? v : acc;
-      } else {
-        const uint64_t v = m == 0 ? rmax : m == 1 ? omax : tmax;
-        acc = v > acc ? v : acc;
-      }
-    }
-  }
-  // C8: one line state for the window, merged into each key not yet FAIL
-  if (lfail_s != 3u) {
-    Facts f;
-    f.addr = x.addr;
-    f.pfail = ISF && (ff & 2u);
-    if (KIND == 0) f.y = (__int128)val;
-    else if (KIND == 1) {
-      constexpr uint32_t sh64 = 64u - (8u << LG);
-      f.y = (__int128)((int64_t)(val << sh64) >> sh64);
-    } else {
-      f.y = (__int128)ival;
-    }
-    LinePts g;
-    g.state = VE_LINE_EMPTY;
-    if (valid) group_line(x.vmask, f, g);
-    const int ps = x.pc0 < P.sp ? (int)x.pc0 : -1;
-    const int os = x.koi0 < P.so ? (int)(P.sp + x.koi0) : -1;
-    uint32_t lf = lfail_s;
-    if (lane == x.l0) {
-      if (!(lf & 1u) && wcache_merge(P, S, wc, x.pc0, ps, g) == VE_LINE_FAIL) lf |= 1u;
-      if (!(lf & 2u) && wcache_merge(P, S, wc, P.n_pcs + x.koi0, os, g) == VE_LINE_FAIL) lf |= 2u;
-    }
-    __syncwarp();
-    lfail_s = __shfl_sync(0xFFFFFFFFu, lf, x.l0);
-  }
-  // S8: exact histogram.  A load that reads an unchanged whole element carries the
-  // pre-snapshot value of that element, so it is counted per element (a coalesced
-  // counter increment) and mapped to its value at report time; every other record
-  // is inserted per distinct value.
-  const bool dl = dense_s != 0ull && eq && (uint32_t)LG == x.ew_lg && (x.off & ((1ull << LG) - 1)) == 0;
-  if (dl) atomicAdd(reinterpret_cast<uint32_t*>(dense_s) + (x.off >> LG), 1u);
-  const unsigned hmask = __ballot_sync(0xFFFFFFFFu, valid && !dl);
-  if (valid && !dl) {
-    const unsigned vg = (LG < 3) ? __match_any_sync(hmask, (uint32_t)val) : __match_any_sync(hmask, val);
-    if (lane == __ffs(vg) - 1) hist_insert(P, S, (x.pc0 << 16) | (x.koi0 & 0xFFFFu), val, __popc(vg));
-  }
+  fold_row(P, pc < P.sp ? (int)pc : -1, pc, f, field, v);
+  fold_row(P, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
 }
 
 struct Rec {
   uint64_t addr, val, pm;
 };
 
-// ---- per-warp TMA ring: cp.async.bulk of whole 768-byte windows into shared memory
+// ---- per-warp TMA ring: cp.async.bulk of 2-window stages into shared memory ----
+constexpr int STAGE_WIN = 2;
+constexpr int NSTAGE = RING / STAGE_WIN;
+constexpr uint32_t STAGE_BYTES = STAGE_WIN * WIN_BYTES;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
 }
 __device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-__device__ __forceinline__ void ring_issue(uint8_t* dst, const void* src, uint64_t* bar) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(WIN_BYTES) : "memory");
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(WIN_BYTES), "r"(smem_u32(bar))
+__device__ __forceinline__ void ring_issue(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
                : "memory");
 }
-__device__ __forceinline__ void ring_wait(uint64_t* bar, uint32_t phase) {
+__device__ __forceinline__ void ring_wait(uint32_t bar, uint32_t phase) {
   uint32_t ok = 0;
   while (!ok) {
     asm volatile(
         "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(ok)
-        : "r"(smem_u32(bar)), "r"(phase)
+        : "r"(bar), "r"(phase)
         : "memory");
+  }
+}
+// fire-and-forget global atomics (no compiler-generated warp aggregation around them)
+__device__ __forceinline__ void red_or(uint32_t* p, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_add(uint32_t* p, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// A warp's ring: NSTAGE stages of STAGE_WIN windows; lane l reads record l of a window.
+struct Ring {
+  const ve_record* src;   // next stage to issue
+  uint32_t left;          // windows not yet consumed
+  uint32_t iss;           // windows not yet issued
+  uint32_t rd;            // ve_smem offset of stage 0 of this warp + lane * 24
+  uint32_t bar;           // shared address of this warp's mbarrier 0
+  uint32_t dst;           // shared address of this warp's stage 0
+  uint32_t d, h, ph;      // current stage, window in it, phase parity
+};
+
+__device__ __forceinline__ void ring_issue_next(Ring& R) {
+  const uint32_t nw = R.iss < (uint32_t)STAGE_WIN ? R.iss : (uint32_t)STAGE_WIN;
+  ring_issue(R.dst + R.d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar + R.d * 8);
+  R.src += nw * 32;
+  R.iss -= nw;
+}
+
+// take the next window out of the ring (lane l gets record l); a stage is refilled
+// as soon as its last window has been read
+__device__ __forceinline__ void ring_next(Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm) {
+  if (R.h == 0) ring_wait(R.bar + R.d * 8, R.ph);
+  const uint32_t o = R.rd + R.d * STAGE_BYTES + R.h * WIN_BYTES;
+  addr = *reinterpret_cast<const unsigned long long*>(ve_smem + o);
+  val = *reinterpret_cast<const unsigned long long*>(ve_smem + o + 8);
+  pm = *reinterpret_cast<const unsigned long long*>(ve_smem + o + 16);
+  --R.left;
+  if (++R.h == (uint32_t)STAGE_WIN) {
+    R.h = 0;
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0 && R.iss) {
+      fence_proxy_async();   // our generic reads of the stage precede the next async write
+      ring_issue_next(R);
+    }
+    if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.ph ^= 1u; }
   }
 }
 
@@ -607,11 +552,403 @@ __device__ __forceinline__ Rec load_rec(const AnalyzeParams& P, uint64_t w, uint
   return r;
 }
 
-__global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
-  extern __shared__ __align__(16) uint8_t smem_raw[];
+// ---- slow path: any window (mixed keys, invalid / shared / unmapped / straddling
+// records, tails).  Returns this lane's (invalid | unmapped << 16) counts.
+__device__ __noinline__ uint32_t slow_window(const AnalyzeParams& P, WarpCache& wc, uint64_t addr,
+                                             uint64_t val, uint64_t pm, bool inrange) {
+  const Smem S = smem_of(P);
+  const int lane = threadIdx.x & 31;
+  const uint32_t pc = (uint32_t)pm, meta = (uint32_t)(pm >> 32);
+  // S1 decode + validate
+  const bool valid = inrange && rec_valid(addr, val, pc, meta, P.n_pcs);
+  const unsigned vmask = __ballot_sync(0xFFFFFFFFu, valid);
+  const uint32_t inv = (inrange && !valid) ? 1u : 0u;
+  if (vmask == 0) return inv;
+  const uint32_t lg = meta & 3u, kind = (meta >> 2) & 3u;
+  const bool st = meta_store(meta), sh = meta_shared(meta);
+
+  // S2 address -> object (binary search)
+  const bool need = valid && !sh;
+  const int oi = need ? find_object(P, addr) : -1;
+  const bool mapped = oi >= 0;
+  uint64_t ob = 0, oe = 0, bmoff = 0, opre = 0;
+  uint32_t oid = 0, ew_lg = 0;
+  if (mapped) {
+    ob = P.objc ? S.sob[oi] : P.o.base[oi];
+    oe = P.objc ? S.soe[oi] : P.o.end[oi];
+    bmoff = P.o.bmoff[oi];
+    opre = P.o.pre[oi];
+    oid = P.o.id[oi];
+    const uint32_t ew = P.o.ew[oi];
+    ew_lg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
+  }
+  const uint32_t unm = (need && !mapped) ? 1u : 0u;
+
+  // S3 snapshot gather + eq_pre
+  const uint64_t off = mapped ? addr - ob : 0ull;
+  const bool inside = mapped && addr + (1u << lg) <= oe;
+  const bool eqdef = inside && opre != 0ull;
+  const uint64_t pv = eqdef ? load_pre(opre + off, lg) : 0ull;
+  const uint32_t koi = sh ? P.n_obj : (mapped ? oid : KO_NONE);
+
+  // W element bitmap (C10) and L start-element bitmap (C3)
+  const uint64_t e0 = off >> ew_lg, e1 = (off + (1u << lg) - 1) >> ew_lg;
+  const uint64_t w0 = bmoff + (e0 >> 5), w1 = bmoff + (e1 >> 5);
+  {
+    const bool wpart = inside && st;
+    if (__any_sync(0xFFFFFFFFu, wpart)) {
+      uint32_t b0 = 0, b1 = 0;
+      if (wpart) {
+        for (uint64_t e = e0; e <= e1; ++e) {
+          if (bmoff + (e >> 5) == w0) b0 |= 1u << (e & 31);
+          else b1 |= 1u << (e & 31);
+        }
+      }
+      bitmap_or(P.t.W, wpart, w0, b0);
+      const bool spill = wpart && w1 != w0;
+      if (__any_sync(0xFFFFFFFFu, spill)) bitmap_or(P.t.W, spill, w1, b1);
+    }
+  }
+  const bool eq = eqdef && pv == val;
+  const bool lpart = inside && !st && eq;
+  if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, w0, 1u << (e0 & 31));
+
+  // per-key groups
+  Facts f;
+  f.addr = addr;
+  f.val = val;
+  f.tc = type_code(kind, lg);
+  f.isf = kind >= 2u;
+  int64_t ival = 0;
+  const uint32_t ff = f.isf ? float_flags(val, kind, lg, ival) : 0u;
+  f.nan = ff & 1u;
+  f.pfail = f.isf && (ff & 2u);
+  f.ordv = ord_key(val, kind, lg);
+  f.truncv = f.isf ? trunc_bits(val, kind, lg, P.mant_bits) : 0ull;
+  if (kind == 0u) f.y = (__int128)val;
+  else if (kind == 1u) {
+    const uint32_t sh64 = 64u - (8u << lg);
+    f.y = (__int128)((int64_t)(val << sh64) >> sh64);
+  } else f.y = (__int128)ival;
+  f.packA = (uint32_t)st | ((uint32_t)(val == 0) << 6) | ((uint32_t)(eq && !st) << 12) |
+            ((uint32_t)(eq && st) << 18) | ((uint32_t)(!eqdef) << 24);
+  f.packB = (ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) | (((ff >> 3) & 1u) << 18) |
+            (((ff >> 4) & 1u) << 24);
+  LinePts gp, go;
+  gp.state = go.state = VE_LINE_EMPTY;
+  bool leadp = false, leado = false;
+  const int pslot = pc < P.sp ? (int)pc : -1;
+  if (valid) {
+    const unsigned gm = __match_any_sync(vmask, pc);
+    apply_group(P, gm, pslot, pc, f, gp);
+    leadp = lane == __ffs(gm) - 1;
+  }
+  const bool opart = valid && koi != KO_NONE;
+  const unsigned omask = __ballot_sync(0xFFFFFFFFu, opart);
+  const int oslot = koi < P.so ? (int)(P.sp + koi) : -1;
+  if (opart) {
+    const unsigned gm = __match_any_sync(omask, koi);
+    apply_group(P, gm, oslot, P.n_pcs + koi, f, go);
+    leado = lane == __ffs(gm) - 1;
+  }
+  merge_lines(P, wc, leadp, pc, pslot, gp);
+  merge_lines(P, wc, leado, P.n_pcs + koi, oslot, go);
+  if (valid) {
+    const uint32_t tag = (pc << 16) | (koi & 0xFFFFu);
+    const unsigned tg = __match_any_sync(vmask, tag);
+    const unsigned vg = __match_any_sync(tg, val);
+    if (lane == __ffs(vg) - 1) hist_insert(P, tag, val, __popc(vg));
+  }
+  return inv | (unm << 16);
+}
+
+// ---- fast path ---------------------------------------------------------------
+// A fast window: all 32 lanes valid, one (pc, access type), global space, every
+// access aligned inside the warp's cached object whose element width equals the
+// access width.  Its type is a compile-time constant of run_fast below.
+
+// warp-uniform cache of the last object windows mapped to
+struct ObjCache {
+  uint64_t base, lim;      // offsets [0, lim] hold a whole element
+  uint64_t bmoff, pre;
+  int oi;
+  uint32_t id, fastlg;     // fastlg: log2 element width, 0xFF = no fast windows
+};
+
+__device__ __noinline__ ObjCache obj_refill(const AnalyzeParams& P, uint64_t a) {
+  const Smem S = smem_of(P);
+  ObjCache oc;
+  oc.oi = find_object(P, a);
+  oc.base = 0; oc.lim = 0; oc.bmoff = 0; oc.pre = 0; oc.id = 0; oc.fastlg = 0xFFu;
+  if (oc.oi >= 0) {
+    const int i = oc.oi;
+    oc.base = P.objc ? S.sob[i] : P.o.base[i];
+    const uint64_t e = P.objc ? S.soe[i] : P.o.end[i];
+    oc.bmoff = P.o.bmoff[i];
+    oc.pre = P.o.pre[i];
+    oc.id = P.o.id[i];
+    const uint32_t ew = P.o.ew[i];
+    const uint32_t lg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
+    // pre must be aligned for element-wide gathers
+    if (e - oc.base >= ew && (oc.pre & (ew - 1)) == 0) {
+      oc.lim = e - oc.base - ew;
+      oc.fastlg = lg;
+    }
+  }
+  return oc;
+}
+
+constexpr uint32_t VALID_KL = 0x2EFFu;  // valid (kind << 2 | log2 w) pairs of include/ve.h
+// a window whose lanes all carry (pc0, meta0): global space, valid type, pc in range
+__device__ __forceinline__ bool meta_fast(uint32_t meta0, uint32_t pc0, uint32_t n_pcs) {
+  return (meta0 >> 5) == 0u && ((VALID_KL >> (meta0 & 15u)) & 1u) && pc0 < n_pcs;
+}
+
+template <int LG>
+__device__ __forceinline__ uint64_t ld_pre(uint64_t p) {
+  if (LG == 0) return __ldg((const unsigned char*)p);
+  if (LG == 1) return __ldg((const unsigned short*)p);
+  if (LG == 2) return __ldg((const unsigned int*)p);
+  return __ldg((const unsigned long long*)p);
+}
+
+// C5 float flags of a <= 32-bit float (same definition as float_flags, 32-bit
+// arithmetic, branch-free)
+template <int KIND, int LG>
+__device__ __forceinline__ uint32_t fflags32(uint32_t b) {
+  constexpr int EB = KIND == 3 ? 8 : (LG == 1 ? 5 : 8);
+  constexpr int MB = KIND == 3 ? 7 : (LG == 1 ? 10 : 23);
+  constexpr int NB = 8 << LG;
+  constexpr uint32_t EMAX = (1u << EB) - 1u;
+  constexpr int BIAS = (1 << (EB - 1)) - 1;
+  const uint32_t E = (b >> MB) & EMAX, M = b & ((1u << MB) - 1u);
+  const bool sign = (b >> (NB - 1)) & 1u;
+  const uint32_t sig = E ? (M | (1u << MB)) : M;
+  const int ex = (E ? (int)E : 1) - BIAS - MB;
+  const int low = ex + __ffs((int)sig) - 1;
+  const int top = ex + 31 - __clz((int)sig);
+  uint32_t f = (top >= 63 || low < 0) ? 2u : 0u;
+  if (!(top <= 15 && low >= max(top - 10, -24))) f |= 4u;
+  if (!(top <= 127 && low >= max(top - 7, -133))) f |= 8u;
+  f = sig == 0u ? (sign ? 2u : 0u) : f;                 // +-0.0 (-0.0 is nonint)
+  return E == EMAX ? (M ? 15u : 2u) : f;                // NaN fails everything, +-Inf nonint only
+}
+
+// one window's OR into an element bitmap; lanes' words are usually one or two
+// consecutive words from lane 0's
+__device__ __forceinline__ void bitmap_or_win(uint32_t* bm, bool part, uint64_t word, uint32_t bit) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t w0 = shfl64(0xFFFFFFFFu, word, 0);
+  const uint64_t d = word - w0;
+  if (__all_sync(0xFFFFFFFFu, !part || d <= 1ull)) {
+    const uint32_t b0 = __reduce_or_sync(0xFFFFFFFFu, (part && d == 0ull) ? bit : 0u);
+    const uint32_t b1 = __reduce_or_sync(0xFFFFFFFFu, (part && d == 1ull) ? bit : 0u);
+    if (lane < 2 && (lane ? b1 : b0)) red_or(&bm[w0 + lane], lane ? b1 : b0);
+  } else {
+    bitmap_or(bm, part, word, bit);
+  }
+}
+
+// C8 for a fast window: one line state over its 32 points, merged into the keys
+// not yet FAIL; returns the updated FAIL bits
+__device__ __noinline__ uint32_t fast_line(const AnalyzeParams& P, WarpCache& wc, uint64_t addr,
+                                           uint64_t val, uint32_t meta0, uint32_t pc0, uint32_t koi0, uint32_t lf) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t lg = meta0 & 3u, kind = (meta0 >> 2) & 3u;
+  Facts f;
+  f.addr = addr;
+  int64_t ival = 0;
+  const uint32_t ff = kind >= 2u ? float_flags(val, kind, lg, ival) : 0u;
+  f.pfail = kind >= 2u && (ff & 2u);
+  if (kind == 0u) f.y = (__int128)val;
+  else if (kind == 1u) {
+    const uint32_t sh64 = 64u - (8u << lg);
+    f.y = (__int128)((int64_t)(val << sh64) >> sh64);
+  } else f.y = (__int128)ival;
+  LinePts g;
+  group_line(0xFFFFFFFFu, f, g);
+  const int ps = pc0 < P.sp ? (int)pc0 : -1;
+  const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
+  if (lane == 0) {
+    if (!(lf & 1u) && wcache_merge(P, wc, pc0, ps, g) == VE_LINE_FAIL) lf |= 1u;
+    if (!(lf & 2u) && wcache_merge(P, wc, P.n_pcs + koi0, os, g) == VE_LINE_FAIL) lf |= 2u;
+  }
+  __syncwarp();
+  return __shfl_sync(0xFFFFFFFFu, lf, 0);
+}
+
+// slot install on a miss: flush the victim, claim its line-FAIL bits and dense array
+__device__ __forceinline__ int slot_install(const AnalyzeParams& P, FastSlots& F, uint64_t& acc, uint64_t key,
+                                           uint32_t pc0, const ObjCache& oc, bool st) {
+  const int lane = threadIdx.x & 31;
+  const int s = (F.key[0] == ~0ull) ? 0 : (F.key[1] == ~0ull) ? 1 : (int)(F.mru ^ 1u);
+  const uint64_t victim = s ? F.key[1] : F.key[0];
+  if (victim != ~0ull) fast_flush(P, victim, s, acc);
+  if ((lane >> 4) == s) acc = fast_identity(lane & 15);
+  const uint32_t lf = slot_lfail(P, pc0, oc.id);
+  const unsigned long long dn = (P.dense_ok && !st) ? dense_lookup(P, oc.oi, pc0) : 0ull;
+  // constant indices only: the slot table stays in registers
+  if (s) { F.key[1] = key; F.lfail[1] = lf; F.dense[1] = dn; }
+  else { F.key[0] = key; F.lfail[0] = lf; F.dense[0] = dn; }
+  return s;
+}
+
+// Consume fast windows of access type (KIND, LG) from the ring, starting with the
+// current one (addr, val, pm; known fast).  Returns true when it stopped at a
+// window it has not consumed (left in addr, val, pm), false when the ring is empty.
+template <int KIND, int LG>
+__device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, const ObjCache& oc, FastSlots& F,
+                                         uint64_t& acc, Ring& R, uint32_t scr, uint64_t& addr, uint64_t& val,
+                                         uint64_t& pm) {
+  constexpr uint32_t W = 1u << LG;
+  constexpr uint32_t KL = ((uint32_t)KIND << 2) | (uint32_t)LG;
+  constexpr int MB = KIND == 3 ? 7 : (LG == 1 ? 10 : LG == 2 ? 23 : 52);
+  const unsigned FULL = 0xFFFFFFFFu;
+  const int lane = threadIdx.x & 31;
+  const uint64_t tmask = P.mant_bits >= (uint32_t)MB ? ~0ull : ~((1ull << (MB - P.mant_bits)) - 1ull);
+  const bool eqdef = oc.pre != 0ull;
+  // this lane's accumulator field (lane & 15) of its slot (lane >> 4): a sum taken
+  // from the packed REDUX results A / B, a constant per window, or a min / max
+  const int fl = lane & 15;
+  const bool f_sum = fl <= 8, f_min = fl >= 9 && (fl & 1), f_fromA = fl <= 3;
+  const uint32_t f_sh = (fl == 1 || fl == 4) ? 0u : (fl == 2 || fl == 5) ? 6u : fl == 6 ? 12u : fl == 7 ? 18u : 24u;
+  const uint32_t f_mask = (fl == 0 || fl == 3 || fl > 8) ? 0u : 63u;
+  const uint32_t f_add = fl == 0 ? 32u : (fl == 3 && !eqdef) ? 32u : 0u;
+  const uint32_t f_mm = scr + 8u * (uint32_t)(fl >= 9 && fl <= 14 ? fl - 9 : 0);
+  uint64_t pm0 = shfl64(FULL, pm, 0);
+  while (true) {
+    const uint32_t pc0 = (uint32_t)pm0, meta0 = (uint32_t)(pm0 >> 32);
+    const bool st = meta_store(meta0);
+    // select / install the register slot of (meta, object, pc)
+    const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
+    const int s = (F.key[0] == key) ? 0 : (F.key[1] == key) ? 1 : slot_install(P, F, acc, key, pc0, oc, st);
+    F.mru = (uint32_t)s;
+    const uint32_t lf_s = s ? F.lfail[1] : F.lfail[0];
+    const unsigned long long dn_s = s ? F.dense[1] : F.dense[0];
+
+    // S3: element, gather, written bitmap
+    const uint64_t off = addr - oc.base;
+    const uint64_t e = off >> LG;
+    const uint64_t pv = eqdef ? ld_pre<LG>(oc.pre + off) : 0ull;
+    const uint64_t word = oc.bmoff + (e >> 5);
+    const uint32_t bit = 1u << ((uint32_t)e & 31u);
+    if (st) bitmap_or_win(P.t.W, true, word, bit);
+
+    // C4-C7 reductions of the window
+    uint64_t rmin, rmax, omin, omax, tmin = ~0ull, tmax = 0ull;
+    uint32_t B = 0;
+    if constexpr (LG < 3) {
+      const uint32_t b = (uint32_t)val;
+      rmin = __reduce_min_sync(FULL, b);
+      rmax = __reduce_max_sync(FULL, b);
+      if constexpr (KIND == 0) {
+        omin = rmin; omax = rmax;
+      } else if constexpr (KIND == 1) {           // sext32(b) ^ 2^31: order-isomorphic to the 64-bit key
+        constexpr uint32_t sh = 32 - (8 << LG);
+        const uint32_t k = (uint32_t)(((int32_t)(b << sh)) >> sh) ^ 0x80000000u;
+        omin = __reduce_min_sync(FULL, k);
+        omax = __reduce_max_sync(FULL, k);
+      } else {
+        constexpr uint32_t SIGN = 1u << ((8 << LG) - 1);
+        constexpr uint32_t MASK = (uint32_t)((1ull << (8 << LG)) - 1ull);
+        const uint32_t ff = fflags32<KIND, LG>(b);
+        const bool okv = !(ff & 1u);              // NaNs excluded from ord / trunc
+        const uint32_t k = (b & SIGN) ? (~b & MASK) : (b | SIGN);
+        const uint32_t t = b & (uint32_t)tmask;
+        // a non-NaN key is never 0xFFFFFFFF, so that is the min identity in 32 bits
+        const uint32_t kmin = __reduce_min_sync(FULL, okv ? k : 0xFFFFFFFFu);
+        omax = __reduce_max_sync(FULL, okv ? k : 0u);
+        const uint32_t tm = __reduce_min_sync(FULL, okv ? t : 0xFFFFFFFFu);
+        tmax = __reduce_max_sync(FULL, okv ? t : 0u);
+        omin = kmin == 0xFFFFFFFFu ? ~0ull : (uint64_t)kmin;
+        tmin = tm == 0xFFFFFFFFu ? ~0ull : (uint64_t)tm;
+        B = __reduce_add_sync(FULL, (ff * 0x108421u) & 0x1041041u);   // flag bit i -> 6-bit field i
+      }
+    } else {
+      rmin = redmin64(FULL, val);
+      rmax = redmax64(FULL, val);
+      if constexpr (KIND == 0) {
+        omin = rmin; omax = rmax;
+      } else if constexpr (KIND == 1) {
+        const uint64_t k = val ^ (1ull << 63);
+        omin = redmin64(FULL, k);
+        omax = redmax64(FULL, k);
+      } else {
+        int64_t ival;
+        const uint32_t ff = float_flags(val, 2u, 3u, ival);
+        const bool okv = !(ff & 1u);
+        const uint64_t k = (val >> 63) ? ~val : (val | (1ull << 63));
+        const uint64_t t = val & tmask;
+        omin = redmin64(FULL, okv ? k : ~0ull);
+        omax = redmax64(FULL, okv ? k : 0ull);
+        tmin = redmin64(FULL, okv ? t : ~0ull);
+        tmax = redmax64(FULL, okv ? t : 0ull);
+        B = __reduce_add_sync(FULL, (ff * 0x108421u) & 0x1041041u);
+      }
+    }
+    // the pre-snapshot gather is consumed only now
+    const bool eq = eqdef && pv == val;
+    const uint32_t A = __reduce_add_sync(FULL, (uint32_t)(val == 0ull) | ((uint32_t)eq << 6));
+    // C3 loaded elements; loads counted per element below get their bits from the
+    // dense counters at report time
+    if (!st && dn_s == 0ull && __any_sync(FULL, eq)) bitmap_or_win(P.t.L, eq, word, bit);
+
+    // fold into slot s: sums from the packed REDUX results, min / max via scratch
+    if (lane == 0) {
+      *reinterpret_cast<ulonglong2*>(ve_smem + scr) = make_ulonglong2(rmin, rmax);
+      *reinterpret_cast<ulonglong2*>(ve_smem + scr + 16) = make_ulonglong2(omin, omax);
+      *reinterpret_cast<ulonglong2*>(ve_smem + scr + 32) = make_ulonglong2(tmin, tmax);
+    }
+    __syncwarp();
+    {
+      const uint64_t m = *reinterpret_cast<const unsigned long long*>(ve_smem + f_mm);
+      const uint32_t sv = (((f_fromA ? A : B) >> f_sh) & f_mask) + f_add;
+      const uint64_t nv = f_sum ? acc + sv : f_min ? (m < acc ? m : acc) : (m > acc ? m : acc);
+      if ((lane >> 4) == s && fl != 15) acc = nv;
+    }
+
+    // C8 line state, only while a key of the slot is not yet FAIL
+    if (lf_s != 3u) {
+      const uint32_t lf = fast_line(P, wc, addr, val, meta0, pc0, oc.id, lf_s);
+      if (s) F.lfail[1] = lf;
+      else F.lfail[0] = lf;
+    }
+
+    // S8: exact histogram.  A load that reads an unchanged element carries that
+    // element's pre value, so it is counted per element (mapped to its value at
+    // report time); every other record is inserted per distinct value.
+    const bool dl = dn_s != 0ull && eq;
+    if (dl) red_add(reinterpret_cast<uint32_t*>(dn_s) + e, 1u);
+    const unsigned hm = __ballot_sync(FULL, !dl);
+    if (hm) {
+      const uint32_t tag = (pc0 << 16) | (oc.id & 0xFFFFu);
+      const int l = __ffs(hm) - 1;
+      const uint64_t v0 = (LG < 3) ? (uint64_t)__shfl_sync(FULL, (uint32_t)val, l) : shfl64(FULL, val, l);
+      if (__all_sync(FULL, dl || val == v0)) {
+        if (lane == l) hist_insert(P, tag, val, __popc(hm));
+      } else if (!dl) {
+        const unsigned vg = (LG < 3) ? __match_any_sync(hm, (uint32_t)val) : __match_any_sync(hm, val);
+        if (lane == __ffs(vg) - 1) hist_insert(P, tag, val, __popc(vg));
+      }
+    }
+
+    // next window: continue while it is fast with the same access type
+    if (R.left == 0) return false;
+    ring_next(R, addr, val, pm);
+    pm0 = shfl64(FULL, pm, 0);
+    const uint64_t o2 = addr - oc.base;
+    bool ok = pm == pm0 && o2 <= oc.lim && (o2 & (W - 1)) == 0;
+    if constexpr (LG < 3) ok = ok && (val >> (8 * W)) == 0ull;
+    const uint32_t m2 = (uint32_t)(pm0 >> 32);
+    if (!__all_sync(FULL, ok) || (m2 & 15u) != KL || !meta_fast(m2, (uint32_t)pm0, P.n_pcs)) return true;
+  }
+}
+
+__global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant__ AnalyzeParams P) {
   const uint32_t nsk = P.sp + P.so;
-  Smem S = carve(smem_raw, nsk, P.hs, P.objc);
+  const Smem S = smem_of(P);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const unsigned FULL = 0xFFFFFFFFu;
 
   for (uint32_t i = tid; i < nsk * NSUM; i += blockDim.x) S.ssum[i] = 0;
   for (uint32_t i = tid; i < nsk * NMM; i += blockDim.x) { S.smin[i] = ~0ull; S.smax[i] = 0; }
@@ -622,7 +959,9 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   for (uint32_t i = tid; i < P.objc; i += blockDim.x) { S.sob[i] = P.o.base[i]; S.soe[i] = P.o.end[i]; }
   if (tid < 4) S.sctr[tid] = 0;
   __shared__ WarpCache s_wc[K1_WARPS];
+  __shared__ __align__(16) uint64_t s_scr[K1_WARPS][8];
   WarpCache& wc = s_wc[warp];
+  const uint32_t scr = (uint32_t)((const uint8_t*)s_scr[warp] - ve_smem);   // ve_smem offset
   if (lane < WC) wc.key1[lane] = 0;
   if (lane == 0) wc.next = 0;
 
@@ -631,248 +970,93 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + warp;
   const uint64_t wbeg = gw * nwin / tw, wend = (gw + 1) * nwin / tw;
   const uint64_t nfull = P.n / 32;
-  const uint64_t rend = P.ring ? (wend < nfull ? wend : nfull) : wbeg;   // ring covers [wbeg, rend)
-  uint8_t (*s_ring)[RING][WIN_BYTES] = reinterpret_cast<uint8_t (*)[RING][WIN_BYTES]>(S.ring);
-  uint64_t (*s_bar)[RING] = reinterpret_cast<uint64_t (*)[RING]>(S.bars);
-  if (lane == 0) {
-    for (int d = 0; d < RING; ++d) mbar_init(&s_bar[warp][d], 1);
+  uint64_t rend = P.ring ? (wend < nfull ? wend : nfull) : wbeg;   // the ring covers [wbeg, rend)
+  if (rend < wbeg) rend = wbeg;
+  Ring R;
+  R.src = P.recs + wbeg * 32;
+  R.left = R.iss = (uint32_t)(rend - wbeg);
+  R.rd = P.o_ring + (uint32_t)warp * RING * WIN_BYTES + (uint32_t)lane * 24u;
+  R.dst = smem_u32(ve_smem + P.o_ring + (uint32_t)warp * RING * WIN_BYTES);
+  R.bar = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
+  R.d = R.h = R.ph = 0;
+  if (lane == 0) {   // only lane 0 issues: its src / iss are the ones that matter
+    for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar + d * 8, 1);
     fence_mbar_init();
-    for (int d = 0; d < RING && wbeg + d < rend; ++d)
-      ring_issue(s_ring[warp][d], P.recs + (wbeg + d) * 32, &s_bar[warp][d]);
+    for (int d = 0; d < NSTAGE && R.iss; ++d) {
+      R.d = d;
+      ring_issue_next(R);
+    }
+    R.d = 0;
   }
   __syncthreads();
   ObjCache oc;
-  oc.oi = -1; oc.base = oc.end = oc.bmoff = oc.pre = 0; oc.id = 0; oc.ewlg = 0;
-  uint32_t n_invalid = 0, n_unmapped = 0;
+  oc.base = 0; oc.lim = 0; oc.bmoff = 0; oc.pre = 0; oc.oi = -1; oc.id = 0; oc.fastlg = 0xFFu;
+  uint32_t n_inv = 0, n_unm = 0;   // this lane's invalid / unmapped records (slow windows)
   FastSlots F;
-  F.used = 0;
   F.mru = 0;
+  F.key[0] = F.key[1] = ~0ull;
+  F.lfail[0] = F.lfail[1] = 3u;
+  F.dense[0] = F.dense[1] = 0ull;
   uint64_t acc = 0;
 
-  for (uint64_t w = wbeg; w < wend; ++w) {
-    Rec cur;
-    if (w < rend) {
-      const uint64_t i = w - wbeg;
-      const int d = (int)(i % RING);
-      ring_wait(&s_bar[warp][d], (uint32_t)((i / RING) & 1));
-      const unsigned long long* q = reinterpret_cast<const unsigned long long*>(s_ring[warp][d] + lane * 24);
-      cur.addr = q[0];
-      cur.val = q[1];
-      cur.pm = q[2];
-      __syncwarp();
-      if (lane == 0 && w + RING < rend) {
-        fence_proxy_async();   // our generic reads of the stage precede the next async write
-        ring_issue(s_ring[warp][d], P.recs + (w + RING) * 32, &s_bar[warp][d]);
+  uint64_t addr = 0, val = 0, pm = 0;
+  bool have = false;
+  while (have || R.left) {
+    if (!have) ring_next(R, addr, val, pm);
+    have = false;
+    const uint64_t pm0 = shfl64(FULL, pm, 0);
+    const uint32_t meta0 = (uint32_t)(pm0 >> 32), pc0 = (uint32_t)pm0;
+    bool fast = false;
+    if (__all_sync(FULL, pm == pm0) && meta_fast(meta0, pc0, P.n_pcs)) {
+      const uint32_t lg0 = meta0 & 3u;
+      const uint64_t wm = (1ull << lg0) - 1ull;
+      const bool vok = lg0 == 3u || (val >> (8u << lg0)) == 0ull;
+      uint64_t off = addr - oc.base;
+      if (!__all_sync(FULL, off <= oc.lim && (off & wm) == 0ull) || lg0 != oc.fastlg) {
+        oc = obj_refill(P, shfl64(FULL, addr, 0));
+        off = addr - oc.base;
       }
-    } else {
-      cur = load_rec(P, w, wend, lane);
+      fast = __all_sync(FULL, vok && off <= oc.lim && (off & wm) == 0ull) && lg0 == oc.fastlg;
     }
-    const uint64_t addr = cur.addr, val = cur.val;
-    const uint32_t pc = (uint32_t)cur.pm, meta = (uint32_t)(cur.pm >> 32);
-    const bool full = (w + 1) * 32 <= P.n;
-    const bool inrange = full || (w * 32 + lane < P.n);
-
-    // S1 decode + validate
-    const bool valid = inrange && rec_valid(addr, val, pc, meta, P.n_pcs);
-    const unsigned vmask = __ballot_sync(0xFFFFFFFFu, valid);
-    if (lane == 0) n_invalid += (full ? 32u : (uint32_t)min((uint64_t)32, P.n - w * 32)) - (uint32_t)__popc(vmask);
-    if (vmask == 0) continue;
-    const uint32_t lg = meta & 3u, kind = (meta >> 2) & 3u;
-    const bool st = meta_store(meta), sh = meta_shared(meta);
-
-    // S2 address -> object: warp-uniform cached object, binary search only on a miss
-    const bool need = valid && !sh;
-    const bool hit = need && oc.oi >= 0 && addr >= oc.base && addr < oc.end;
-    int oi = hit ? oc.oi : -1;
-    uint64_t ob = oc.base, oe = oc.end, obm = oc.bmoff, opre = oc.pre;
-    uint32_t oid = oc.id, oewlg = oc.ewlg;
-    const unsigned missm = __ballot_sync(0xFFFFFFFFu, need && !hit);
-    if (missm) {
-      if (need && !hit) {
-        oi = find_object(P, S, addr);
-        if (oi >= 0) {
-          ob = P.objc ? S.sob[oi] : P.o.base[oi];
-          oe = P.objc ? S.soe[oi] : P.o.end[oi];
-          obm = P.o.bmoff[oi];
-          opre = P.o.pre[oi];
-          oid = P.o.id[oi];
-          const uint32_t ew = P.o.ew[oi];
-          oewlg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
-        }
-      }
-      const unsigned mm = __ballot_sync(0xFFFFFFFFu, need && !hit && oi >= 0);
-      if (mm) {                                    // adopt the first newly found object
-        const int src = __ffs(mm) - 1;
-        oc.oi = __shfl_sync(0xFFFFFFFFu, oi, src);
-        oc.base = __shfl_sync(0xFFFFFFFFu, ob, src);
-        oc.end = __shfl_sync(0xFFFFFFFFu, oe, src);
-        oc.bmoff = __shfl_sync(0xFFFFFFFFu, obm, src);
-        oc.pre = __shfl_sync(0xFFFFFFFFu, opre, src);
-        oc.id = __shfl_sync(0xFFFFFFFFu, oid, src);
-        oc.ewlg = __shfl_sync(0xFFFFFFFFu, oewlg, src);
-      }
-      const unsigned um = __ballot_sync(0xFFFFFFFFu, need && oi < 0);
-      if (lane == 0) n_unmapped += __popc(um);
-    }
-    const bool mapped = oi >= 0;
-
-    // S3 snapshot gather + eq_pre
-    const uint32_t ew_lg = mapped ? oewlg : 0u;
-    const uint64_t off = mapped ? addr - ob : 0ull;
-    const uint64_t bmoff = mapped ? obm : 0ull;
-    const bool inside = mapped && addr + (1u << lg) <= oe;
-    const bool eqdef = inside && opre != 0ull;
-    // issue the pre-snapshot gather now, consume it as late as possible (latency hiding)
-    const uint64_t pv = eqdef ? load_pre(opre + off, lg) : 0ull;
-    const uint32_t koi = sh ? P.n_obj : (mapped ? oid : KO_NONE);
-    const uint64_t lw0 = bmoff + ((off >> ew_lg) >> 5);        // L bitmap word / bit of the first element
-    const uint32_t lbit = 1u << ((off >> ew_lg) & 31);
-
-    // W element bitmap (C10); L is set once eq_pre is known
-    {
-      const bool wpart = inside && st;
-      const uint64_t e0 = off >> ew_lg, e1 = (off + (1u << lg) - 1) >> ew_lg;
-      const uint64_t w0 = bmoff + (e0 >> 5), w1 = bmoff + (e1 >> 5);
-      const unsigned wany = __ballot_sync(0xFFFFFFFFu, wpart);
-      if (wany) {
-        uint32_t b0 = 0, b1 = 0;
-        if (wpart) {
-          for (uint64_t e = e0; e <= e1; ++e) {
-            if (bmoff + (e >> 5) == w0) b0 |= 1u << (e & 31);
-            else b1 |= 1u << (e & 31);
-          }
-        }
-        bitmap_or(P.t.W, wpart, w0, b0);
-        const bool spill = wpart && w1 != w0;
-        if (__any_sync(0xFFFFFFFFu, spill)) bitmap_or(P.t.W, spill, w1, b1);
-      }
-    }
-
-    // uniform window? (pc, access type and object shared by every valid lane)
-    const int l0 = __ffs(vmask) - 1;
-    const uint32_t pc0 = __shfl_sync(0xFFFFFFFFu, pc, l0);
-    const uint32_t meta0 = __shfl_sync(0xFFFFFFFFu, meta, l0);
-    const uint32_t koi0 = __shfl_sync(0xFFFFFFFFu, koi, l0);
-    const bool uniform = __all_sync(0xFFFFFFFFu, !valid || (pc == pc0 && meta == meta0 && koi == koi0));
-
-    if (uniform) {
-      // ---------------- fast path ----------------
-      // select / install the register slot for (pc, object key, access type)
-      int s;
-      if ((F.used & 1u) && F.pc[0] == pc0 && F.koi[0] == koi0 && F.meta[0] == meta0) s = 0;
-      else if ((F.used & 2u) && F.pc[1] == pc0 && F.koi[1] == koi0 && F.meta[1] == meta0) s = 1;
-      else {
-        s = !(F.used & 1u) ? 0 : !(F.used & 2u) ? 1 : (int)(F.mru ^ 1u);
-        if (F.used & (1u << s)) {
-          if (s) fast_flush(P, S, F.pc[1], F.koi[1], F.meta[1], 1, acc);
-          else fast_flush(P, S, F.pc[0], F.koi[0], F.meta[0], 0, acc);
-        }
-        F.used |= 1u << s;
-        // constant indices only: the slot table stays in registers
-        if (s) { F.pc[1] = pc0; F.koi[1] = koi0; F.meta[1] = meta0; }
-        else { F.pc[0] = pc0; F.koi[0] = koi0; F.meta[0] = meta0; }
-        if ((lane >> 4) == s) acc = fast_identity(lane & 15);
-        // line states this warp can skip (already FAIL in the CTA state)
-        const int ps = pc0 < P.sp ? (int)pc0 : -1;
-        uint32_t lf = (line_target(P, S, ps, pc0)->state == VE_LINE_FAIL) ? 1u : 0u;
-        if (koi0 == KO_NONE) lf |= 2u;
-        else {
-          const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
-          if (line_target(P, S, os, P.n_pcs + koi0)->state == VE_LINE_FAIL) lf |= 2u;
-        }
-        lf = __shfl_sync(0xFFFFFFFFu, lf, 0);
-        // dense per-element counting for loads of a real object that read the pre value
-        const int oi0 = __shfl_sync(0xFFFFFFFFu, oi, l0);
-        const unsigned long long dn =
-            (P.dense_ok && oi0 >= 0 && !meta_store(meta0)) ? dense_lookup(P, oi0, pc0) : 0ull;
-        if (s) { F.lfail[1] = lf; F.dense[1] = dn; }
-        else { F.lfail[0] = lf; F.dense[0] = dn; }
-      }
-      F.mru = (uint32_t)s;
-      uint32_t lf_s = s ? F.lfail[1] : F.lfail[0];
-      const unsigned long long dn_s = s ? F.dense[1] : F.dense[0];
-      WinCtx x;
-      x.addr = addr; x.val = val; x.off = off; x.ew_lg = ew_lg;
-      x.valid = valid; x.eqdef = eqdef; x.inside = inside; x.st = st;
-      x.pv = pv; x.lw0 = lw0; x.lbit = lbit;
-      x.vmask = vmask; x.l0 = l0; x.pc0 = pc0; x.koi0 = koi0;
+    if (fast) {
       // specialised on the window's access type (compile-time width / kind)
       switch (meta0 & 15u) {
-        case 0: fast_window<0, 0>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 1: fast_window<0, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 2: fast_window<0, 2>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 3: fast_window<0, 3>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 4: fast_window<1, 0>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 5: fast_window<1, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 6: fast_window<1, 2>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 7: fast_window<1, 3>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 9: fast_window<2, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 10: fast_window<2, 2>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        case 11: fast_window<2, 3>(P, S, lf_s, dn_s, s, acc, wc, x); break;
-        default: fast_window<3, 1>(P, S, lf_s, dn_s, s, acc, wc, x); break;   // 13: bfloat16
+        case 0: have = run_fast<0, 0>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 1: have = run_fast<0, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 2: have = run_fast<0, 2>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 3: have = run_fast<0, 3>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 4: have = run_fast<1, 0>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 5: have = run_fast<1, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 6: have = run_fast<1, 2>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 7: have = run_fast<1, 3>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 9: have = run_fast<2, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 10: have = run_fast<2, 2>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        case 11: have = run_fast<2, 3>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
+        default: have = run_fast<3, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;   // 13: bfloat16
       }
-      if (s) F.lfail[1] = lf_s;
-      else F.lfail[0] = lf_s;
     } else {
-      // ---------------- slow path: per-key groups ----------------
-      const bool eq = eqdef && pv == val;
-      const bool lpart = inside && !st && eq;
-      if (__any_sync(0xFFFFFFFFu, lpart)) bitmap_or(P.t.L, lpart, lw0, lbit);   // C3 loaded elements
-      Facts f;
-      f.addr = addr;
-      f.val = val;
-      f.tc = type_code(kind, lg);
-      f.isf = kind >= 2u;
-      int64_t ival = 0;
-      const uint32_t ff = f.isf ? float_flags(val, kind, lg, ival) : 0u;
-      f.nan = ff & 1u;
-      f.pfail = f.isf && (ff & 2u);
-      f.ordv = ord_key(val, kind, lg);
-      f.truncv = f.isf ? trunc_bits(val, kind, lg, P.mant_bits) : 0ull;
-      if (kind == 0u) f.y = (__int128)val;
-      else if (kind == 1u) {
-        const uint32_t sh64 = 64u - (8u << lg);
-        f.y = (__int128)((int64_t)(val << sh64) >> sh64);
-      } else f.y = (__int128)ival;
-      f.packA = (uint32_t)st | ((uint32_t)(val == 0) << 6) | ((uint32_t)(eq && !st) << 12) |
-                ((uint32_t)(eq && st) << 18) | ((uint32_t)(!eqdef) << 24);
-      f.packB = (ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) | (((ff >> 3) & 1u) << 18) |
-                (((ff >> 4) & 1u) << 24);
-      LinePts gp, go;
-      gp.state = go.state = VE_LINE_EMPTY;
-      bool leadp = false, leado = false;
-      const int pslot = pc < P.sp ? (int)pc : -1;
-      if (valid) {
-        const unsigned gm = __match_any_sync(vmask, pc);
-        apply_group(P, S, gm, pslot, pc, f, gp);
-        leadp = lane == __ffs(gm) - 1;
-      }
-      const bool opart = valid && koi != KO_NONE;
-      const unsigned omask = __ballot_sync(0xFFFFFFFFu, opart);
-      const int oslot = koi < P.so ? (int)(P.sp + koi) : -1;
-      if (opart) {
-        const unsigned gm = __match_any_sync(omask, koi);
-        apply_group(P, S, gm, oslot, P.n_pcs + koi, f, go);
-        leado = lane == __ffs(gm) - 1;
-      }
-      merge_lines(P, S, wc, leadp, pc, pslot, gp);
-      merge_lines(P, S, wc, leado, P.n_pcs + koi, oslot, go);
-      if (valid) {
-        const uint32_t tag = (pc << 16) | (koi & 0xFFFFu);
-        const unsigned tg = __match_any_sync(vmask, tag);
-        const unsigned vg = __match_any_sync(tg, val);
-        if (lane == __ffs(vg) - 1) hist_insert(P, S, tag, val, __popc(vg));
-      }
+      const uint32_t cnt = slow_window(P, wc, addr, val, pm, true);
+      n_inv += cnt & 0xFFFFu;
+      n_unm += cnt >> 16;
     }
+  }
+  // windows outside the ring (partial tail, or records not 16-byte aligned)
+  for (uint64_t w = rend; w < wend; ++w) {
+    const Rec cur = load_rec(P, w, wend, lane);
+    const uint32_t cnt = slow_window(P, wc, cur.addr, cur.val, cur.pm, w * 32 + lane < P.n);
+    n_inv += cnt & 0xFFFFu;
+    n_unm += cnt >> 16;
   }
 
   // fold the warp's register slots and line cache, then the CTA's shared state
-  if (F.used & 1u) fast_flush(P, S, F.pc[0], F.koi[0], F.meta[0], 0, acc);
-  if (F.used & 2u) fast_flush(P, S, F.pc[1], F.koi[1], F.meta[1], 1, acc);
+  if (F.key[0] != ~0ull) fast_flush(P, F.key[0], 0, acc);
+  if (F.key[1] != ~0ull) fast_flush(P, F.key[1], 1, acc);
+  n_inv = __reduce_add_sync(FULL, n_inv);
+  n_unm = __reduce_add_sync(FULL, n_unm);
   if (lane == 0) {
-    if (n_invalid) atomicAdd(&S.sctr[0], n_invalid);
-    if (n_unmapped) atomicAdd(&S.sctr[1], n_unmapped);
-    wcache_flush(P, S, wc);
+    if (n_inv) atomicAdd(&S.sctr[0], n_inv);
+    if (n_unm) atomicAdd(&S.sctr[1], n_unm);
+    wcache_flush(P, wc);
   }
   __syncthreads();
 
@@ -906,6 +1090,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(AnalyzeParams P) {
   }
 }
 
+
 ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
   AnalyzeParams P;
   P.recs = d;
@@ -935,6 +1120,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   uint32_t hs = 8192;
   while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > budget) hs >>= 1;
   P.hs = hs;
+  carve_offsets(P, sp + so);
   const size_t sb = smem_bytes(sp + so, hs, P.objc);
   cudaError_t e = cudaFuncSetAttribute(k_analyze, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
   if (e != cudaSuccess) return cuda_fail(c, e, "cudaFuncSetAttribute(k_analyze)");

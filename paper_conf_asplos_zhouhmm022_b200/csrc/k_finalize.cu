@@ -562,7 +562,7 @@ constexpr int DF_SLOTS = 1024;
 constexpr uint64_t DF_CHUNK = 16384;
 
 __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
-                                                           uint32_t ew, uint32_t tag, DevTables t) {
+                                                           uint32_t ew, uint32_t tag, uint64_t bmoff, DevTables t) {
   __shared__ unsigned long long sbits[DF_SLOTS], scnt[DF_SLOTS];
   for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS) { sbits[i] = ~0ull; scnt[i] = 0; }
   __syncthreads();
@@ -585,6 +585,9 @@ __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint6
       }
     }
     const unsigned km = __ballot_sync(0xFFFFFFFFu, k != 0);
+    // C3: a counted load started at element e (K1 leaves these L bits to us); the
+    // warp's 32 elements are one aligned bitmap word
+    if (lane == 0 && km) atomicOr(&t.L[bmoff + ((base + threadIdx.x) >> 5)], km);
     if (k) {
       const unsigned g = __match_any_sync(km, bits);
       const unsigned long long sum = __reduce_add_sync(g, k);   // < 32 * 2^32? counts are < 2^32 each
@@ -625,7 +628,7 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
       const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
       count_launch();
       k_dense_flush<<<(unsigned)blocks, DF_THREADS, 0, s>>>((uint32_t*)c->dense_pool + c->dense_off_h[DENSE_PER_OBJ * i + j],
-                                                    o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, c->t);
+                                                    o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, o.bmoff, c->t);
       any = true;
     }
   }
