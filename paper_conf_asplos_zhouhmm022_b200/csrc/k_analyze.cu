@@ -22,6 +22,8 @@
 // same bits (C12).
 #include <cuda_runtime.h>
 
+#include <type_traits>
+
 #include "ve_internal.cuh"
 
 namespace ve {
@@ -372,18 +374,26 @@ __device__ __forceinline__ void bitmap_or(uint32_t* bm, bool part, uint64_t word
   }
 }
 
-// ---- fast path: lane-distributed register accumulators -----------------------
-// Two key slots per warp; lane l holds field (l & 15) of slot (l >> 4):
-//  0 n   1 n_zero   2 n_eq_pre   3 n_nosnap   4 nan   5 nonint   6 not_f16   7 not_bf16
-//  8 not_f32   9 raw_min 10 raw_max 11 ord_min 12 ord_max 13 trunc_min 14 trunc_max
-// For w <= 4 the ord fields of signed types hold sext32(b)^2^31 (order-isomorphic),
-// converted to the 64-bit key at flush.  A slot is keyed by (meta, object id, pc).
-struct FastSlots {
-  uint64_t key[2];              // meta << 32 | object id << 16 | pc; ~0 = unused
-  uint32_t mru;
-  uint32_t lfail[2];            // bit0: PC key line FAIL, bit1: object key line FAIL (known to this warp)
-  unsigned long long dense[2];  // per-element counters of this (pc, object), or 0
+// ---- fast path key slots ------------------------------------------------------
+// A fast window's statistics are warp-uniform REDUX results, accumulated into the
+// totals of its key slot (pc, object, access type).  The active slot lives in
+// registers inside run_fast; each warp keeps NSLOT slots in a private shared-memory
+// cache and folds a slot into the PC-key and object-key rows only on eviction and
+// at exit.  For w <= 4 the min / max totals are 32-bit forms: ord of signed types
+// is sext32(b)^2^31 (order-isomorphic to the 64-bit key), and 0xFFFFFFFF is the min
+// identity of ord / trunc of floats (no non-NaN key has that value).
+constexpr int NSLOT = 4;
+struct __align__(16) SlotE {
+  uint64_t key;                 // meta << 32 | object id << 16 | pc; ~0 = free
+  unsigned long long dense;     // per-element counters of (pc, object), or 0
+  uint64_t mm[6];               // raw min, raw max, ord min, ord max, trunc min, trunc max
+  uint32_t nwin;                // windows (32 records each)
+  uint32_t lfail;               // bit0: PC key line FAIL, bit1: object key line FAIL (known to this warp)
+  uint32_t nosnap;              // the object has no pre snapshot
+  uint32_t pad;
+  uint32_t sum[8];              // zero, eq_pre, nan, nonint, not_f16, not_bf16, not_f32, -
 };
+static_assert(sizeof(SlotE) == 112, "SlotE layout");
 
 // claim (or find) a dense counter array of sorted object oi for pc (lane 0), broadcast
 __device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t pc) {
@@ -416,12 +426,9 @@ __device__ __noinline__ uint32_t slot_lfail(const AnalyzeParams& P, uint32_t pc,
   return __shfl_sync(0xFFFFFFFFu, lf, 0);
 }
 
-__device__ __forceinline__ uint64_t fast_identity(int f) {
-  return (f >= 9 && (f & 1)) ? ~0ull : 0ull;
-}
-
-__device__ __forceinline__ void fold_row(const AnalyzeParams& P, int slot, uint32_t key, int f,
-                                         uint32_t field, uint64_t v) {
+// field f of a key row: f <= 8 or 15 a sum, f = 9..14 min (odd) / max (even)
+__device__ __forceinline__ void fold_row(const AnalyzeParams& P, int slot, uint32_t key, int f, uint32_t field,
+                                         uint64_t v) {
   const Smem S = smem_of(P);
   if (f <= 8 || f == 15) {
     if (slot >= 0) atomicAdd(&S.ssum[slot * NSUM + field], (uint32_t)v);
@@ -433,34 +440,78 @@ __device__ __forceinline__ void fold_row(const AnalyzeParams& P, int slot, uint3
   }
 }
 
-// fold slot s's accumulators into the PC-key row and the object-key row (lanes of half s)
-__device__ __noinline__ void fast_flush(const AnalyzeParams& P, uint64_t skey, int s, uint64_t acc) {
-  const Smem S = smem_of(P);
-  const int lane = threadIdx.x & 31;
-  const uint64_t nrec = __shfl_sync(0xFFFFFFFFu, acc, s * 16);   // field 0 of slot s
-  if ((lane >> 4) != s) return;
-  const uint32_t pc = (uint32_t)skey & 0xFFFFu, koi = (uint32_t)(skey >> 16) & 0xFFFFu;
-  const uint32_t meta = (uint32_t)(skey >> 32);
-  const int f = lane & 15;
-  const uint32_t lg = meta & 3u, kind = (meta >> 2) & 3u;
+// fold a slot into its PC-key row (lanes 0-15) and object-key row (lanes 16-31);
+// lane field f: 0 n  1 zero  2 eq_pre  3 nosnap  4-8 float flags  9-14 min / max  15 n_type
+__device__ __noinline__ void slot_flush(const AnalyzeParams& P, const SlotE* e) {
+  const int lane = threadIdx.x & 31, f = lane & 15;
+  const uint64_t key = e->key;
+  const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
+  const uint32_t meta = (uint32_t)(key >> 32), lg = meta & 3u, kind = (meta >> 2) & 3u;
   const bool st = meta_store(meta);
-  uint64_t v = (f == 15) ? nrec : acc;
-  if (v == fast_identity(f) && f != 15) return;
-  if (f == 15 && v == 0) return;
-  uint32_t field;
-  if (f == 0) field = st ? F_ST : F_LD;
-  else if (f == 1) field = F_ZERO;
-  else if (f == 2) field = st ? F_STEQ : F_LDEQ;
-  else if (f == 3) field = F_NOSNAP;
-  else if (f <= 8) field = F_NAN + (uint32_t)(f - 4);
-  else if (f == 15) field = F_TYPE0 + type_code(kind, lg);
-  else field = 0;
-  if ((f == 11 || f == 12) && kind == 1u && lg < 3u) {
-    const int32_t sv = (int32_t)((uint32_t)v ^ 0x80000000u);
-    v = (uint64_t)(int64_t)sv ^ (1ull << 63);
+  const uint64_t n = (uint64_t)e->nwin * 32u;
+  uint64_t v = 0;
+  uint32_t field = 0;
+  bool skip;
+  if (f == 0) { v = n; field = st ? F_ST : F_LD; }
+  else if (f == 1) { v = e->sum[0]; field = F_ZERO; }
+  else if (f == 2) { v = e->sum[1]; field = st ? F_STEQ : F_LDEQ; }
+  else if (f == 3) { v = e->nosnap ? n : 0; field = F_NOSNAP; }
+  else if (f <= 8) { v = e->sum[f - 2]; field = F_NAN + (uint32_t)(f - 4); }
+  else if (f == 15) { v = n; field = F_TYPE0 + type_code(kind, lg); }
+  else v = e->mm[f - 9];
+  if (f <= 8 || f == 15) {
+    skip = v == 0;
+  } else {
+    const int m = f - 9;                       // 0 raw min 1 raw max 2 ord min 3 ord max 4 trunc min 5 trunc max
+    if (m >= 4 && kind < 2u) v = (m & 1) ? 0ull : ~0ull;        // no trunc for integers
+    else if (lg < 3u) {
+      if (kind == 1u && (m == 2 || m == 3)) {  // sext32(b)^2^31 -> 64-bit ord key
+        const int32_t sv = (int32_t)((uint32_t)v ^ 0x80000000u);
+        v = (uint64_t)(int64_t)sv ^ (1ull << 63);
+      } else if (kind >= 2u && (m == 2 || m == 4) && v == 0xFFFFFFFFull) {
+        v = ~0ull;                             // 32-bit min identity (all NaN)
+      }
+    }
+    skip = (m & 1) ? v == 0ull : v == ~0ull;
   }
-  fold_row(P, pc < P.sp ? (int)pc : -1, pc, f, field, v);
-  fold_row(P, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
+  if (skip) return;
+  if (lane < 16) fold_row(P, pc < P.sp ? (int)pc : -1, pc, f, field, v);
+  else fold_row(P, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
+}
+
+// index of key's slot in the warp's cache; a miss evicts round-robin (folding the
+// victim) and initialises the slot for key's access type
+__device__ __noinline__ int slot_acquire(const AnalyzeParams& P, SlotE* slots, uint32_t* next, uint64_t key,
+                                         int oi, bool nosnap) {
+  for (int i = 0; i < NSLOT; ++i)
+    if (slots[i].key == key) return i;
+  int v = -1;
+  for (int i = 0; i < NSLOT; ++i)
+    if (slots[i].key == ~0ull) { v = i; break; }
+  if (v < 0) {
+    v = (int)(*next % NSLOT);
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) *next = *next + 1;
+    slot_flush(P, &slots[v]);
+  }
+  const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
+  const uint32_t meta = (uint32_t)(key >> 32);
+  const uint32_t lf = slot_lfail(P, pc, koi);
+  const unsigned long long dn = (P.dense_ok && !meta_store(meta)) ? dense_lookup(P, oi, pc) : 0ull;
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) {
+    SlotE& e = slots[v];
+    e.key = key;
+    e.dense = dn;
+    const uint64_t mid = (meta & 3u) < 3u ? 0xFFFFFFFFull : ~0ull;
+    for (int m = 0; m < 6; ++m) e.mm[m] = (m & 1) ? 0ull : mid;
+    e.nwin = 0;
+    e.lfail = lf;
+    e.nosnap = nosnap ? 1u : 0u;
+    for (int i = 0; i < 8; ++i) e.sum[i] = 0;
+  }
+  __syncwarp();
+  return v;
 }
 
 struct Rec {
@@ -502,42 +553,43 @@ __device__ __forceinline__ void red_add(uint32_t* p, uint32_t v) {
   asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// A warp's ring: NSTAGE stages of STAGE_WIN windows; lane l reads record l of a window.
+// A warp's ring: NSTAGE stages of STAGE_WIN (= 2) windows; lane l reads record l.
 struct Ring {
-  const ve_record* src;   // next stage to issue
+  const ve_record* src;   // next stage to issue (lane 0)
   uint32_t left;          // windows not yet consumed
-  uint32_t iss;           // windows not yet issued
-  uint32_t rd;            // ve_smem offset of stage 0 of this warp + lane * 24
-  uint32_t bar;           // shared address of this warp's mbarrier 0
-  uint32_t dst;           // shared address of this warp's stage 0
-  uint32_t d, h, ph;      // current stage, window in it, phase parity
+  uint32_t iss;           // windows not yet issued (lane 0)
+  uint32_t o, o0;         // ve_smem offset of this lane's record in the next window / in stage 0
+  uint32_t bar, bar0;     // shared address of the current / first stage's mbarrier
+  uint32_t dst0;          // shared address of stage 0
+  uint32_t h, ph;         // window within the stage, phase parity
 };
 
-__device__ __forceinline__ void ring_issue_next(Ring& R) {
+__device__ __forceinline__ void ring_issue_stage(Ring& R, uint32_t d) {
   const uint32_t nw = R.iss < (uint32_t)STAGE_WIN ? R.iss : (uint32_t)STAGE_WIN;
-  ring_issue(R.dst + R.d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar + R.d * 8);
+  ring_issue(R.dst0 + d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar0 + d * 8u);
   R.src += nw * 32;
   R.iss -= nw;
 }
 
-// take the next window out of the ring (lane l gets record l); a stage is refilled
-// as soon as its last window has been read
+// take the next window out of the ring; a stage is refilled as soon as its last
+// window has been read
 __device__ __forceinline__ void ring_next(Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm) {
-  if (R.h == 0) ring_wait(R.bar + R.d * 8, R.ph);
-  const uint32_t o = R.rd + R.d * STAGE_BYTES + R.h * WIN_BYTES;
-  addr = *reinterpret_cast<const unsigned long long*>(ve_smem + o);
-  val = *reinterpret_cast<const unsigned long long*>(ve_smem + o + 8);
-  pm = *reinterpret_cast<const unsigned long long*>(ve_smem + o + 16);
+  if (R.h == 0) ring_wait(R.bar, R.ph);
+  addr = *reinterpret_cast<const unsigned long long*>(ve_smem + R.o);
+  val = *reinterpret_cast<const unsigned long long*>(ve_smem + R.o + 8);
+  pm = *reinterpret_cast<const unsigned long long*>(ve_smem + R.o + 16);
   --R.left;
-  if (++R.h == (uint32_t)STAGE_WIN) {
-    R.h = 0;
+  R.o += WIN_BYTES;
+  if (R.h) {
     __syncwarp();
     if ((threadIdx.x & 31) == 0 && R.iss) {
       fence_proxy_async();   // our generic reads of the stage precede the next async write
-      ring_issue_next(R);
+      ring_issue_stage(R, (R.bar - R.bar0) >> 3);
     }
-    if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.ph ^= 1u; }
+    R.bar += 8u;
+    if (R.bar == R.bar0 + NSTAGE * 8u) { R.bar = R.bar0; R.o = R.o0; R.ph ^= 1u; }
   }
+  R.h ^= 1u;
 }
 
 __device__ __forceinline__ Rec load_rec(const AnalyzeParams& P, uint64_t w, uint64_t wend, int lane) {
@@ -704,6 +756,8 @@ __device__ __forceinline__ bool meta_fast(uint32_t meta0, uint32_t pc0, uint32_t
   return (meta0 >> 5) == 0u && ((VALID_KL >> (meta0 & 15u)) & 1u) && pc0 < n_pcs;
 }
 
+__device__ const unsigned long long ve_zero_word = 0ull;
+
 template <int LG>
 __device__ __forceinline__ uint64_t ld_pre(uint64_t p) {
   if (LG == 0) return __ldg((const unsigned char*)p);
@@ -777,149 +831,135 @@ __device__ __noinline__ uint32_t fast_line(const AnalyzeParams& P, WarpCache& wc
   return __shfl_sync(0xFFFFFFFFu, lf, 0);
 }
 
-// slot install on a miss: flush the victim, claim its line-FAIL bits and dense array
-__device__ __forceinline__ int slot_install(const AnalyzeParams& P, FastSlots& F, uint64_t& acc, uint64_t key,
-                                           uint32_t pc0, const ObjCache& oc, bool st) {
-  const int lane = threadIdx.x & 31;
-  const int s = (F.key[0] == ~0ull) ? 0 : (F.key[1] == ~0ull) ? 1 : (int)(F.mru ^ 1u);
-  const uint64_t victim = s ? F.key[1] : F.key[0];
-  if (victim != ~0ull) fast_flush(P, victim, s, acc);
-  if ((lane >> 4) == s) acc = fast_identity(lane & 15);
-  const uint32_t lf = slot_lfail(P, pc0, oc.id);
-  const unsigned long long dn = (P.dense_ok && !st) ? dense_lookup(P, oc.oi, pc0) : 0ull;
-  // constant indices only: the slot table stays in registers
-  if (s) { F.key[1] = key; F.lfail[1] = lf; F.dense[1] = dn; }
-  else { F.key[0] = key; F.lfail[0] = lf; F.dense[0] = dn; }
-  return s;
-}
-
 // Consume fast windows of access type (KIND, LG) from the ring, starting with the
 // current one (addr, val, pm; known fast).  Returns true when it stopped at a
 // window it has not consumed (left in addr, val, pm), false when the ring is empty.
 template <int KIND, int LG>
-__device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, const ObjCache& oc, FastSlots& F,
-                                         uint64_t& acc, Ring& R, uint32_t scr, uint64_t& addr, uint64_t& val,
-                                         uint64_t& pm) {
+__device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, const ObjCache& oc, SlotE* slots,
+                                         uint32_t* snext, Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm) {
+  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;   // min / max totals
+  constexpr bool ISF = KIND >= 2;
   constexpr uint32_t W = 1u << LG;
   constexpr uint32_t KL = ((uint32_t)KIND << 2) | (uint32_t)LG;
   constexpr int MB = KIND == 3 ? 7 : (LG == 1 ? 10 : LG == 2 ? 23 : 52);
   const unsigned FULL = 0xFFFFFFFFu;
   const int lane = threadIdx.x & 31;
-  const uint64_t tmask = P.mant_bits >= (uint32_t)MB ? ~0ull : ~((1ull << (MB - P.mant_bits)) - 1ull);
+  const MT tmask = (MT)(P.mant_bits >= (uint32_t)MB ? ~0ull : ~((1ull << (MB - P.mant_bits)) - 1ull));
   const bool eqdef = oc.pre != 0ull;
-  // this lane's accumulator field (lane & 15) of its slot (lane >> 4): a sum taken
-  // from the packed REDUX results A / B, a constant per window, or a min / max
-  const int fl = lane & 15;
-  const bool f_sum = fl <= 8, f_min = fl >= 9 && (fl & 1), f_fromA = fl <= 3;
-  const uint32_t f_sh = (fl == 1 || fl == 4) ? 0u : (fl == 2 || fl == 5) ? 6u : fl == 6 ? 12u : fl == 7 ? 18u : 24u;
-  const uint32_t f_mask = (fl == 0 || fl == 3 || fl > 8) ? 0u : 63u;
-  const uint32_t f_add = fl == 0 ? 32u : (fl == 3 && !eqdef) ? 32u : 0u;
-  const uint32_t f_mm = scr + 8u * (uint32_t)(fl >= 9 && fl <= 14 ? fl - 9 : 0);
   uint64_t pm0 = shfl64(FULL, pm, 0);
+  // the active slot, in registers
+  uint64_t akey = ~0ull;
+  int a = 0;
+  uint32_t nwin = 0, lf = 3u, c0 = 0, c1 = 0, c2 = 0, c3 = 0, c4 = 0, c5 = 0, c6 = 0;
+  unsigned long long dn = 0;
+  MT m0 = 0, m1 = 0, m2 = 0, m3 = 0, m4 = 0, m5 = 0;
+  auto save = [&]() {
+    __syncwarp();
+    if (lane == 0) {
+      SlotE& e = slots[a];
+      e.nwin = nwin; e.lfail = lf;
+      e.sum[0] = c0; e.sum[1] = c1; e.sum[2] = c2; e.sum[3] = c3; e.sum[4] = c4; e.sum[5] = c5; e.sum[6] = c6;
+      e.mm[0] = m0; e.mm[1] = m1; e.mm[2] = m2; e.mm[3] = m3; e.mm[4] = m4; e.mm[5] = m5;
+    }
+    __syncwarp();
+  };
   while (true) {
     const uint32_t pc0 = (uint32_t)pm0, meta0 = (uint32_t)(pm0 >> 32);
     const bool st = meta_store(meta0);
-    // select / install the register slot of (meta, object, pc)
     const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
-    const int s = (F.key[0] == key) ? 0 : (F.key[1] == key) ? 1 : slot_install(P, F, acc, key, pc0, oc, st);
-    F.mru = (uint32_t)s;
-    const uint32_t lf_s = s ? F.lfail[1] : F.lfail[0];
-    const unsigned long long dn_s = s ? F.dense[1] : F.dense[0];
+    if (key != akey) {
+      if (akey != ~0ull) save();
+      a = slot_acquire(P, slots, snext, key, oc.oi, !eqdef);
+      akey = key;
+      const SlotE& e = slots[a];
+      nwin = e.nwin; lf = e.lfail; dn = e.dense;
+      c0 = e.sum[0]; c1 = e.sum[1]; c2 = e.sum[2]; c3 = e.sum[3]; c4 = e.sum[4]; c5 = e.sum[5]; c6 = e.sum[6];
+      m0 = (MT)e.mm[0]; m1 = (MT)e.mm[1]; m2 = (MT)e.mm[2]; m3 = (MT)e.mm[3]; m4 = (MT)e.mm[4]; m5 = (MT)e.mm[5];
+    }
 
-    // S3: element, gather, written bitmap
+    // S3: element, gather (unconditional: a zero word when the object has no
+    // snapshot, so nothing waits on a merge of the loaded value), written bitmap
     const uint64_t off = addr - oc.base;
     const uint64_t e = off >> LG;
-    const uint64_t pv = eqdef ? ld_pre<LG>(oc.pre + off) : 0ull;
+    const uint64_t pv = ld_pre<LG>(eqdef ? oc.pre + off : (uint64_t)&ve_zero_word);
     const uint64_t word = oc.bmoff + (e >> 5);
     const uint32_t bit = 1u << ((uint32_t)e & 31u);
     if (st) bitmap_or_win(P.t.W, true, word, bit);
 
-    // C4-C7 reductions of the window
-    uint64_t rmin, rmax, omin, omax, tmin = ~0ull, tmax = 0ull;
-    uint32_t B = 0;
+    // C4-C7: the window's REDUX totals
+    ++nwin;
     if constexpr (LG < 3) {
       const uint32_t b = (uint32_t)val;
-      rmin = __reduce_min_sync(FULL, b);
-      rmax = __reduce_max_sync(FULL, b);
+      m0 = min(m0, __reduce_min_sync(FULL, b));
+      m1 = max(m1, __reduce_max_sync(FULL, b));
       if constexpr (KIND == 0) {
-        omin = rmin; omax = rmax;
-      } else if constexpr (KIND == 1) {           // sext32(b) ^ 2^31: order-isomorphic to the 64-bit key
+        m2 = m0; m3 = m1;
+      } else if constexpr (KIND == 1) {           // sext32(b) ^ 2^31
         constexpr uint32_t sh = 32 - (8 << LG);
         const uint32_t k = (uint32_t)(((int32_t)(b << sh)) >> sh) ^ 0x80000000u;
-        omin = __reduce_min_sync(FULL, k);
-        omax = __reduce_max_sync(FULL, k);
+        m2 = min(m2, __reduce_min_sync(FULL, k));
+        m3 = max(m3, __reduce_max_sync(FULL, k));
       } else {
         constexpr uint32_t SIGN = 1u << ((8 << LG) - 1);
         constexpr uint32_t MASK = (uint32_t)((1ull << (8 << LG)) - 1ull);
         const uint32_t ff = fflags32<KIND, LG>(b);
         const bool okv = !(ff & 1u);              // NaNs excluded from ord / trunc
         const uint32_t k = (b & SIGN) ? (~b & MASK) : (b | SIGN);
-        const uint32_t t = b & (uint32_t)tmask;
-        // a non-NaN key is never 0xFFFFFFFF, so that is the min identity in 32 bits
-        const uint32_t kmin = __reduce_min_sync(FULL, okv ? k : 0xFFFFFFFFu);
-        omax = __reduce_max_sync(FULL, okv ? k : 0u);
-        const uint32_t tm = __reduce_min_sync(FULL, okv ? t : 0xFFFFFFFFu);
-        tmax = __reduce_max_sync(FULL, okv ? t : 0u);
-        omin = kmin == 0xFFFFFFFFu ? ~0ull : (uint64_t)kmin;
-        tmin = tm == 0xFFFFFFFFu ? ~0ull : (uint64_t)tm;
-        B = __reduce_add_sync(FULL, (ff * 0x108421u) & 0x1041041u);   // flag bit i -> 6-bit field i
+        const uint32_t t = b & tmask;
+        m2 = min(m2, __reduce_min_sync(FULL, okv ? k : 0xFFFFFFFFu));
+        m3 = max(m3, __reduce_max_sync(FULL, okv ? k : 0u));
+        m4 = min(m4, __reduce_min_sync(FULL, okv ? t : 0xFFFFFFFFu));
+        m5 = max(m5, __reduce_max_sync(FULL, okv ? t : 0u));
+        c2 += __popc(__ballot_sync(FULL, ff & 1u));
+        c3 += __popc(__ballot_sync(FULL, ff & 2u));
+        c4 += __popc(__ballot_sync(FULL, ff & 4u));
+        c5 += __popc(__ballot_sync(FULL, ff & 8u));
       }
     } else {
-      rmin = redmin64(FULL, val);
-      rmax = redmax64(FULL, val);
+      m0 = min(m0, redmin64(FULL, val));
+      m1 = max(m1, redmax64(FULL, val));
       if constexpr (KIND == 0) {
-        omin = rmin; omax = rmax;
+        m2 = m0; m3 = m1;
       } else if constexpr (KIND == 1) {
         const uint64_t k = val ^ (1ull << 63);
-        omin = redmin64(FULL, k);
-        omax = redmax64(FULL, k);
+        m2 = min(m2, redmin64(FULL, k));
+        m3 = max(m3, redmax64(FULL, k));
       } else {
         int64_t ival;
         const uint32_t ff = float_flags(val, 2u, 3u, ival);
         const bool okv = !(ff & 1u);
         const uint64_t k = (val >> 63) ? ~val : (val | (1ull << 63));
         const uint64_t t = val & tmask;
-        omin = redmin64(FULL, okv ? k : ~0ull);
-        omax = redmax64(FULL, okv ? k : 0ull);
-        tmin = redmin64(FULL, okv ? t : ~0ull);
-        tmax = redmax64(FULL, okv ? t : 0ull);
-        B = __reduce_add_sync(FULL, (ff * 0x108421u) & 0x1041041u);
+        m2 = min(m2, redmin64(FULL, okv ? k : ~0ull));
+        m3 = max(m3, redmax64(FULL, okv ? k : 0ull));
+        m4 = min(m4, redmin64(FULL, okv ? t : ~0ull));
+        m5 = max(m5, redmax64(FULL, okv ? t : 0ull));
+        c2 += __popc(__ballot_sync(FULL, ff & 1u));
+        c3 += __popc(__ballot_sync(FULL, ff & 2u));
+        c4 += __popc(__ballot_sync(FULL, ff & 4u));
+        c5 += __popc(__ballot_sync(FULL, ff & 8u));
+        c6 += __popc(__ballot_sync(FULL, ff & 16u));
       }
     }
+    (void)ISF;
     // the pre-snapshot gather is consumed only now
     const bool eq = eqdef && pv == val;
-    const uint32_t A = __reduce_add_sync(FULL, (uint32_t)(val == 0ull) | ((uint32_t)eq << 6));
+    c0 += __popc(__ballot_sync(FULL, val == 0ull));
+    const unsigned eqm = __ballot_sync(FULL, eq);
+    c1 += __popc(eqm);
     // C3 loaded elements; loads counted per element below get their bits from the
     // dense counters at report time
-    if (!st && dn_s == 0ull && __any_sync(FULL, eq)) bitmap_or_win(P.t.L, eq, word, bit);
-
-    // fold into slot s: sums from the packed REDUX results, min / max via scratch
-    if (lane == 0) {
-      *reinterpret_cast<ulonglong2*>(ve_smem + scr) = make_ulonglong2(rmin, rmax);
-      *reinterpret_cast<ulonglong2*>(ve_smem + scr + 16) = make_ulonglong2(omin, omax);
-      *reinterpret_cast<ulonglong2*>(ve_smem + scr + 32) = make_ulonglong2(tmin, tmax);
-    }
-    __syncwarp();
-    {
-      const uint64_t m = *reinterpret_cast<const unsigned long long*>(ve_smem + f_mm);
-      const uint32_t sv = (((f_fromA ? A : B) >> f_sh) & f_mask) + f_add;
-      const uint64_t nv = f_sum ? acc + sv : f_min ? (m < acc ? m : acc) : (m > acc ? m : acc);
-      if ((lane >> 4) == s && fl != 15) acc = nv;
-    }
+    if (!st && dn == 0ull && eqm) bitmap_or_win(P.t.L, eq, word, bit);
 
     // C8 line state, only while a key of the slot is not yet FAIL
-    if (lf_s != 3u) {
-      const uint32_t lf = fast_line(P, wc, addr, val, meta0, pc0, oc.id, lf_s);
-      if (s) F.lfail[1] = lf;
-      else F.lfail[0] = lf;
-    }
+    if (lf != 3u) lf = fast_line(P, wc, addr, val, meta0, pc0, oc.id, lf);
 
     // S8: exact histogram.  A load that reads an unchanged element carries that
     // element's pre value, so it is counted per element (mapped to its value at
     // report time); every other record is inserted per distinct value.
-    const bool dl = dn_s != 0ull && eq;
-    if (dl) red_add(reinterpret_cast<uint32_t*>(dn_s) + e, 1u);
-    const unsigned hm = __ballot_sync(FULL, !dl);
+    const bool dl = dn != 0ull && eq;
+    if (dl) red_add(reinterpret_cast<uint32_t*>(dn) + e, 1u);
+    const unsigned hm = dn != 0ull ? ~eqm : FULL;
     if (hm) {
       const uint32_t tag = (pc0 << 16) | (oc.id & 0xFFFFu);
       const int l = __ffs(hm) - 1;
@@ -933,14 +973,14 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, 
     }
 
     // next window: continue while it is fast with the same access type
-    if (R.left == 0) return false;
+    if (R.left == 0) { save(); return false; }
     ring_next(R, addr, val, pm);
     pm0 = shfl64(FULL, pm, 0);
     const uint64_t o2 = addr - oc.base;
     bool ok = pm == pm0 && o2 <= oc.lim && (o2 & (W - 1)) == 0;
     if constexpr (LG < 3) ok = ok && (val >> (8 * W)) == 0ull;
-    const uint32_t m2 = (uint32_t)(pm0 >> 32);
-    if (!__all_sync(FULL, ok) || (m2 & 15u) != KL || !meta_fast(m2, (uint32_t)pm0, P.n_pcs)) return true;
+    const uint32_t mt = (uint32_t)(pm0 >> 32);
+    if (!__all_sync(FULL, ok) || (mt & 15u) != KL || !meta_fast(mt, (uint32_t)pm0, P.n_pcs)) { save(); return true; }
   }
 }
 
@@ -959,11 +999,13 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   for (uint32_t i = tid; i < P.objc; i += blockDim.x) { S.sob[i] = P.o.base[i]; S.soe[i] = P.o.end[i]; }
   if (tid < 4) S.sctr[tid] = 0;
   __shared__ WarpCache s_wc[K1_WARPS];
-  __shared__ __align__(16) uint64_t s_scr[K1_WARPS][8];
+  __shared__ SlotE s_slot[K1_WARPS][NSLOT];
+  __shared__ uint32_t s_snext[K1_WARPS];
   WarpCache& wc = s_wc[warp];
-  const uint32_t scr = (uint32_t)((const uint8_t*)s_scr[warp] - ve_smem);   // ve_smem offset
+  SlotE* slots = s_slot[warp];
   if (lane < WC) wc.key1[lane] = 0;
-  if (lane == 0) wc.next = 0;
+  if (lane < NSLOT) slots[lane].key = ~0ull;
+  if (lane == 0) { wc.next = 0; s_snext[warp] = 0; }
 
   // this warp's contiguous range of windows; full windows stream through a TMA ring
   const uint64_t nwin = (P.n + 31) / 32;
@@ -975,29 +1017,19 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   Ring R;
   R.src = P.recs + wbeg * 32;
   R.left = R.iss = (uint32_t)(rend - wbeg);
-  R.rd = P.o_ring + (uint32_t)warp * RING * WIN_BYTES + (uint32_t)lane * 24u;
-  R.dst = smem_u32(ve_smem + P.o_ring + (uint32_t)warp * RING * WIN_BYTES);
-  R.bar = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
-  R.d = R.h = R.ph = 0;
+  R.o0 = R.o = P.o_ring + (uint32_t)warp * RING * WIN_BYTES + (uint32_t)lane * 24u;
+  R.dst0 = smem_u32(ve_smem + P.o_ring + (uint32_t)warp * RING * WIN_BYTES);
+  R.bar0 = R.bar = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
+  R.h = R.ph = 0;
   if (lane == 0) {   // only lane 0 issues: its src / iss are the ones that matter
-    for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar + d * 8, 1);
+    for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar0 + d * 8u, 1);
     fence_mbar_init();
-    for (int d = 0; d < NSTAGE && R.iss; ++d) {
-      R.d = d;
-      ring_issue_next(R);
-    }
-    R.d = 0;
+    for (int d = 0; d < NSTAGE && R.iss; ++d) ring_issue_stage(R, (uint32_t)d);
   }
   __syncthreads();
   ObjCache oc;
   oc.base = 0; oc.lim = 0; oc.bmoff = 0; oc.pre = 0; oc.oi = -1; oc.id = 0; oc.fastlg = 0xFFu;
   uint32_t n_inv = 0, n_unm = 0;   // this lane's invalid / unmapped records (slow windows)
-  FastSlots F;
-  F.mru = 0;
-  F.key[0] = F.key[1] = ~0ull;
-  F.lfail[0] = F.lfail[1] = 3u;
-  F.dense[0] = F.dense[1] = 0ull;
-  uint64_t acc = 0;
 
   uint64_t addr = 0, val = 0, pm = 0;
   bool have = false;
@@ -1021,18 +1053,18 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
     if (fast) {
       // specialised on the window's access type (compile-time width / kind)
       switch (meta0 & 15u) {
-        case 0: have = run_fast<0, 0>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 1: have = run_fast<0, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 2: have = run_fast<0, 2>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 3: have = run_fast<0, 3>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 4: have = run_fast<1, 0>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 5: have = run_fast<1, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 6: have = run_fast<1, 2>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 7: have = run_fast<1, 3>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 9: have = run_fast<2, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 10: have = run_fast<2, 2>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        case 11: have = run_fast<2, 3>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;
-        default: have = run_fast<3, 1>(P, wc, oc, F, acc, R, scr, addr, val, pm); break;   // 13: bfloat16
+        case 0: have = run_fast<0, 0>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 1: have = run_fast<0, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 2: have = run_fast<0, 2>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 3: have = run_fast<0, 3>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 4: have = run_fast<1, 0>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 5: have = run_fast<1, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 6: have = run_fast<1, 2>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 7: have = run_fast<1, 3>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 9: have = run_fast<2, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 10: have = run_fast<2, 2>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        case 11: have = run_fast<2, 3>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
+        default: have = run_fast<3, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;   // 13: bfloat16
       }
     } else {
       const uint32_t cnt = slow_window(P, wc, addr, val, pm, true);
@@ -1048,9 +1080,9 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
     n_unm += cnt >> 16;
   }
 
-  // fold the warp's register slots and line cache, then the CTA's shared state
-  if (F.key[0] != ~0ull) fast_flush(P, F.key[0], 0, acc);
-  if (F.key[1] != ~0ull) fast_flush(P, F.key[1], 1, acc);
+  // fold the warp's key slots and line cache, then the CTA's shared state
+  for (int i = 0; i < NSLOT; ++i)
+    if (slots[i].key != ~0ull) slot_flush(P, &slots[i]);
   n_inv = __reduce_add_sync(FULL, n_inv);
   n_unm = __reduce_add_sync(FULL, n_unm);
   if (lane == 0) {
