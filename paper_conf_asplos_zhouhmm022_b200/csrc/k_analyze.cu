@@ -22,13 +22,23 @@
 // same bits (C12).
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <type_traits>
 
 #include "ve_internal.cuh"
 
 namespace ve {
 
-constexpr int K1_THREADS = 512;  // 16 warps x 128 registers
+#ifndef VE_K1_THREADS
+#define VE_K1_THREADS 512
+#endif
+#ifndef VE_STEAL
+#define VE_STEAL 0   // 1: dynamic chunk claiming (measured slower at 512 threads: L1 locality), 0: one static range per warp
+#endif
+#ifndef VE_PIPE
+#define VE_PIPE 0    // 1: software-pipelined pre gather (helps at 384 threads, not at 512: register pressure)
+#endif
+constexpr int K1_THREADS = VE_K1_THREADS;  // 16 warps x 128 registers
 constexpr int K1_WARPS = K1_THREADS / 32;
 constexpr int RING = 6;                      // record windows in flight per warp (TMA ring)
 constexpr uint32_t WIN_BYTES = 32 * sizeof(ve_record);
@@ -43,6 +53,8 @@ struct AnalyzeParams {
   uint32_t objc;            // objects cached in shared memory (0 = use global table)
   uint32_t dense_ok;        // dense per-element counting enabled for this launch
   uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
+  uint64_t nring;           // full windows, claimed in CHUNK-window chunks through *work
+  unsigned long long* work; // chunk counter (zeroed before the launch)
   // byte offsets of the dynamic shared-memory regions (see carve_offsets)
   uint32_t o_ssum, o_smin, o_smax, o_sline, o_shs, o_shc, o_sob, o_soe, o_sctr, o_ring, o_bars;
   DevObjects o;
@@ -545,6 +557,15 @@ __device__ __forceinline__ void ring_wait(uint32_t bar, uint32_t phase) {
         : "memory");
   }
 }
+__device__ __forceinline__ bool mbar_ready(uint32_t bar, uint32_t phase) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(bar), "r"(phase)
+      : "memory");
+  return ok != 0;
+}
 // fire-and-forget global atomics (no compiler-generated warp aggregation around them)
 __device__ __forceinline__ void red_or(uint32_t* p, uint32_t v) {
   asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
@@ -554,38 +575,71 @@ __device__ __forceinline__ void red_add(uint32_t* p, uint32_t v) {
 }
 
 // A warp's ring: NSTAGE stages of STAGE_WIN (= 2) windows; lane l reads record l.
+// Warps claim CHUNK-window chunks of the full windows dynamically (the next chunk
+// index is claimed one chunk ahead), so no warp idles while others still work.
+constexpr uint32_t CHUNK = 64;
 struct Ring {
-  const ve_record* src;   // next stage to issue (lane 0)
-  uint32_t left;          // windows not yet consumed
-  uint32_t iss;           // windows not yet issued (lane 0)
-  uint32_t o, o0;         // ve_smem offset of this lane's record in the next window / in stage 0
+  const ve_record* src;   // next window to issue (lane 0)
+  unsigned long long nextc;  // chunk claimed for after the current one (lane 0)
+  uint32_t iss;           // windows of the current chunk not yet issued (lane 0)
+  uint32_t left;          // windows issued and not yet consumed
+  uint32_t o, o0;         // shared address of this lane's record in the next window / in stage 0
   uint32_t bar, bar0;     // shared address of the current / first stage's mbarrier
   uint32_t dst0;          // shared address of stage 0
   uint32_t h, ph;         // window within the stage, phase parity
 };
 
-__device__ __forceinline__ void ring_issue_stage(Ring& R, uint32_t d) {
+// lane 0: move to the claimed chunk (if any) and claim the one after it
+__device__ __forceinline__ void ring_chunk(const AnalyzeParams& P, Ring& R) {
+#if !VE_STEAL
+  if (R.nextc != ~0ull) {     // static: this warp's range, once
+    const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + (threadIdx.x >> 5);
+    const uint64_t b = gw * P.nring / tw, e = (gw + 1) * P.nring / tw;
+    R.src = P.recs + b * 32;
+    R.iss = (uint32_t)(e - b);
+    R.nextc = ~0ull;
+  } else {
+    R.iss = 0;
+  }
+  return;
+#endif
+  const uint64_t w0 = (uint64_t)R.nextc * CHUNK;
+  if (w0 < P.nring) {
+    R.src = P.recs + w0 * 32;
+    R.iss = (uint32_t)(P.nring - w0 < CHUNK ? P.nring - w0 : CHUNK);
+    R.nextc = atomicAdd(P.work, 1ull);
+  } else {
+    R.iss = 0;
+  }
+}
+
+__device__ __forceinline__ void ring_issue_stage(const AnalyzeParams& P, Ring& R, uint32_t d) {
   const uint32_t nw = R.iss < (uint32_t)STAGE_WIN ? R.iss : (uint32_t)STAGE_WIN;
   ring_issue(R.dst0 + d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar0 + d * 8u);
   R.src += nw * 32;
   R.iss -= nw;
+  R.left += nw;
+  if (R.iss == 0) ring_chunk(P, R);
 }
 
 // take the next window out of the ring; a stage is refilled as soon as its last
 // window has been read
-__device__ __forceinline__ void ring_next(Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm) {
+__device__ __forceinline__ void ring_next(const AnalyzeParams& P, Ring& R, uint64_t& addr, uint64_t& val,
+                                          uint64_t& pm) {
   if (R.h == 0) ring_wait(R.bar, R.ph);
-  addr = *reinterpret_cast<const unsigned long long*>(ve_smem + R.o);
-  val = *reinterpret_cast<const unsigned long long*>(ve_smem + R.o + 8);
-  pm = *reinterpret_cast<const unsigned long long*>(ve_smem + R.o + 16);
+  asm volatile("ld.shared.u64 %0, [%3];\n\tld.shared.u64 %1, [%3+8];\n\tld.shared.u64 %2, [%3+16];"
+               : "=l"(addr), "=l"(val), "=l"(pm)
+               : "r"(R.o)
+               : "memory");
   --R.left;
   R.o += WIN_BYTES;
   if (R.h) {
     __syncwarp();
     if ((threadIdx.x & 31) == 0 && R.iss) {
       fence_proxy_async();   // our generic reads of the stage precede the next async write
-      ring_issue_stage(R, (R.bar - R.bar0) >> 3);
+      ring_issue_stage(P, R, (R.bar - R.bar0) >> 3);
     }
+    R.left = __shfl_sync(0xFFFFFFFFu, R.left, 0);
     R.bar += 8u;
     if (R.bar == R.bar0 + NSTAGE * 8u) { R.bar = R.bar0; R.o = R.o0; R.ph ^= 1u; }
   }
@@ -838,6 +892,7 @@ template <int KIND, int LG>
 __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, const ObjCache& oc, SlotE* slots,
                                          uint32_t* snext, Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm) {
   using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;   // min / max totals
+  using PT = MT;                                                                // one gathered value
   constexpr bool ISF = KIND >= 2;
   constexpr uint32_t W = 1u << LG;
   constexpr uint32_t KL = ((uint32_t)KIND << 2) | (uint32_t)LG;
@@ -863,25 +918,45 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, 
     }
     __syncwarp();
   };
+  bool newkey = true;
+  bool have_npv = false;
+  PT npv = 0;
   while (true) {
     const uint32_t pc0 = (uint32_t)pm0, meta0 = (uint32_t)(pm0 >> 32);
     const bool st = meta_store(meta0);
-    const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
-    if (key != akey) {
-      if (akey != ~0ull) save();
-      a = slot_acquire(P, slots, snext, key, oc.oi, !eqdef);
-      akey = key;
-      const SlotE& e = slots[a];
-      nwin = e.nwin; lf = e.lfail; dn = e.dense;
-      c0 = e.sum[0]; c1 = e.sum[1]; c2 = e.sum[2]; c3 = e.sum[3]; c4 = e.sum[4]; c5 = e.sum[5]; c6 = e.sum[6];
-      m0 = (MT)e.mm[0]; m1 = (MT)e.mm[1]; m2 = (MT)e.mm[2]; m3 = (MT)e.mm[3]; m4 = (MT)e.mm[4]; m5 = (MT)e.mm[5];
+    if (newkey) {
+      const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
+      if (key != akey) {
+        if (akey != ~0ull) save();
+        a = slot_acquire(P, slots, snext, key, oc.oi, !eqdef);
+        akey = key;
+        const SlotE& e = slots[a];
+        nwin = e.nwin; lf = e.lfail; dn = e.dense;
+        c0 = e.sum[0]; c1 = e.sum[1]; c2 = e.sum[2]; c3 = e.sum[3]; c4 = e.sum[4]; c5 = e.sum[5]; c6 = e.sum[6];
+        m0 = (MT)e.mm[0]; m1 = (MT)e.mm[1]; m2 = (MT)e.mm[2]; m3 = (MT)e.mm[3]; m4 = (MT)e.mm[4]; m5 = (MT)e.mm[5];
+      }
+      newkey = false;
     }
 
     // S3: element, gather (unconditional: a zero word when the object has no
     // snapshot, so nothing waits on a merge of the loaded value), written bitmap
     const uint64_t off = addr - oc.base;
     const uint64_t e = off >> LG;
-    const uint64_t pv = ld_pre<LG>(eqdef ? oc.pre + off : (uint64_t)&ve_zero_word);
+    // software-pipelined gather: this window's pre value was loaded during the
+    // previous window when that one could see it in the ring; the next window's
+    // is issued now, so a gather's latency overlaps a whole window of work
+    if (!have_npv) npv = (PT)ld_pre<LG>(eqdef ? oc.pre + off : (uint64_t)&ve_zero_word);
+    const PT pv = npv;
+    have_npv = false;
+    if (VE_PIPE && eqdef && R.left && (R.h == 1u || mbar_ready(R.bar, R.ph))) {
+      unsigned long long na;
+      asm volatile("ld.shared.u64 %0, [%1];" : "=l"(na) : "r"(R.o));
+      const uint64_t no = na - oc.base;
+      if (no <= oc.lim && (no & (W - 1)) == 0) {
+        npv = (PT)ld_pre<LG>(oc.pre + no);
+        have_npv = true;
+      }
+    }
     const uint64_t word = oc.bmoff + (e >> 5);
     const uint32_t bit = 1u << ((uint32_t)e & 31u);
     if (st) bitmap_or_win(P.t.W, true, word, bit);
@@ -902,7 +977,9 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, 
       } else {
         constexpr uint32_t SIGN = 1u << ((8 << LG) - 1);
         constexpr uint32_t MASK = (uint32_t)((1ull << (8 << LG)) - 1ull);
-        const uint32_t ff = fflags32<KIND, LG>(b);
+        uint32_t ff;
+        if constexpr (KIND == 2 && LG == 2) ff = fflags_f32(b);
+        else ff = fflags32<KIND, LG>(b);
         const bool okv = !(ff & 1u);              // NaNs excluded from ord / trunc
         const uint32_t k = (b & SIGN) ? (~b & MASK) : (b | SIGN);
         const uint32_t t = b & tmask;
@@ -943,7 +1020,7 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, 
     }
     (void)ISF;
     // the pre-snapshot gather is consumed only now
-    const bool eq = eqdef && pv == val;
+    const bool eq = eqdef && (uint64_t)pv == val;
     c0 += __popc(__ballot_sync(FULL, val == 0ull));
     const unsigned eqm = __ballot_sync(FULL, eq);
     c1 += __popc(eqm);
@@ -974,13 +1051,19 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, 
 
     // next window: continue while it is fast with the same access type
     if (R.left == 0) { save(); return false; }
-    ring_next(R, addr, val, pm);
-    pm0 = shfl64(FULL, pm, 0);
+    ring_next(P, R, addr, val, pm);
     const uint64_t o2 = addr - oc.base;
-    bool ok = pm == pm0 && o2 <= oc.lim && (o2 & (W - 1)) == 0;
+    bool ok = o2 <= oc.lim && (o2 & (W - 1)) == 0;
     if constexpr (LG < 3) ok = ok && (val >> (8 * W)) == 0ull;
-    const uint32_t mt = (uint32_t)(pm0 >> 32);
-    if (!__all_sync(FULL, ok) || (mt & 15u) != KL || !meta_fast(mt, (uint32_t)pm0, P.n_pcs)) { save(); return true; }
+    if (__all_sync(FULL, ok && pm == pm0)) continue;        // same pc and type: same slot
+    const uint64_t pmn = shfl64(FULL, pm, 0);
+    const uint32_t mt = (uint32_t)(pmn >> 32);
+    if (!__all_sync(FULL, ok && pm == pmn) || (mt & 15u) != KL || !meta_fast(mt, (uint32_t)pmn, P.n_pcs)) {
+      save();
+      return true;
+    }
+    pm0 = pmn;
+    newkey = true;
   }
 }
 
@@ -1007,25 +1090,25 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   if (lane < NSLOT) slots[lane].key = ~0ull;
   if (lane == 0) { wc.next = 0; s_snext[warp] = 0; }
 
-  // this warp's contiguous range of windows; full windows stream through a TMA ring
+  // full windows stream through the TMA ring in dynamically claimed chunks; without
+  // the ring (records not 16-byte aligned) each warp takes a static range
   const uint64_t nwin = (P.n + 31) / 32;
   const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + warp;
-  const uint64_t wbeg = gw * nwin / tw, wend = (gw + 1) * nwin / tw;
-  const uint64_t nfull = P.n / 32;
-  uint64_t rend = P.ring ? (wend < nfull ? wend : nfull) : wbeg;   // the ring covers [wbeg, rend)
-  if (rend < wbeg) rend = wbeg;
   Ring R;
-  R.src = P.recs + wbeg * 32;
-  R.left = R.iss = (uint32_t)(rend - wbeg);
-  R.o0 = R.o = P.o_ring + (uint32_t)warp * RING * WIN_BYTES + (uint32_t)lane * 24u;
+  R.left = 0;
+  R.iss = 0;
   R.dst0 = smem_u32(ve_smem + P.o_ring + (uint32_t)warp * RING * WIN_BYTES);
+  R.o0 = R.o = R.dst0 + (uint32_t)lane * 24u;
   R.bar0 = R.bar = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
   R.h = R.ph = 0;
-  if (lane == 0) {   // only lane 0 issues: its src / iss are the ones that matter
+  if (lane == 0 && P.nring) {   // only lane 0 issues: its src / iss / nextc are the ones that matter
     for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar0 + d * 8u, 1);
     fence_mbar_init();
-    for (int d = 0; d < NSTAGE && R.iss; ++d) ring_issue_stage(R, (uint32_t)d);
+    R.nextc = atomicAdd(P.work, 1ull);
+    ring_chunk(P, R);
+    for (int d = 0; d < NSTAGE && R.iss; ++d) ring_issue_stage(P, R, (uint32_t)d);
   }
+  R.left = __shfl_sync(FULL, R.left, 0);
   __syncthreads();
   ObjCache oc;
   oc.base = 0; oc.lim = 0; oc.bmoff = 0; oc.pre = 0; oc.oi = -1; oc.id = 0; oc.fastlg = 0xFFu;
@@ -1034,7 +1117,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   uint64_t addr = 0, val = 0, pm = 0;
   bool have = false;
   while (have || R.left) {
-    if (!have) ring_next(R, addr, val, pm);
+    if (!have) ring_next(P, R, addr, val, pm);
     have = false;
     const uint64_t pm0 = shfl64(FULL, pm, 0);
     const uint32_t meta0 = (uint32_t)(pm0 >> 32), pc0 = (uint32_t)pm0;
@@ -1072,8 +1155,11 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       n_unm += cnt >> 16;
     }
   }
-  // windows outside the ring (partial tail, or records not 16-byte aligned)
-  for (uint64_t w = rend; w < wend; ++w) {
+  // windows outside the ring: the partial last window, or (records not 16-byte
+  // aligned) a static range of every warp
+  uint64_t wbeg = P.nring, wend = gw == 0 ? nwin : P.nring;
+  if (!P.nring) { wbeg = gw * nwin / tw; wend = (gw + 1) * nwin / tw; }
+  for (uint64_t w = wbeg; w < wend; ++w) {
     const Rec cur = load_rec(P, w, wend, lane);
     const uint32_t cnt = slow_window(P, wc, cur.addr, cur.val, cur.pm, w * 32 + lane < P.n);
     n_inv += cnt & 0xFFFFu;
@@ -1133,6 +1219,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   // u32 per-element counters cannot overflow while the ctx has seen < 2^32 records
   P.dense_ok = (c->dense_used > 0 && c->records_analyzed + n < (1ull << 32)) ? 1u : 0u;
   P.ring = ((uintptr_t)d % 16 == 0) ? 1u : 0u;
+  P.nring = P.ring ? n / 32 : 0;
+  P.work = c->t.glob + G_WORK;
   c->records_analyzed += n;
   // shared stat rows: up to 256 keys, PCs first then object keys (incl. SHARED)
   const uint32_t NSK_MAX = 256;
@@ -1149,7 +1237,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   cudaFuncAttributes fa;
   cudaFuncGetAttributes(&fa, k_analyze);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring
-  uint32_t hs = 8192;
+  uint32_t hs = getenv("VE_HS") ? (uint32_t)atoi(getenv("VE_HS")) : 8192;
   while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > budget) hs >>= 1;
   P.hs = hs;
   carve_offsets(P, sp + so);
@@ -1160,6 +1248,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   uint64_t windows = (n + 31) / 32;
   uint64_t blocks = (windows + K1_WARPS - 1) / K1_WARPS;
   if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+  e = cudaMemsetAsync(P.work, 0, sizeof(unsigned long long), s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze work counter");
   count_launch();
   k_analyze<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();

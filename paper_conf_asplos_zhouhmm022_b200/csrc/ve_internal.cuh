@@ -61,7 +61,7 @@ struct DevTables {
   unsigned long long* hcount;  // [hcap]
   uint64_t hmask;           // hcap - 1
 };
-enum : int { G_RECORDS = 0, G_INVALID = 1, G_UNMAPPED = 2, G_OVERFLOW = 3 };
+enum : int { G_RECORDS = 0, G_INVALID = 1, G_UNMAPPED = 2, G_OVERFLOW = 3, G_WORK = 7 };  // 7: K1 chunk counter
 
 struct DevObjects {          // sorted by base
   const uint64_t* base;
@@ -266,6 +266,25 @@ __device__ __forceinline__ uint32_t float_flags(uint64_t b, uint32_t kind, uint3
   if (!(top <= 127 && low >= max(top - 7, -133))) f |= 8u;              // bfloat16
   if (is_f64 && !(top <= 127 && low >= max(top - 23, -149))) f |= 16u;  // binary32
   return f;
+}
+
+// float_flags of an IEEE binary32 value in closed form (same results as
+// float_flags(b, 2, 2, .) for every bit pattern; checked exhaustively by
+// scripts/check_fflags.cu).  E = exponent field, tz = trailing zeros of the
+// significand with its implicit bit: the value is sig * 2^(E-150), its lowest set
+// bit has exponent E-150+tz and its leading bit E-127, so
+//   integer           <=> E + tz >= 150 and E <= 189 (|v| < 2^63)
+//   binary16 exact    <=> E <= 142, tz >= 13, E + tz >= 126 (normal or subnormal f16)
+//   bfloat16 exact    <=> the low 16 bits are zero (same exponent range as binary32)
+__device__ __forceinline__ uint32_t fflags_f32(uint32_t b) {
+  const uint32_t E = (b >> 23) & 0xFFu, M = b & 0x7FFFFFu;
+  const uint32_t tz = (uint32_t)__ffs((int)(M | 0x800000u)) - 1u;
+  const uint32_t t = E + tz;
+  const bool special = E == 0xFFu;                        // Inf or NaN
+  uint32_t f = (b != 0u && !(t >= 150u && E <= 189u)) ? 2u : 0u;
+  if (!((b << 1) == 0u || (special && M == 0u) || (E <= 142u && tz >= 13u && t >= 126u))) f |= 4u;
+  if (b & 0xFFFFu) f |= 8u;
+  return (special && M != 0u) ? 15u : f;                  // NaN fails everything
 }
 
 // C7 mantissa truncation

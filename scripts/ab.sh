@@ -1,8 +1,10 @@
 #!/bin/bash
-# A/B timing of alternative libve builds (VE_LIB_PATH)
+# A/B timing of alternative libve builds (build/libve_*.so via VE_LIB_PATH), 2 rounds
 cd "${GRAFT_REPO_ROOT:-.}"; mkdir -p gpurun_out; rm -f gpurun_out/ab.log
-for lib in paper_conf_asplos_zhouhmm022_b200/libve.so build/libve_384.so; do
+for r in 1 2; do
+for lib in build/libve_*.so; do
   echo "== $lib" >> gpurun_out/ab.log
-  VE_LIB_PATH=$lib timeout 300 python scripts/step_timing.py 2>/dev/null | grep "analyze\[" | tail -2 >> gpurun_out/ab.log
+  VE_LIB_PATH=$lib timeout 300 python scripts/step_timing.py 2>/dev/null | grep "analyze\[" | tail -2 | tr '\n' ' ' >> gpurun_out/ab.log
+  echo >> gpurun_out/ab.log
 done
-timeout 900 python -m pytest tests/ -x -q -m gpu > gpurun_out/gpu_tests.log 2>&1; echo "exit $?" >> gpurun_out/gpu_tests.log
+done
