@@ -21,6 +21,12 @@ VEG_FN uint64_t snap_word(int cfg, int epoch, uint64_t seed, uint32_t obj, int p
     uint64_t hi = veg_cfg2_elem(seed, (uint32_t)epoch, obj, post, e + 1);
     return lo | (hi << 32);
   }
+  if (VEG_BASE(cfg) == VEG_CFG3) {
+    const uint32_t sh = VEG_SHIFT(cfg);
+    if (veg_c3_object(sh, obj).elem_width == 8) return veg_c3_elem(seed, sh, obj, post, j);
+    return veg_c3_elem(seed, sh, obj, post, 2 * j) | (veg_c3_elem(seed, sh, obj, post, 2 * j + 1) << 32);
+  }
+  if (VEG_BASE(cfg) == VEG_CFG4) return veg_c4_elem(seed, VEG_SHIFT(cfg), (uint32_t)epoch, obj, post, j);
   if (cfg == VEG_FUZZ) return veg_fuzz_word(seed, obj, post, j);
   return 0;
 }
@@ -28,6 +34,8 @@ VEG_FN uint64_t snap_word(int cfg, int epoch, uint64_t seed, uint32_t obj, int p
 VEG_FN void record_at(int cfg, int epoch, uint64_t seed, uint64_t r, veg_record* out) {
   if (cfg == VEG_CFG1) veg_cfg1_record(seed, r, out);
   else if (cfg == VEG_CFG2) veg_cfg2_record(seed, (uint32_t)epoch, r, out);
+  else if (VEG_BASE(cfg) == VEG_CFG3) veg_cfg3_record(seed, VEG_SHIFT(cfg), r, out);
+  else if (VEG_BASE(cfg) == VEG_CFG4) veg_cfg4_record(seed, VEG_SHIFT(cfg), (uint32_t)epoch, r, out);
   else veg_fuzz_record(seed, r, out);
 }
 
@@ -43,6 +51,18 @@ extern "C" int veg_info_get(int cfg, int epoch, veg_info* out) {
     if (epoch < 0 || epoch > 1) return -1;
     out->n_records = epoch == 0 ? VEG_C2_FILL_N : VEG_C2_GEMM_N;
     out->n_pcs = 5; out->n_obj = 4; out->n_epochs = 2;
+    return 0;
+  }
+  if (VEG_BASE(cfg) == VEG_CFG3) {                /* one epoch per training iteration (seed 3 + it) */
+    if (epoch < 0 || epoch > 3 || VEG_SHIFT(cfg) > 7 || (cfg & ~0xFFF)) return -1;
+    out->n_records = veg_c3_n(VEG_SHIFT(cfg)); out->n_pcs = VEG_C3_NPCS; out->n_obj = VEG_C3_NOBJ;
+    out->n_epochs = 4;
+    return 0;
+  }
+  if (VEG_BASE(cfg) == VEG_CFG4) {                /* epoch 0 hotspot3D-like, epoch 1 Castro-like */
+    if (epoch < 0 || epoch > 1 || VEG_SHIFT(cfg) > 4 || (cfg & ~0xFFF)) return -1;
+    out->n_records = veg_c4_n(VEG_SHIFT(cfg), (uint32_t)epoch); out->n_pcs = VEG_C4_NPCS; out->n_obj = 6;
+    out->n_epochs = 2;
     return 0;
   }
   if (cfg == VEG_FUZZ) {
@@ -61,6 +81,10 @@ extern "C" int veg_object_get(int cfg, int epoch, uint32_t i, veg_object* out) {
     out->has_pre = 1; out->has_post = 1;
   } else if (cfg == VEG_CFG2) {
     *out = veg_cfg2_object(i);
+  } else if (VEG_BASE(cfg) == VEG_CFG3) {
+    *out = veg_c3_object(VEG_SHIFT(cfg), i);
+  } else if (VEG_BASE(cfg) == VEG_CFG4) {
+    *out = veg_c4_object(VEG_SHIFT(cfg), i);
   } else {
     *out = veg_fuzz_object(i);
   }
@@ -90,9 +114,11 @@ extern "C" int veg_records_device(int cfg, int epoch, uint64_t seed, uint64_t r0
 
 extern "C" void veg_snapshot_host(int cfg, int epoch, uint64_t seed, uint32_t obj, int post, uint64_t off,
                                   uint64_t len, uint8_t* out) {
+  uint64_t wj = ~0ull, w = 0;
   for (uint64_t p = 0; p < len; ++p) {
     uint64_t b = off + p;
-    out[p] = (uint8_t)(snap_word(cfg, epoch, seed, obj, post, b / 8) >> (8 * (b % 8)));
+    if (b / 8 != wj) { wj = b / 8; w = snap_word(cfg, epoch, seed, obj, post, wj); }
+    out[p] = (uint8_t)(w >> (8 * (b % 8)));
   }
 }
 

@@ -40,7 +40,11 @@ typedef struct veg_info {
   uint32_t n_epochs, pad;
 } veg_info;
 
-enum { VEG_CFG1 = 1, VEG_CFG2 = 2, VEG_FUZZ = 100, VEG_DEDUP = 101 };
+enum { VEG_CFG1 = 1, VEG_CFG2 = 2, VEG_CFG3 = 3, VEG_CFG4 = 4, VEG_FUZZ = 100, VEG_DEDUP = 101 };
+/* cfg codes of the scalable configs carry a size shift s in bits 8..11:
+ * VEG_CFG3 | (s << 8) is cfg3 with every tensor 2^s times smaller (s = 0: full size) */
+#define VEG_BASE(cfg) ((cfg) & 0xFF)
+#define VEG_SHIFT(cfg) (((cfg) >> 8) & 15)
 
 /* meta encoding (include/ve.h): [1:0] log2 w, [3:2] kind, [4] store, [5] shared */
 #define VEG_META(lg, kind, st) ((uint32_t)(lg) | ((uint32_t)(kind) << 2) | ((uint32_t)(st) << 4))
@@ -267,6 +271,270 @@ VEG_FN void veg_cfg2_record(uint64_t seed, uint32_t epoch, uint64_t r, veg_recor
   out->value = is_st ? veg_cfg2_out(seed, e) : 0;
   out->pc = is_st ? 4 : 3;
   out->meta = is_st ? st : ld;
+}
+
+/* f64 bits of (x * 2^-k), x exact in f64, result normal */
+VEG_FN uint64_t veg_f64_scaled(int64_t x, int k) {
+  uint64_t u = veg_f64_of_int(x);
+  if ((u & 0x7FFFFFFFFFFFFFFFull) == 0) return u;
+  return u - ((uint64_t)k << 52);
+}
+
+/* =========================================================================
+ * cfg3: PyTorch op mix (BASELINE.json configs[2]), one epoch
+ * per training iteration (seed 3 + iteration), 16 objects, 20 PCs:
+ *   S0 embedding      ld ids (i64), then per token 24 x (ld weight row chunk, st out)
+ *   S1 masked_fill_   st weight row 0 (padding) = +0.0 over a zero row (redundant)
+ *   S2 add            ld a, ld b, st c = a + b        (c: the high-cardinality PC)
+ *   S3 relu           ld c (new values), st r = max(c, +0)
+ *   S4 mul by ones    ld r, ld ones (1.0), st m = r
+ *   S5 sum-reduce     per row: 1024 x ld x, then ONE st (partial group: later
+ *                     windows are not 32-aligned)
+ *   S6 index_select   ld idx (i64 arange, structured), ld src, st dst = src
+ *   S7 zeros_like, zero_, ones fill: st grad 0, st grad 0, st ones_t 1.0 (all
+ *                     over equal pre values: redundant)
+ * Sizes at shift s: T = 32768>>s tokens, D = 768, V = 30522, M = 16 Mi>>s,
+ * R = 16384>>s rows of 1024, NI = 4 Mi>>s; 264,291,072 records at s = 0.
+ * Values are exact binary fractions k * 2^-10 (sums stay exact).
+ * ========================================================================= */
+#define VEG_C3_V 30522ull
+#define VEG_C3_D 768ull
+#define VEG_C3_BASE 0x7c0000000000ull
+#define VEG_C3_NOBJ 16u
+#define VEG_C3_NPCS 20u
+
+typedef struct veg_c3dims { uint64_t T, M, R, NI; } veg_c3dims;
+VEG_FN veg_c3dims veg_c3_dims(uint32_t sh) {
+  veg_c3dims d;
+  d.T = 32768ull >> sh; d.M = (16ull << 20) >> sh; d.R = 16384ull >> sh; d.NI = (4ull << 20) >> sh;
+  return d;
+}
+/* records per segment */
+VEG_FN void veg_c3_seglen(uint32_t sh, uint64_t* L) {
+  veg_c3dims d = veg_c3_dims(sh);
+  L[0] = d.T + 2 * d.T * VEG_C3_D;
+  L[1] = VEG_C3_D;
+  L[2] = 3 * d.M;
+  L[3] = 2 * d.M;
+  L[4] = 3 * d.M;
+  L[5] = 1025 * d.R;
+  L[6] = 3 * d.NI;
+  L[7] = 3 * d.M;
+}
+VEG_FN uint64_t veg_c3_n(uint32_t sh) {
+  uint64_t L[8], n = 0;
+  veg_c3_seglen(sh, L);
+  for (int i = 0; i < 8; ++i) n += L[i];
+  return n;
+}
+VEG_FN veg_object veg_c3_object(uint32_t sh, uint32_t i) {
+  veg_c3dims d = veg_c3_dims(sh);
+  const uint64_t elems[16] = {VEG_C3_V * VEG_C3_D, d.T, d.T * VEG_C3_D, d.M, d.M, d.M, d.M, d.M, d.M,
+                              d.R * 1024, d.R, d.NI, d.NI, d.NI, d.M, d.M};
+  veg_object o;
+  o.id = i;
+  o.base = VEG_C3_BASE + (uint64_t)i * (1ull << 36);
+  o.elem_width = (i == 1 || i == 11) ? 8 : 4;
+  o.size = elems[i] * o.elem_width;
+  o.has_pre = 1;
+  o.has_post = 1;
+  return o;
+}
+/* embedding weights: N(0, ~0.02)-shaped, 2^16-entry table; the padding row 0 is zero */
+VEG_FN uint32_t veg_c3_w(uint64_t seed, uint64_t e) {
+  if (e < VEG_C3_D) return 0;
+  uint64_t t = veg_h(seed, 30, e) & 0xFFFFu;
+  int64_t s = 0;
+  for (int j = 0; j < 4; ++j) s += (int64_t)(veg_h(seed, 300 + j, t) & 0xFFFFu);
+  return veg_f32_scaled(s - 131070, 21);
+}
+/* token ids: 10% padding id 0, else a skewed (Zipf-like) id in [1, V) */
+VEG_FN uint64_t veg_c3_id(uint64_t seed, uint64_t t) {
+  uint64_t h = veg_h(seed, 31, t);
+  if (h % 10 == 0) return 0;
+  uint64_t span = 1 + (h >> 32) % (VEG_C3_V - 1);
+  return 1 + ((h >> 8) & 0xFFFFFFu) % span;
+}
+VEG_FN int64_t veg_c3_k20(uint64_t seed, uint64_t st, uint64_t e) {   /* k in [-2^19, 2^19) */
+  return (int64_t)(veg_h(seed, st, e) & 0xFFFFFu) - 524288;
+}
+VEG_FN int64_t veg_c3_kc(uint64_t seed, uint64_t e) { return veg_c3_k20(seed, 33, e) + veg_c3_k20(seed, 34, e); }
+VEG_FN uint32_t veg_c3_r(uint64_t seed, uint64_t e) {
+  int64_t k = veg_c3_kc(seed, e);
+  return k > 0 ? veg_f32_scaled(k, 10) : 0u;
+}
+VEG_FN int64_t veg_c3_kx(uint64_t seed, uint64_t e) {                 /* reduce input, k in [-2^12, 2^12) */
+  return (int64_t)(veg_h(seed, 35, e) & 0x1FFFu) - 4096;
+}
+VEG_FN uint32_t veg_c3_rowsum(uint64_t seed, uint64_t i) {
+  int64_t s = 0;
+  for (uint64_t j = 0; j < 1024; ++j) s += veg_c3_kx(seed, i * 1024 + j);
+  return veg_f32_scaled(s, 10);
+}
+/* element e of object i: pre (post = 0) or post (post = 1) snapshot */
+VEG_FN uint64_t veg_c3_elem(uint64_t seed, uint32_t sh, uint32_t i, int post, uint64_t e) {
+  switch (i) {
+    case 0: return veg_c3_w(seed, e);
+    case 1: return veg_c3_id(seed, e);
+    case 2: return post ? veg_c3_w(seed, veg_c3_id(seed, e / VEG_C3_D) * VEG_C3_D + e % VEG_C3_D) : 0;
+    case 3: return veg_f32_scaled(veg_c3_k20(seed, 33, e), 10);
+    case 4: return veg_f32_scaled(veg_c3_k20(seed, 34, e), 10);
+    case 5: return post ? veg_f32_scaled(veg_c3_kc(seed, e), 10) : 0;
+    case 6: return post ? veg_c3_r(seed, e) : 0;
+    case 7: return 0x3F800000u;
+    case 8: return post ? veg_c3_r(seed, e) : 0;
+    case 9: return veg_f32_scaled(veg_c3_kx(seed, e), 10);
+    case 10: return post ? veg_c3_rowsum(seed, e) : 0;
+    case 11: return e;
+    case 12: return veg_f32_scaled(veg_c3_k20(seed, 36, e), 10);
+    case 13: return post ? veg_f32_scaled(veg_c3_k20(seed, 36, e), 10) : 0;
+    case 14: return 0;
+    default: return 0x3F800000u;
+  }
+  (void)sh;
+}
+VEG_FN void veg_c3_put(veg_record* out, uint32_t sh, uint32_t obj, uint64_t e, uint64_t v, uint32_t pc, int st) {
+  veg_object o = veg_c3_object(sh, obj);
+  out->addr = o.base + e * o.elem_width;
+  out->value = v;
+  out->pc = pc;
+  out->meta = VEG_META(o.elem_width == 8 ? 3 : 2, o.elem_width == 8 ? 1 : 2, st);
+}
+VEG_FN void veg_cfg3_record(uint64_t seed, uint32_t sh, uint64_t r, veg_record* out) {
+  uint64_t L[8];
+  veg_c3_seglen(sh, L);
+  int sg = 0;
+  while (sg < 7 && r >= L[sg]) r -= L[sg++];
+  const uint64_t D = VEG_C3_D;
+  if (sg == 0) {                                   /* embedding: per 32-token block */
+    const uint64_t blk = 32 + 32 * 24 * 64;
+    uint64_t b = r / blk, u = r % blk;
+    if (u < 32) { uint64_t t = b * 32 + u; veg_c3_put(out, sh, 1, t, veg_c3_id(seed, t), 0, 0); return; }
+    u -= 32;
+    uint64_t t = b * 32 + u / (24 * 64), v = u % (24 * 64);
+    uint64_t d = (v / 64) * 32 + v % 32;
+    uint64_t we = veg_c3_id(seed, t) * D + d;
+    if (v % 64 < 32) veg_c3_put(out, sh, 0, we, veg_c3_w(seed, we), 1, 0);
+    else veg_c3_put(out, sh, 2, t * D + d, veg_c3_w(seed, we), 2, 1);
+    return;
+  }
+  if (sg == 1) { veg_c3_put(out, sh, 0, r, 0, 3, 1); return; }
+  if (sg == 2 || sg == 4 || sg == 6) {             /* 3 groups per 32-element block */
+    uint64_t e = (r / 96) * 32 + r % 32, g = (r % 96) / 32;
+    if (sg == 2) {
+      if (g == 0) veg_c3_put(out, sh, 3, e, veg_f32_scaled(veg_c3_k20(seed, 33, e), 10), 4, 0);
+      else if (g == 1) veg_c3_put(out, sh, 4, e, veg_f32_scaled(veg_c3_k20(seed, 34, e), 10), 5, 0);
+      else veg_c3_put(out, sh, 5, e, veg_f32_scaled(veg_c3_kc(seed, e), 10), 6, 1);
+    } else if (sg == 4) {
+      if (g == 0) veg_c3_put(out, sh, 6, e, veg_c3_r(seed, e), 9, 0);
+      else if (g == 1) veg_c3_put(out, sh, 7, e, 0x3F800000u, 10, 0);
+      else veg_c3_put(out, sh, 8, e, veg_c3_r(seed, e), 11, 1);
+    } else {
+      if (g == 0) veg_c3_put(out, sh, 11, e, e, 14, 0);
+      else if (g == 1) veg_c3_put(out, sh, 12, e, veg_f32_scaled(veg_c3_k20(seed, 36, e), 10), 15, 0);
+      else veg_c3_put(out, sh, 13, e, veg_f32_scaled(veg_c3_k20(seed, 36, e), 10), 16, 1);
+    }
+    return;
+  }
+  if (sg == 3) {                                   /* relu */
+    uint64_t e = (r / 64) * 32 + r % 32;
+    if ((r % 64) < 32) veg_c3_put(out, sh, 5, e, veg_f32_scaled(veg_c3_kc(seed, e), 10), 7, 0);
+    else veg_c3_put(out, sh, 6, e, veg_c3_r(seed, e), 8, 1);
+    return;
+  }
+  if (sg == 5) {                                   /* sum-reduce rows */
+    uint64_t i = r / 1025, u = r % 1025;
+    if (u < 1024) veg_c3_put(out, sh, 9, i * 1024 + u, veg_f32_scaled(veg_c3_kx(seed, i * 1024 + u), 10), 12, 0);
+    else veg_c3_put(out, sh, 10, i, veg_c3_rowsum(seed, i), 13, 1);
+    return;
+  }
+  {                                                /* zeros_like, zero_, ones fill */
+    veg_c3dims d = veg_c3_dims(sh);
+    uint64_t pass = r / d.M, e = r % d.M;
+    if (pass < 2) veg_c3_put(out, sh, 14, e, 0, 17 + (uint32_t)pass, 1);
+    else veg_c3_put(out, sh, 15, e, 0x3F800000u, 19, 1);
+  }
+}
+
+/* =========================================================================
+ * cfg4: LAMMPS / Castro-style f64 stencils (BASELINE.json configs[3]; SURVEY
+ * 8(d) cfg4) on a G^3 grid, G = 512 >> s, point p = (z G + y) G + x.  Warps
+ * take 32 consecutive points; each memory instruction is one 32-record group.
+ *   epoch 0 (hotspot3D-like): 7 loads of T_in (centre, x-1, x+1, y-1, y+1, z-1,
+ *     z+1; faces clamped), st T_out = T_in(centre).  T_in = 300 + 3q/8192,
+ *     q = hash mod 4096: one K=7 truncation bucket (approximate), n_ld_reload
+ *     = 6/7 of the T_in loads.
+ *   epoch 1 (cellconslin_slopes-like): ld a (1.0 except every 20th point: 2.0),
+ *     ld xc[x] (= x + 64: structured), ld vol (1.0), ld s[x-1], s, s[x+1]
+ *     (clamped), st s (= s_pre where a == 1: redundant, else s_pre + 1).
+ * Objects (f64, ew 8): 0 T_in, 1 T_out, 2 a, 3 s, 4 vol (G^3 each), 5 xc (G).
+ * ========================================================================= */
+#define VEG_C4_BASE 0x7b0000000000ull
+#define VEG_C4_NPCS 15u
+
+VEG_FN uint64_t veg_c4_g(uint32_t sh) { return 512ull >> sh; }
+VEG_FN veg_object veg_c4_object(uint32_t sh, uint32_t i) {
+  uint64_t G = veg_c4_g(sh);
+  veg_object o;
+  o.id = i;
+  o.base = VEG_C4_BASE + (uint64_t)i * (1ull << 36);
+  o.elem_width = 8;
+  o.size = 8 * (i == 5 ? G : G * G * G);
+  o.has_pre = 1;
+  o.has_post = 1;
+  return o;
+}
+VEG_FN uint64_t veg_c4_tin(uint64_t seed, uint64_t p) {
+  return veg_f64_scaled(300 * 8192 + 3 * (int64_t)(veg_h(seed, 41, p) % 4096), 13);
+}
+VEG_FN int64_t veg_c4_spre(uint64_t seed, uint64_t p) { return (int64_t)(veg_h(seed, 42, p) % 1000); }
+VEG_FN uint64_t veg_c4_elem(uint64_t seed, uint32_t sh, uint32_t epoch, uint32_t i, int post, uint64_t e) {
+  uint64_t G = veg_c4_g(sh);
+  switch (i) {
+    case 0: return veg_c4_tin(seed, e);
+    case 1: return (post && epoch == 0) ? veg_c4_tin(seed, e) : 0;
+    case 2: return (e % 20 != 0) ? 0x3FF0000000000000ull : 0x4000000000000000ull;
+    case 3: return veg_f64_of_int(veg_c4_spre(seed, e) + ((post && epoch == 1 && e % 20 == 0) ? 1 : 0));
+    case 4: return 0x3FF0000000000000ull;
+    default: return veg_f64_of_int((int64_t)(e % G) + 64);
+  }
+}
+VEG_FN uint64_t veg_c4_n(uint32_t sh, uint32_t epoch) {
+  uint64_t G = veg_c4_g(sh);
+  return (epoch == 0 ? 8 : 7) * G * G * G;
+}
+VEG_FN void veg_cfg4_record(uint64_t seed, uint32_t sh, uint32_t epoch, uint64_t r, veg_record* out) {
+  const uint64_t G = veg_c4_g(sh);
+  const uint32_t ng = epoch == 0 ? 8 : 7;
+  const uint64_t b = r / (32 * ng), g = (r % (32 * ng)) / 32, p = b * 32 + r % 32;
+  const uint64_t x = p % G, y = (p / G) % G, z = p / (G * G);
+  uint32_t obj;
+  uint64_t e = p;
+  int st = 0;
+  if (epoch == 0) {
+    obj = 0;
+    if (g == 1) e = p - (x > 0);
+    else if (g == 2) e = p + (x + 1 < G);
+    else if (g == 3) e = p - (y > 0) * G;
+    else if (g == 4) e = p + (y + 1 < G) * G;
+    else if (g == 5) e = p - (z > 0) * G * G;
+    else if (g == 6) e = p + (z + 1 < G) * G * G;
+    else if (g == 7) { obj = 1; st = 1; }
+    out->value = veg_c4_tin(seed, e);
+    out->pc = (uint32_t)g;
+  } else {
+    const uint32_t objs[7] = {2, 5, 4, 3, 3, 3, 3};
+    obj = objs[g];
+    if (g == 1) e = x;
+    else if (g == 3) e = p - (x > 0);
+    else if (g == 5) e = p + (x + 1 < G);
+    st = g == 6;
+    out->value = veg_c4_elem(seed, sh, 1, obj, st, e);
+    out->pc = 8 + (uint32_t)g;
+  }
+  const veg_object o = veg_c4_object(sh, obj);
+  out->addr = o.base + 8 * e;
+  out->meta = VEG_META(3, 2, st);
 }
 
 /* =========================================================================

@@ -8,8 +8,13 @@ import os
 
 import numpy as np
 
-CFG1, CFG2, FUZZ = 1, 2, 100
-SEEDS = {CFG1: 1, CFG2: 2}
+CFG1, CFG2, CFG3, CFG4, FUZZ = 1, 2, 3, 4, 100
+SEEDS = {CFG1: 1, CFG2: 2, CFG3: 3, CFG4: 4}
+
+
+def scaled(cfg, shift):
+    """cfg code of cfg3 / cfg4 with every tensor 2^shift times smaller (0 = full size)."""
+    return cfg | (shift << 8)
 
 REC_DTYPE = np.dtype([("addr", "<u8"), ("value", "<u8"), ("pc", "<u4"), ("meta", "<u4")])
 assert REC_DTYPE.itemsize == 24

@@ -8,6 +8,9 @@
  *
  *   cfg: VEG_CFG1 (1)  single kernel, 2^20 4-byte records, 16 PCs, one 4 MiB object
  *        VEG_CFG2 (2)  Darknet YOLOv4 conv layer; epoch 0 fill_ongpu, epoch 1 gemm
+ *        VEG_CFG3 (3)  PyTorch op mix (4 epochs = iterations, seed 3 + iteration)
+ *        VEG_CFG4 (4)  f64 stencils; epoch 0 hotspot3D-like, epoch 1 Castro-like
+ *                      (cfg3 / cfg4 | s << 8: tensors 2^s times smaller)
  *        VEG_FUZZ (100) adversarial mixed trace (unbounded record stream)
  *   Dedup sets: veg_dedup_* (object i of a set keyed by seed and size unit).
  *
