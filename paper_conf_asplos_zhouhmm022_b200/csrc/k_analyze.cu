@@ -32,15 +32,12 @@ namespace ve {
 #ifndef VE_K1_THREADS
 #define VE_K1_THREADS 512
 #endif
-#ifndef VE_STEAL
-#define VE_STEAL 0   // 1: dynamic chunk claiming (measured slower at 512 threads: L1 locality), 0: one static range per warp
-#endif
-#ifndef VE_PIPE
-#define VE_PIPE 0    // 1: software-pipelined pre gather (helps at 384 threads, not at 512: register pressure)
-#endif
 constexpr int K1_THREADS = VE_K1_THREADS;  // 16 warps x 128 registers
 constexpr int K1_WARPS = K1_THREADS / 32;
-constexpr int RING = 6;                      // record windows in flight per warp (TMA ring)
+#ifndef VE_RING
+#define VE_RING 6
+#endif
+constexpr int RING = VE_RING;                // record windows per warp ring (2 stages)
 constexpr uint32_t WIN_BYTES = 32 * sizeof(ve_record);
 
 struct AnalyzeParams {
@@ -53,8 +50,8 @@ struct AnalyzeParams {
   uint32_t objc;            // objects cached in shared memory (0 = use global table)
   uint32_t dense_ok;        // dense per-element counting enabled for this launch
   uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
-  uint64_t nring;           // full windows, claimed in CHUNK-window chunks through *work
-  unsigned long long* work; // chunk counter (zeroed before the launch)
+  uint64_t nring;           // full windows (streamed through the per-warp rings)
+  unsigned long long* work; // chunk claim counter (zeroed before the launch)
   // byte offsets of the dynamic shared-memory regions (see carve_offsets)
   uint32_t o_ssum, o_smin, o_smax, o_sline, o_shs, o_shc, o_sob, o_soe, o_sctr, o_ring, o_bars;
   DevObjects o;
@@ -407,8 +404,9 @@ struct __align__(16) SlotE {
 };
 static_assert(sizeof(SlotE) == 112, "SlotE layout");
 
-// claim (or find) a dense counter array of sorted object oi for pc (lane 0), broadcast
-__device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t pc) {
+// claim (or find) a dense counter array of sorted object oi for the loads of one
+// (pc, access type): claim key ck = meta << 16 | pc (lane 0), broadcast
+__device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t ck) {
   unsigned long long dp = 0;
   if ((threadIdx.x & 31) == 0) {
     for (int j = 0; j < DENSE_PER_OBJ; ++j) {
@@ -416,10 +414,10 @@ __device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, 
       uint32_t d = *(volatile uint32_t*)slot;
       if (d == DENSE_OFF) break;
       if (d == DENSE_FREE) {
-        d = atomicCAS(slot, DENSE_FREE, pc);
-        if (d == DENSE_FREE) d = pc;
+        d = atomicCAS(slot, DENSE_FREE, ck);
+        if (d == DENSE_FREE) d = ck;
       }
-      if (d == pc) {
+      if (d == ck) {
         dp = (unsigned long long)(P.o.dense_pool + P.o.dense_off[DENSE_PER_OBJ * oi + j]);
         break;
       }
@@ -509,7 +507,7 @@ __device__ __noinline__ int slot_acquire(const AnalyzeParams& P, SlotE* slots, u
   const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
   const uint32_t meta = (uint32_t)(key >> 32);
   const uint32_t lf = slot_lfail(P, pc, koi);
-  const unsigned long long dn = (P.dense_ok && !meta_store(meta)) ? dense_lookup(P, oi, pc) : 0ull;
+  const unsigned long long dn = (P.dense_ok && !meta_store(meta)) ? dense_lookup(P, oi, (meta << 16) | pc) : 0ull;
   __syncwarp();
   if ((threadIdx.x & 31) == 0) {
     SlotE& e = slots[v];
@@ -531,7 +529,14 @@ struct Rec {
 };
 
 // ---- per-warp TMA ring: cp.async.bulk of 2-window stages into shared memory ----
-constexpr int STAGE_WIN = 2;
+// Each warp streams its own contiguous range of full windows.  The ring state is
+// warp-uniform (every lane computes it; lane 0 alone issues the copies), so no
+// per-window broadcast is needed.  Records are read once: the copies carry an
+// L2 evict-first policy so the stream does not push snapshots and counters out.
+#ifndef VE_STAGE_WIN
+#define VE_STAGE_WIN 3
+#endif
+constexpr int STAGE_WIN = VE_STAGE_WIN;
 constexpr int NSTAGE = RING / STAGE_WIN;
 constexpr uint32_t STAGE_BYTES = STAGE_WIN * WIN_BYTES;
 
@@ -541,73 +546,91 @@ __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
 }
 __device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-__device__ __forceinline__ void ring_issue(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void ring_issue(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar, uint64_t pol) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          dst),
+      "l"(src), "r"(bytes), "r"(bar), "l"(pol)
+      : "memory");
 }
 __device__ __forceinline__ void ring_wait(uint32_t bar, uint32_t phase) {
-  uint32_t ok = 0;
-  while (!ok) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(ok)
-        : "r"(bar), "r"(phase)
-        : "memory");
-  }
-}
-__device__ __forceinline__ bool mbar_ready(uint32_t bar, uint32_t phase) {
-  uint32_t ok;
   asm volatile(
-      "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-      : "=r"(ok)
-      : "r"(bar), "r"(phase)
+      "{\n\t.reg .pred p;\n\tRW_LOOP:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra RW_LOOP;\n\t}" ::"r"(bar), "r"(phase)
       : "memory");
-  return ok != 0;
 }
-// fire-and-forget global atomics (no compiler-generated warp aggregation around them)
-__device__ __forceinline__ void red_or(uint32_t* p, uint32_t v) {
-  asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+// fire-and-forget global atomics under a predicate (no branch, no compiler-generated
+// warp aggregation around them)
+__device__ __forceinline__ void red_or(uint32_t* p, uint32_t v, bool on = true) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.relaxed.gpu.global.or.b32 [%0], %1;\n\t}" ::"l"(p),
+               "r"(v), "r"((uint32_t)on)
+               : "memory");
 }
-__device__ __forceinline__ void red_add(uint32_t* p, uint32_t v) {
-  asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+__device__ __forceinline__ void red_add(uint32_t* p, uint32_t v, bool on = true) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.relaxed.gpu.global.add.u32 [%0], %1;\n\t}" ::"l"(p),
+               "r"(v), "r"((uint32_t)on)
+               : "memory");
+}
+// the same, with an L2 evict-last policy (per-element counters that are re-hit)
+__device__ __forceinline__ void red_add_keep(uint32_t* p, uint32_t v, bool on = true) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\t.reg .b64 pol;\n\tsetp.ne.u32 q, %2, 0;\n\t"
+      "createpolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+      "@q red.relaxed.gpu.global.add.L2::cache_hint.u32 [%0], %1, pol;\n\t}" ::"l"(p),
+      "r"(v), "r"((uint32_t)on)
+      : "memory");
+}
+// lane predicate `on`: order the warp's generic reads of the stage before the async
+// write, arm the stage's mbarrier and start its bulk copy (branch-free)
+__device__ __forceinline__ void ring_issue_pred(bool on, uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %4, 0;\n\t"
+      "@q fence.proxy.async.shared::cta;\n\t"
+      "@q mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n\t"
+      "@q cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%2], [%3], %1, [%0], %5;\n\t}" ::"r"(
+          bar),
+      "r"(bytes), "r"(dst), "l"(src), "r"((uint32_t)on), "l"(policy_evict_first())
+      : "memory");
 }
 
-// A warp's ring: NSTAGE stages of STAGE_WIN (= 2) windows; lane l reads record l.
-// Warps claim CHUNK-window chunks of the full windows dynamically (the next chunk
-// index is claimed one chunk ahead), so no warp idles while others still work.
-constexpr uint32_t CHUNK = 64;
+// A warp's ring: NSTAGE (= 2) stages of STAGE_WIN windows.  The state is warp-
+// uniform; lane 0 alone issues the copies.  A consumed stage is refilled at the
+// start of the following ring_next, once the window read last has been fully
+// processed, so the proxy fence before the refill finds no loads outstanding.
+// With VE_CLAIM the warps claim CHUNK-window chunks of the trace dynamically
+// (balanced finish), else each warp streams one static contiguous range.
+static_assert(NSTAGE * STAGE_WIN == RING, "whole stages");
+#ifndef VE_CLAIM
+#define VE_CLAIM 1
+#endif
+constexpr uint32_t CHUNK = 32 * STAGE_WIN;   // windows per claim (whole stages)
 struct Ring {
-  const ve_record* src;   // next window to issue (lane 0)
-  unsigned long long nextc;  // chunk claimed for after the current one (lane 0)
-  uint32_t iss;           // windows of the current chunk not yet issued (lane 0)
+  const ve_record* src;   // next window to issue
+  uint32_t iss;           // windows of the current range / chunk not yet issued
   uint32_t left;          // windows issued and not yet consumed
-  uint32_t o, o0;         // shared address of this lane's record in the next window / in stage 0
-  uint32_t bar, bar0;     // shared address of the current / first stage's mbarrier
+  uint32_t o, o0;         // shared address of this lane's record in the current slot / in slot 0
+  uint32_t bar0;          // shared address of stage 0's mbarrier
   uint32_t dst0;          // shared address of stage 0
-  uint32_t h, ph;         // window within the stage, phase parity
+  uint32_t d, sw, ph;     // stage and window within it of the next read, phase parity of the current pass
+  uint32_t pend;          // stage + 1 to refill at the next read, 0 = none
 };
 
-// lane 0: move to the claimed chunk (if any) and claim the one after it
-__device__ __forceinline__ void ring_chunk(const AnalyzeParams& P, Ring& R) {
-#if !VE_STEAL
-  if (R.nextc != ~0ull) {     // static: this warp's range, once
-    const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + (threadIdx.x >> 5);
-    const uint64_t b = gw * P.nring / tw, e = (gw + 1) * P.nring / tw;
-    R.src = P.recs + b * 32;
-    R.iss = (uint32_t)(e - b);
-    R.nextc = ~0ull;
-  } else {
-    R.iss = 0;
-  }
-  return;
-#endif
-  const uint64_t w0 = (uint64_t)R.nextc * CHUNK;
+// claim the next chunk of full windows (all lanes; lane 0 does the atomic)
+__device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
+  unsigned long long c = 0;
+  if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
+  c = __shfl_sync(0xFFFFFFFFu, c, 0);
+  const uint64_t w0 = (uint64_t)c * CHUNK;
   if (w0 < P.nring) {
     R.src = P.recs + w0 * 32;
     R.iss = (uint32_t)(P.nring - w0 < CHUNK ? P.nring - w0 : CHUNK);
-    R.nextc = atomicAdd(P.work, 1ull);
   } else {
     R.iss = 0;
   }
@@ -615,35 +638,37 @@ __device__ __forceinline__ void ring_chunk(const AnalyzeParams& P, Ring& R) {
 
 __device__ __forceinline__ void ring_issue_stage(const AnalyzeParams& P, Ring& R, uint32_t d) {
   const uint32_t nw = R.iss < (uint32_t)STAGE_WIN ? R.iss : (uint32_t)STAGE_WIN;
-  ring_issue(R.dst0 + d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar0 + d * 8u);
+  if (nw == 0u) return;
+  ring_issue_pred((threadIdx.x & 31) == 0, R.dst0 + d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar0 + d * 8u);
   R.src += nw * 32;
   R.iss -= nw;
   R.left += nw;
-  if (R.iss == 0) ring_chunk(P, R);
+#if VE_CLAIM
+  if (R.iss == 0u) ring_claim(P, R);
+#endif
 }
 
-// take the next window out of the ring; a stage is refilled as soon as its last
-// window has been read
+// take the next window out of the ring (R.left > 0)
 __device__ __forceinline__ void ring_next(const AnalyzeParams& P, Ring& R, uint64_t& addr, uint64_t& val,
                                           uint64_t& pm) {
-  if (R.h == 0) ring_wait(R.bar, R.ph);
+  if (R.pend) {
+    __syncwarp();
+    ring_issue_stage(P, R, R.pend - 1u);
+    R.pend = 0;
+  }
+  const uint32_t d = R.d;
+  ring_wait(R.bar0 + d * 8u, R.ph);
   asm volatile("ld.shared.u64 %0, [%3];\n\tld.shared.u64 %1, [%3+8];\n\tld.shared.u64 %2, [%3+16];"
                : "=l"(addr), "=l"(val), "=l"(pm)
                : "r"(R.o)
                : "memory");
   --R.left;
   R.o += WIN_BYTES;
-  if (R.h) {
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0 && R.iss) {
-      fence_proxy_async();   // our generic reads of the stage precede the next async write
-      ring_issue_stage(P, R, (R.bar - R.bar0) >> 3);
-    }
-    R.left = __shfl_sync(0xFFFFFFFFu, R.left, 0);
-    R.bar += 8u;
-    if (R.bar == R.bar0 + NSTAGE * 8u) { R.bar = R.bar0; R.o = R.o0; R.ph ^= 1u; }
+  if (++R.sw == (uint32_t)STAGE_WIN) {   // stage consumed: refill it at the next read
+    R.sw = 0;
+    R.pend = R.iss ? d + 1u : 0u;
+    if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.o = R.o0; R.ph ^= 1u; }
   }
-  R.h ^= 1u;
 }
 
 __device__ __forceinline__ Rec load_rec(const AnalyzeParams& P, uint64_t w, uint64_t wend, int lane) {
@@ -812,12 +837,39 @@ __device__ __forceinline__ bool meta_fast(uint32_t meta0, uint32_t pc0, uint32_t
 
 __device__ const unsigned long long ve_zero_word = 0ull;
 
+// The pre-snapshot gather of a window is prefetched into L1 when the window is read
+// ahead (VE_PREFETCH) instead of being loaded into a register there: a register in
+// flight would stall the register rotation of the read-ahead pipeline.
+#ifndef VE_PREFETCH
+#define VE_PREFETCH 0
+#endif
+__device__ __forceinline__ void prefetch_l1(uint64_t p) { asm volatile("prefetch.global.L1 [%0];" ::"l"(p)); }
+// L2 policy of the data K1 re-reads (snapshot gathers, per-element counters): keep it
+// over the record stream (evict-first) and the histogram
+#ifndef VE_KEEP_HINT
+#define VE_KEEP_HINT 1
+#endif
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
 template <int LG>
 __device__ __forceinline__ uint64_t ld_pre(uint64_t p) {
+#if VE_KEEP_HINT
+  const uint64_t pol = policy_evict_last();
+  if (LG == 0) { uint16_t v; asm("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol)); return v & 0xFFu; }
+  if (LG == 1) { uint16_t v; asm("ld.global.nc.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol)); return v; }
+  if (LG == 2) { uint32_t v; asm("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol)); return v; }
+  uint64_t v;
+  asm("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
+#else
   if (LG == 0) return __ldg((const unsigned char*)p);
   if (LG == 1) return __ldg((const unsigned short*)p);
   if (LG == 2) return __ldg((const unsigned int*)p);
   return __ldg((const unsigned long long*)p);
+#endif
 }
 
 // C5 float flags of a <= 32-bit float (same definition as float_flags, 32-bit
@@ -851,30 +903,32 @@ __device__ __forceinline__ void bitmap_or_win(uint32_t* bm, bool part, uint64_t 
   if (__all_sync(0xFFFFFFFFu, !part || d <= 1ull)) {
     const uint32_t b0 = __reduce_or_sync(0xFFFFFFFFu, (part && d == 0ull) ? bit : 0u);
     const uint32_t b1 = __reduce_or_sync(0xFFFFFFFFu, (part && d == 1ull) ? bit : 0u);
-    if (lane < 2 && (lane ? b1 : b0)) red_or(&bm[w0 + lane], lane ? b1 : b0);
+    const uint32_t bv = lane ? b1 : b0;
+    red_or(&bm[w0 + lane], bv, lane < 2 && bv != 0u);
   } else {
     bitmap_or(bm, part, word, bit);
   }
 }
 
-// C8 for a fast window: one line state over its 32 points, merged into the keys
-// not yet FAIL; returns the updated FAIL bits
-__device__ __noinline__ uint32_t fast_line(const AnalyzeParams& P, WarpCache& wc, uint64_t addr,
-                                           uint64_t val, uint32_t meta0, uint32_t pc0, uint32_t koi0, uint32_t lf) {
-  const int lane = threadIdx.x & 31;
-  const uint32_t lg = meta0 & 3u, kind = (meta0 >> 2) & 3u;
-  Facts f;
-  f.addr = addr;
+// C8 point of a value: y = the integer the bits denote (uint, sint, or an integral
+// float); pfail = a float that is not a finite integer below 2^63 (no point)
+__device__ __forceinline__ __int128 line_y(uint64_t val, uint32_t kind, uint32_t lg, bool& pfail) {
   int64_t ival = 0;
   const uint32_t ff = kind >= 2u ? float_flags(val, kind, lg, ival) : 0u;
-  f.pfail = kind >= 2u && (ff & 2u);
-  if (kind == 0u) f.y = (__int128)val;
-  else if (kind == 1u) {
+  pfail = kind >= 2u && (ff & 2u);
+  if (kind == 0u) return (__int128)val;
+  if (kind == 1u) {
     const uint32_t sh64 = 64u - (8u << lg);
-    f.y = (__int128)((int64_t)(val << sh64) >> sh64);
-  } else f.y = (__int128)ival;
-  LinePts g;
-  group_line(0xFFFFFFFFu, f, g);
+    return (__int128)((int64_t)(val << sh64) >> sh64);
+  }
+  return (__int128)ival;
+}
+
+// merge a window's line state into the keys of its slot not yet FAIL (lane 0);
+// returns the updated FAIL bits (warp-uniform)
+__device__ __forceinline__ uint32_t line_apply(const AnalyzeParams& P, WarpCache& wc, const LinePts& g,
+                                               uint32_t pc0, uint32_t koi0, uint32_t lf) {
+  const int lane = threadIdx.x & 31;
   const int ps = pc0 < P.sp ? (int)pc0 : -1;
   const int os = koi0 < P.so ? (int)(P.sp + koi0) : -1;
   if (lane == 0) {
@@ -885,160 +939,215 @@ __device__ __noinline__ uint32_t fast_line(const AnalyzeParams& P, WarpCache& wc
   return __shfl_sync(0xFFFFFFFFu, lf, 0);
 }
 
+// C8 for a fast window: one line state over its 32 points
+__device__ __noinline__ uint32_t fast_line(const AnalyzeParams& P, WarpCache& wc, uint64_t addr,
+                                           uint64_t val, uint32_t meta0, uint32_t pc0, uint32_t koi0, uint32_t lf) {
+  Facts f;
+  f.addr = addr;
+  f.y = line_y(val, (meta0 >> 2) & 3u, meta0 & 3u, f.pfail);
+  LinePts g;
+  group_line(0xFFFFFFFFu, f, g);
+  return line_apply(P, wc, g, pc0, koi0, lf);
+}
+
+// C8 for a run of windows that all carry the one value cy: its points (x, y(cy))
+// span [xmin, xmax], so the run is POINT or a slope-0 LINE between its extremes
+__device__ __noinline__ uint32_t const_line(const AnalyzeParams& P, WarpCache& wc, uint64_t xmin, uint64_t xmax,
+                                            uint64_t cy, uint32_t meta0, uint32_t pc0, uint32_t koi0, uint32_t lf) {
+  bool pfail;
+  const __int128 y = line_y(cy, (meta0 >> 2) & 3u, meta0 & 3u, pfail);
+  LinePts g;
+  g.state = pfail ? VE_LINE_FAIL : (xmin == xmax ? VE_LINE_POINT : VE_LINE_LINE);
+  g.px = xmin; g.qx = xmax;
+  g.py = g.qy = y;
+  return line_apply(P, wc, g, pc0, koi0, lf);
+}
+
 // Consume fast windows of access type (KIND, LG) from the ring, starting with the
 // current one (addr, val, pm; known fast).  Returns true when it stopped at a
 // window it has not consumed (left in addr, val, pm), false when the ring is empty.
+//
+// Every lane folds its own record of each window into per-lane accumulators of the
+// active slot (counts in 16-bit fields, min / max in MT); the warp reduces them
+// only when the slot is switched out, so a window costs no warp reductions.
+template <typename MT>
+__device__ __forceinline__ MT wmin(MT v) {
+  if constexpr (sizeof(MT) == 4) return __reduce_min_sync(0xFFFFFFFFu, v);
+  else return redmin64(0xFFFFFFFFu, v);
+}
+template <typename MT>
+__device__ __forceinline__ MT wmax(MT v) {
+  if constexpr (sizeof(MT) == 4) return __reduce_max_sync(0xFFFFFFFFu, v);
+  else return redmax64(0xFFFFFFFFu, v);
+}
+__device__ __forceinline__ uint32_t wsum16(uint32_t v, int hi) {
+  return __reduce_add_sync(0xFFFFFFFFu, hi ? (v >> 16) : (v & 0xFFFFu));
+}
+
 template <int KIND, int LG>
-__device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, const ObjCache& oc, SlotE* slots,
-                                         uint32_t* snext, Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm) {
-  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;   // min / max totals
-  using PT = MT;                                                                // one gathered value
+__device__ __forceinline__ bool run_fast(const AnalyzeParams& P, const ObjCache& oc, SlotE* se, bool one, bool cmode,
+                                         uint64_t cy, uint64_t& xmin, uint64_t& xmax, Ring& R, uint64_t& addr,
+                                         uint64_t& val, uint64_t& pm) {
+  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;   // min / max accumulators
   constexpr bool ISF = KIND >= 2;
   constexpr uint32_t W = 1u << LG;
-  constexpr uint32_t KL = ((uint32_t)KIND << 2) | (uint32_t)LG;
   constexpr int MB = KIND == 3 ? 7 : (LG == 1 ? 10 : LG == 2 ? 23 : 52);
+  constexpr MT MID = (MT)~0ull;                                                 // min identity
   const unsigned FULL = 0xFFFFFFFFu;
   const int lane = threadIdx.x & 31;
   const MT tmask = (MT)(P.mant_bits >= (uint32_t)MB ? ~0ull : ~((1ull << (MB - P.mant_bits)) - 1ull));
   const bool eqdef = oc.pre != 0ull;
-  uint64_t pm0 = shfl64(FULL, pm, 0);
-  // the active slot, in registers
-  uint64_t akey = ~0ull;
-  int a = 0;
-  uint32_t nwin = 0, lf = 3u, c0 = 0, c1 = 0, c2 = 0, c3 = 0, c4 = 0, c5 = 0, c6 = 0;
-  unsigned long long dn = 0;
-  MT m0 = 0, m1 = 0, m2 = 0, m3 = 0, m4 = 0, m5 = 0;
-  auto save = [&]() {
+  const uint64_t pm0 = shfl64(FULL, pm, 0);
+  const uint32_t pc0 = (uint32_t)pm0, meta0 = (uint32_t)(pm0 >> 32);
+  const bool st = meta_store(meta0);
+  const unsigned long long dn = se->dense;
+  const uint32_t tag = (pc0 << 16) | (oc.id & 0xFFFFu);
+  // per-lane accumulators
+  uint32_t nwin = 0;
+  uint32_t cz = 0, cf0 = 0, cf1 = 0, cf2 = 0;   // zero | eq_pre<<16, nan | nonint<<16, not_f16 | not_bf16<<16, not_f32
+  MT m0 = MID, m1 = 0, m2 = MID, m3 = 0, m4 = MID, m5 = 0;
+  auto save = [&]() {   // fold the accumulators into the slot and reset them
+    const uint32_t s0 = wsum16(cz, 0), s1 = wsum16(cz, 1);
+    uint32_t s2 = 0, s3 = 0, s4 = 0, s5 = 0, s6 = 0;
+    if constexpr (ISF) {
+      s2 = wsum16(cf0, 0); s3 = wsum16(cf0, 1); s4 = wsum16(cf1, 0); s5 = wsum16(cf1, 1);
+      if constexpr (LG == 3) s6 = __reduce_add_sync(FULL, cf2);
+    }
+    const MT r0 = wmin(m0), r1 = wmax(m1);
+    MT r2 = r0, r3 = r1, r4 = MID, r5 = 0;
+    if constexpr (KIND != 0) { r2 = wmin(m2); r3 = wmax(m3); }
+    if constexpr (ISF) { r4 = wmin(m4); r5 = wmax(m5); }
     __syncwarp();
     if (lane == 0) {
-      SlotE& e = slots[a];
-      e.nwin = nwin; e.lfail = lf;
-      e.sum[0] = c0; e.sum[1] = c1; e.sum[2] = c2; e.sum[3] = c3; e.sum[4] = c4; e.sum[5] = c5; e.sum[6] = c6;
-      e.mm[0] = m0; e.mm[1] = m1; e.mm[2] = m2; e.mm[3] = m3; e.mm[4] = m4; e.mm[5] = m5;
+      SlotE& e = *se;
+      e.nwin += nwin;
+      e.sum[0] += s0; e.sum[1] += s1; e.sum[2] += s2; e.sum[3] += s3; e.sum[4] += s4; e.sum[5] += s5; e.sum[6] += s6;
+      e.mm[0] = min(e.mm[0], (uint64_t)r0); e.mm[1] = max(e.mm[1], (uint64_t)r1);
+      e.mm[2] = min(e.mm[2], (uint64_t)r2); e.mm[3] = max(e.mm[3], (uint64_t)r3);
+      e.mm[4] = min(e.mm[4], (uint64_t)r4); e.mm[5] = max(e.mm[5], (uint64_t)r5);
     }
     __syncwarp();
+    cz = cf0 = cf1 = cf2 = 0;
+    m0 = MID; m1 = 0; m2 = MID; m3 = 0; m4 = MID; m5 = 0;
+    nwin = 0;
   };
-  bool newkey = true;
-  bool have_npv = false;
-  PT npv = 0;
+  // S3 gather of a window's pre-snapshot elements (a zero word when the object has
+  // no snapshot).  Software-pipelined: the next window is read from the ring and its
+  // gather issued before the current window is processed.
+  auto gather = [&](uint64_t o) -> MT { return (MT)ld_pre<LG>(eqdef ? oc.pre + o : (uint64_t)&ve_zero_word); };
+  // window i+1 read ahead: a continuing window's record is in (a1, v1) with its
+  // gather pv1 in flight; a window that does not continue is left in (a1, v1, p1)
+  auto peek = [&](uint64_t& a, uint64_t& v, uint64_t& p, uint64_t& o, MT& g, bool& c) {
+    ring_next(P, R, a, v, p);
+    o = a - oc.base;
+    bool ok = o <= oc.lim && (o & (W - 1)) == 0;
+    if constexpr (LG < 3) ok = ok && (v >> (8 * W)) == 0ull;
+    c = __all_sync(FULL, ok && p == pm0 && (!cmode || v == cy));
+#if VE_PREFETCH
+    if (c && eqdef) prefetch_l1(oc.pre + o);
+#else
+    if (c) g = gather(o);
+#endif
+  };
+  uint64_t off = addr - oc.base;
+  MT pv = gather(off);
+  uint64_t a1 = 0, v1 = 0, p1 = 0, off1 = 0;
+  MT pv1 = 0;
+  bool more1 = !one && R.left != 0u, cont1 = false;
+  if (more1) peek(a1, v1, p1, off1, pv1, cont1);
   while (true) {
-    const uint32_t pc0 = (uint32_t)pm0, meta0 = (uint32_t)(pm0 >> 32);
-    const bool st = meta_store(meta0);
-    if (newkey) {
-      const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
-      if (key != akey) {
-        if (akey != ~0ull) save();
-        a = slot_acquire(P, slots, snext, key, oc.oi, !eqdef);
-        akey = key;
-        const SlotE& e = slots[a];
-        nwin = e.nwin; lf = e.lfail; dn = e.dense;
-        c0 = e.sum[0]; c1 = e.sum[1]; c2 = e.sum[2]; c3 = e.sum[3]; c4 = e.sum[4]; c5 = e.sum[5]; c6 = e.sum[6];
-        m0 = (MT)e.mm[0]; m1 = (MT)e.mm[1]; m2 = (MT)e.mm[2]; m3 = (MT)e.mm[3]; m4 = (MT)e.mm[4]; m5 = (MT)e.mm[5];
-      }
-      newkey = false;
-    }
+    // window i+2, two windows ahead of the one processed now
+    uint64_t a2 = 0, v2 = 0, p2 = 0, off2 = 0;
+    MT pv2 = 0;
+    const bool more2 = cont1 && R.left != 0u;
+    bool cont2 = false;
+    if (more2) peek(a2, v2, p2, off2, pv2, cont2);
 
-    // S3: element, gather (unconditional: a zero word when the object has no
-    // snapshot, so nothing waits on a merge of the loaded value), written bitmap
-    const uint64_t off = addr - oc.base;
-    const uint64_t e = off >> LG;
-    // software-pipelined gather: this window's pre value was loaded during the
-    // previous window when that one could see it in the ring; the next window's
-    // is issued now, so a gather's latency overlaps a whole window of work
-    if (!have_npv) npv = (PT)ld_pre<LG>(eqdef ? oc.pre + off : (uint64_t)&ve_zero_word);
-    const PT pv = npv;
-    have_npv = false;
-    if (VE_PIPE && eqdef && R.left && (R.h == 1u || mbar_ready(R.bar, R.ph))) {
-      unsigned long long na;
-      asm volatile("ld.shared.u64 %0, [%1];" : "=l"(na) : "r"(R.o));
-      const uint64_t no = na - oc.base;
-      if (no <= oc.lim && (no & (W - 1)) == 0) {
-        npv = (PT)ld_pre<LG>(oc.pre + no);
-        have_npv = true;
-      }
+#if VE_PREFETCH
+    pv = gather(off);                     // prefetched into L1 two windows ago
+#endif
+#ifndef VE_EXP
+#define VE_EXP 0   // timing experiments only (wrong results): 1 stream only, 2 + gather/eq, 3 + dense counts
+#endif
+#if VE_EXP == 1
+    cz += 1u;
+#elif VE_EXP == 2
+    cz += ((MT)val == pv) ? 1u : 0u;
+#elif VE_EXP == 3
+    {
+      const bool eq = (MT)val == pv;
+      cz += eq ? 1u : 0u;
+      red_add_keep(reinterpret_cast<uint32_t*>(dn) + (off >> LG), 1u, eq && dn != 0ull);
     }
+#else
+    // element, written bitmap
+    const uint64_t e = off >> LG;
     const uint64_t word = oc.bmoff + (e >> 5);
     const uint32_t bit = 1u << ((uint32_t)e & 31u);
     if (st) bitmap_or_win(P.t.W, true, word, bit);
-
-    // C4-C7: the window's REDUX totals
-    ++nwin;
-    if constexpr (LG < 3) {
-      const uint32_t b = (uint32_t)val;
-      m0 = min(m0, __reduce_min_sync(FULL, b));
-      m1 = max(m1, __reduce_max_sync(FULL, b));
-      if constexpr (KIND == 0) {
-        m2 = m0; m3 = m1;
-      } else if constexpr (KIND == 1) {           // sext32(b) ^ 2^31
-        constexpr uint32_t sh = 32 - (8 << LG);
-        const uint32_t k = (uint32_t)(((int32_t)(b << sh)) >> sh) ^ 0x80000000u;
-        m2 = min(m2, __reduce_min_sync(FULL, k));
-        m3 = max(m3, __reduce_max_sync(FULL, k));
-      } else {
-        constexpr uint32_t SIGN = 1u << ((8 << LG) - 1);
-        constexpr uint32_t MASK = (uint32_t)((1ull << (8 << LG)) - 1ull);
-        uint32_t ff;
-        if constexpr (KIND == 2 && LG == 2) ff = fflags_f32(b);
-        else ff = fflags32<KIND, LG>(b);
-        const bool okv = !(ff & 1u);              // NaNs excluded from ord / trunc
-        const uint32_t k = (b & SIGN) ? (~b & MASK) : (b | SIGN);
-        const uint32_t t = b & tmask;
-        m2 = min(m2, __reduce_min_sync(FULL, okv ? k : 0xFFFFFFFFu));
-        m3 = max(m3, __reduce_max_sync(FULL, okv ? k : 0u));
-        m4 = min(m4, __reduce_min_sync(FULL, okv ? t : 0xFFFFFFFFu));
-        m5 = max(m5, __reduce_max_sync(FULL, okv ? t : 0u));
-        c2 += __popc(__ballot_sync(FULL, ff & 1u));
-        c3 += __popc(__ballot_sync(FULL, ff & 2u));
-        c4 += __popc(__ballot_sync(FULL, ff & 4u));
-        c5 += __popc(__ballot_sync(FULL, ff & 8u));
-      }
-    } else {
-      m0 = min(m0, redmin64(FULL, val));
-      m1 = max(m1, redmax64(FULL, val));
-      if constexpr (KIND == 0) {
-        m2 = m0; m3 = m1;
-      } else if constexpr (KIND == 1) {
-        const uint64_t k = val ^ (1ull << 63);
-        m2 = min(m2, redmin64(FULL, k));
-        m3 = max(m3, redmax64(FULL, k));
-      } else {
-        int64_t ival;
-        const uint32_t ff = float_flags(val, 2u, 3u, ival);
-        const bool okv = !(ff & 1u);
-        const uint64_t k = (val >> 63) ? ~val : (val | (1ull << 63));
-        const uint64_t t = val & tmask;
-        m2 = min(m2, redmin64(FULL, okv ? k : ~0ull));
-        m3 = max(m3, redmax64(FULL, okv ? k : 0ull));
-        m4 = min(m4, redmin64(FULL, okv ? t : ~0ull));
-        m5 = max(m5, redmax64(FULL, okv ? t : 0ull));
-        c2 += __popc(__ballot_sync(FULL, ff & 1u));
-        c3 += __popc(__ballot_sync(FULL, ff & 2u));
-        c4 += __popc(__ballot_sync(FULL, ff & 4u));
-        c5 += __popc(__ballot_sync(FULL, ff & 8u));
-        c6 += __popc(__ballot_sync(FULL, ff & 16u));
-      }
+    if (cmode) {                          // C8 of a constant run: the extreme addresses
+      xmin = addr < xmin ? addr : xmin;
+      xmax = addr > xmax ? addr : xmax;
     }
-    (void)ISF;
-    // the pre-snapshot gather is consumed only now
-    const bool eq = eqdef && (uint64_t)pv == val;
-    c0 += __popc(__ballot_sync(FULL, val == 0ull));
-    const unsigned eqm = __ballot_sync(FULL, eq);
-    c1 += __popc(eqm);
+
+    const MT b = (MT)val;
+    const bool eq = eqdef && pv == b;
+    const bool dl = dn != 0ull && eq;
+    if (dn != 0ull && __all_sync(FULL, dl)) {
+      // a dense window: every load reads its element's unchanged pre value, so its
+      // value statistics (C1 zero, C4-C7, C9) are those of the pre snapshot at the
+      // counted elements, taken once per element at report time (k_dense_flush)
+      cz += 0x10000u;
+      red_add_keep(reinterpret_cast<uint32_t*>(dn) + e, 1u, true);
+    } else {
+    // C1/C4-C7: per-lane folds of the records not counted per element
+    const bool fo = !dl;
+    m0 = min(m0, fo ? b : MID);
+    m1 = max(m1, fo ? b : (MT)0);
+    if constexpr (KIND == 1) {
+      MT k;
+      if constexpr (LG < 3) {               // sext32(b) ^ 2^31 (order-isomorphic to the 64-bit key)
+        constexpr uint32_t sh = 32 - (8 << LG);
+        k = (uint32_t)(((int32_t)(b << sh)) >> sh) ^ 0x80000000u;
+      } else {
+        k = b ^ (1ull << 63);
+      }
+      m2 = min(m2, fo ? k : MID);
+      m3 = max(m3, fo ? k : (MT)0);
+    } else if constexpr (ISF) {
+      uint32_t ff;
+      if constexpr (KIND == 2 && LG == 2) ff = fflags_f32((uint32_t)b);
+      else if constexpr (LG < 3) ff = fflags32<KIND, LG>((uint32_t)b);
+      else { int64_t ival; ff = float_flags(val, 2u, 3u, ival); }
+      ff = fo ? ff : 1u;                    // counted elements: as NaN below, then masked out
+      const bool okv = !(ff & 1u);          // NaNs excluded from ord / trunc
+      constexpr MT SIGN = (MT)1 << ((8 << LG) - 1);
+      constexpr MT MASK = (MT)((8 << LG) == 64 ? ~0ull : ((1ull << (8 << LG)) - 1ull));
+      const MT k = (b & SIGN) ? (~b & MASK) : (b | SIGN);
+      const MT t = b & tmask;
+      m2 = min(m2, okv ? k : MID);
+      m3 = max(m3, okv ? k : (MT)0);
+      m4 = min(m4, okv ? t : MID);
+      m5 = max(m5, okv ? t : (MT)0);
+      ff = fo ? ff : 0u;
+      cf0 += (ff & 1u) | ((ff & 2u) << 15);
+      cf1 += ((ff >> 2) & 1u) | ((ff & 8u) << 13);
+      if constexpr (LG == 3) cf2 += (ff >> 4) & 1u;
+    }
+    cz += (fo && b == (MT)0 ? 1u : 0u) + (eq ? 0x10000u : 0u);
+
     // C3 loaded elements; loads counted per element below get their bits from the
     // dense counters at report time
-    if (!st && dn == 0ull && eqm) bitmap_or_win(P.t.L, eq, word, bit);
-
-    // C8 line state, only while a key of the slot is not yet FAIL
-    if (lf != 3u) lf = fast_line(P, wc, addr, val, meta0, pc0, oc.id, lf);
+    if (!st && dn == 0ull) {
+      if (__any_sync(FULL, eq)) bitmap_or_win(P.t.L, eq, word, bit);
+    }
 
     // S8: exact histogram.  A load that reads an unchanged element carries that
     // element's pre value, so it is counted per element (mapped to its value at
     // report time); every other record is inserted per distinct value.
-    const bool dl = dn != 0ull && eq;
-    if (dl) red_add(reinterpret_cast<uint32_t*>(dn) + e, 1u);
-    const unsigned hm = dn != 0ull ? ~eqm : FULL;
+    red_add_keep(reinterpret_cast<uint32_t*>(dn) + e, 1u, dl);
+    const unsigned hm = __ballot_sync(FULL, !dl);
     if (hm) {
-      const uint32_t tag = (pc0 << 16) | (oc.id & 0xFFFFu);
       const int l = __ffs(hm) - 1;
       const uint64_t v0 = (LG < 3) ? (uint64_t)__shfl_sync(FULL, (uint32_t)val, l) : shfl64(FULL, val, l);
       if (__all_sync(FULL, dl || val == v0)) {
@@ -1048,22 +1157,18 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, WarpCache& wc, 
         if (lane == __ffs(vg) - 1) hist_insert(P, tag, val, __popc(vg));
       }
     }
-
-    // next window: continue while it is fast with the same access type
-    if (R.left == 0) { save(); return false; }
-    ring_next(P, R, addr, val, pm);
-    const uint64_t o2 = addr - oc.base;
-    bool ok = o2 <= oc.lim && (o2 & (W - 1)) == 0;
-    if constexpr (LG < 3) ok = ok && (val >> (8 * W)) == 0ull;
-    if (__all_sync(FULL, ok && pm == pm0)) continue;        // same pc and type: same slot
-    const uint64_t pmn = shfl64(FULL, pm, 0);
-    const uint32_t mt = (uint32_t)(pmn >> 32);
-    if (!__all_sync(FULL, ok && pm == pmn) || (mt & 15u) != KL || !meta_fast(mt, (uint32_t)pmn, P.n_pcs)) {
-      save();
-      return true;
     }
-    pm0 = pmn;
-    newkey = true;
+#endif
+    if (++nwin == 0xFFFFu) save();          // 16-bit per-lane count fields
+
+    // next window: continue while it is fast with the same key
+    if (!cont1) {
+      save();
+      if (more1) { addr = a1; val = v1; pm = p1; }
+      return more1;
+    }
+    addr = a1; val = v1; off = off1; pv = pv1;
+    a1 = a2; v1 = v2; p1 = p2; off1 = off2; pv1 = pv2; more1 = more2; cont1 = cont2;
   }
 }
 
@@ -1090,25 +1195,32 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   if (lane < NSLOT) slots[lane].key = ~0ull;
   if (lane == 0) { wc.next = 0; s_snext[warp] = 0; }
 
-  // full windows stream through the TMA ring in dynamically claimed chunks; without
-  // the ring (records not 16-byte aligned) each warp takes a static range
+  // full windows stream through the warp's TMA ring (a static contiguous range per
+  // warp); without the ring (records not 16-byte aligned) each warp takes a static
+  // range of plain loads
   const uint64_t nwin = (P.n + 31) / 32;
   const uint64_t tw = (uint64_t)gridDim.x * K1_WARPS, gw = (uint64_t)blockIdx.x * K1_WARPS + warp;
   Ring R;
-  R.left = 0;
-  R.iss = 0;
   R.dst0 = smem_u32(ve_smem + P.o_ring + (uint32_t)warp * RING * WIN_BYTES);
   R.o0 = R.o = R.dst0 + (uint32_t)lane * 24u;
-  R.bar0 = R.bar = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
-  R.h = R.ph = 0;
-  if (lane == 0 && P.nring) {   // only lane 0 issues: its src / iss / nextc are the ones that matter
+  R.bar0 = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
+  R.d = R.sw = R.ph = R.pend = 0;
+  R.left = 0;
+  if (lane == 0 && P.nring) {
     for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar0 + d * 8u, 1);
     fence_mbar_init();
-    R.nextc = atomicAdd(P.work, 1ull);
-    ring_chunk(P, R);
-    for (int d = 0; d < NSTAGE && R.iss; ++d) ring_issue_stage(P, R, (uint32_t)d);
   }
-  R.left = __shfl_sync(FULL, R.left, 0);
+  __syncwarp();
+#if VE_CLAIM
+  ring_claim(P, R);
+#else
+  {
+    const uint64_t b = gw * P.nring / tw, e = (gw + 1) * P.nring / tw;
+    R.src = P.recs + b * 32;
+    R.iss = (uint32_t)(e - b);
+  }
+#endif
+  for (int d = 0; d < NSTAGE; ++d) ring_issue_stage(P, R, (uint32_t)d);
   __syncthreads();
   ObjCache oc;
   oc.base = 0; oc.lim = 0; oc.bmoff = 0; oc.pre = 0; oc.oi = -1; oc.id = 0; oc.fastlg = 0xFFu;
@@ -1134,20 +1246,49 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       fast = __all_sync(FULL, vok && off <= oc.lim && (off & wm) == 0ull) && lg0 == oc.fastlg;
     }
     if (fast) {
+      // the window's key slot (pc, object, access type); while one of its line states
+      // is still live, windows go one at a time through the line check
+      const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
+      SlotE* se = &slots[slot_acquire(P, slots, &s_snext[warp], key, oc.oi, oc.pre == 0ull)];
+      const uint32_t lf = se->lfail;
+      // a live line state: runs of one value take the constant-run path, other windows
+      // go one at a time through the per-window line check
+      bool one = false, cm = false;
+      uint64_t cy = 0, xmin = ~0ull, xmax = 0;
+      if (lf != 3u) {
+        cy = shfl64(FULL, val, 0);
+        cm = __all_sync(FULL, val == cy);
+        one = !cm;
+      }
       // specialised on the window's access type (compile-time width / kind)
+#define VE_RF(K, L) have = run_fast<K, L>(P, oc, se, one, cm, cy, xmin, xmax, R, addr, val, pm)
       switch (meta0 & 15u) {
-        case 0: have = run_fast<0, 0>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 1: have = run_fast<0, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 2: have = run_fast<0, 2>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 3: have = run_fast<0, 3>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 4: have = run_fast<1, 0>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 5: have = run_fast<1, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 6: have = run_fast<1, 2>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 7: have = run_fast<1, 3>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 9: have = run_fast<2, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 10: have = run_fast<2, 2>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        case 11: have = run_fast<2, 3>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;
-        default: have = run_fast<3, 1>(P, wc, oc, slots, &s_snext[warp], R, addr, val, pm); break;   // 13: bfloat16
+        case 0: VE_RF(0, 0); break;
+        case 1: VE_RF(0, 1); break;
+        case 2: VE_RF(0, 2); break;
+        case 3: VE_RF(0, 3); break;
+        case 4: VE_RF(1, 0); break;
+        case 5: VE_RF(1, 1); break;
+        case 6: VE_RF(1, 2); break;
+        case 7: VE_RF(1, 3); break;
+        case 9: VE_RF(2, 1); break;
+        case 10: VE_RF(2, 2); break;
+        case 11: VE_RF(2, 3); break;
+        default: VE_RF(3, 1); break;   // 13: bfloat16
+      }
+#undef VE_RF
+      if (lf != 3u) {
+        uint32_t nlf;
+        if (one) {   // C8 for the window just consumed (still in addr / val)
+          nlf = fast_line(P, wc, addr, val, meta0, pc0, oc.id, lf);
+        } else {
+          xmin = redmin64(FULL, xmin);
+          xmax = redmax64(FULL, xmax);
+          nlf = const_line(P, wc, xmin, xmax, cy, meta0, pc0, oc.id, lf);
+        }
+        __syncwarp();
+        if (lane == 0) se->lfail = nlf;
+        __syncwarp();
       }
     } else {
       const uint32_t cnt = slow_window(P, wc, addr, val, pm, true);
@@ -1192,12 +1333,8 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
     if (S.smin[i] != ~0ull) atomic_min_u64(&P.t.mn[(uint64_t)key * NMM + fld], S.smin[i]);
     if (S.smax[i] != 0ull) atomic_max_u64(&P.t.mx[(uint64_t)key * NMM + fld], S.smax[i]);
   }
-  for (uint32_t s = tid; s < nsk; s += blockDim.x) {
-    if (S.sline[s].state != VE_LINE_EMPTY) {
-      const uint32_t key = s < P.sp ? s : P.n_pcs + (s - P.sp);
-      line_merge_locked(&P.t.line[key], line_load(S.sline[s]));
-    }
-  }
+  // line states of the shared keys: one row per CTA, folded by K2 (no global locks)
+  for (uint32_t s = tid; s < nsk; s += blockDim.x) P.t.lcta[(uint64_t)blockIdx.x * nsk + s] = S.sline[s];
   for (uint32_t i = tid; i < P.hs; i += blockDim.x) {
     if (S.shs[i].tag != EMPTY_TAG) hist_insert_global(P.t, S.shs[i].tag, S.shs[i].bits, S.shc[i]);
   }
@@ -1208,6 +1345,27 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   }
 }
 
+
+// K2: fold the per-CTA line states of every shared key (C8's (+) monoid, order-free)
+// into the key's global state.  One thread per key; runs after K1 on the same stream.
+__global__ void k_line_fold(const LineState* lcta, uint32_t grid, uint32_t nsk, uint32_t sp, uint32_t n_pcs,
+                            LineState* line) {
+  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nsk) return;
+  LinePts r;
+  r.state = VE_LINE_EMPTY;
+  r.px = r.qx = 0;
+  r.py = r.qy = 0;
+  for (uint32_t b = 0; b < grid; ++b) {
+    const LineState& x = lcta[(uint64_t)b * nsk + s];
+    if (x.state != VE_LINE_EMPTY) r = line_merge(r, line_load(x));
+  }
+  if (r.state == VE_LINE_EMPTY) return;
+  const uint32_t key = s < sp ? s : n_pcs + (s - sp);
+  LineState& g = line[key];
+  const LinePts m = line_merge(line_load(g), r);
+  line_store(g, m);
+}
 
 ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
   AnalyzeParams P;
@@ -1223,7 +1381,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.work = c->t.glob + G_WORK;
   c->records_analyzed += n;
   // shared stat rows: up to 256 keys, PCs first then object keys (incl. SHARED)
-  const uint32_t NSK_MAX = 256;
+  const uint32_t NSK_MAX = K1_NSK;
   uint32_t so = c->n_obj + 1 < 128 ? c->n_obj + 1 : 128;
   uint32_t sp = c->cfg.n_pcs < NSK_MAX - so ? c->cfg.n_pcs : NSK_MAX - so;
   so = (c->n_obj + 1 < NSK_MAX - sp) ? c->n_obj + 1 : NSK_MAX - sp;
@@ -1248,12 +1406,19 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   uint64_t windows = (n + 31) / 32;
   uint64_t blocks = (windows + K1_WARPS - 1) / K1_WARPS;
   if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+#if VE_CLAIM
   e = cudaMemsetAsync(P.work, 0, sizeof(unsigned long long), s);
-  if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze work counter");
+  if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze claim counter");
+#endif
   count_launch();
   k_analyze<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze launch");
+  const uint32_t nsk = sp + so;
+  count_launch();
+  k_line_fold<<<(nsk + 127) / 128, 128, 0, s>>>(c->t.lcta, (uint32_t)blocks, nsk, sp, c->cfg.n_pcs, c->t.line);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "k_line_fold launch");
   return VE_OK;
 }
 

@@ -561,10 +561,38 @@ constexpr int DF_THREADS = 256;
 constexpr int DF_SLOTS = 1024;
 constexpr uint64_t DF_CHUNK = 16384;
 
+// The value statistics of the counted loads (C1 n_zero, C5 flags and ord range, C4 raw
+// range, C7 truncated range) are taken here too, once per element weighted by its
+// count: a counted load's value IS the element's pre value (k_analyze skips them).
+struct DenseVal {
+  unsigned long long s[6];   // zero, nan, nonint, not_f16, not_bf16, not_f32
+  unsigned long long mn[3], mx[3];   // raw, ord, trunc
+};
+__device__ __forceinline__ unsigned long long wsum64(unsigned long long v) {
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
+  return v;
+}
+__device__ __forceinline__ unsigned long long wmin64(unsigned long long v) {
+  for (int o = 16; o; o >>= 1) { const unsigned long long w = __shfl_xor_sync(0xFFFFFFFFu, v, o); v = w < v ? w : v; }
+  return v;
+}
+__device__ __forceinline__ unsigned long long wmax64(unsigned long long v) {
+  for (int o = 16; o; o >>= 1) { const unsigned long long w = __shfl_xor_sync(0xFFFFFFFFu, v, o); v = w > v ? w : v; }
+  return v;
+}
+
 __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
-                                                           uint32_t ew, uint32_t tag, uint64_t bmoff, DevTables t) {
+                                                           uint32_t ew, uint32_t tag, uint64_t bmoff, DevTables t,
+                                                           uint32_t meta, uint32_t mant_bits, uint32_t kp, uint32_t ko) {
   __shared__ unsigned long long sbits[DF_SLOTS], scnt[DF_SLOTS];
+  __shared__ DenseVal sv;
   for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS) { sbits[i] = ~0ull; scnt[i] = 0; }
+  if (threadIdx.x < 6) sv.s[threadIdx.x] = 0;
+  if (threadIdx.x < 3) { sv.mn[threadIdx.x] = ~0ull; sv.mx[threadIdx.x] = 0; }
+  const uint32_t kind = (meta >> 2) & 3u, lg = meta & 3u;
+  DenseVal v;
+  for (int i = 0; i < 6; ++i) v.s[i] = 0;
+  for (int i = 0; i < 3; ++i) { v.mn[i] = ~0ull; v.mx[i] = 0; }
   __syncthreads();
   const uint64_t lo = blockIdx.x * DF_CHUNK, hi = lo + DF_CHUNK < n_elems ? lo + DF_CHUNK : n_elems;
   const int lane = threadIdx.x & 31;
@@ -581,6 +609,28 @@ __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint6
           bits = ew == 1 ? *p : ew == 2 ? *(const uint16_t*)p : ew == 4 ? *(const uint32_t*)p : *(const uint64_t*)p;
         } else {
           for (uint32_t i = 0; i < ew; ++i) bits |= (uint64_t)p[i] << (8 * i);
+        }
+      }
+    }
+    if (k) {
+      const uint64_t b = bits;
+      if (b == 0ull) v.s[0] += k;
+      uint32_t ff = 0;
+      if (kind >= 2u) {
+        int64_t ival;
+        ff = float_flags(b, kind, lg, ival);
+        for (int j = 0; j < 5; ++j) if (ff & (1u << j)) v.s[1 + j] += k;
+      }
+      v.mn[0] = b < v.mn[0] ? b : v.mn[0];
+      v.mx[0] = b > v.mx[0] ? b : v.mx[0];
+      if (!(ff & 1u)) {                    // NaNs excluded from ord / trunc (C5, C7)
+        const uint64_t o = ord_key(b, kind, lg);
+        v.mn[1] = o < v.mn[1] ? o : v.mn[1];
+        v.mx[1] = o > v.mx[1] ? o : v.mx[1];
+        if (kind >= 2u) {
+          const uint64_t tr = trunc_bits(b, kind, lg, mant_bits);
+          v.mn[2] = tr < v.mn[2] ? tr : v.mn[2];
+          v.mx[2] = tr > v.mx[2] ? tr : v.mx[2];
         }
       }
     }
@@ -608,9 +658,28 @@ __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint6
       }
     }
   }
+  // value statistics: warp, block, then both keys' rows (PC key kp, object key ko)
+  for (int i = 0; i < 6; ++i) {
+    const unsigned long long x = wsum64(v.s[i]);
+    if (lane == 0 && x) atomicAdd(&sv.s[i], x);
+  }
+  for (int i = 0; i < 3; ++i) {
+    const unsigned long long a = wmin64(v.mn[i]), b = wmax64(v.mx[i]);
+    if (lane == 0) { atomicMin(&sv.mn[i], a); atomicMax(&sv.mx[i], b); }
+  }
   __syncthreads();
   for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS)
     if (sbits[i] != ~0ull && scnt[i]) hist_insert_global(t, tag, sbits[i], scnt[i]);
+  if (threadIdx.x < 2) {
+    const uint64_t key = threadIdx.x ? ko : kp;
+    const int f[6] = {F_ZERO, F_NAN, F_NONINT, F_NF16, F_NBF16, F_NF32};
+    for (int i = 0; i < 6; ++i)
+      if (sv.s[i]) atomicAdd(&t.sum[key * NSUM + f[i]], sv.s[i]);
+    for (int i = 0; i < 3; ++i) {
+      if (sv.mn[i] != ~0ull) atomicMin(&t.mn[key * NMM + i], sv.mn[i]);
+      if (sv.mx[i] != 0ull) atomicMax(&t.mx[key * NMM + i], sv.mx[i]);
+    }
+  }
 }
 
 ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
@@ -622,13 +691,15 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   bool any = false;
   for (uint32_t i = 0; i < c->n_obj; ++i) {
     for (int j = 0; j < DENSE_PER_OBJ; ++j) {
-      const uint32_t pc = dpc[DENSE_PER_OBJ * i + j];
-      if (pc == DENSE_FREE || pc == DENSE_OFF) continue;
+      const uint32_t ck = dpc[DENSE_PER_OBJ * i + j];   // claim key: meta << 16 | pc
+      if (ck == DENSE_FREE || ck == DENSE_OFF) continue;
+      const uint32_t pc = ck & 0xFFFFu, meta = ck >> 16;
       const HostObject& o = c->objs[i];
       const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
       count_launch();
       k_dense_flush<<<(unsigned)blocks, DF_THREADS, 0, s>>>((uint32_t*)c->dense_pool + c->dense_off_h[DENSE_PER_OBJ * i + j],
-                                                    o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, o.bmoff, c->t);
+                                                    o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, o.bmoff, c->t,
+                                                    meta, c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id);
       any = true;
     }
   }

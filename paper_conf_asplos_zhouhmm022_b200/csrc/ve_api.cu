@@ -34,6 +34,7 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->t.mn);
   cudaFree(c->t.mx);
   cudaFree(c->t.line);
+  cudaFree(c->t.lcta);
   cudaFree(c->t.glob);
   cudaFree(c->t.W);
   cudaFree(c->t.L);
@@ -192,6 +193,7 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
             cudaMalloc(&c->t.mn, nk_max * NMM * 8) == cudaSuccess &&
             cudaMalloc(&c->t.mx, nk_max * NMM * 8) == cudaSuccess &&
             cudaMalloc(&c->t.line, nk_max * sizeof(LineState)) == cudaSuccess &&
+            cudaMalloc(&c->t.lcta, (size_t)c->num_sms * K1_NSK * sizeof(LineState)) == cudaSuccess &&
             cudaMalloc(&c->t.glob, 8 * 8) == cudaSuccess &&
             cudaMalloc(&c->t.hslot, hcap * sizeof(HSlot)) == cudaSuccess &&
             cudaMalloc(&c->t.hcount, hcap * 8) == cudaSuccess;
@@ -421,6 +423,19 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
     c->poisoned = true;
     return fail(c, VE_ERR_CAPACITY, "value histogram capacity exceeded (hist_capacity)");
   }
+  // counted loads contribute their value statistics and histogram entries first
+  const bool tm = getenv("VE_TIMING") != nullptr;
+  auto t0 = std::chrono::steady_clock::now();
+  if (!c->hist_merged) {
+    ve_status st = dense_flush(c, 0);
+    if (st != VE_OK) return st;
+    if (tm) {
+      cudaDeviceSynchronize();
+      fprintf(stderr, "[ve] dense_flush %.3f ms\n",
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+      t0 = std::chrono::steady_clock::now();
+    }
+  }
   const uint32_t nk = c->n_keys, K = c->cfg.topk;
   std::vector<uint64_t> sum((size_t)nk * NSUM), mn((size_t)nk * NMM), mx((size_t)nk * NMM);
   std::vector<LineState> line(nk);
@@ -440,16 +455,6 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
     nd = c->merged_ndistinct;
     r->top = c->merged_topk;
   } else {
-    const bool tm = getenv("VE_TIMING") != nullptr;
-    auto t0 = std::chrono::steady_clock::now();
-    st = dense_flush(c, 0);
-    if (st != VE_OK) { delete r; return st; }
-    if (tm) {
-      cudaDeviceSynchronize();
-      fprintf(stderr, "[ve] dense_flush %.3f ms\n",
-              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
-      t0 = std::chrono::steady_clock::now();
-    }
     st = finalize_hist(c, 0, nd, r->top);
     if (tm) {
       cudaDeviceSynchronize();

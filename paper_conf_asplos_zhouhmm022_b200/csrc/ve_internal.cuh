@@ -28,6 +28,7 @@ enum : int { M_RAW = 0, M_ORD = 1, M_TRUNC = 2 };
 constexpr uint32_t EMPTY_TAG = 0xFFFFFFFFu;  // histogram slot free
 constexpr uint32_t KO_NONE = 0xFFFFu;        // record maps to no object key
 constexpr int WARP = 32;
+constexpr uint32_t K1_NSK = 256;              // K1 keys with shared-memory rows (PCs first, then objects)
 
 // line state of C8 / the (+) monoid of DESIGN.md 3.3; y is signed 128-bit
 struct __align__(16) LineState {
@@ -54,6 +55,7 @@ struct DevTables {
   unsigned long long* mn;   // [n_keys][NMM]
   unsigned long long* mx;   // [n_keys][NMM]
   LineState* line;          // [n_keys]
+  LineState* lcta;          // [grid][K1_NSK]: per-CTA line states of K1's shared keys, folded by K2
   unsigned long long* glob; // [8]: n_records, n_invalid, n_unmapped, overflow
   uint32_t* W;              // written-element bitmaps (all objects)
   uint32_t* L;              // eq_pre-load start-element bitmaps
@@ -335,23 +337,17 @@ __device__ __forceinline__ void ld128_volatile(const void* p, uint64_t& lo, uint
 }
 
 // Insert (tag, bits) += cnt into the global exact histogram; false on overflow.
+// CAS first (an empty slot is all-ones; an occupied one has pad 0): one L2 round
+// trip claims a free slot or returns the occupant, so a probe never needs a
+// separate read; the count update is a fire-and-forget reduction.
 __device__ __forceinline__ bool hist_insert_global(const DevTables& t, uint32_t tag, uint64_t bits,
                                                    unsigned long long cnt) {
   uint64_t h = hist_hash(tag, bits) & t.hmask;
   for (uint64_t probe = 0; probe <= t.hmask; ++probe) {
     HSlot* s = &t.hslot[h];
-    uint64_t lo, hi;
-    ld128_volatile(s, lo, hi);
-    uint32_t stag = (uint32_t)hi;
-    if (stag == EMPTY_TAG) {
-      uint64_t olo, ohi;
-      cas128_global(s, lo, hi, bits, (uint64_t)tag, olo, ohi);
-      if ((uint32_t)ohi == EMPTY_TAG || (olo == bits && (uint32_t)ohi == tag)) {
-        atomicAdd(&t.hcount[h], cnt);
-        return true;
-      }
-      if (olo == bits && (uint32_t)ohi == tag) { atomicAdd(&t.hcount[h], cnt); return true; }
-    } else if (stag == tag && lo == bits) {
+    uint64_t olo, ohi;
+    cas128_global(s, ~0ull, ~0ull, bits, (uint64_t)tag, olo, ohi);
+    if ((olo == ~0ull && ohi == ~0ull) || (olo == bits && ohi == (uint64_t)tag)) {
       atomicAdd(&t.hcount[h], cnt);
       return true;
     }

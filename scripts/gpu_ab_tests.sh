@@ -1,0 +1,5 @@
+#!/bin/bash
+# parity tests of the default build, then A/B timing of build/libve_*.so
+cd "${GRAFT_REPO_ROOT:-.}"; mkdir -p gpurun_out
+timeout 900 python -m pytest tests/ -x -q -m gpu ${PYTEST_ARGS} > gpurun_out/gpu_tests.log 2>&1; echo "exit $?" >> gpurun_out/gpu_tests.log
+bash scripts/ab.sh
