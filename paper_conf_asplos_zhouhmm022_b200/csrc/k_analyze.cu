@@ -35,7 +35,7 @@ namespace ve {
 constexpr int K1_THREADS = VE_K1_THREADS;  // 16 warps x 128 registers
 constexpr int K1_WARPS = K1_THREADS / 32;
 #ifndef VE_RING
-#define VE_RING 6
+#define VE_RING 8
 #endif
 constexpr int RING = VE_RING;                // record windows per warp ring (2 stages)
 constexpr uint32_t WIN_BYTES = 32 * sizeof(ve_record);
@@ -534,7 +534,7 @@ struct Rec {
 // per-window broadcast is needed.  Records are read once: the copies carry an
 // L2 evict-first policy so the stream does not push snapshots and counters out.
 #ifndef VE_STAGE_WIN
-#define VE_STAGE_WIN 3
+#define VE_STAGE_WIN 4
 #endif
 constexpr int STAGE_WIN = VE_STAGE_WIN;
 constexpr int NSTAGE = RING / STAGE_WIN;
@@ -608,7 +608,7 @@ __device__ __forceinline__ void ring_issue_pred(bool on, uint32_t dst, const voi
 // (balanced finish), else each warp streams one static contiguous range.
 static_assert(NSTAGE * STAGE_WIN == RING, "whole stages");
 #ifndef VE_CLAIM
-#define VE_CLAIM 1
+#define VE_CLAIM 0
 #endif
 constexpr uint32_t CHUNK = 32 * STAGE_WIN;   // windows per claim (whole stages)
 struct Ring {
@@ -622,15 +622,21 @@ struct Ring {
   uint32_t pend;          // stage + 1 to refill at the next read, 0 = none
 };
 
-// claim the next chunk of full windows (all lanes; lane 0 does the atomic)
+// claim the next chunk of full windows (all lanes; lane 0 does the atomic).  Guided:
+// CHUNK-window chunks cover the first 7/8 of the trace, then chunks of one stage, so
+// the warps finish together even where windows differ much in cost.
+constexpr uint32_t CHUNK_TAIL = STAGE_WIN;
 __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
   unsigned long long c = 0;
   if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
   c = __shfl_sync(0xFFFFFFFFu, c, 0);
-  const uint64_t w0 = (uint64_t)c * CHUNK;
+  const uint64_t nbig = (P.nring - P.nring / 8) / CHUNK;
+  uint64_t w0, len;
+  if (c < nbig) { w0 = (uint64_t)c * CHUNK; len = CHUNK; }
+  else { w0 = nbig * CHUNK + (uint64_t)(c - nbig) * CHUNK_TAIL; len = CHUNK_TAIL; }
   if (w0 < P.nring) {
     R.src = P.recs + w0 * 32;
-    R.iss = (uint32_t)(P.nring - w0 < CHUNK ? P.nring - w0 : CHUNK);
+    R.iss = (uint32_t)(P.nring - w0 < len ? P.nring - w0 : len);
   } else {
     R.iss = 0;
   }
@@ -669,6 +675,32 @@ __device__ __forceinline__ void ring_next(const AnalyzeParams& P, Ring& R, uint6
     R.pend = R.iss ? d + 1u : 0u;
     if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.o = R.o0; R.ph ^= 1u; }
   }
+}
+
+// whole-stage access (the dense batch path): refill a pending stage, wait for the
+// current stage (the next read is its first window), read window j of it, and
+// consume the stage
+__device__ __forceinline__ bool ring_stage_full(const Ring& R) { return R.sw == 0u && R.left >= (uint32_t)STAGE_WIN; }
+__device__ __forceinline__ void ring_stage_wait(const AnalyzeParams& P, Ring& R) {
+  if (R.pend) {
+    __syncwarp();
+    ring_issue_stage(P, R, R.pend - 1u);
+    R.pend = 0;
+  }
+  ring_wait(R.bar0 + R.d * 8u, R.ph);
+}
+__device__ __forceinline__ void ring_stage_read(const Ring& R, uint32_t j, uint64_t& addr, uint64_t& val,
+                                                uint64_t& pm) {
+  asm volatile("ld.shared.u64 %0, [%3];\n\tld.shared.u64 %1, [%3+8];\n\tld.shared.u64 %2, [%3+16];"
+               : "=l"(addr), "=l"(val), "=l"(pm)
+               : "r"(R.o + j * WIN_BYTES)
+               : "memory");
+}
+__device__ __forceinline__ void ring_stage_consume(Ring& R) {
+  R.left -= STAGE_WIN;
+  R.o += STAGE_WIN * WIN_BYTES;
+  R.pend = R.iss ? R.d + 1u : 0u;
+  if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.o = R.o0; R.ph ^= 1u; }
 }
 
 __device__ __forceinline__ Rec load_rec(const AnalyzeParams& P, uint64_t w, uint64_t wend, int lane) {
@@ -961,6 +993,81 @@ __device__ __noinline__ uint32_t const_line(const AnalyzeParams& P, WarpCache& w
   g.px = xmin; g.qx = xmax;
   g.py = g.qy = y;
   return line_apply(P, wc, g, pc0, koi0, lf);
+}
+
+// Dense batch path for a key whose loads are counted per element (C3 / S8 dense
+// counters): such a window's statistics are its record count, its eq_pre count and
+// one counter increment per element -- every value statistic is taken from the
+// pre snapshot at report time (k_dense_flush).  Whole ring stages are consumed at
+// once (one barrier wait, STAGE_WIN gathers in flight together).  Stops at a key
+// change (returns true, window left in addr / val / pm), at the end of the ring
+// (false), or at a window that is not entirely dense: then nd is set and that
+// window, unprocessed, is left in addr / val / pm for run_fast.
+template <int LG>
+__device__ __forceinline__ bool run_dense(const AnalyzeParams& P, const ObjCache& oc, SlotE* se, Ring& R,
+                                          uint64_t& addr, uint64_t& val, uint64_t& pm, bool& nd) {
+  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;
+  constexpr uint32_t W = 1u << LG;
+  const unsigned FULL = 0xFFFFFFFFu;
+  const uint64_t pm0 = shfl64(FULL, pm, 0);
+  uint32_t* const dn = reinterpret_cast<uint32_t*>(se->dense);
+  uint32_t ndw = 0;                                  // dense windows processed
+  auto fits = [&](uint64_t a, uint64_t v, uint64_t p, uint64_t& o) -> bool {
+    o = a - oc.base;
+    bool ok = o <= oc.lim && (o & (W - 1)) == 0 && p == pm0;
+    if constexpr (LG < 3) ok = ok && (v >> (8 * W)) == 0ull;
+    return ok;
+  };
+  auto done = [&]() {
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) { se->nwin += ndw; se->sum[1] += ndw * 32u; }
+    __syncwarp();
+  };
+  nd = false;
+  // the current window (already read from the ring)
+  {
+    const uint64_t o = addr - oc.base;
+    const MT pv = (MT)ld_pre<LG>(oc.pre + o);
+    if (!__all_sync(FULL, pv == (MT)val)) { nd = true; done(); return true; }
+    red_add_keep(dn + (o >> LG), 1u, true);
+    ++ndw;
+  }
+  while (true) {
+    if (ring_stage_full(R)) {
+      ring_stage_wait(P, R);
+      uint64_t a[STAGE_WIN], v[STAGE_WIN], p[STAGE_WIN], o[STAGE_WIN];
+      bool ok = true;
+#pragma unroll
+      for (int j = 0; j < STAGE_WIN; ++j) {
+        ring_stage_read(R, (uint32_t)j, a[j], v[j], p[j]);
+        ok = ok && fits(a[j], v[j], p[j], o[j]);
+      }
+      if (__all_sync(FULL, ok)) {
+        MT pv[STAGE_WIN];
+#pragma unroll
+        for (int j = 0; j < STAGE_WIN; ++j) pv[j] = (MT)ld_pre<LG>(oc.pre + o[j]);
+        bool eq = true;
+#pragma unroll
+        for (int j = 0; j < STAGE_WIN; ++j) eq = eq && pv[j] == (MT)v[j];
+        if (__all_sync(FULL, eq)) {
+#pragma unroll
+          for (int j = 0; j < STAGE_WIN; ++j) red_add_keep(dn + (o[j] >> LG), 1u, true);
+          ndw += STAGE_WIN;
+          ring_stage_consume(R);
+          continue;
+        }
+      }
+      // not a whole dense stage of this key: go on window by window
+    }
+    if (R.left == 0u) { done(); return false; }
+    ring_next(P, R, addr, val, pm);
+    uint64_t o;
+    if (!__all_sync(FULL, fits(addr, val, pm, o))) { done(); return true; }
+    const MT pv = (MT)ld_pre<LG>(oc.pre + o);
+    if (!__all_sync(FULL, pv == (MT)val)) { nd = true; done(); return true; }
+    red_add_keep(dn + (o >> LG), 1u, true);
+    ++ndw;
+  }
 }
 
 // Consume fast windows of access type (KIND, LG) from the ring, starting with the
@@ -1260,6 +1367,17 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
         cm = __all_sync(FULL, val == cy);
         one = !cm;
       }
+      // dense loads of a key without live line state: the stage-batched dense path
+      bool nd = true;
+      if (!one && !cm && se->dense != 0ull) {
+        switch (meta0 & 3u) {
+          case 0: have = run_dense<0>(P, oc, se, R, addr, val, pm, nd); break;
+          case 1: have = run_dense<1>(P, oc, se, R, addr, val, pm, nd); break;
+          case 2: have = run_dense<2>(P, oc, se, R, addr, val, pm, nd); break;
+          default: have = run_dense<3>(P, oc, se, R, addr, val, pm, nd); break;
+        }
+      }
+      if (nd) {
       // specialised on the window's access type (compile-time width / kind)
 #define VE_RF(K, L) have = run_fast<K, L>(P, oc, se, one, cm, cy, xmin, xmax, R, addr, val, pm)
       switch (meta0 & 15u) {
@@ -1277,6 +1395,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
         default: VE_RF(3, 1); break;   // 13: bfloat16
       }
 #undef VE_RF
+      }
       if (lf != 3u) {
         uint32_t nlf;
         if (one) {   // C8 for the window just consumed (still in addr / val)
@@ -1347,24 +1466,35 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
 
 
 // K2: fold the per-CTA line states of every shared key (C8's (+) monoid, order-free)
-// into the key's global state.  One thread per key; runs after K1 on the same stream.
-__global__ void k_line_fold(const LineState* lcta, uint32_t grid, uint32_t nsk, uint32_t sp, uint32_t n_pcs,
-                            LineState* line) {
-  const uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
-  if (s >= nsk) return;
+// into the key's global state.  One block per key, a shared-memory tree over the CTAs.
+constexpr int LF_THREADS = 256;
+__global__ void __launch_bounds__(LF_THREADS) k_line_fold(const LineState* lcta, uint32_t grid, uint32_t nsk,
+                                                          uint32_t sp, uint32_t n_pcs, LineState* line) {
+  __shared__ LineState st[LF_THREADS];
+  const uint32_t s = blockIdx.x, t = threadIdx.x;
   LinePts r;
   r.state = VE_LINE_EMPTY;
   r.px = r.qx = 0;
   r.py = r.qy = 0;
-  for (uint32_t b = 0; b < grid; ++b) {
+  for (uint32_t b = t; b < grid; b += LF_THREADS) {
     const LineState& x = lcta[(uint64_t)b * nsk + s];
     if (x.state != VE_LINE_EMPTY) r = line_merge(r, line_load(x));
   }
-  if (r.state == VE_LINE_EMPTY) return;
-  const uint32_t key = s < sp ? s : n_pcs + (s - sp);
-  LineState& g = line[key];
-  const LinePts m = line_merge(line_load(g), r);
-  line_store(g, m);
+  line_store(st[t], r);
+  __syncthreads();
+  for (uint32_t h = LF_THREADS / 2; h > 0; h >>= 1) {
+    if (t < h && st[t + h].state != VE_LINE_EMPTY) {
+      const LinePts m = line_merge(line_load(st[t]), line_load(st[t + h]));
+      line_store(st[t], m);
+    }
+    __syncthreads();
+  }
+  if (t == 0 && st[0].state != VE_LINE_EMPTY) {
+    const uint32_t key = s < sp ? s : n_pcs + (s - sp);
+    LineState& g = line[key];
+    const LinePts m = line_merge(line_load(g), line_load(st[0]));
+    line_store(g, m);
+  }
 }
 
 ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
@@ -1416,7 +1546,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze launch");
   const uint32_t nsk = sp + so;
   count_launch();
-  k_line_fold<<<(nsk + 127) / 128, 128, 0, s>>>(c->t.lcta, (uint32_t)blocks, nsk, sp, c->cfg.n_pcs, c->t.line);
+  k_line_fold<<<nsk, LF_THREADS, 0, s>>>(c->t.lcta, (uint32_t)blocks, nsk, sp, c->cfg.n_pcs, c->t.line);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_line_fold launch");
   return VE_OK;

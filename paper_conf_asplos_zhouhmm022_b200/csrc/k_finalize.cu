@@ -371,41 +371,154 @@ ve_status select_topk(ve_ctx* c, cudaStream_t s, uint64_t* gb[2], uint64_t* gc[2
 // view table.
 constexpr uint32_t TAG_CAP = 1u << 16;
 
+// Block-local key counters in shared memory: a block scans one contiguous chunk of
+// the table and touches each hot global counter once (same-address global atomics
+// from every warp serialise in L2).  Keys that do not fit the shared table fall
+// back to warp-aggregated global atomics.
+constexpr int BK_SLOTS = 512;
+struct BlockKeys {
+  uint32_t key[BK_SLOTS];
+  unsigned long long cnt[BK_SLOTS];
+  unsigned long long base[BK_SLOTS];
+};
+__device__ __forceinline__ void bk_init(BlockKeys& B) {
+  for (int i = threadIdx.x; i < BK_SLOTS; i += blockDim.x) { B.key[i] = EMPTY_TAG; B.cnt[i] = 0; B.base[i] = 0; }
+}
+// slot of key in B (claimed if absent), -1 when the table is full
+__device__ __forceinline__ int bk_slot(BlockKeys& B, uint32_t key) {
+  uint32_t h = (uint32_t)mix64(key) & (BK_SLOTS - 1);
+  for (int p = 0; p < 32; ++p) {
+    uint32_t old = *(volatile uint32_t*)&B.key[h];
+    if (old == EMPTY_TAG) old = atomicCAS(&B.key[h], EMPTY_TAG, key);
+    if (old == EMPTY_TAG || old == key) return (int)h;
+    h = (h + 1) & (BK_SLOTS - 1);
+  }
+  return -1;
+}
+// warp-aggregated add of 1 per active lane to B[key]; returns the lane's slot (or -1)
+__device__ __forceinline__ int bk_add(BlockKeys& B, bool active, uint32_t key) {
+  const unsigned am = __ballot_sync(0xFFFFFFFFu, active);
+  int sl = -1;
+  if (active) {
+    const unsigned g = __match_any_sync(am, key);
+    const int lead = __ffs(g) - 1, lane = threadIdx.x & 31;
+    if (lane == lead) {
+      sl = bk_slot(B, key);
+      if (sl >= 0) atomicAdd(&B.cnt[sl], (unsigned long long)__popc(g));
+    }
+    sl = __shfl_sync(g, sl, lead);
+  }
+  return sl;
+}
+__device__ __forceinline__ void block_chunk(uint64_t n, uint64_t& lo, uint64_t& hi) {
+  const uint64_t per = (n + gridDim.x - 1) / gridDim.x;
+  lo = (uint64_t)blockIdx.x * per;
+  hi = lo + per < n ? lo + per : n;
+  if (lo > hi) lo = hi;
+}
+
 __global__ void k_tagscan(const HSlot* hs, uint64_t cap, uint32_t* tags, unsigned long long* tcnt,
                           unsigned long long* ovf) {
-  VE_WARP_LOOP(i, cap) {
-    const uint32_t tag = i < cap ? hs[i].tag : EMPTY_TAG;
+  __shared__ BlockKeys B;
+  bk_init(B);
+  __syncthreads();
+  uint64_t lo, hi;
+  block_chunk(cap, lo, hi);
+  for (uint64_t b = lo; b < hi; b += blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
+    const bool act = tag != EMPTY_TAG;
+    const int sl = bk_add(B, act, tag);
+    if (act && sl < 0) {   // shared table full: count this entry globally
+      uint32_t h = (uint32_t)mix64(tag) & (TAG_CAP - 1);
+      bool done = false;
+      for (int p = 0; p < 64 && !done; ++p) {
+        uint32_t old = *(volatile uint32_t*)&tags[h];
+        if (old == EMPTY_TAG) old = atomicCAS(&tags[h], EMPTY_TAG, tag);
+        if (old == EMPTY_TAG || old == tag) done = true;
+        else h = (h + 1) & (TAG_CAP - 1);
+      }
+      if (done) atomicAdd(&tcnt[h], 1ull);
+      else atomicExch(ovf, 1ull);
+    }
+  }
+  __syncthreads();
+  for (int j = threadIdx.x; j < BK_SLOTS; j += blockDim.x) {
+    const uint32_t tag = B.key[j];
+    if (tag == EMPTY_TAG || !B.cnt[j]) continue;
     uint32_t h = (uint32_t)mix64(tag) & (TAG_CAP - 1);
-    bool done = tag == EMPTY_TAG;
+    bool done = false;
     for (int p = 0; p < 64 && !done; ++p) {
-      uint32_t old = *(volatile uint32_t*)&tags[h];            // read first: the hot tags are already in
+      uint32_t old = *(volatile uint32_t*)&tags[h];
       if (old == EMPTY_TAG) old = atomicCAS(&tags[h], EMPTY_TAG, tag);
       if (old == EMPTY_TAG || old == tag) done = true;
       else h = (h + 1) & (TAG_CAP - 1);
     }
-    if (!done) atomicExch(ovf, 1ull);
-    const bool act = tag != EMPTY_TAG && done;
-    warp_count(&tcnt[act ? h : 0], act, h);
+    if (done) atomicAdd(&tcnt[h], B.cnt[j]);
+    else atomicExch(ovf, 1ull);
   }
 }
 
+// Direct keys' entries are written to their segment at positions reserved per block
+// (count pass, one global reservation per key, scatter pass); the other keys'
+// entries are aggregated in the view table.
 __global__ void k_emit(const HSlot* hs, const unsigned long long* hc, uint64_t cap, uint32_t n_pcs,
                        const uint8_t* direct, const unsigned long long* off, unsigned long long* cur, uint64_t* gb,
                        uint64_t* gc, HSlot* vs, unsigned long long* vc, uint64_t vmask, unsigned long long* ovf) {
-  VE_WARP_LOOP(i, cap) {
-    const uint32_t tag = i < cap ? hs[i].tag : EMPTY_TAG;
+  __shared__ BlockKeys B;
+  bk_init(B);
+  __syncthreads();
+  uint64_t lo, hi;
+  block_chunk(cap, lo, hi);
+  auto key_of = [&](uint32_t tag, int side, bool occ, bool& act, bool& dir) -> uint32_t {
+    const uint32_t koi = tag & 0xFFFFu;
+    act = occ && !(side == 1 && koi == KO_NONE);
+    const uint32_t key = act ? (side == 0 ? (tag >> 16) : n_pcs + koi) : 0;
+    dir = act && direct[key];
+    return key;
+  };
+  // pass 1: per-key entry counts of the chunk
+  for (uint64_t b = lo; b < hi; b += blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
+    for (int side = 0; side < 2; ++side) {
+      bool act, dir;
+      const uint32_t key = key_of(tag, side, tag != EMPTY_TAG, act, dir);
+      bk_add(B, dir, key);
+    }
+  }
+  __syncthreads();
+  // one reservation per key; the counts become the block's cursors
+  for (int j = threadIdx.x; j < BK_SLOTS; j += blockDim.x) {
+    const uint32_t key = B.key[j];
+    if (key != EMPTY_TAG && B.cnt[j]) B.base[j] = off[key] + atomicAdd(&cur[key], B.cnt[j]);
+    B.cnt[j] = 0;
+  }
+  __syncthreads();
+  // pass 2: scatter (entries of keys that missed the shared table reserve globally)
+  for (uint64_t b = lo; b < hi; b += blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
     const bool occ = tag != EMPTY_TAG;
     const uint64_t bits = occ ? hs[i].bits : 0;
     const unsigned long long cnt = occ ? hc[i] : 0;
-    const uint32_t koi = tag & 0xFFFFu;
     for (int side = 0; side < 2; ++side) {
-      const bool act = occ && !(side == 1 && koi == KO_NONE);
-      const uint32_t key = act ? (side == 0 ? (tag >> 16) : n_pcs + koi) : 0;
-      const bool dir = act && direct[key];
-      const unsigned long long p = warp_count(&cur[key], dir, key);
+      bool act, dir;
+      const uint32_t key = key_of(tag, side, occ, act, dir);
+      const int lane = threadIdx.x & 31;
+      const unsigned am = __ballot_sync(0xFFFFFFFFu, dir);
       if (dir) {
-        gb[off[key] + p] = bits;
-        gc[off[key] + p] = cnt;
+        const unsigned g = __match_any_sync(am, key);
+        const int lead = __ffs(g) - 1;
+        unsigned long long p = 0;
+        if (lane == lead) {
+          const int sl = bk_slot(B, key);
+          p = sl >= 0 ? B.base[sl] + atomicAdd(&B.cnt[sl], (unsigned long long)__popc(g))
+                      : off[key] + atomicAdd(&cur[key], (unsigned long long)__popc(g));
+        }
+        p = __shfl_sync(g, p, lead) + __popc(g & ((1u << lane) - 1u));
+        gb[p] = bits;
+        gc[p] = cnt;
       } else if (act) {
         vinsert(vs, vc, vmask, ovf, key, bits, cnt);
       }
@@ -559,7 +672,7 @@ ve_status finalize_hist_views(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& 
 // shared table) so runs of equal values (zero-filled regions) cost one global insert.
 constexpr int DF_THREADS = 256;
 constexpr int DF_SLOTS = 1024;
-constexpr uint64_t DF_CHUNK = 16384;
+constexpr uint64_t DF_CHUNK = 1024;    // elements per block: many blocks keep the global inserts in flight
 
 // The value statistics of the counted loads (C1 n_zero, C5 flags and ord range, C4 raw
 // range, C7 truncated range) are taken here too, once per element weighted by its
