@@ -42,19 +42,12 @@ static cudaError_t scratch_need(ve_ctx* c, size_t bytes) {
 __device__ __forceinline__ bool vinsert(HSlot* slots, unsigned long long* counts, uint64_t mask,
                                         unsigned long long* overflow, uint32_t tag, uint64_t bits,
                                         unsigned long long cnt) {
+  // CAS first (empty slots are all-ones, occupied ones have pad 0): one round trip per probe
   uint64_t h = hist_hash(tag, bits) & mask;
   for (uint64_t probe = 0; probe <= mask; ++probe) {
-    HSlot* s = &slots[h];
-    uint64_t lo, hi;
-    ld128_volatile(s, lo, hi);
-    if ((uint32_t)hi == EMPTY_TAG) {
-      uint64_t olo, ohi;
-      cas128_global(s, lo, hi, bits, (uint64_t)tag, olo, ohi);
-      if (((uint32_t)ohi == EMPTY_TAG && olo == lo) || ((uint32_t)ohi == tag && olo == bits)) {
-        atomicAdd(&counts[h], cnt);
-        return true;
-      }
-    } else if ((uint32_t)hi == tag && lo == bits) {
+    uint64_t olo, ohi;
+    cas128_global(&slots[h], ~0ull, ~0ull, bits, (uint64_t)tag, olo, ohi);
+    if ((olo == ~0ull && ohi == ~0ull) || (olo == bits && ohi == (uint64_t)tag)) {
       atomicAdd(&counts[h], cnt);
       return true;
     }
@@ -418,16 +411,20 @@ __device__ __forceinline__ void block_chunk(uint64_t n, uint64_t& lo, uint64_t& 
 }
 
 __global__ void k_tagscan(const HSlot* hs, uint64_t cap, uint32_t* tags, unsigned long long* tcnt,
-                          unsigned long long* ovf) {
+                          unsigned long long* ovf, uint32_t* occ_idx, unsigned long long* n_occ) {
   __shared__ BlockKeys B;
+  __shared__ unsigned long long s_cur;
   bk_init(B);
+  if (threadIdx.x == 0) s_cur = 0;
   __syncthreads();
   uint64_t lo, hi;
   block_chunk(cap, lo, hi);
+  unsigned long long my = 0;   // occupied slots seen by this thread
   for (uint64_t b = lo; b < hi; b += blockDim.x) {
     const uint64_t i = b + threadIdx.x;
     const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
     const bool act = tag != EMPTY_TAG;
+    my += act ? 1u : 0u;
     const int sl = bk_add(B, act, tag);
     if (act && sl < 0) {   // shared table full: count this entry globally
       uint32_t h = (uint32_t)mix64(tag) & (TAG_CAP - 1);
@@ -457,19 +454,42 @@ __global__ void k_tagscan(const HSlot* hs, uint64_t cap, uint32_t* tags, unsigne
     if (done) atomicAdd(&tcnt[h], B.cnt[j]);
     else atomicExch(ovf, 1ull);
   }
+  // the chunk's occupied slots, compacted (one reservation per block; order within
+  // the block's range is irrelevant)
+  my = __reduce_add_sync(0xFFFFFFFFu, (unsigned)my);
+  if ((threadIdx.x & 31) == 0 && my) atomicAdd(&s_cur, my);
+  __syncthreads();
+  const unsigned long long nb = s_cur;
+  __syncthreads();
+  if (threadIdx.x == 0) s_cur = nb ? atomicAdd(n_occ, nb) : 0;
+  __syncthreads();
+  const unsigned long long base = s_cur;
+  __syncthreads();
+  if (threadIdx.x == 0) s_cur = 0;
+  __syncthreads();
+  for (uint64_t b = lo; b < hi && nb; b += blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    const bool occ = i < hi && hs[i].tag != EMPTY_TAG;
+    const unsigned m = __ballot_sync(0xFFFFFFFFu, occ);
+    unsigned long long wb = 0;
+    if ((threadIdx.x & 31) == 0 && m) wb = atomicAdd(&s_cur, (unsigned long long)__popc(m));
+    wb = __shfl_sync(0xFFFFFFFFu, wb, 0);
+    if (occ) occ_idx[base + wb + __popc(m & ((1u << (threadIdx.x & 31)) - 1u))] = (uint32_t)i;
+  }
 }
 
 // Direct keys' entries are written to their segment at positions reserved per block
 // (count pass, one global reservation per key, scatter pass); the other keys'
 // entries are aggregated in the view table.
-__global__ void k_emit(const HSlot* hs, const unsigned long long* hc, uint64_t cap, uint32_t n_pcs,
-                       const uint8_t* direct, const unsigned long long* off, unsigned long long* cur, uint64_t* gb,
-                       uint64_t* gc, HSlot* vs, unsigned long long* vc, uint64_t vmask, unsigned long long* ovf) {
+__global__ void k_emit(const HSlot* hs, const unsigned long long* hc, const uint32_t* occ_idx,
+                       const unsigned long long* n_occ, uint32_t n_pcs, const uint8_t* direct,
+                       const unsigned long long* off, unsigned long long* cur, uint64_t* gb, uint64_t* gc, HSlot* vs,
+                       unsigned long long* vc, uint64_t vmask, unsigned long long* ovf) {
   __shared__ BlockKeys B;
   bk_init(B);
   __syncthreads();
   uint64_t lo, hi;
-  block_chunk(cap, lo, hi);
+  block_chunk(*n_occ, lo, hi);
   auto key_of = [&](uint32_t tag, int side, bool occ, bool& act, bool& dir) -> uint32_t {
     const uint32_t koi = tag & 0xFFFFu;
     act = occ && !(side == 1 && koi == KO_NONE);
@@ -477,10 +497,11 @@ __global__ void k_emit(const HSlot* hs, const unsigned long long* hc, uint64_t c
     dir = act && direct[key];
     return key;
   };
-  // pass 1: per-key entry counts of the chunk
+  // pass 1: per-key entry counts of the chunk (of the occupied-slot list)
   for (uint64_t b = lo; b < hi; b += blockDim.x) {
-    const uint64_t i = b + threadIdx.x;
-    const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
+    const uint64_t j = b + threadIdx.x;
+    const uint64_t i = j < hi ? occ_idx[j] : 0;
+    const uint32_t tag = j < hi ? hs[i].tag : EMPTY_TAG;
     for (int side = 0; side < 2; ++side) {
       bool act, dir;
       const uint32_t key = key_of(tag, side, tag != EMPTY_TAG, act, dir);
@@ -497,8 +518,9 @@ __global__ void k_emit(const HSlot* hs, const unsigned long long* hc, uint64_t c
   __syncthreads();
   // pass 2: scatter (entries of keys that missed the shared table reserve globally)
   for (uint64_t b = lo; b < hi; b += blockDim.x) {
-    const uint64_t i = b + threadIdx.x;
-    const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
+    const uint64_t j = b + threadIdx.x;
+    const uint64_t i = j < hi ? occ_idx[j] : 0;
+    const uint32_t tag = j < hi ? hs[i].tag : EMPTY_TAG;
     const bool occ = tag != EMPTY_TAG;
     const uint64_t bits = occ ? hs[i].bits : 0;
     const unsigned long long cnt = occ ? hc[i] : 0;
@@ -526,6 +548,22 @@ __global__ void k_emit(const HSlot* hs, const unsigned long long* hc, uint64_t c
   }
 }
 
+// the distinct tags found by k_tagscan, compacted: out[0] = count, then (tag, entries)
+// pairs (up to TAGL_MAX; the host falls back to the full table beyond)
+constexpr uint32_t TAGL_MAX = 8192;
+__global__ void k_tag_compact(const uint32_t* tags, const unsigned long long* tcnt, unsigned long long* out) {
+  __shared__ unsigned int n;
+  if (threadIdx.x == 0) n = 0;
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < TAG_CAP; i += blockDim.x) {
+    if (tags[i] == EMPTY_TAG) continue;
+    const unsigned p = atomicAdd(&n, 1u);
+    if (p < TAGL_MAX) { out[1 + 2 * p] = tags[i]; out[2 + 2 * p] = tcnt[i]; }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) out[0] = n;
+}
+
 // Exact n_distinct and top-k of every key (PC keys, then object keys).
 ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
                         std::vector<ve_topk_entry>& top) {
@@ -534,32 +572,57 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   top.assign((size_t)nk * K, ve_topk_entry{0, 0});
   cudaError_t e;
   const int grid = c->num_sms * 4;
-  // 1. distinct tags and their entry counts
+  // 1. distinct tags and their entry counts; the occupied slots, compacted
   uint32_t* d_tags = nullptr;
   unsigned long long* d_tcnt = nullptr;
-  unsigned long long* d_small = nullptr;     // [0] overflow
+  unsigned long long* d_small = nullptr;     // [0] overflow, [1] occupied slots
+  unsigned long long* d_tl = nullptr;        // compacted tag list
+  uint32_t* d_occ = nullptr;                 // occupied slot indices
+  if (c->hcap > 0xFFFFFFFFull) return fail(c, VE_ERR_INVALID, "finalize: hist_capacity above 2^32");
   e = cudaMallocAsync((void**)&d_tags, TAG_CAP * 4, s);
   if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_tcnt, TAG_CAP * 8, s);
   if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_small, 16, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_tl, (1 + 2 * TAGL_MAX) * 8, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_occ, c->hcap * 4, s);
   if (e != cudaSuccess) return cuda_fail(c, e, "finalize alloc");
+  if (!c->pin) {
+    e = cudaMallocHost(&c->pin, (1 + 2 * TAGL_MAX) * 8 + 64);
+    if (e != cudaSuccess) { c->pin = nullptr; return cuda_fail(c, e, "finalize pinned buffer"); }
+  }
+  unsigned long long* hp = (unsigned long long*)c->pin;
   cudaMemsetAsync(d_tags, 0xFF, TAG_CAP * 4, s);
   cudaMemsetAsync(d_tcnt, 0, TAG_CAP * 8, s);
   cudaMemsetAsync(d_small, 0, 16, s);
   stage("start", s);
   count_launch();
-  k_tagscan<<<grid, 256, 0, s>>>(c->t.hslot, c->hcap, d_tags, d_tcnt, d_small);
-  std::vector<uint32_t> tags(TAG_CAP);
-  std::vector<unsigned long long> tcnt(TAG_CAP);
-  unsigned long long ovf = 0;
-  cudaMemcpyAsync(tags.data(), d_tags, TAG_CAP * 4, cudaMemcpyDeviceToHost, s);
-  cudaMemcpyAsync(tcnt.data(), d_tcnt, TAG_CAP * 8, cudaMemcpyDeviceToHost, s);
-  cudaMemcpyAsync(&ovf, d_small, 8, cudaMemcpyDeviceToHost, s);
-  cudaFreeAsync(d_tags, s);
-  cudaFreeAsync(d_tcnt, s);
+  k_tagscan<<<grid, 256, 0, s>>>(c->t.hslot, c->hcap, d_tags, d_tcnt, d_small, d_occ, d_small + 1);
+  count_launch();
+  k_tag_compact<<<1, 1024, 0, s>>>(d_tags, d_tcnt, d_tl);
+  cudaMemcpyAsync(hp, d_tl, (1 + 2 * TAGL_MAX) * 8, cudaMemcpyDeviceToHost, s);
+  cudaMemcpyAsync(hp + 1 + 2 * TAGL_MAX, d_small, 8, cudaMemcpyDeviceToHost, s);
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize tags"); }
+  unsigned long long ovf = hp[1 + 2 * TAGL_MAX];
+  std::vector<uint32_t> tags;
+  std::vector<unsigned long long> tcnt;
+  if (hp[0] <= TAGL_MAX) {
+    tags.resize(hp[0]);
+    tcnt.resize(hp[0]);
+    for (size_t i = 0; i < hp[0]; ++i) { tags[i] = (uint32_t)hp[1 + 2 * i]; tcnt[i] = hp[2 + 2 * i]; }
+  } else {
+    tags.resize(TAG_CAP);
+    tcnt.resize(TAG_CAP);
+    cudaMemcpyAsync(tags.data(), d_tags, TAG_CAP * 4, cudaMemcpyDeviceToHost, s);
+    cudaMemcpyAsync(tcnt.data(), d_tcnt, TAG_CAP * 8, cudaMemcpyDeviceToHost, s);
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) { cudaFreeAsync(d_small, s); return cuda_fail(c, e, "finalize tags"); }
+  }
+  cudaFreeAsync(d_tags, s);
+  cudaFreeAsync(d_tcnt, s);
+  cudaFreeAsync(d_tl, s);
   stage("tagscan+d2h", s);
   if (ovf) {                                  // too many distinct tags: aggregate every key
+    cudaFreeAsync(d_occ, s);
     cudaFreeAsync(d_small, s);
     ViewTable V;
     ve_status st = build_views(c, s, V);
@@ -570,7 +633,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   // 2. classify keys: direct (one tag) or aggregated (several tags)
   std::vector<uint32_t> ntag(nk, 0);
   std::vector<uint64_t> ent(nk, 0);
-  for (uint32_t i = 0; i < TAG_CAP; ++i) {
+  for (size_t i = 0; i < tags.size(); ++i) {
     if (tags[i] == EMPTY_TAG) continue;
     const uint32_t pk = tags[i] >> 16, koi = tags[i] & 0xFFFFu;
     ntag[pk]++;
@@ -613,8 +676,8 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   stage("alloc", s);
   // 3. emit direct keys' entries, aggregate the others in the view table
   count_launch();
-  k_emit<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, npc, d_direct, d_off, d_off + nk, gb[0], gc[0],
-                              V.vs, V.vc, V.vcap ? V.vcap - 1 : 0, d_small);
+  k_emit<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, d_occ, d_small + 1, npc, d_direct, d_off, d_off + nk, gb[0],
+                              gc[0], V.vs, V.vc, V.vcap ? V.vcap - 1 : 0, d_small);
   if (agg_in) {
     unsigned long long* d_nd = nullptr;
     cudaMallocAsync((void**)&d_nd, 8ull * nk, s);
@@ -644,6 +707,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   unsigned long long h_ovf = 0;
   cudaMemcpyAsync(&h_ovf, d_small, 8, cudaMemcpyDeviceToHost, s);
   free_views(V, s);
+  cudaFreeAsync(d_occ, s);
   cudaFreeAsync(gbuf, s);
   cudaFreeAsync(d_direct, s);
   cudaFreeAsync(d_off, s);

@@ -42,6 +42,7 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->t.hcount);
   cudaFree(c->obj_block);
   cudaFree(c->scratch);
+  if (c->pin) cudaFreeHost(c->pin);
   cudaFree(c->dense_pool);
   for (int i = 0; i < 2; ++i) {
     if (c->stage[i]) cudaFree(c->stage[i]);

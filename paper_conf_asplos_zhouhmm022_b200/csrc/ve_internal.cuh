@@ -120,6 +120,7 @@ struct ve_ctx {
   uint64_t records_analyzed = 0;
   // finalize scratch
   void* scratch = nullptr;
+  void* pin = nullptr;                       // pinned host staging of small report-time copies
   size_t scratch_bytes = 0;
   // merged histogram results (NCCL path)
   std::vector<uint64_t> merged_ndistinct;
