@@ -39,6 +39,7 @@ constexpr int K1_WARPS = K1_THREADS / 32;
 #endif
 constexpr int RING = VE_RING;                // record windows per warp ring (2 stages)
 constexpr uint32_t WIN_BYTES = 32 * sizeof(ve_record);
+constexpr uint64_t STAGE_RS_MAX = 16384;      // S8 staging entries per warp (16 B each)
 
 struct AnalyzeParams {
   const ve_record* recs;
@@ -52,6 +53,13 @@ struct AnalyzeParams {
   uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
   uint64_t nring;           // full windows (streamed through the per-warp rings)
   unsigned long long* work; // chunk claim counter (zeroed before the launch)
+  // S8 insert staging: a private region of stage_rs 16-byte entries per warp for the
+  // (tag, bits, count) groups the shared table cannot take; k_hist_drain inserts them
+  // into the HBM table after K1, at full occupancy, instead of K1's 16 warps/SM
+  // waiting on one global CAS round trip per group
+  uint4* stage;             // [grid * K1_WARPS][stage_rs]
+  uint32_t* stage_cnt;      // [grid * K1_WARPS] entries written (<= stage_rs)
+  uint32_t stage_rs;
   // byte offsets of the dynamic shared-memory regions (see carve_offsets)
   uint32_t o_ssum, o_smin, o_smax, o_sline, o_shs, o_shc, o_sob, o_soe, o_sctr, o_ring, o_bars;
   DevObjects o;
@@ -333,32 +341,82 @@ __device__ __noinline__ void merge_lines(const AnalyzeParams& P, WarpCache& C, b
   }
 }
 
-// Insert a group of equal (tag, bits) with count c: shared table first, HBM table on miss/full.
-__device__ __forceinline__ void hist_insert(const AnalyzeParams& P, uint32_t tag, uint64_t bits,
-                                            uint32_t c) {
+__shared__ uint32_t s_stage_n[K1_WARPS];   // entries claimed in the warp's staging region
+
+// Stage a (tag, bits, c) group for k_hist_drain; the HBM table directly once the
+// warp's region is full.  A plain store: the warp does not wait on it.
+__device__ __forceinline__ void hist_stage(const AnalyzeParams& P, uint32_t tag, uint64_t bits, uint32_t c) {
+  const uint32_t w = threadIdx.x >> 5;
+  const uint32_t pos = atomicAdd(&s_stage_n[w], 1u);
+  if (pos < P.stage_rs) {
+    uint4* q = P.stage + ((uint64_t)blockIdx.x * K1_WARPS + w) * P.stage_rs + pos;
+    __stcg(q, make_uint4((uint32_t)bits, (uint32_t)(bits >> 32), tag, c));
+  } else {
+    hist_insert_global(P.t, tag, bits, c);
+  }
+}
+
+// Shared-table part of an S8 insert: add count c to (tag, bits) in the CTA's table.
+// Returns false if the group was not placed.  The table is kept at most half full;
+// once it is, only the first two probe positions are searched for an existing entry.
+// (Placing a group in the shared table, the staging region or the HBM table is
+// equally exact: every part is summed into the HBM table in the end.)
+__device__ __forceinline__ bool hist_insert_shared(const AnalyzeParams& P, uint32_t tag, uint64_t bits, uint32_t c) {
   const Smem S = smem_of(P);
   const uint32_t hmask = P.hs - 1;
+  const bool full = *(volatile uint32_t*)&S.sctr[2] >= (P.hs >> 1);
+  const int np = full ? 2 : 16;
   uint32_t h = (uint32_t)hist_hash(tag, bits) & hmask;
-  for (int probe = 0; probe < 16; ++probe) {
+  for (int probe = 0; probe < np; ++probe) {
     HSlot* s = &S.shs[h];
     uint64_t lo = *(volatile uint64_t*)&s->bits;
     uint32_t stag = *(volatile uint32_t*)&s->tag;
-    if (stag == tag && lo == bits) { atomicAdd(&S.shc[h], c); return; }
+    if (stag == tag && lo == bits) { atomicAdd(&S.shc[h], c); return true; }
     if (stag == EMPTY_TAG) {
-      if (*(volatile uint32_t*)&S.sctr[2] >= (P.hs >> 1)) break;     // keep the table at most half full
+      if (*(volatile uint32_t*)&S.sctr[2] >= (P.hs >> 1)) return false;   // keep the table at most half full
       uint64_t ehi = ((uint64_t)(*(volatile uint32_t*)&s->pad) << 32) | EMPTY_TAG;
       uint64_t olo, ohi;
       cas128_shared(s, lo, ehi, bits, (uint64_t)tag, olo, ohi);
       if ((uint32_t)ohi == EMPTY_TAG && olo == lo) {
         atomicAdd(&S.sctr[2], 1u);
         atomicAdd(&S.shc[h], c);
-        return;
+        return true;
       }
-      if ((uint32_t)ohi == tag && olo == bits) { atomicAdd(&S.shc[h], c); return; }
+      if ((uint32_t)ohi == tag && olo == bits) { atomicAdd(&S.shc[h], c); return true; }
     }
     h = (h + 1) & hmask;
   }
-  hist_insert_global(P.t, tag, bits, c);
+  return false;
+}
+
+// Insert a group of equal (tag, bits) with count c: shared table first, then the
+// warp's staging region (HBM table on miss/full, via k_hist_drain).
+__device__ __forceinline__ void hist_insert(const AnalyzeParams& P, uint32_t tag, uint64_t bits,
+                                            uint32_t c) {
+  if (!hist_insert_shared(P, tag, bits, c)) hist_stage(P, tag, bits, c);
+}
+
+// Warp-collective insert of the groups led by the lanes with lead set (act = the
+// lanes executing this call): shared table, then one staging claim for the warp.
+__device__ __forceinline__ void hist_insert_warp(const AnalyzeParams& P, unsigned act, bool lead, uint32_t tag,
+                                                 uint64_t bits, uint32_t c) {
+  const bool need = lead && !hist_insert_shared(P, tag, bits, c);
+  const unsigned F = __ballot_sync(act, need);
+  if (!F) return;
+  const int lane = threadIdx.x & 31, l0 = __ffs(act) - 1;
+  const uint32_t w = threadIdx.x >> 5;
+  uint32_t base = 0;
+  if (lane == l0) base = atomicAdd(&s_stage_n[w], (uint32_t)__popc(F));
+  base = __shfl_sync(act, base, l0);
+  if (need) {
+    const uint32_t pos = base + (uint32_t)__popc(F & ((1u << lane) - 1u));
+    if (pos < P.stage_rs) {
+      uint4* q = P.stage + ((uint64_t)blockIdx.x * K1_WARPS + w) * P.stage_rs + pos;
+      __stcg(q, make_uint4((uint32_t)bits, (uint32_t)(bits >> 32), tag, c));
+    } else {
+      hist_insert_global(P.t, tag, bits, c);
+    }
+  }
 }
 
 __device__ __noinline__ int find_object(const AnalyzeParams& P, uint64_t addr) {
@@ -607,10 +665,27 @@ __device__ __forceinline__ void ring_issue_pred(bool on, uint32_t dst, const voi
 // With VE_CLAIM the warps claim CHUNK-window chunks of the trace dynamically
 // (balanced finish), else each warp streams one static contiguous range.
 static_assert(NSTAGE * STAGE_WIN == RING, "whole stages");
+#ifndef VE_WCLK
+#define VE_WCLK 0
+#endif
+#if VE_WCLK
+__shared__ uint32_t s_dbg[K1_WARPS][6];   // dense stages, dense singles, fast windows, hist inserts, dense exits nd, dense exits fit
+#define VE_DBG(i, n) do { if ((threadIdx.x & 31) == 0) s_dbg[threadIdx.x >> 5][i] += (n); } while (0)
+__shared__ unsigned long long s_dbgc[K1_WARPS][6];   // cycles: run_fast, run_dense, line, slot_acquire, refill, slow
+#define VE_TBEG(v) const long long v = clock64()
+#define VE_TEND(i, v) do { if ((threadIdx.x & 31) == 0) s_dbgc[threadIdx.x >> 5][i] += clock64() - (v); } while (0)
+#else
+#define VE_TBEG(v) do { } while (0)
+#define VE_TEND(i, v) do { } while (0)
+#define VE_DBG(i, n) do { } while (0)
+#endif
 #ifndef VE_CLAIM
 #define VE_CLAIM 0
 #endif
-constexpr uint32_t CHUNK = 32 * STAGE_WIN;   // windows per claim (whole stages)
+#ifndef VE_CHUNK_STAGES
+#define VE_CHUNK_STAGES 32
+#endif
+constexpr uint32_t CHUNK = VE_CHUNK_STAGES * STAGE_WIN;   // windows per claim (whole stages)
 struct Ring {
   const ve_record* src;   // next window to issue
   uint32_t iss;           // windows of the current range / chunk not yet issued
@@ -1053,6 +1128,7 @@ __device__ __forceinline__ bool run_dense(const AnalyzeParams& P, const ObjCache
 #pragma unroll
           for (int j = 0; j < STAGE_WIN; ++j) red_add_keep(dn + (o[j] >> LG), 1u, true);
           ndw += STAGE_WIN;
+          VE_DBG(0, 1);
           ring_stage_consume(R);
           continue;
         }
@@ -1062,10 +1138,11 @@ __device__ __forceinline__ bool run_dense(const AnalyzeParams& P, const ObjCache
     if (R.left == 0u) { done(); return false; }
     ring_next(P, R, addr, val, pm);
     uint64_t o;
-    if (!__all_sync(FULL, fits(addr, val, pm, o))) { done(); return true; }
+    if (!__all_sync(FULL, fits(addr, val, pm, o))) { VE_DBG(5, 1); done(); return true; }
     const MT pv = (MT)ld_pre<LG>(oc.pre + o);
-    if (!__all_sync(FULL, pv == (MT)val)) { nd = true; done(); return true; }
+    if (!__all_sync(FULL, pv == (MT)val)) { VE_DBG(4, 1); nd = true; done(); return true; }
     red_add_keep(dn + (o >> LG), 1u, true);
+    VE_DBG(1, 1);
     ++ndw;
   }
 }
@@ -1156,13 +1233,19 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, const ObjCache&
     if (c) g = gather(o);
 #endif
   };
+  VE_TBEG(tf0);
   uint64_t off = addr - oc.base;
   MT pv = gather(off);
   uint64_t a1 = 0, v1 = 0, p1 = 0, off1 = 0;
   MT pv1 = 0;
   bool more1 = !one && R.left != 0u, cont1 = false;
   if (more1) peek(a1, v1, p1, off1, pv1, cont1);
+#if VE_WCLK
+  { volatile MT sink = pv; (void)sink; }
+#endif
+  VE_TEND(1, tf0);
   while (true) {
+    VE_TBEG(tw0);
     // window i+2, two windows ahead of the one processed now
     uint64_t a2 = 0, v2 = 0, p2 = 0, off2 = 0;
     MT pv2 = 0;
@@ -1254,23 +1337,31 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, const ObjCache&
     // report time); every other record is inserted per distinct value.
     red_add_keep(reinterpret_cast<uint32_t*>(dn) + e, 1u, dl);
     const unsigned hm = __ballot_sync(FULL, !dl);
+    VE_TBEG(th0);
     if (hm) {
       const int l = __ffs(hm) - 1;
       const uint64_t v0 = (LG < 3) ? (uint64_t)__shfl_sync(FULL, (uint32_t)val, l) : shfl64(FULL, val, l);
       if (__all_sync(FULL, dl || val == v0)) {
+        VE_DBG(3, 1);
         if (lane == l) hist_insert(P, tag, val, __popc(hm));
       } else if (!dl) {
         const unsigned vg = (LG < 3) ? __match_any_sync(hm, (uint32_t)val) : __match_any_sync(hm, val);
-        if (lane == __ffs(vg) - 1) hist_insert(P, tag, val, __popc(vg));
+        VE_DBG(3, 32);
+        hist_insert_warp(P, hm, lane == __ffs(vg) - 1, tag, val, __popc(vg));
       }
     }
+    VE_TEND(0, th0);
     }
 #endif
+    VE_DBG(2, 1);
     if (++nwin == 0xFFFFu) save();          // 16-bit per-lane count fields
+    VE_TEND(2, tw0);
 
     // next window: continue while it is fast with the same key
     if (!cont1) {
+      VE_TBEG(ts0);
       save();
+      VE_TEND(5, ts0);
       if (more1) { addr = a1; val = v1; pm = p1; }
       return more1;
     }
@@ -1300,7 +1391,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   SlotE* slots = s_slot[warp];
   if (lane < WC) wc.key1[lane] = 0;
   if (lane < NSLOT) slots[lane].key = ~0ull;
-  if (lane == 0) { wc.next = 0; s_snext[warp] = 0; }
+  if (lane == 0) { wc.next = 0; s_snext[warp] = 0; s_stage_n[warp] = 0; }
 
   // full windows stream through the warp's TMA ring (a static contiguous range per
   // warp); without the ring (records not 16-byte aligned) each warp takes a static
@@ -1332,6 +1423,12 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   ObjCache oc;
   oc.base = 0; oc.lim = 0; oc.bmoff = 0; oc.pre = 0; oc.oi = -1; oc.id = 0; oc.fastlg = 0xFFu;
   uint32_t n_inv = 0, n_unm = 0;   // this lane's invalid / unmapped records (slow windows)
+#if VE_WCLK
+  const long long wclk0 = clock64();
+  if (lane < 6) { s_dbg[warp][lane] = 0; s_dbgc[warp][lane] = 0; }
+  __syncwarp();
+  uint32_t wslow = 0, wfast = 0;
+#endif
 
   uint64_t addr = 0, val = 0, pm = 0;
   bool have = false;
@@ -1369,6 +1466,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       }
       // dense loads of a key without live line state: the stage-batched dense path
       bool nd = true;
+      VE_TBEG(t1);
       if (!one && !cm && se->dense != 0ull) {
         switch (meta0 & 3u) {
           case 0: have = run_dense<0>(P, oc, se, R, addr, val, pm, nd); break;
@@ -1377,6 +1475,8 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
           default: have = run_dense<3>(P, oc, se, R, addr, val, pm, nd); break;
         }
       }
+      VE_TEND(3, t1);
+      VE_TBEG(t0);
       if (nd) {
       // specialised on the window's access type (compile-time width / kind)
 #define VE_RF(K, L) have = run_fast<K, L>(P, oc, se, one, cm, cy, xmin, xmax, R, addr, val, pm)
@@ -1396,6 +1496,8 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       }
 #undef VE_RF
       }
+      VE_TEND(0, t0);
+      VE_TBEG(t2);
       if (lf != 3u) {
         uint32_t nlf;
         if (one) {   // C8 for the window just consumed (still in addr / val)
@@ -1409,7 +1511,14 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
         if (lane == 0) se->lfail = nlf;
         __syncwarp();
       }
+      VE_TEND(4, t2);
+#if VE_WCLK
+      ++wfast;
+#endif
     } else {
+#if VE_WCLK
+      ++wslow;
+#endif
       const uint32_t cnt = slow_window(P, wc, addr, val, pm, true);
       n_inv += cnt & 0xFFFFu;
       n_unm += cnt >> 16;
@@ -1426,12 +1535,24 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
     n_unm += cnt >> 16;
   }
 
+#if VE_WCLK
+  if (lane == 0 && P.n > 100000000ull && (blockIdx.x < 3 || blockIdx.x == 147))
+    printf("WCLK %d %d %lld fast %u slow %u dstage %u dsingle %u fwin %u hist %u exnd %u exfit %u\n", blockIdx.x, warp,
+           clock64() - wclk0, wfast, wslow, s_dbg[warp][0], s_dbg[warp][1], s_dbg[warp][2], s_dbg[warp][3],
+           s_dbg[warp][4], s_dbg[warp][5]);
+  if (lane == 0 && P.n > 100000000ull && (blockIdx.x < 3 || blockIdx.x == 147))
+    printf("WCYC %d %d hist %llu fill %llu body %llu dense %llu line %llu save %llu\n", blockIdx.x, warp, s_dbgc[warp][0],
+           s_dbgc[warp][1], s_dbgc[warp][2], s_dbgc[warp][3], s_dbgc[warp][4], s_dbgc[warp][5]);
+#endif
   // fold the warp's key slots and line cache, then the CTA's shared state
   for (int i = 0; i < NSLOT; ++i)
     if (slots[i].key != ~0ull) slot_flush(P, &slots[i]);
   n_inv = __reduce_add_sync(FULL, n_inv);
   n_unm = __reduce_add_sync(FULL, n_unm);
+  __syncwarp();
   if (lane == 0) {
+    const uint32_t ns = s_stage_n[warp];
+    P.stage_cnt[gw] = ns < P.stage_rs ? ns : P.stage_rs;
     if (n_inv) atomicAdd(&S.sctr[0], n_inv);
     if (n_unm) atomicAdd(&S.sctr[1], n_unm);
     wcache_flush(P, wc);
@@ -1464,6 +1585,17 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   }
 }
 
+
+// K1b: insert the staged S8 groups into the HBM table (one block per warp region).
+__global__ void __launch_bounds__(256) k_hist_drain(const uint4* __restrict__ stage, const uint32_t* __restrict__ cnt,
+                                                    uint32_t rs, DevTables t) {
+  const uint32_t n = cnt[blockIdx.x];
+  const uint4* q = stage + (uint64_t)blockIdx.x * rs;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const uint4 e = __ldcs(q + i);
+    hist_insert_global(t, e.z, (uint64_t)e.x | ((uint64_t)e.y << 32), e.w);
+  }
+}
 
 // K2: fold the per-CTA line states of every shared key (C8's (+) monoid, order-free)
 // into the key's global state.  One block per key, a shared-memory tree over the CTAs.
@@ -1536,6 +1668,23 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   uint64_t windows = (n + 31) / 32;
   uint64_t blocks = (windows + K1_WARPS - 1) / K1_WARPS;
   if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+  // staging regions: a warp stages at most one group per record of its static range
+  {
+    const uint64_t tw = blocks * K1_WARPS;
+    const uint64_t per = 32 * ((windows + tw - 1) / tw + 2);
+    P.stage_rs = (uint32_t)(per < STAGE_RS_MAX ? per : STAGE_RS_MAX);
+    const size_t need = (size_t)tw * P.stage_rs * sizeof(uint4) + tw * sizeof(uint32_t);
+    if (c->hstage_bytes < need) {
+      if (c->hstage) cudaFree(c->hstage);
+      c->hstage = nullptr;
+      c->hstage_bytes = 0;
+      e = cudaMalloc(&c->hstage, need);
+      if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze staging");
+      c->hstage_bytes = need;
+    }
+    P.stage = (uint4*)c->hstage;
+    P.stage_cnt = (uint32_t*)((uint8_t*)c->hstage + (size_t)tw * P.stage_rs * sizeof(uint4));
+  }
 #if VE_CLAIM
   e = cudaMemsetAsync(P.work, 0, sizeof(unsigned long long), s);
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze claim counter");
@@ -1544,6 +1693,10 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   k_analyze<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze launch");
+  count_launch();
+  k_hist_drain<<<(unsigned)(blocks * K1_WARPS), 256, 0, s>>>(P.stage, P.stage_cnt, P.stage_rs, P.t);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "k_hist_drain launch");
   const uint32_t nsk = sp + so;
   count_launch();
   k_line_fold<<<nsk, LF_THREADS, 0, s>>>(c->t.lcta, (uint32_t)blocks, nsk, sp, c->cfg.n_pcs, c->t.line);

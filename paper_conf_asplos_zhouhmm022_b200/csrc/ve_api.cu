@@ -44,6 +44,7 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->scratch);
   if (c->pin) cudaFreeHost(c->pin);
   cudaFree(c->dense_pool);
+  cudaFree(c->hstage);
   for (int i = 0; i < 2; ++i) {
     if (c->stage[i]) cudaFree(c->stage[i]);
     if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);

@@ -129,6 +129,9 @@ struct ve_ctx {
   void* stage[2] = {nullptr, nullptr};
   cudaEvent_t stage_ev[2] = {nullptr, nullptr};
   size_t stage_bytes = 0;
+  // K1's S8 insert staging (k_hist_drain)
+  void* hstage = nullptr;
+  size_t hstage_bytes = 0;
 };
 
 struct ve_rep {
