@@ -177,6 +177,45 @@ ve_status ve_report_globals(const ve_rep* r, ve_globals* out);
 /* format 0: binary (magic "VERP", header, then the arrays above); 1: JSON */
 ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
 
+/* ---- accessed intervals and the adaptive copy plan --------
+ * PAPER.md section 6.1: "We define an interval [start, end] as
+ * the memory range accessed by each GPU instruction" and merge intervals "if
+ * they are adjacent or overlapped", on the GPU (Figure 4);
+ * the merged intervals drive the choice between segment copy and min-max copy
+ * of a data object's snapshot (Figure 5).  DESIGN.md 3 (R1-R4). */
+typedef struct ve_interval { uint64_t start, end; } ve_interval;   /* inclusive bytes */
+
+enum { VE_COPY_NONE = 0, VE_COPY_SEGMENT = 1, VE_COPY_MINMAX = 2 };
+typedef struct ve_copy_plan {
+  uint64_t n_segments;      /* merged intervals clipped to the object (segment copies)  */
+  uint64_t accessed_bytes;  /* bytes they cover (segment copy volume, Fig. 5c)          */
+  uint64_t lo, hi;          /* min / max accessed byte address, inclusive (0, 0: none)  */
+  uint64_t direct_bytes;    /* object size (direct copy, Fig. 5a)                       */
+  uint64_t minmax_bytes;    /* hi - lo + 1 (min-max copy, Fig. 5b); 0 when untouched     */
+  uint32_t choice;          /* VE_COPY_*: SEGMENT iff n_segments <= seg_max and          */
+                            /* 100*accessed_bytes < dense_pct*minmax_bytes (R4)          */
+  uint32_t pad;
+} ve_copy_plan;
+
+/* Merge n device intervals d_in (start > end = empty, skipped) into the sorted
+ * maximal runs of their union: out[k].end + 1 < out[k+1].start.  d_out (device,
+ * room for n) receives *h_n_out intervals.  n < 2^32.  Synchronizes s. */
+ve_status ve_interval_merge(ve_ctx* ctx, const ve_interval* d_in, uint64_t n, ve_interval* d_out,
+                            uint64_t* h_n_out, cudaStream_t s);
+
+/* The merged intervals accessed by n device records: [addr, addr + w - 1] of
+ * every valid global-space record (shared-space and invalid records skipped;
+ * validity uses the ctx's n_pcs).  d_out needs room for n.  n < 2^32.
+ * Synchronizes s. */
+ve_status ve_record_intervals(ve_ctx* ctx, const ve_record* d_records, uint64_t n, ve_interval* d_out,
+                              uint64_t* h_n_out, cudaStream_t s);
+
+/* Copy plan of every object of the ctx (h_plan[id], n_objects entries) from a
+ * merged interval set (output of the two calls above; VE_ERR_INVALID if it is
+ * not sorted, disjoint and non-adjacent).  Synchronizes s. */
+ve_status ve_plan_copies(ve_ctx* ctx, const ve_interval* d_merged, uint64_t n, uint32_t seg_max,
+                         uint32_t dense_pct, ve_copy_plan* h_plan, cudaStream_t s);
+
 /* Number of libve kernels launched by this process so far (all contexts). */
 uint64_t  ve_kernel_launches(void);
 

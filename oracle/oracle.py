@@ -35,6 +35,10 @@ KEY_DTYPE = np.dtype(
 GLOB_DTYPE = np.dtype([("n_records", "<u8"), ("n_invalid", "<u8"), ("n_unmapped", "<u8"), ("u_touched", "<u8")])
 OBJSTAT_DTYPE = np.dtype([("n_elems", "<u8"), ("n_written", "<u8"), ("n_loaded_eq", "<u8"),
                           ("n_ld_reload", "<u8"), ("n_touched", "<u8")])
+INTERVAL_DTYPE = np.dtype([("start", "<u8"), ("end", "<u8")])
+COPY_NONE, COPY_SEGMENT, COPY_MINMAX = 0, 1, 2
+PLAN_DTYPE = np.dtype([(f, "<u8") for f in ("n_segments", "accessed_bytes", "lo", "hi", "direct_bytes",
+                                           "minmax_bytes")] + [("choice", "<u4"), ("pad", "<u4")])
 DIFF_DTYPE = np.dtype([("n_elems", "<u8"), ("n_masked", "<u8"), ("n_unchanged", "<u8"), ("n_changed", "<u8"),
                        ("n_untouched", "<u8"), ("redundant", "<u4"), ("pad", "<u4")])
 
@@ -61,6 +65,11 @@ def lib():
         L.vo_analyze.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_snapshot_diff.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, u32, u32, vp, vp]
         L.vo_object_dedup.argtypes = [vp, u32, vp]
+        L.vo_interval_merge.argtypes = [vp, u64, vp]
+        L.vo_interval_merge.restype = u64
+        L.vo_record_intervals.argtypes = [u32, vp, u64, vp]
+        L.vo_record_intervals.restype = u64
+        L.vo_plan_copies.argtypes = [vp, u32, vp, u64, u32, u32, vp]
         L.vo_ord.argtypes = [u64, u32, u32]
         L.vo_ord.restype = u64
         L.vo_float_flags.argtypes = [u64, u32, u32]
@@ -72,6 +81,7 @@ def lib():
         for which, dt in enumerate([KEY_DTYPE, GLOB_DTYPE, OBJSTAT_DTYPE, DIFF_DTYPE]):
             assert L.vo_sizeof(which) == dt.itemsize, (which, L.vo_sizeof(which), dt.itemsize)
         assert L.vo_sizeof(4) == ctypes.sizeof(VoObject)
+        assert L.vo_sizeof(6) == PLAN_DTYPE.itemsize
         _LIB = L
     return _LIB
 
@@ -147,3 +157,30 @@ def float_flags(b, kind, w):
 
 def trunc(b, kind, w, K):
     return lib().vo_trunc(b, kind, w, K)
+
+
+def interval_merge(intervals):
+    """C13: intervals = INTERVAL_DTYPE array (or (n, 2) u64); returns the merged INTERVAL_DTYPE array."""
+    iv = np.ascontiguousarray(np.asarray(intervals).view(np.uint64).reshape(-1, 2)).view(INTERVAL_DTYPE).ravel()
+    out = np.zeros(max(len(iv), 1), dtype=INTERVAL_DTYPE)
+    k = lib().vo_interval_merge(iv.ctypes.data, len(iv), out.ctypes.data)
+    return out[:k]
+
+
+def record_intervals(n_pcs, recs):
+    """C14: merged intervals [addr, addr + w - 1] of the valid global-space records."""
+    recs = np.ascontiguousarray(recs)
+    out = np.zeros(max(len(recs), 1), dtype=INTERVAL_DTYPE)
+    k = lib().vo_record_intervals(n_pcs, recs.ctypes.data, len(recs), out.ctypes.data)
+    return out[:k]
+
+
+def plan_copies(objs, merged, seg_max=32, dense_pct=50):
+    """C15: per-object copy plan (PLAN_DTYPE indexed by object id)."""
+    arr, _keep = _objects(objs)
+    m = np.ascontiguousarray(merged, dtype=INTERVAL_DTYPE)
+    out = np.zeros(max(len(objs), 1), dtype=PLAN_DTYPE)
+    rc = lib().vo_plan_copies(arr, len(objs), m.ctypes.data, len(m), seg_max, dense_pct, out.ctypes.data)
+    if rc != 0:
+        raise ValueError("vo_plan_copies rejected its arguments")
+    return out[:len(objs)]

@@ -577,6 +577,85 @@ int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of) {
   return 0;
 }
 
+/* ---- C13-C15: accessed intervals and the adaptive copy plan ---------------
+ * PAPER.md 6.1.  The merged set is the definition itself: sort
+ * the intervals by start and sweep, extending the current run while the next
+ * interval starts at or before (run end + 1) -- "adjacent or overlapped"
+ * (P:L305).  This is the textbook sequential merge the paper names as the CPU
+ * alternative (O(N log N)); tests pin it against brute-force byte
+ * coverage and against a literal transcription of Figure 4's steps 1-9. */
+
+static int cmp_interval(const void* a, const void* b) {
+  const vo_interval* x = (const vo_interval*)a;
+  const vo_interval* y = (const vo_interval*)b;
+  if (x->start != y->start) return (x->start > y->start) - (x->start < y->start);
+  return (x->end > y->end) - (x->end < y->end);
+}
+
+uint64_t vo_interval_merge(const vo_interval* in, uint64_t n, vo_interval* out) {
+  vo_interval* v = (vo_interval*)malloc(sizeof(*v) * (n ? n : 1));
+  uint64_t m = 0;
+  for (uint64_t i = 0; i < n; ++i)
+    if (in[i].start <= in[i].end) v[m++] = in[i];      /* R1: start > end is the empty set */
+  qsort(v, m, sizeof(*v), cmp_interval);
+  uint64_t k = 0;
+  for (uint64_t i = 0; i < m; ++i) {
+    if (k > 0 && (out[k - 1].end == UINT64_MAX || v[i].start <= out[k - 1].end + 1)) {
+      if (v[i].end > out[k - 1].end) out[k - 1].end = v[i].end;   /* overlapped or adjacent */
+    } else {
+      out[k++] = v[i];
+    }
+  }
+  free(v);
+  return k;
+}
+
+uint64_t vo_record_intervals(uint32_t n_pcs, const vo_record* recs, uint64_t n, vo_interval* out) {
+  vo_interval* v = (vo_interval*)malloc(sizeof(*v) * (n ? n : 1));
+  uint64_t m = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    if (!rec_valid(&recs[i], n_pcs) || rec_shared(recs[i].meta)) continue;   /* R2 */
+    v[m].start = recs[i].addr;
+    v[m].end = recs[i].addr + rec_w(recs[i].meta) - 1;
+    ++m;
+  }
+  uint64_t k = vo_interval_merge(v, m, out);
+  free(v);
+  return k;
+}
+
+int vo_plan_copies(const vo_object* objs, uint32_t n_obj, const vo_interval* merged, uint64_t n,
+                 uint32_t seg_max, uint32_t dense_pct, vo_copy_plan* plan) {
+  for (uint32_t j = 0; j < n_obj; ++j) {
+    const vo_object* o = &objs[j];
+    if (o->id >= n_obj || o->size == 0) return -1;
+    vo_copy_plan* p = &plan[o->id];
+    memset(p, 0, sizeof(*p));
+    p->lo = UINT64_MAX;
+    p->direct_bytes = o->size;
+    const uint64_t ob = o->base, oe = o->base + o->size - 1;
+    for (uint64_t i = 0; i < n; ++i) {                  /* R3: clip every merged interval */
+      if (merged[i].end < ob || merged[i].start > oe) continue;
+      uint64_t s = merged[i].start > ob ? merged[i].start : ob;
+      uint64_t e = merged[i].end < oe ? merged[i].end : oe;
+      p->n_segments++;
+      p->accessed_bytes += e - s + 1;
+      if (s < p->lo) p->lo = s;
+      if (e > p->hi) p->hi = e;
+    }
+    if (p->n_segments == 0) {
+      p->lo = 0;
+      p->choice = VO_COPY_NONE;
+      continue;
+    }
+    p->minmax_bytes = p->hi - p->lo + 1;
+    /* R4: segment copy when sparse AND few intervals, else min-max */
+    int sparse = (unsigned __int128)100 * p->accessed_bytes < (unsigned __int128)dense_pct * p->minmax_bytes;
+    p->choice = (sparse && p->n_segments <= seg_max) ? VO_COPY_SEGMENT : VO_COPY_MINMAX;
+  }
+  return 0;
+}
+
 /* struct sizes, for the ctypes harness to check its mirrors */
 uint64_t vo_sizeof(int which) {
   switch (which) {
@@ -585,6 +664,7 @@ uint64_t vo_sizeof(int which) {
     case 2: return sizeof(vo_objstat);
     case 3: return sizeof(vo_diff);
     case 4: return sizeof(vo_object);
+    case 6: return sizeof(vo_copy_plan);
     default: return sizeof(vo_record);
   }
 }

@@ -116,6 +116,39 @@ int vo_snapshot_diff(const vo_config* cfg, const vo_object* objs, uint32_t n_obj
 /* C11: duplicate objects; group_of[i] = min id of i's class. */
 int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of);
 
+/* ---- accessed intervals and the adaptive copy plan -------
+ * PAPER.md section 6.1 (Figures 4 and 5).  The paper defines an
+ * interval [start, end] as the memory range accessed by a GPU instruction and
+ * merges intervals that are "adjacent or overlapped"; the merged set
+ * is the union's maximal runs of consecutive byte addresses.
+ * readings R1-R4. */
+typedef struct vo_interval { uint64_t start, end; } vo_interval;   /* inclusive */
+
+typedef struct vo_copy_plan {
+  uint64_t n_segments;      /* merged intervals clipped to the object        */
+  uint64_t accessed_bytes;  /* bytes they cover (segment copy, Fig. 5c)      */
+  uint64_t lo, hi;          /* min / max accessed byte address (inclusive)   */
+  uint64_t direct_bytes;    /* object size (direct copy, Fig. 5a)            */
+  uint64_t minmax_bytes;    /* hi - lo + 1 (min-max copy, Fig. 5b), 0 if none */
+  uint32_t choice;          /* VO_COPY_*                                     */
+  uint32_t pad;
+} vo_copy_plan;
+
+enum { VO_COPY_NONE = 0, VO_COPY_SEGMENT = 1, VO_COPY_MINMAX = 2 };
+
+/* C13: merge n intervals (start > end = empty, ignored) into the sorted
+ * maximal runs of their union; out needs room for n.  Returns the count. */
+uint64_t vo_interval_merge(const vo_interval* in, uint64_t n, vo_interval* out);
+
+/* C14: the merged intervals accessed by the valid global-space records
+ * ([addr, addr + w - 1] per record). */
+uint64_t vo_record_intervals(uint32_t n_pcs, const vo_record* recs, uint64_t n, vo_interval* out);
+
+/* C15: adaptive copy plan per object; merged must be the output
+ * of C13/C14.  plan[id] for every object id. */
+int vo_plan_copies(const vo_object* objs, uint32_t n_obj, const vo_interval* merged, uint64_t n,
+                 uint32_t seg_max, uint32_t dense_pct, vo_copy_plan* plan);
+
 /* helpers exposed for pinning */
 uint64_t vo_ord(uint64_t b, uint32_t kind, uint32_t w);
 uint32_t vo_float_flags(uint64_t b, uint32_t kind, uint32_t w);   /* bit0 nan, 1 nonint, 2 not_f16, 3 not_bf16, 4 not_f32 */

@@ -34,6 +34,10 @@ KEY_DTYPE = np.dtype(
 TOPK_DTYPE = np.dtype([("bits", "<u8"), ("count", "<u8")])
 OBJ_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_written", "n_loaded_eq", "n_ld_reload", "n_touched")])
 GLOB_DTYPE = np.dtype([(f, "<u8") for f in ("n_records", "n_invalid", "n_unmapped", "hist_entries")])
+INTERVAL_DTYPE = np.dtype([("start", "<u8"), ("end", "<u8")])   # ve_interval (inclusive)
+COPY_NONE, COPY_SEGMENT, COPY_MINMAX = 0, 1, 2
+PLAN_DTYPE = np.dtype([(f, "<u8") for f in ("n_segments", "accessed_bytes", "lo", "hi", "direct_bytes",
+                                           "minmax_bytes")] + [("choice", "<u4"), ("pad", "<u4")])
 DIFF_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_masked", "n_unchanged", "n_changed", "n_untouched")]
                       + [("redundant", "<u4"), ("pad", "<u4")])
 
@@ -90,6 +94,9 @@ def lib():
             "ve_nccl_get_unique_id": ([vp], st),
             "ve_nccl_comm_init": ([ctypes.POINTER(vp), i32, vp, i32], st),
             "ve_nccl_comm_destroy": ([vp], st),
+            "ve_interval_merge": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
+            "ve_record_intervals": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
+            "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -287,6 +294,27 @@ class Context:
         self._check(lib().ve_merge_stats(self._h, other._h if other is not None else None,
                                          ctypes.c_void_p(comm) if comm else None, _stream(stream)),
                     "ve_merge_stats")
+
+    def interval_merge(self, d_in, n, d_out, stream=None):
+        """ve_interval_merge: merge n device intervals (16 B each) into d_out; returns the merged count."""
+        m = ctypes.c_uint64(0)
+        self._check(lib().ve_interval_merge(self._h, _ptr(d_in), n, _ptr(d_out), ctypes.byref(m), _stream(stream)),
+                    "ve_interval_merge")
+        return m.value
+
+    def record_intervals(self, d_records, n, d_out, stream=None):
+        """ve_record_intervals: merged byte intervals accessed by n device records; returns the count."""
+        m = ctypes.c_uint64(0)
+        self._check(lib().ve_record_intervals(self._h, _ptr(d_records), n, _ptr(d_out), ctypes.byref(m),
+                                              _stream(stream)), "ve_record_intervals")
+        return m.value
+
+    def plan_copies(self, d_merged, n, seg_max=32, dense_pct=50, stream=None):
+        """ve_plan_copies: per-object adaptive copy plan (PLAN_DTYPE, indexed by object id)."""
+        out = np.zeros(max(getattr(self, "n_objects", 0), 1), dtype=PLAN_DTYPE)
+        self._check(lib().ve_plan_copies(self._h, _ptr(d_merged), n, seg_max, dense_pct, out.ctypes.data,
+                                         _stream(stream)), "ve_plan_copies")
+        return out[:getattr(self, "n_objects", 0)]
 
     def report(self):
         h = ctypes.c_void_p()
