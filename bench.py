@@ -242,6 +242,7 @@ def main():
     ap.add_argument("--cpu-sample", type=int, default=16_000_000)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-f1", action="store_true")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -259,7 +260,8 @@ def main():
     from paper_conf_asplos_zhouhmm022_b200 import ve
 
     wl = Workload(rank, world, dev)
-    ctx = ve.Context(n_pcs=5, max_objects=8, hist_capacity=1 << 23, device=local)
+    ctx = ve.Context(n_pcs=5, max_objects=8, hist_capacity=int(os.environ.get("VE_BENCH_HCAP", 1 << 23)),
+                     device=local)
     comm = None
     if world > 1:
         comm = ve.nccl_comm_from_torch(rank, world)
@@ -314,6 +316,10 @@ def main():
         "dedup_output_xgpu": int(groups[4]) == 3 and int(groups[3]) == 3,
     }
 
+    f1 = None
+    if rank == 0 and not args.no_f1:
+        f1 = measure_f1(ve, ctx, wl, stream, peak)
+
     e2e = None
     if not args.no_e2e and rank == 0 and world == 1:
         e2e = measure_e2e(ve, ctx, wl, stream, max(1, min(args.steps, 3)))
@@ -337,10 +343,35 @@ def main():
                              "alg_bytes_per_launch": alg[1]},
                 "analyze_ms_per_step": [round(statistics.mean(a[i] for a in an_ms), 4) for i in (0, 1)],
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
+                "f1_record_intervals": f1,
                 "parity_spot_check": spot}
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def measure_f1(ve, ctx, wl, stream, peak, reps=3):
+    """SURVEY 8(f) f1, measured outside the step: ve_record_intervals (warp compaction, radix sort,
+    merge scans) over this rank's gemm-epoch records; device time by CUDA events around the call."""
+    import torch
+    e = wl.epochs[1]
+    n = e["n"]
+    out = torch.empty(n * 16, dtype=torch.uint8, device=wl.device)
+    ctx.record_intervals(e["recs"], n, out, stream=stream.cuda_stream)   # warm-up (workspace pool)
+    ts, k = [], 0
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        a.record(stream)
+        k = ctx.record_intervals(e["recs"], n, out, stream=stream.cuda_stream)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    ms = statistics.median(ts)
+    del out
+    return {"records": n, "ms": ms, "records_per_s": n / (ms / 1e3), "merged_intervals": k,
+            "trace_gbs": n * REC_BYTES / (ms / 1e3) / 1e9, "frac_of_hbm_peak": n * REC_BYTES / (ms / 1e3) / 1e9 / peak,
+            "note": "f1 leg, not part of the step; the call synchronizes (count read-backs) inside the timed region"}
 
 
 def measure_e2e(ve, ctx, wl, stream, steps):

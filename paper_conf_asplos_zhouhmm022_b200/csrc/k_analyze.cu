@@ -459,8 +459,28 @@ struct __align__(16) SlotE {
   uint32_t nosnap;              // the object has no pre snapshot
   uint32_t pad;
   uint32_t sum[8];              // zero, eq_pre, nan, nonint, not_f16, not_bf16, not_f32, -
+  // C8 of constant runs, deferred: while the key's line is live, consecutive runs of
+  // one value cy only widen [cx0, cx1]; the horizontal segment is merged once (the
+  // (+) monoid keeps only the extreme points, so this equals merging every run)
+  uint64_t cy, cx0, cx1;
+  uint32_t cpend;               // a deferred constant segment is held
+  uint32_t pad2;
 };
-static_assert(sizeof(SlotE) == 112, "SlotE layout");
+static_assert(sizeof(SlotE) == 144, "SlotE layout");
+
+__device__ __noinline__ uint32_t const_line(const AnalyzeParams& P, WarpCache& wc, uint64_t xmin, uint64_t xmax,
+                                            uint64_t cy, uint32_t meta0, uint32_t pc0, uint32_t koi0, uint32_t lf);
+
+// merge a slot's deferred constant segment into the line states (all lanes)
+__device__ __noinline__ void slot_line_flush(const AnalyzeParams& P, WarpCache& wc, SlotE* e) {
+  if (!e->cpend) return;
+  const uint64_t key = e->key;
+  const uint32_t lf = const_line(P, wc, e->cx0, e->cx1, e->cy, (uint32_t)(key >> 32), (uint32_t)key & 0xFFFFu,
+                                 (uint32_t)(key >> 16) & 0xFFFFu, e->lfail);
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) { e->lfail = lf; e->cpend = 0; }
+  __syncwarp();
+}
 
 // claim (or find) a dense counter array of sorted object oi for the loads of one
 // (pc, access type): claim key ck = meta << 16 | pc (lane 0), broadcast
@@ -549,8 +569,8 @@ __device__ __noinline__ void slot_flush(const AnalyzeParams& P, const SlotE* e) 
 
 // index of key's slot in the warp's cache; a miss evicts round-robin (folding the
 // victim) and initialises the slot for key's access type
-__device__ __noinline__ int slot_acquire(const AnalyzeParams& P, SlotE* slots, uint32_t* next, uint64_t key,
-                                         int oi, bool nosnap) {
+__device__ __noinline__ int slot_acquire(const AnalyzeParams& P, WarpCache& wc, SlotE* slots, uint32_t* next,
+                                         uint64_t key, int oi, bool nosnap) {
   for (int i = 0; i < NSLOT; ++i)
     if (slots[i].key == key) return i;
   int v = -1;
@@ -560,6 +580,7 @@ __device__ __noinline__ int slot_acquire(const AnalyzeParams& P, SlotE* slots, u
     v = (int)(*next % NSLOT);
     __syncwarp();
     if ((threadIdx.x & 31) == 0) *next = *next + 1;
+    slot_line_flush(P, wc, &slots[v]);
     slot_flush(P, &slots[v]);
   }
   const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
@@ -576,6 +597,7 @@ __device__ __noinline__ int slot_acquire(const AnalyzeParams& P, SlotE* slots, u
     e.nwin = 0;
     e.lfail = lf;
     e.nosnap = nosnap ? 1u : 0u;
+    e.cpend = 0;
     for (int i = 0; i < 8; ++i) e.sum[i] = 0;
   }
   __syncwarp();
@@ -1350,7 +1372,7 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, const ObjCache&
         hist_insert_warp(P, hm, lane == __ffs(vg) - 1, tag, val, __popc(vg));
       }
     }
-    VE_TEND(0, th0);
+    VE_TEND(3, th0);
     }
 #endif
     VE_DBG(2, 1);
@@ -1453,7 +1475,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       // the window's key slot (pc, object, access type); while one of its line states
       // is still live, windows go one at a time through the line check
       const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
-      SlotE* se = &slots[slot_acquire(P, slots, &s_snext[warp], key, oc.oi, oc.pre == 0ull)];
+      SlotE* se = &slots[slot_acquire(P, wc, slots, &s_snext[warp], key, oc.oi, oc.pre == 0ull)];
       const uint32_t lf = se->lfail;
       // a live line state: runs of one value take the constant-run path, other windows
       // go one at a time through the per-window line check
@@ -1475,7 +1497,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
           default: have = run_dense<3>(P, oc, se, R, addr, val, pm, nd); break;
         }
       }
-      VE_TEND(3, t1);
+      (void)0;
       VE_TBEG(t0);
       if (nd) {
       // specialised on the window's access type (compile-time width / kind)
@@ -1505,7 +1527,17 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
         } else {
           xmin = redmin64(FULL, xmin);
           xmax = redmax64(FULL, xmax);
-          nlf = const_line(P, wc, xmin, xmax, cy, meta0, pc0, oc.id, lf);
+          nlf = lf;
+          if (se->cpend && se->cy == cy) {         // same constant: widen the deferred segment
+            if (lane == 0) {
+              se->cx0 = xmin < se->cx0 ? xmin : se->cx0;
+              se->cx1 = xmax > se->cx1 ? xmax : se->cx1;
+            }
+          } else {
+            slot_line_flush(P, wc, se);            // another constant: merge the held one first
+            nlf = se->lfail;
+            if (nlf != 3u && lane == 0) { se->cpend = 1; se->cy = cy; se->cx0 = xmin; se->cx1 = xmax; }
+          }
         }
         __syncwarp();
         if (lane == 0) se->lfail = nlf;
@@ -1541,12 +1573,15 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
            clock64() - wclk0, wfast, wslow, s_dbg[warp][0], s_dbg[warp][1], s_dbg[warp][2], s_dbg[warp][3],
            s_dbg[warp][4], s_dbg[warp][5]);
   if (lane == 0 && P.n > 100000000ull && (blockIdx.x < 3 || blockIdx.x == 147))
-    printf("WCYC %d %d hist %llu fill %llu body %llu dense %llu line %llu save %llu\n", blockIdx.x, warp, s_dbgc[warp][0],
+    printf("WCYC %d %d runfast %llu fill %llu body %llu hist %llu line %llu save %llu\n", blockIdx.x, warp, s_dbgc[warp][0],
            s_dbgc[warp][1], s_dbgc[warp][2], s_dbgc[warp][3], s_dbgc[warp][4], s_dbgc[warp][5]);
 #endif
   // fold the warp's key slots and line cache, then the CTA's shared state
   for (int i = 0; i < NSLOT; ++i)
-    if (slots[i].key != ~0ull) slot_flush(P, &slots[i]);
+    if (slots[i].key != ~0ull) {
+      slot_line_flush(P, wc, &slots[i]);
+      slot_flush(P, &slots[i]);
+    }
   n_inv = __reduce_add_sync(FULL, n_inv);
   n_unm = __reduce_add_sync(FULL, n_unm);
   __syncwarp();
