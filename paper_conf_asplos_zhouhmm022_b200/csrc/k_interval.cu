@@ -62,24 +62,48 @@ __device__ __forceinline__ bool warp_compact(bool ok, uint64_t& s, uint64_t& e) 
   return ok && !next_join;
 }
 
-// append the emitting lanes' intervals at a warp-claimed position of (S, E)
-__device__ __forceinline__ void warp_append(bool emit, uint64_t s, uint64_t e, uint64_t* S, uint64_t* E,
-                                            unsigned long long* cnt) {
+// Emitted intervals collect in a per-warp shared buffer and go to (S, E) 32+ at a
+// time with one global claim (a claim per window would serialise ~N/32 atomics on
+// one counter).  n is warp-uniform; the buffer never holds more than 63 entries.
+constexpr int WB = 64;
+struct WarpBuf {
+  uint64_t s[WB], e[WB];
+};
+
+__device__ __forceinline__ void wb_flush(WarpBuf& b, uint32_t& n, uint64_t* S, uint64_t* E,
+                                         unsigned long long* cnt) {
+  const int lane = threadIdx.x & 31;
+  if (n == 0) return;
+  unsigned long long base = 0;
+  if (lane == 0) base = atomicAdd(cnt, (unsigned long long)n);
+  base = __shfl_sync(FULLM, base, 0);
+  for (uint32_t i = lane; i < n; i += 32) {
+    S[base + i] = b.s[i];
+    E[base + i] = b.e[i];
+  }
+  __syncwarp();
+  n = 0;
+}
+
+__device__ __forceinline__ void wb_append(WarpBuf& b, uint32_t& n, bool emit, uint64_t s, uint64_t e, uint64_t* S,
+                                          uint64_t* E, unsigned long long* cnt) {
   const int lane = threadIdx.x & 31;
   const unsigned m = __ballot_sync(FULLM, emit);
-  if (!m) return;
-  unsigned long long base = 0;
-  if (lane == 0) base = atomicAdd(cnt, (unsigned long long)__popc(m));
-  base = __shfl_sync(FULLM, base, 0);
   if (emit) {
-    const uint64_t p = base + __popc(m & ((1u << lane) - 1u));
-    S[p] = s;
-    E[p] = e;
+    const uint32_t p = n + __popc(m & ((1u << lane) - 1u));
+    b.s[p] = s;
+    b.e[p] = e;
   }
+  n += __popc(m);
+  __syncwarp();
+  if (n >= 32) wb_flush(b, n, S, E, cnt);
 }
 
 __global__ void __launch_bounds__(IV_T) k_iv_in(const ve_interval* in, uint64_t n, uint64_t* S, uint64_t* E,
                                                 unsigned long long* cnt) {
+  __shared__ WarpBuf wbuf[IV_NW];
+  WarpBuf& b = wbuf[threadIdx.x >> 5];
+  uint32_t bn = 0;
   const uint64_t nw = (n + 31) / 32, stride = (uint64_t)gridDim.x * IV_NW;
   for (uint64_t w = (uint64_t)blockIdx.x * IV_NW + (threadIdx.x >> 5); w < nw; w += stride) {
     const uint64_t i = w * 32 + (threadIdx.x & 31);
@@ -87,12 +111,16 @@ __global__ void __launch_bounds__(IV_T) k_iv_in(const ve_interval* in, uint64_t 
     if (i < n) { s = in[i].start; e = in[i].end; }
     const bool ok = i < n && s <= e;      // start > end: the empty set (R1)
     const bool emit = warp_compact(ok, s, e);
-    warp_append(emit, s, e, S, E, cnt);
+    wb_append(b, bn, emit, s, e, S, E, cnt);
   }
+  wb_flush(b, bn, S, E, cnt);
 }
 
 __global__ void __launch_bounds__(IV_T) k_iv_rec(const ve_record* r, uint64_t n, uint32_t n_pcs, uint64_t* S,
                                                  uint64_t* E, unsigned long long* cnt) {
+  __shared__ WarpBuf wbuf[IV_NW];
+  WarpBuf& b = wbuf[threadIdx.x >> 5];
+  uint32_t bn = 0;
   const uint64_t nw = (n + 31) / 32, stride = (uint64_t)gridDim.x * IV_NW;
   for (uint64_t w = (uint64_t)blockIdx.x * IV_NW + (threadIdx.x >> 5); w < nw; w += stride) {
     const uint64_t i = w * 32 + (threadIdx.x & 31);
@@ -107,8 +135,9 @@ __global__ void __launch_bounds__(IV_T) k_iv_rec(const ve_record* r, uint64_t n,
       e = addr + (1ull << meta_lg(meta)) - 1ull;
     }
     const bool emit = warp_compact(ok, s, e);
-    warp_append(emit, s, e, S, E, cnt);
+    wb_append(b, bn, emit, s, e, S, E, cnt);
   }
+  wb_flush(b, bn, S, E, cnt);
 }
 
 // out[0] = min start, out[1] = max start, out[2] = number of i with S[i] < S[i-1]
