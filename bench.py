@@ -243,6 +243,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-f1", action="store_true")
+    ap.add_argument("--no-cfg5", action="store_true")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -320,6 +321,10 @@ def main():
     if rank == 0 and not args.no_f1:
         f1 = measure_f1(ve, ctx, wl, stream, peak)
 
+    dd5 = None
+    if rank == 0 and not args.no_cfg5:
+        dd5 = measure_cfg5_dedup(ve, ctx, stream, peak)
+
     e2e = None
     if not args.no_e2e and rank == 0 and world == 1:
         e2e = measure_e2e(ve, ctx, wl, stream, max(1, min(args.steps, 3)))
@@ -343,7 +348,7 @@ def main():
                              "alg_bytes_per_launch": alg[1]},
                 "analyze_ms_per_step": [round(statistics.mean(a[i] for a in an_ms), 4) for i in (0, 1)],
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
-                "f1_record_intervals": f1,
+                "f1_record_intervals": f1, "cfg5_dedup": dd5,
                 "parity_spot_check": spot}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -372,6 +377,44 @@ def measure_f1(ve, ctx, wl, stream, peak, reps=3):
     return {"records": n, "ms": ms, "records_per_s": n / (ms / 1e3), "merged_intervals": k,
             "trace_gbs": n * REC_BYTES / (ms / 1e3) / 1e9, "frac_of_hbm_peak": n * REC_BYTES / (ms / 1e3) / 1e9 / peak,
             "note": "f1 leg, not part of the step; the call synchronizes (count read-backs) inside the timed region"}
+
+
+def measure_cfg5_dedup(ve, ctx, stream, peak, reps=3):
+    """BASELINE configs[4] (cfg5), duplicate-object half: ve_object_dedup over 1000 objects / ~19.7 GiB of
+    post snapshots generated on the device (untimed); CUDA events around the (synchronizing) call.
+    Algorithmic bytes: every byte hashed once + 2 x size per non-representative duplicate."""
+    import torch
+    from gen import vegen as G
+    from tests import workloads as W
+    objs = W.cfg5_dedup_objects()
+    sp = stream.cuda_stream
+    dobjs = []
+    for o in objs:
+        t = torch.empty(o["size"], dtype=torch.uint8, device="cuda")
+        G.dedup_device(W.CFG5_SEED, o["id"], W.CFG5_UNIT, t.data_ptr(), sp)
+        dobjs.append(dict(o, pre=None, post=t))
+    torch.cuda.synchronize()
+    want = W.cfg5_expected_groups(objs)
+    g = ctx.object_dedup(dobjs, stream=sp)                     # warm-up
+    ts = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        a.record(stream)
+        g = ctx.object_dedup(dobjs, stream=sp)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    ms = statistics.median(ts)
+    total = sum(o["size"] for o in objs)
+    dup = sum(o["size"] for o, w in zip(objs, want) if w != o["id"])
+    alg = total + 2 * dup
+    del dobjs
+    torch.cuda.empty_cache()
+    return {"workload": "cfg5 duplicate-object scan: 1000 objects, 4 sizes (8-32 MiB), 30% zero / 10% copies / "
+                        "5% one-bit flips / 55% random", "objects": len(objs), "bytes": total, "ms": ms,
+            "alg_bytes": alg, "alg_gbs": alg / (ms / 1e3) / 1e9, "frac_of_hbm_peak": alg / (ms / 1e3) / 1e9 / peak,
+            "groups": len(set(want)), "parity_closed_form": [int(x) for x in g] == want}
 
 
 def measure_e2e(ve, ctx, wl, stream, steps):

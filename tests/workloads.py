@@ -30,3 +30,33 @@ def device_objects(host_objs, device="cuda"):
 def device_records(recs, device="cuda"):
     import torch
     return torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).to(device)
+
+
+# ---- cfg5 duplicate-object scan (dedup half) ------------------------------
+CFG5_SEED, CFG5_N, CFG5_UNIT = 5, 1000, 8 << 20     # 1000 objects, 4 sizes of 8-32 MiB: ~19.5 GiB
+
+
+def cfg5_dedup_objects(n=CFG5_N, unit=CFG5_UNIT, seed=CFG5_SEED):
+    """Object table of the cfg5 duplicate scan (generator metadata: size, content class, copy source)."""
+    return [G.dedup_object(seed, i, unit) for i in range(n)]
+
+
+def cfg5_expected_groups(objs):
+    """Closed form of the duplicate classes from the generator's construction (not from any analysis):
+    class 0 = zeros, 3 = random (own content), 1 = exact copy of src, 2 = copy of src with one bit
+    flipped (a content of its own).  group_of[i] = min id with the same content."""
+    key = {}
+    for o in objs:
+        c, s = o["cls"], o["src"]
+        if c == 0 or (c == 1 and objs[s]["cls"] == 0):
+            key[o["id"]] = ("z", o["size"])
+        elif c == 3:
+            key[o["id"]] = ("r", o["id"])
+        elif c == 1:
+            key[o["id"]] = ("r", s)
+        else:
+            key[o["id"]] = ("f", o["id"])
+    first = {}
+    for o in objs:
+        first.setdefault(key[o["id"]], o["id"])
+    return [first[key[o["id"]]] for o in objs]
