@@ -33,7 +33,19 @@ __global__ void __launch_bounds__(256) k_hash(const HashJob* jobs, unsigned long
   if (((uintptr_t)jb.p & 15) == 0) {
     const uint64_t nv = jb.size / 16;
     const uint4* v = (const uint4*)jb.p;
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nv; i += stride) {
+    // four independent 16-byte loads in flight per thread per iteration
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    for (; i + 3 * stride < nv; i += 4 * stride) {
+      uint4 x[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) x[u] = __ldcs(v + i + u * stride);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint64_t k = i + u * stride;
+        acc += word_mix(((uint64_t)x[u].y << 32) | x[u].x, 2 * k) + word_mix(((uint64_t)x[u].w << 32) | x[u].z, 2 * k + 1);
+      }
+    }
+    for (; i < nv; i += stride) {
       const uint4 x = __ldcs(v + i);
       acc += word_mix(((uint64_t)x.y << 32) | x.x, 2 * i) + word_mix(((uint64_t)x.w << 32) | x.z, 2 * i + 1);
     }
@@ -63,7 +75,7 @@ struct CmpJob {
   uint32_t pad;
 };
 
-// K8: bytewise verification of (member, representative) pairs, 64 KiB per CTA
+// K8: bytewise verification of (member, representative) pairs, 256 KiB per CTA
 __global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned int* differs) {
   const CmpJob jb = jobs[blockIdx.x];
   if (*(volatile unsigned int*)&differs[jb.pair]) return;
@@ -72,7 +84,18 @@ __global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned in
   const uint8_t* b = jb.b + jb.off;
   if ((((uintptr_t)a | (uintptr_t)b) & 15) == 0) {
     const uint64_t nv = jb.len / 16;
-    for (uint64_t i = threadIdx.x; i < nv; i += blockDim.x) {
+    uint64_t i = threadIdx.x;
+    for (; i + 3 * blockDim.x < nv; i += 4 * blockDim.x) {   // 8 independent 16-byte loads in flight
+      uint4 x[4], y[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        x[u] = __ldcs((const uint4*)a + i + u * blockDim.x);
+        y[u] = __ldcs((const uint4*)b + i + u * blockDim.x);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) diff |= (x[u].x != y[u].x) | (x[u].y != y[u].y) | (x[u].z != y[u].z) | (x[u].w != y[u].w);
+    }
+    for (; i < nv; i += blockDim.x) {
       const uint4 x = __ldcs((const uint4*)a + i), y = __ldcs((const uint4*)b + i);
       diff |= (x.x != y.x) | (x.y != y.y) | (x.z != y.z) | (x.w != y.w);
     }
@@ -104,9 +127,11 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
   unsigned long long* d_hash = (unsigned long long*)((uint8_t*)d + hj.size() * sizeof(HashJob));
   cudaMemcpyAsync(d_jobs, hj.data(), hj.size() * sizeof(HashJob), cudaMemcpyHostToDevice, s);
   cudaMemsetAsync(d_hash, 0, hj.size() * 8, s);
-  // grid.x sized so the largest object gets ~8 KiB per CTA-iteration, capped
-  uint64_t gx = (maxsz / 16 + 255) / 256;
-  gx = std::min<uint64_t>(std::max<uint64_t>(gx / 4, 1), 1024);
+  // grid.x: ~256 KiB of the largest object per CTA (16 KiB per CTA-iteration, 4 loads deep),
+  // at least two CTAs per SM over the whole set
+  uint64_t gx = (maxsz + (256u << 10) - 1) / (256u << 10);
+  const uint64_t want = (2ull * c->num_sms + elig.size() - 1) / elig.size();
+  gx = std::min<uint64_t>(std::max<uint64_t>(std::max<uint64_t>(gx, want), 1), 1024);
   for (size_t y0 = 0; y0 < hj.size(); y0 += 65535) {
     const unsigned gy = (unsigned)std::min<size_t>(65535, hj.size() - y0);
     count_launch();
@@ -128,7 +153,7 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
     pending.push_back(g.second);
   }
   // K8: verify against the representative (lowest id); mismatches form a new pending group
-  const uint64_t CH = 1 << 16;
+  const uint64_t CH = 1 << 18;   // 256 KiB per verification CTA
   while (!pending.empty()) {
     std::vector<CmpJob> jobs;
     std::vector<std::pair<uint32_t, uint32_t>> pairs;  // (group index, member index)
