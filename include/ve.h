@@ -177,6 +177,18 @@ ve_status ve_report_globals(const ve_rep* r, ve_globals* out);
 /* format 0: binary (magic "VERP", header, then the arrays above); 1: JSON */
 ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
 
+/* ---- approximate frequent values ---------------------------
+ * Def 3.3 (frequent values) over the truncated values of Def 3.8
+ * (P:L191-L193): for every key whose records all have one float type (Q15),
+ * the exact histogram of its values with the low (m - K) mantissa bits cleared
+ * (K = cfg.mant_bits; NaNs keep their bits, R5): h_ndistinct[n_keys] distinct
+ * truncated values and h_top[n_keys * topk] by (count desc, bits asc), zero-
+ * filled; integer and mixed-type keys report 0.  "Approximate frequent" holds
+ * when 100 * h_top[k*topk].count > t_frequent_pct * (n_ld + n_st).  Works on
+ * the ctx's statistics as accumulated so far (local merges included);
+ * VE_ERR_STATE after an NCCL rank merge.  Synchronizes s. */
+ve_status ve_approx_topk(ve_ctx* ctx, uint64_t* h_ndistinct, ve_topk_entry* h_top, cudaStream_t s);
+
 /* ---- accessed intervals and the adaptive copy plan --------
  * PAPER.md section 6.1: "We define an interval [start, end] as
  * the memory range accessed by each GPU instruction" and merge intervals "if

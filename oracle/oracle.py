@@ -65,6 +65,7 @@ def lib():
         L.vo_analyze.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_snapshot_diff.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, u32, u32, vp, vp]
         L.vo_object_dedup.argtypes = [vp, u32, vp]
+        L.vo_approx_topk.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_interval_merge.argtypes = [vp, u64, vp]
         L.vo_interval_merge.restype = u64
         L.vo_record_intervals.argtypes = [u32, vp, u64, vp]
@@ -184,3 +185,18 @@ def plan_copies(objs, merged, seg_max=32, dense_pct=50):
     if rc != 0:
         raise ValueError("vo_plan_copies rejected its arguments")
     return out[:len(objs)]
+
+
+def approx_topk(cfg, objs, recs):
+    """C16: (ndistinct[n_keys], top_bits[n_keys, topk], top_count[n_keys, topk]) of the truncated values."""
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    nk = cfg.n_pcs + len(objs) + 1
+    nd = np.zeros(nk, dtype=np.uint64)
+    tb = np.zeros((nk, cfg.topk), dtype=np.uint64)
+    tc = np.zeros((nk, cfg.topk), dtype=np.uint64)
+    rc = lib().vo_approx_topk(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), nd.ctypes.data,
+                              tb.ctypes.data, tc.ctypes.data)
+    if rc != 0:
+        raise ValueError("vo_approx_topk rejected its arguments")
+    return nd, tb, tc

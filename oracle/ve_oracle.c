@@ -577,6 +577,78 @@ int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of) {
   return 0;
 }
 
+/* ---- C16: approximate frequent values (f2; Def 3.3 over Def 3.8) ---------- */
+
+int vo_approx_topk(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                   uint64_t n, uint64_t* ndistinct, uint64_t* top_bits, uint64_t* top_count) {
+  if (!cfg || cfg->topk > VO_MAX_TOPK || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t n_keys = (uint64_t)cfg->n_pcs + n_obj + 1;
+  const uint64_t key_shared = (uint64_t)cfg->n_pcs + n_obj;
+  const uint32_t K = cfg->topk;
+  memset(ndistinct, 0, sizeof(uint64_t) * n_keys);
+  memset(top_bits, 0, sizeof(uint64_t) * n_keys * K);
+  memset(top_count, 0, sizeof(uint64_t) * n_keys * K);
+  /* pass 1: the type codes of every key (Q15: one type only) */
+  uint32_t* types = (uint32_t*)calloc(n_keys, sizeof(uint32_t));   /* bit tc set if seen */
+  for (uint64_t i = 0; i < n; ++i) {
+    dec_t d;
+    decode(cfg, &t, &recs[i], &d);
+    if (!d.valid) continue;
+    types[recs[i].pc] |= 1u << d.tc;
+    if (d.shared) types[key_shared] |= 1u << d.tc;
+    else if (d.obj) types[(uint64_t)cfg->n_pcs + d.obj->id] |= 1u << d.tc;
+  }
+  /* pass 2: (key, truncated bits) of every record of a single-float-type key */
+  hent* pairs = (hent*)malloc(sizeof(hent) * (2 * n + 1));
+  uint64_t np = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    const vo_record* r = &recs[i];
+    dec_t d;
+    decode(cfg, &t, r, &d);
+    if (!d.valid || d.kind < 2) continue;
+    uint64_t kset[2];
+    int nk = 0;
+    kset[nk++] = r->pc;
+    if (d.shared) kset[nk++] = key_shared;
+    else if (d.obj) kset[nk++] = (uint64_t)cfg->n_pcs + d.obj->id;
+    /* R5: NaNs keep their bits (clearing mantissa bits could turn a NaN into an infinity) */
+    uint64_t tb = (d.fflags & 1u) ? r->value : vo_trunc(r->value, d.kind, d.w, cfg->mant_bits);
+    for (int j = 0; j < nk; ++j) {
+      if (types[kset[j]] != (1u << d.tc)) continue;          /* mixed types: no approximate histogram */
+      pairs[np].key = kset[j];
+      pairs[np].bits = tb;
+      pairs[np].count = 1;
+      ++np;
+    }
+  }
+  qsort(pairs, np, sizeof(hent), cmp_key_bits);
+  uint64_t nr = 0;
+  for (uint64_t i = 0; i < np;) {
+    uint64_t j = i;
+    while (j < np && pairs[j].key == pairs[i].key && pairs[j].bits == pairs[i].bits) ++j;
+    pairs[nr].key = pairs[i].key;
+    pairs[nr].bits = pairs[i].bits;
+    pairs[nr].count = j - i;
+    ++nr;
+    i = j;
+  }
+  qsort(pairs, nr, sizeof(hent), cmp_key_count_bits);
+  for (uint64_t i = 0; i < nr; ++i) {
+    const uint64_t k = pairs[i].key;
+    if (ndistinct[k] < K) {
+      top_bits[k * K + ndistinct[k]] = pairs[i].bits;
+      top_count[k * K + ndistinct[k]] = pairs[i].count;
+    }
+    ndistinct[k]++;
+  }
+  free(pairs);
+  free(types);
+  free(t.by_base);
+  return 0;
+}
+
 /* ---- C13-C15: accessed intervals and the adaptive copy plan ---------------
  * PAPER.md 6.1.  The merged set is the definition itself: sort
  * the intervals by start and sweep, extending the current run while the next

@@ -149,6 +149,17 @@ uint64_t vo_record_intervals(uint32_t n_pcs, const vo_record* recs, uint64_t n, 
 int vo_plan_copies(const vo_object* objs, uint32_t n_obj, const vo_interval* merged, uint64_t n,
                  uint32_t seg_max, uint32_t dense_pct, vo_copy_plan* plan);
 
+/* ---- approximate frequent values -------------------------
+ * Def 3.3 (frequent values) over the truncated values of Def 3.8
+ * ("approximate values ... some fine-grained patterns"): for every
+ * key whose records all have one float type (Q15), each value's low (m - K)
+ * mantissa bits are cleared (C7; NaNs keep their bits, R5) and the exact
+ * histogram of the truncated values gives n_distinct and the top-k by (count
+ * desc, bits asc).  Keys of mixed or integer type report 0 / nothing (C16).
+ * ndistinct[n_keys], top_bits / top_count[n_keys * topk] (0-filled). */
+int vo_approx_topk(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                   uint64_t n, uint64_t* ndistinct, uint64_t* top_bits, uint64_t* top_count);
+
 /* helpers exposed for pinning */
 uint64_t vo_ord(uint64_t b, uint32_t kind, uint32_t w);
 uint32_t vo_float_flags(uint64_t b, uint32_t kind, uint32_t w);   /* bit0 nan, 1 nonint, 2 not_f16, 3 not_bf16, 4 not_f32 */

@@ -73,6 +73,68 @@ __global__ void k_views(const HSlot* hs, const unsigned long long* hc, uint64_t 
   }
 }
 
+__global__ void k_occupancy(const HSlot* hs, uint64_t cap, unsigned long long* cnt);
+
+// the exact histogram's entries of single-float-type keys, with
+// their values truncated to K mantissa bits (NaNs kept), -> a view table of the
+// approximate values.  akind[key] = kind << 2 | lg, or 0xFF (no approximate histogram).
+__global__ void k_approx_views(const HSlot* hs, const unsigned long long* hc, uint64_t hcap, uint32_t n_pcs,
+                               const uint8_t* akind, uint32_t K, HSlot* vs, unsigned long long* vc, uint64_t vmask,
+                               unsigned long long* overflow) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < hcap; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t tag = hs[i].tag;
+    if (tag == EMPTY_TAG) continue;
+    const uint64_t bits = hs[i].bits;
+    const unsigned long long cnt = hc[i];
+    const uint32_t pc = tag >> 16, koi = tag & 0xFFFFu;
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+      if (j == 1 && koi == KO_NONE) break;
+      const uint32_t key = j == 0 ? pc : n_pcs + koi;
+      const uint32_t ak = akind[key];
+      if (ak == 0xFFu) continue;
+      const uint32_t kind = ak >> 2, lg = ak & 3u;
+      int64_t ival;
+      const bool nan = float_flags(bits, kind, lg, ival) & 1u;
+      vinsert(vs, vc, vmask, overflow, key, nan ? bits : trunc_bits(bits, kind, lg, K), cnt);
+    }
+  }
+}
+
+ve_status approx_topk(ve_ctx* c, cudaStream_t s, const std::vector<uint8_t>& akind, std::vector<uint64_t>& ndistinct,
+                      std::vector<ve_topk_entry>& top) {
+  cudaError_t e;
+  unsigned long long* d_small = nullptr;   // [0] overflow, [1] occupied
+  uint8_t* d_ak = nullptr;
+  e = cudaMallocAsync((void**)&d_small, 16, s);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_ak, akind.size(), s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "approx alloc");
+  cudaMemsetAsync(d_small, 0, 16, s);
+  cudaMemcpyAsync(d_ak, akind.data(), akind.size(), cudaMemcpyHostToDevice, s);
+  count_launch();
+  k_occupancy<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->hcap, d_small + 1);
+  unsigned long long occ = 0;
+  e = cudaMemcpyAsync(&occ, d_small + 1, 8, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_small, s); cudaFreeAsync(d_ak, s); return cuda_fail(c, e, "approx occupancy"); }
+  ViewTable V;
+  ve_status st = alloc_views(c, s, 2 * occ + 1, V);
+  if (st != VE_OK) { cudaFreeAsync(d_small, s); cudaFreeAsync(d_ak, s); return st; }
+  count_launch();
+  k_approx_views<<<c->num_sms * 4, 256, 0, s>>>(c->t.hslot, c->t.hcount, c->hcap, c->cfg.n_pcs, d_ak,
+                                                c->cfg.mant_bits, V.vs, V.vc, V.vcap - 1, d_small);
+  unsigned long long ovf = 0;
+  e = cudaMemcpyAsync(&ovf, d_small, 8, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d_small, s);
+  cudaFreeAsync(d_ak, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { free_views(V, s); return cuda_fail(c, e, "approx views"); }
+  if (ovf) { free_views(V, s); return fail(c, VE_ERR_CAPACITY, "approx: view table overflow"); }
+  st = view_topk(c, V, s, ndistinct, top);
+  free_views(V, s);
+  return st;
+}
+
 // Warp-aggregated counter increment: lanes with equal keys share one atomic (the
 // per-key counters are few and hot, so plain per-entry atomics serialise).
 // Every lane of the warp must call it; returns this lane's slot (cursor value).

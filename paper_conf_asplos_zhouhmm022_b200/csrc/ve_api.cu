@@ -504,6 +504,38 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
   return VE_OK;
 }
 
+// approximate frequent values (C16; Def 3.3 over Def 3.8's truncation)
+ve_status ve_approx_topk(ve_ctx* c, uint64_t* h_ndistinct, ve_topk_entry* h_top, cudaStream_t s) {
+  if (!ctx_ok(c) || !h_ndistinct || !h_top) return VE_ERR_INVALID;
+  cudaSetDevice(c->device);
+  if (c->poisoned) return fail(c, VE_ERR_STATE, "ve_approx_topk: ctx poisoned by histogram overflow; ve_reset");
+  if (c->hist_merged)
+    return fail(c, VE_ERR_STATE, "ve_approx_topk: the histogram of a rank-merged ctx is partitioned over ranks");
+  ve_status st = dense_flush(c, s);   // counted loads -> exact histogram (idempotent)
+  if (st != VE_OK) return st;
+  const uint32_t nk = c->n_keys, K = c->cfg.topk;
+  std::vector<uint64_t> sum((size_t)nk * NSUM);
+  cudaError_t e = cudaMemcpyAsync(sum.data(), c->t.sum, sum.size() * 8, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_approx_topk");
+  // keys whose records all have one float type (Q15): type codes 8 f16, 9 f32, 10 f64, 11 bf16
+  std::vector<uint8_t> akind(nk, 0xFF);
+  static const uint8_t code[4] = {(2u << 2) | 1u, (2u << 2) | 2u, (2u << 2) | 3u, (3u << 2) | 1u};
+  for (uint32_t k = 0; k < nk; ++k) {
+    int nt = 0, tc = -1;
+    for (int t = 0; t < 12; ++t)
+      if (sum[(size_t)k * NSUM + F_TYPE0 + t]) { ++nt; tc = t; }
+    if (nt == 1 && tc >= 8) akind[k] = code[tc - 8];
+  }
+  std::vector<uint64_t> nd;
+  std::vector<ve_topk_entry> top;
+  st = approx_topk(c, s, akind, nd, top);
+  if (st != VE_OK) return st;
+  for (uint32_t k = 0; k < nk; ++k) h_ndistinct[k] = nd[k];
+  memcpy(h_top, top.data(), (size_t)nk * K * sizeof(ve_topk_entry));
+  return VE_OK;
+}
+
 void ve_report_free(ve_rep* r) { delete r; }
 uint64_t ve_kernel_launches(void) { return g_launches.load(std::memory_order_relaxed); }
 uint32_t ve_report_n_keys(const ve_rep* r) { return r ? r->n_keys : 0; }

@@ -157,6 +157,8 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
 ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s);
 ve_status merge_nccl(ve_ctx* c, void* comm, cudaStream_t s);
 ve_status dense_flush(ve_ctx* c, cudaStream_t s);  // move dense counts into the exact histogram
+ve_status approx_topk(ve_ctx* c, cudaStream_t s, const std::vector<uint8_t>& akind, std::vector<uint64_t>& ndistinct,
+                      std::vector<ve_topk_entry>& top);
 struct ViewTable {                                 // per-key (PC view, object view) value counts
   HSlot* vs = nullptr;
   unsigned long long* vc = nullptr;

@@ -95,6 +95,7 @@ def lib():
             "ve_nccl_comm_init": ([ctypes.POINTER(vp), i32, vp, i32], st),
             "ve_nccl_comm_destroy": ([vp], st),
             "ve_interval_merge": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
+            "ve_approx_topk": ([vp, vp, vp, vp], st),
             "ve_record_intervals": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
         }
@@ -236,6 +237,7 @@ class Context:
             raise VeError(rc, "ve_create")
         self._h = h
         self.n_pcs = n_pcs
+        self.topk = topk
         self._keep = []
 
     def _check(self, rc, what):
@@ -294,6 +296,15 @@ class Context:
         self._check(lib().ve_merge_stats(self._h, other._h if other is not None else None,
                                          ctypes.c_void_p(comm) if comm else None, _stream(stream)),
                     "ve_merge_stats")
+
+    def approx_topk(self, stream=None):
+        """ve_approx_topk: (ndistinct[n_keys], top[n_keys, topk] of TOPK_DTYPE) of the truncated values."""
+        nk = self.n_pcs + getattr(self, "n_objects", 0) + 1
+        nd = np.zeros(nk, dtype=np.uint64)
+        top = np.zeros(nk * self.topk, dtype=TOPK_DTYPE)
+        self._check(lib().ve_approx_topk(self._h, nd.ctypes.data, top.ctypes.data, _stream(stream)),
+                    "ve_approx_topk")
+        return nd, top.reshape(nk, self.topk)
 
     def interval_merge(self, d_in, n, d_out, stream=None):
         """ve_interval_merge: merge n device intervals (16 B each) into d_out; returns the merged count."""
