@@ -177,6 +177,17 @@ ve_status ve_report_globals(const ve_rep* r, ve_globals* out);
 /* format 0: binary (magic "VERP", header, then the arrays above); 1: JSON */
 ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
 
+/* ---- LoadSpy temporal load redundancy in trace order --------
+ * Q1 / R6 (Table 5; LoadSpy, ref [47]): for every valid
+ * global-space load r of the n device records, in array order, let r' be the
+ * most recent earlier valid global-space load of the same address.  r is
+ * temporal if r' exists and temporally redundant if r' also has r's width and
+ * value bits.  h_out[2*key] = temporal, h_out[2*key + 1] = redundant, for the
+ * ctx's n_keys keys (PC key; object key of the object holding addr, from the
+ * ctx's object table).  Order-dependent: one call covers one ordered trace.
+ * n < 2^32.  Synchronizes s. */
+ve_status ve_temporal_loads(ve_ctx* ctx, const ve_record* d_records, uint64_t n, uint64_t* h_out, cudaStream_t s);
+
 /* ---- approximate frequent values ---------------------------
  * Def 3.3 (frequent values) over the truncated values of Def 3.8
  * (P:L191-L193): for every key whose records all have one float type (Q15),

@@ -65,6 +65,7 @@ def lib():
         L.vo_analyze.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_snapshot_diff.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, u32, u32, vp, vp]
         L.vo_object_dedup.argtypes = [vp, u32, vp]
+        L.vo_temporal_loads.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp]
         L.vo_approx_topk.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_interval_merge.argtypes = [vp, u64, vp]
         L.vo_interval_merge.restype = u64
@@ -200,3 +201,13 @@ def approx_topk(cfg, objs, recs):
     if rc != 0:
         raise ValueError("vo_approx_topk rejected its arguments")
     return nd, tb, tc
+
+
+def temporal_loads(cfg, objs, recs):
+    """C17: uint64[n_keys, 2] = (temporal loads, temporally redundant loads) per key."""
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    out = np.zeros((cfg.n_pcs + len(objs) + 1, 2), dtype=np.uint64)
+    if lib().vo_temporal_loads(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), out.ctypes.data) != 0:
+        raise ValueError("vo_temporal_loads rejected its arguments")
+    return out

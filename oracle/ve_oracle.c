@@ -577,6 +577,48 @@ int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of) {
   return 0;
 }
 
+/* ---- C17: LoadSpy temporal load redundancy in record order (f3; Q1, R6) ----
+ * The definition, walked in record order with a table of the last load seen at
+ * every address (open addressing on the address; a plain map). */
+typedef struct { uint64_t addr; uint64_t value; uint32_t w; uint32_t used; } lastload;
+
+int vo_temporal_loads(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                      uint64_t n, uint64_t* out) {
+  if (!cfg || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t n_keys = (uint64_t)cfg->n_pcs + n_obj + 1;
+  memset(out, 0, sizeof(uint64_t) * 2 * n_keys);
+  uint64_t cap = 16;
+  while (cap < 2 * n + 2) cap <<= 1;
+  lastload* tab = (lastload*)calloc(cap, sizeof(lastload));
+  for (uint64_t i = 0; i < n; ++i) {
+    const vo_record* r = &recs[i];
+    dec_t d;
+    decode(cfg, &t, r, &d);
+    if (!d.valid || d.shared || d.store) continue;
+    uint64_t h = (r->addr * 0x9E3779B97F4A7C15ull) >> 17 & (cap - 1);
+    while (tab[h].used && tab[h].addr != r->addr) h = (h + 1) & (cap - 1);
+    if (tab[h].used) {                                     /* r' = the last load of this address */
+      const int red = tab[h].w == d.w && tab[h].value == r->value;
+      out[2 * r->pc]++;
+      out[2 * r->pc + 1] += red;
+      if (d.obj) {
+        const uint64_t ko = (uint64_t)cfg->n_pcs + d.obj->id;
+        out[2 * ko]++;
+        out[2 * ko + 1] += red;
+      }
+    }
+    tab[h].used = 1;
+    tab[h].addr = r->addr;
+    tab[h].value = r->value;
+    tab[h].w = d.w;
+  }
+  free(tab);
+  free(t.by_base);
+  return 0;
+}
+
 /* ---- C16: approximate frequent values (f2; Def 3.3 over Def 3.8) ---------- */
 
 int vo_approx_topk(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,

@@ -149,6 +149,16 @@ uint64_t vo_record_intervals(uint32_t n_pcs, const vo_record* recs, uint64_t n, 
 int vo_plan_copies(const vo_object* objs, uint32_t n_obj, const vo_interval* merged, uint64_t n,
                  uint32_t seg_max, uint32_t dense_pct, vo_copy_plan* plan);
 
+/* ---- LoadSpy temporal load redundancy in trace order --------
+ * Q1 / R6 (Table 5 "redundancy analysis"; LoadSpy, ref [47]): for
+ * every valid global-space load r, in record order, let r' be the most recent
+ * earlier valid global-space load of the same address.  r is *temporal* if r'
+ * exists, and *temporally redundant* if moreover r' has r's width and value
+ * bits.  Counted per key (PC key; object key of r's first byte, unmapped loads
+ * PC only): out[2 * key] = temporal, out[2 * key + 1] = redundant (C17). */
+int vo_temporal_loads(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                      uint64_t n, uint64_t* out);
+
 /* ---- approximate frequent values -------------------------
  * Def 3.3 (frequent values) over the truncated values of Def 3.8
  * ("approximate values ... some fine-grained patterns"): for every

@@ -428,8 +428,17 @@ static void scan_sum(uint32_t* a, uint64_t n, uint32_t* part, cudaStream_t s) {
 }
 
 // Sort + merge the m compacted intervals in (S, E) (ping-pong buffers S2, E2) into d_out.
-static ve_status merge_sorted_pass(ve_ctx* c, uint64_t* S, uint64_t* E, uint64_t* S2, uint64_t* E2, uint64_t m,
-                                   uint8_t* scr, ve_interval* d_out, uint64_t* h_n, cudaStream_t s) {
+// Stable LSD radix sort of the pairs (S[i], E[i]), i < m, by S (ping-pong with S2/E2; on
+// return S/E point at the sorted arrays).  Skipped when S is already non-decreasing.
+// scr: sort_scratch_bytes(m) bytes of device scratch.  Also used by f3 (k_temporal.cu).
+size_t sort_scratch_bytes(uint64_t m) {
+  const uint64_t ntile = (m + IV_TILE - 1) / IV_TILE;
+  const uint64_t nh = ntile * 256;
+  return 64 + 4 * nh + 4 * (nh / SC_TILE + 2) + 16;
+}
+
+ve_status sort_pairs(ve_ctx* c, uint64_t*& S, uint64_t*& E, uint64_t*& S2, uint64_t*& E2, uint64_t m, uint8_t* scr,
+                     cudaStream_t s) {
   unsigned long long* rng = (unsigned long long*)scr;   // [4]
   const unsigned long long init[4] = {~0ull, 0ull, 0ull, 0ull};
   cudaError_t e = cudaMemcpyAsync(rng, init, sizeof(init), cudaMemcpyHostToDevice, s);
@@ -457,6 +466,17 @@ static ve_status merge_sorted_pass(ve_ctx* c, uint64_t* S, uint64_t* E, uint64_t
       std::swap(E, E2);
     }
   }
+  return VE_OK;
+}
+
+static ve_status merge_sorted_pass(ve_ctx* c, uint64_t* S, uint64_t* E, uint64_t* S2, uint64_t* E2, uint64_t m,
+                                   uint8_t* scr, ve_interval* d_out, uint64_t* h_n, cudaStream_t s) {
+  ve_status st = sort_pairs(c, S, E, S2, E2, m, scr, s);
+  if (st != VE_OK) return st;
+  cudaError_t e;
+  const uint64_t ntile = (m + IV_TILE - 1) / IV_TILE;
+  const uint64_t nh = ntile * 256;
+  uint32_t* part = (uint32_t*)(scr + 64) + nh;
   // merge: tile maxima -> exclusive carries, flag counts -> offsets, emit
   unsigned long long* tcar = (unsigned long long*)(((uintptr_t)(part + nh / SC_TILE + 2) + 15) & ~(uintptr_t)15);
   uint32_t* fcnt = (uint32_t*)(tcar + ntile);
@@ -497,11 +517,154 @@ static ve_status iv_alloc(ve_ctx* c, uint64_t cap, uint8_t** buf, cudaStream_t s
   return VE_OK;
 }
 
+// ---- LoadSpy temporal load redundancy in record order (C17) ----------
+// 1. ordered compaction of the valid global-space loads into (address, record index)
+// 2. stable sort by address (sort_pairs): each address's loads stay in record order
+// 3. every sorted neighbour pair of one address is (last load, load): judge it
+__device__ __forceinline__ bool tl_load(const ve_record* r, uint64_t i, uint64_t n, uint32_t n_pcs, uint64_t& addr) {
+  if (i >= n) return false;
+  const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&r[i]);
+  addr = __ldg(q);
+  const uint64_t val = __ldg(q + 1), pm = __ldg(q + 2);
+  const uint32_t meta = (uint32_t)(pm >> 32);
+  return rec_valid(addr, val, (uint32_t)pm, meta, n_pcs) && !meta_shared(meta) && !meta_store(meta);
+}
+
+__global__ void __launch_bounds__(IV_T) k_tl_count(const ve_record* r, uint64_t n, uint32_t n_pcs, uint32_t* cnt) {
+  const uint64_t t0 = (uint64_t)blockIdx.x * IV_TILE;
+  uint32_t c = 0;
+  for (int j = 0; j < IV_ITEMS; ++j) {
+    uint64_t a;
+    c += tl_load(r, t0 + (uint64_t)j * IV_T + threadIdx.x, n, n_pcs, a) ? 1u : 0u;
+  }
+  c = __reduce_add_sync(FULLM, c);
+  __shared__ uint32_t sm[IV_NW];
+  if ((threadIdx.x & 31) == 0) sm[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int k = 0; k < IV_NW; ++k) t += sm[k];
+    cnt[blockIdx.x] = t;
+  }
+}
+
+__global__ void __launch_bounds__(IV_T) k_tl_write(const ve_record* r, uint64_t n, uint32_t n_pcs, const uint32_t* off,
+                                                   uint64_t* S, uint64_t* E) {
+  __shared__ uint32_t sm[IV_NW];
+  const uint64_t t0 = (uint64_t)blockIdx.x * IV_TILE;
+  uint32_t carry = off[blockIdx.x];
+  for (int j = 0; j < IV_ITEMS; ++j) {
+    const uint64_t i = t0 + (uint64_t)j * IV_T + threadIdx.x;
+    uint64_t a = 0;
+    const bool f = tl_load(r, i, n, n_pcs, a);
+    uint32_t tot;
+    const uint32_t ex = block_excl_scan(f ? 1u : 0u, OpAdd(), 0u, sm, tot);
+    if (f) {
+      S[carry + ex] = a;
+      E[carry + ex] = i;
+    }
+    carry += tot;
+  }
+}
+
+// out[2 * key] += temporal, out[2 * key + 1] += redundant; lanes of equal keys share one atomic
+__device__ __forceinline__ void tl_add(unsigned long long* out, bool act, uint32_t key, uint32_t red) {
+  const unsigned am = __ballot_sync(FULLM, act);
+  if (!act) return;
+  const unsigned g = __match_any_sync(am, key);
+  const uint32_t nr = __popc(__ballot_sync(g, red != 0u) & g);
+  if ((int)(threadIdx.x & 31) == __ffs(g) - 1) {
+    atomicAdd(&out[2 * (uint64_t)key], (unsigned long long)__popc(g));
+    if (nr) atomicAdd(&out[2 * (uint64_t)key + 1], (unsigned long long)nr);
+  }
+}
+
+__global__ void __launch_bounds__(IV_T) k_tl_judge(const ve_record* r, const uint64_t* S, const uint64_t* E,
+                                                   uint64_t m, const uint64_t* ob, const uint64_t* oe,
+                                                   const uint32_t* oid, uint32_t nobj, uint32_t n_pcs,
+                                                   unsigned long long* out) {
+  const uint64_t stride = (uint64_t)gridDim.x * IV_T;
+  for (uint64_t b = (uint64_t)blockIdx.x * IV_T; b < m; b += stride) {   // warp-uniform trip count
+    const uint64_t j = b + threadIdx.x;
+    bool temporal = false;
+    uint32_t red = 0, pc = 0, okey = 0;
+    bool has_obj = false;
+    if (j > 0 && j < m && S[j] == S[j - 1]) {
+      temporal = true;
+      const unsigned long long* qi = reinterpret_cast<const unsigned long long*>(&r[E[j]]);
+      const unsigned long long* qp = reinterpret_cast<const unsigned long long*>(&r[E[j - 1]]);
+      const uint64_t vi = __ldg(qi + 1), pmi = __ldg(qi + 2), vp = __ldg(qp + 1), pmp = __ldg(qp + 2);
+      red = (vi == vp && ((pmi >> 32) & 3u) == ((pmp >> 32) & 3u)) ? 1u : 0u;
+      pc = (uint32_t)pmi;
+      const uint64_t a = S[j];
+      uint32_t lo = 0, hi = nobj;          // first object with base > a
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (ob[mid] <= a) lo = mid + 1; else hi = mid;
+      }
+      if (lo > 0 && a < oe[lo - 1]) { has_obj = true; okey = n_pcs + oid[lo - 1]; }
+    }
+    tl_add(out, temporal, pc, red);
+    tl_add(out, has_obj, okey, red);
+  }
+}
+
 }  // namespace ve
 
 using namespace ve;
 
 extern "C" {
+
+ve_status ve_temporal_loads(ve_ctx* c, const ve_record* d_records, uint64_t n, uint64_t* h_out, cudaStream_t s) {
+  if (!c || !h_out) return VE_ERR_INVALID;
+  const uint32_t nk = c->n_keys;
+  memset(h_out, 0, sizeof(uint64_t) * 2 * nk);
+  if (n == 0) return VE_OK;
+  if (!d_records || ((uintptr_t)d_records & 7)) return fail(c, VE_ERR_INVALID, "ve_temporal_loads: null or misaligned");
+  if (n >= (1ull << 32)) return fail(c, VE_ERR_INVALID, "ve_temporal_loads: n >= 2^32");
+  cudaSetDevice(c->device);
+  const uint64_t ntile = (n + IV_TILE - 1) / IV_TILE;
+  const size_t need = 32 * n + sort_scratch_bytes(n) + 4 * ntile + 4 * (ntile / SC_TILE + 2) + 16 * (size_t)nk + 64;
+  uint8_t* buf = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&buf, need, s);
+  if (e != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "ve_temporal_loads: workspace"); }
+  uint64_t* S = (uint64_t*)buf;
+  uint64_t* E = S + n;
+  uint64_t* S2 = E + n;
+  uint64_t* E2 = S2 + n;
+  uint8_t* scr = (uint8_t*)(E2 + n);
+  uint32_t* tcnt = (uint32_t*)(scr + sort_scratch_bytes(n));
+  uint32_t* part = tcnt + ntile;
+  unsigned long long* d_out =
+      (unsigned long long*)(((uintptr_t)(part + ntile / SC_TILE + 2) + 15) & ~(uintptr_t)15);
+  count_launch();
+  k_tl_count<<<(unsigned)ntile, IV_T, 0, s>>>(d_records, n, c->cfg.n_pcs, tcnt);
+  uint32_t last = 0, last_off = 0;
+  cudaMemcpyAsync(&last, tcnt + ntile - 1, 4, cudaMemcpyDeviceToHost, s);
+  scan_sum(tcnt, ntile, part, s);
+  cudaMemcpyAsync(&last_off, tcnt + ntile - 1, 4, cudaMemcpyDeviceToHost, s);
+  count_launch();
+  k_tl_write<<<(unsigned)ntile, IV_T, 0, s>>>(d_records, n, c->cfg.n_pcs, tcnt, S, E);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) { cudaFreeAsync(buf, s); return cuda_fail(c, e, "ve_temporal_loads: compaction"); }
+  const uint64_t m = (uint64_t)last_off + last;
+  ve_status st = VE_OK;
+  if (m > 1) {
+    st = sort_pairs(c, S, E, S2, E2, m, scr, s);
+    if (st == VE_OK) {
+      cudaMemsetAsync(d_out, 0, 16 * (size_t)nk, s);
+      count_launch();
+      k_tl_judge<<<grid_for(c, IV_T, m), IV_T, 0, s>>>(d_records, S, E, m, c->o.base, c->o.end, c->o.id, c->n_obj,
+                                                       c->cfg.n_pcs, d_out);
+      e = cudaMemcpyAsync(h_out, d_out, 16 * (size_t)nk, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) st = cuda_fail(c, e, "ve_temporal_loads");
+    }
+  }
+  cudaFreeAsync(buf, s);
+  return st;
+}
+
 
 ve_status ve_interval_merge(ve_ctx* c, const ve_interval* d_in, uint64_t n, ve_interval* d_out, uint64_t* h_n_out,
                             cudaStream_t s) {

@@ -170,6 +170,9 @@ void free_views(ViewTable& V, cudaStream_t s);
 ve_status view_topk(ve_ctx* c, const ViewTable& V, cudaStream_t s, std::vector<uint64_t>& ndistinct,
                     std::vector<ve_topk_entry>& top);
 void count_launch();  // process-wide kernel launch counter (ve_kernel_launches)
+size_t sort_scratch_bytes(uint64_t m);              // k_interval.cu: stable LSD radix sort of u64 pairs
+ve_status sort_pairs(ve_ctx* c, uint64_t*& S, uint64_t*& E, uint64_t*& S2, uint64_t*& E2, uint64_t m, uint8_t* scr,
+                     cudaStream_t s);
 }  // namespace ve
 
 // ============================================================================

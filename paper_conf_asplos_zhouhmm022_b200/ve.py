@@ -96,6 +96,7 @@ def lib():
             "ve_nccl_comm_destroy": ([vp], st),
             "ve_interval_merge": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_approx_topk": ([vp, vp, vp, vp], st),
+            "ve_temporal_loads": ([vp, vp, u64, vp, vp], st),
             "ve_record_intervals": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
         }
@@ -305,6 +306,14 @@ class Context:
         self._check(lib().ve_approx_topk(self._h, nd.ctypes.data, top.ctypes.data, _stream(stream)),
                     "ve_approx_topk")
         return nd, top.reshape(nk, self.topk)
+
+    def temporal_loads(self, d_records, n, stream=None):
+        """ve_temporal_loads: uint64[n_keys, 2] = (temporal, temporally redundant) loads per key."""
+        nk = self.n_pcs + getattr(self, "n_objects", 0) + 1
+        out = np.zeros((nk, 2), dtype=np.uint64)
+        self._check(lib().ve_temporal_loads(self._h, _ptr(d_records), n, out.ctypes.data, _stream(stream)),
+                    "ve_temporal_loads")
+        return out
 
     def interval_merge(self, d_in, n, d_out, stream=None):
         """ve_interval_merge: merge n device intervals (16 B each) into d_out; returns the merged count."""
