@@ -319,7 +319,7 @@ def main():
 
     f1 = None
     if rank == 0 and not args.no_f1:
-        f1 = measure_f1(ve, ctx, wl, stream, peak)
+        f1 = measure_next_rows(ve, ctx, wl, stream, peak)
 
     dd5 = None
     if rank == 0 and not args.no_cfg5:
@@ -348,35 +348,57 @@ def main():
                              "alg_bytes_per_launch": alg[1]},
                 "analyze_ms_per_step": [round(statistics.mean(a[i] for a in an_ms), 4) for i in (0, 1)],
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
-                "f1_record_intervals": f1, "cfg5_dedup": dd5,
+                "next_rows": f1, "cfg5_dedup": dd5,
                 "parity_spot_check": spot}
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
 
 
-def measure_f1(ve, ctx, wl, stream, peak, reps=3):
-    """SURVEY 8(f) f1, measured outside the step: ve_record_intervals (warp compaction, radix sort,
-    merge scans) over this rank's gemm-epoch records; device time by CUDA events around the call."""
+def measure_next_rows(ve, ctx, wl, stream, peak, reps=3):
+    """SURVEY 8(f) rows, measured outside the step on this rank's cfg2 gemm-epoch records (CUDA events
+    around each synchronizing call, median of `reps`):
+      f1 ve_record_intervals (warp compaction, radix sort, merge scans),
+      f2 ve_approx_topk on the ctx's gemm-epoch histogram (re-keyed by truncated value),
+      f3 ve_temporal_loads (ordered load compaction, radix sort by address, neighbour judging)."""
     import torch
     e = wl.epochs[1]
     n = e["n"]
+    sp = stream.cuda_stream
+
+    def timed(fn):
+        fn()                                    # warm-up (workspace pool)
+        ts, r = [], None
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            a.record(stream)
+            r = fn()
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        return statistics.median(ts), r
+
     out = torch.empty(n * 16, dtype=torch.uint8, device=wl.device)
-    ctx.record_intervals(e["recs"], n, out, stream=stream.cuda_stream)   # warm-up (workspace pool)
-    ts, k = [], 0
-    for _ in range(reps):
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        torch.cuda.synchronize()
-        a.record(stream)
-        k = ctx.record_intervals(e["recs"], n, out, stream=stream.cuda_stream)
-        b.record(stream)
-        torch.cuda.synchronize()
-        ts.append(a.elapsed_time(b))
-    ms = statistics.median(ts)
+    ms1, k = timed(lambda: ctx.record_intervals(e["recs"], n, out, stream=sp))
     del out
-    return {"records": n, "ms": ms, "records_per_s": n / (ms / 1e3), "merged_intervals": k,
-            "trace_gbs": n * REC_BYTES / (ms / 1e3) / 1e9, "frac_of_hbm_peak": n * REC_BYTES / (ms / 1e3) / 1e9 / peak,
-            "note": "f1 leg, not part of the step; the call synchronizes (count read-backs) inside the timed region"}
+    ctx.set_objects(e["objs"])
+    ctx.analyze_records(e["recs"], n, stream=sp)
+    ms2, (nd, _top) = timed(lambda: ctx.approx_topk(stream=sp))
+    ms3, tl = timed(lambda: ctx.temporal_loads(e["recs"], n, stream=sp))
+    gbs = lambda ms: n * REC_BYTES / (ms / 1e3) / 1e9
+    return {
+        "note": "SURVEY 8(f) rows, not part of the step; each call synchronizes (count read-backs) inside its "
+                "timed region",
+        "f1_record_intervals": {"records": n, "ms": ms1, "records_per_s": n / (ms1 / 1e3), "trace_gbs": gbs(ms1),
+                                "frac_of_hbm_peak": gbs(ms1) / peak, "merged_intervals": k},
+        "f2_approx_topk": {"ms": ms2, "keys_with_approx_histogram": int((nd > 0).sum()),
+                           "approx_distinct_total": int(nd.sum())},
+        "f3_temporal_loads": {"records": n, "ms": ms3, "records_per_s": n / (ms3 / 1e3), "trace_gbs": gbs(ms3),
+                              "frac_of_hbm_peak": gbs(ms3) / peak, "temporal_loads_pc": [int(x) for x in tl[:5, 0]],
+                              "closed_form_ok": bool(int(tl[1, 1]) == 363 * 256 * 1152
+                                                     and int(tl[2, 1]) == 15 * 1152 * 5776)},
+    }
 
 
 def measure_cfg5_dedup(ve, ctx, stream, peak, reps=3):

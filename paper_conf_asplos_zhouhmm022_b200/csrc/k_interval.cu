@@ -222,7 +222,11 @@ __global__ void __launch_bounds__(IV_T) k_rs_scatter(const uint64_t* __restrict_
     __syncwarp();
   }
   __syncthreads();
-  {   // exclusive prefix over the warps of the tile, per digit
+  // per digit: exclusive prefix over the warps of the tile, and the tile-local start of
+  // the digit (exclusive scan of the digit totals over the 256 threads)
+  __shared__ uint32_t ls[256];
+  __shared__ uint32_t wsum[IV_NW];
+  {
     const int d = threadIdx.x;
     uint32_t run = 0;
     for (int k = 0; k < IV_NW; ++k) {
@@ -230,15 +234,39 @@ __global__ void __launch_bounds__(IV_T) k_rs_scatter(const uint64_t* __restrict_
       wc[k][d] = run;
       run += c;
     }
+    uint32_t x = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULLM, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[w] = x;
+    __syncthreads();
+    uint32_t pre = 0;
+    for (int k = 0; k < w; ++k) pre += wsum[k];
+    ls[d] = pre + x - run;
   }
   __syncthreads();
+  // stage the tile in shared memory in (digit, rank) order, then write every digit's run
+  // out contiguously: consecutive threads store consecutive addresses
+  __shared__ uint64_t sk[IV_TILE], sv[IV_TILE];
 #pragma unroll
   for (int j = 0; j < IV_ITEMS; ++j) {
     if (dg[j] < 256u) {
-      const uint64_t p = (uint64_t)go[dg[j]] + wc[w][dg[j]] + rk[j];
-      So[p] = s[j];
-      Eo[p] = e[j];
+      const uint32_t lp = ls[dg[j]] + wc[w][dg[j]] + rk[j];
+      sk[lp] = s[j];
+      sv[lp] = e[j];
     }
+  }
+  __syncthreads();
+  const uint64_t t0 = (uint64_t)blockIdx.x * IV_TILE;
+  const uint32_t nv = (uint32_t)(n - t0 < (uint64_t)IV_TILE ? n - t0 : (uint64_t)IV_TILE);
+  for (uint32_t idx = threadIdx.x; idx < nv; idx += IV_T) {
+    const uint64_t key = sk[idx];
+    const uint32_t d = rs_digit(key, kmin, shift);
+    const uint64_t p = (uint64_t)go[d] + (idx - ls[d]);
+    So[p] = key;
+    Eo[p] = sv[idx];
   }
 }
 
@@ -520,7 +548,8 @@ static ve_status iv_alloc(ve_ctx* c, uint64_t cap, uint8_t** buf, cudaStream_t s
 // ---- LoadSpy temporal load redundancy in record order (C17) ----------
 // 1. ordered compaction of the valid global-space loads into (address, record index)
 // 2. stable sort by address (sort_pairs): each address's loads stay in record order
-// 3. every sorted neighbour pair of one address is (last load, load): judge it
+// 3. gather each sorted load's value / meta (one random read per load), then judge every
+//    sorted neighbour pair of one address, i.e. (last load, load), sequentially
 __device__ __forceinline__ bool tl_load(const ve_record* r, uint64_t i, uint64_t n, uint32_t n_pcs, uint64_t& addr) {
   if (i >= n) return false;
   const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&r[i]);
@@ -567,34 +596,66 @@ __global__ void __launch_bounds__(IV_T) k_tl_write(const ve_record* r, uint64_t 
   }
 }
 
-// out[2 * key] += temporal, out[2 * key + 1] += redundant; lanes of equal keys share one atomic
-__device__ __forceinline__ void tl_add(unsigned long long* out, bool act, uint32_t key, uint32_t red) {
+// (temporal, redundant) += (group size, redundant lanes) for key; lanes of equal keys share one
+// update, into the block's shared counters for keys < TL_SK (flushed at exit), else global
+constexpr uint32_t TL_SK = 1024;
+__device__ __forceinline__ void tl_add(uint32_t* sc, unsigned long long* out, bool act, uint32_t key, uint32_t red) {
   const unsigned am = __ballot_sync(FULLM, act);
   if (!act) return;
   const unsigned g = __match_any_sync(am, key);
   const uint32_t nr = __popc(__ballot_sync(g, red != 0u) & g);
   if ((int)(threadIdx.x & 31) == __ffs(g) - 1) {
-    atomicAdd(&out[2 * (uint64_t)key], (unsigned long long)__popc(g));
-    if (nr) atomicAdd(&out[2 * (uint64_t)key + 1], (unsigned long long)nr);
+    if (key < TL_SK) {
+      atomicAdd(&sc[2 * key], (uint32_t)__popc(g));
+      if (nr) atomicAdd(&sc[2 * key + 1], nr);
+    } else {
+      atomicAdd(&out[2 * (uint64_t)key], (unsigned long long)__popc(g));
+      if (nr) atomicAdd(&out[2 * (uint64_t)key + 1], (unsigned long long)nr);
+    }
   }
 }
 
-__global__ void __launch_bounds__(IV_T) k_tl_judge(const ve_record* r, const uint64_t* S, const uint64_t* E,
+// sorted position j -> the value bits and (pc | meta << 32) of its record: the one random
+// gather of the pass (the judge then reads neighbours sequentially)
+__global__ void __launch_bounds__(IV_T) k_tl_gather(const ve_record* r, const uint64_t* E, uint64_t m, uint64_t* V,
+                                                    uint64_t* PM) {
+  const uint64_t stride = (uint64_t)gridDim.x * IV_T;
+  uint64_t j = (uint64_t)blockIdx.x * IV_T + threadIdx.x;
+  for (; j + 3 * stride < m; j += 4 * stride) {     // four random reads in flight per thread
+    uint64_t v[4], pm[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&r[E[j + u * stride]]);
+      v[u] = __ldg(q + 1);
+      pm[u] = __ldg(q + 2);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) { V[j + u * stride] = v[u]; PM[j + u * stride] = pm[u]; }
+  }
+  for (; j < m; j += stride) {
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&r[E[j]]);
+    V[j] = __ldg(q + 1);
+    PM[j] = __ldg(q + 2);
+  }
+}
+
+__global__ void __launch_bounds__(IV_T) k_tl_judge(const uint64_t* S, const uint64_t* V, const uint64_t* PM,
                                                    uint64_t m, const uint64_t* ob, const uint64_t* oe,
                                                    const uint32_t* oid, uint32_t nobj, uint32_t n_pcs,
                                                    unsigned long long* out) {
+  __shared__ uint32_t sc[2 * TL_SK];   // per-block counters of the first TL_SK keys (< 2^32 per block)
+  for (uint32_t i = threadIdx.x; i < 2 * TL_SK; i += IV_T) sc[i] = 0;
+  __syncthreads();
   const uint64_t stride = (uint64_t)gridDim.x * IV_T;
-  for (uint64_t b = (uint64_t)blockIdx.x * IV_T; b < m; b += stride) {   // warp-uniform trip count
+  for (uint64_t b = (uint64_t)blockIdx.x * IV_T; b < m; b += stride) {   // block-uniform trip count
     const uint64_t j = b + threadIdx.x;
     bool temporal = false;
     uint32_t red = 0, pc = 0, okey = 0;
     bool has_obj = false;
     if (j > 0 && j < m && S[j] == S[j - 1]) {
       temporal = true;
-      const unsigned long long* qi = reinterpret_cast<const unsigned long long*>(&r[E[j]]);
-      const unsigned long long* qp = reinterpret_cast<const unsigned long long*>(&r[E[j - 1]]);
-      const uint64_t vi = __ldg(qi + 1), pmi = __ldg(qi + 2), vp = __ldg(qp + 1), pmp = __ldg(qp + 2);
-      red = (vi == vp && ((pmi >> 32) & 3u) == ((pmp >> 32) & 3u)) ? 1u : 0u;
+      const uint64_t pmi = PM[j], pmp = PM[j - 1];
+      red = (V[j] == V[j - 1] && ((pmi >> 32) & 3u) == ((pmp >> 32) & 3u)) ? 1u : 0u;
       pc = (uint32_t)pmi;
       const uint64_t a = S[j];
       uint32_t lo = 0, hi = nobj;          // first object with base > a
@@ -604,9 +665,12 @@ __global__ void __launch_bounds__(IV_T) k_tl_judge(const ve_record* r, const uin
       }
       if (lo > 0 && a < oe[lo - 1]) { has_obj = true; okey = n_pcs + oid[lo - 1]; }
     }
-    tl_add(out, temporal, pc, red);
-    tl_add(out, has_obj, okey, red);
+    tl_add(sc, out, temporal, pc, red);
+    tl_add(sc, out, has_obj, okey, red);
   }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < 2 * TL_SK; i += IV_T)
+    if (sc[i]) atomicAdd(&out[i], (unsigned long long)sc[i]);
 }
 
 }  // namespace ve
@@ -654,7 +718,9 @@ ve_status ve_temporal_loads(ve_ctx* c, const ve_record* d_records, uint64_t n, u
     if (st == VE_OK) {
       cudaMemsetAsync(d_out, 0, 16 * (size_t)nk, s);
       count_launch();
-      k_tl_judge<<<grid_for(c, IV_T, m), IV_T, 0, s>>>(d_records, S, E, m, c->o.base, c->o.end, c->o.id, c->n_obj,
+      k_tl_gather<<<grid_for(c, IV_T, m), IV_T, 0, s>>>(d_records, E, m, S2, E2);   // the sort's spare buffers
+      count_launch();
+      k_tl_judge<<<grid_for(c, IV_T, m), IV_T, 0, s>>>(S, S2, E2, m, c->o.base, c->o.end, c->o.id, c->n_obj,
                                                        c->cfg.n_pcs, d_out);
       e = cudaMemcpyAsync(h_out, d_out, 16 * (size_t)nk, cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaStreamSynchronize(s);
