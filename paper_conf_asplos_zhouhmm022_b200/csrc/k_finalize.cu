@@ -798,7 +798,10 @@ ve_status finalize_hist_views(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& 
 // shared table) so runs of equal values (zero-filled regions) cost one global insert.
 constexpr int DF_THREADS = 256;
 constexpr int DF_SLOTS = 1024;
-constexpr uint64_t DF_CHUNK = 1024;    // elements per block: many blocks keep the global inserts in flight
+#ifndef VE_DF_CHUNK
+#define VE_DF_CHUNK 1024
+#endif
+constexpr uint64_t DF_CHUNK = VE_DF_CHUNK;    // elements per block: many blocks keep the global inserts in flight
 
 // The value statistics of the counted loads (C1 n_zero, C5 flags and ord range, C4 raw
 // range, C7 truncated range) are taken here too, once per element weighted by its
