@@ -239,6 +239,55 @@ ve_status ve_record_intervals(ve_ctx* ctx, const ve_record* d_records, uint64_t 
 ve_status ve_plan_copies(ve_ctx* ctx, const ve_interval* d_merged, uint64_t n, uint32_t seg_max,
                          uint32_t dense_pct, ve_copy_plan* h_plan, cudaStream_t s);
 
+/* ---- value flow graph (Defs 5.1-5.3) ----------
+ * Host-side bookkeeping over an API-event log (no device work, no ctx).  The
+ * log is the program-order list of data-object accesses of GPU API
+ * invocations; accesses of one invocation share a sequence number.  Readings
+ * R7-R9 in DESIGN.md section 3. */
+#define VE_HOST_VERTEX 0xFFFFFFFFu                 /* v_host */
+enum { VE_ACC_READ = 1, VE_ACC_WRITE = 2 };         /* edge labels (bit set)                     */
+enum { VE_EV_DEVICE = 0, VE_EV_ALLOC = 1, VE_EV_H2D = 2, VE_EV_D2H = 3 };
+
+typedef struct ve_api_access {
+  uint64_t seq;        /* invocation sequence number, non-decreasing over the log         */
+  uint64_t bytes;      /* bytes accessed: the edge importance I(e)                */
+  uint32_t vertex;     /* vertex id = the API's call path: equal ids merge        */
+  uint32_t object;     /* data object id (dense, < 2^32 - 1)                              */
+  uint32_t mode;       /* VE_ACC_READ | VE_ACC_WRITE (ALLOC / H2D imply WRITE, D2H READ)   */
+  uint32_t kind;       /* VE_EV_*: ALLOC creates the object (its first writer);   */
+                       /* H2D adds a source edge host -> vertex, D2H a sink edge vertex -> host */
+} ve_api_access;
+
+typedef struct ve_vfg_edge {
+  uint32_t src, dst;   /* vertex ids; VE_HOST_VERTEX for source / sink edges              */
+  uint32_t object;     /* D_{v_k}                                                         */
+  uint32_t label;      /* VE_ACC_* of the accessing (dst) side, ORed over merged invocations */
+  uint64_t bytes;      /* summed accessed bytes                                           */
+  uint64_t count;      /* invocations merged into the edge                                */
+} ve_vfg_edge;
+
+typedef struct ve_vfg_vertex {
+  uint32_t vertex, pad;
+  uint64_t invocations;   /* I(v) */
+} ve_vfg_vertex;
+
+typedef struct ve_vfg ve_vfg;   /* opaque, host memory */
+
+/* Def 5.1: build the graph.  VE_ERR_INVALID if seq decreases or an object is
+ * accessed before its allocation.  Edges sorted by (src, dst, object),
+ * vertices by id (v_host not listed). */
+ve_status ve_vfg_build(const ve_api_access* log, uint64_t n, ve_vfg** out);
+/* Def 5.2: the vertex slice graph of vertex v (VE_ERR_INVALID if v is absent). */
+ve_status ve_vfg_slice(const ve_vfg* g, uint32_t v, ve_vfg** out);
+/* Def 5.3: edges with bytes >= min_edge_bytes; vertices on a kept edge or with
+ * invocations >= min_vertex_invocations. */
+ve_status ve_vfg_important(const ve_vfg* g, uint64_t min_edge_bytes, uint64_t min_vertex_invocations,
+                           ve_vfg** out);
+ve_status ve_vfg_size(const ve_vfg* g, uint64_t* n_vertices, uint64_t* n_edges);
+ve_status ve_vfg_vertices(const ve_vfg* g, ve_vfg_vertex* out);   /* n_vertices entries */
+ve_status ve_vfg_edges(const ve_vfg* g, ve_vfg_edge* out);         /* n_edges entries    */
+void      ve_vfg_free(ve_vfg* g);
+
 /* Number of libve kernels launched by this process so far (all contexts). */
 uint64_t  ve_kernel_launches(void);
 

@@ -65,6 +65,9 @@ def lib():
         L.vo_analyze.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_snapshot_diff.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, u32, u32, vp, vp]
         L.vo_object_dedup.argtypes = [vp, u32, vp]
+        L.vo_vfg_build.argtypes = [vp, u64, vp, vp, vp, vp]
+        L.vo_vfg_slice.argtypes = [vp, u64, vp, u64, u32, vp, vp, vp, vp]
+        L.vo_vfg_important.argtypes = [vp, u64, vp, u64, u64, u64, vp, vp, vp, vp]
         L.vo_temporal_loads.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp]
         L.vo_approx_topk.argtypes = [ctypes.POINTER(VoConfig), vp, u32, vp, u64, vp, vp, vp]
         L.vo_interval_merge.argtypes = [vp, u64, vp]
@@ -211,3 +214,46 @@ def temporal_loads(cfg, objs, recs):
     if lib().vo_temporal_loads(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), out.ctypes.data) != 0:
         raise ValueError("vo_temporal_loads rejected its arguments")
     return out
+
+
+# ---- C18-C20: value flow graph (layouts of ve.h's ve_api_access / ve_vfg_edge / ve_vfg_vertex)
+HOST_VERTEX = 0xFFFFFFFF
+ACCESS_DTYPE = np.dtype([("seq", "<u8"), ("bytes", "<u8"), ("vertex", "<u4"), ("object", "<u4"), ("mode", "<u4"),
+                         ("kind", "<u4")])
+VFG_EDGE_DTYPE = np.dtype([("src", "<u4"), ("dst", "<u4"), ("object", "<u4"), ("label", "<u4"), ("bytes", "<u8"),
+                           ("count", "<u8")])
+VFG_VERTEX_DTYPE = np.dtype([("vertex", "<u4"), ("pad", "<u4"), ("invocations", "<u8")])
+
+
+def vfg_build(log):
+    """C18 (Def 5.1): (edges, vertices) of an ACCESS_DTYPE log."""
+    log = np.ascontiguousarray(log, dtype=ACCESS_DTYPE)
+    n = len(log)
+    e = np.zeros(2 * n + 1, dtype=VFG_EDGE_DTYPE)
+    v = np.zeros(n + 1, dtype=VFG_VERTEX_DTYPE)
+    ne, nv = ctypes.c_uint64(), ctypes.c_uint64()
+    if lib().vo_vfg_build(log.ctypes.data, n, e.ctypes.data, ctypes.byref(ne), v.ctypes.data, ctypes.byref(nv)) != 0:
+        raise ValueError("vo_vfg_build: an access before its allocation")
+    return e[:ne.value], v[:nv.value]
+
+
+def vfg_slice(edges, verts, vertex):
+    """C19 (Def 5.2): the vertex slice graph of `vertex`."""
+    edges, verts = np.ascontiguousarray(edges), np.ascontiguousarray(verts)
+    oe = np.zeros(len(edges) + 1, dtype=VFG_EDGE_DTYPE)
+    ov = np.zeros(len(verts) + 1, dtype=VFG_VERTEX_DTYPE)
+    ne, nv = ctypes.c_uint64(), ctypes.c_uint64()
+    lib().vo_vfg_slice(edges.ctypes.data, len(edges), verts.ctypes.data, len(verts), vertex, oe.ctypes.data,
+                       ctypes.byref(ne), ov.ctypes.data, ctypes.byref(nv))
+    return oe[:ne.value], ov[:nv.value]
+
+
+def vfg_important(edges, verts, min_edge_bytes, min_vertex_invocations):
+    """C20 (Def 5.3): the important graph."""
+    edges, verts = np.ascontiguousarray(edges), np.ascontiguousarray(verts)
+    oe = np.zeros(len(edges) + 1, dtype=VFG_EDGE_DTYPE)
+    ov = np.zeros(len(verts) + 1, dtype=VFG_VERTEX_DTYPE)
+    ne, nv = ctypes.c_uint64(), ctypes.c_uint64()
+    lib().vo_vfg_important(edges.ctypes.data, len(edges), verts.ctypes.data, len(verts), min_edge_bytes,
+                           min_vertex_invocations, oe.ctypes.data, ctypes.byref(ne), ov.ctypes.data, ctypes.byref(nv))
+    return oe[:ne.value], ov[:nv.value]

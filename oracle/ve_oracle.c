@@ -577,6 +577,144 @@ int vo_object_dedup(const vo_object* objs, uint32_t n, uint32_t* group_of) {
   return 0;
 }
 
+/* ---- C18-C20: value flow graph (f4; Defs 5.1-5.3) ------------- */
+
+enum { VO_ACC_R = 1, VO_ACC_W = 2, VO_EV_DEV = 0, VO_EV_ALLOC = 1, VO_EV_H2D = 2, VO_EV_D2H = 3 };
+
+static int vo_writes(const vo_access* a, uint32_t k) {
+  return a->object == k && (a->kind == VO_EV_ALLOC || a->kind == VO_EV_H2D || (a->kind == VO_EV_DEV && (a->mode & VO_ACC_W)));
+}
+
+static void vo_edge_add(vo_vfg_edge* E, uint64_t* ne, uint64_t* last, uint32_t src, uint32_t dst, uint32_t k,
+                        uint32_t label, uint64_t bytes, uint64_t seq) {
+  for (uint64_t i = 0; i < *ne; ++i)
+    if (E[i].src == src && E[i].dst == dst && E[i].object == k) {
+      E[i].label |= label;
+      E[i].bytes += bytes;
+      if (last[i] != seq) { E[i].count++; last[i] = seq; }
+      return;
+    }
+  E[*ne].src = src; E[*ne].dst = dst; E[*ne].object = k; E[*ne].label = label;
+  E[*ne].bytes = bytes; E[*ne].count = 1;
+  last[*ne] = seq;
+  (*ne)++;
+}
+
+static int cmp_edge(const void* a, const void* b) {
+  const vo_vfg_edge* x = (const vo_vfg_edge*)a;
+  const vo_vfg_edge* y = (const vo_vfg_edge*)b;
+  if (x->src != y->src) return (x->src > y->src) - (x->src < y->src);
+  if (x->dst != y->dst) return (x->dst > y->dst) - (x->dst < y->dst);
+  return (x->object > y->object) - (x->object < y->object);
+}
+static int cmp_vertex(const void* a, const void* b) {
+  const vo_vfg_vertex* x = (const vo_vfg_vertex*)a;
+  const vo_vfg_vertex* y = (const vo_vfg_vertex*)b;
+  return (x->vertex > y->vertex) - (x->vertex < y->vertex);
+}
+
+int vo_vfg_build(const vo_access* log, uint64_t n, vo_vfg_edge* edges, uint64_t* ne, vo_vfg_vertex* verts,
+                 uint64_t* nv) {
+  uint64_t* last = (uint64_t*)malloc(sizeof(uint64_t) * (2 * n + 1));
+  *ne = 0;
+  *nv = 0;
+  for (uint64_t j = 0; j < n; ++j) {
+    const vo_access* a = &log[j];
+    /* I(v): the number of distinct invocations (sequence numbers) of the vertex */
+    int first = 1;
+    for (uint64_t i = 0; i < j; ++i)
+      if (log[i].vertex == a->vertex && log[i].seq == a->seq) first = 0;
+    if (first) {
+      uint64_t q = 0;
+      while (q < *nv && verts[q].vertex != a->vertex) ++q;
+      if (q == *nv) { verts[q].vertex = a->vertex; verts[q].pad = 0; verts[q].invocations = 0; (*nv)++; }
+      verts[q].invocations++;
+    }
+    if (a->kind == VO_EV_ALLOC) continue;
+    /* Def 5.1: v_i writes D_k and no v_u writes D_k after it and before v_j */
+    int64_t w = -1;
+    for (int64_t i = (int64_t)j - 1; i >= 0; --i)
+      if (log[i].seq < a->seq && vo_writes(&log[i], a->object)) { w = i; break; }
+    if (w < 0) { free(last); return -1; }
+    uint32_t mode = a->mode & (VO_ACC_R | VO_ACC_W);
+    if (a->kind == VO_EV_H2D) mode = VO_ACC_W;
+    if (a->kind == VO_EV_D2H) mode = VO_ACC_R;
+    vo_edge_add(edges, ne, last, log[w].vertex, a->vertex, a->object, mode, a->bytes, a->seq);
+    if (a->kind == VO_EV_H2D) vo_edge_add(edges, ne, last, VO_HOST, a->vertex, a->object, VO_ACC_W, a->bytes, a->seq);
+    if (a->kind == VO_EV_D2H) vo_edge_add(edges, ne, last, a->vertex, VO_HOST, a->object, VO_ACC_R, a->bytes, a->seq);
+  }
+  free(last);
+  qsort(edges, *ne, sizeof(vo_vfg_edge), cmp_edge);
+  qsort(verts, *nv, sizeof(vo_vfg_vertex), cmp_vertex);
+  return 0;
+}
+
+static int in_set(const uint32_t* s, uint64_t n, uint32_t x) {
+  for (uint64_t i = 0; i < n; ++i) if (s[i] == x) return 1;
+  return 0;
+}
+
+static void vo_keep_vertices(const vo_vfg_edge* oe, uint64_t one, const vo_vfg_vertex* verts, uint64_t nv,
+                             vo_vfg_vertex* ov, uint64_t* onv, uint64_t min_inv) {
+  *onv = 0;
+  for (uint64_t q = 0; q < nv; ++q) {
+    int on = verts[q].invocations >= min_inv;
+    for (uint64_t i = 0; i < one && !on; ++i) on = oe[i].src == verts[q].vertex || oe[i].dst == verts[q].vertex;
+    if (on) ov[(*onv)++] = verts[q];
+  }
+}
+
+int vo_vfg_slice(const vo_vfg_edge* edges, uint64_t ne, const vo_vfg_vertex* verts, uint64_t nv, uint32_t v,
+                 vo_vfg_edge* oe, uint64_t* one, vo_vfg_vertex* ov, uint64_t* onv) {
+  *one = 0;
+  uint32_t* rin = (uint32_t*)malloc(sizeof(uint32_t) * (2 * ne + 2));
+  uint32_t* rout = (uint32_t*)malloc(sizeof(uint32_t) * (2 * ne + 2));
+  for (uint64_t e0 = 0; e0 < ne; ++e0) {                 /* every object v reads or writes */
+    if (edges[e0].src != v && edges[e0].dst != v) continue;
+    const uint32_t k = edges[e0].object;
+    int dup = 0;
+    for (uint64_t e1 = 0; e1 < e0; ++e1)
+      if ((edges[e1].src == v || edges[e1].dst == v) && edges[e1].object == k) dup = 1;
+    if (dup) continue;
+    uint64_t nin = 1, nout = 1;
+    rin[0] = v; rout[0] = v;
+    for (int changed = 1; changed;) {                    /* fixpoint: vertices with a D_k path to v */
+      changed = 0;
+      for (uint64_t i = 0; i < ne; ++i)
+        if (edges[i].object == k && in_set(rin, nin, edges[i].dst) && !in_set(rin, nin, edges[i].src)) {
+          rin[nin++] = edges[i].src;
+          changed = 1;
+        }
+    }
+    for (int changed = 1; changed;) {                    /* ... and with a D_k path from v */
+      changed = 0;
+      for (uint64_t i = 0; i < ne; ++i)
+        if (edges[i].object == k && in_set(rout, nout, edges[i].src) && !in_set(rout, nout, edges[i].dst)) {
+          rout[nout++] = edges[i].dst;
+          changed = 1;
+        }
+    }
+    for (uint64_t i = 0; i < ne; ++i)
+      if (edges[i].object == k && (in_set(rin, nin, edges[i].dst) || in_set(rout, nout, edges[i].src)))
+        oe[(*one)++] = edges[i];
+  }
+  free(rin);
+  free(rout);
+  qsort(oe, *one, sizeof(vo_vfg_edge), cmp_edge);
+  vo_keep_vertices(oe, *one, verts, nv, ov, onv, ~0ull);
+  return 0;
+}
+
+int vo_vfg_important(const vo_vfg_edge* edges, uint64_t ne, const vo_vfg_vertex* verts, uint64_t nv,
+                     uint64_t min_edge_bytes, uint64_t min_vertex_invocations,
+                     vo_vfg_edge* oe, uint64_t* one, vo_vfg_vertex* ov, uint64_t* onv) {
+  *one = 0;
+  for (uint64_t i = 0; i < ne; ++i)
+    if (edges[i].bytes >= min_edge_bytes) oe[(*one)++] = edges[i];
+  vo_keep_vertices(oe, *one, verts, nv, ov, onv, min_vertex_invocations);
+  return 0;
+}
+
 /* ---- C17: LoadSpy temporal load redundancy in record order (f3; Q1, R6) ----
  * The definition, walked in record order with a table of the last load seen at
  * every address (open addressing on the address; a plain map). */

@@ -149,6 +149,28 @@ uint64_t vo_record_intervals(uint32_t n_pcs, const vo_record* recs, uint64_t n, 
 int vo_plan_copies(const vo_object* objs, uint32_t n_obj, const vo_interval* merged, uint64_t n,
                  uint32_t seg_max, uint32_t dense_pct, vo_copy_plan* plan);
 
+/* ---- value flow graph (Defs 5.1-5.3) -------------
+ * Layouts equal ve.h's ve_api_access / ve_vfg_edge / ve_vfg_vertex (re-declared).
+ * Build (C18): for every non-allocation access of D_k by v_j, the edge from the
+ * vertex of the latest earlier invocation that writes D_k (allocation, host copy
+ * or a write access), found by scanning the log backwards -- Def 5.1 read
+ * literally -- plus source / sink edges of host copies.  Slice (C19): a fixpoint
+ * of "reaches v" / "reached from v" over each object's edges.  Important (C20):
+ * the two thresholds of Def 5.3.  Edges sorted by (src, dst, object). */
+#define VO_HOST 0xFFFFFFFFu
+typedef struct vo_access { uint64_t seq, bytes; uint32_t vertex, object, mode, kind; } vo_access;
+typedef struct vo_vfg_edge { uint32_t src, dst, object, label; uint64_t bytes, count; } vo_vfg_edge;
+typedef struct vo_vfg_vertex { uint32_t vertex, pad; uint64_t invocations; } vo_vfg_vertex;
+
+/* edges: room for 2n, verts: room for n.  Returns -1 on an access before allocation. */
+int vo_vfg_build(const vo_access* log, uint64_t n, vo_vfg_edge* edges, uint64_t* ne, vo_vfg_vertex* verts,
+                 uint64_t* nv);
+int vo_vfg_slice(const vo_vfg_edge* edges, uint64_t ne, const vo_vfg_vertex* verts, uint64_t nv, uint32_t v,
+                 vo_vfg_edge* oe, uint64_t* one, vo_vfg_vertex* ov, uint64_t* onv);
+int vo_vfg_important(const vo_vfg_edge* edges, uint64_t ne, const vo_vfg_vertex* verts, uint64_t nv,
+                     uint64_t min_edge_bytes, uint64_t min_vertex_invocations,
+                     vo_vfg_edge* oe, uint64_t* one, vo_vfg_vertex* ov, uint64_t* onv);
+
 /* ---- LoadSpy temporal load redundancy in trace order --------
  * Q1 / R6 (Table 5 "redundancy analysis"; LoadSpy, ref [47]): for
  * every valid global-space load r, in record order, let r' be the most recent

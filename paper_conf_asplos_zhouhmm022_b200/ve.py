@@ -36,6 +36,15 @@ OBJ_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_written", "n_loaded_eq"
 GLOB_DTYPE = np.dtype([(f, "<u8") for f in ("n_records", "n_invalid", "n_unmapped", "hist_entries")])
 INTERVAL_DTYPE = np.dtype([("start", "<u8"), ("end", "<u8")])   # ve_interval (inclusive)
 COPY_NONE, COPY_SEGMENT, COPY_MINMAX = 0, 1, 2
+# value flow graph (ve_api_access / ve_vfg_edge / ve_vfg_vertex)
+HOST_VERTEX = 0xFFFFFFFF
+ACC_READ, ACC_WRITE = 1, 2
+EV_DEVICE, EV_ALLOC, EV_H2D, EV_D2H = 0, 1, 2, 3
+ACCESS_DTYPE = np.dtype([("seq", "<u8"), ("bytes", "<u8"), ("vertex", "<u4"), ("object", "<u4"), ("mode", "<u4"),
+                         ("kind", "<u4")])
+VFG_EDGE_DTYPE = np.dtype([("src", "<u4"), ("dst", "<u4"), ("object", "<u4"), ("label", "<u4"), ("bytes", "<u8"),
+                           ("count", "<u8")])
+VFG_VERTEX_DTYPE = np.dtype([("vertex", "<u4"), ("pad", "<u4"), ("invocations", "<u8")])
 PLAN_DTYPE = np.dtype([(f, "<u8") for f in ("n_segments", "accessed_bytes", "lo", "hi", "direct_bytes",
                                            "minmax_bytes")] + [("choice", "<u4"), ("pad", "<u4")])
 DIFF_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_masked", "n_unchanged", "n_changed", "n_untouched")]
@@ -97,6 +106,13 @@ def lib():
             "ve_interval_merge": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_approx_topk": ([vp, vp, vp, vp], st),
             "ve_temporal_loads": ([vp, vp, u64, vp, vp], st),
+            "ve_vfg_build": ([vp, u64, ctypes.POINTER(vp)], st),
+            "ve_vfg_slice": ([vp, u32, ctypes.POINTER(vp)], st),
+            "ve_vfg_important": ([vp, u64, u64, ctypes.POINTER(vp)], st),
+            "ve_vfg_size": ([vp, ctypes.POINTER(u64), ctypes.POINTER(u64)], st),
+            "ve_vfg_vertices": ([vp, vp], st),
+            "ve_vfg_edges": ([vp, vp], st),
+            "ve_vfg_free": ([vp], None),
             "ve_record_intervals": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
         }
@@ -143,6 +159,47 @@ def kernel_launches():
 def rank_chunk(n, rank, world):
     """[lo, hi) of the contiguous share of n records analyzed by `rank` of `world` (strong scaling)."""
     return n * rank // world, n * (rank + 1) // world
+
+
+class ValueFlowGraph:
+    """ve_vfg_* (Defs 5.1-5.3): built from an ACCESS_DTYPE log in program order (host-side, no device)."""
+
+    def __init__(self, handle):
+        self._h = handle
+        nv, ne = ctypes.c_uint64(), ctypes.c_uint64()
+        lib().ve_vfg_size(handle, ctypes.byref(nv), ctypes.byref(ne))
+        self.vertices = np.zeros(nv.value, dtype=VFG_VERTEX_DTYPE)
+        self.edges = np.zeros(ne.value, dtype=VFG_EDGE_DTYPE)
+        lib().ve_vfg_vertices(handle, self.vertices.ctypes.data if nv.value else None)
+        lib().ve_vfg_edges(handle, self.edges.ctypes.data if ne.value else None)
+
+    @classmethod
+    def build(cls, log):
+        log = np.ascontiguousarray(log, dtype=ACCESS_DTYPE)
+        h = ctypes.c_void_p()
+        rc = lib().ve_vfg_build(log.ctypes.data if len(log) else None, len(log), ctypes.byref(h))
+        if rc != OK:
+            raise VeError(rc, "ve_vfg_build: seq not in program order or an access before its allocation")
+        return cls(h)
+
+    def slice(self, vertex):
+        h = ctypes.c_void_p()
+        rc = lib().ve_vfg_slice(self._h, vertex, ctypes.byref(h))
+        if rc != OK:
+            raise VeError(rc, f"ve_vfg_slice: no vertex {vertex}")
+        return ValueFlowGraph(h)
+
+    def important(self, min_edge_bytes, min_vertex_invocations):
+        h = ctypes.c_void_p()
+        rc = lib().ve_vfg_important(self._h, min_edge_bytes, min_vertex_invocations, ctypes.byref(h))
+        if rc != OK:
+            raise VeError(rc, "ve_vfg_important")
+        return ValueFlowGraph(h)
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _LIB is not None:
+            _LIB.ve_vfg_free(self._h)
+            self._h = None
 
 
 def merge_group(contexts, stream=None):

@@ -14,10 +14,15 @@ for r in rows[hi + 1:]:
     k = r[ki].split("(")[0]
     d[k] += float(r[vi].replace(",", ""))
     n[k] += 1
-tot = sum(d.values())
+gen = {k for k in d if not k.startswith("ve::") and not k.startswith("void ve::")}   # input generator (untimed)
+tot = sum(v for k, v in d.items() if k not in gen)
 print("# ncu launch list (gpu__time_duration.sum, --clock-control none), bench.py --steps 1 --warmup 1"
-      " (2 steps: warm-up + timed)\n# cold-cache serialised per-launch times: compare SHARES, not absolutes")
+      " --no-e2e --no-cpu --no-f1 --no-cfg5 (2 steps: warm-up + timed)\n# cold-cache serialised per-launch times:"
+      " compare SHARES, not absolutes; shares are of the libve kernels (the step)")
 print(f"{'ms':>10} launches  share  kernel")
 for k, v in d.most_common():
-    print(f"{v / 1e6:10.3f} {n[k]:8d} {100 * v / tot:5.1f}%  {k}")
-print(f"total {tot / 1e6:.3f} ms")
+    if k not in gen:
+        print(f"{v / 1e6:10.3f} {n[k]:8d} {100 * v / tot:5.1f}%  {k}")
+print(f"total {tot / 1e6:.3f} ms (libve)")
+for k in sorted(gen):
+    print(f"# input generator, outside the timed region: {k} {d[k] / 1e6:.3f} ms x {n[k]}")
