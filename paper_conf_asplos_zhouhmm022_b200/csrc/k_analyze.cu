@@ -646,6 +646,17 @@ __device__ __forceinline__ void ring_wait(uint32_t bar, uint32_t phase) {
       "@!p bra RW_LOOP;\n\t}" ::"r"(bar), "r"(phase)
       : "memory");
 }
+// non-blocking: has the phase with this parity completed?
+__device__ __forceinline__ bool mbar_test(uint32_t bar, uint32_t phase) {
+  uint32_t r;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(r) : "r"(bar), "r"(phase) : "memory");
+  return r != 0u;
+}
+#ifndef VE_PF_NEXT
+#define VE_PF_NEXT 0
+#endif
 // fire-and-forget global atomics under a predicate (no branch, no compiler-generated
 // warp aggregation around them)
 __device__ __forceinline__ void red_or(uint32_t* p, uint32_t v, bool on = true) {
@@ -1152,6 +1163,24 @@ __device__ __forceinline__ bool run_dense(const AnalyzeParams& P, const ObjCache
         ring_stage_read(R, (uint32_t)j, a[j], v[j], p[j]);
         ok = ok && fits(a[j], v[j], p[j], o[j]);
       }
+#if VE_PF_NEXT
+      // the following stage, if already landed: pull its pre elements into L1 now, so
+      // its gathers hit L1 instead of waiting on L2 one stage later
+      if (NSTAGE >= 3 && R.left >= 2u * STAGE_WIN) {
+        const uint32_t dn = R.d + 1u == (uint32_t)NSTAGE ? 0u : R.d + 1u;
+        const uint32_t phn = R.d + 1u == (uint32_t)NSTAGE ? (R.ph ^ 1u) : R.ph;
+        if (mbar_test(R.bar0 + dn * 8u, phn)) {
+#pragma unroll
+          for (int j = 0; j < STAGE_WIN; ++j) {
+            uint64_t an;
+            asm volatile("ld.shared.u64 %0, [%1];" : "=l"(an) : "r"(R.o0 + dn * STAGE_BYTES + (uint32_t)j * WIN_BYTES)
+                         : "memory");
+            const uint64_t on = an - oc.base;
+            if (on <= oc.lim) prefetch_l1(oc.pre + on);
+          }
+        }
+      }
+#endif
       if (__all_sync(FULL, ok)) {
         MT pv[STAGE_WIN];
 #pragma unroll
