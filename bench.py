@@ -244,6 +244,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-f1", action="store_true")
     ap.add_argument("--no-cfg5", action="store_true")
+    ap.add_argument("--no-cfg34", action="store_true")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))
@@ -324,6 +325,9 @@ def main():
     dd5 = None
     if rank == 0 and not args.no_cfg5:
         dd5 = measure_cfg5_dedup(ve, ctx, stream, peak)
+    c34 = None
+    if rank == 0 and not args.no_cfg34:
+        c34 = measure_other_configs(ve, stream, peak)
 
     e2e = None
     if not args.no_e2e and rank == 0 and world == 1:
@@ -348,7 +352,7 @@ def main():
                              "alg_bytes_per_launch": alg[1]},
                 "analyze_ms_per_step": [round(statistics.mean(a[i] for a in an_ms), 4) for i in (0, 1)],
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
-                "next_rows": f1, "cfg5_dedup": dd5,
+                "next_rows": f1, "cfg5_dedup": dd5, "cfg3_cfg4": c34,
                 "parity_spot_check": spot}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -399,6 +403,62 @@ def measure_next_rows(ve, ctx, wl, stream, peak, reps=3):
                               "closed_form_ok": bool(int(tl[1, 1]) == 363 * 256 * 1152
                                                      and int(tl[2, 1]) == 15 * 1152 * 5776)},
     }
+
+
+def measure_other_configs(ve, stream, peak):
+    """BASELINE configs[2] (cfg3, PyTorch op mix: 4 iterations x 264 M records) and configs[3] (cfg4, f64
+    stencils: 1.07 G + 0.94 G records), full size, outside the step: per epoch the records and snapshots
+    are generated on the device (untimed), then set_objects + ve_analyze_records + ve_report are timed with
+    CUDA events.  Parity at full size: the recipe's closed forms (tests/cfg34.py)."""
+    import torch
+    from gen import vegen as G
+    from tests import cfg34
+    sp = stream.cuda_stream
+    out = {}
+    plans = [("cfg3", G.scaled(G.CFG3, 0), [(0, 3), (0, 4), (0, 5), (0, 6)], 1 << 25),
+             ("cfg4", G.scaled(G.CFG4, 0), [(0, 4), (1, 4)], 1 << 22)]
+    for name, cfg, runs, hcap in plans:
+        tot_n, tot_ms, ok = 0, 0.0, True
+        for epoch, seed in runs:
+            inf = G.info(cfg, epoch)
+            n = inf["n_records"]
+            dobjs = []
+            for i, o in enumerate(G.objects(cfg, epoch)):
+                d = {k: o[k] for k in ("base", "size", "id", "elem_width")}
+                for side in ("pre", "post"):
+                    t = torch.empty(o["size"], dtype=torch.uint8, device="cuda")
+                    G.snapshot_device(cfg, epoch, seed, i, side == "post", t.data_ptr(), sp)
+                    d[side] = t
+                dobjs.append(d)
+            recs = torch.empty(n * REC_BYTES, dtype=torch.uint8, device="cuda")
+            G.records_device(cfg, epoch, seed, 0, n, recs.data_ptr(), sp)
+            ctx = ve.Context(n_pcs=inf["n_pcs"], max_objects=len(dobjs), hist_capacity=hcap)
+            for rep_i in range(2):           # pass 0 warms the context (allocations, pools), pass 1 is timed
+                torch.cuda.synchronize()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                ctx.set_objects(dobjs)
+                ctx.analyze_records(recs, n, stream=sp)
+                rep = ctx.report()
+                b.record(stream)
+                torch.cuda.synchronize()
+            tot_ms += a.elapsed_time(b)
+            tot_n += n
+            if seed == runs[0][1] and epoch in (0, 1):
+                k = {f: rep.keys[f] for f in rep.keys.dtype.names}
+                k["top_bits"], k["top_count"] = rep.topk["bits"], rep.topk["count"]
+                bad = (cfg34.check_cfg3(k, int(rep.globals["n_records"]), 0, rep.objects) if name == "cfg3" else
+                       cfg34.check_cfg4(k, int(rep.globals["n_records"]), 0, epoch, rep.objects))
+                ok = ok and not bad
+            ctx.close()
+            del dobjs, recs
+            torch.cuda.empty_cache()
+        gbs = tot_n * REC_BYTES / (tot_ms / 1e3) / 1e9
+        out[name] = {"records": tot_n, "ms": tot_ms, "records_per_s": tot_n / (tot_ms / 1e3), "trace_gbs": gbs,
+                     "trace_frac_of_hbm_peak": gbs / peak, "closed_forms_ok": ok,
+                     "timed": "set_objects + analyze + report per epoch (no diff / dedup), second pass on a warm "
+                              "context"}
+    return out
 
 
 def measure_cfg5_dedup(ve, ctx, stream, peak, reps=3):

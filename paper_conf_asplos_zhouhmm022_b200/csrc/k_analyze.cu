@@ -449,7 +449,10 @@ __device__ __forceinline__ void bitmap_or(uint32_t* bm, bool part, uint64_t word
 // at exit.  For w <= 4 the min / max totals are 32-bit forms: ord of signed types
 // is sext32(b)^2^31 (order-isomorphic to the 64-bit key), and 0xFFFFFFFF is the min
 // identity of ord / trunc of floats (no non-NaN key has that value).
-constexpr int NSLOT = 4;
+#ifndef VE_NSLOT
+#define VE_NSLOT 8
+#endif
+constexpr int NSLOT = VE_NSLOT;
 struct __align__(16) SlotE {
   uint64_t key;                 // meta << 32 | object id << 16 | pc; ~0 = free
   unsigned long long dense;     // per-element counters of (pc, object), or 0
@@ -483,20 +486,31 @@ __device__ __noinline__ void slot_line_flush(const AnalyzeParams& P, WarpCache& 
 }
 
 // claim (or find) a dense counter array of sorted object oi for the loads of one
-// (pc, access type): claim key ck = meta << 16 | pc (lane 0), broadcast
+// (pc, access type): claim key ck = meta << 16 | pc (lane 0), broadcast.  The claimer
+// takes the array from the pool (bump allocation) and publishes its offset; a warp
+// finding the slot already claimed by ck waits for that offset (a few cycles).
 __device__ __noinline__ unsigned long long dense_lookup(const AnalyzeParams& P, int oi, uint32_t ck) {
   unsigned long long dp = 0;
   if ((threadIdx.x & 31) == 0) {
+    const uint64_t ne = (P.o.end[oi] - P.o.base[oi] + P.o.ew[oi] - 1) / P.o.ew[oi];
     for (int j = 0; j < DENSE_PER_OBJ; ++j) {
-      uint32_t* slot = &P.o.dense_pc[DENSE_PER_OBJ * oi + j];
+      const int si = DENSE_PER_OBJ * oi + j;
+      uint32_t* slot = &P.o.dense_pc[si];
       uint32_t d = *(volatile uint32_t*)slot;
       if (d == DENSE_OFF) break;
       if (d == DENSE_FREE) {
         d = atomicCAS(slot, DENSE_FREE, ck);
-        if (d == DENSE_FREE) d = ck;
+        if (d == DENSE_FREE) {                       // ours: allocate and publish
+          const unsigned long long off = atomicAdd(P.o.dense_next, (unsigned long long)ne);
+          atomicExch(&P.o.dense_off[si], off + ne <= P.o.dense_cap ? off : DENSE_NONE);
+          d = ck;
+        }
       }
       if (d == ck) {
-        dp = (unsigned long long)(P.o.dense_pool + P.o.dense_off[DENSE_PER_OBJ * oi + j]);
+        unsigned long long off;
+        while ((off = *(volatile unsigned long long*)&P.o.dense_off[si]) == DENSE_NOT_READY) {
+        }
+        if (off != DENSE_NONE) dp = (unsigned long long)(P.o.dense_pool + off);
         break;
       }
     }
@@ -1715,7 +1729,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.n_obj = c->n_obj;
   P.mant_bits = c->cfg.mant_bits;
   // u32 per-element counters cannot overflow while the ctx has seen < 2^32 records
-  P.dense_ok = (c->dense_used > 0 && c->records_analyzed + n < (1ull << 32)) ? 1u : 0u;
+  P.dense_ok = (c->dense_cap > 0 && c->records_analyzed + n < (1ull << 32)) ? 1u : 0u;
+  if (P.dense_ok) c->dense_dirty = true;
   P.ring = ((uintptr_t)d % 16 == 0) ? 1u : 0u;
   P.nring = P.ring ? n / 32 : 0;
   P.work = c->t.glob + G_WORK;

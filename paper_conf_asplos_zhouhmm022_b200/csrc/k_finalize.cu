@@ -823,22 +823,81 @@ __device__ __forceinline__ unsigned long long wmax64(unsigned long long v) {
   return v;
 }
 
-__global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
+// Shared table of `ts` slots (dynamic shared memory: ts u64 value bits, then ts u32
+// counts).  Blocks walk chunks of DF_CHUNK elements (chunk c, c + grid, ...).  The many-
+// block launch (one chunk per block, ts = DF_SLOTS) keeps many HBM-table inserts in
+// flight for high-cardinality arrays; the persistent launch (two blocks per SM, ts =
+// DF_LC_SLOTS) aggregates a low-cardinality array across all its chunks, so each block
+// inserts each distinct value about once.  A table filled past half is emptied into the
+// HBM table between chunks.  Counts per block stay < 2^32 (dense counting is on only
+// while the ctx has seen < 2^32 records).
+constexpr uint32_t DF_LC_SLOTS = 8192;
+constexpr uint32_t DF_LC_CHUNK = 32768;
+constexpr uint64_t DF_PROBE_MIN = 1ull << 24;   // arrays probed for low cardinality   // elements between table-fill checks (persistent blocks)
+
+// value statistics of `k` counted loads that read the value bits b (C1 n_zero, C5 flags
+// and ord range, C4 raw range, C7 truncated range), accumulated per thread
+__device__ __forceinline__ void df_stats(DenseVal& v, uint64_t b, unsigned long long k, uint32_t kind, uint32_t lg,
+                                         uint32_t mant_bits) {
+  if (b == 0ull) v.s[0] += k;
+  uint32_t ff = 0;
+  if (kind >= 2u) {
+    int64_t ival;
+    ff = float_flags(b, kind, lg, ival);
+    for (int j = 0; j < 5; ++j) if (ff & (1u << j)) v.s[1 + j] += k;
+  }
+  v.mn[0] = b < v.mn[0] ? b : v.mn[0];
+  v.mx[0] = b > v.mx[0] ? b : v.mx[0];
+  if (!(ff & 1u)) {                    // NaNs excluded from ord / trunc (C5, C7)
+    const uint64_t o = ord_key(b, kind, lg);
+    v.mn[1] = o < v.mn[1] ? o : v.mn[1];
+    v.mx[1] = o > v.mx[1] ? o : v.mx[1];
+    if (kind >= 2u) {
+      const uint64_t tr = trunc_bits(b, kind, lg, mant_bits);
+      v.mn[2] = tr < v.mn[2] ? tr : v.mn[2];
+      v.mx[2] = tr > v.mx[2] ? tr : v.mx[2];
+    }
+  }
+}
+
+// empty the block's table into the HBM table, taking each entry's value statistics once
+__device__ __forceinline__ void df_table_flush(unsigned long long* sbits, uint32_t* scnt, uint32_t ts, uint32_t tag,
+                                               DevTables& t, DenseVal& v, uint32_t kind, uint32_t lg,
+                                               uint32_t mant_bits) {
+  for (uint32_t i = threadIdx.x; i < ts; i += blockDim.x) {
+    if (sbits[i] != ~0ull && scnt[i]) {
+      df_stats(v, sbits[i], scnt[i], kind, lg, mant_bits);
+      hist_insert_global(t, tag, sbits[i], scnt[i]);
+    }
+    sbits[i] = ~0ull;
+    scnt[i] = 0;
+  }
+}
+
+template <int NT>
+__global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
                                                            uint32_t ew, uint32_t tag, uint64_t bmoff, DevTables t,
-                                                           uint32_t meta, uint32_t mant_bits, uint32_t kp, uint32_t ko) {
-  __shared__ unsigned long long sbits[DF_SLOTS], scnt[DF_SLOTS];
+                                                           uint32_t meta, uint32_t mant_bits, uint32_t kp, uint32_t ko,
+                                                           uint32_t ts, uint32_t csz) {
+  extern __shared__ unsigned long long df_smem[];
+  unsigned long long* sbits = df_smem;
+  uint32_t* scnt = reinterpret_cast<uint32_t*>(df_smem + ts);
   __shared__ DenseVal sv;
-  for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS) { sbits[i] = ~0ull; scnt[i] = 0; }
+  __shared__ uint32_t sfill;
+  for (uint32_t i = threadIdx.x; i < ts; i += NT) { sbits[i] = ~0ull; scnt[i] = 0; }
   if (threadIdx.x < 6) sv.s[threadIdx.x] = 0;
   if (threadIdx.x < 3) { sv.mn[threadIdx.x] = ~0ull; sv.mx[threadIdx.x] = 0; }
+  if (threadIdx.x == 0) sfill = 0;
   const uint32_t kind = (meta >> 2) & 3u, lg = meta & 3u;
   DenseVal v;
   for (int i = 0; i < 6; ++i) v.s[i] = 0;
   for (int i = 0; i < 3; ++i) { v.mn[i] = ~0ull; v.mx[i] = 0; }
   __syncthreads();
-  const uint64_t lo = blockIdx.x * DF_CHUNK, hi = lo + DF_CHUNK < n_elems ? lo + DF_CHUNK : n_elems;
   const int lane = threadIdx.x & 31;
-  for (uint64_t base = lo; base < hi; base += DF_THREADS) {
+  const uint64_t nchunks = (n_elems + csz - 1) / csz;
+  for (uint64_t ch = blockIdx.x; ch < nchunks; ch += gridDim.x) {
+  const uint64_t lo = ch * csz, hi = lo + csz < n_elems ? lo + csz : n_elems;
+  for (uint64_t base = lo; base < hi; base += NT) {
     const uint64_t e = base + threadIdx.x;
     uint32_t k = 0;
     uint64_t bits = 0;
@@ -854,52 +913,52 @@ __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint6
         }
       }
     }
-    if (k) {
-      const uint64_t b = bits;
-      if (b == 0ull) v.s[0] += k;
-      uint32_t ff = 0;
-      if (kind >= 2u) {
-        int64_t ival;
-        ff = float_flags(b, kind, lg, ival);
-        for (int j = 0; j < 5; ++j) if (ff & (1u << j)) v.s[1 + j] += k;
-      }
-      v.mn[0] = b < v.mn[0] ? b : v.mn[0];
-      v.mx[0] = b > v.mx[0] ? b : v.mx[0];
-      if (!(ff & 1u)) {                    // NaNs excluded from ord / trunc (C5, C7)
-        const uint64_t o = ord_key(b, kind, lg);
-        v.mn[1] = o < v.mn[1] ? o : v.mn[1];
-        v.mx[1] = o > v.mx[1] ? o : v.mx[1];
-        if (kind >= 2u) {
-          const uint64_t tr = trunc_bits(b, kind, lg, mant_bits);
-          v.mn[2] = tr < v.mn[2] ? tr : v.mn[2];
-          v.mx[2] = tr > v.mx[2] ? tr : v.mx[2];
-        }
-      }
-    }
     const unsigned km = __ballot_sync(0xFFFFFFFFu, k != 0);
     // C3: a counted load started at element e (K1 leaves these L bits to us); the
     // warp's 32 elements are one aligned bitmap word
     if (lane == 0 && km) atomicOr(&t.L[bmoff + ((base + threadIdx.x) >> 5)], km);
     if (k) {
       const unsigned g = __match_any_sync(km, bits);
-      const unsigned long long sum = __reduce_add_sync(g, k);   // < 32 * 2^32? counts are < 2^32 each
+      // (a REDUX under per-lane group masks runs once per distinct mask: singletons skip it)
+      const unsigned long long sum = __popc(g) == 1 ? (unsigned long long)k : __reduce_add_sync(g, k);
       if (lane == __ffs(g) - 1) {
         // shared slots are claimed by a 64-bit CAS of the value itself (empty = ~0, which
         // only an 8-byte element can hold: such values go straight to the global table)
-        uint32_t h = (uint32_t)hist_hash(tag, bits) & (DF_SLOTS - 1);
+        uint32_t h = (uint32_t)hist_hash(tag, bits) & (ts - 1);
         bool done = false;
         for (int probe = 0; probe < 8 && !done && bits != ~0ull; ++probe) {
-          const unsigned long long old = atomicCAS(&sbits[h], ~0ull, bits);
-          if (old == ~0ull || old == bits) {
-            atomicAdd(&scnt[h], sum);
+          // look first (a warm table mostly holds the value already), claim only empty slots
+          unsigned long long cur = *(volatile unsigned long long*)&sbits[h];
+          if (cur == ~0ull) {
+            cur = atomicCAS(&sbits[h], ~0ull, bits);
+            if (cur == ~0ull) {
+              atomicAdd(&sfill, 1u);
+              cur = bits;
+            }
+          }
+          if (cur == bits) {
+            atomicAdd(&scnt[h], (uint32_t)sum);
             done = true;
           }
-          h = (h + 1) & (DF_SLOTS - 1);
+          h = (h + 1) & (ts - 1);
         }
-        if (!done) hist_insert_global(t, tag, bits, sum);
+        if (!done) {                     // straight to the HBM table: its statistics now
+          df_stats(v, bits, sum, kind, lg, mant_bits);
+          hist_insert_global(t, tag, bits, sum);
+        }
       }
     }
   }
+  __syncthreads();
+  if (sfill > ts / 2) {                    // a table past half full: empty it between chunks
+    df_table_flush(sbits, scnt, ts, tag, t, v, kind, lg, mant_bits);
+    __syncthreads();
+    if (threadIdx.x == 0) sfill = 0;
+    __syncthreads();
+  }
+  }
+  __syncthreads();
+  df_table_flush(sbits, scnt, ts, tag, t, v, kind, lg, mant_bits);
   // value statistics: warp, block, then both keys' rows (PC key kp, object key ko)
   for (int i = 0; i < 6; ++i) {
     const unsigned long long x = wsum64(v.s[i]);
@@ -910,8 +969,6 @@ __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint6
     if (lane == 0) { atomicMin(&sv.mn[i], a); atomicMax(&sv.mx[i], b); }
   }
   __syncthreads();
-  for (int i = threadIdx.x; i < DF_SLOTS; i += DF_THREADS)
-    if (sbits[i] != ~0ull && scnt[i]) hist_insert_global(t, tag, sbits[i], scnt[i]);
   if (threadIdx.x < 2) {
     const uint64_t key = threadIdx.x ? ko : kp;
     const int f[6] = {F_ZERO, F_NAN, F_NONINT, F_NF16, F_NBF16, F_NF32};
@@ -924,27 +981,118 @@ __global__ void __launch_bounds__(DF_THREADS) k_dense_flush(uint32_t* cnt, uint6
   }
 }
 
+// Cardinality probe of a dense array: the distinct values among up to 64 Ki counted
+// elements sampled at a fixed stride (one block); out[0] = distinct (capped near 4096).
+__global__ void __launch_bounds__(1024) k_dense_sample(const uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
+                                                      uint32_t ew, unsigned int* out) {
+  extern __shared__ unsigned long long tb[];   // 8192 slots (dynamic: 64 KiB)
+  __shared__ unsigned int nd;
+  for (int i = threadIdx.x; i < 8192; i += 1024) tb[i] = ~0ull;
+  if (threadIdx.x == 0) nd = 0;
+  __syncthreads();
+  const uint64_t stride = n_elems > 65536 ? n_elems / 65536 : 1;
+  for (uint64_t s = threadIdx.x; s < 65536 && s * stride < n_elems; s += 1024) {
+    if (*(volatile unsigned int*)&nd > 4096) break;
+    const uint64_t e = s * stride;
+    if (!cnt[e]) continue;
+    const uint8_t* p = pre + e * ew;
+    uint64_t bits = 0;
+    for (uint32_t i = 0; i < ew; ++i) bits |= (uint64_t)p[i] << (8 * i);
+    if (bits == ~0ull) bits = ~1ull;   // (the probe only estimates)
+    uint32_t h = (uint32_t)mix64(bits) & 8191u;
+    for (int probe = 0; probe < 64; ++probe) {
+      unsigned long long old = *(volatile unsigned long long*)&tb[h];   // look first: no CAS storm on one value
+      if (old == bits) break;
+      if (old == ~0ull) {
+        old = atomicCAS(&tb[h], ~0ull, bits);
+        if (old == ~0ull) { atomicAdd(&nd, 1u); break; }
+        if (old == bits) break;
+      }
+      h = (h + 1) & 8191u;
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) out[0] = nd;
+}
+
 ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
-  if (!c->dense_used || !c->n_obj) return VE_OK;
-  std::vector<uint32_t> dpc((size_t)DENSE_PER_OBJ * c->n_obj);
-  cudaError_t e = cudaMemcpyAsync(dpc.data(), c->o.dense_pc, dpc.size() * 4, cudaMemcpyDeviceToHost, s);
+  if (!c->dense_cap || !c->n_obj || !c->dense_dirty) return VE_OK;
+  const size_t ns = (size_t)DENSE_PER_OBJ * c->n_obj;
+  std::vector<uint32_t> dpc(ns);
+  std::vector<unsigned long long> doff(ns);
+  cudaError_t e = cudaMemcpyAsync(dpc.data(), c->o.dense_pc, ns * 4, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(doff.data(), c->o.dense_off, ns * 8, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush");
   bool any = false;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaFuncSetAttribute(k_dense_flush<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_LC_SLOTS * 12));
+    cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)(DF_SLOTS * 12));
+    cudaFuncSetAttribute(k_dense_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
+    attr_set = true;
+  }
+  struct Arr { uint32_t i, pc, meta; unsigned long long off; };
+  std::vector<Arr> arrs;
   for (uint32_t i = 0; i < c->n_obj; ++i) {
     for (int j = 0; j < DENSE_PER_OBJ; ++j) {
       const uint32_t ck = dpc[DENSE_PER_OBJ * i + j];   // claim key: meta << 16 | pc
-      if (ck == DENSE_FREE || ck == DENSE_OFF) continue;
-      const uint32_t pc = ck & 0xFFFFu, meta = ck >> 16;
-      const HostObject& o = c->objs[i];
-      const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
-      count_launch();
-      k_dense_flush<<<(unsigned)blocks, DF_THREADS, 0, s>>>((uint32_t*)c->dense_pool + c->dense_off_h[DENSE_PER_OBJ * i + j],
-                                                    o.n_elems, (const uint8_t*)o.pre, o.ew, (pc << 16) | o.id, o.bmoff, c->t,
-                                                    meta, c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id);
-      any = true;
+      const unsigned long long off = doff[DENSE_PER_OBJ * i + j];
+      if (ck == DENSE_FREE || ck == DENSE_OFF || off == DENSE_NOT_READY || off == DENSE_NONE) continue;
+      arrs.push_back(Arr{i, ck & 0xFFFFu, ck >> 16, off});
     }
   }
+  // cardinality probes of the large arrays, one sync for all of them
+  std::vector<unsigned int> nd(arrs.size(), ~0u);
+  unsigned int* d_probe = nullptr;
+  if (!arrs.empty()) {
+    e = cudaMallocAsync((void**)&d_probe, 4 * arrs.size(), s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush probe alloc");
+    cudaMemsetAsync(d_probe, 0xFF, 4 * arrs.size(), s);
+    bool probed = false;
+    for (size_t a = 0; a < arrs.size(); ++a) {
+      const HostObject& o = c->objs[arrs[a].i];
+      if (o.n_elems < DF_PROBE_MIN) continue;   // small arrays: the many-block path, no probe sync
+      count_launch();
+      k_dense_sample<<<1, 1024, 8192 * 8, s>>>((uint32_t*)c->dense_pool + arrs[a].off, o.n_elems,
+                                               (const uint8_t*)o.pre, o.ew, d_probe + a);
+      probed = true;
+    }
+    if (probed) {
+      e = cudaMemcpyAsync(nd.data(), d_probe, 4 * arrs.size(), cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) { cudaFreeAsync(d_probe, s); return cuda_fail(c, e, "dense_flush probe"); }
+    }
+  }
+  for (size_t a = 0; a < arrs.size(); ++a) {
+    const HostObject& o = c->objs[arrs[a].i];
+    const uint32_t pc = arrs[a].pc, meta = arrs[a].meta;
+    uint32_t* arr = (uint32_t*)c->dense_pool + arrs[a].off;
+    // low-cardinality arrays (a sampled distinct count that fits half a large table):
+    // one persistent 1024-thread block per SM aggregates across chunks; otherwise one
+    // chunk per 256-thread block
+    const bool lc = nd[a] <= DF_LC_SLOTS / 2;
+    const uint32_t ts = lc ? DF_LC_SLOTS : (uint32_t)DF_SLOTS;
+    const size_t smem = (size_t)ts * 12;
+    uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
+    count_launch();
+    if (lc) {
+      if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+      k_dense_flush<1024><<<(unsigned)blocks, 1024, smem, s>>>(arr, o.n_elems, (const uint8_t*)o.pre, o.ew,
+                                                              (pc << 16) | o.id, o.bmoff, c->t, meta,
+                                                              c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id, ts,
+                                                              DF_LC_CHUNK);
+    } else {
+      k_dense_flush<DF_THREADS><<<(unsigned)blocks, DF_THREADS, smem, s>>>(arr, o.n_elems, (const uint8_t*)o.pre,
+                                                                          o.ew, (pc << 16) | o.id, o.bmoff, c->t,
+                                                                          meta, c->cfg.mant_bits, pc,
+                                                                          c->cfg.n_pcs + o.id, ts, (uint32_t)DF_CHUNK);
+    }
+    any = true;
+  }
+  if (d_probe) cudaFreeAsync(d_probe, s);
+  c->dense_dirty = false;      // every claimed array is read and re-zeroed by its flush
   if (!any) return VE_OK;
   unsigned long long glob[8];
   e = cudaMemcpyAsync(glob, c->t.glob, sizeof(glob), cudaMemcpyDeviceToHost, s);

@@ -57,15 +57,25 @@ ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
   cudaMemsetAsync(c->t.mn, 0xFF, nk_max * NMM * 8, s);
   cudaMemsetAsync(c->t.mx, 0, nk_max * NMM * 8, s);
   cudaMemsetAsync(c->t.line, 0, nk_max * sizeof(LineState), s);
+  // counts claimed arrays still hold (analysed, never flushed): clear the used pool
+  if (c->dense_dirty && c->dense_pool) {
+    unsigned long long used = 0;
+    cudaMemcpyAsync(&used, c->t.glob + G_DENSE_NEXT, 8, cudaMemcpyDeviceToHost, s);
+    cudaStreamSynchronize(s);
+    if (used > c->dense_cap) used = c->dense_cap;
+    if (used) cudaMemsetAsync(c->dense_pool, 0, used * 4, s);
+    c->dense_dirty = false;
+  }
   cudaMemsetAsync(c->t.glob, 0, 8 * 8, s);
   if (c->bm_words) {
     cudaMemsetAsync(c->t.W, 0, c->bm_words * 4, s);
     cudaMemsetAsync(c->t.L, 0, c->bm_words * 4, s);
   }
   cudaMemsetAsync(c->t.hslot, 0xFF, c->hcap * sizeof(HSlot), s);
-  if (c->dense_used) cudaMemsetAsync(c->dense_pool, 0, c->dense_used * 4, s);
-  if (c->n_obj)
+  if (c->n_obj) {
     cudaMemcpyAsync(c->o.dense_pc, c->dense_pc_init.data(), 4ull * DENSE_PER_OBJ * c->n_obj, cudaMemcpyHostToDevice, s);
+    cudaMemsetAsync(c->o.dense_off, 0xFF, 8ull * DENSE_PER_OBJ * c->n_obj, s);   // DENSE_NOT_READY
+  }
   c->records_analyzed = 0;
   cudaError_t e = cudaMemsetAsync(c->t.hcount, 0, c->hcap * 8, s);
   if (e != cudaSuccess) return cuda_fail(c, e, "reset");
@@ -265,36 +275,37 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     }
   }
   c->bm_words = words;
-  // dense per-element counters: DENSE_PER_OBJ arrays per object with a pre snapshot,
-  // smallest objects first, within a budget of 2^30 counters (4 GiB)
-  const uint64_t DENSE_BUDGET = 1ull << 30;
-  std::vector<uint32_t> order(n);
-  for (uint32_t i = 0; i < n; ++i) order[i] = i;
-  std::sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return v[a].n_elems < v[b].n_elems; });
-  c->dense_off_h.assign((size_t)DENSE_PER_OBJ * n, ~0ull);
+  // dense per-element counters: up to DENSE_PER_OBJ arrays per object with a pre
+  // snapshot, allocated from one pool when a (pc, access type) first claims one
+  // (k_analyze's dense_lookup); the pool holds min(2^31, DENSE_PER_OBJ * sum of the
+  // objects' elements) counters (<= 8 GiB), claims beyond it take the hash path
+  const uint64_t DENSE_BUDGET = 1ull << 31;
   c->dense_pc_init.assign((size_t)DENSE_PER_OBJ * n, DENSE_OFF);
-  uint64_t dense = 0;
-  for (uint32_t i : order) {
-    if (!v[i].pre || dense + DENSE_PER_OBJ * v[i].n_elems > DENSE_BUDGET) continue;
-    for (int j = 0; j < DENSE_PER_OBJ; ++j) {
-      c->dense_off_h[DENSE_PER_OBJ * i + j] = dense;
-      c->dense_pc_init[DENSE_PER_OBJ * i + j] = DENSE_FREE;
-      dense += v[i].n_elems;
-    }
+  uint64_t want = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (!v[i].pre) continue;
+    for (int j = 0; j < DENSE_PER_OBJ; ++j) c->dense_pc_init[DENSE_PER_OBJ * i + j] = DENSE_FREE;
+    want += DENSE_PER_OBJ * v[i].n_elems;
   }
-  if (dense > c->dense_cap) {
-    cudaFree(c->dense_pool);
+  if (want > DENSE_BUDGET) want = DENSE_BUDGET;
+  if (want > c->dense_cap) {
+    if (c->dense_pool) {
+      cudaDeviceSynchronize();
+      cudaFree(c->dense_pool);
+    }
     c->dense_pool = nullptr;
     c->dense_cap = 0;
-    if (cudaMalloc(&c->dense_pool, dense * 4) != cudaSuccess) {
+    if (cudaMalloc(&c->dense_pool, want * 4) != cudaSuccess ||
+        cudaMemset(c->dense_pool, 0, want * 4) != cudaSuccess) {
       cudaGetLastError();
-      dense = 0;                                       // no memory: everything goes to the hash path
+      if (c->dense_pool) cudaFree(c->dense_pool);
+      c->dense_pool = nullptr;                         // no memory: everything goes to the hash path
       std::fill(c->dense_pc_init.begin(), c->dense_pc_init.end(), DENSE_OFF);
     } else {
-      c->dense_cap = dense;
+      c->dense_cap = want;
     }
+    c->dense_dirty = false;
   }
-  c->dense_used = dense;
   // device object table (SoA, sorted by base)
   cudaFree(c->obj_block);
   c->obj_block = nullptr;
@@ -316,18 +327,20 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     hid[i] = v[i].id; hew[i] = v[i].ew;
     c->sorted_of_id[v[i].id] = i;
   }
-  for (size_t k = 0; k < (size_t)DENSE_PER_OBJ * n; ++k) { hdo[k] = c->dense_off_h[k]; hdp[k] = c->dense_pc_init[k]; }
+  for (size_t k = 0; k < (size_t)DENSE_PER_OBJ * n; ++k) { hdo[k] = DENSE_NOT_READY; hdp[k] = c->dense_pc_init[k]; }
   cudaMemcpy(c->obj_block, host.data(), nb, cudaMemcpyHostToDevice);
   uint64_t* db = (uint64_t*)c->obj_block;
   c->o.base = db;
   c->o.end = db + n;
   c->o.pre = db + 2 * n;
   c->o.bmoff = db + 3 * n;
-  c->o.dense_off = db + 4 * n;
+  c->o.dense_off = (unsigned long long*)(db + 4 * n);
   c->o.id = (const uint32_t*)(db + 4 * n + DENSE_PER_OBJ * n);
   c->o.ew = c->o.id + n;
   c->o.dense_pc = const_cast<uint32_t*>(c->o.ew + n);
   c->o.dense_pool = (uint32_t*)c->dense_pool;
+  c->o.dense_cap = c->dense_cap;
+  c->o.dense_next = c->t.glob + G_DENSE_NEXT;
   c->o.n = n;
   c->objs = v;
   c->n_obj = n;

@@ -72,17 +72,24 @@ struct DevObjects {          // sorted by base
   const uint32_t* ew;
   const uint64_t* pre;       // device pointers as integers (0 = none)
   const uint64_t* bmoff;     // first bitmap word of the object
-  // dense per-element access counters for loads that read the pre value
-  // (2 arrays per object, each claimed by one PC): dense_pc[2*i+j] = claimed pc,
-  // DENSE_FREE or DENSE_OFF; dense_off[2*i+j] = first counter in dense_pool
+  // dense per-element access counters for loads that read the pre value: up to
+  // DENSE_PER_OBJ arrays per object, each claimed by one (pc, access type):
+  // dense_pc[D*i+j] = claim key, DENSE_FREE or DENSE_OFF; the claimer allocates the
+  // array from the pool (bump cursor *dense_next) and publishes its first counter in
+  // dense_off[D*i+j] (DENSE_NOT_READY until then, DENSE_NONE if the pool is full)
   uint32_t* dense_pc;
-  const uint64_t* dense_off;
+  unsigned long long* dense_off;
   uint32_t* dense_pool;
+  unsigned long long* dense_next;
+  uint64_t dense_cap;        // counters in the pool
   uint32_t n;
 };
 constexpr uint32_t DENSE_FREE = 0xFFFFFFFFu;
 constexpr uint32_t DENSE_OFF = 0xFFFFFFFEu;
-constexpr int DENSE_PER_OBJ = 2;
+constexpr unsigned long long DENSE_NOT_READY = ~0ull;
+constexpr unsigned long long DENSE_NONE = ~1ull;
+constexpr int DENSE_PER_OBJ = 8;
+constexpr int G_DENSE_NEXT = 4;   // glob slot of the dense pool cursor
 
 // ---- host-side context ------------------------------------------------------
 struct HostObject {
@@ -114,9 +121,8 @@ struct ve_ctx {
   // dense counters (see DevObjects); disabled once 2^32 records could overflow a u32 counter
   void* dense_pool = nullptr;
   uint64_t dense_cap = 0;                    // counters allocated
-  uint64_t dense_used = 0;                   // counters in use by the current object table
-  std::vector<uint64_t> dense_off_h;         // [2*n_obj]
-  std::vector<uint32_t> dense_pc_init;       // [2*n_obj]: DENSE_FREE or DENSE_OFF
+  bool dense_dirty = false;                  // pool may hold counts not yet flushed
+  std::vector<uint32_t> dense_pc_init;       // [DENSE_PER_OBJ*n_obj]: DENSE_FREE or DENSE_OFF
   uint64_t records_analyzed = 0;
   // finalize scratch
   void* scratch = nullptr;
