@@ -1225,6 +1225,140 @@ __device__ __forceinline__ bool run_dense(const AnalyzeParams& P, const ObjCache
   }
 }
 
+// Multi-key dense path (VE_MULTI_DENSE): like run_dense, but a following window may
+// belong to ANY key of the warp's slot cache that counts its loads densely and has no
+// live line state (loads of one object by several PCs interleaved window by window:
+// stencil neighbours, Darknet's C rows).  Whole stages are taken up to the first
+// window that does not qualify, their STAGE_WIN gathers in flight together; each
+// window's record count and eq count go to its own slot.  Stops (returns true, window
+// left in addr / val / pm for the main loop) at a window that does not qualify; nd is
+// set only when the entry window itself is not entirely dense.
+#ifndef VE_MULTI_DENSE
+#define VE_MULTI_DENSE 1
+#endif
+#ifndef VE_MULTI_MIN_PCS
+#define VE_MULTI_MIN_PCS 8
+#endif
+template <int LG>
+__device__ __forceinline__ bool run_dense_multi(const AnalyzeParams& P, const ObjCache& oc, SlotE* slots, SlotE* se,
+                                                Ring& R, uint64_t& addr, uint64_t& val, uint64_t& pm, bool& nd) {
+  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;
+  constexpr uint32_t W = 1u << LG;
+  const unsigned FULL = 0xFFFFFFFFu;
+  const int lane = threadIdx.x & 31;
+  uint64_t lastp = shfl64(FULL, pm, 0);      // the key seen last, its slot, and the windows
+  SlotE* lasts = se;                          // counted for it but not yet added to the slot
+  uint32_t nlast = 0;
+  auto settle = [&]() {
+    __syncwarp();
+    if (lane == 0 && nlast) { lasts->nwin += nlast; lasts->sum[1] += nlast * 32u; }
+    __syncwarp();
+    nlast = 0;
+  };
+  // the slot of a window (warp-uniform pm) if it is a dense load key of this object
+  // without live line state, else nullptr; it becomes the "last" slot
+  auto slot_of = [&](uint64_t p) -> SlotE* {
+    if (__all_sync(FULL, p == lastp)) return lasts;
+    const uint64_t p0 = shfl64(FULL, p, 0);
+    if (!__all_sync(FULL, p == p0)) return nullptr;
+    const uint32_t meta = (uint32_t)(p0 >> 32), pc = (uint32_t)p0;
+    if ((meta & 3u) != (uint32_t)LG || meta_store(meta) || meta_shared(meta)) return nullptr;
+    const uint64_t key = ((uint64_t)meta << 32) | ((uint64_t)oc.id << 16) | pc;
+#pragma unroll
+    for (int i = 0; i < NSLOT; ++i)
+      if (slots[i].key == key) {
+        if (slots[i].dense == 0ull || slots[i].lfail != 3u) return nullptr;
+        settle();
+        lastp = p0;
+        lasts = &slots[i];
+        return lasts;
+      }
+    return nullptr;
+  };
+  auto lane_fits = [&](uint64_t a, uint64_t v, uint64_t& o) -> bool {
+    o = a - oc.base;
+    bool ok = o <= oc.lim && (o & (W - 1)) == 0;
+    if constexpr (LG < 3) ok = ok && (v >> (8 * W)) == 0ull;
+    return ok;
+  };
+  nd = false;
+  {   // the entry window (its slot is se)
+    const uint64_t o = addr - oc.base;
+    const MT pv = (MT)ld_pre<LG>(oc.pre + o);
+    if (!__all_sync(FULL, pv == (MT)val)) { nd = true; return true; }
+    red_add_keep(reinterpret_cast<uint32_t*>(se->dense) + (o >> LG), 1u, true);
+    ++nlast;
+  }
+  while (true) {
+    if (ring_stage_full(R)) {
+      ring_stage_wait(P, R);
+      uint64_t a[STAGE_WIN], v[STAGE_WIN], p[STAGE_WIN], o[STAGE_WIN];
+      bool same = true;
+#pragma unroll
+      for (int j = 0; j < STAGE_WIN; ++j) {
+        ring_stage_read(R, (uint32_t)j, a[j], v[j], p[j]);
+        same = same && p[j] == lastp && lane_fits(a[j], v[j], o[j]);
+      }
+      if (__all_sync(FULL, same)) {           // a whole stage of the last key: as run_dense
+        MT pv[STAGE_WIN];
+#pragma unroll
+        for (int j = 0; j < STAGE_WIN; ++j) pv[j] = (MT)ld_pre<LG>(oc.pre + o[j]);
+        bool eq = true;
+#pragma unroll
+        for (int j = 0; j < STAGE_WIN; ++j) eq = eq && pv[j] == (MT)v[j];
+        if (__all_sync(FULL, eq)) {
+          uint32_t* const dn = reinterpret_cast<uint32_t*>(lasts->dense);
+#pragma unroll
+          for (int j = 0; j < STAGE_WIN; ++j) red_add_keep(dn + (o[j] >> LG), 1u, true);
+          nlast += STAGE_WIN;
+          VE_DBG(0, 1);
+          ring_stage_consume(R);
+          continue;
+        }
+      } else {                                 // several keys: each window's own slot
+        SlotE* es[STAGE_WIN];
+        bool ok = true;
+#pragma unroll
+        for (int j = 0; j < STAGE_WIN; ++j) {
+          es[j] = ok ? slot_of(p[j]) : nullptr;
+          ok = ok && es[j] != nullptr && __all_sync(FULL, lane_fits(a[j], v[j], o[j]));
+        }
+        if (ok) {
+          MT pv[STAGE_WIN];
+#pragma unroll
+          for (int j = 0; j < STAGE_WIN; ++j) pv[j] = (MT)ld_pre<LG>(oc.pre + o[j]);
+          bool eq = true;
+#pragma unroll
+          for (int j = 0; j < STAGE_WIN; ++j) eq = eq && pv[j] == (MT)v[j];
+          if (__all_sync(FULL, eq)) {
+            settle();
+#pragma unroll
+            for (int j = 0; j < STAGE_WIN; ++j) {
+              red_add_keep(reinterpret_cast<uint32_t*>(es[j]->dense) + (o[j] >> LG), 1u, true);
+              if (lane == 0) { es[j]->nwin += 1u; es[j]->sum[1] += 32u; }
+            }
+            __syncwarp();
+            VE_DBG(0, 1);
+            ring_stage_consume(R);
+            continue;
+          }
+        }
+      }
+      // not a whole stage of qualifying windows: go on window by window
+    }
+    if (R.left == 0u) { settle(); return false; }
+    ring_next(P, R, addr, val, pm);
+    SlotE* e = slot_of(pm);
+    uint64_t o;
+    if (e == nullptr || !__all_sync(FULL, lane_fits(addr, val, o))) { VE_DBG(5, 1); settle(); return true; }
+    const MT pv = (MT)ld_pre<LG>(oc.pre + o);
+    if (!__all_sync(FULL, pv == (MT)val)) { VE_DBG(4, 1); settle(); return true; }   // re-dispatched by the main loop
+    red_add_keep(reinterpret_cast<uint32_t*>(e->dense) + (o >> LG), 1u, true);
+    ++nlast;
+    VE_DBG(1, 1);
+  }
+}
+
 // Consume fast windows of access type (KIND, LG) from the ring, starting with the
 // current one (addr, val, pm; known fast).  Returns true when it stopped at a
 // window it has not consumed (left in addr, val, pm), false when the ring is empty.
@@ -1448,6 +1582,10 @@ __device__ __forceinline__ bool run_fast(const AnalyzeParams& P, const ObjCache&
   }
 }
 
+// MULTI: take the multi-key dense path (run_dense_multi) for keys without live line
+// state.  A separate instantiation, so traces with few PCs keep the register
+// allocation of the single-key kernel (launch_analyze picks by the PC count).
+template <bool MULTI>
 __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant__ AnalyzeParams P) {
   const uint32_t nsk = P.sp + P.so;
   const Smem S = smem_of(P);
@@ -1547,6 +1685,16 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       bool nd = true;
       VE_TBEG(t1);
       if (!one && !cm && se->dense != 0ull) {
+#if VE_MULTI_DENSE
+        if (MULTI && lf == 3u) {
+          switch (meta0 & 3u) {
+            case 0: have = run_dense_multi<0>(P, oc, slots, se, R, addr, val, pm, nd); break;
+            case 1: have = run_dense_multi<1>(P, oc, slots, se, R, addr, val, pm, nd); break;
+            case 2: have = run_dense_multi<2>(P, oc, slots, se, R, addr, val, pm, nd); break;
+            default: have = run_dense_multi<3>(P, oc, slots, se, R, addr, val, pm, nd); break;
+          }
+        } else
+#endif
         switch (meta0 & 3u) {
           case 0: have = run_dense<0>(P, oc, se, R, addr, val, pm, nd); break;
           case 1: have = run_dense<1>(P, oc, se, R, addr, val, pm, nd); break;
@@ -1748,14 +1896,18 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   int dev_smem = 0;
   cudaDeviceGetAttribute(&dev_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device);
   cudaFuncAttributes fa;
-  cudaFuncGetAttributes(&fa, k_analyze);
+  // many PCs interleave their warp instructions window by window (stencils, op mixes):
+  // the multi-key dense kernel; few PCs (long runs per key): the single-key kernel
+  const bool multi = VE_MULTI_DENSE && c->cfg.n_pcs >= VE_MULTI_MIN_PCS;
+  auto kfn = multi ? k_analyze<true> : k_analyze<false>;
+  cudaFuncGetAttributes(&fa, kfn);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring
   uint32_t hs = getenv("VE_HS") ? (uint32_t)atoi(getenv("VE_HS")) : 8192;
   while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > budget) hs >>= 1;
   P.hs = hs;
   carve_offsets(P, sp + so);
   const size_t sb = smem_bytes(sp + so, hs, P.objc);
-  cudaError_t e = cudaFuncSetAttribute(k_analyze, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
+  cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
   if (e != cudaSuccess) return cuda_fail(c, e, "cudaFuncSetAttribute(k_analyze)");
   if (n == 0) return VE_OK;
   uint64_t windows = (n + 31) / 32;
@@ -1783,7 +1935,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze claim counter");
 #endif
   count_launch();
-  k_analyze<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
+  kfn<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze launch");
   count_launch();
