@@ -279,7 +279,9 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   // snapshot, allocated from one pool when a (pc, access type) first claims one
   // (k_analyze's dense_lookup); the pool holds min(2^31, DENSE_PER_OBJ * sum of the
   // objects' elements) counters (<= 8 GiB), claims beyond it take the hash path
-  const uint64_t DENSE_BUDGET = 1ull << 31;
+  // (VE_DENSE_BUDGET: a smaller pool, for tests of the pool-exhausted path)
+  const uint64_t DENSE_BUDGET = getenv("VE_DENSE_BUDGET") ? strtoull(getenv("VE_DENSE_BUDGET"), nullptr, 10)
+                                                          : (1ull << 31);
   c->dense_pc_init.assign((size_t)DENSE_PER_OBJ * n, DENSE_OFF);
   uint64_t want = 0;
   for (uint32_t i = 0; i < n; ++i) {

@@ -168,3 +168,24 @@ def test_nccl_merge_single_rank(torch_cuda):
     c.merge(comm=comm)
     bad = parity.compare_with_oracle(c.report(), okeys, oglob, oobj)
     assert not bad, "\n".join(bad[:20])
+
+
+@pytest.mark.parametrize("budget", ["0", "70000", "300000"])
+def test_dense_pool_exhausted_parity(torch_cuda, budget):
+    """Dense counter arrays are allocated from one pool when a (pc, access type) first claims
+    one; claims beyond the pool take the hash path.  Results must not depend on the pool size."""
+    import os
+    old = os.environ.get("VE_DENSE_BUDGET")
+    os.environ["VE_DENSE_BUDGET"] = budget
+    try:
+        hobjs = W.host_objects(G.FUZZ, 0, 12)
+        recs = G.records_host(G.FUZZ, 0, 12, 0, 120000)
+        _check(torch_cuda, 64, hobjs, recs)
+        hobjs = W.host_objects(G.CFG1, 0, 1)
+        recs = G.records_host(G.CFG1, 0, 1, 0, 1 << 20)
+        _check(torch_cuda, 16, hobjs, recs)
+    finally:
+        if old is None:
+            del os.environ["VE_DENSE_BUDGET"]
+        else:
+            os.environ["VE_DENSE_BUDGET"] = old
