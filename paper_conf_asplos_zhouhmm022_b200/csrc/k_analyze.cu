@@ -452,7 +452,11 @@ __device__ __forceinline__ void bitmap_or(uint32_t* bm, bool part, uint64_t word
 #ifndef VE_NSLOT
 #define VE_NSLOT 8
 #endif
-constexpr int NSLOT = VE_NSLOT;
+constexpr int NSLOT = VE_NSLOT;          // slots of the multi-key kernel (cfg4 rotates 8 PCs)
+#ifndef VE_NSLOT_SINGLE
+#define VE_NSLOT_SINGLE 4
+#endif
+constexpr int NSLOT_SINGLE = VE_NSLOT_SINGLE;   // slots of the single-key kernel (few-PC traces)
 struct __align__(16) SlotE {
   uint64_t key;                 // meta << 32 | object id << 16 | pc; ~0 = free
   unsigned long long dense;     // per-element counters of (pc, object), or 0
@@ -583,15 +587,16 @@ __device__ __noinline__ void slot_flush(const AnalyzeParams& P, const SlotE* e) 
 
 // index of key's slot in the warp's cache; a miss evicts round-robin (folding the
 // victim) and initialises the slot for key's access type
+template <int NS>
 __device__ __noinline__ int slot_acquire(const AnalyzeParams& P, WarpCache& wc, SlotE* slots, uint32_t* next,
                                          uint64_t key, int oi, bool nosnap) {
-  for (int i = 0; i < NSLOT; ++i)
+  for (int i = 0; i < NS; ++i)
     if (slots[i].key == key) return i;
   int v = -1;
-  for (int i = 0; i < NSLOT; ++i)
+  for (int i = 0; i < NS; ++i)
     if (slots[i].key == ~0ull) { v = i; break; }
   if (v < 0) {
-    v = (int)(*next % NSLOT);
+    v = (int)(*next % NS);
     __syncwarp();
     if ((threadIdx.x & 31) == 0) *next = *next + 1;
     slot_line_flush(P, wc, &slots[v]);
@@ -1601,12 +1606,13 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   for (uint32_t i = tid; i < P.objc; i += blockDim.x) { S.sob[i] = P.o.base[i]; S.soe[i] = P.o.end[i]; }
   if (tid < 4) S.sctr[tid] = 0;
   __shared__ WarpCache s_wc[K1_WARPS];
-  __shared__ SlotE s_slot[K1_WARPS][NSLOT];
+  constexpr int NS = MULTI ? NSLOT : NSLOT_SINGLE;
+  __shared__ SlotE s_slot[K1_WARPS][NS];
   __shared__ uint32_t s_snext[K1_WARPS];
   WarpCache& wc = s_wc[warp];
   SlotE* slots = s_slot[warp];
   if (lane < WC) wc.key1[lane] = 0;
-  if (lane < NSLOT) slots[lane].key = ~0ull;
+  if (lane < NS) slots[lane].key = ~0ull;
   if (lane == 0) { wc.next = 0; s_snext[warp] = 0; s_stage_n[warp] = 0; }
 
   // full windows stream through the warp's TMA ring (a static contiguous range per
@@ -1670,7 +1676,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
       // the window's key slot (pc, object, access type); while one of its line states
       // is still live, windows go one at a time through the line check
       const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)oc.id << 16) | pc0;
-      SlotE* se = &slots[slot_acquire(P, wc, slots, &s_snext[warp], key, oc.oi, oc.pre == 0ull)];
+      SlotE* se = &slots[slot_acquire<NS>(P, wc, slots, &s_snext[warp], key, oc.oi, oc.pre == 0ull)];
       const uint32_t lf = se->lfail;
       // a live line state: runs of one value take the constant-run path, other windows
       // go one at a time through the per-window line check
@@ -1782,7 +1788,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
            s_dbgc[warp][1], s_dbgc[warp][2], s_dbgc[warp][3], s_dbgc[warp][4], s_dbgc[warp][5]);
 #endif
   // fold the warp's key slots and line cache, then the CTA's shared state
-  for (int i = 0; i < NSLOT; ++i)
+  for (int i = 0; i < NS; ++i)
     if (slots[i].key != ~0ull) {
       slot_line_flush(P, wc, &slots[i]);
       slot_flush(P, &slots[i]);
