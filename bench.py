@@ -319,14 +319,14 @@ def main():
     }
 
     f1 = None
-    if rank == 0 and not args.no_f1:
+    if rank == 0 and world == 1 and not args.no_f1:       # single-GPU legs: not under torchrun
         f1 = measure_next_rows(ve, ctx, wl, stream, peak)
 
     dd5 = None
-    if rank == 0 and not args.no_cfg5:
+    if rank == 0 and world == 1 and not args.no_cfg5:
         dd5 = measure_cfg5_dedup(ve, ctx, stream, peak)
     c34 = None
-    if rank == 0 and not args.no_cfg34:
+    if rank == 0 and world == 1 and not args.no_cfg34:
         c34 = measure_other_configs(ve, stream, peak)
 
     e2e = None
