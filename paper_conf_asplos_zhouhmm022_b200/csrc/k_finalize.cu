@@ -1025,14 +1025,10 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush");
   bool any = false;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaFuncSetAttribute(k_dense_flush<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_LC_SLOTS * 12));
-    cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)(DF_SLOTS * 12));
-    cudaFuncSetAttribute(k_dense_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
-    attr_set = true;
-  }
+  // (per call: the attribute belongs to the current device, and a process may drive several)
+  cudaFuncSetAttribute(k_dense_flush<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_LC_SLOTS * 12));
+  cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_SLOTS * 12));
+  cudaFuncSetAttribute(k_dense_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
   struct Arr { uint32_t i, pc, meta; unsigned long long off; };
   std::vector<Arr> arrs;
   for (uint32_t i = 0; i < c->n_obj; ++i) {
