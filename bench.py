@@ -262,7 +262,9 @@ def main():
     from paper_conf_asplos_zhouhmm022_b200 import ve
 
     wl = Workload(rank, world, dev)
-    ctx = ve.Context(n_pcs=5, max_objects=8, hist_capacity=int(os.environ.get("VE_BENCH_HCAP", 1 << 23)),
+    # hist_capacity >= 2x the distinct (pc, object, value) entries of an epoch:
+    # cfg2's gemm epoch has 1,274,116 (scripts/cfg2_ndistinct.py), so 2^22 slots (30% load)
+    ctx = ve.Context(n_pcs=5, max_objects=8, hist_capacity=int(os.environ.get("VE_BENCH_HCAP", 1 << 22)),
                      device=local)
     comm = None
     if world > 1:

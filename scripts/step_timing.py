@@ -11,7 +11,7 @@ from paper_conf_asplos_zhouhmm022_b200 import ve  # noqa: E402
 
 torch.cuda.set_device(0)
 wl = bench.Workload(0, 1, torch.device("cuda", 0))
-ctx = ve.Context(n_pcs=5, max_objects=8, hist_capacity=1 << 23, device=0)
+ctx = ve.Context(n_pcs=5, max_objects=8, hist_capacity=1 << 22, device=0)
 s = torch.cuda.current_stream()
 
 
