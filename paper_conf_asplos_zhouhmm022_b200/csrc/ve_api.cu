@@ -308,12 +308,19 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     }
     c->dense_dirty = false;
   }
-  // device object table (SoA, sorted by base)
-  cudaFree(c->obj_block);
-  c->obj_block = nullptr;
+  // device object table (SoA, sorted by base); the block is reused when it is large
+  // enough (after the device is idle: earlier launches may still read the old table)
   const size_t nn = n ? n : 1;
   const size_t nb = nn * (8 * 4 + 8 * DENSE_PER_OBJ + 4 * 2 + 4 * DENSE_PER_OBJ) + 64;
-  if (cudaMalloc(&c->obj_block, nb) != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "objects"); }
+  if (nb > c->obj_block_bytes) {
+    cudaFree(c->obj_block);
+    c->obj_block = nullptr;
+    c->obj_block_bytes = 0;
+    if (cudaMalloc(&c->obj_block, nb) != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "objects"); }
+    c->obj_block_bytes = nb;
+  } else {
+    cudaDeviceSynchronize();
+  }
   std::vector<uint8_t> host(nb, 0);
   uint64_t* hb = (uint64_t*)host.data();
   uint64_t* he = hb + n;

@@ -116,6 +116,7 @@ struct ve_ctx {
   ve::DevTables t{};
   ve::DevObjects o{};
   void* obj_block = nullptr;                 // backing store of DevObjects arrays
+  size_t obj_block_bytes = 0;
   uint64_t bm_words = 0;
   uint64_t hcap = 0;
   // dense counters (see DevObjects); disabled once 2^32 records could overflow a u32 counter
