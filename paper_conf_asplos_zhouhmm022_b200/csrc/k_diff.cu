@@ -104,8 +104,24 @@ __global__ void k_diff_scalar(const uint8_t* pre, const uint8_t* post, uint64_t 
   if (cu) atomicAdd(&out[1], cu);
 }
 
+// |W u L| of one object's bitmap words (n_untouched = n_elems - this)
+__global__ void __launch_bounds__(256) k_touched(const uint32_t* __restrict__ W, const uint32_t* __restrict__ L,
+                                                 uint64_t nw, unsigned long long* out) {
+  unsigned long long n = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x)
+    n += __popc(W[i] | L[i]);
+  for (int o = 16; o; o >>= 1) n += __shfl_xor_sync(0xFFFFFFFFu, n, o);
+  if ((threadIdx.x & 31) == 0 && n) atomicAdd(out, n);
+}
+
 ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask, ve_diff* out, cudaStream_t s) {
   const HostObject& o = c->objs[oi];
+  // counted loads set their L bits when flushed: flush first, so n_untouched does not
+  // depend on whether ve_report ran before this call (idempotent; ve_report skips it then)
+  if (!c->hist_merged) {
+    ve_status st = dense_flush(c, s);
+    if (st != VE_OK) return st;
+  }
   if (!o.pre || !o.post) return fail(c, VE_ERR_INVALID, "ve_snapshot_diff: object needs pre and post snapshots");
   const uint32_t* mask = nullptr;
   if (mode == VE_DIFF_WRITTEN) mask = c->t.W + o.bmoff;
@@ -116,10 +132,10 @@ ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask
     return fail(c, VE_ERR_INVALID, "ve_snapshot_diff: bad mode");
   }
   const uint32_t ew_lg = o.ew == 1 ? 0 : o.ew == 2 ? 1 : o.ew == 4 ? 2 : 3;
-  unsigned long long* d_out = nullptr;
-  cudaError_t e = cudaMallocAsync((void**)&d_out, 16, s);
+  unsigned long long* d_out = nullptr;   // [0] masked, [1] unchanged, [2] |W u L|
+  cudaError_t e = cudaMallocAsync((void**)&d_out, 24, s);
   if (e != cudaSuccess) return cuda_fail(c, e, "diff alloc");
-  cudaMemsetAsync(d_out, 0, 16, s);
+  cudaMemsetAsync(d_out, 0, 24, s);
   const bool aligned = (o.pre % 16 == 0) && (o.post % 16 == 0);
   uint64_t e_begin = 0;
   if (aligned) {
@@ -142,20 +158,23 @@ ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask
     k_diff_scalar<<<(unsigned)blocks, 256, 0, s>>>((const uint8_t*)o.pre, (const uint8_t*)o.post, o.size, o.ew,
                                                   e_begin, o.n_elems, mask, d_out);
   }
-  unsigned long long h[2];
-  cudaMemcpyAsync(h, d_out, 16, cudaMemcpyDeviceToHost, s);
+  // n_untouched = n_elems - |W u L|, counted in the same stream (one read-back)
+  if (o.bmwords) {
+    uint64_t blocks = (o.bmwords + 255) / 256;
+    if (blocks > (uint64_t)c->num_sms * 4) blocks = (uint64_t)c->num_sms * 4;
+    count_launch();
+    k_touched<<<(unsigned)blocks, 256, 0, s>>>(c->t.W + o.bmoff, c->t.L + o.bmoff, o.bmwords, d_out + 2);
+  }
+  unsigned long long h[3];
+  cudaMemcpyAsync(h, d_out, 24, cudaMemcpyDeviceToHost, s);
   cudaFreeAsync(d_out, s);
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "ve_snapshot_diff");
-  // n_untouched = n_elems - |W u L|
-  std::vector<ve_obj_stats> bc;
-  ve_status st = bitmap_counts(c, s, bc);
-  if (st != VE_OK) return st;
   out->n_elems = o.n_elems;
   out->n_masked = h[0];
   out->n_unchanged = h[1];
   out->n_changed = h[0] - h[1];
-  out->n_untouched = o.n_elems - bc[o.id].n_touched;
+  out->n_untouched = o.n_elems - h[2];
   out->redundant = (h[0] > 0 && (unsigned __int128)100 * h[1] > (unsigned __int128)c->cfg.t_redundant_pct * h[0]);
   out->pad = 0;
   return VE_OK;

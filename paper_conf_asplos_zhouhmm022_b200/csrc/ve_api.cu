@@ -43,6 +43,7 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->obj_block);
   cudaFree(c->scratch);
   if (c->pin) cudaFreeHost(c->pin);
+  if (c->rpin) cudaFreeHost(c->rpin);
   cudaFree(c->dense_pool);
   cudaFree(c->hstage);
   for (int i = 0; i < 2; ++i) {
@@ -447,6 +448,7 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
     c->poisoned = true;
     return fail(c, VE_ERR_CAPACITY, "value histogram capacity exceeded (hist_capacity)");
   }
+  if (glob[G_DENSE_NEXT] == 0) c->dense_dirty = false;   // no dense array was claimed: nothing to flush
   // counted loads contribute their value statistics and histogram entries first
   const bool tm = getenv("VE_TIMING") != nullptr;
   auto t0 = std::chrono::steady_clock::now();
@@ -463,11 +465,29 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
   const uint32_t nk = c->n_keys, K = c->cfg.topk;
   std::vector<uint64_t> sum((size_t)nk * NSUM), mn((size_t)nk * NMM), mx((size_t)nk * NMM);
   std::vector<LineState> line(nk);
-  cudaMemcpy(sum.data(), c->t.sum, sum.size() * 8, cudaMemcpyDeviceToHost);
-  cudaMemcpy(mn.data(), c->t.mn, mn.size() * 8, cudaMemcpyDeviceToHost);
-  cudaMemcpy(mx.data(), c->t.mx, mx.size() * 8, cudaMemcpyDeviceToHost);
-  e = cudaMemcpy(line.data(), c->t.line, nk * sizeof(LineState), cudaMemcpyDeviceToHost);
-  if (e != cudaSuccess) return cuda_fail(c, e, "ve_report copy");
+  {   // the four tables through one pinned staging area, one synchronisation
+    const size_t bs = sum.size() * 8, bm = mn.size() * 8, bl = nk * sizeof(LineState);
+    const size_t need = bs + 2 * bm + bl;
+    if (c->rpin_bytes < need) {
+      if (c->rpin) cudaFreeHost(c->rpin);
+      c->rpin = nullptr;
+      c->rpin_bytes = 0;
+      e = cudaMallocHost(&c->rpin, need);
+      if (e != cudaSuccess) { c->rpin = nullptr; return cuda_fail(c, e, "ve_report staging"); }
+      c->rpin_bytes = need;
+    }
+    uint8_t* hp = (uint8_t*)c->rpin;
+    cudaMemcpyAsync(hp, c->t.sum, bs, cudaMemcpyDeviceToHost, 0);
+    cudaMemcpyAsync(hp + bs, c->t.mn, bm, cudaMemcpyDeviceToHost, 0);
+    cudaMemcpyAsync(hp + bs + bm, c->t.mx, bm, cudaMemcpyDeviceToHost, 0);
+    cudaMemcpyAsync(hp + bs + 2 * bm, c->t.line, bl, cudaMemcpyDeviceToHost, 0);
+    e = cudaStreamSynchronize(0);
+    if (e != cudaSuccess) return cuda_fail(c, e, "ve_report copy");
+    memcpy(sum.data(), hp, bs);
+    memcpy(mn.data(), hp + bs, bm);
+    memcpy(mx.data(), hp + bs + bm, bm);
+    memcpy(line.data(), hp + bs + 2 * bm, bl);
+  }
   ve_rep* r = new (std::nothrow) ve_rep();
   if (!r) return VE_ERR_NOMEM;
   r->n_keys = nk;

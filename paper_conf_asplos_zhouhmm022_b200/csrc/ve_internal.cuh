@@ -128,6 +128,8 @@ struct ve_ctx {
   // finalize scratch
   void* scratch = nullptr;
   void* pin = nullptr;                       // pinned host staging of small report-time copies
+  void* rpin = nullptr;                      // pinned staging of the report's table copies
+  size_t rpin_bytes = 0;
   size_t scratch_bytes = 0;
   // merged histogram results (NCCL path)
   std::vector<uint64_t> merged_ndistinct;

@@ -189,3 +189,25 @@ def test_dense_pool_exhausted_parity(torch_cuda, budget):
             del os.environ["VE_DENSE_BUDGET"]
         else:
             os.environ["VE_DENSE_BUDGET"] = old
+
+
+def test_diff_before_report(torch_cuda):
+    """ve_snapshot_diff before ve_report (the bench order): n_untouched must already count the
+    elements of loads that are counted densely (their L bits are set when the counts are flushed)."""
+    ve = _ve()
+    for cfgc, seed, n, npcs in ((G.FUZZ, 7, 100000, 64), (G.CFG1, 1, 1 << 20, 16)):
+        hobjs = W.host_objects(cfgc, 0, seed)
+        recs = G.records_host(cfgc, 0, seed, 0, n)
+        ctx = ve.Context(n_pcs=npcs, max_objects=max(len(hobjs), 1), hist_capacity=1 << 20)
+        ctx.set_objects(W.device_objects(hobjs))
+        ctx.analyze_records(W.device_records(recs), n)
+        cfg = O.make_config(npcs)
+        for o in hobjs:
+            if o.get("pre") is None or o.get("post") is None:
+                continue
+            gd = ctx.snapshot_diff(o["id"], O.DIFF_WRITTEN)
+            od = O.snapshot_diff(cfg, hobjs, recs, o["id"], O.DIFF_WRITTEN)
+            assert not parity.compare_diff(gd, od), (cfgc, o["id"])
+        okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
+        assert not parity.compare_with_oracle(ctx.report(), okeys, oglob, oobj)
+        ctx.close()
