@@ -1839,7 +1839,7 @@ __global__ void __launch_bounds__(256) k_hist_drain(const uint4* __restrict__ st
   const uint4* q = stage + (uint64_t)blockIdx.x * rs;
   for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
     const uint4 e = __ldcs(q + i);
-    hist_insert_global(t, e.z, (uint64_t)e.x | ((uint64_t)e.y << 32), e.w);
+    hist_insert_global_rf(t, e.z, (uint64_t)e.x | ((uint64_t)e.y << 32), e.w);
   }
 }
 

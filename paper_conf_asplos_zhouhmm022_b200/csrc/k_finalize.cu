@@ -867,7 +867,7 @@ __device__ __forceinline__ void df_table_flush(unsigned long long* sbits, uint32
   for (uint32_t i = threadIdx.x; i < ts; i += blockDim.x) {
     if (sbits[i] != ~0ull && scnt[i]) {
       df_stats(v, sbits[i], scnt[i], kind, lg, mant_bits);
-      hist_insert_global(t, tag, sbits[i], scnt[i]);
+      hist_insert_global_rf(t, tag, sbits[i], scnt[i]);
     }
     sbits[i] = ~0ull;
     scnt[i] = 0;
@@ -944,7 +944,7 @@ __global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n
         }
         if (!done) {                     // straight to the HBM table: its statistics now
           df_stats(v, bits, sum, kind, lg, mant_bits);
-          hist_insert_global(t, tag, bits, sum);
+          hist_insert_global_rf(t, tag, bits, sum);
         }
       }
     }

@@ -375,6 +375,43 @@ __device__ __forceinline__ bool hist_insert_global(const DevTables& t, uint32_t 
   return false;
 }
 
+// Read-first insert for hit-heavy callers (report-time flushes, the K1 drain): a plain
+// 16-byte load finds an existing entry with one atomic (the count add) instead of two.
+// Slots go from empty to their final (bits, tag) once, by CAS, so a load whose low word is
+// neither empty nor `bits` proves another key (skip); any other observation (a possibly
+// torn read of a slot being claimed) is settled by the CAS itself.
+#ifndef VE_READ_FIRST
+#define VE_READ_FIRST 1
+#endif
+__device__ __forceinline__ bool hist_insert_global_rf(const DevTables& t, uint32_t tag, uint64_t bits,
+                                                      unsigned long long cnt) {
+#if VE_READ_FIRST
+  uint64_t h = hist_hash(tag, bits) & t.hmask;
+  for (uint64_t probe = 0; probe <= t.hmask; ++probe) {
+    HSlot* s = &t.hslot[h];
+    uint64_t lo, hi;
+    asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(lo), "=l"(hi) : "l"(s) : "memory");
+    if (lo == bits && hi == (uint64_t)tag) {
+      atomicAdd(&t.hcount[h], cnt);
+      return true;
+    }
+    if (lo == ~0ull || lo == bits) {
+      uint64_t olo, ohi;
+      cas128_global(s, ~0ull, ~0ull, bits, (uint64_t)tag, olo, ohi);
+      if ((olo == ~0ull && ohi == ~0ull) || (olo == bits && ohi == (uint64_t)tag)) {
+        atomicAdd(&t.hcount[h], cnt);
+        return true;
+      }
+    }
+    h = (h + 1) & t.hmask;
+  }
+  atomicExch(&t.glob[G_OVERFLOW], 1ull);
+  return false;
+#else
+  return hist_insert_global(t, tag, bits, cnt);
+#endif
+}
+
 // ---- line-state monoid (+) --------------------------------
 __device__ __forceinline__ __int128 mk128(uint64_t lo, int64_t hi) {
   return (__int128)(((unsigned __int128)(uint64_t)hi << 64) | lo);
