@@ -1822,7 +1822,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   // line states of the shared keys: one row per CTA, folded by K2 (no global locks)
   for (uint32_t s = tid; s < nsk; s += blockDim.x) P.t.lcta[(uint64_t)blockIdx.x * nsk + s] = S.sline[s];
   for (uint32_t i = tid; i < P.hs; i += blockDim.x) {
-    if (S.shs[i].tag != EMPTY_TAG) hist_insert_global(P.t, S.shs[i].tag, S.shs[i].bits, S.shc[i]);
+    if (S.shs[i].tag != EMPTY_TAG) hist_insert_global_rf(P.t, S.shs[i].tag, S.shs[i].bits, S.shc[i]);
   }
   if (tid == 0) {
     if (S.sctr[0]) atomicAdd(&P.t.glob[G_INVALID], (unsigned long long)S.sctr[0]);

@@ -33,7 +33,7 @@ __global__ void k_merge_tables(DevTables d, DevTables s, uint32_t n_keys, uint64
 __global__ void k_merge_hist(DevTables d, const HSlot* shs, const unsigned long long* shc, uint64_t scap) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < scap; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t tag = shs[i].tag;
-    if (tag != EMPTY_TAG) hist_insert_global(d, tag, shs[i].bits, shc[i]);
+    if (tag != EMPTY_TAG) hist_insert_global_rf(d, tag, shs[i].bits, shc[i]);
   }
 }
 

@@ -214,7 +214,7 @@ __global__ void k_insert_entries(const Entry* in, uint64_t n, HSlot* vs, unsigne
   t.hmask = vmask;
   t.glob = overflow - G_OVERFLOW;   // hist_insert_global flags glob[G_OVERFLOW]
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-    hist_insert_global(t, in[i].key, in[i].bits, in[i].count);
+    hist_insert_global_rf(t, in[i].key, in[i].bits, in[i].count);
 }
 
 static bool same_layout(const ve_ctx* a, const ve_ctx* b) {
