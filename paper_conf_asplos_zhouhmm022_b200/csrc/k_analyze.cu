@@ -369,15 +369,20 @@ __device__ __forceinline__ bool hist_insert_shared(const AnalyzeParams& P, uint3
   uint32_t h = (uint32_t)hist_hash(tag, bits) & hmask;
   for (int probe = 0; probe < np; ++probe) {
     HSlot* s = &S.shs[h];
-    uint64_t lo = *(volatile uint64_t*)&s->bits;
-    uint32_t stag = *(volatile uint32_t*)&s->tag;
-    if (stag == tag && lo == bits) { atomicAdd(&S.shc[h], c); return true; }
-    if (stag == EMPTY_TAG) {
-      if (*(volatile uint32_t*)&S.sctr[2] >= (P.hs >> 1)) return false;   // keep the table at most half full
-      uint64_t ehi = ((uint64_t)(*(volatile uint32_t*)&s->pad) << 32) | EMPTY_TAG;
+    // one 16-byte read of the slot.  An empty slot is (bits 0, EMPTY_TAG, pad 0) and a claim
+    // replaces both words by one 128-bit CAS; should a read ever combine the old bits with
+    // the new tag, it would look like an entry of value 0 -- so a match of value 0 is
+    // confirmed by the CAS, never taken from the read
+    uint64_t lo, hi;
+    asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];"
+                 : "=l"(lo), "=l"(hi) : "r"((uint32_t)__cvta_generic_to_shared(s)) : "memory");
+    const uint32_t stag = (uint32_t)hi;
+    if (stag == tag && lo == bits && bits != 0ull) { atomicAdd(&S.shc[h], c); return true; }
+    if (stag == EMPTY_TAG || (stag == tag && lo == bits)) {
+      if (stag == EMPTY_TAG && *(volatile uint32_t*)&S.sctr[2] >= (P.hs >> 1)) return false;   // at most half full
       uint64_t olo, ohi;
-      cas128_shared(s, lo, ehi, bits, (uint64_t)tag, olo, ohi);
-      if ((uint32_t)ohi == EMPTY_TAG && olo == lo) {
+      cas128_shared(s, 0ull, (uint64_t)EMPTY_TAG, bits, (uint64_t)tag, olo, ohi);
+      if ((uint32_t)ohi == EMPTY_TAG && olo == 0ull) {
         atomicAdd(&S.sctr[2], 1u);
         atomicAdd(&S.shc[h], c);
         return true;

@@ -391,7 +391,7 @@ __device__ __forceinline__ bool hist_insert_global_rf(const DevTables& t, uint32
     HSlot* s = &t.hslot[h];
     uint64_t lo, hi;
     asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(lo), "=l"(hi) : "l"(s) : "memory");
-    if (lo == bits && hi == (uint64_t)tag) {
+    if (lo == bits && hi == (uint64_t)tag && bits != ~0ull) {   // (value ~0: confirmed by the CAS below)
       atomicAdd(&t.hcount[h], cnt);
       return true;
     }
