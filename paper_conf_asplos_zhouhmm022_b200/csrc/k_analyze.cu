@@ -1913,7 +1913,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   auto kfn = multi ? k_analyze<true> : k_analyze<false>;
   cudaFuncGetAttributes(&fa, kfn);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring
-  uint32_t hs = getenv("VE_HS") ? (uint32_t)atoi(getenv("VE_HS")) : 8192;
+  // 2048 slots measured best on cfg2 / cfg3 / cfg4 (the HBM table behind it stays L2-resident)
+  uint32_t hs = getenv("VE_HS") ? (uint32_t)atoi(getenv("VE_HS")) : 2048;
   while (hs > 256 && smem_bytes(sp + so, hs, P.objc) > budget) hs >>= 1;
   P.hs = hs;
   carve_offsets(P, sp + so);
