@@ -799,7 +799,7 @@ ve_status finalize_hist_views(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& 
 constexpr int DF_THREADS = 256;
 constexpr int DF_SLOTS = 1024;
 #ifndef VE_DF_CHUNK
-#define VE_DF_CHUNK 1024
+#define VE_DF_CHUNK 2048
 #endif
 constexpr uint64_t DF_CHUNK = VE_DF_CHUNK;    // elements per block: many blocks keep the global inserts in flight
 
