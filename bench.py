@@ -541,7 +541,7 @@ def measure_e2e(ve, ctx, wl, stream, steps):
     torch.cuda.synchronize()
     dt = (time.perf_counter() - t) / steps
     return {"value": wl.total_records / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-            "ms_per_step": dt * 1e3, "steps": steps, "path": "ve_analyze_records_host (pinned, double-buffered)"}
+            "ms_per_step": dt * 1e3, "steps": steps, "path": "ve_analyze_records_host (pinned; two staging buffers, H2D on a side stream overlapped with the analysis)"}
 
 
 if __name__ == "__main__":

@@ -49,7 +49,9 @@ static void free_dev(ve_ctx* c) {
   for (int i = 0; i < 2; ++i) {
     if (c->stage[i]) cudaFree(c->stage[i]);
     if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);
+    if (c->copied_ev[i]) cudaEventDestroy(c->copied_ev[i]);
   }
+  if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
 }
 
 ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
@@ -401,12 +403,26 @@ ve_status ve_analyze_records_host(ve_ctx* c, const ve_record* h, uint64_t n, cud
     }
     c->stage_bytes = CH * sizeof(ve_record);
   }
-  // chunk i: copy into stage[i%2] (after that buffer's previous analysis), then analyze it
+  if (!c->copy_stream) {
+    if (cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->copied_ev[0], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->copied_ev[1], cudaEventDisableTiming) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(c, VE_ERR_NOMEM, "copy stream");
+    }
+  }
+  // chunk i: the copy stream fills stage[i%2] once that buffer's previous analysis is done,
+  // and stream s analyses it once the copy is done -- copy i+1 overlaps analysis i
+  cudaEventRecord(c->stage_ev[0], s);   // nothing of this call may overtake earlier work on s
+  cudaEventRecord(c->stage_ev[1], s);
   for (uint64_t off = 0, i = 0; off < n; off += CH, ++i) {
     const int b = (int)(i & 1);
     const uint64_t m = std::min(CH, n - off);
-    cudaError_t e = cudaStreamWaitEvent(s, c->stage_ev[b], 0);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(c->stage[b], h + off, m * sizeof(ve_record), cudaMemcpyHostToDevice, s);
+    cudaError_t e = cudaStreamWaitEvent(c->copy_stream, c->stage_ev[b], 0);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(c->stage[b], h + off, m * sizeof(ve_record), cudaMemcpyHostToDevice, c->copy_stream);
+    if (e == cudaSuccess) e = cudaEventRecord(c->copied_ev[b], c->copy_stream);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(s, c->copied_ev[b], 0);
     if (e != cudaSuccess) return cuda_fail(c, e, "ve_analyze_records_host copy");
     ve_status st = launch_analyze(c, (const ve_record*)c->stage[b], m, s);
     if (st != VE_OK) return st;

@@ -137,6 +137,8 @@ struct ve_ctx {
   // host staging for ve_analyze_records_host
   void* stage[2] = {nullptr, nullptr};
   cudaEvent_t stage_ev[2] = {nullptr, nullptr};
+  cudaEvent_t copied_ev[2] = {nullptr, nullptr};
+  cudaStream_t copy_stream = nullptr;        // H2D of the staging buffers, overlapped with analysis
   size_t stage_bytes = 0;
   // K1's S8 insert staging (k_hist_drain)
   void* hstage = nullptr;

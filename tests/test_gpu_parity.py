@@ -211,3 +211,25 @@ def test_diff_before_report(torch_cuda):
         okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
         assert not parity.compare_with_oracle(ctx.report(), okeys, oglob, oobj)
         ctx.close()
+
+
+def test_analyze_records_host_parity(torch_cuda):
+    """ve_analyze_records_host: host records streamed through the two staging buffers (2 Mi records
+    each, copies on a side stream overlapped with the analysis) -- several chunks, a ragged tail."""
+    ve = _ve()
+    seed, n = 13, (1 << 21) * 2 + 12345
+    hobjs = W.host_objects(G.FUZZ, 0, seed)
+    recs = G.records_host(G.FUZZ, 0, seed, 0, n)
+    cfg = O.make_config(64)
+    okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
+    import torch
+    ctx = ve.Context(n_pcs=64, max_objects=8, hist_capacity=1 << 22)
+    ctx.set_objects(W.device_objects(hobjs))
+    pinned = torch.from_numpy(recs.view(np.uint8)).pin_memory()
+    ctx.analyze_records_host(pinned, n)
+    assert not parity.compare_with_oracle(ctx.report(), okeys, oglob, oobj)
+    ctx.reset()
+    ctx.set_objects(W.device_objects(hobjs))
+    ctx.analyze_records_host(recs, n)                 # pageable numpy memory
+    assert not parity.compare_with_oracle(ctx.report(), okeys, oglob, oobj)
+    ctx.close()
