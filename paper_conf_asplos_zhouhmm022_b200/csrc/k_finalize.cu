@@ -613,17 +613,21 @@ __global__ void k_emit(const HSlot* hs, const unsigned long long* hc, const uint
 // the distinct tags found by k_tagscan, compacted: out[0] = count, then (tag, entries)
 // pairs (up to TAGL_MAX; the host falls back to the full table beyond)
 constexpr uint32_t TAGL_MAX = 8192;
-__global__ void k_tag_compact(const uint32_t* tags, const unsigned long long* tcnt, unsigned long long* out) {
-  __shared__ unsigned int n;
-  if (threadIdx.x == 0) n = 0;
-  __syncthreads();
-  for (uint32_t i = threadIdx.x; i < TAG_CAP; i += blockDim.x) {
-    if (tags[i] == EMPTY_TAG) continue;
-    const unsigned p = atomicAdd(&n, 1u);
+// one thread per tag-table entry, one claim per warp (out[0] zeroed before the launch)
+__global__ void __launch_bounds__(256) k_tag_compact(const uint32_t* tags, const unsigned long long* tcnt,
+                                                    unsigned long long* out) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  const bool f = i < TAG_CAP && tags[i] != EMPTY_TAG;
+  const unsigned m = __ballot_sync(0xFFFFFFFFu, f);
+  if (!m) return;
+  const int lane = threadIdx.x & 31;
+  unsigned long long base = 0;
+  if (lane == 0) base = atomicAdd(&out[0], (unsigned long long)__popc(m));
+  base = __shfl_sync(0xFFFFFFFFu, base, 0);
+  if (f) {
+    const unsigned long long p = base + __popc(m & ((1u << lane) - 1u));
     if (p < TAGL_MAX) { out[1 + 2 * p] = tags[i]; out[2 + 2 * p] = tcnt[i]; }
   }
-  __syncthreads();
-  if (threadIdx.x == 0) out[0] = n;
 }
 
 // Exact n_distinct and top-k of every key (PC keys, then object keys).
@@ -659,7 +663,8 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   count_launch();
   k_tagscan<<<grid, 256, 0, s>>>(c->t.hslot, c->hcap, d_tags, d_tcnt, d_small, d_occ, d_small + 1);
   count_launch();
-  k_tag_compact<<<1, 1024, 0, s>>>(d_tags, d_tcnt, d_tl);
+  cudaMemsetAsync(d_tl, 0, 8, s);
+  k_tag_compact<<<(TAG_CAP + 255) / 256, 256, 0, s>>>(d_tags, d_tcnt, d_tl);
   cudaMemcpyAsync(hp, d_tl, (1 + 2 * TAGL_MAX) * 8, cudaMemcpyDeviceToHost, s);
   cudaMemcpyAsync(hp + 1 + 2 * TAGL_MAX, d_small, 8, cudaMemcpyDeviceToHost, s);
   e = cudaStreamSynchronize(s);
