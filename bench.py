@@ -324,9 +324,10 @@ def main():
     if rank == 0 and world == 1 and not args.no_f1:       # single-GPU legs: not under torchrun
         f1 = measure_next_rows(ve, ctx, wl, stream, peak)
 
-    dd5 = None
+    dd5 = r5 = None
     if rank == 0 and world == 1 and not args.no_cfg5:
         dd5 = measure_cfg5_dedup(ve, ctx, stream, peak)
+        r5 = measure_cfg5_records(ve, stream, peak)
     c34 = None
     if rank == 0 and world == 1 and not args.no_cfg34:
         c34 = measure_other_configs(ve, stream, peak)
@@ -354,7 +355,7 @@ def main():
                              "alg_bytes_per_launch": alg[1]},
                 "analyze_ms_per_step": [round(statistics.mean(a[i] for a in an_ms), 4) for i in (0, 1)],
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
-                "next_rows": f1, "cfg5_dedup": dd5, "cfg3_cfg4": c34,
+                "next_rows": f1, "cfg5_dedup": dd5, "cfg5_records": r5, "cfg3_cfg4": c34,
                 "parity_spot_check": spot}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -499,6 +500,81 @@ def measure_cfg5_dedup(ve, ctx, stream, peak, reps=3):
                         "5% one-bit flips / 55% random", "objects": len(objs), "bytes": total, "ms": ms,
             "alg_bytes": alg, "alg_gbs": alg / (ms / 1e3) / 1e9, "frac_of_hbm_peak": alg / (ms / 1e3) / 1e9 / peak,
             "groups": len(set(want)), "parity_closed_form": [int(x) for x in g] == want}
+
+
+def measure_cfg5_records(ve, stream, peak):
+    """BASELINE configs[4] (cfg5), records half: 4000 independent kernels, 10^9 records in total (4..64 PCs,
+    1..4 objects, 2,987 .. 1,676,166 records each; gen/ve_gen_core.h veg_cfg5_record).  All records and
+    snapshots are generated on the device first (untimed, 24 GB + 2 x 4 GB); the timed region is the
+    per-kernel analysis a user runs -- ve_set_objects + ve_analyze_records + ve_report for every kernel
+    on ONE context -- bracketed by CUDA events; events around each ve_analyze_records give the share of
+    the analysis kernels.  Parity at full size: the recipe's closed forms (tests/cfg5k.py) on every 50th
+    kernel (kernel-by-kernel oracle parity is tests/test_gpu_cfg5.py)."""
+    import torch
+    from gen import vegen as G
+    from tests import cfg5k
+    sp = stream.cuda_stream
+    cfg, seed, K = G.scaled(G.CFG5, 0), 5, 4000
+    infos = [G.info(cfg, k) for k in range(K)]
+    n_tot = sum(i["n_records"] for i in infos)
+    recs = torch.empty(n_tot * REC_BYTES, dtype=torch.uint8, device="cuda")
+    objs_of = [G.objects(cfg, k) for k in range(K)]
+    snap_tot = sum(o["size"] for objs in objs_of for o in objs)
+    snaps = torch.empty(2 * snap_tot, dtype=torch.uint8, device="cuda")
+    r0, s0, plan = 0, 0, []
+    for k in range(K):
+        n = infos[k]["n_records"]
+        G.records_device(cfg, k, seed, 0, n, recs.data_ptr() + r0 * REC_BYTES, sp)
+        dobjs = []
+        for i, o in enumerate(objs_of[k]):
+            d = {f: o[f] for f in ("base", "size", "id", "elem_width")}
+            for side in ("pre", "post"):
+                t = snaps[s0:s0 + o["size"]]
+                s0 += o["size"]
+                G.snapshot_device(cfg, k, seed, i, side == "post", t.data_ptr(), sp)
+                d[side] = t
+            dobjs.append(d)
+        plan.append((recs[r0 * REC_BYTES:(r0 + n) * REC_BYTES], n, dobjs))
+        r0 += n
+    ctx = ve.Context(n_pcs=64, max_objects=4, hist_capacity=1 << 23)
+    for buf, n, dobjs in plan[:8]:                                 # warm the context (untimed)
+        ctx.set_objects(dobjs)
+        ctx.analyze_records(buf, n, stream=sp)
+        ctx.report().close()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    bad, checked = [], 0
+    a.record(stream)
+    for k, (buf, n, dobjs) in enumerate(plan):
+        ctx.set_objects(dobjs)
+        ev[k][0].record(stream)
+        ctx.analyze_records(buf, n, stream=sp)
+        ev[k][1].record(stream)
+        rep = ctx.report()
+        if k % 50 == 0:
+            keys = {f: rep.keys[f].copy() for f in ("n_ld", "n_st", "n_ld_eq_pre", "n_st_eq_pre", "raw_min",
+                                                     "raw_max", "single_zero", "single_value")}
+            plan[k] = (buf, n, dobjs, keys, int(rep.globals["n_records"]))
+        rep.close()
+    b.record(stream)
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b)
+    an_ms = sum(x.elapsed_time(y) for x, y in ev)
+    for k in range(0, K, 50):
+        bad += cfg5k.check_cfg5_kernel(plan[k][3], plan[k][4], cfg, k)
+        checked += 1
+    ctx.close()
+    del plan, recs, snaps
+    torch.cuda.empty_cache()
+    gbs = n_tot * REC_BYTES / (ms / 1e3) / 1e9
+    return {"workload": "cfg5 records: 4000 kernels, 4-64 PCs with cfg1 roles, 1-4 objects, 10^9 records",
+            "kernels": K, "records": n_tot, "snapshot_bytes": 2 * snap_tot, "ms": ms,
+            "records_per_s": n_tot / (ms / 1e3), "trace_gbs": gbs, "trace_frac_of_hbm_peak": gbs / peak,
+            "analyze_ms": an_ms, "analyze_records_per_s": n_tot / (an_ms / 1e3),
+            "per_kernel_overhead_ms": (ms - an_ms) / K, "closed_forms_kernels_checked": checked,
+            "closed_forms_ok": not bad, "closed_form_mismatches": bad[:5],
+            "timed": "set_objects + analyze + report per kernel on one context, CUDA events around the loop"}
 
 
 def measure_e2e(ve, ctx, wl, stream, steps):

@@ -27,6 +27,11 @@ VEG_FN uint64_t snap_word(int cfg, int epoch, uint64_t seed, uint32_t obj, int p
     return veg_c3_elem(seed, sh, obj, post, 2 * j) | (veg_c3_elem(seed, sh, obj, post, 2 * j + 1) << 32);
   }
   if (VEG_BASE(cfg) == VEG_CFG4) return veg_c4_elem(seed, VEG_SHIFT(cfg), (uint32_t)epoch, obj, post, j);
+  if (VEG_BASE(cfg) == VEG_CFG5) {
+    const uint32_t sh = VEG_SHIFT(cfg);
+    return (uint64_t)veg_c5_elem(seed, sh, (uint32_t)epoch, obj, post, 2 * j) |
+           ((uint64_t)veg_c5_elem(seed, sh, (uint32_t)epoch, obj, post, 2 * j + 1) << 32);
+  }
   if (cfg == VEG_FUZZ) return veg_fuzz_word(seed, obj, post, j);
   return 0;
 }
@@ -36,6 +41,7 @@ VEG_FN void record_at(int cfg, int epoch, uint64_t seed, uint64_t r, veg_record*
   else if (cfg == VEG_CFG2) veg_cfg2_record(seed, (uint32_t)epoch, r, out);
   else if (VEG_BASE(cfg) == VEG_CFG3) veg_cfg3_record(seed, VEG_SHIFT(cfg), r, out);
   else if (VEG_BASE(cfg) == VEG_CFG4) veg_cfg4_record(seed, VEG_SHIFT(cfg), (uint32_t)epoch, r, out);
+  else if (VEG_BASE(cfg) == VEG_CFG5) veg_cfg5_record(seed, VEG_SHIFT(cfg), (uint32_t)epoch, r, out);
   else veg_fuzz_record(seed, r, out);
 }
 
@@ -65,6 +71,13 @@ extern "C" int veg_info_get(int cfg, int epoch, veg_info* out) {
     out->n_epochs = 2;
     return 0;
   }
+  if (VEG_BASE(cfg) == VEG_CFG5) {                /* one epoch per kernel of the 4000-kernel application */
+    if (epoch < 0 || epoch >= (int)VEG_C5_KERNELS || VEG_SHIFT(cfg) > 7 || (cfg & ~0xFFF)) return -1;
+    out->n_records = veg_c5_n(VEG_SHIFT(cfg), (uint32_t)epoch);
+    out->n_pcs = veg_c5_npcs((uint32_t)epoch); out->n_obj = veg_c5_nobj((uint32_t)epoch);
+    out->n_epochs = VEG_C5_KERNELS;
+    return 0;
+  }
   if (cfg == VEG_FUZZ) {
     if (epoch != 0) return -1;
     out->n_records = 0; out->n_pcs = VEG_FZ_NPCS; out->n_obj = VEG_FZ_NOBJ; out->n_epochs = 1;
@@ -85,6 +98,8 @@ extern "C" int veg_object_get(int cfg, int epoch, uint32_t i, veg_object* out) {
     *out = veg_c3_object(VEG_SHIFT(cfg), i);
   } else if (VEG_BASE(cfg) == VEG_CFG4) {
     *out = veg_c4_object(VEG_SHIFT(cfg), i);
+  } else if (VEG_BASE(cfg) == VEG_CFG5) {
+    *out = veg_c5_object(VEG_SHIFT(cfg), (uint32_t)epoch, i);
   } else {
     *out = veg_fuzz_object(i);
   }

@@ -40,7 +40,7 @@ typedef struct veg_info {
   uint32_t n_epochs, pad;
 } veg_info;
 
-enum { VEG_CFG1 = 1, VEG_CFG2 = 2, VEG_CFG3 = 3, VEG_CFG4 = 4, VEG_FUZZ = 100, VEG_DEDUP = 101 };
+enum { VEG_CFG1 = 1, VEG_CFG2 = 2, VEG_CFG3 = 3, VEG_CFG4 = 4, VEG_CFG5 = 5, VEG_FUZZ = 100, VEG_DEDUP = 101 };
 /* cfg codes of the scalable configs carry a size shift s in bits 8..11:
  * VEG_CFG3 | (s << 8) is cfg3 with every tensor 2^s times smaller (s = 0: full size) */
 #define VEG_BASE(cfg) ((cfg) & 0xFF)
@@ -766,6 +766,99 @@ VEG_FN uint64_t veg_dedup_word(uint64_t seed, uint32_t i, uint32_t cls, uint32_t
   uint64_t v = (src_cls == 0) ? 0 : veg_h(seed, 5000 + src, j);
   if (cls == 2 && j == veg_h(seed, 4002, i) % words) v ^= 1ull << (veg_h(seed, 4003, i) % 64);
   return v;
+}
+
+
+/* =========================================================================
+ * cfg5 records half (BASELINE.json configs[4]; SURVEY 8(d) cfg5 "Kernels"):
+ * 4000 independent kernels, epoch = kernel index k.  Kernel k has P = 4..64
+ * PCs whose roles are drawn from cfg1's 16 roles, touches O = 1..4 objects
+ * of 4-byte elements, and has n_k records: octave-uniform raw draws in
+ * [10^4, 2*10^6), rescaled in groups of 8 kernels so every group sums to
+ * exactly 2*10^6 records (500 groups: 1,000,000,000 records in total).
+ * The geometry (P, O, roles, n_k) is drawn from the fixed seed 5 so that it
+ * does not depend on the value seed; shift s divides every n_k by 2^s.
+ *
+ * Record r of kernel k: warp g = r / 32 belongs to PC p = g % P (round robin,
+ * like cfg1), PC p lives on object o = p % O in slot s = p / O of L elements
+ * (L = 32 * ceil(ceil(n/32) / P)); its element is e = s L + (g / P) 32 + r % 32
+ * and it carries veg_cfg1_value(seed, role, e).  pre follows cfg1's per-role
+ * rule; post = pre + the stores (elements no record covers keep pre).
+ * ========================================================================= */
+#define VEG_C5_KERNELS 4000u
+#define VEG_C5_GROUP 8u
+#define VEG_C5_GROUP_N 2000000ull
+#define VEG_C5_GEOM_SEED 5ull
+#define VEG_C5_BASE 0x7c0000000000ull
+
+VEG_FN uint64_t veg_c5_raw(uint32_t k) {              /* octave-uniform in [1e4, 2e6) */
+  uint64_t h = veg_h(VEG_C5_GEOM_SEED, 500, k);
+  uint64_t lo = 10000ull << (h % 8);
+  uint64_t hi = 2 * lo < 2000000ull ? 2 * lo : 2000000ull;
+  return lo + (h >> 8) % (hi - lo);
+}
+VEG_FN uint64_t veg_c5_n(uint32_t sh, uint32_t k) {
+  uint32_t g0 = k - k % VEG_C5_GROUP;
+  uint64_t S = 0, part = 0;
+  for (uint32_t j = 0; j < VEG_C5_GROUP; ++j) S += veg_c5_raw(g0 + j);
+  uint64_t n;
+  if (k % VEG_C5_GROUP != VEG_C5_GROUP - 1) {
+    n = veg_c5_raw(k) * VEG_C5_GROUP_N / S;
+  } else {
+    for (uint32_t j = 0; j + 1 < VEG_C5_GROUP; ++j) part += veg_c5_raw(g0 + j) * VEG_C5_GROUP_N / S;
+    n = VEG_C5_GROUP_N - part;
+  }
+  return n >> sh;
+}
+VEG_FN uint32_t veg_c5_npcs(uint32_t k) { return 4u + (uint32_t)(veg_h(VEG_C5_GEOM_SEED, 501, k) % 61u); }
+VEG_FN uint32_t veg_c5_nobj(uint32_t k) { return 1u + (uint32_t)((veg_h(VEG_C5_GEOM_SEED, 501, k) >> 8) % 4u); }
+VEG_FN uint32_t veg_c5_role(uint32_t k, uint32_t p) {
+  return (uint32_t)(veg_h(VEG_C5_GEOM_SEED, 502, (uint64_t)k * 64u + p) % 16u);
+}
+/* elements per PC slot */
+VEG_FN uint64_t veg_c5_slot(uint64_t n, uint32_t P) { return 32ull * ((((n + 31) / 32) + P - 1) / P); }
+
+VEG_FN veg_object veg_c5_object(uint32_t sh, uint32_t k, uint32_t i) {
+  veg_object o;
+  uint32_t P = veg_c5_npcs(k), O = veg_c5_nobj(k);
+  uint64_t L = veg_c5_slot(veg_c5_n(sh, k), P);
+  uint32_t slots = (P - i + O - 1) / O;                /* PCs p = i, i + O, ... */
+  o.base = VEG_C5_BASE + ((uint64_t)i << 36);
+  o.size = 4ull * L * slots;
+  o.id = i;
+  o.elem_width = 4;
+  o.has_pre = 1;
+  o.has_post = 1;
+  return o;
+}
+
+VEG_FN void veg_cfg5_record(uint64_t seed, uint32_t sh, uint32_t k, uint64_t r, veg_record* out) {
+  uint32_t P = veg_c5_npcs(k), O = veg_c5_nobj(k);
+  uint64_t L = veg_c5_slot(veg_c5_n(sh, k), P);
+  uint64_t g = r / 32;
+  uint32_t p = (uint32_t)(g % P), o = p % O, role = veg_c5_role(k, p);
+  uint64_t e = (uint64_t)(p / O) * L + (g / P) * 32 + r % 32;
+  out->addr = VEG_C5_BASE + ((uint64_t)o << 36) + 4 * e;
+  out->value = veg_cfg1_value(seed, role, e);
+  out->pc = p;
+  out->meta = veg_cfg1_meta(role);
+}
+
+/* element e of object i (pre or post) */
+VEG_FN uint32_t veg_c5_elem(uint64_t seed, uint32_t sh, uint32_t k, uint32_t i, int post, uint64_t e) {
+  uint32_t P = veg_c5_npcs(k), O = veg_c5_nobj(k);
+  uint64_t n = veg_c5_n(sh, k), L = veg_c5_slot(n, P);
+  uint32_t p = (uint32_t)(e / L) * O + i, role = veg_c5_role(k, p);
+  uint64_t w = e % L;
+  uint32_t v = veg_cfg1_value(seed, role, e);
+  uint32_t pre = v;                                    /* cfg1's per-role pre rule */
+  if (role >= 8) {
+    if (role == 8 || role == 11 || role == 13) pre = 0;
+    else if (role == 9) pre = (e % 2 == 0) ? v : (v ^ 1u);
+    else pre = v ^ 1u;
+  }
+  int covered = ((w / 32) * P + p) * 32 + w % 32 < n;
+  return (post && role >= 8 && covered) ? v : pre;
 }
 
 #endif /* VE_GEN_CORE_H */

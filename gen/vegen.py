@@ -8,12 +8,12 @@ import os
 
 import numpy as np
 
-CFG1, CFG2, CFG3, CFG4, FUZZ = 1, 2, 3, 4, 100
-SEEDS = {CFG1: 1, CFG2: 2, CFG3: 3, CFG4: 4}
+CFG1, CFG2, CFG3, CFG4, CFG5, FUZZ = 1, 2, 3, 4, 5, 100
+SEEDS = {CFG1: 1, CFG2: 2, CFG3: 3, CFG4: 4, CFG5: 5}
 
 
 def scaled(cfg, shift):
-    """cfg code of cfg3 / cfg4 with every tensor 2^shift times smaller (0 = full size)."""
+    """cfg code of cfg3 / cfg4 / cfg5 with every tensor 2^shift times smaller (0 = full size)."""
     return cfg | (shift << 8)
 
 REC_DTYPE = np.dtype([("addr", "<u8"), ("value", "<u8"), ("pc", "<u4"), ("meta", "<u4")])
@@ -126,3 +126,22 @@ def dedup_host(seed, i, unit):
 def dedup_device(seed, i, unit, d_ptr, stream_ptr=0):
     if lib().veg_dedup_device(seed, i, unit, ctypes.c_void_p(d_ptr), ctypes.c_void_p(stream_ptr)) != 0:
         raise RuntimeError("veg_dedup_device failed")
+
+
+_M64 = (1 << 64) - 1
+
+
+def _mix64(z):
+    z = (z + 0x9E3779B97F4A7C15) & _M64
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & _M64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & _M64
+    return z ^ (z >> 31)
+
+
+def _h(seed, stream, i):
+    return _mix64((_mix64(seed ^ ((stream * 0xD1B54A32D192ED03) & _M64)) + i) & _M64)
+
+
+def c5_role(k, p):
+    """cfg1 role of PC p of cfg5 kernel k (ve_gen_core.h veg_c5_role, geometry seed 5)"""
+    return _h(5, 502, k * 64 + p) % 16
