@@ -216,6 +216,23 @@ def temporal_loads(cfg, objs, recs):
     return out
 
 
+DYADIC_DTYPE = np.dtype([("state", "<u4"), ("scale", "<u4"), ("px", "<u8"), ("qx", "<u8"), ("py", "<i8"),
+                         ("qy", "<i8")])
+
+
+def dyadic_fit(cfg, objs, recs):
+    """C21 (f2): DYADIC_DTYPE[n_keys] -- exact linear fit over the records' exact values."""
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    out = np.zeros(cfg.n_pcs + len(objs) + 1, dtype=DYADIC_DTYPE)
+    L = lib()
+    L.vo_dyadic_fit.argtypes = [ctypes.POINTER(VoConfig), ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+                                ctypes.c_uint64, ctypes.c_void_p]
+    if L.vo_dyadic_fit(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), out.ctypes.data) != 0:
+        raise ValueError("vo_dyadic_fit rejected its arguments")
+    return out
+
+
 # ---- C18-C20: value flow graph (layouts of ve.h's ve_api_access / ve_vfg_edge / ve_vfg_vertex)
 HOST_VERTEX = 0xFFFFFFFF
 ACCESS_DTYPE = np.dtype([("seq", "<u8"), ("bytes", "<u8"), ("vertex", "<u4"), ("object", "<u4"), ("mode", "<u4"),

@@ -920,3 +920,123 @@ uint64_t vo_sizeof(int which) {
     default: return sizeof(vo_record);
   }
 }
+
+/* ---- C21: dyadic-scaled exact linear fit (f2; Def 3.7 P:L187-L189 over exact float values) ----
+ * DESIGN.md reading R10.  Every valid record of a key is a point (x = addr, y = the exact real
+ * value of its bits: integers as such, floats as the dyadic rational (-1)^s M 2^E they encode).
+ * The key is a *dyadic line* when all points lie on one straight line.  Steps, in order:
+ *  1. NaN or infinity among the key's records -> FAIL;
+ *  2. T = the largest number of fractional bits of any y (0 for integers), so that every
+ *     Y = y 2^T is an integer; some |Y| >= 2^62 -> FAIL (the bound of the exact check);
+ *  3. P = (min x, smallest Y at that x), Q = (max x, smallest Y at that x);
+ *  4. every point collinear with P and Q (exact 128-bit cross product), and a point at P.x or
+ *     Q.x equal to that anchor (one value per address) -> LINE (POINT when P.x == Q.x), else FAIL.  No valid record -> EMPTY. */
+
+/* exact value of a record as M * 2^E with M odd (or M = 0, E = 0); returns 0 for NaN / inf */
+static int exact_value(uint64_t b, uint32_t kind, uint32_t w, int64_t* M, int* E) {
+  if (kind == 0 || kind == 1) {
+    if (kind == 0 && b >= (1ull << 63)) { *M = INT64_MAX; *E = 0; return 1; }   /* overflows step 2 */
+    *M = (kind == 0) ? (int64_t)b : sext(b, w);
+    *E = 0;
+  } else {
+    int eb, mb;
+    if (kind == 3) { eb = 8; mb = 7; }
+    else if (w == 2) { eb = 5; mb = 10; }
+    else if (w == 4) { eb = 8; mb = 23; }
+    else { eb = 11; mb = 52; }
+    const uint64_t sign = (b >> (eb + mb)) & 1u;
+    const uint64_t ex = (b >> mb) & ((1ull << eb) - 1);
+    const uint64_t man = b & ((1ull << mb) - 1);
+    const int bias = (1 << (eb - 1)) - 1;
+    if (ex == (1ull << eb) - 1) return 0;                  /* inf / NaN */
+    uint64_t sig;
+    int e2;
+    if (ex == 0) { sig = man; e2 = 1 - bias - mb; }         /* zero / subnormal */
+    else { sig = man | (1ull << mb); e2 = (int)ex - bias - mb; }
+    *M = sign ? -(int64_t)sig : (int64_t)sig;
+    *E = e2;
+  }
+  if (*M == 0) { *E = 0; return 1; }
+  while ((*M & 1) == 0) { *M /= 2; *E += 1; }
+  return 1;
+}
+
+/* Y = M 2^s (s >= 0); returns 0 if |Y| >= 2^62 */
+static int scaled_y(int64_t M, int s, i128* Y) {
+  if (M == 0) { *Y = 0; return 1; }
+  const uint64_t a = M < 0 ? (uint64_t)(-(M + 1)) + 1u : (uint64_t)M;
+  int bits = 64 - __builtin_clzll(a);
+  if (bits + s > 62) return 0;
+  *Y = (i128)M * ((i128)1 << s);
+  return 1;
+}
+
+int vo_dyadic_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs, uint64_t n,
+                  vo_dyadic* out) {
+  if (!cfg || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t n_keys = (uint64_t)cfg->n_pcs + n_obj + 1;
+  int* have = (int*)calloc(n_keys, sizeof(int));
+  int* fail = (int*)calloc(n_keys, sizeof(int));
+  int* T = (int*)calloc(n_keys, sizeof(int));
+  int* hp = (int*)calloc(n_keys, sizeof(int));
+  int* hq = (int*)calloc(n_keys, sizeof(int));
+  i128* py = (i128*)calloc(n_keys, sizeof(i128));
+  i128* qy = (i128*)calloc(n_keys, sizeof(i128));
+  memset(out, 0, sizeof(vo_dyadic) * n_keys);
+  for (int pass = 1; pass <= 3; ++pass) {
+    for (uint64_t i = 0; i < n; ++i) {
+      const vo_record* r = &recs[i];
+      dec_t d;
+      decode(cfg, &t, r, &d);
+      if (!d.valid) continue;
+      uint64_t kset[2];
+      int nk = 0;
+      kset[nk++] = r->pc;                                  /* PC key, object key as in C1 */
+      if (d.shared) kset[nk++] = (uint64_t)cfg->n_pcs + n_obj;
+      else if (d.obj) kset[nk++] = (uint64_t)cfg->n_pcs + d.obj->id;
+      int64_t M = 0;
+      int E = 0;
+      const int finite = exact_value(r->value, d.kind, d.w, &M, &E);
+      for (int j = 0; j < nk; ++j) {
+        const uint64_t k = kset[j];
+        vo_dyadic* o = &out[k];
+        if (pass == 1) {                                   /* step 1, T of step 2, extreme x */
+          if (!finite) { fail[k] = 1; continue; }
+          if (-E > T[k]) T[k] = -E;
+          if (!have[k] || r->addr < o->px) o->px = r->addr;
+          if (!have[k] || r->addr > o->qx) o->qx = r->addr;
+          have[k] = 1;
+          continue;
+        }
+        if (fail[k]) continue;
+        i128 Y;
+        if (!scaled_y(M, E + T[k], &Y)) { fail[k] = 1; continue; }   /* step 2 bound */
+        if (pass == 2) {                                   /* step 3: anchors */
+          if (r->addr == o->px && (!hp[k] || Y < py[k])) { py[k] = Y; hp[k] = 1; }
+          if (r->addr == o->qx && (!hq[k] || Y < qy[k])) { qy[k] = Y; hq[k] = 1; }
+        } else if (!collinear((i128)o->px, py[k], (i128)o->qx, qy[k], (i128)r->addr, Y) ||
+                   (r->addr == o->px && Y != py[k]) || (r->addr == o->qx && Y != qy[k])) {
+          fail[k] = 1;                                     /* step 4 (one value per x) */
+        }
+      }
+    }
+  }
+  for (uint64_t k = 0; k < n_keys; ++k) {
+    vo_dyadic* o = &out[k];
+    if (fail[k] || !have[k]) {
+      memset(o, 0, sizeof(*o));
+      o->state = fail[k] ? VO_LINE_FAIL : VO_LINE_EMPTY;
+      continue;
+    }
+    o->state = (o->px == o->qx) ? VO_LINE_POINT : VO_LINE_LINE;
+    o->scale = (uint32_t)T[k];
+    o->py = (int64_t)py[k];
+    o->qy = (int64_t)qy[k];
+  }
+  free(hp); free(hq);
+  free(have); free(fail); free(T); free(py); free(qy);
+  free(t.by_base);
+  return 0;
+}

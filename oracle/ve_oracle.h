@@ -192,6 +192,17 @@ int vo_temporal_loads(const vo_config* cfg, const vo_object* objs, uint32_t n_ob
 int vo_approx_topk(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
                    uint64_t n, uint64_t* ndistinct, uint64_t* top_bits, uint64_t* top_count);
 
+/* ---- dyadic-scaled exact linear fit (C21) ----------------
+ * Def 3.7 (structured values) over the EXACT values of the
+ * records (floats as the dyadic rationals they encode; R10): per key,
+ * NaN / inf -> FAIL; T = max fractional bits; every Y = y 2^T must satisfy
+ * |Y| < 2^62 (else FAIL); anchors P = (min x, min Y at that x), Q = (max x,
+ * min Y at that x); all points collinear -> LINE (POINT if one x), else FAIL.
+ * out[n_keys]; EMPTY / FAIL entries are zero apart from state. */
+typedef struct vo_dyadic { uint32_t state, scale; uint64_t px, qx; int64_t py, qy; } vo_dyadic;
+int vo_dyadic_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs, uint64_t n,
+                  vo_dyadic* out);
+
 /* helpers exposed for pinning */
 uint64_t vo_ord(uint64_t b, uint32_t kind, uint32_t w);
 uint32_t vo_float_flags(uint64_t b, uint32_t kind, uint32_t w);   /* bit0 nan, 1 nonint, 2 not_f16, 3 not_bf16, 4 not_f32 */
