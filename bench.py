@@ -367,7 +367,8 @@ def measure_next_rows(ve, ctx, wl, stream, peak, reps=3):
     around each synchronizing call, median of `reps`):
       f1 ve_record_intervals (warp compaction, radix sort, merge scans),
       f2 ve_approx_topk on the ctx's gemm-epoch histogram (re-keyed by truncated value),
-      f3 ve_temporal_loads (ordered load compaction, radix sort by address, neighbour judging)."""
+      f3 ve_temporal_loads (ordered load compaction, radix sort by address, neighbour judging),
+      f2 ve_dyadic_fit (three streaming passes over the records: algorithmic bytes 3 x 24 B per record)."""
     import torch
     e = wl.epochs[1]
     n = e["n"]
@@ -393,6 +394,7 @@ def measure_next_rows(ve, ctx, wl, stream, peak, reps=3):
     ctx.analyze_records(e["recs"], n, stream=sp)
     ms2, (nd, _top) = timed(lambda: ctx.approx_topk(stream=sp))
     ms3, tl = timed(lambda: ctx.temporal_loads(e["recs"], n, stream=sp))
+    ms4, dy = timed(lambda: ctx.dyadic_fit(e["recs"], n, stream=sp))
     gbs = lambda ms: n * REC_BYTES / (ms / 1e3) / 1e9
     return {
         "note": "SURVEY 8(f) rows, not part of the step; each call synchronizes (count read-backs) inside its "
@@ -405,6 +407,9 @@ def measure_next_rows(ve, ctx, wl, stream, peak, reps=3):
                               "frac_of_hbm_peak": gbs(ms3) / peak, "temporal_loads_pc": [int(x) for x in tl[:5, 0]],
                               "closed_form_ok": bool(int(tl[1, 1]) == 363 * 256 * 1152
                                                      and int(tl[2, 1]) == 15 * 1152 * 5776)},
+        "f2_dyadic_fit": {"records": n, "ms": ms4, "records_per_s": n / (ms4 / 1e3),
+                          "alg_gbs": 3 * gbs(ms4), "frac_of_hbm_peak": 3 * gbs(ms4) / peak,
+                          "states": [int(x) for x in np.bincount(dy["state"], minlength=4)]},
     }
 
 

@@ -200,6 +200,24 @@ ve_status ve_temporal_loads(ve_ctx* ctx, const ve_record* d_records, uint64_t n,
  * VE_ERR_STATE after an NCCL rank merge.  Synchronizes s. */
 ve_status ve_approx_topk(ve_ctx* ctx, uint64_t* h_ndistinct, ve_topk_entry* h_top, cudaStream_t s);
 
+/* ---- dyadic-scaled exact linear fit ------------------------
+ * Def 3.7 (structured values) over the EXACT values of the
+ * records (R10): a float encodes the dyadic rational (-1)^s M 2^E,
+ * so structured floats with non-integral values (k/64 ramps, 3 + i 2^-40) are
+ * recognised, which C8's integral-value fit cannot.  Per key of the ctx (PC key,
+ * object key of the first byte from the ctx's object table, SHARED key):
+ * NaN / inf -> FAIL; scale = T = the largest number of fractional bits, every
+ * Y = value * 2^T must satisfy |Y| < 2^62 (else FAIL); P = (min addr, min Y at
+ * that addr), Q = (max addr, min Y at that addr); every point collinear with P
+ * and Q and equal to the anchor at P.x / Q.x -> LINE (POINT if one address),
+ * else FAIL.  Invalid records are skipped.  "Dyadic structured" holds when
+ * state == VE_LINE_LINE and py != qy; the line is y = (py + (x - px)(qy - py)
+ * / (qx - px)) 2^-scale.  h_out[n_keys] (host memory; EMPTY / FAIL entries
+ * zero apart from state).  d_records: device, 8-byte aligned.  Three passes
+ * over the records; independent of the ctx's statistics.  Synchronizes s. */
+typedef struct ve_dyadic { uint32_t state, scale; uint64_t px, qx; int64_t py, qy; } ve_dyadic;
+ve_status ve_dyadic_fit(ve_ctx* ctx, const ve_record* d_records, uint64_t n, ve_dyadic* h_out, cudaStream_t s);
+
 /* ---- accessed intervals and the adaptive copy plan --------
  * PAPER.md section 6.1: "We define an interval [start, end] as
  * the memory range accessed by each GPU instruction" and merge intervals "if

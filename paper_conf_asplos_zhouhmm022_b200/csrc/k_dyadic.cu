@@ -1,0 +1,227 @@
+// k_dyadic.cu -- SURVEY 8(f) f2: dyadic-scaled exact linear fit (ve_dyadic_fit).
+//
+// Def 3.7 (structured values) over the EXACT values of the records
+// (reading R10): a float encodes the dyadic rational (-1)^s M 2^E, so with
+// T = the key's largest number of fractional bits every Y = y 2^T is an integer and the
+// points (addr, Y) are collinear exactly when the points (addr, y) are.  Three streaming
+// passes over the AoS records (24 B each, read once per pass; HBM-bound):
+//   D1  per key: NaN / inf -> fail; T = max fractional bits; min / max address
+//   D2  per key: Y = M 2^(E+T) must fit |Y| < 2^62 (else fail); anchors P = (min x, min Y
+//       at that x), Q = (max x, min Y at that x) -- only records at the extreme x touch them
+//   D3  every record: collinear with P and Q (exact 128-bit cross product) and, at P.x or
+//       Q.x, equal to the anchor; else fail
+// Keys as in K1: the PC key and the object key of the first byte (SHARED pseudo-object for
+// shared-space records); invalid records are skipped.  D1 aggregates keys < DY_SK in shared
+// memory per CTA (flushed at exit), the rest with global atomics.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <vector>
+
+#include "ve_internal.cuh"
+
+namespace ve {
+
+constexpr uint32_t DY_T = 256;
+constexpr uint32_t DY_SK = 512;
+constexpr unsigned long long DY_NONE = ~0ull;
+
+struct DyKey {                  // global per-key state (32 B)
+  unsigned int T, fail;
+  unsigned long long minx, maxx;
+  unsigned long long py, qy;    // Y + 2^63 (order-preserving), DY_NONE = no anchor yet
+};
+
+// exact value of the bits as M 2^E with M odd or zero; false for NaN / inf.  Unsigned values
+// >= 2^63 report M = 2^62 (they fail the |Y| < 2^62 bound for any T).
+__device__ __forceinline__ bool dy_exact(uint64_t b, uint32_t kind, uint32_t lg, long long& M, int& E) {
+  if (kind < 2u) {
+    if (kind == 0u) {
+      M = (b >> 63) ? (1ll << 62) : (long long)b;
+    } else {
+      const uint32_t sh = 64u - (8u << lg);
+      M = (long long)(b << sh) >> sh;
+    }
+    E = 0;
+  } else {
+    int eb, mb;
+    if (kind == 3u) { eb = 8; mb = 7; }
+    else if (lg == 1u) { eb = 5; mb = 10; }
+    else if (lg == 2u) { eb = 8; mb = 23; }
+    else { eb = 11; mb = 52; }
+    const uint64_t ex = (b >> mb) & ((1ull << eb) - 1ull);
+    if (ex == (1ull << eb) - 1ull) return false;
+    const uint64_t man = b & ((1ull << mb) - 1ull);
+    const int bias = (1 << (eb - 1)) - 1;
+    const uint64_t sig = ex ? (man | (1ull << mb)) : man;
+    E = ex ? (int)ex - bias - mb : 1 - bias - mb;
+    M = ((b >> (eb + mb)) & 1ull) ? -(long long)sig : (long long)sig;
+  }
+  if (M == 0) { E = 0; return true; }
+  const int tz = __ffsll(M) - 1;        // strip trailing zero bits: M odd
+  M >>= tz;
+  E += tz;
+  return true;
+}
+
+// Y = M 2^s, s >= 0; false if |Y| >= 2^62
+__device__ __forceinline__ bool dy_scaled(long long M, int s, long long& Y) {
+  if (M == 0) { Y = 0; return true; }
+  const unsigned long long a = M < 0 ? (unsigned long long)(-(M + 1)) + 1ull : (unsigned long long)M;
+  const int bits = 64 - __clzll(a);
+  if (bits + s > 62) return false;
+  Y = M * (1ll << s);
+  return true;
+}
+
+struct DyRec {
+  uint64_t x, v;
+  uint32_t pc, meta;
+  uint32_t nk, k[2];
+};
+
+__device__ __forceinline__ bool dy_load(const ve_record* r, uint64_t i, const DevObjects& o, uint32_t n_pcs,
+                                        DyRec& d) {
+  const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&r[i]);
+  d.x = __ldg(q);
+  d.v = __ldg(q + 1);
+  const unsigned long long pm = __ldg(q + 2);
+  d.pc = (uint32_t)pm;
+  d.meta = (uint32_t)(pm >> 32);
+  if (!rec_valid(d.x, d.v, d.pc, d.meta, n_pcs)) return false;
+  d.nk = 1;
+  d.k[0] = d.pc;
+  if (meta_shared(d.meta)) {
+    d.k[d.nk++] = n_pcs + o.n;
+  } else {
+    uint32_t lo = 0, hi = o.n;          // first object with base > x
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (o.base[mid] <= d.x) lo = mid + 1; else hi = mid;
+    }
+    if (lo > 0 && d.x < o.end[lo - 1]) d.k[d.nk++] = n_pcs + o.id[lo - 1];
+  }
+  return true;
+}
+
+__global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n, DevObjects o, uint32_t n_pcs,
+                                                  uint32_t nk, DyKey* K) {
+  __shared__ unsigned int sT[DY_SK], sF[DY_SK];
+  __shared__ unsigned long long sMin[DY_SK], sMax[DY_SK];
+  const uint32_t ns = nk < DY_SK ? nk : DY_SK;
+  for (uint32_t i = threadIdx.x; i < ns; i += DY_T) { sT[i] = 0; sF[i] = 0; sMin[i] = DY_NONE; sMax[i] = 0; }
+  __syncthreads();
+  for (uint64_t i = (uint64_t)blockIdx.x * DY_T + threadIdx.x; i < n; i += (uint64_t)gridDim.x * DY_T) {
+    DyRec d;
+    if (!dy_load(r, i, o, n_pcs, d)) continue;
+    long long M;
+    int E;
+    const bool fin = dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E);
+    const unsigned int t = (fin && E < 0) ? (unsigned int)(-E) : 0u;
+    for (uint32_t j = 0; j < d.nk; ++j) {
+      const uint32_t k = d.k[j];
+      if (k < ns) {
+        if (!fin) { sF[k] = 1u; continue; }
+        if (t) atomicMax(&sT[k], t);
+        atomicMin(&sMin[k], (unsigned long long)d.x);
+        atomicMax(&sMax[k], (unsigned long long)d.x);
+      } else {
+        if (!fin) { K[k].fail = 1u; continue; }
+        if (t) atomicMax(&K[k].T, t);
+        atomicMin(&K[k].minx, (unsigned long long)d.x);
+        atomicMax(&K[k].maxx, (unsigned long long)d.x);
+      }
+    }
+  }
+  __syncthreads();
+  for (uint32_t k = threadIdx.x; k < ns; k += DY_T) {
+    if (sF[k]) K[k].fail = 1u;
+    if (sMin[k] == DY_NONE) continue;
+    if (sT[k]) atomicMax(&K[k].T, sT[k]);
+    atomicMin(&K[k].minx, sMin[k]);
+    atomicMax(&K[k].maxx, sMax[k]);
+  }
+}
+
+// D2 (anchors and the |Y| bound) when pass == 0, D3 (collinearity) when pass == 1
+__global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t n, DevObjects o, uint32_t n_pcs,
+                                                   DyKey* K, int pass) {
+  for (uint64_t i = (uint64_t)blockIdx.x * DY_T + threadIdx.x; i < n; i += (uint64_t)gridDim.x * DY_T) {
+    DyRec d;
+    if (!dy_load(r, i, o, n_pcs, d)) continue;
+    long long M;
+    int E;
+    if (!dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E)) continue;   // its keys failed in D1
+    for (uint32_t j = 0; j < d.nk; ++j) {
+      DyKey& k = K[d.k[j]];
+      if (*(volatile unsigned int*)&k.fail) continue;
+      long long Y;
+      if (!dy_scaled(M, E + (int)k.T, Y)) { k.fail = 1u; continue; }
+      const unsigned long long yo = (unsigned long long)Y ^ (1ull << 63);
+      if (pass == 0) {
+        if (d.x == k.minx) atomicMin(&k.py, yo);
+        if (d.x == k.maxx) atomicMin(&k.qy, yo);
+        continue;
+      }
+      const long long py = (long long)(k.py ^ (1ull << 63)), qy = (long long)(k.qy ^ (1ull << 63));
+      const __int128 dx = (__int128)(long long)(d.x - k.minx), qx = (__int128)(long long)(k.maxx - k.minx);
+      bool ok = (__int128)(Y - py) * qx == (__int128)(qy - py) * dx;   // |Y - py| < 2^63, |dx| < 2^48
+      ok = ok && !(d.x == k.minx && Y != py) && !(d.x == k.maxx && Y != qy);
+      if (!ok) k.fail = 1u;
+    }
+  }
+}
+
+__global__ void k_dy_init(DyKey* K, uint32_t nk) {
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < nk; k += gridDim.x * blockDim.x) {
+    K[k].T = 0; K[k].fail = 0;
+    K[k].minx = DY_NONE; K[k].maxx = 0;
+    K[k].py = DY_NONE; K[k].qy = DY_NONE;
+  }
+}
+
+}  // namespace ve
+
+using namespace ve;
+
+extern "C" ve_status ve_dyadic_fit(ve_ctx* c, const ve_record* d_records, uint64_t n, ve_dyadic* h_out,
+                                   cudaStream_t s) {
+  if (!c || !h_out) return VE_ERR_INVALID;
+  const uint32_t nk = c->n_keys;
+  if (n && (!d_records || ((uintptr_t)d_records & 7))) return fail(c, VE_ERR_INVALID, "ve_dyadic_fit: null or misaligned");
+  cudaSetDevice(c->device);
+  DyKey* K = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&K, sizeof(DyKey) * (size_t)nk, s);
+  if (e != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "ve_dyadic_fit: workspace"); }
+  count_launch();
+  k_dy_init<<<(nk + 255) / 256, 256, 0, s>>>(K, nk);
+  if (n) {
+    uint64_t b = (n + DY_T - 1) / DY_T;
+    const uint64_t cap = (uint64_t)c->num_sms * 8;
+    const unsigned grid = (unsigned)(b < cap ? b : cap);
+    count_launch();
+    k_dy_scan<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, nk, K);
+    count_launch();
+    k_dy_check<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, K, 0);
+    count_launch();
+    k_dy_check<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, K, 1);
+  }
+  std::vector<DyKey> hk(nk);
+  e = cudaMemcpyAsync(hk.data(), K, sizeof(DyKey) * (size_t)nk, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaFreeAsync(K, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_dyadic_fit");
+  for (uint32_t k = 0; k < nk; ++k) {
+    ve_dyadic& o = h_out[k];
+    o = ve_dyadic{};
+    if (hk[k].fail) { o.state = VE_LINE_FAIL; continue; }
+    if (hk[k].minx == DY_NONE) { o.state = VE_LINE_EMPTY; continue; }
+    o.state = hk[k].minx == hk[k].maxx ? VE_LINE_POINT : VE_LINE_LINE;
+    o.scale = hk[k].T;
+    o.px = hk[k].minx;
+    o.qx = hk[k].maxx;
+    o.py = (int64_t)(hk[k].py ^ (1ull << 63));
+    o.qy = (int64_t)(hk[k].qy ^ (1ull << 63));
+  }
+  return VE_OK;
+}

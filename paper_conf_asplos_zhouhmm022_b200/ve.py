@@ -51,6 +51,10 @@ DIFF_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_masked", "n_unchanged"
                       + [("redundant", "<u4"), ("pad", "<u4")])
 
 
+DYADIC_DTYPE = np.dtype([("state", "<u4"), ("scale", "<u4"), ("px", "<u8"), ("qx", "<u8"), ("py", "<i8"),
+                         ("qy", "<i8")])
+
+
 class VeError(RuntimeError):
     def __init__(self, status, msg):
         super().__init__(f"{STATUS_NAMES[status] if 0 <= status < 7 else status}: {msg}")
@@ -106,6 +110,7 @@ def lib():
             "ve_interval_merge": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_approx_topk": ([vp, vp, vp, vp], st),
             "ve_temporal_loads": ([vp, vp, u64, vp, vp], st),
+            "ve_dyadic_fit": ([vp, vp, u64, vp, vp], st),
             "ve_vfg_build": ([vp, u64, ctypes.POINTER(vp)], st),
             "ve_vfg_slice": ([vp, u32, ctypes.POINTER(vp)], st),
             "ve_vfg_important": ([vp, u64, u64, ctypes.POINTER(vp)], st),
@@ -363,6 +368,14 @@ class Context:
         self._check(lib().ve_approx_topk(self._h, nd.ctypes.data, top.ctypes.data, _stream(stream)),
                     "ve_approx_topk")
         return nd, top.reshape(nk, self.topk)
+
+    def dyadic_fit(self, d_records, n, stream=None):
+        """ve_dyadic_fit: DYADIC_DTYPE[n_keys] -- exact linear fit over the records' exact values (f2)."""
+        nk = self.n_pcs + getattr(self, "n_objects", 0) + 1
+        out = np.zeros(nk, dtype=DYADIC_DTYPE)
+        self._check(lib().ve_dyadic_fit(self._h, _ptr(d_records), n, out.ctypes.data, _stream(stream)),
+                    "ve_dyadic_fit")
+        return out
 
     def temporal_loads(self, d_records, n, stream=None):
         """ve_temporal_loads: uint64[n_keys, 2] = (temporal, temporally redundant) loads per key."""
