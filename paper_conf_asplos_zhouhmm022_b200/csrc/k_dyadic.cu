@@ -111,15 +111,54 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
   const uint32_t ns = nk < DY_SK ? nk : DY_SK;
   for (uint32_t i = threadIdx.x; i < ns; i += DY_T) { sT[i] = 0; sF[i] = 0; sMin[i] = DY_NONE; sMax[i] = 0; }
   __syncthreads();
-  for (uint64_t i = (uint64_t)blockIdx.x * DY_T + threadIdx.x; i < n; i += (uint64_t)gridDim.x * DY_T) {
+  // block-uniform trip count: every lane takes part in the warp aggregation below
+  for (uint64_t b = (uint64_t)blockIdx.x * DY_T; b < n; b += (uint64_t)gridDim.x * DY_T) {
+    const uint64_t i = b + threadIdx.x;
     DyRec d;
-    if (!dy_load(r, i, o, n_pcs, d)) continue;
-    long long M;
-    int E;
-    const bool fin = dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E);
-    const unsigned int t = (fin && E < 0) ? (unsigned int)(-E) : 0u;
-    for (uint32_t j = 0; j < d.nk; ++j) {
-      const uint32_t k = d.k[j];
+    d.nk = 0;
+    const bool act = i < n && dy_load(r, i, o, n_pcs, d);
+    long long M = 0;
+    int E = 0;
+    const bool fin = act && dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E);
+    unsigned int t = (fin && E < 0) ? (unsigned int)(-E) : 0u;
+    for (uint32_t j = 0; j < 2; ++j) {
+      const uint32_t k = j < d.nk ? d.k[j] : 0xFFFFFFFFu;
+      const unsigned g = __match_any_sync(0xFFFFFFFFu, k);
+      if (g == 0xFFFFFFFFu) {
+        // the whole warp on one key (the common case: a warp-wide access of one PC / object):
+        // one update per warp instead of 32 contended shared-memory atomics
+        if (k == 0xFFFFFFFFu) continue;
+        unsigned long long mn = fin ? d.x : DY_NONE, mx = fin ? d.x : 0ull;
+        unsigned int tt = t, ff = (!fin) ? 1u : 0u, hv = fin ? 1u : 0u;
+        for (int off = 16; off > 0; off >>= 1) {
+          const unsigned long long a = __shfl_xor_sync(0xFFFFFFFFu, mn, off);
+          const unsigned long long c = __shfl_xor_sync(0xFFFFFFFFu, mx, off);
+          mn = a < mn ? a : mn;
+          mx = c > mx ? c : mx;
+        }
+        tt = __reduce_max_sync(0xFFFFFFFFu, tt);
+        ff = __reduce_or_sync(0xFFFFFFFFu, ff);
+        hv = __reduce_or_sync(0xFFFFFFFFu, hv);
+        if ((threadIdx.x & 31u) == 0u) {
+          if (k < ns) {
+            if (ff) sF[k] = 1u;
+            if (hv) {
+              if (tt) atomicMax(&sT[k], tt);
+              atomicMin(&sMin[k], mn);
+              atomicMax(&sMax[k], mx);
+            }
+          } else {
+            if (ff) K[k].fail = 1u;
+            if (hv) {
+              if (tt) atomicMax(&K[k].T, tt);
+              atomicMin(&K[k].minx, mn);
+              atomicMax(&K[k].maxx, mx);
+            }
+          }
+        }
+        continue;
+      }
+      if (k == 0xFFFFFFFFu) continue;
       if (k < ns) {
         if (!fin) { sF[k] = 1u; continue; }
         if (t) atomicMax(&sT[k], t);
@@ -154,7 +193,7 @@ __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t 
     if (!dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E)) continue;   // its keys failed in D1
     for (uint32_t j = 0; j < d.nk; ++j) {
       DyKey& k = K[d.k[j]];
-      if (*(volatile unsigned int*)&k.fail) continue;
+      if (k.fail) continue;                  // a stale 0 only costs the check below
       long long Y;
       if (!dy_scaled(M, E + (int)k.T, Y)) { k.fail = 1u; continue; }
       const unsigned long long yo = (unsigned long long)Y ^ (1ull << 63);
