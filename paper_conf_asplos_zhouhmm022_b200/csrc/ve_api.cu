@@ -292,6 +292,7 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     for (int j = 0; j < DENSE_PER_OBJ; ++j) c->dense_pc_init[DENSE_PER_OBJ * i + j] = DENSE_FREE;
     want += DENSE_PER_OBJ * v[i].n_elems;
   }
+  c->pre_elems = want / DENSE_PER_OBJ;
   if (want > DENSE_BUDGET) want = DENSE_BUDGET;
   if (want > c->dense_cap) {
     if (c->dense_pool) {

@@ -125,6 +125,7 @@ struct ve_ctx {
   bool dense_dirty = false;                  // pool may hold counts not yet flushed
   std::vector<uint32_t> dense_pc_init;       // [DENSE_PER_OBJ*n_obj]: DENSE_FREE or DENSE_OFF
   uint64_t records_analyzed = 0;
+  uint64_t pre_elems = 0;                    // elements of the objects with a pre snapshot
   // finalize scratch
   void* scratch = nullptr;
   void* pin = nullptr;                       // pinned host staging of small report-time copies

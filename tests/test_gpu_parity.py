@@ -191,6 +191,29 @@ def test_dense_pool_exhausted_parity(torch_cuda, budget):
             os.environ["VE_DENSE_BUDGET"] = old
 
 
+@pytest.mark.parametrize("always", ["1", None])
+def test_dense_gate_parity(torch_cuda, always):
+    """The dense counters are used only by calls with >= 1 record per pre-snapshot element
+    (VE_DENSE_ALWAYS=1 forces them): a chunked trace then mixes dense-counted and hash-counted
+    calls for the same keys.  Results must not depend on which path counted what."""
+    import os
+    old = os.environ.get("VE_DENSE_ALWAYS")
+    if always:
+        os.environ["VE_DENSE_ALWAYS"] = always
+    try:
+        hobjs = W.host_objects(G.FUZZ, 0, 13)
+        recs = G.records_host(G.FUZZ, 0, 13, 0, 150000)
+        _check(torch_cuda, 64, hobjs, recs, chunks=[7, 40000, 41000, 100000])
+        hobjs = W.host_objects(G.CFG1, 0, 1)
+        recs = G.records_host(G.CFG1, 0, 1, 0, 1 << 20)
+        _check(torch_cuda, 16, hobjs, recs, chunks=[5000, 1 << 19, (1 << 19) + 3])
+    finally:
+        if old is None:
+            os.environ.pop("VE_DENSE_ALWAYS", None)
+        else:
+            os.environ["VE_DENSE_ALWAYS"] = old
+
+
 def test_diff_before_report(torch_cuda):
     """ve_snapshot_diff before ve_report (the bench order): n_untouched must already count the
     elements of loads that are counted densely (their L bits are set when the counts are flushed)."""
