@@ -52,6 +52,7 @@ struct AnalyzeParams {
   uint32_t dense_ok;        // dense per-element counting enabled for this launch
   uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
   uint64_t nring;           // full windows (streamed through the per-warp rings)
+  uint32_t chunk;           // windows per static chunk (VE_CLAIM 2): CHUNK, or one stage for short traces
   unsigned long long* work; // chunk claim counter (zeroed before the launch)
   // S8 insert staging: a private region of stage_rs 16-byte entries per warp for the
   // (tag, bits, count) groups the shared table cannot take; k_hist_drain inserts them
@@ -768,8 +769,8 @@ __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
 #if VE_CLAIM == 2
   // static interleave: chunk c goes to warp c mod (all warps); no atomics, and every
   // warp sees the same mix of the trace
-  w0 = R.nextc * CHUNK;
-  len = CHUNK;
+  w0 = R.nextc * P.chunk;
+  len = P.chunk;
   R.nextc += (uint64_t)gridDim.x * K1_WARPS;
 #else
   unsigned long long c = 0;
@@ -1636,7 +1637,9 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
     fence_mbar_init();
   }
   __syncwarp();
-  R.nextc = gw;
+  // short traces (one-stage chunks): chunk c goes to CTA c mod grid first, so the few chunks
+  // spread over all SMs instead of filling the first CTAs' warps
+  R.nextc = P.chunk == CHUNK ? gw : (uint64_t)warp * gridDim.x + blockIdx.x;
 #if VE_CLAIM
   ring_claim(P, R);
 #else
@@ -1929,6 +1932,9 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   uint64_t windows = (n + 31) / 32;
   uint64_t blocks = (windows + K1_WARPS - 1) / K1_WARPS;
   if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+  // a trace too short to give every warp a few CHUNK-window chunks (cfg5's kernels: a warp's
+  // serial share of a 16-window chunk set a ~0.3 ms floor) is split into one-stage chunks
+  P.chunk = P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? CHUNK : (uint32_t)STAGE_WIN;
   // staging regions: a warp stages at most one group per record of its static range
   {
     const uint64_t tw = blocks * K1_WARPS;
