@@ -166,6 +166,22 @@ def rank_chunk(n, rank, world):
     return n * rank // world, n * (rank + 1) // world
 
 
+def lpt_assign(costs, world):
+    """Rank of each unit under longest-processing-time-first (cfg5's independent
+    kernels by record count): units in decreasing cost (ties by index) go to the least-loaded rank
+    (ties by rank).  Deterministic, so every rank computes the same plan without communication;
+    max load <= (4/3 - 1/(3 world)) x the optimum (Graham's bound)."""
+    import heapq
+    order = sorted(range(len(costs)), key=lambda i: (-int(costs[i]), i))
+    heap = [(0, r) for r in range(world)]
+    owner = [0] * len(costs)
+    for i in order:
+        load, r = heapq.heappop(heap)
+        owner[i] = r
+        heapq.heappush(heap, (load + int(costs[i]), r))
+    return owner
+
+
 class ValueFlowGraph:
     """ve_vfg_* (Defs 5.1-5.3): built from an ACCESS_DTYPE log in program order (host-side, no device)."""
 

@@ -41,7 +41,17 @@ def _worker(rank, world, port, q):
         dist.all_gather(ids, uid)
         # 3. the max-over-ranks timing reduction of bench.py
         ms = bench.max_over_ranks(10.0 + rank, device="cpu")
-        q.put((rank, [c.tolist() for c in allc], [bytes(i.tolist()) for i in ids], ms))
+        # 4. cfg5's kernel plan (LPT on record count), computed independently on every rank
+        from gen import vegen as G
+        cfg = G.scaled(G.CFG5, 0)
+        costs = [G.info(cfg, k)["n_records"] for k in range(4000)]
+        owner = ve.lpt_assign(costs, world)
+        mine = [k for k in range(4000) if owner[k] == rank]
+        t = torch.tensor([len(mine), sum(costs[k] for k in mine), sum(mine), hash(tuple(owner)) & 0x7FFFFFFF],
+                         dtype=torch.int64)
+        plans = [torch.zeros(4, dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(plans, t)
+        q.put((rank, [c.tolist() for c in allc], [bytes(i.tolist()) for i in ids], ms, [p.tolist() for p in plans]))
     finally:
         dist.destroy_process_group()
 
@@ -59,8 +69,32 @@ def test_gloo_two_ranks():
         p.join(timeout=60)
         assert p.exitcode == 0
     n = 231555071
-    for rank, chunks, ids, ms in res:
+    for rank, chunks, ids, ms, plans in res:
+        # the kernel plan: the same on both ranks, covering every kernel once, balanced
+        assert len({p[3] for p in plans}) == 1
+        assert sum(p[0] for p in plans) == 4000 and sum(p[2] for p in plans) == 4000 * 3999 // 2
+        assert sum(p[1] for p in plans) == 1_000_000_000
+        loads = [p[1] for p in plans]
+        assert max(loads) <= (4 / 3 - 1 / (3 * world)) * max(1_000_000_000 / world, 1_676_166)
         assert chunks[0][0] == 0 and chunks[-1][1] == n
         assert all(chunks[i][1] == chunks[i + 1][0] for i in range(world - 1))
         assert len(set(ids)) == 1 and ids[0] == bytes((i ^ 0x5A) for i in range(128))
         assert ms == 11.0
+
+
+def test_lpt_assign_bound():
+    """LPT against the brute-force optimum on small random instances: every unit assigned,
+    max load within Graham's (4/3 - 1/(3m)) bound, deterministic."""
+    import itertools
+    import random
+    from paper_conf_asplos_zhouhmm022_b200 import ve
+    rng = random.Random(5)
+    for _ in range(40):
+        m = rng.choice([2, 3])
+        costs = [rng.randint(1, 50) for _ in range(rng.randint(1, 8))]
+        owner = ve.lpt_assign(costs, m)
+        assert owner == ve.lpt_assign(list(costs), m) and all(0 <= r < m for r in owner)
+        loads = [sum(c for c, r in zip(costs, owner) if r == q) for q in range(m)]
+        opt = min(max(sum(c for c, r in zip(costs, a) if r == q) for q in range(m))
+                  for a in itertools.product(range(m), repeat=len(costs)))
+        assert max(loads) <= (4 / 3 - 1 / (3 * m)) * opt + 1e-9
