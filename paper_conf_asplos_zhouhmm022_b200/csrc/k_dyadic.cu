@@ -80,8 +80,14 @@ struct DyRec {
   uint32_t nk, k[2];
 };
 
+// the thread's last object [cb, ce) -> key: records of a warp window mostly stay in one object
+struct DyObjCache {
+  uint64_t cb = 1, ce = 0;
+  uint32_t key = 0;
+};
+
 __device__ __forceinline__ bool dy_load(const ve_record* r, uint64_t i, const DevObjects& o, uint32_t n_pcs,
-                                        DyRec& d) {
+                                        DyRec& d, DyObjCache& oc) {
   const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&r[i]);
   d.x = __ldg(q);
   d.v = __ldg(q + 1);
@@ -93,13 +99,20 @@ __device__ __forceinline__ bool dy_load(const ve_record* r, uint64_t i, const De
   d.k[0] = d.pc;
   if (meta_shared(d.meta)) {
     d.k[d.nk++] = n_pcs + o.n;
+  } else if (d.x >= oc.cb && d.x < oc.ce) {
+    d.k[d.nk++] = oc.key;
   } else {
     uint32_t lo = 0, hi = o.n;          // first object with base > x
     while (lo < hi) {
       const uint32_t mid = (lo + hi) >> 1;
       if (o.base[mid] <= d.x) lo = mid + 1; else hi = mid;
     }
-    if (lo > 0 && d.x < o.end[lo - 1]) d.k[d.nk++] = n_pcs + o.id[lo - 1];
+    if (lo > 0 && d.x < o.end[lo - 1]) {
+      oc.cb = o.base[lo - 1];
+      oc.ce = o.end[lo - 1];
+      oc.key = n_pcs + o.id[lo - 1];
+      d.k[d.nk++] = oc.key;
+    }
   }
   return true;
 }
@@ -111,12 +124,13 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
   const uint32_t ns = nk < DY_SK ? nk : DY_SK;
   for (uint32_t i = threadIdx.x; i < ns; i += DY_T) { sT[i] = 0; sF[i] = 0; sMin[i] = DY_NONE; sMax[i] = 0; }
   __syncthreads();
+  DyObjCache oc;
   // block-uniform trip count: every lane takes part in the warp aggregation below
   for (uint64_t b = (uint64_t)blockIdx.x * DY_T; b < n; b += (uint64_t)gridDim.x * DY_T) {
     const uint64_t i = b + threadIdx.x;
     DyRec d;
     d.nk = 0;
-    const bool act = i < n && dy_load(r, i, o, n_pcs, d);
+    const bool act = i < n && dy_load(r, i, o, n_pcs, d, oc);
     long long M = 0;
     int E = 0;
     const bool fin = act && dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E);
@@ -130,11 +144,13 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
         if (k == 0xFFFFFFFFu) continue;
         unsigned long long mn = fin ? d.x : DY_NONE, mx = fin ? d.x : 0ull;
         unsigned int tt = t, ff = (!fin) ? 1u : 0u, hv = fin ? 1u : 0u;
-        for (int off = 16; off > 0; off >>= 1) {
-          const unsigned long long a = __shfl_xor_sync(0xFFFFFFFFu, mn, off);
-          const unsigned long long c = __shfl_xor_sync(0xFFFFFFFFu, mx, off);
-          mn = a < mn ? a : mn;
-          mx = c > mx ? c : mx;
+        {                                  // 64-bit min / max from 32-bit warp reductions
+          const unsigned mh = __reduce_min_sync(0xFFFFFFFFu, (unsigned)(mn >> 32));
+          const unsigned ml = __reduce_min_sync(0xFFFFFFFFu, (unsigned)(mn >> 32) == mh ? (unsigned)mn : ~0u);
+          const unsigned xh = __reduce_max_sync(0xFFFFFFFFu, (unsigned)(mx >> 32));
+          const unsigned xl = __reduce_max_sync(0xFFFFFFFFu, (unsigned)(mx >> 32) == xh ? (unsigned)mx : 0u);
+          mn = ((unsigned long long)mh << 32) | ml;
+          mx = ((unsigned long long)xh << 32) | xl;
         }
         tt = __reduce_max_sync(0xFFFFFFFFu, tt);
         ff = __reduce_or_sync(0xFFFFFFFFu, ff);
@@ -185,9 +201,10 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
 // D2 (anchors and the |Y| bound) when pass == 0, D3 (collinearity) when pass == 1
 __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t n, DevObjects o, uint32_t n_pcs,
                                                    DyKey* K, int pass) {
+  DyObjCache oc;
   for (uint64_t i = (uint64_t)blockIdx.x * DY_T + threadIdx.x; i < n; i += (uint64_t)gridDim.x * DY_T) {
     DyRec d;
-    if (!dy_load(r, i, o, n_pcs, d)) continue;
+    if (!dy_load(r, i, o, n_pcs, d, oc)) continue;
     long long M;
     int E;
     if (!dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E)) continue;   // its keys failed in D1
