@@ -6,8 +6,9 @@
 // points (addr, Y) are collinear exactly when the points (addr, y) are.  Three streaming
 // passes over the AoS records (24 B each, read once per pass; HBM-bound):
 //   D1  per key: NaN / inf -> fail; T = max fractional bits; min / max address
-//   D2  per key: Y = M 2^(E+T) must fit |Y| < 2^62 (else fail); anchors P = (min x, min Y
-//       at that x), Q = (max x, min Y at that x) -- only records at the extreme x touch them
+//   D2  anchors P = (min x, min Y at that x), Q = (max x, min Y at that x), Y = M 2^(E+T);
+//       only records at a key's extreme x decode their value
+//   (every record's |Y| < 2^62 bound is checked in D3, which computes Y anyway)
 //   D3  every record: collinear with P and Q (exact 128-bit cross product) and, at P.x or
 //       Q.x, equal to the anchor; else fail
 // Keys as in K1: the PC key and the object key of the first byte (SHARED pseudo-object for
@@ -205,6 +206,14 @@ __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t 
   for (uint64_t i = (uint64_t)blockIdx.x * DY_T + threadIdx.x; i < n; i += (uint64_t)gridDim.x * DY_T) {
     DyRec d;
     if (!dy_load(r, i, o, n_pcs, d, oc)) continue;
+    if (pass == 0) {                       // D2 needs only the records at a key's extreme address
+      bool any = false;
+      for (uint32_t j = 0; j < d.nk; ++j) {
+        const DyKey& k = K[d.k[j]];
+        any |= d.x == k.minx || d.x == k.maxx;
+      }
+      if (!any) continue;
+    }
     long long M;
     int E;
     if (!dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E)) continue;   // its keys failed in D1
