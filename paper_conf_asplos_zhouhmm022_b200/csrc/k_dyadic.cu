@@ -213,6 +213,10 @@ __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t 
         any |= d.x == k.minx || d.x == k.maxx;
       }
       if (!any) continue;
+    } else {                               // D3: nothing left to check once every key of the record failed
+      bool any = false;
+      for (uint32_t j = 0; j < d.nk; ++j) any |= K[d.k[j]].fail == 0u;
+      if (!any) continue;
     }
     long long M;
     int E;
