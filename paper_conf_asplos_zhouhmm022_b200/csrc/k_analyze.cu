@@ -1916,7 +1916,9 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   cudaFuncAttributes fa;
   // many PCs interleave their warp instructions window by window (stencils, op mixes):
   // the multi-key dense kernel; few PCs (long runs per key): the single-key kernel
-  const bool multi = VE_MULTI_DENSE && c->cfg.n_pcs >= VE_MULTI_MIN_PCS;
+  // (VE_K1_MULTI=0/1 forces one instantiation: the parity tests run both on the same traces)
+  const char* fm = getenv("VE_K1_MULTI");
+  const bool multi = VE_MULTI_DENSE && (fm && *fm ? *fm == '1' : c->cfg.n_pcs >= VE_MULTI_MIN_PCS);
   auto kfn = multi ? k_analyze<true> : k_analyze<false>;
   cudaFuncGetAttributes(&fa, kfn);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring

@@ -78,7 +78,12 @@ struct CmpJob {
 // K8: bytewise verification of (member, representative) pairs, 256 KiB per CTA
 __global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned int* differs) {
   const CmpJob jb = jobs[blockIdx.x];
-  if (*(volatile unsigned int*)&differs[jb.pair]) return;
+  // early exit when another chunk of the pair already differs: decided once per block (thread 0
+  // reads the flag) so every thread takes the same branch before __syncthreads_or below
+  __shared__ unsigned int s_skip;
+  if (threadIdx.x == 0) s_skip = *(volatile unsigned int*)&differs[jb.pair];
+  __syncthreads();
+  if (s_skip) return;
   bool diff = false;
   const uint8_t* a = jb.a + jb.off;
   const uint8_t* b = jb.b + jb.off;

@@ -368,9 +368,13 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
 ve_status ve_reset(ve_ctx* c) {
   if (!ctx_ok(c)) return VE_ERR_INVALID;
   cudaSetDevice(c->device);
+  // work still queued on other (non-blocking) streams may write the tables: let it finish
+  // before the reset memsets, which run on the legacy stream
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_reset (pending work)");
   ve_status st = launch_reset(c, 0);
   if (st != VE_OK) return st;
-  cudaError_t e = cudaDeviceSynchronize();
+  e = cudaDeviceSynchronize();
   return e == cudaSuccess ? VE_OK : cuda_fail(c, e, "ve_reset");
 }
 
@@ -379,8 +383,9 @@ ve_status ve_analyze_records(ve_ctx* c, const ve_record* d, uint64_t n, cudaStre
   if (c->poisoned || c->hist_merged) return fail(c, VE_ERR_STATE, "ve_analyze_records: ctx poisoned or merged; ve_reset first");
   if (n == 0) return VE_OK;
   if (!d || ((uintptr_t)d & 7)) return fail(c, VE_ERR_INVALID, "ve_analyze_records: d_records null or not 8-byte aligned");
-  // per-CTA shared counters are 32-bit: keep each launch well below 2^32 records per CTA
-  const uint64_t CH = 1ull << 36;
+  // per-CTA shared counters are 32-bit: keep each launch below 2^31 records per CTA (the
+  // grid is one CTA per SM, so the cap scales with the SM count: MIG slices have few SMs)
+  const uint64_t CH = (uint64_t)(c->num_sms > 0 ? c->num_sms : 1) << 31;
   for (uint64_t off = 0; off < n; off += CH) {
     ve_status st = launch_analyze(c, d + off, std::min(CH, n - off), s);
     if (st != VE_OK) return st;
@@ -394,13 +399,22 @@ ve_status ve_analyze_records_host(ve_ctx* c, const ve_record* h, uint64_t n, cud
   if (n == 0) return VE_OK;
   if (!h) return fail(c, VE_ERR_INVALID, "ve_analyze_records_host: null records");
   const uint64_t CH = 1ull << 21;  // 2 Mi records = 48 MiB per staging buffer
-  if (!c->stage[0]) {
-    for (int i = 0; i < 2; ++i) {
-      if (cudaMalloc(&c->stage[i], CH * sizeof(ve_record)) != cudaSuccess ||
-          cudaEventCreateWithFlags(&c->stage_ev[i], cudaEventDisableTiming) != cudaSuccess) {
-        cudaGetLastError();
-        return fail(c, VE_ERR_NOMEM, "staging buffers");
+  if (!c->stage[0] || !c->stage[1] || !c->stage_ev[0] || !c->stage_ev[1]) {
+    // all or nothing: a partial allocation is released, so a later call retries from scratch
+    bool ok = true;
+    for (int i = 0; i < 2 && ok; ++i) {
+      ok = cudaMalloc(&c->stage[i], CH * sizeof(ve_record)) == cudaSuccess &&
+           cudaEventCreateWithFlags(&c->stage_ev[i], cudaEventDisableTiming) == cudaSuccess;
+    }
+    if (!ok) {
+      cudaGetLastError();
+      for (int i = 0; i < 2; ++i) {
+        if (c->stage[i]) cudaFree(c->stage[i]);
+        if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);
+        c->stage[i] = nullptr;
+        c->stage_ev[i] = nullptr;
       }
+      return fail(c, VE_ERR_NOMEM, "staging buffers");
     }
     c->stage_bytes = CH * sizeof(ve_record);
   }
@@ -413,9 +427,15 @@ ve_status ve_analyze_records_host(ve_ctx* c, const ve_record* h, uint64_t n, cud
     }
   }
   // chunk i: the copy stream fills stage[i%2] once that buffer's previous analysis is done,
-  // and stream s analyses it once the copy is done -- copy i+1 overlaps analysis i
-  cudaEventRecord(c->stage_ev[0], s);   // nothing of this call may overtake earlier work on s
-  cudaEventRecord(c->stage_ev[1], s);
+  // and stream s analyses it once the copy is done -- copy i+1 overlaps analysis i.
+  // stage_ev[b] always marks the last analysis that read stage[b], on whatever stream an
+  // earlier call used: the copy stream waits on it before overwriting (cross-call and
+  // cross-stream safe); the first copy of this call also waits for earlier work on s.
+  cudaError_t e0 = cudaStreamWaitEvent(c->copy_stream, c->stage_ev[0], 0);
+  if (e0 == cudaSuccess) e0 = cudaStreamWaitEvent(c->copy_stream, c->stage_ev[1], 0);
+  if (e0 == cudaSuccess) e0 = cudaEventRecord(c->copied_ev[0], s);
+  if (e0 == cudaSuccess) e0 = cudaStreamWaitEvent(c->copy_stream, c->copied_ev[0], 0);
+  if (e0 != cudaSuccess) return cuda_fail(c, e0, "ve_analyze_records_host order");
   for (uint64_t off = 0, i = 0; off < n; off += CH, ++i) {
     const int b = (int)(i & 1);
     const uint64_t m = std::min(CH, n - off);
