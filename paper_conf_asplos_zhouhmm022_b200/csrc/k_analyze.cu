@@ -611,7 +611,7 @@ __device__ __noinline__ int slot_acquire(const AnalyzeParams& P, WarpCache& wc, 
   const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
   const uint32_t meta = (uint32_t)(key >> 32);
   const uint32_t lf = slot_lfail(P, pc, koi);
-  const unsigned long long dn = (P.dense_ok && !meta_store(meta)) ? dense_lookup(P, oi, (meta << 16) | pc) : 0ull;
+  const unsigned long long dn = (P.dense_ok && !meta_store(meta) && !nosnap) ? dense_lookup(P, oi, (meta << 16) | pc) : 0ull;
   __syncwarp();
   if ((threadIdx.x & 31) == 0) {
     SlotE& e = slots[v];
@@ -758,6 +758,7 @@ struct Ring {
   uint32_t d, sw, ph;     // stage and window within it of the next read, phase parity of the current pass
   uint32_t pend;          // stage + 1 to refill at the next read, 0 = none
   uint64_t nextc;         // VE_CLAIM == 2: the warp's next static chunk (gw, gw + warps, ...)
+  uint32_t cstride;       // warps of the grid (the static interleave's stride)
 };
 
 // claim the next chunk of full windows (all lanes; lane 0 does the atomic).  Guided:
@@ -771,7 +772,7 @@ __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
   // warp sees the same mix of the trace
   w0 = R.nextc * P.chunk;
   len = P.chunk;
-  R.nextc += (uint64_t)gridDim.x * K1_WARPS;
+  R.nextc += R.cstride;
 #else
   unsigned long long c = 0;
   if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
@@ -867,6 +868,7 @@ __device__ __noinline__ uint32_t slow_window(const AnalyzeParams& P, WarpCache& 
                                              uint64_t val, uint64_t pm, bool inrange) {
   const Smem S = smem_of(P);
   const int lane = threadIdx.x & 31;
+  __syncwarp();
   const uint32_t pc = (uint32_t)pm, meta = (uint32_t)(pm >> 32);
   // S1 decode + validate
   const bool valid = inrange && rec_valid(addr, val, pc, meta, P.n_pcs);
@@ -968,6 +970,7 @@ __device__ __noinline__ uint32_t slow_window(const AnalyzeParams& P, WarpCache& 
     const unsigned vg = __match_any_sync(tg, val);
     if (lane == __ffs(vg) - 1) hist_insert(P, tag, val, __popc(vg));
   }
+  __syncwarp();
   return inv | (unm << 16);
 }
 
@@ -1640,6 +1643,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   // short traces (one-stage chunks): chunk c goes to CTA c mod grid first, so the few chunks
   // spread over all SMs instead of filling the first CTAs' warps
   R.nextc = P.chunk == CHUNK ? gw : (uint64_t)warp * gridDim.x + blockIdx.x;
+  R.cstride = gridDim.x * K1_WARPS;
 #if VE_CLAIM
   ring_claim(P, R);
 #else
@@ -1840,6 +1844,558 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
 }
 
 
+// ============================================================================
+// K1 v2: register-resident key slots for traces whose PCs and objects alternate
+// window by window (stencil neighbours, op mixes, multi-PC kernels).
+//
+// Slot s of a warp lives in lane s's registers (32 slots per warp), so a window
+// switches key at the cost of one ballot: the warp reduces the window's value
+// statistics with REDUX (counts packed 6 bits apart, 32-bit min / max) and lane s
+// folds them into its accumulators with predicated instructions.  A slot is folded
+// into the PC-key and object-key rows (shared memory, or the global table) only on
+// eviction and at exit, by its own lane.  Objects (<= 32) are cached one per lane:
+// an address is mapped by one ballot, the metadata moves by shuffles.  Everything
+// else (slow windows, S8 inserts, line states, dense counters) is shared with v1.
+// ============================================================================
+constexpr int NS2 = 32;
+struct SlotLine {            // deferred C8 constant segment of slot s (see SlotE::cy)
+  uint64_t cy, cx0, cx1;
+  uint32_t cpend, pad;
+};
+struct LaneSlot {            // the registers of lane s that hold slot s
+  uint64_t key;              // meta << 32 | object id << 16 | pc; ~0 = free
+  unsigned long long dn;     // dense counter array of (pc, object) loads that read the pre value, or 0
+  unsigned long long dq;     // dense counter array of records that carry the post value (DENSE_POST), or 0
+  uint32_t info;             // bits 0-1: line FAIL (PC key, object key); bit 2: object has no pre snapshot
+  uint32_t n, zero, eq, nan, nonint, nf16, nbf16, nf32;
+  uint64_t mm[6];            // raw min, raw max, ord min, ord max, trunc min, trunc max (64-bit keys)
+};
+
+__device__ __forceinline__ void lslot_clear_acc(LaneSlot& L) {
+  L.n = L.zero = L.eq = L.nan = L.nonint = L.nf16 = L.nbf16 = L.nf32 = 0;
+#pragma unroll
+  for (int m = 0; m < 6; ++m) L.mm[m] = (m & 1) ? 0ull : ~0ull;
+}
+
+// A slot leaves lane s's registers through a per-warp shared-memory record (lane s writes it),
+// then the whole warp folds it into the PC-key row (lanes 0-15) and the object-key row (lanes
+// 16-31), one field per lane: f 0 n  1 zero  2 eq_pre  3 nosnap  4-8 float flags  9-14 min / max
+// 15 n_type (the layout of slot_flush)
+struct SlotSave {
+  uint64_t key;
+  uint32_t info, n, zero, eq, nan, nonint, nf16, nbf16, nf32, pad;
+  uint64_t mm[6];
+};
+__device__ __forceinline__ void lslot_save(SlotSave* sv, const LaneSlot& L) {
+  sv->key = L.key; sv->info = L.info; sv->n = L.n; sv->zero = L.zero; sv->eq = L.eq; sv->nan = L.nan;
+  sv->nonint = L.nonint; sv->nf16 = L.nf16; sv->nbf16 = L.nbf16; sv->nf32 = L.nf32;
+#pragma unroll
+  for (int m = 0; m < 6; ++m) sv->mm[m] = L.mm[m];
+}
+__device__ __noinline__ void lslot_fold(const AnalyzeParams& P, const SlotSave* sv) {
+  __syncwarp();
+  const int lane = threadIdx.x & 31, f = lane & 15;
+  const uint64_t key = sv->key;
+  const uint32_t n = sv->n;
+  if (key == ~0ull || n == 0u) { __syncwarp(); return; }
+  const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
+  const uint32_t meta = (uint32_t)(key >> 32), lg = meta & 3u, kind = (meta >> 2) & 3u;
+  const bool st = meta_store(meta);
+  uint64_t v = 0;
+  uint32_t field = 0;
+  if (f == 0) { v = n; field = st ? F_ST : F_LD; }
+  else if (f == 1) { v = sv->zero; field = F_ZERO; }
+  else if (f == 2) { v = sv->eq; field = st ? F_STEQ : F_LDEQ; }
+  else if (f == 3) { v = (sv->info & 4u) ? n : 0u; field = F_NOSNAP; }
+  else if (f == 4) { v = sv->nan; field = F_NAN; }
+  else if (f == 5) { v = sv->nonint; field = F_NONINT; }
+  else if (f == 6) { v = sv->nf16; field = F_NF16; }
+  else if (f == 7) { v = sv->nbf16; field = F_NBF16; }
+  else if (f == 8) { v = sv->nf32; field = F_NF32; }
+  else if (f == 15) { v = n; field = F_TYPE0 + type_code(kind, lg); }
+  else v = sv->mm[f - 9];
+  bool skip;
+  if (f <= 8 || f == 15) skip = v == 0;
+  else {
+    const int m = f - 9;
+    skip = (m >= 4 && kind < 2u) || ((m & 1) ? v == 0ull : v == ~0ull);
+  }
+  if (!skip) {
+    if (lane < 16) fold_row(P, pc < P.sp ? (int)pc : -1, pc, f, field, v);
+    else fold_row(P, koi < P.so ? (int)(P.sp + koi) : -1, P.n_pcs + koi, f, field, v);
+  }
+  __syncwarp();
+}
+
+// merge slot v's deferred constant segment into the line states (all lanes); returns the new FAIL bits
+__device__ __noinline__ uint32_t sl_flush(const AnalyzeParams& P, WarpCache& wc, SlotLine* sl, int v, uint64_t key,
+                                          uint32_t lf) {
+  if (!sl[v].cpend) return lf;
+  const uint32_t nlf = const_line(P, wc, sl[v].cx0, sl[v].cx1, sl[v].cy, (uint32_t)(key >> 32), (uint32_t)key & 0xFFFFu,
+                                  (uint32_t)(key >> 16) & 0xFFFFu, lf);
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) sl[v].cpend = 0;
+  __syncwarp();
+  return nlf;
+}
+
+// a slot for key (all lanes): the caller picked slot v (a free one, else round robin: the victim
+// key vk with FAIL bits vlf, whose pending segment is merged here); returns the new slot's dense
+// array and, in lf, its FAIL bits
+__device__ __noinline__ unsigned long long lslot_prepare(const AnalyzeParams& P, WarpCache& wc, SlotLine* sl, int v,
+                                                        bool evict, uint64_t vk, uint32_t vlf, uint64_t key, int oi,
+                                                        bool nosnap, bool postok, uint32_t* lf,
+                                                        unsigned long long* dq) {
+  if (evict) sl_flush(P, wc, sl, v, vk, vlf);
+  const uint32_t pc = (uint32_t)key & 0xFFFFu, koi = (uint32_t)(key >> 16) & 0xFFFFu;
+  const uint32_t meta = (uint32_t)(key >> 32);
+  *lf = slot_lfail(P, pc, koi);
+  const unsigned long long dn = (P.dense_ok && !meta_store(meta) && !nosnap) ? dense_lookup(P, oi, (meta << 16) | pc) : 0ull;
+  (void)postok;
+  *dq = 0ull;   // a post array is claimed on demand (win_fast), so keys counted against pre use no slot
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) sl[v].cpend = 0;
+  __syncwarp();
+  return dn;
+}
+
+// C8 of one fast window of a key with a live line state (all lanes); returns the new FAIL bits
+__device__ __noinline__ uint32_t win_line(const AnalyzeParams& P, WarpCache& wc, SlotLine* sl, int s, uint64_t key,
+                                          uint32_t lf, uint64_t addr, uint64_t val) {
+  const unsigned FULL = 0xFFFFFFFFu;
+  const uint32_t pc0 = (uint32_t)key & 0xFFFFu, koi0 = (uint32_t)(key >> 16) & 0xFFFFu, meta0 = (uint32_t)(key >> 32);
+  const uint64_t cy = shfl64(FULL, val, 0);
+  if (!__all_sync(FULL, val == cy)) return fast_line(P, wc, addr, val, meta0, pc0, koi0, lf);
+  // a window of one value: its points lie on y = cy between its extreme addresses; consecutive
+  // windows of one value only widen a held segment (the (+) monoid keeps the extreme points)
+  const uint64_t xmin = redmin64(FULL, addr), xmax = redmax64(FULL, addr);
+  SlotLine& e = sl[s];
+  if (e.cpend && e.cy == cy) {
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) {
+      e.cx0 = xmin < e.cx0 ? xmin : e.cx0;
+      e.cx1 = xmax > e.cx1 ? xmax : e.cx1;
+    }
+    __syncwarp();
+    return lf;
+  }
+  lf = sl_flush(P, wc, sl, s, key, lf);
+  if (lf != 3u && (threadIdx.x & 31) == 0) { e.cpend = 1; e.cy = cy; e.cx0 = xmin; e.cx1 = xmax; }
+  __syncwarp();
+  return lf;
+}
+
+// The value statistics of a fast window of type (KIND, LG) that is not entirely counted
+// densely (lanes with dl are: their values are taken from the pre snapshot at report time).
+template <int KIND, int LG>
+__device__ __forceinline__ void win_value(const AnalyzeParams& P, LaneSlot& L, int s, bool st, bool eq, bool dl,
+                                          uint64_t val, uint64_t word, uint32_t bit, bool dense_key, uint32_t tag) {
+  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;
+  constexpr bool ISF = KIND >= 2;
+  constexpr int MB = KIND == 3 ? 7 : (LG == 1 ? 10 : LG == 2 ? 23 : 52);
+  constexpr MT MID = (MT)~0ull;
+  const unsigned FULL = 0xFFFFFFFFu;
+  const int lane = threadIdx.x & 31;
+  const MT b = (MT)val;
+  const bool fo = !dl;
+  const uint32_t zc = __popc(__ballot_sync(FULL, fo && b == (MT)0));
+  const uint32_t ec = __popc(__ballot_sync(FULL, eq));
+  const MT r0 = wmin<MT>(fo ? b : MID), r1 = wmax<MT>(fo ? b : (MT)0);
+  uint64_t R[6] = {(uint64_t)r0, (uint64_t)r1, ~0ull, 0ull, ~0ull, 0ull};
+  uint32_t fsum = 0, nf32 = 0;
+  if constexpr (KIND == 0) {
+    R[2] = R[0]; R[3] = R[1];
+  } else if constexpr (KIND == 1) {
+    if constexpr (LG < 3) {                 // sext32(b) ^ 2^31 (order-isomorphic to the 64-bit key)
+      constexpr uint32_t sh = 32 - (8 << LG);
+      const uint32_t k = (uint32_t)(((int32_t)(b << sh)) >> sh) ^ 0x80000000u;
+      const uint32_t a = __reduce_min_sync(FULL, fo ? k : 0xFFFFFFFFu), c = __reduce_max_sync(FULL, fo ? k : 0u);
+      R[2] = (uint64_t)(int64_t)(int32_t)(a ^ 0x80000000u) ^ (1ull << 63);
+      R[3] = (uint64_t)(int64_t)(int32_t)(c ^ 0x80000000u) ^ (1ull << 63);
+    } else {
+      R[2] = redmin64(FULL, fo ? (b ^ (1ull << 63)) : ~0ull);
+      R[3] = redmax64(FULL, fo ? (b ^ (1ull << 63)) : 0ull);
+    }
+  } else {
+    uint32_t ff;
+    if constexpr (KIND == 2 && LG == 2) ff = fflags_f32((uint32_t)b);
+    else if constexpr (LG < 3) ff = fflags32<KIND, LG>((uint32_t)b);
+    else { int64_t ival; ff = float_flags(val, 2u, 3u, ival); }
+    const bool okv = fo && !(ff & 1u);      // NaNs excluded from ord / trunc
+    ff = fo ? ff : 0u;
+    constexpr MT SIGN = (MT)1 << ((8 << LG) - 1);
+    constexpr MT MASK = (MT)((8 << LG) == 64 ? ~0ull : ((1ull << (8 << LG)) - 1ull));
+    const MT k = (b & SIGN) ? (~b & MASK) : (b | SIGN);
+    const MT tmask = (MT)(P.mant_bits >= (uint32_t)MB ? ~0ull : ~((1ull << (MB - P.mant_bits)) - 1ull));
+    const MT t = b & tmask;
+    const MT k0 = wmin<MT>(okv ? k : MID), k1 = wmax<MT>(okv ? k : (MT)0);
+    const MT t0 = wmin<MT>(okv ? t : MID), t1 = wmax<MT>(okv ? t : (MT)0);
+    R[2] = (LG < 3 && k0 == MID) ? ~0ull : (uint64_t)k0; R[3] = (uint64_t)k1;
+    R[4] = (LG < 3 && t0 == MID) ? ~0ull : (uint64_t)t0; R[5] = (uint64_t)t1;
+    fsum = __reduce_add_sync(FULL, (ff & 1u) | (((ff >> 1) & 1u) << 6) | (((ff >> 2) & 1u) << 12) | (((ff >> 3) & 1u) << 18));
+    if constexpr (LG == 3) nf32 = __popc(__ballot_sync(FULL, (ff >> 4) & 1u));
+  }
+  if (lane == s) {
+    L.n += 32u; L.zero += zc; L.eq += ec;
+    if constexpr (ISF) {
+      L.nan += fsum & 63u; L.nonint += (fsum >> 6) & 63u; L.nf16 += (fsum >> 12) & 63u; L.nbf16 += (fsum >> 18) & 63u;
+      L.nf32 += nf32;
+    }
+#pragma unroll
+    for (int m = 0; m < 6; ++m) L.mm[m] = (m & 1) ? (R[m] > L.mm[m] ? R[m] : L.mm[m]) : (R[m] < L.mm[m] ? R[m] : L.mm[m]);
+  }
+  // C10 written elements; C3 loaded elements of loads not counted per element
+  if (st) bitmap_or_win(P.t.W, true, word, bit);
+  else if (!dense_key && __any_sync(FULL, eq)) bitmap_or_win(P.t.L, eq, word, bit);
+  // S8: every record not counted per element is inserted per distinct value
+  const unsigned hm = __ballot_sync(FULL, fo);
+  const int l = __ffs(hm) - 1;
+  const uint64_t v0 = (LG < 3) ? (uint64_t)__shfl_sync(FULL, (uint32_t)val, l) : shfl64(FULL, val, l);
+  if (__all_sync(FULL, !fo || val == v0)) {
+    if (lane == l) hist_insert(P, tag, val, __popc(hm));
+  } else if (fo) {
+    const unsigned vg = (LG < 3) ? __match_any_sync(hm, (uint32_t)val) : __match_any_sync(hm, val);
+    hist_insert_warp(P, hm, lane == __ffs(vg) - 1, tag, val, __popc(vg));
+  }
+  __syncwarp();   // reconverge before the next window's warp-collectives
+}
+
+// one fast window of access width LG: eq_pre, then the per-element counted lanes -- loads that read
+// the pre value (dn) and records that carry the post value (dq, gathered here) -- and the value path
+// of the window's type for the rest
+template <int LG>
+__device__ __forceinline__ bool win_fast(const AnalyzeParams& P, LaneSlot& L, int s, uint32_t meta0, uint32_t pc0,
+                                         uint32_t oid, uint64_t opre, uint64_t obm, uint64_t off, uint64_t val,
+                                         uint64_t pv, unsigned long long dn, uint64_t qv, unsigned long long dq) {
+  using MT = typename std::conditional<(LG < 3), uint32_t, uint64_t>::type;
+  constexpr MT WMASK = (MT)(LG == 3 ? ~0ull : ((1ull << (8u << LG)) - 1ull));
+  const unsigned FULL = 0xFFFFFFFFu;
+  const int lane = threadIdx.x & 31;
+  const bool st = meta_store(meta0);
+  bool eq = false;
+  if (opre) eq = ((MT)pv & WMASK) == (MT)val;   // pv: the gathered pre element (low 8w bits)
+  const uint64_t e = off >> LG;
+  const bool dl = dn != 0ull && eq;
+  if (dn != 0ull && __all_sync(FULL, dl)) {
+    red_add_keep(reinterpret_cast<uint32_t*>(dn) + e, 1u, true);
+    if (lane == s) { L.n += 32u; L.eq += 32u; }
+    return false;
+  }
+  const bool dql = dq != 0ull && !dl && ((MT)qv & WMASK) == (MT)val;   // qv: the gathered post element
+  const bool dc = dl || dql;                   // counted per element: value statistics at the flush
+  red_add_keep(reinterpret_cast<uint32_t*>(dn) + e, 1u, dl);
+  red_add_keep(reinterpret_cast<uint32_t*>(dq) + e, 1u, dql);
+  const uint64_t word = obm + (e >> 5);
+  const uint32_t bit = 1u << ((uint32_t)e & 31u);
+  if (__all_sync(FULL, dc)) {
+    const uint32_t ec = __popc(__ballot_sync(FULL, eq));
+    if (lane == s) { L.n += 32u; L.eq += ec; }
+    if (st) bitmap_or_win(P.t.W, true, word, bit);
+    else if (dn == 0ull && __any_sync(FULL, eq)) bitmap_or_win(P.t.L, eq, word, bit);
+    return false;
+  }
+  const uint32_t tag = (pc0 << 16) | (oid & 0xFFFFu);
+  const bool dk = dn != 0ull;
+  switch (meta0 & 15u) {
+#define VE_WV(K) win_value<K, LG>(P, L, s, st, eq, dc, val, word, bit, dk, tag)
+    case 0u | LG: VE_WV(0); break;
+    case 4u | LG: VE_WV(1); break;
+    default:
+      if constexpr (LG == 1) {
+        if ((meta0 & 15u) == 13u) { VE_WV(3); break; }
+      }
+      if constexpr (LG != 0) VE_WV(2);
+      break;
+#undef VE_WV
+  }
+  return dq == 0ull;    // lanes went the value path: a post array may count them per element
+}
+
+// claim the post-value array of the current slot's key (all lanes; on the first window that needs it)
+__device__ __noinline__ unsigned long long post_claim(const AnalyzeParams& P, int oi, uint64_t key) {
+  const uint32_t pc = (uint32_t)key & 0xFFFFu, meta = (uint32_t)(key >> 32);
+  return dense_lookup(P, oi, DENSE_POST | (meta << 16) | pc);
+}
+
+// K1 v2 runs K2_WARPS warps per CTA (168 registers: the slots and the object state stay in registers)
+// inside the 16-warp shared-memory layout of v1 (rings and staging regions of warps >= K2_WARPS unused)
+#ifndef VE_K2_THREADS
+#define VE_K2_THREADS 384
+#endif
+constexpr int K2_THREADS = VE_K2_THREADS;
+constexpr int K2_WARPS = K2_THREADS / 32;
+static_assert(K2_WARPS <= K1_WARPS, "v2 uses the v1 shared-memory layout");
+
+__global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constant__ AnalyzeParams P) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const unsigned FULL = 0xFFFFFFFFu;
+  {
+    const uint32_t nsk = P.sp + P.so;
+    const Smem S = smem_of(P);
+    for (uint32_t i = tid; i < nsk * NSUM; i += blockDim.x) S.ssum[i] = 0;
+    for (uint32_t i = tid; i < nsk * NMM; i += blockDim.x) { S.smin[i] = ~0ull; S.smax[i] = 0; }
+    for (uint32_t i = tid; i < nsk; i += blockDim.x) { S.sline[i].state = VE_LINE_EMPTY; S.sline[i].lock = 0; }
+    for (uint32_t i = tid; i < P.hs; i += blockDim.x) {
+      S.shs[i].bits = 0; S.shs[i].tag = EMPTY_TAG; S.shs[i].pad = 0; S.shc[i] = 0;
+    }
+    for (uint32_t i = tid; i < P.objc; i += blockDim.x) { S.sob[i] = P.o.base[i]; S.soe[i] = P.o.end[i]; }
+    if (tid < 4) S.sctr[tid] = 0;
+    if (tid < K1_WARPS - K2_WARPS) P.stage_cnt[(uint64_t)blockIdx.x * K1_WARPS + K2_WARPS + tid] = 0;
+  }
+  __shared__ WarpCache s_wc[K1_WARPS];
+  __shared__ SlotLine s_sl[K1_WARPS][NS2];
+  __shared__ SlotSave s_save[K1_WARPS];
+  WarpCache& wc = s_wc[warp];
+  SlotLine* sl = s_sl[warp];
+  if (lane < WC) wc.key1[lane] = 0;
+  sl[lane].cpend = 0;
+  if (lane == 0) { wc.next = 0; s_stage_n[warp] = 0; }
+  LaneSlot L;
+  L.key = ~0ull; L.dn = 0; L.dq = 0; L.info = 0;
+  lslot_clear_acc(L);
+  uint32_t snext = 0;
+
+  // objects: the CTA caches sorted objects 0..31 (base, end, pre, bitmap offset, id | log2 ew << 16 |
+  // fast << 20); an address is mapped by one ballot over them when there are at most 32, else by
+  // binary search
+  const bool ob32 = P.o.n <= 32u;
+  __shared__ uint64_t s_ob[32], s_oe[32], s_opre[32], s_obm[32], s_opost[32];
+  __shared__ uint32_t s_ometa[32];
+  if (tid < 32 && (uint32_t)tid < P.o.n) {
+    const uint64_t b = P.o.base[tid], e = P.o.end[tid], pr = P.o.pre[tid], po = P.o.post[tid];
+    s_ob[tid] = b; s_oe[tid] = e; s_opre[tid] = pr; s_obm[tid] = P.o.bmoff[tid];
+    const uint32_t ew = P.o.ew[tid];
+    const uint32_t lg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
+    const bool fast = e - b >= ew && (pr & (ew - 1)) == 0;
+    s_opost[tid] = (po & (ew - 1)) == 0 ? po : 0ull;   // post values counted per element need aligned elements
+    s_ometa[tid] = (P.o.id[tid] & 0xFFFFu) | (lg << 16) | (fast ? (1u << 20) : 0u);
+  }
+
+  Ring R;
+  R.dst0 = smem_u32(ve_smem + P.o_ring + (uint32_t)warp * RING * WIN_BYTES);
+  R.o0 = R.o = R.dst0 + (uint32_t)lane * 24u;
+  R.bar0 = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
+  R.d = R.sw = R.ph = R.pend = 0;
+  R.left = 0;
+  if (lane == 0 && P.nring) {
+    for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar0 + d * 8u, 1);
+    fence_mbar_init();
+  }
+  __syncwarp();
+  R.nextc = P.chunk == CHUNK ? (uint64_t)blockIdx.x * K2_WARPS + warp : (uint64_t)warp * gridDim.x + blockIdx.x;
+  R.cstride = gridDim.x * K2_WARPS;
+  ring_claim(P, R);
+  for (int d = 0; d < NSTAGE; ++d) ring_issue_stage(P, R, (uint32_t)d);
+  __syncthreads();
+
+  // the current object (warp-uniform): offsets [0, clim] hold a whole element
+  uint64_t cb = 1, clim = 0, cpre = 0, cbm = 0, cpost = 0;
+  uint32_t cid = 0, clg = 0xFFu;
+  int coi = -1;
+  // the current slot's warp-uniform copies (dense arrays, FAIL bits)
+  unsigned long long ldn = 0, ldq = 0;
+  bool lpt = false;          // the post array of the current slot was claimed (or tried)
+  uint32_t llf = 3;
+  uint32_t n_inv = 0, n_unm = 0;
+
+  // make sorted object oi (-1: none) the current object
+  auto obj_set = [&](int oi) {
+    coi = oi;
+    if (oi < 0) {
+      cb = 1; clim = 0; clg = 0xFFu; cpre = 0; cpost = 0;
+    } else if (ob32) {
+      cb = s_ob[oi];
+      const uint64_t ce = s_oe[oi];
+      cpre = s_opre[oi];
+      cpost = s_opost[oi];
+      cbm = s_obm[oi];
+      const uint32_t mt = s_ometa[oi];
+      cid = mt & 0xFFFFu;
+      const bool fok = (mt >> 20) & 1u;
+      clg = fok ? (mt >> 16) & 3u : 0xFFu;
+      clim = fok ? ce - cb - (1ull << ((mt >> 16) & 3u)) : 0ull;
+    } else {
+      cb = P.o.base[oi];
+      const uint64_t ce = P.o.end[oi];
+      cpre = P.o.pre[oi]; cbm = P.o.bmoff[oi]; cid = P.o.id[oi];
+      const uint32_t ew = P.o.ew[oi];
+      cpost = (P.o.post[oi] & (ew - 1)) == 0 ? P.o.post[oi] : 0ull;
+      const uint32_t lg = (ew == 1) ? 0 : (ew == 2) ? 1 : (ew == 4) ? 2 : 3;
+      const bool fok = ce - cb >= ew && (cpre & (ew - 1)) == 0;
+      clg = fok ? lg : 0xFFu;
+      clim = fok ? ce - cb - ew : 0ull;
+    }
+  };
+  // the object holding address a0 (warp-uniform) becomes current, unless it already is
+  auto obj_find = [&](uint64_t a0) {
+    if (a0 - cb <= clim && coi >= 0) return;
+    int oi;
+    if (ob32) {
+      const unsigned m = __ballot_sync(FULL, (uint32_t)lane < P.o.n && s_ob[lane] <= a0 && a0 < s_oe[lane]);
+      oi = m ? __ffs(m) - 1 : -1;
+    } else {
+      oi = find_object(P, a0);
+    }
+    obj_set(oi);
+  };
+  // the key of the current slot: kpm = its (pc | meta << 32) word, klg its access width, kwm / kvm
+  // the alignment and value-bit masks; a window continues it when every lane carries kpm, lies in
+  // the current object at an aligned element and has no value bits above its width
+  uint64_t kpm = ~0ull, kvm = 0;
+  uint32_t kwm = 0, klg = 0;
+  uint64_t kkey = ~0ull;
+  int s = 0;
+
+  while (R.left) {
+    uint64_t addr, val, pm;
+    ring_next(P, R, addr, val, pm);
+    const uint64_t off = addr - cb;
+    if (!__all_sync(FULL, pm == kpm && off <= clim && ((uint32_t)off & kwm) == 0u && (val & kvm) == val)) {
+      // another key, another object, or a window for the slow path
+      const uint64_t pm0 = shfl64(FULL, pm, 0);
+      const uint32_t meta0 = (uint32_t)(pm0 >> 32), pc0 = (uint32_t)pm0;
+      bool fast = false;
+      if (__all_sync(FULL, pm == pm0) && meta_fast(meta0, pc0, P.n_pcs)) {
+        const uint32_t lg0 = meta0 & 3u;
+        const uint64_t wm = (1ull << lg0) - 1ull;
+        const bool vok = lg0 == 3u || (val >> (8u << lg0)) == 0ull;
+        obj_find(shfl64(FULL, addr, 0));
+        const uint64_t o = addr - cb;
+        fast = lg0 == clg && __all_sync(FULL, vok && o <= clim && (o & wm) == 0ull);
+      }
+      if (!fast) {
+        const uint32_t cnt = slow_window(P, wc, addr, val, pm, true);
+        n_inv += cnt & 0xFFFFu;
+        n_unm += cnt >> 16;
+        kpm = ~0ull;          // (the object may have changed under the key)
+        continue;
+      }
+      const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)cid << 16) | pc0;
+      if (key != kkey) {
+        const unsigned hit = __ballot_sync(FULL, L.key == key);
+        if (hit) {
+          s = __ffs(hit) - 1;
+        } else {
+          const unsigned fr = __ballot_sync(FULL, L.key == ~0ull);
+          const bool evict = fr == 0u;
+          s = evict ? (int)(snext++ & 31u) : __ffs(fr) - 1;
+          const uint64_t vk = shfl64(FULL, L.key, s);
+          const uint32_t vlf = __shfl_sync(FULL, L.info, s) & 3u;
+          uint32_t nlf;
+          unsigned long long dq;
+          const unsigned long long dn = lslot_prepare(P, wc, sl, s, evict, vk, vlf, key, coi, cpre == 0ull,
+                                                      cpost != 0ull, &nlf, &dq);
+          if (evict) {
+            if (lane == s) lslot_save(&s_save[warp], L);
+            lslot_fold(P, &s_save[warp]);
+          }
+          if (lane == s) {
+            L.key = key;
+            L.dn = dn;
+            L.dq = dq;
+            L.info = nlf | (cpre == 0ull ? 4u : 0u);
+            lslot_clear_acc(L);
+          }
+        }
+        kkey = key;
+        ldn = shfl64(FULL, L.dn, s);
+        ldq = shfl64(FULL, L.dq, s);
+        lpt = (__shfl_sync(FULL, L.info, s) >> 3) & 1u;
+        llf = __shfl_sync(FULL, L.info, s) & 3u;
+      }
+      kpm = pm0;
+      klg = meta0 & 3u;
+      kwm = (1u << klg) - 1u;
+      kvm = klg == 3u ? ~0ull : ((1ull << (8u << klg)) - 1ull);
+    }
+    // a fast window of the current key in the current object
+    const uint64_t o = addr - cb;
+    uint64_t pv = 0, qv = 0;
+    if (cpre != 0ull) pv = ld_pre<3>((cpre + o) & ~7ull) >> (8u * (uint32_t)((cpre + o) & 7ull));
+    if (ldq != 0ull) qv = ld_pre<3>((cpost + o) & ~7ull) >> (8u * (uint32_t)((cpost + o) & 7ull));
+    const uint32_t meta0 = (uint32_t)(kpm >> 32), pc0 = (uint32_t)kpm;
+    bool wantq = false;
+    switch (klg) {
+      case 0: wantq = win_fast<0>(P, L, s, meta0, pc0, cid, cpre, cbm, o, val, pv, ldn, qv, ldq); break;
+      case 1: wantq = win_fast<1>(P, L, s, meta0, pc0, cid, cpre, cbm, o, val, pv, ldn, qv, ldq); break;
+      case 2: wantq = win_fast<2>(P, L, s, meta0, pc0, cid, cpre, cbm, o, val, pv, ldn, qv, ldq); break;
+      default: wantq = win_fast<3>(P, L, s, meta0, pc0, cid, cpre, cbm, o, val, pv, ldn, qv, ldq); break;
+    }
+    if (wantq && !lpt && cpost != 0ull && P.dense_ok) {       // first value-path window of the key
+      lpt = true;
+      ldq = post_claim(P, coi, kkey);
+      if (lane == s) { L.dq = ldq; L.info |= 8u; }
+    }
+    // (no overflow check: a launch gives a warp < 2^31 records, so the 32-bit accumulators hold)
+    if (llf != 3u) {
+      const uint32_t nlf = win_line(P, wc, sl, s, kkey, llf, addr, val);
+      if (nlf != llf) {
+        llf = nlf;
+        if (lane == s) L.info = (L.info & ~3u) | nlf;
+      }
+    }
+  }
+  // windows outside the ring: the partial last window, or (records not 16-byte aligned) a
+  // static range of every warp
+  const uint64_t nwin = (P.n + 31) / 32;
+  const uint64_t tw = (uint64_t)gridDim.x * K2_WARPS, gw = (uint64_t)blockIdx.x * K2_WARPS + warp;
+  uint64_t wbeg = P.nring, wend = gw == 0 ? nwin : P.nring;
+  if (!P.nring) { wbeg = gw * nwin / tw; wend = (gw + 1) * nwin / tw; }
+  for (uint64_t w = wbeg; w < wend; ++w) {
+    const Rec cur = load_rec(P, w, wend, lane);
+    const uint32_t cnt = slow_window(P, wc, cur.addr, cur.val, cur.pm, w * 32 + lane < P.n);
+    n_inv += cnt & 0xFFFFu;
+    n_unm += cnt >> 16;
+  }
+  // fold the slots (pending constant segments first), the line cache, then the CTA's shared state
+  for (int v = 0; v < NS2; ++v) {
+    const uint64_t vk = shfl64(FULL, L.key, v);
+    if (vk == ~0ull) continue;
+    sl_flush(P, wc, sl, v, vk, __shfl_sync(FULL, L.info, v) & 3u);
+  }
+  for (int v = 0; v < NS2; ++v) {
+    if (lane == v) lslot_save(&s_save[warp], L);
+    lslot_fold(P, &s_save[warp]);
+  }
+  n_inv = __reduce_add_sync(FULL, n_inv);
+  n_unm = __reduce_add_sync(FULL, n_unm);
+  __syncwarp();
+  const Smem S = smem_of(P);
+  const uint32_t nsk = P.sp + P.so;
+  if (lane == 0) {
+    const uint32_t ns = s_stage_n[warp];
+    P.stage_cnt[(uint64_t)blockIdx.x * K1_WARPS + warp] = ns < P.stage_rs ? ns : P.stage_rs;
+    if (n_inv) atomicAdd(&S.sctr[0], n_inv);
+    if (n_unm) atomicAdd(&S.sctr[1], n_unm);
+    wcache_flush(P, wc);
+  }
+  __syncthreads();
+
+  for (uint32_t i = tid; i < nsk * NSUM; i += blockDim.x) {
+    const uint32_t v = S.ssum[i];
+    if (v) {
+      const uint32_t s = i / NSUM, fld = i % NSUM;
+      const uint32_t key = s < P.sp ? s : P.n_pcs + (s - P.sp);
+      atomicAdd(&P.t.sum[(uint64_t)key * NSUM + fld], (unsigned long long)v);
+    }
+  }
+  for (uint32_t i = tid; i < nsk * NMM; i += blockDim.x) {
+    const uint32_t s = i / NMM, fld = i % NMM;
+    const uint32_t key = s < P.sp ? s : P.n_pcs + (s - P.sp);
+    if (S.smin[i] != ~0ull) atomic_min_u64(&P.t.mn[(uint64_t)key * NMM + fld], S.smin[i]);
+    if (S.smax[i] != 0ull) atomic_max_u64(&P.t.mx[(uint64_t)key * NMM + fld], S.smax[i]);
+  }
+  for (uint32_t s = tid; s < nsk; s += blockDim.x) P.t.lcta[(uint64_t)blockIdx.x * nsk + s] = S.sline[s];
+  for (uint32_t i = tid; i < P.hs; i += blockDim.x) {
+    if (S.shs[i].tag != EMPTY_TAG) hist_insert_global_rf(P.t, S.shs[i].tag, S.shs[i].bits, S.shc[i]);
+  }
+  if (tid == 0) {
+    if (S.sctr[0]) atomicAdd(&P.t.glob[G_INVALID], (unsigned long long)S.sctr[0]);
+    if (S.sctr[1]) atomicAdd(&P.t.glob[G_UNMAPPED], (unsigned long long)S.sctr[1]);
+    if (blockIdx.x == 0) atomicAdd(&P.t.glob[G_RECORDS], (unsigned long long)P.n);
+  }
+}
+
 // K1b: insert the staged S8 groups into the HBM table (one block per warp region).
 __global__ void __launch_bounds__(256) k_hist_drain(const uint4* __restrict__ stage, const uint32_t* __restrict__ cnt,
                                                     uint32_t rs, DevTables t) {
@@ -1919,7 +2475,10 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   // (VE_K1_MULTI=0/1 forces one instantiation: the parity tests run both on the same traces)
   const char* fm = getenv("VE_K1_MULTI");
   const bool multi = VE_MULTI_DENSE && (fm && *fm ? *fm == '1' : c->cfg.n_pcs >= VE_MULTI_MIN_PCS);
-  auto kfn = multi ? k_analyze<true> : k_analyze<false>;
+  // K1 v2 (register key slots) unless VE_K1=1 selects the v1 kernels
+  const char* kv = getenv("VE_K1");
+  const bool v2 = !(kv && *kv == '1');
+  auto kfn = v2 ? k_analyze2 : multi ? k_analyze<true> : k_analyze<false>;
   cudaFuncGetAttributes(&fa, kfn);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring
   // 2048 slots measured best on cfg2 / cfg3 / cfg4 (the HBM table behind it stays L2-resident)
@@ -1940,7 +2499,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   // staging regions: a warp stages at most one group per record of its static range
   {
     const uint64_t tw = blocks * K1_WARPS;
-    const uint64_t per = 32 * ((windows + tw - 1) / tw + 2);
+    const uint64_t twa = blocks * (v2 ? K2_WARPS : K1_WARPS);   // warps that take windows
+    const uint64_t per = 32 * ((windows + twa - 1) / twa + 2);
     P.stage_rs = (uint32_t)(per < STAGE_RS_MAX ? per : STAGE_RS_MAX);
     const size_t need = (size_t)tw * P.stage_rs * sizeof(uint4) + tw * sizeof(uint32_t);
     if (c->hstage_bytes < need) {
@@ -1959,7 +2519,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze claim counter");
 #endif
   count_launch();
-  kfn<<<(unsigned)blocks, K1_THREADS, sb, s>>>(P);
+  kfn<<<(unsigned)blocks, v2 ? K2_THREADS : K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze launch");
   count_launch();

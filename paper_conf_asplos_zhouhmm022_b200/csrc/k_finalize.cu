@@ -797,6 +797,7 @@ ve_status finalize_hist_views(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& 
 }
 
 // ---- dense per-element counts -> exact histogram ------------------------------
+// (one array per launch: the path of claims whose counts are mostly 0 -- sparse or high-cardinality reads)
 // A dense counter cnt[e] of (pc, object) counts loads that read element e's unchanged
 // pre-snapshot value, so it contributes cnt[e] occurrences of that value (C9).
 // Each block aggregates its chunk of elements by value (warp match, then a small
@@ -883,7 +884,7 @@ template <int NT>
 __global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
                                                            uint32_t ew, uint32_t tag, uint64_t bmoff, DevTables t,
                                                            uint32_t meta, uint32_t mant_bits, uint32_t kp, uint32_t ko,
-                                                           uint32_t ts, uint32_t csz) {
+                                                           uint32_t ts, uint32_t csz, uint32_t setL) {
   extern __shared__ unsigned long long df_smem[];
   unsigned long long* sbits = df_smem;
   uint32_t* scnt = reinterpret_cast<uint32_t*>(df_smem + ts);
@@ -921,7 +922,7 @@ __global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n
     const unsigned km = __ballot_sync(0xFFFFFFFFu, k != 0);
     // C3: a counted load started at element e (K1 leaves these L bits to us); the
     // warp's 32 elements are one aligned bitmap word
-    if (lane == 0 && km) atomicOr(&t.L[bmoff + ((base + threadIdx.x) >> 5)], km);
+    if (setL && lane == 0 && km) atomicOr(&t.L[bmoff + ((base + threadIdx.x) >> 5)], km);
     if (k) {
       const unsigned g = __match_any_sync(km, bits);
       // (a REDUX under per-lane group masks runs once per distinct mask: singletons skip it)
@@ -1020,6 +1021,328 @@ __global__ void __launch_bounds__(1024) k_dense_sample(const uint32_t* cnt, uint
   if (threadIdx.x == 0) out[0] = nd;
 }
 
+// ---- fused per-object flush of the dense counters (all claims of one object in one pass) --------
+// Every claim j of object o counts, per element e, the records of one (pc, access type) whose value
+// was e's PRE value (side 0, loads) or e's POST value (side 1, DENSE_POST): their histogram entries
+// are (tag_j, side value of e) with count c_j(e).  One pass over the object reads each snapshot side
+// once and every claim's counters, and aggregates in a block-local table:
+//   H0_side(v) = #elements of the pass with side value v (one insert per element and side), and
+//   D_j(v)    = sum of (c_j(e) - m_j) over the elements where c_j(e) != m_j,
+// m_j being a per-block base multiplicity (the mode of c_j over 32 sampled elements): stencils read
+// every element once per PC, so H0 carries the whole count and corrections are few (clamped faces).
+// When the table is emptied, the local count of (j, v) is m_j * H0_side(v) + D_j(v) -- exactly the
+// number of counted records of claim j with value v among the elements of this table generation
+// (every D_j(v) of the generation has its H0_side(v) beside it); positive counts go to the HBM
+// table with their value statistics (C1 n_zero, C4-C7), so no zero-count entry is ever created.
+constexpr int DO_THREADS = 1024;
+// block table: 16-byte slots {value bits, cls << 56 | (count + 2^55)}: cls 0 / 1 = H0 of the pre / post
+// side, 2 + j = correction of claim j, 0xFF = empty; the biased 56-bit count takes signed adds
+constexpr uint32_t DO_TS = 12288;                // 192 KiB of shared memory
+constexpr uint64_t DO_EMPTY = 0xFFull << 56;
+constexpr uint64_t DO_BIAS = 1ull << 55;
+constexpr uint64_t DO_M56 = (1ull << 56) - 1ull;
+constexpr int DO_MAXC = DENSE_PER_OBJ;
+constexpr uint64_t DO_CH = 65536;               // elements per chunk
+struct DoClaim {
+  uint32_t* cnt;        // counters (zeroed by the flush)
+  uint32_t tag, meta;   // (pc << 16 | object id), access type
+  uint32_t side, kp;    // 0 pre / 1 post; PC key row
+  uint32_t m, pad;      // base multiplicity (>= 1): the mode of the counts, sampled by k_dense_mode
+};
+struct DoArgs {
+  DoClaim c[DO_MAXC];
+  uint32_t nc, ew, ko, mant_bits;
+  uint64_t ne;          // whole elements
+  const uint8_t* snap[2];
+  uint64_t bmoff;
+};
+struct DoStat {          // per-claim value statistics (shared, then the two key rows)
+  unsigned long long s[6];   // zero, nan, nonint, not_f16, not_bf16, not_f32
+  unsigned long long mn[3], mx[3];
+};
+
+__device__ __forceinline__ uint64_t do_load(const uint8_t* p, uint32_t ew) {
+  return ew == 1 ? *p : ew == 2 ? *(const uint16_t*)p : ew == 4 ? *(const uint32_t*)p : *(const uint64_t*)p;
+}
+
+struct DoSlot {
+  uint64_t v, w;        // value bits; cls << 56 | biased count
+};
+__device__ __forceinline__ uint32_t do_h(uint32_t cls, uint64_t v) {
+  uint32_t h = ((uint32_t)v ^ (uint32_t)(v >> 32) ^ (cls * 0x9E3779B9u)) * 0x85EBCA6Bu;
+  h ^= h >> 15;
+  h *= 0xC2B2AE35u;
+  h ^= h >> 13;
+  return (uint32_t)(((uint64_t)h * DO_TS) >> 32);
+}
+// add d to (cls, v) in the block table (claims a slot with a 128-bit CAS); false when 64 probes found
+// no place
+__device__ __forceinline__ bool do_add(DoSlot* ts, uint32_t cls, uint64_t v, long long d, uint32_t* fill) {
+  uint32_t h = do_h(cls, v);
+  for (int probe = 0; probe < 64; ++probe) {
+    DoSlot* s = &ts[h];
+    uint64_t lo, hi;
+    asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];"
+                 : "=l"(lo), "=l"(hi) : "r"((uint32_t)__cvta_generic_to_shared(s)) : "memory");
+    const uint32_t sc = (uint32_t)(hi >> 56);
+    // (an empty slot reads (0, EMPTY): a match of value 0 is confirmed by the CAS, never taken from the read)
+    if (sc == cls && lo == v && v != 0ull) { atomicAdd((unsigned long long*)&s->w, (unsigned long long)d); return true; }
+    if (sc == 0xFFu || (sc == cls && lo == v)) {
+      uint64_t olo, ohi;
+      cas128_shared(s, 0ull, DO_EMPTY, v, ((uint64_t)cls << 56) | DO_BIAS, olo, ohi);
+      if (ohi == DO_EMPTY && olo == 0ull) {
+        atomicAdd(fill, 1u);
+        atomicAdd((unsigned long long*)&s->w, (unsigned long long)d);
+        return true;
+      }
+      if ((uint32_t)(ohi >> 56) == cls && olo == v) {
+        atomicAdd((unsigned long long*)&s->w, (unsigned long long)d);
+        return true;
+      }
+    }
+    h = h + 1 == DO_TS ? 0u : h + 1;
+  }
+  return false;
+}
+__device__ __forceinline__ long long do_cnt(uint64_t w) { return (long long)(w & DO_M56) - (long long)DO_BIAS; }
+// read-only lookup (no concurrent writers): the count of (cls, v), 0 if absent
+__device__ __forceinline__ long long do_get(const DoSlot* ts, uint32_t cls, uint64_t v) {
+  uint32_t h = do_h(cls, v);
+  for (int probe = 0; probe < 64; ++probe) {
+    const DoSlot& s = ts[h];
+    const uint32_t sc = (uint32_t)(s.w >> 56);
+    if (sc == 0xFFu) return 0;
+    if (sc == cls && s.v == v) return do_cnt(s.w);
+    h = h + 1 == DO_TS ? 0u : h + 1;
+  }
+  return 0;
+}
+
+// value statistics of k counted records that carry the bits v (C1 n_zero, C5 flags and ord range,
+// C4 raw range, C7 truncated range), accumulated per thread
+struct DoAcc {
+  unsigned long long s[6];
+  unsigned long long mn[3], mx[3];
+};
+__device__ __forceinline__ void do_acc_init(DoAcc& a) {
+#pragma unroll
+  for (int i = 0; i < 6; ++i) a.s[i] = 0;
+#pragma unroll
+  for (int i = 0; i < 3; ++i) { a.mn[i] = ~0ull; a.mx[i] = 0; }
+}
+__device__ __forceinline__ void do_acc(DoAcc& a, uint64_t v, unsigned long long k, uint32_t meta, uint32_t mant_bits) {
+  const uint32_t kind = (meta >> 2) & 3u, lg = meta & 3u;
+  if (v == 0ull) a.s[0] += k;
+  uint32_t ff = 0;
+  if (kind >= 2u) {
+    int64_t ival;
+    ff = float_flags(v, kind, lg, ival);
+#pragma unroll
+    for (int i = 0; i < 5; ++i) if (ff & (1u << i)) a.s[1 + i] += k;
+  }
+  a.mn[0] = v < a.mn[0] ? v : a.mn[0];
+  a.mx[0] = v > a.mx[0] ? v : a.mx[0];
+  if (!(ff & 1u)) {                        // NaNs excluded from ord / trunc (C5, C7)
+    const uint64_t o = ord_key(v, kind, lg);
+    a.mn[1] = o < a.mn[1] ? o : a.mn[1];
+    a.mx[1] = o > a.mx[1] ? o : a.mx[1];
+    if (kind >= 2u) {
+      const uint64_t tr = trunc_bits(v, kind, lg, mant_bits);
+      a.mn[2] = tr < a.mn[2] ? tr : a.mn[2];
+      a.mx[2] = tr > a.mx[2] ? tr : a.mx[2];
+    }
+  }
+}
+// fold a thread's statistics into the block's row of claim j (a warp reduction first)
+__device__ __forceinline__ void do_acc_fold(DoStat& S, DoAcc& a) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int i = 0; i < 6; ++i) {
+    unsigned long long x = a.s[i];
+    for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(0xFFFFFFFFu, x, o);
+    if (lane == 0 && x) atomicAdd(&S.s[i], x);
+  }
+#pragma unroll
+  for (int i = 0; i < 3; ++i) {
+    unsigned long long x = a.mn[i], y = a.mx[i];
+    for (int o = 16; o; o >>= 1) {
+      const unsigned long long xx = __shfl_xor_sync(0xFFFFFFFFu, x, o), yy = __shfl_xor_sync(0xFFFFFFFFu, y, o);
+      x = xx < x ? xx : x;
+      y = yy > y ? yy : y;
+    }
+    if (lane == 0) {
+      if (x != ~0ull) atomicMin(&S.mn[i], x);
+      if (y != 0ull) atomicMax(&S.mx[i], y);
+    }
+  }
+}
+
+// base multiplicity of every claim: the most frequent count among 32 pseudo-random elements
+// (one warp per claim; a regular stride could land on a stencil's faces every time)
+__global__ void k_dense_mode(const uint32_t* const* cnt, const uint64_t* ne, uint32_t* m) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t j = blockIdx.x;
+  const uint64_t n = ne[j];
+  const uint64_t e = n ? mix64(((uint64_t)j << 32) ^ (uint64_t)lane ^ 0x5bd1e995ull) % n : 0;
+  const uint32_t c = n ? cnt[j][e] : 0u;
+  const unsigned g = __match_any_sync(0xFFFFFFFFu, c);
+  const uint32_t best = __reduce_max_sync(0xFFFFFFFFu, ((uint32_t)__popc(g) << 5) | (31u - (uint32_t)lane));
+  const uint32_t mm = __shfl_sync(0xFFFFFFFFu, c, 31 - (int)(best & 31u));
+  if (lane == 0) m[j] = mm;
+}
+
+__global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_constant__ DoArgs A, DevTables t) {
+  extern __shared__ __align__(16) uint8_t do_smem[];
+  DoSlot* ts = reinterpret_cast<DoSlot*>(do_smem);
+  __shared__ DoStat st[DO_MAXC];
+  __shared__ uint32_t s_fill;
+  const int tid = threadIdx.x, lane = tid & 31;
+  for (uint32_t i = tid; i < DO_TS; i += blockDim.x) { ts[i].v = 0; ts[i].w = DO_EMPTY; }
+  if (tid < DO_MAXC * 6) st[tid / 6].s[tid % 6] = 0;
+  if (tid < DO_MAXC * 3) { st[tid / 3].mn[tid % 3] = ~0ull; st[tid / 3].mx[tid % 3] = 0; }
+  if (tid == 0) s_fill = 0;
+  uint32_t sides = 0;                                  // bit s: some claim reads side s
+  for (uint32_t j = 0; j < A.nc; ++j) sides |= 1u << A.c[j].side;
+  __syncthreads();
+  // empty the table: positive local counts of every (claim, value) -> HBM table + statistics
+  auto drain = [&]() {
+    __syncthreads();
+    for (uint32_t j = 0; j < A.nc; ++j) {
+      const uint32_t sd = A.c[j].side;
+      DoAcc acc;
+      do_acc_init(acc);
+      for (uint32_t i = tid; i < DO_TS; i += blockDim.x) {
+        const uint64_t w = ts[i].w;
+        if ((uint32_t)(w >> 56) != sd) continue;
+        const uint64_t v = ts[i].v;
+        const long long k = (long long)A.c[j].m * do_cnt(w) + do_get(ts, 2u + j, v);
+        if (k > 0) {
+          hist_insert_global_rf(t, A.c[j].tag, v, (unsigned long long)k);
+          do_acc(acc, v, (unsigned long long)k, A.c[j].meta, A.mant_bits);
+        }
+      }
+      do_acc_fold(st[j], acc);
+    }
+    __syncthreads();
+    for (uint32_t i = tid; i < DO_TS; i += blockDim.x) { ts[i].v = 0; ts[i].w = DO_EMPTY; }
+    if (tid == 0) s_fill = 0;
+    __syncthreads();
+  };
+  const uint64_t nch = (A.ne + DO_CH - 1) / DO_CH;
+  for (uint64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
+  const uint64_t lo = ch * DO_CH, hi = lo + DO_CH < A.ne ? lo + DO_CH : A.ne;
+  for (uint64_t base = lo; base < hi; base += DO_THREADS) {
+    const uint64_t e = base + tid;
+    const bool in = e < hi;
+    // every load of the batch first (the counters of all claims, the snapshot sides), then the rest
+    uint32_t cj[DO_MAXC];
+#pragma unroll
+    for (int j = 0; j < DO_MAXC; ++j) cj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
+    uint64_t sv0 = 0, sv1 = 0;
+    if (in && A.snap[0]) sv0 = do_load(A.snap[0] + e * A.ew, A.ew);
+    if (in && A.snap[1]) sv1 = do_load(A.snap[1] + e * A.ew, A.ew);
+    uint32_t corr = 0;                                 // claims whose count differs from their base
+    bool lbit = false;
+#pragma unroll
+    for (int j = 0; j < DO_MAXC; ++j) {
+      if ((uint32_t)j >= A.nc) break;
+      if (cj[j]) { __stcs(A.c[j].cnt + e, 0u); if (A.c[j].side == 0u) lbit = true; }
+      if (in && cj[j] != A.c[j].m) corr |= 1u << j;
+    }
+    // C3: a counted pre-value load started at element e (K1 leaves these L bits to the flush)
+    const unsigned lm = __ballot_sync(0xFFFFFFFFu, lbit);
+    if (lane == 0 && lm) atomicOr(&t.L[A.bmoff + (base + (uint64_t)(tid & ~31)) / 32], lm);
+    // the groups this lane leads: bit b (0, 1: H0 of a side; 2 + j: correction of claim j), sum gd[b]
+    uint32_t pend = 0;
+    long long gd[2 + DO_MAXC];
+#pragma unroll
+    for (int sd = 0; sd < 2; ++sd) {
+      gd[sd] = 0;
+      if (!((sides >> sd) & 1u)) continue;
+      const uint64_t v = sd ? sv1 : sv0;
+      const unsigned am = __ballot_sync(0xFFFFFFFFu, in);
+      if (in) {
+        const unsigned g = __match_any_sync(am, v);
+        if (lane == __ffs(g) - 1) { pend |= 1u << sd; gd[sd] = __popc(g); }
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < DO_MAXC; ++j) gd[2 + j] = 0;
+    if (__any_sync(0xFFFFFFFFu, corr != 0u)) {         // (stencils: only at their faces)
+#pragma unroll
+      for (int j = 0; j < DO_MAXC; ++j) {
+        if ((uint32_t)j >= A.nc) break;
+        const bool act = (corr >> j) & 1u;
+        const unsigned am = __ballot_sync(0xFFFFFFFFu, act);
+        if (act) {
+          const long long d = (long long)cj[j] - (long long)A.c[j].m;
+          const uint64_t v = A.c[j].side ? sv1 : sv0;
+          const unsigned g = __match_any_sync(am, v);
+          long long sum = d;
+          if (__popc(g) > 1) {                         // group sum: a shuffle from each member
+            sum = 0;
+            for (unsigned gg = g; gg; gg &= gg - 1) sum += __shfl_sync(g, d, __ffs(gg) - 1);
+          }
+          if (lane == __ffs(g) - 1) { pend |= 1u << (2 + j); gd[2 + j] = sum; }
+        }
+      }
+    }
+    // insert the led groups.  A table generation must hold all groups of a batch (H0 and
+    // corrections of the same elements), so should one not fit (64 probes full: adversarial
+    // cardinality), the batch's inserted groups are taken out again and its counts go to the HBM
+    // table element by element instead -- exact either way
+    uint32_t done = 0;
+#pragma unroll
+    for (int b = 0; b < 2 + DO_MAXC; ++b) {
+      if (!((pend >> b) & 1u)) continue;
+      const uint64_t v = (b == 1 || (b >= 2 && A.c[b - 2].side)) ? sv1 : sv0;
+      if (do_add(ts, (uint32_t)b, v, gd[b], &s_fill)) done |= 1u << b;
+    }
+    if (__syncthreads_or(pend != done)) {
+#pragma unroll
+      for (int b = 0; b < 2 + DO_MAXC; ++b) {
+        if (!((done >> b) & 1u)) continue;
+        const uint64_t v = (b == 1 || (b >= 2 && A.c[b - 2].side)) ? sv1 : sv0;
+        do_add(ts, (uint32_t)b, v, -gd[b], &s_fill);    // present: always found
+      }
+      for (uint32_t j = 0; j < A.nc; ++j) {
+        DoAcc acc;
+        do_acc_init(acc);
+        const uint32_t c = cj[j];
+        if (c) {
+          const uint64_t v = A.c[j].side ? sv1 : sv0;
+          hist_insert_global_rf(t, A.c[j].tag, v, c);
+          do_acc(acc, v, c, A.c[j].meta, A.mant_bits);
+        }
+        do_acc_fold(st[j], acc);
+      }
+      __syncthreads();
+    }
+    if (s_fill > DO_TS * 7 / 10) drain();   // (block-uniform: read after the barrier above)
+  }
+  }
+  drain();
+  // statistics of every claim into its PC-key and object-key rows
+  if (tid < 2 * DO_MAXC) {
+    const uint32_t j = tid >> 1;
+    if (j < A.nc) {
+      const uint64_t key = (tid & 1) ? A.ko : A.c[j].kp;
+      const DoStat& S = st[j];
+      const int f[6] = {F_ZERO, F_NAN, F_NONINT, F_NF16, F_NBF16, F_NF32};
+      for (int i = 0; i < 6; ++i)
+        if (S.s[i]) atomicAdd(&t.sum[key * NSUM + f[i]], S.s[i]);
+      for (int i = 0; i < 3; ++i) {
+        if (S.mn[i] != ~0ull) atomicMin(&t.mn[key * NMM + i], S.mn[i]);
+        if (S.mx[i] != 0ull) atomicMax(&t.mx[key * NMM + i], S.mx[i]);
+      }
+    }
+  }
+}
+
+// Flush every claimed dense array into the exact histogram.  The base multiplicity m of every
+// claim is sampled first (k_dense_mode, one sync): claims read about m >= 1 times per element
+// (stencils, re-read weights) are flushed per object by k_dense_obj (H0 + corrections); claims
+// whose counts are mostly 0 (sparse or one-off reads) take the per-array k_dense_flush.
 ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   if (!c->dense_cap || !c->n_obj || !c->dense_dirty) return VE_OK;
   const size_t ns = (size_t)DENSE_PER_OBJ * c->n_obj;
@@ -1029,72 +1352,98 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   if (e == cudaSuccess) e = cudaMemcpyAsync(doff.data(), c->o.dense_off, ns * 8, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush");
-  bool any = false;
-  // (per call: the attribute belongs to the current device, and a process may drive several)
-  cudaFuncSetAttribute(k_dense_flush<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_LC_SLOTS * 12));
-  cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_SLOTS * 12));
-  cudaFuncSetAttribute(k_dense_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
-  struct Arr { uint32_t i, pc, meta; unsigned long long off; };
-  std::vector<Arr> arrs;
-  for (uint32_t i = 0; i < c->n_obj; ++i) {
+  struct Cl { uint32_t i, ck; unsigned long long off; };
+  std::vector<Cl> cl;
+  for (uint32_t i = 0; i < c->n_obj; ++i)
     for (int j = 0; j < DENSE_PER_OBJ; ++j) {
-      const uint32_t ck = dpc[DENSE_PER_OBJ * i + j];   // claim key: meta << 16 | pc
+      const uint32_t ck = dpc[DENSE_PER_OBJ * i + j];
       const unsigned long long off = doff[DENSE_PER_OBJ * i + j];
       if (ck == DENSE_FREE || ck == DENSE_OFF || off == DENSE_NOT_READY || off == DENSE_NONE) continue;
-      arrs.push_back(Arr{i, ck & 0xFFFFu, ck >> 16, off});
+      const HostObject& o = c->objs[i];
+      if (!((ck & DENSE_POST) ? o.post : o.pre)) continue;   // (claims are made only where the side exists)
+      cl.push_back(Cl{i, ck, off});
     }
-  }
-  // cardinality probes of the large arrays, one sync for all of them
-  std::vector<unsigned int> nd(arrs.size(), ~0u);
-  unsigned int* d_probe = nullptr;
-  if (!arrs.empty()) {
-    e = cudaMallocAsync((void**)&d_probe, 4 * arrs.size(), s);
-    if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush probe alloc");
-    cudaMemsetAsync(d_probe, 0xFF, 4 * arrs.size(), s);
-    bool probed = false;
-    for (size_t a = 0; a < arrs.size(); ++a) {
-      const HostObject& o = c->objs[arrs[a].i];
-      if (o.n_elems < DF_PROBE_MIN) continue;   // small arrays: the many-block path, no probe sync
-      count_launch();
-      k_dense_sample<<<1, 1024, 8192 * 8, s>>>((uint32_t*)c->dense_pool + arrs[a].off, o.n_elems,
-                                               (const uint8_t*)o.pre, o.ew, d_probe + a);
-      probed = true;
-    }
-    if (probed) {
-      e = cudaMemcpyAsync(nd.data(), d_probe, 4 * arrs.size(), cudaMemcpyDeviceToHost, s);
-      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-      if (e != cudaSuccess) { cudaFreeAsync(d_probe, s); return cuda_fail(c, e, "dense_flush probe"); }
-    }
-  }
-  for (size_t a = 0; a < arrs.size(); ++a) {
-    const HostObject& o = c->objs[arrs[a].i];
-    const uint32_t pc = arrs[a].pc, meta = arrs[a].meta;
-    uint32_t* arr = (uint32_t*)c->dense_pool + arrs[a].off;
-    // low-cardinality arrays (a sampled distinct count that fits half a large table):
-    // one persistent 1024-thread block per SM aggregates across chunks; otherwise one
-    // chunk per 256-thread block
-    const bool lc = nd[a] <= DF_LC_SLOTS / 2;
-    const uint32_t ts = lc ? DF_LC_SLOTS : (uint32_t)DF_SLOTS;
-    const size_t smem = (size_t)ts * 12;
-    uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
-    count_launch();
-    if (lc) {
-      if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
-      k_dense_flush<1024><<<(unsigned)blocks, 1024, smem, s>>>(arr, o.n_elems, (const uint8_t*)o.pre, o.ew,
-                                                              (pc << 16) | o.id, o.bmoff, c->t, meta,
-                                                              c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id, ts,
-                                                              DF_LC_CHUNK);
-    } else {
-      k_dense_flush<DF_THREADS><<<(unsigned)blocks, DF_THREADS, smem, s>>>(arr, o.n_elems, (const uint8_t*)o.pre,
-                                                                          o.ew, (pc << 16) | o.id, o.bmoff, c->t,
-                                                                          meta, c->cfg.mant_bits, pc,
-                                                                          c->cfg.n_pcs + o.id, ts, (uint32_t)DF_CHUNK);
-    }
-    any = true;
-  }
-  if (d_probe) cudaFreeAsync(d_probe, s);
   c->dense_dirty = false;      // every claimed array is read and re-zeroed by its flush
-  if (!any) return VE_OK;
+  if (cl.empty()) return VE_OK;
+  // base multiplicities
+  const size_t nc = cl.size();
+  std::vector<uint64_t> hb(2 * nc);
+  for (size_t k = 0; k < nc; ++k) {
+    hb[k] = (uint64_t)(uintptr_t)((uint32_t*)c->dense_pool + cl[k].off);
+    hb[nc + k] = c->objs[cl[k].i].size / c->objs[cl[k].i].ew;
+  }
+  void* dm = nullptr;
+  e = cudaMallocAsync(&dm, 2 * nc * 8 + nc * 4, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush alloc");
+  std::vector<uint32_t> mh(nc);
+  cudaMemcpyAsync(dm, hb.data(), 2 * nc * 8, cudaMemcpyHostToDevice, s);
+  count_launch();
+  k_dense_mode<<<(unsigned)nc, 32, 0, s>>>((const uint32_t* const*)dm, (const uint64_t*)dm + nc,
+                                          (uint32_t*)((uint8_t*)dm + 2 * nc * 8));
+  // and the cardinality of each claim's side values (the H0 table holds ~DO_TS * 0.7 distinct values)
+  unsigned int* dnd = (unsigned int*)((uint8_t*)dm + 2 * nc * 8);   // (reuses nothing: a second buffer below)
+  (void)dnd;
+  std::vector<unsigned int> nd(nc, ~0u);
+  unsigned int* d_probe = nullptr;
+  e = cudaMallocAsync((void**)&d_probe, 4 * nc, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush probe alloc");
+  cudaFuncSetAttribute(k_dense_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
+  for (size_t k = 0; k < nc; ++k) {
+    const HostObject& o = c->objs[cl[k].i];
+    count_launch();
+    k_dense_sample<<<1, 1024, 8192 * 8, s>>>((uint32_t*)c->dense_pool + cl[k].off, o.n_elems,
+                                             (const uint8_t*)((cl[k].ck & DENSE_POST) ? o.post : o.pre), o.ew,
+                                             d_probe + k);
+  }
+  cudaMemcpyAsync(mh.data(), (uint8_t*)dm + 2 * nc * 8, nc * 4, cudaMemcpyDeviceToHost, s);
+  cudaMemcpyAsync(nd.data(), d_probe, 4 * nc, cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(dm, s);
+  cudaFreeAsync(d_probe, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "k_dense_mode");
+  const size_t smem = (size_t)DO_TS * sizeof(DoSlot);
+  cudaFuncSetAttribute(k_dense_obj, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_SLOTS * 12));
+  for (uint32_t i = 0; i < c->n_obj; ++i) {
+    const HostObject& o = c->objs[i];
+    DoArgs A;
+    memset(&A, 0, sizeof(A));
+    for (size_t k = 0; k < nc; ++k) {
+      if (cl[k].i != i) continue;
+      const uint32_t ck = cl[k].ck, pc = ck & 0xFFFFu, meta = (ck >> 16) & 0x3Fu;
+      const bool post = (ck & DENSE_POST) != 0u;
+      uint32_t* arr = (uint32_t*)c->dense_pool + cl[k].off;
+      if (mh[k] == 0u || nd[k] > 4096u) {   // mostly unread elements, or many values: per-array flush
+        const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
+        count_launch();
+        k_dense_flush<DF_THREADS><<<(unsigned)blocks, DF_THREADS, DF_SLOTS * 12, s>>>(
+            arr, o.n_elems, (const uint8_t*)(post ? o.post : o.pre), o.ew, (pc << 16) | o.id, o.bmoff, c->t, meta,
+            c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id, (uint32_t)DF_SLOTS, (uint32_t)DF_CHUNK, post ? 0u : 1u);
+        continue;
+      }
+      DoClaim& d = A.c[A.nc++];
+      d.cnt = arr;
+      d.meta = meta;
+      d.side = post ? 1u : 0u;
+      d.tag = (pc << 16) | (o.id & 0xFFFFu);
+      d.kp = pc;
+      d.m = mh[k];
+      A.snap[d.side] = (const uint8_t*)(post ? o.post : o.pre);
+    }
+    if (!A.nc) continue;
+    A.ew = o.ew;
+    A.ko = c->cfg.n_pcs + o.id;
+    A.mant_bits = c->cfg.mant_bits;
+    A.ne = o.size / o.ew;                  // whole elements (K1 counts only those)
+    A.bmoff = o.bmoff;
+    uint64_t blocks = (A.ne + DO_CH - 1) / DO_CH;
+    if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+    if (blocks == 0) blocks = 1;
+    count_launch();
+    k_dense_obj<<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t);
+  }
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "dense flush launch");
   unsigned long long glob[8];
   e = cudaMemcpyAsync(glob, c->t.glob, sizeof(glob), cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);

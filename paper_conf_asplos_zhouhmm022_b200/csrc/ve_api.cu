@@ -287,12 +287,14 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
                                                           : (1ull << 31);
   c->dense_pc_init.assign((size_t)DENSE_PER_OBJ * n, DENSE_OFF);
   uint64_t want = 0;
+  uint64_t pre_elems = 0;
   for (uint32_t i = 0; i < n; ++i) {
-    if (!v[i].pre) continue;
+    if (!v[i].pre && !v[i].post) continue;
     for (int j = 0; j < DENSE_PER_OBJ; ++j) c->dense_pc_init[DENSE_PER_OBJ * i + j] = DENSE_FREE;
     want += DENSE_PER_OBJ * v[i].n_elems;
+    if (v[i].pre) pre_elems += v[i].n_elems;
   }
-  c->pre_elems = want / DENSE_PER_OBJ;
+  c->pre_elems = pre_elems;
   if (want > DENSE_BUDGET) want = DENSE_BUDGET;
   if (want > c->dense_cap) {
     if (c->dense_pool) {
@@ -315,7 +317,7 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   // device object table (SoA, sorted by base); the block is reused when it is large
   // enough (after the device is idle: earlier launches may still read the old table)
   const size_t nn = n ? n : 1;
-  const size_t nb = nn * (8 * 4 + 8 * DENSE_PER_OBJ + 4 * 2 + 4 * DENSE_PER_OBJ) + 64;
+  const size_t nb = nn * (8 * 5 + 8 * DENSE_PER_OBJ + 4 * 2 + 4 * DENSE_PER_OBJ) + 64;
   if (nb > c->obj_block_bytes) {
     cudaFree(c->obj_block);
     c->obj_block = nullptr;
@@ -330,13 +332,14 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   uint64_t* he = hb + n;
   uint64_t* hp = he + n;
   uint64_t* hm = hp + n;
-  uint64_t* hdo = hm + n;
+  uint64_t* hq = hm + n;
+  uint64_t* hdo = hq + n;
   uint32_t* hid = (uint32_t*)(hdo + DENSE_PER_OBJ * n);
   uint32_t* hew = hid + n;
   uint32_t* hdp = hew + n;
   c->sorted_of_id.assign(n, 0);
   for (uint32_t i = 0; i < n; ++i) {
-    hb[i] = v[i].base; he[i] = v[i].base + v[i].size; hp[i] = v[i].pre; hm[i] = v[i].bmoff;
+    hb[i] = v[i].base; he[i] = v[i].base + v[i].size; hp[i] = v[i].pre; hm[i] = v[i].bmoff; hq[i] = v[i].post;
     hid[i] = v[i].id; hew[i] = v[i].ew;
     c->sorted_of_id[v[i].id] = i;
   }
@@ -347,8 +350,9 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   c->o.end = db + n;
   c->o.pre = db + 2 * n;
   c->o.bmoff = db + 3 * n;
-  c->o.dense_off = (unsigned long long*)(db + 4 * n);
-  c->o.id = (const uint32_t*)(db + 4 * n + DENSE_PER_OBJ * n);
+  c->o.post = db + 4 * n;
+  c->o.dense_off = (unsigned long long*)(db + 5 * n);
+  c->o.id = (const uint32_t*)(db + 5 * n + DENSE_PER_OBJ * n);
   c->o.ew = c->o.id + n;
   c->o.dense_pc = const_cast<uint32_t*>(c->o.ew + n);
   c->o.dense_pool = (uint32_t*)c->dense_pool;

@@ -71,6 +71,7 @@ struct DevObjects {          // sorted by base
   const uint32_t* id;
   const uint32_t* ew;
   const uint64_t* pre;       // device pointers as integers (0 = none)
+  const uint64_t* post;      // post snapshot (0 = none)
   const uint64_t* bmoff;     // first bitmap word of the object
   // dense per-element access counters for loads that read the pre value: up to
   // DENSE_PER_OBJ arrays per object, each claimed by one (pc, access type):
@@ -89,6 +90,10 @@ constexpr uint32_t DENSE_OFF = 0xFFFFFFFEu;
 constexpr unsigned long long DENSE_NOT_READY = ~0ull;
 constexpr unsigned long long DENSE_NONE = ~1ull;
 constexpr int DENSE_PER_OBJ = 8;
+// A claim key is meta << 16 | pc; DENSE_POST marks an array that counts records whose value equals the
+// POST snapshot's element (records that read a value written earlier by the same API call, and stores
+// of an element's final value): their histogram entry is that post value (K1 v2 claims these)
+constexpr uint32_t DENSE_POST = 1u << 31;
 constexpr int G_DENSE_NEXT = 4;   // glob slot of the dense pool cursor
 
 // ---- host-side context ------------------------------------------------------
