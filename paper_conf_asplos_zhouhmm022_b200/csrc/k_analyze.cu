@@ -1862,8 +1862,14 @@ struct SlotLine {            // deferred C8 constant segment of slot s (see Slot
   uint64_t cy, cx0, cx1;
   uint32_t cpend, pad;
 };
+struct SlotRec {             // slot s's object and arrays (per warp, shared memory; read by every lane)
+  uint64_t cb, clim, cpre, cpost, cbm;
+  unsigned long long dn, dq;
+  uint32_t cidlg, coi;       // object id | log2 element width << 16 (every register of the object is restored); sorted index
+};
 struct LaneSlot {            // the registers of lane s that hold slot s
   uint64_t key;              // meta << 32 | object id << 16 | pc; ~0 = free
+  uint64_t pmw, ob, olim;    // pc | meta << 32, and the object's range [ob, ob + olim] (the hit test)
   unsigned long long dn;     // dense counter array of (pc, object) loads that read the pre value, or 0
   unsigned long long dq;     // dense counter array of records that carry the post value (DENSE_POST), or 0
   uint32_t info;             // bits 0-1: line FAIL (PC key, object key); bit 2: object has no pre snapshot
@@ -2142,16 +2148,16 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
     if (tid < 4) S.sctr[tid] = 0;
     if (tid < K1_WARPS - K2_WARPS) P.stage_cnt[(uint64_t)blockIdx.x * K1_WARPS + K2_WARPS + tid] = 0;
   }
-  __shared__ WarpCache s_wc[K1_WARPS];
-  __shared__ SlotLine s_sl[K1_WARPS][NS2];
-  __shared__ SlotSave s_save[K1_WARPS];
+  __shared__ WarpCache s_wc[K2_WARPS];
+  __shared__ SlotLine s_sl[K2_WARPS][NS2];
+  __shared__ SlotSave s_save[K2_WARPS];
   WarpCache& wc = s_wc[warp];
   SlotLine* sl = s_sl[warp];
   if (lane < WC) wc.key1[lane] = 0;
   sl[lane].cpend = 0;
   if (lane == 0) { wc.next = 0; s_stage_n[warp] = 0; }
   LaneSlot L;
-  L.key = ~0ull; L.dn = 0; L.dq = 0; L.info = 0;
+  L.key = ~0ull; L.pmw = ~0ull; L.ob = 1; L.olim = 0; L.dn = 0; L.dq = 0; L.info = 0;
   lslot_clear_acc(L);
   uint32_t snext = 0;
 
@@ -2238,28 +2244,51 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
     }
     obj_set(oi);
   };
-  // the key of the current slot: kpm = its (pc | meta << 32) word, klg its access width, kwm / kvm
-  // the alignment and value-bit masks; a window continues it when every lane carries kpm, lies in
-  // the current object at an aligned element and has no value bits above its width
-  uint64_t kpm = ~0ull, kvm = 0;
+  // Slot s also holds, in lane s's registers, its (pc | meta << 32) word pmw and its object's range
+  // [ob, ob + olim]; its object / array data sits in the warp's shared-memory record sr[s].  A window
+  // whose lane 0 carries (pmw, an address in that range) is found by ONE ballot; the registers below
+  // hold the data of the slot ls used last, so runs of one key reload nothing.
+  __shared__ SlotRec s_rec[K2_WARPS][NS2];
+  SlotRec* const sr = s_rec[warp];
+  uint64_t kvm = 0, kkey = ~0ull;
   uint32_t kwm = 0, klg = 0;
-  uint64_t kkey = ~0ull;
-  int s = 0;
+  int s = 0, ls = -1;
 
   while (R.left) {
     uint64_t addr, val, pm;
     ring_next(P, R, addr, val, pm);
-    const uint64_t off = addr - cb;
-    if (!__all_sync(FULL, pm == kpm && off <= clim && ((uint32_t)off & kwm) == 0u && (val & kvm) == val)) {
-      // another key, another object, or a window for the slow path
-      const uint64_t pm0 = shfl64(FULL, pm, 0);
+    const uint64_t pm0 = shfl64(FULL, pm, 0);
+    const uint64_t a0 = shfl64(FULL, addr, 0);
+    const unsigned hit = __ballot_sync(FULL, L.pmw == pm0 && a0 - L.ob <= L.olim);
+    bool ok = false;
+    if (hit) {
+      s = __ffs(hit) - 1;
+      if (s != ls) {
+        ls = s;
+        const SlotRec& r = sr[s];
+        cb = r.cb; clim = r.clim; cpre = r.cpre; cpost = r.cpost; cbm = r.cbm; ldn = r.dn; ldq = r.dq;
+        cid = r.cidlg & 0xFFFFu; coi = (int)r.coi; clg = r.cidlg >> 16;
+        kkey = ((uint64_t)(uint32_t)(pm0 >> 32) << 32) | ((uint64_t)cid << 16) | (uint32_t)pm0;
+        klg = (uint32_t)(pm0 >> 32) & 3u;
+        kwm = (1u << klg) - 1u;
+        kvm = klg == 3u ? 0ull : ~((1ull << (8u << klg)) - 1ull);
+        const uint32_t inf = __shfl_sync(FULL, L.info, s);
+        llf = inf & 3u;
+        lpt = (inf >> 3) & 1u;
+      }
+      const uint64_t o = addr - cb;
+      ok = __all_sync(FULL, pm == pm0 && o <= clim && ((uint32_t)o & kwm) == 0u && (val & kvm) == 0ull);
+    }
+    if (!ok) {
+      // another key or object, or a window for the slow path
       const uint32_t meta0 = (uint32_t)(pm0 >> 32), pc0 = (uint32_t)pm0;
       bool fast = false;
       if (__all_sync(FULL, pm == pm0) && meta_fast(meta0, pc0, P.n_pcs)) {
         const uint32_t lg0 = meta0 & 3u;
         const uint64_t wm = (1ull << lg0) - 1ull;
         const bool vok = lg0 == 3u || (val >> (8u << lg0)) == 0ull;
-        obj_find(shfl64(FULL, addr, 0));
+        ls = -1;                                     // the object registers change
+        obj_find(a0);
         const uint64_t o = addr - cb;
         fast = lg0 == clg && __all_sync(FULL, vok && o <= clim && (o & wm) == 0ull);
       }
@@ -2267,53 +2296,58 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
         const uint32_t cnt = slow_window(P, wc, addr, val, pm, true);
         n_inv += cnt & 0xFFFFu;
         n_unm += cnt >> 16;
-        kpm = ~0ull;          // (the object may have changed under the key)
         continue;
       }
       const uint64_t key = ((uint64_t)meta0 << 32) | ((uint64_t)cid << 16) | pc0;
-      if (key != kkey) {
-        const unsigned hit = __ballot_sync(FULL, L.key == key);
-        if (hit) {
-          s = __ffs(hit) - 1;
-        } else {
-          const unsigned fr = __ballot_sync(FULL, L.key == ~0ull);
-          const bool evict = fr == 0u;
-          s = evict ? (int)(snext++ & 31u) : __ffs(fr) - 1;
-          const uint64_t vk = shfl64(FULL, L.key, s);
-          const uint32_t vlf = __shfl_sync(FULL, L.info, s) & 3u;
-          uint32_t nlf;
-          unsigned long long dq;
-          const unsigned long long dn = lslot_prepare(P, wc, sl, s, evict, vk, vlf, key, coi, cpre == 0ull,
-                                                      cpost != 0ull, &nlf, &dq);
-          if (evict) {
-            if (lane == s) lslot_save(&s_save[warp], L);
-            lslot_fold(P, &s_save[warp]);
-          }
-          if (lane == s) {
-            L.key = key;
-            L.dn = dn;
-            L.dq = dq;
-            L.info = nlf | (cpre == 0ull ? 4u : 0u);
-            lslot_clear_acc(L);
-          }
+      const unsigned kh = __ballot_sync(FULL, L.key == key);
+      if (kh) {
+        s = __ffs(kh) - 1;
+      } else {
+        const unsigned fr = __ballot_sync(FULL, L.key == ~0ull);
+        const bool evict = fr == 0u;
+        s = evict ? (int)(snext++ & 31u) : __ffs(fr) - 1;
+        const uint64_t vk = shfl64(FULL, L.key, s);
+        const uint32_t vlf = __shfl_sync(FULL, L.info, s) & 3u;
+        uint32_t nlf;
+        unsigned long long dq;
+        const unsigned long long dn = lslot_prepare(P, wc, sl, s, evict, vk, vlf, key, coi, cpre == 0ull,
+                                                    cpost != 0ull, &nlf, &dq);
+        if (evict) {
+          if (lane == s) lslot_save(&s_save[warp], L);
+          lslot_fold(P, &s_save[warp]);
         }
-        kkey = key;
-        ldn = shfl64(FULL, L.dn, s);
-        ldq = shfl64(FULL, L.dq, s);
-        lpt = (__shfl_sync(FULL, L.info, s) >> 3) & 1u;
-        llf = __shfl_sync(FULL, L.info, s) & 3u;
+        if (lane == s) {
+          L.key = key;
+          L.pmw = pm0;
+          L.ob = cb;
+          L.olim = clim;
+          L.dn = dn;
+          L.dq = dq;
+          L.info = nlf | (cpre == 0ull ? 4u : 0u);
+          lslot_clear_acc(L);
+          SlotRec& r = sr[s];
+          r.cb = cb; r.clim = clim; r.cpre = cpre; r.cpost = cpost; r.cbm = cbm; r.dn = dn; r.dq = dq;
+          r.cidlg = (cid & 0xFFFFu) | (clg << 16); r.coi = (uint32_t)coi;
+        }
+        __syncwarp();
       }
-      kpm = pm0;
+      ls = s;
+      kkey = key;
+      ldn = shfl64(FULL, L.dn, s);
+      ldq = shfl64(FULL, L.dq, s);
+      const uint32_t inf = __shfl_sync(FULL, L.info, s);
+      llf = inf & 3u;
+      lpt = (inf >> 3) & 1u;
       klg = meta0 & 3u;
       kwm = (1u << klg) - 1u;
-      kvm = klg == 3u ? ~0ull : ((1ull << (8u << klg)) - 1ull);
+      kvm = klg == 3u ? 0ull : ~((1ull << (8u << klg)) - 1ull);
     }
-    // a fast window of the current key in the current object
+    // a fast window of slot s (its object in cb ..)
     const uint64_t o = addr - cb;
     uint64_t pv = 0, qv = 0;
     if (cpre != 0ull) pv = ld_pre<3>((cpre + o) & ~7ull) >> (8u * (uint32_t)((cpre + o) & 7ull));
     if (ldq != 0ull) qv = ld_pre<3>((cpost + o) & ~7ull) >> (8u * (uint32_t)((cpost + o) & 7ull));
-    const uint32_t meta0 = (uint32_t)(kpm >> 32), pc0 = (uint32_t)kpm;
+    const uint32_t meta0 = (uint32_t)(kkey >> 32), pc0 = (uint32_t)kkey & 0xFFFFu;
     bool wantq = false;
     switch (klg) {
       case 0: wantq = win_fast<0>(P, L, s, meta0, pc0, cid, cpre, cbm, o, val, pv, ldn, qv, ldq); break;
@@ -2324,7 +2358,8 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
     if (wantq && !lpt && cpost != 0ull && P.dense_ok) {       // first value-path window of the key
       lpt = true;
       ldq = post_claim(P, coi, kkey);
-      if (lane == s) { L.dq = ldq; L.info |= 8u; }
+      if (lane == s) { L.dq = ldq; L.info |= 8u; sr[s].dq = ldq; }
+      __syncwarp();
     }
     // (no overflow check: a launch gives a warp < 2^31 records, so the 32-bit accumulators hold)
     if (llf != 3u) {
