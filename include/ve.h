@@ -146,6 +146,28 @@ ve_status ve_snapshot_diff(ve_ctx* ctx, uint32_t obj_id, uint32_t mode, const ui
 ve_status ve_object_dedup(ve_ctx* ctx, const ve_object* objs, uint32_t n, uint32_t* h_group_of,
                           cudaStream_t s);
 
+/* S10 / S11 sharded by memory object (the paper claims
+ * multi-GPU support without a mechanism).  Every rank holds the same
+ * objects (after ve_merge_stats the W / L bitmaps are merged).
+ *   ve_snapshot_diff_all: C10 of EVERY object with both snapshots, mode
+ *     VE_DIFF_WRITTEN or VE_DIFF_ALL; the object at position k of the sorted
+ *     object table is diffed by rank k mod G, the partial results are
+ *     SUM-allreduced: h_out[id] (n_objects entries, indexed by object id;
+ *     objects without both snapshots report n_elems only).  nccl_comm NULL: one
+ *     rank (every object diffed locally).  Synchronizes s.
+ *   ve_object_dedup_comm: C11 over NCCL: eligible object k is hashed by rank
+ *     k mod G (hashes SUM-allreduced), candidate pair p is byte-verified by rank
+ *     p mod G (flags SUM-allreduced); every rank gets the full h_group_of.
+ *     Objects' post snapshots must be readable on every rank.  Synchronizes s.
+ *   ..._group: the same algorithms with n contexts on one device playing ranks
+ *     0..n-1 (device copies instead of NCCL; the tests' transport). */
+ve_status ve_snapshot_diff_all(ve_ctx* ctx, uint32_t mode, void* nccl_comm_or_null, ve_diff* h_out, cudaStream_t s);
+ve_status ve_object_dedup_comm(ve_ctx* ctx, const ve_object* objs, uint32_t n, void* nccl_comm, uint32_t* h_group_of,
+                               cudaStream_t s);
+ve_status ve_snapshot_diff_all_group(ve_ctx** ctxs, uint32_t n, uint32_t mode, ve_diff* h_out, cudaStream_t s);
+ve_status ve_object_dedup_group(ve_ctx** ctxs, uint32_t n, const ve_object* objs, uint32_t n_objs,
+                                uint32_t* h_group_of, cudaStream_t s);
+
 /* S12 / C12: merge statistics.  src != NULL: dst <- dst (+) src on one device
  * (same config and object table).  nccl_comm != NULL (an ncclComm_t over all
  * ranks, each holding a ctx with the same config/objects): every rank ends

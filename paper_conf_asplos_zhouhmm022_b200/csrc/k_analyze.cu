@@ -2510,9 +2510,10 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   // (VE_K1_MULTI=0/1 forces one instantiation: the parity tests run both on the same traces)
   const char* fm = getenv("VE_K1_MULTI");
   const bool multi = VE_MULTI_DENSE && (fm && *fm ? *fm == '1' : c->cfg.n_pcs >= VE_MULTI_MIN_PCS);
-  // K1 v2 (register key slots) unless VE_K1=1 selects the v1 kernels
+  // K1 v2 (register key slots, post-value counting) for traces of many PCs, whose windows alternate
+  // keys; v1 (single-key runs, stage-batched dense gathers) for few PCs.  VE_K1=1 / 2 forces one.
   const char* kv = getenv("VE_K1");
-  const bool v2 = !(kv && *kv == '1');
+  const bool v2 = (kv && *kv) ? *kv == '2' : c->cfg.n_pcs >= VE_MULTI_MIN_PCS;
   auto kfn = v2 ? k_analyze2 : multi ? k_analyze<true> : k_analyze<false>;
   cudaFuncGetAttributes(&fa, kfn);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring

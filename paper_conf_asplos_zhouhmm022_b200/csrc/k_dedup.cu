@@ -76,12 +76,12 @@ struct CmpJob {
 };
 
 // K8: bytewise verification of (member, representative) pairs, 256 KiB per CTA
-__global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned int* differs) {
+__global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned long long* differs) {
   const CmpJob jb = jobs[blockIdx.x];
   // early exit when another chunk of the pair already differs: decided once per block (thread 0
   // reads the flag) so every thread takes the same branch before __syncthreads_or below
   __shared__ unsigned int s_skip;
-  if (threadIdx.x == 0) s_skip = *(volatile unsigned int*)&differs[jb.pair];
+  if (threadIdx.x == 0) s_skip = *(volatile unsigned long long*)&differs[jb.pair] != 0ull;
   __syncthreads();
   if (s_skip) return;
   bool diff = false;
@@ -108,90 +108,122 @@ __global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned in
   } else {
     for (uint64_t k = threadIdx.x; k < jb.len; k += blockDim.x) diff |= a[k] != b[k];
   }
-  if (__syncthreads_or(diff) && threadIdx.x == 0) atomicOr(&differs[jb.pair], 1u);
+  if (__syncthreads_or(diff) && threadIdx.x == 0) atomicOr(&differs[jb.pair], 1ull);
 }
 
-ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* group_of, cudaStream_t s) {
+// K7 of the eligible objects k (positions in elig) with k mod G == rank into d_hash[k]
+static void hash_launch(ve_ctx* c, const ve_object* objs, const std::vector<uint32_t>& elig, int G, int rank,
+                        HashJob* d_jobs, std::vector<HashJob>& hj, unsigned long long* d_hash, cudaStream_t s) {
+  hj.clear();
+  std::vector<uint32_t> pos;
+  uint64_t maxsz = 0;
+  for (size_t k = 0; k < elig.size(); ++k) {
+    if ((int)(k % G) != rank) continue;
+    hj.push_back(HashJob{(const uint8_t*)objs[elig[k]].post, objs[elig[k]].size});
+    pos.push_back((uint32_t)k);
+    maxsz = std::max<uint64_t>(maxsz, objs[elig[k]].size);
+  }
+  if (hj.empty()) return;
+  // a rank's owned objects are not contiguous in elig: hash into a compact array, then scatter
+  cudaMemcpyAsync(d_jobs, hj.data(), hj.size() * sizeof(HashJob), cudaMemcpyHostToDevice, s);
+  unsigned long long* d_tmp = d_hash + elig.size();
+  cudaMemsetAsync(d_tmp, 0, hj.size() * 8, s);
+  // grid.x: ~256 KiB of the largest object per CTA (16 KiB per CTA-iteration, 4 loads deep),
+  // at least two CTAs per SM over the whole set
+  uint64_t gx = (maxsz + (256u << 10) - 1) / (256u << 10);
+  const uint64_t want = (2ull * c->num_sms + hj.size() - 1) / hj.size();
+  gx = std::min<uint64_t>(std::max<uint64_t>(std::max<uint64_t>(gx, want), 1), 1024);
+  for (size_t y0 = 0; y0 < hj.size(); y0 += 65535) {
+    const unsigned gy = (unsigned)std::min<size_t>(65535, hj.size() - y0);
+    count_launch();
+    k_hash<<<dim3((unsigned)gx, gy), 256, 0, s>>>(d_jobs + y0, d_tmp + y0);
+  }
+  for (size_t q = 0; q < pos.size(); ++q)      // (small: one 8-byte copy per owned object)
+    cudaMemcpyAsync(d_hash + pos[q], d_tmp + q, 8, cudaMemcpyDeviceToDevice, s);
+}
+
+ve_status dedup_ranks(const std::vector<ve_ctx*>& cs, Comm& comm, const ve_object* objs, uint32_t n,
+                      uint32_t* group_of, cudaStream_t s) {
+  ve_ctx* c0 = cs[0];
+  const int G = comm.G;
   for (uint32_t i = 0; i < n; ++i) group_of[i] = objs[i].id;
   std::vector<uint32_t> elig;
   for (uint32_t i = 0; i < n; ++i)
     if (objs[i].size > 0 && objs[i].post) elig.push_back(i);
   if (elig.size() < 2) return VE_OK;
-  // K7: content hash of every eligible object
-  std::vector<HashJob> hj(elig.size());
-  uint64_t maxsz = 0;
-  for (size_t k = 0; k < elig.size(); ++k) {
-    hj[k] = HashJob{(const uint8_t*)objs[elig[k]].post, objs[elig[k]].size};
-    maxsz = std::max<uint64_t>(maxsz, objs[elig[k]].size);
+  const size_t ne = elig.size();
+  // K7 on the owned objects, then a SUM allreduce: every rank holds every hash
+  std::vector<void*> hb(cs.size());
+  std::vector<void*> jb(cs.size());
+  std::vector<HashJob> hj;
+  for (size_t i = 0; i < cs.size(); ++i) {
+    cudaError_t e = cudaMallocAsync(&hb[i], 2 * ne * 8, s);
+    if (e == cudaSuccess) e = cudaMallocAsync(&jb[i], ne * sizeof(HashJob), s);
+    if (e != cudaSuccess) return cuda_fail(c0, e, "dedup alloc");
+    cudaMemsetAsync(hb[i], 0, ne * 8, s);
+    hash_launch(cs[i], objs, elig, G, comm.local[i], (HashJob*)jb[i], hj, (unsigned long long*)hb[i], s);
+    // (hj is reused by the next rank only after this rank's H2D copy is ordered on s)
+    cudaStreamSynchronize(s);
   }
-  void* d = nullptr;
-  const size_t nb = hj.size() * (sizeof(HashJob) + 8);
-  cudaError_t e = cudaMallocAsync(&d, nb, s);
-  if (e != cudaSuccess) return cuda_fail(c, e, "dedup alloc");
-  HashJob* d_jobs = (HashJob*)d;
-  unsigned long long* d_hash = (unsigned long long*)((uint8_t*)d + hj.size() * sizeof(HashJob));
-  cudaMemcpyAsync(d_jobs, hj.data(), hj.size() * sizeof(HashJob), cudaMemcpyHostToDevice, s);
-  cudaMemsetAsync(d_hash, 0, hj.size() * 8, s);
-  // grid.x: ~256 KiB of the largest object per CTA (16 KiB per CTA-iteration, 4 loads deep),
-  // at least two CTAs per SM over the whole set
-  uint64_t gx = (maxsz + (256u << 10) - 1) / (256u << 10);
-  const uint64_t want = (2ull * c->num_sms + elig.size() - 1) / elig.size();
-  gx = std::min<uint64_t>(std::max<uint64_t>(std::max<uint64_t>(gx, want), 1), 1024);
-  for (size_t y0 = 0; y0 < hj.size(); y0 += 65535) {
-    const unsigned gy = (unsigned)std::min<size_t>(65535, hj.size() - y0);
-    count_launch();
-    k_hash<<<dim3((unsigned)gx, gy), 256, 0, s>>>(d_jobs + y0, d_hash + y0);
-  }
-  std::vector<unsigned long long> h(hj.size());
-  cudaMemcpyAsync(h.data(), d_hash, hj.size() * 8, cudaMemcpyDeviceToHost, s);
-  cudaFreeAsync(d, s);
-  e = cudaStreamSynchronize(s);
-  if (e != cudaSuccess) return cuda_fail(c, e, "dedup hash");
+  if (!comm.allreduce(hb, ne, OP_SUM, s)) return fail(c0, VE_ERR_NCCL, "dedup hash allreduce: " + comm.err);
+  std::vector<unsigned long long> h(ne);
+  cudaMemcpyAsync(h.data(), hb[0], ne * 8, cudaMemcpyDeviceToHost, s);
+  for (size_t i = 0; i < cs.size(); ++i) { cudaFreeAsync(hb[i], s); cudaFreeAsync(jb[i], s); }
+  cudaError_t e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c0, e, "dedup hash");
 
-  // candidate groups: equal (size, hash); members ordered by id
+  // candidate groups: equal (size, hash); members ordered by id (the same on every rank)
   std::map<std::pair<uint64_t, uint64_t>, std::vector<uint32_t>> groups;
-  for (size_t k = 0; k < elig.size(); ++k) groups[{objs[elig[k]].size, h[k]}].push_back(elig[k]);
+  for (size_t k = 0; k < ne; ++k) groups[{objs[elig[k]].size, h[k]}].push_back(elig[k]);
   std::vector<std::vector<uint32_t>> pending;
   for (auto& g : groups) {
     if (g.second.size() < 2) continue;
     std::sort(g.second.begin(), g.second.end(), [&](uint32_t a, uint32_t b) { return objs[a].id < objs[b].id; });
     pending.push_back(g.second);
   }
-  // K8: verify against the representative (lowest id); mismatches form a new pending group
+  // K8: verify every member against its class representative (lowest id); pair p is checked by rank
+  // p mod G, the flags are SUM-allreduced; mismatches form a new pending group
   const uint64_t CH = 1 << 18;   // 256 KiB per verification CTA
   while (!pending.empty()) {
-    std::vector<CmpJob> jobs;
     std::vector<std::pair<uint32_t, uint32_t>> pairs;  // (group index, member index)
-    for (uint32_t gi = 0; gi < pending.size(); ++gi) {
-      const auto& g = pending[gi];
-      const ve_object& rep = objs[g[0]];
-      for (uint32_t mi = 1; mi < g.size(); ++mi) {
-        const ve_object& m = objs[g[mi]];
-        const uint32_t pid = (uint32_t)pairs.size();
-        pairs.push_back({gi, mi});
+    for (uint32_t gi = 0; gi < pending.size(); ++gi)
+      for (uint32_t mi = 1; mi < pending[gi].size(); ++mi) pairs.push_back({gi, mi});
+    const size_t np = pairs.size();
+    std::vector<void*> db(cs.size());
+    for (size_t i = 0; i < cs.size(); ++i) {
+      std::vector<CmpJob> jobs;
+      for (size_t p = 0; p < np; ++p) {
+        if ((int)(p % G) != comm.local[i]) continue;
+        const auto& g = pending[pairs[p].first];
+        const ve_object& rep = objs[g[0]];
+        const ve_object& m = objs[g[pairs[p].second]];
         for (uint64_t off = 0; off < m.size; off += CH)
-          jobs.push_back(CmpJob{(const uint8_t*)m.post, (const uint8_t*)rep.post, off, std::min(CH, m.size - off), pid, 0});
+          jobs.push_back(CmpJob{(const uint8_t*)m.post, (const uint8_t*)rep.post, off, std::min(CH, m.size - off),
+                                (uint32_t)p, 0});
       }
+      e = cudaMallocAsync(&db[i], np * 8 + jobs.size() * sizeof(CmpJob), s);
+      if (e != cudaSuccess) return cuda_fail(c0, e, "dedup verify alloc");
+      unsigned long long* d_diff = (unsigned long long*)db[i];
+      CmpJob* d_cj = (CmpJob*)((uint8_t*)db[i] + np * 8);
+      cudaMemsetAsync(d_diff, 0, np * 8, s);
+      if (!jobs.empty()) {
+        cudaMemcpyAsync(d_cj, jobs.data(), jobs.size() * sizeof(CmpJob), cudaMemcpyHostToDevice, s);
+        for (size_t j0 = 0; j0 < jobs.size(); j0 += (1u << 30)) {
+          const unsigned gxx = (unsigned)std::min<size_t>(jobs.size() - j0, 1u << 30);
+          count_launch();
+          k_compare<<<gxx, 256, 0, s>>>(d_cj + j0, d_diff);
+        }
+      }
+      cudaStreamSynchronize(s);   // (jobs is a host vector of this iteration)
     }
-    void* dd = nullptr;
-    e = cudaMallocAsync(&dd, jobs.size() * sizeof(CmpJob) + pairs.size() * 4, s);
-    if (e != cudaSuccess) return cuda_fail(c, e, "dedup verify alloc");
-    CmpJob* d_cj = (CmpJob*)dd;
-    unsigned int* d_diff = (unsigned int*)((uint8_t*)dd + jobs.size() * sizeof(CmpJob));
-    cudaMemcpyAsync(d_cj, jobs.data(), jobs.size() * sizeof(CmpJob), cudaMemcpyHostToDevice, s);
-    cudaMemsetAsync(d_diff, 0, pairs.size() * 4, s);
-    for (size_t j0 = 0; j0 < jobs.size(); j0 += (1u << 30)) {
-      const unsigned gxx = (unsigned)std::min<size_t>(jobs.size() - j0, 1u << 30);
-      count_launch();
-      k_compare<<<gxx, 256, 0, s>>>(d_cj + j0, d_diff);
-    }
-    std::vector<unsigned int> diff(pairs.size());
-    cudaMemcpyAsync(diff.data(), d_diff, pairs.size() * 4, cudaMemcpyDeviceToHost, s);
-    cudaFreeAsync(dd, s);
+    if (!comm.allreduce(db, np, OP_SUM, s)) return fail(c0, VE_ERR_NCCL, "dedup verify allreduce: " + comm.err);
+    std::vector<unsigned long long> diff(np);
+    cudaMemcpyAsync(diff.data(), db[0], np * 8, cudaMemcpyDeviceToHost, s);
+    for (size_t i = 0; i < cs.size(); ++i) cudaFreeAsync(db[i], s);
     e = cudaStreamSynchronize(s);
-    if (e != cudaSuccess) return cuda_fail(c, e, "dedup verify");
+    if (e != cudaSuccess) return cuda_fail(c0, e, "dedup verify");
     std::vector<std::vector<uint32_t>> next(pending.size());
-    for (size_t p = 0; p < pairs.size(); ++p) {
+    for (size_t p = 0; p < np; ++p) {
       const auto& g = pending[pairs[p].first];
       const uint32_t mem = g[pairs[p].second];
       if (!diff[p]) group_of[mem] = objs[g[0]].id;
@@ -202,6 +234,11 @@ ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* grou
       if (g.size() >= 2) pending.push_back(g);
   }
   return VE_OK;
+}
+
+ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* group_of, cudaStream_t s) {
+  LocalComm one;
+  return dedup_ranks({c}, one, objs, n, group_of, s);
 }
 
 }  // namespace ve

@@ -8,6 +8,7 @@
 // compares per element, and counts masked / unchanged elements with popcounts.
 #include <cuda_runtime.h>
 
+#include <cstring>
 #include <vector>
 
 #include "ve_internal.cuh"
@@ -46,26 +47,34 @@ __global__ void __launch_bounds__(256) k_diff_vec(const uint4* __restrict__ pre,
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   constexpr int U = 4;
+  // the mask bits of a 16-byte block are read first: blocks without masked elements load nothing
+  // (B_diff = 2 x masked bytes + mask)
+  const uint32_t full = (per == 32u) ? 0xFFFFFFFFu : ((1u << per) - 1u);
   for (; i + (U - 1) * stride < nvec; i += U * stride) {
-    uint4 a[U], b[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) { a[u] = __ldcs(pre + i + u * stride); b[u] = __ldcs(post + i + u * stride); }
+    uint32_t m[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      const uint64_t v = i + u * stride;
-      const uint64_t e0 = v * per;
-      uint32_t m = (per == 32u) ? 0xFFFFFFFFu : ((1u << per) - 1u);
-      if (mask) m &= __ldg(mask + (e0 >> 5)) >> (e0 & 31);
+      const uint64_t e0 = (i + u * stride) * per;
+      m[u] = mask ? full & (__ldg(mask + (e0 >> 5)) >> (e0 & 31)) : full;
+    }
+    uint4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      a[u] = b[u] = make_uint4(0, 0, 0, 0);
+      if (m[u]) { a[u] = __ldcs(pre + i + u * stride); b[u] = __ldcs(post + i + u * stride); }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
       const uint32_t q = eq_bits16(a[u], b[u], ew_lg);
-      cm += __popc(m);
-      cu += __popc(m & q);
+      cm += __popc(m[u]);
+      cu += __popc(m[u] & q);
     }
   }
   for (; i < nvec; i += stride) {
-    const uint4 a = __ldcs(pre + i), b = __ldcs(post + i);
     const uint64_t e0 = i * per;
-    uint32_t m = (per == 32u) ? 0xFFFFFFFFu : ((1u << per) - 1u);
-    if (mask) m &= __ldg(mask + (e0 >> 5)) >> (e0 & 31);
+    const uint32_t m = mask ? full & (__ldg(mask + (e0 >> 5)) >> (e0 & 31)) : full;
+    if (!m) continue;
+    const uint4 a = __ldcs(pre + i), b = __ldcs(post + i);
     const uint32_t q = eq_bits16(a, b, ew_lg);
     cm += __popc(m);
     cu += __popc(m & q);
@@ -180,4 +189,62 @@ ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask
   return VE_OK;
 }
 
+}  // namespace ve
+
+namespace ve {
+// S10 of every object with both snapshots (mode WRITTEN or ALL), sharded by object over comm: the
+// object at position k of the ctx's sorted table is diffed by rank k mod G; each rank's results go
+// into a u64 table [n_obj][5] (zero where it does not own), SUM-allreduced, then unpacked by id.
+// Objects without both snapshots report n_elems only.  Every context must hold the same objects
+// (the merged state of a rank merge).
+ve_status diff_ranks(const std::vector<ve_ctx*>& cs, Comm& comm, uint32_t mode, ve_diff* out_by_id, cudaStream_t s) {
+  ve_ctx* c0 = cs[0];
+  if (mode != VE_DIFF_WRITTEN && mode != VE_DIFF_ALL)
+    return fail(c0, VE_ERR_INVALID, "ve_snapshot_diff_all: mode must be VE_DIFF_WRITTEN or VE_DIFF_ALL");
+  const uint32_t n = c0->n_obj;
+  for (ve_ctx* c : cs)
+    if (c->n_obj != n) return fail(c0, VE_ERR_INVALID, "ve_snapshot_diff_all: contexts hold different objects");
+  if (n == 0) return VE_OK;
+  const int G = comm.G;
+  std::vector<void*> bufs(cs.size());
+  for (size_t i = 0; i < cs.size(); ++i) {
+    ve_ctx* c = cs[i];
+    std::vector<unsigned long long> tab((size_t)n * 5, 0ull);
+    for (uint32_t k = 0; k < n; ++k) {
+      if ((int)(k % G) != comm.local[i]) continue;
+      const HostObject& o = c->objs[k];
+      if (!o.pre || !o.post) continue;
+      ve_diff d;
+      ve_status st = run_diff(c, k, mode, nullptr, &d, s);
+      if (st != VE_OK) return st;
+      unsigned long long* r = &tab[(size_t)k * 5];
+      r[0] = 1; r[1] = d.n_masked; r[2] = d.n_unchanged; r[3] = d.n_untouched; r[4] = 0;
+    }
+    cudaError_t e = cudaMallocAsync(&bufs[i], tab.size() * 8, s);
+    if (e != cudaSuccess) return cuda_fail(c0, e, "diff_all alloc");
+    cudaMemcpyAsync(bufs[i], tab.data(), tab.size() * 8, cudaMemcpyHostToDevice, s);
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(c0, e, "diff_all");
+  }
+  if (!comm.allreduce(bufs, (size_t)n * 5, OP_SUM, s)) return fail(c0, VE_ERR_NCCL, "diff allreduce: " + comm.err);
+  std::vector<unsigned long long> tab((size_t)n * 5);
+  cudaMemcpyAsync(tab.data(), bufs[0], tab.size() * 8, cudaMemcpyDeviceToHost, s);
+  for (void* b : bufs) cudaFreeAsync(b, s);
+  cudaError_t e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c0, e, "diff_all");
+  for (uint32_t k = 0; k < n; ++k) {
+    const HostObject& o = c0->objs[k];
+    const unsigned long long* r = &tab[(size_t)k * 5];
+    ve_diff& d = out_by_id[o.id];
+    memset(&d, 0, sizeof(d));
+    d.n_elems = o.n_elems;
+    if (!r[0]) continue;
+    d.n_masked = r[1];
+    d.n_unchanged = r[2];
+    d.n_changed = r[1] - r[2];
+    d.n_untouched = r[3];
+    d.redundant = (r[1] > 0 && (unsigned __int128)100 * r[2] > (unsigned __int128)c0->cfg.t_redundant_pct * r[1]);
+  }
+  return VE_OK;
+}
 }  // namespace ve

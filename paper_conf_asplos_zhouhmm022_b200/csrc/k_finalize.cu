@@ -989,8 +989,25 @@ __global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n
 
 // Cardinality probe of a dense array: the distinct values among up to 64 Ki counted
 // elements sampled at a fixed stride (one block); out[0] = distinct (capped near 4096).
+struct SampleJob {
+  const uint32_t* cnt;
+  const uint8_t* pre;     // the claim's side snapshot
+  uint64_t n_elems;
+  uint32_t ew, pad;
+};
+__device__ void dense_sample_body(const uint32_t* cnt, uint64_t n_elems, const uint8_t* pre, uint32_t ew,
+                                  unsigned int* out);
+// every claim's cardinality probe in one launch (one block per claim)
+__global__ void __launch_bounds__(1024) k_dense_sample_many(const SampleJob* jobs, unsigned int* out) {
+  const SampleJob j = jobs[blockIdx.x];
+  dense_sample_body(j.cnt, j.n_elems, j.pre, j.ew, out + blockIdx.x);
+}
 __global__ void __launch_bounds__(1024) k_dense_sample(const uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
                                                       uint32_t ew, unsigned int* out) {
+  dense_sample_body(cnt, n_elems, pre, ew, out);
+}
+__device__ void dense_sample_body(const uint32_t* cnt, uint64_t n_elems, const uint8_t* pre, uint32_t ew,
+                                  unsigned int* out) {
   extern __shared__ unsigned long long tb[];   // 8192 slots (dynamic: 64 KiB)
   __shared__ unsigned int nd;
   for (int i = threadIdx.x; i < 8192; i += 1024) tb[i] = ~0ull;
@@ -1287,10 +1304,10 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
         }
       }
     }
-    // insert the led groups.  A table generation must hold all groups of a batch (H0 and
-    // corrections of the same elements), so should one not fit (64 probes full: adversarial
-    // cardinality), the batch's inserted groups are taken out again and its counts go to the HBM
-    // table element by element instead -- exact either way
+    // insert the warp's groups.  A table generation must hold all groups of the warp's 32 elements
+    // (H0 and corrections of the same elements), so should one not fit (64 probes full), the warp
+    // takes its inserted groups out again and sends its elements' counts to the HBM table one by one
+    // -- exact either way, and without a block barrier
     uint32_t done = 0;
 #pragma unroll
     for (int b = 0; b < 2 + DO_MAXC; ++b) {
@@ -1298,7 +1315,7 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
       const uint64_t v = (b == 1 || (b >= 2 && A.c[b - 2].side)) ? sv1 : sv0;
       if (do_add(ts, (uint32_t)b, v, gd[b], &s_fill)) done |= 1u << b;
     }
-    if (__syncthreads_or(pend != done)) {
+    if (__any_sync(0xFFFFFFFFu, pend != done)) {
 #pragma unroll
       for (int b = 0; b < 2 + DO_MAXC; ++b) {
         if (!((done >> b) & 1u)) continue;
@@ -1316,9 +1333,12 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
         }
         do_acc_fold(st[j], acc);
       }
-      __syncthreads();
     }
-    if (s_fill > DO_TS * 7 / 10) drain();   // (block-uniform: read after the barrier above)
+    // every 4 batches (block-uniform): drain a table past 60 %
+    if ((((base - lo) / DO_THREADS) & 3u) == 3u) {
+      __syncthreads();
+      if (s_fill > DO_TS * 6 / 10) drain();
+    }
   }
   }
   drain();
@@ -1387,13 +1407,23 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   unsigned int* d_probe = nullptr;
   e = cudaMallocAsync((void**)&d_probe, 4 * nc, s);
   if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush probe alloc");
-  cudaFuncSetAttribute(k_dense_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
-  for (size_t k = 0; k < nc; ++k) {
-    const HostObject& o = c->objs[cl[k].i];
+  cudaFuncSetAttribute(k_dense_sample_many, cudaFuncAttributeMaxDynamicSharedMemorySize, 8192 * 8);
+  {
+    std::vector<SampleJob> sj(nc);
+    for (size_t k = 0; k < nc; ++k) {
+      const HostObject& o = c->objs[cl[k].i];
+      sj[k] = SampleJob{(const uint32_t*)((uint32_t*)c->dense_pool + cl[k].off),
+                        (const uint8_t*)((cl[k].ck & DENSE_POST) ? o.post : o.pre), o.n_elems, o.ew, 0};
+    }
+    SampleJob* d_sj = nullptr;
+    e = cudaMallocAsync((void**)&d_sj, nc * sizeof(SampleJob), s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush probe jobs");
+    cudaMemcpyAsync(d_sj, sj.data(), nc * sizeof(SampleJob), cudaMemcpyHostToDevice, s);
     count_launch();
-    k_dense_sample<<<1, 1024, 8192 * 8, s>>>((uint32_t*)c->dense_pool + cl[k].off, o.n_elems,
-                                             (const uint8_t*)((cl[k].ck & DENSE_POST) ? o.post : o.pre), o.ew,
-                                             d_probe + k);
+    k_dense_sample_many<<<(unsigned)nc, 1024, 8192 * 8, s>>>(d_sj, d_probe);
+    cudaFreeAsync(d_sj, s);
+    e = cudaStreamSynchronize(s);     // (sj is a host vector of this scope)
+    if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush probe");
   }
   cudaMemcpyAsync(mh.data(), (uint8_t*)dm + 2 * nc * 8, nc * 4, cudaMemcpyDeviceToHost, s);
   cudaMemcpyAsync(nd.data(), d_probe, 4 * nc, cudaMemcpyDeviceToHost, s);

@@ -25,26 +25,7 @@
 
 namespace ve {
 
-// ---- transports -----------------------------------------------------------------
-enum { OP_SUM = 0, OP_MIN = 1, OP_MAX = 2 };
-
-struct Comm {
-  int G = 1;                      // number of ranks
-  std::vector<int> local;         // global rank of each local context
-  std::string err;
-  virtual ~Comm() {}
-  // u64 in-place allreduce of count elements in bufs[i] (one per local rank)
-  virtual bool allreduce(const std::vector<void*>& bufs, size_t count, int op, cudaStream_t s) = 0;
-  // recv[i] receives G blocks of bytes, block g from global rank g
-  virtual bool allgather(const std::vector<const void*>& send, const std::vector<void*>& recv, size_t bytes,
-                         cudaStream_t s) = 0;
-  // send[i] + soff[i][g] (sbytes[i][g]) goes to rank g; recv[i] + roff[i][g] gets rbytes[i][g] from rank g
-  virtual bool alltoallv(const std::vector<const uint8_t*>& send, const std::vector<std::vector<size_t>>& soff,
-                         const std::vector<std::vector<size_t>>& sbytes, const std::vector<uint8_t*>& recv,
-                         const std::vector<std::vector<size_t>>& roff, const std::vector<std::vector<size_t>>& rbytes,
-                         cudaStream_t s) = 0;
-};
-
+// ---- transports (Comm: ve_internal.cuh) --------------------------------------------
 __global__ void k_reduce_u64(unsigned long long* dst, const unsigned long long* src, size_t n, int op) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
     const unsigned long long a = dst[i], b = src[i];
@@ -436,6 +417,64 @@ ve_status ve_merge_group(ve_ctx** ctxs, uint32_t n, cudaStream_t s) {
   comm.G = (int)n;
   for (uint32_t i = 0; i < n; ++i) comm.local.push_back((int)i);
   return merge_ranks(cs, comm, s);
+}
+
+// S10 / S11 sharded by object: see diff_ranks / dedup_ranks
+static ve_status comm_of(ve_ctx* c, void* comm_ptr, NcclComm& comm) {
+  if (!nccl().ok) return fail(c, VE_ERR_NCCL, "NCCL library not available");
+  comm.comm = (ncclComm_t)comm_ptr;
+  int G = 0, me = 0;
+  if (nccl().CommCount(comm.comm, &G) != ncclSuccess || nccl().CommUserRank(comm.comm, &me) != ncclSuccess)
+    return fail(c, VE_ERR_NCCL, "bad NCCL communicator");
+  comm.G = G;
+  comm.local = {me};
+  return VE_OK;
+}
+
+ve_status ve_snapshot_diff_all(ve_ctx* ctx, uint32_t mode, void* nccl_comm_or_null, ve_diff* h_out, cudaStream_t s) {
+  if (!ctx || !h_out) return VE_ERR_INVALID;
+  cudaSetDevice(ctx->device);
+  if (!nccl_comm_or_null) {
+    LocalComm one;
+    return diff_ranks({ctx}, one, mode, h_out, s);
+  }
+  NcclComm comm;
+  ve_status st = comm_of(ctx, nccl_comm_or_null, comm);
+  return st != VE_OK ? st : diff_ranks({ctx}, comm, mode, h_out, s);
+}
+
+ve_status ve_object_dedup_comm(ve_ctx* ctx, const ve_object* objs, uint32_t n, void* nccl_comm, uint32_t* h_group_of,
+                               cudaStream_t s) {
+  if (!ctx || !nccl_comm || (n && (!objs || !h_group_of))) return VE_ERR_INVALID;
+  cudaSetDevice(ctx->device);
+  NcclComm comm;
+  ve_status st = comm_of(ctx, nccl_comm, comm);
+  return st != VE_OK ? st : dedup_ranks({ctx}, comm, objs, n, h_group_of, s);
+}
+
+ve_status ve_snapshot_diff_all_group(ve_ctx** ctxs, uint32_t n, uint32_t mode, ve_diff* h_out, cudaStream_t s) {
+  if (!ctxs || n == 0 || !h_out) return VE_ERR_INVALID;
+  std::vector<ve_ctx*> cs(ctxs, ctxs + n);
+  for (ve_ctx* c : cs)
+    if (!c || c->device != cs[0]->device) return VE_ERR_INVALID;
+  cudaSetDevice(cs[0]->device);
+  SimComm comm;
+  comm.G = (int)n;
+  for (uint32_t i = 0; i < n; ++i) comm.local.push_back((int)i);
+  return diff_ranks(cs, comm, mode, h_out, s);
+}
+
+ve_status ve_object_dedup_group(ve_ctx** ctxs, uint32_t n, const ve_object* objs, uint32_t n_objs, uint32_t* h_group_of,
+                                cudaStream_t s) {
+  if (!ctxs || n == 0 || (n_objs && (!objs || !h_group_of))) return VE_ERR_INVALID;
+  std::vector<ve_ctx*> cs(ctxs, ctxs + n);
+  for (ve_ctx* c : cs)
+    if (!c || c->device != cs[0]->device) return VE_ERR_INVALID;
+  cudaSetDevice(cs[0]->device);
+  SimComm comm;
+  comm.G = (int)n;
+  for (uint32_t i = 0; i < n; ++i) comm.local.push_back((int)i);
+  return dedup_ranks(cs, comm, objs, n_objs, h_group_of, s);
 }
 
 ve_status ve_nccl_get_unique_id(void* out128) {

@@ -172,6 +172,43 @@ ve_status run_diff(ve_ctx* c, uint32_t obj_index, uint32_t mode, const uint32_t*
                    cudaStream_t s);
 ve_status run_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* group_of, cudaStream_t s);
 ve_status merge_local(ve_ctx* dst, const ve_ctx* src, cudaStream_t s);
+// ---- rank transports (nccl_merge.cu: NCCL, and same-device simulated ranks) ----
+enum { OP_SUM = 0, OP_MIN = 1, OP_MAX = 2 };
+struct Comm {
+  int G = 1;                      // number of ranks
+  std::vector<int> local;         // global rank of each local context
+  std::string err;
+  virtual ~Comm() {}
+  // u64 in-place allreduce of count elements in bufs[i] (one per local rank)
+  virtual bool allreduce(const std::vector<void*>& bufs, size_t count, int op, cudaStream_t s) = 0;
+  // recv[i] receives G blocks of bytes, block g from global rank g
+  virtual bool allgather(const std::vector<const void*>& send, const std::vector<void*>& recv, size_t bytes,
+                         cudaStream_t s) = 0;
+  // send[i] + soff[i][g] (sbytes[i][g]) goes to rank g; recv[i] + roff[i][g] gets rbytes[i][g] from rank g
+  virtual bool alltoallv(const std::vector<const uint8_t*>& send, const std::vector<std::vector<size_t>>& soff,
+                         const std::vector<std::vector<size_t>>& sbytes, const std::vector<uint8_t*>& recv,
+                         const std::vector<std::vector<size_t>>& roff, const std::vector<std::vector<size_t>>& rbytes,
+                         cudaStream_t s) = 0;
+};
+struct LocalComm : Comm {        // one rank: every exchange is the identity
+  LocalComm() { G = 1; local = {0}; }
+  bool allreduce(const std::vector<void*>&, size_t, int, cudaStream_t) override { return true; }
+  bool allgather(const std::vector<const void*>& send, const std::vector<void*>& recv, size_t bytes,
+                 cudaStream_t s) override {
+    return !bytes || cudaMemcpyAsync(recv[0], send[0], bytes, cudaMemcpyDeviceToDevice, s) == cudaSuccess;
+  }
+  bool alltoallv(const std::vector<const uint8_t*>&, const std::vector<std::vector<size_t>>&,
+                 const std::vector<std::vector<size_t>>&, const std::vector<uint8_t*>&,
+                 const std::vector<std::vector<size_t>>&, const std::vector<std::vector<size_t>>&,
+                 cudaStream_t) override { return false; }
+};
+// S11 / S10 sharded by object over the ranks of comm (cs: one context per local rank): the owner
+// rank of object k (position k of the eligible list, k mod G) hashes / diffs it, candidate pairs
+// are verified by rank (pair index mod G), and the partial results are allreduced -- every rank
+// ends with the same full result.  One rank (LocalComm) is the plain call.
+ve_status dedup_ranks(const std::vector<ve_ctx*>& cs, Comm& comm, const ve_object* objs, uint32_t n,
+                      uint32_t* group_of, cudaStream_t s);
+ve_status diff_ranks(const std::vector<ve_ctx*>& cs, Comm& comm, uint32_t mode, ve_diff* out_by_id, cudaStream_t s);
 ve_status merge_nccl(ve_ctx* c, void* comm, cudaStream_t s);
 ve_status dense_flush(ve_ctx* c, cudaStream_t s);  // move dense counts into the exact histogram
 ve_status approx_topk(ve_ctx* c, cudaStream_t s, const std::vector<uint8_t>& akind, std::vector<uint64_t>& ndistinct,

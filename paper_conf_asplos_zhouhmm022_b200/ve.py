@@ -120,6 +120,10 @@ def lib():
             "ve_vfg_free": ([vp], None),
             "ve_record_intervals": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
+            "ve_snapshot_diff_all": ([vp, u32, vp, vp, vp], st),
+            "ve_object_dedup_comm": ([vp, vp, u32, vp, vp, vp], st),
+            "ve_snapshot_diff_all_group": ([ctypes.POINTER(vp), u32, u32, vp, vp], st),
+            "ve_object_dedup_group": ([ctypes.POINTER(vp), u32, vp, u32, vp, vp], st),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -229,6 +233,34 @@ def merge_group(contexts, stream=None):
     rc = lib().ve_merge_group(arr, len(contexts), _stream(stream))
     if rc != OK:
         raise VeError(rc, "ve_merge_group: " + lib().ve_last_error(contexts[0].handle).decode())
+
+
+def _objects_arr(objs):
+    arr = (_Object * max(len(objs), 1))()
+    for i, o in enumerate(objs):
+        arr[i] = _Object(o["base"], o["size"], _ptr(o.get("pre")), _ptr(o.get("post")), o["id"], o.get("elem_width", 8))
+    return arr
+
+
+def snapshot_diff_all_group(contexts, mode=DIFF_WRITTEN, stream=None):
+    """ve_snapshot_diff_all_group: the object-sharded diff with context i playing rank i (one device)."""
+    arr = (ctypes.c_void_p * len(contexts))(*[c.handle.value for c in contexts])
+    n = getattr(contexts[0], "n_objects", 0)
+    out = np.zeros(max(n, 1), dtype=DIFF_DTYPE)
+    rc = lib().ve_snapshot_diff_all_group(arr, len(contexts), mode, out.ctypes.data, _stream(stream))
+    if rc != OK:
+        raise VeError(rc, "ve_snapshot_diff_all_group: " + lib().ve_last_error(contexts[0].handle).decode())
+    return out[:n]
+
+
+def object_dedup_group(contexts, objs, stream=None):
+    """ve_object_dedup_group: the object-sharded duplicate scan with context i playing rank i."""
+    arr = (ctypes.c_void_p * len(contexts))(*[c.handle.value for c in contexts])
+    g = np.zeros(max(len(objs), 1), dtype=np.uint32)
+    rc = lib().ve_object_dedup_group(arr, len(contexts), _objects_arr(objs), len(objs), g.ctypes.data, _stream(stream))
+    if rc != OK:
+        raise VeError(rc, "ve_object_dedup_group: " + lib().ve_last_error(contexts[0].handle).decode())
+    return g[:len(objs)]
 
 
 def nccl_unique_id():
@@ -360,15 +392,26 @@ class Context:
                     "ve_snapshot_diff")
         return out[0]
 
-    def object_dedup(self, objs, stream=None):
-        arr = (_Object * max(len(objs), 1))()
-        for i, o in enumerate(objs):
-            arr[i] = _Object(o["base"], o["size"], _ptr(o.get("pre")), _ptr(o.get("post")), o["id"],
-                             o.get("elem_width", 8))
+    def object_dedup(self, objs, comm=None, stream=None):
+        """ve_object_dedup (comm: ve_object_dedup_comm, sharded over the ranks of an NCCL comm)."""
+        arr = _objects_arr(objs)
         g = np.zeros(max(len(objs), 1), dtype=np.uint32)
-        self._check(lib().ve_object_dedup(self._h, arr, len(objs), g.ctypes.data, _stream(stream)),
-                    "ve_object_dedup")
+        if comm:
+            self._check(lib().ve_object_dedup_comm(self._h, arr, len(objs), ctypes.c_void_p(comm), g.ctypes.data,
+                                                   _stream(stream)), "ve_object_dedup_comm")
+        else:
+            self._check(lib().ve_object_dedup(self._h, arr, len(objs), g.ctypes.data, _stream(stream)),
+                        "ve_object_dedup")
         return g[:len(objs)]
+
+    def snapshot_diff_all(self, mode=DIFF_WRITTEN, comm=None, stream=None):
+        """ve_snapshot_diff_all: DIFF_DTYPE[n_objects] (by id) of every object with both snapshots,
+        sharded by object over the ranks of an NCCL comm (None: this rank alone)."""
+        n = getattr(self, "n_objects", 0)
+        out = np.zeros(max(n, 1), dtype=DIFF_DTYPE)
+        self._check(lib().ve_snapshot_diff_all(self._h, mode, ctypes.c_void_p(comm) if comm else None,
+                                               out.ctypes.data, _stream(stream)), "ve_snapshot_diff_all")
+        return out[:n]
 
     def merge(self, other=None, comm=None, stream=None):
         """ve_merge_stats: with another same-device context, or over all ranks of an NCCL comm."""

@@ -1,8 +1,8 @@
 """GPU parity of every K1 (k_analyze) code path the bench runs, against the CPU oracle, bit-exact.
 
-launch_analyze picks k_analyze<false> (single-key slots, run_dense) for traces with < 8 PCs and
-k_analyze<true> (multi-key dense batches) otherwise; VE_K1_MULTI=0/1 forces one, so each trace
-below runs through BOTH instantiations.  Traces of >= 4 x 148 x 16 x 16 windows (~4.85 M records)
+launch_analyze picks K1 v1 k_analyze<false> (single-key slots, run_dense) for traces with < 8 PCs
+and K1 v2 k_analyze2 (register key slots, post-value counting) otherwise; VE_K1=1/2 and
+VE_K1_MULTI=0/1 force one, so each trace below runs through v1 single-key, v1 multi-key and v2.  Traces of >= 4 x 148 x 16 x 16 windows (~4.85 M records)
 take the 16-window static-interleave chunk path (multi-stage chunks), shorter ones one-stage chunks:
 the large cases cover the chunk path the full-size configs use.
 
@@ -33,23 +33,26 @@ def torch_cuda():
 from tests.gpu_run import _check, _run_gpu  # noqa: E402
 
 
-class _k1:
-    """force one k_analyze instantiation for the block"""
+KERNELS = [("1", "0"), ("1", "1"), ("2", "")]     # (VE_K1, VE_K1_MULTI): v1 single-key, v1 multi-key, v2
 
-    def __init__(self, multi):
-        self.v = None if multi is None else ("1" if multi else "0")
+
+class _k1:
+    """force one k_analyze kernel for the block"""
+
+    def __init__(self, k):
+        self.k = k
 
     def __enter__(self):
-        self.old = os.environ.get("VE_K1_MULTI")
-        if self.v is not None:
-            os.environ["VE_K1_MULTI"] = self.v
+        self.old = (os.environ.get("VE_K1"), os.environ.get("VE_K1_MULTI"))
+        os.environ["VE_K1"], os.environ["VE_K1_MULTI"] = self.k
         return self
 
     def __exit__(self, *a):
-        if self.old is None:
-            os.environ.pop("VE_K1_MULTI", None)
-        else:
-            os.environ["VE_K1_MULTI"] = self.old
+        for name, v in zip(("VE_K1", "VE_K1_MULTI"), self.old):
+            if v is None:
+                os.environ.pop(name, None)
+            else:
+                os.environ[name] = v
 
 
 def fuzz5(seed, n, r0=0):
@@ -63,11 +66,11 @@ def fuzz5(seed, n, r0=0):
 def _parity(torch_cuda, n_pcs, hobjs, recs, hcap=1 << 22, chunks=None):
     cfg = O.make_config(n_pcs)
     okeys, oglob, oobj = O.analyze(cfg, hobjs, recs)
-    for multi in (False, True):
-        with _k1(multi):
+    for k in KERNELS:
+        with _k1(k):
             rep, _ = _run_gpu(torch_cuda, n_pcs, hobjs, recs, hist_capacity=hcap, chunks=chunks)
         bad = parity.compare_with_oracle(rep, okeys, oglob, oobj)
-        assert not bad, f"multi={multi}:\n" + "\n".join(bad[:30])
+        assert not bad, f"kernel {k}:\n" + "\n".join(bad[:30])
 
 
 @pytest.mark.parametrize("seed,n", [(21, 4096), (22, 100003), (23, 300001), (24, 1 << 20)])
