@@ -1248,16 +1248,27 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
   const uint64_t nch = (A.ne + DO_CH - 1) / DO_CH;
   for (uint64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
   const uint64_t lo = ch * DO_CH, hi = lo + DO_CH < A.ne ? lo + DO_CH : A.ne;
+  // the loads of a batch (the counters of all claims, the snapshot sides) are issued one batch
+  // ahead, so they are in flight while the previous batch is inserted
+  uint32_t ncj[DO_MAXC];
+  uint64_t nsv0 = 0, nsv1 = 0;
+  auto issue = [&](uint64_t b) {
+    const uint64_t e = b + tid;
+    const bool in = e < hi;
+#pragma unroll
+    for (int j = 0; j < DO_MAXC; ++j) ncj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
+    nsv0 = (in && A.snap[0]) ? do_load(A.snap[0] + e * A.ew, A.ew) : 0ull;
+    nsv1 = (in && A.snap[1]) ? do_load(A.snap[1] + e * A.ew, A.ew) : 0ull;
+  };
+  issue(lo);
   for (uint64_t base = lo; base < hi; base += DO_THREADS) {
     const uint64_t e = base + tid;
     const bool in = e < hi;
-    // every load of the batch first (the counters of all claims, the snapshot sides), then the rest
     uint32_t cj[DO_MAXC];
 #pragma unroll
-    for (int j = 0; j < DO_MAXC; ++j) cj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
-    uint64_t sv0 = 0, sv1 = 0;
-    if (in && A.snap[0]) sv0 = do_load(A.snap[0] + e * A.ew, A.ew);
-    if (in && A.snap[1]) sv1 = do_load(A.snap[1] + e * A.ew, A.ew);
+    for (int j = 0; j < DO_MAXC; ++j) cj[j] = ncj[j];
+    const uint64_t sv0 = nsv0, sv1 = nsv1;
+    if (base + DO_THREADS < hi) issue(base + DO_THREADS);
     uint32_t corr = 0;                                 // claims whose count differs from their base
     bool lbit = false;
 #pragma unroll
@@ -1334,8 +1345,8 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
         do_acc_fold(st[j], acc);
       }
     }
-    // every 4 batches (block-uniform): drain a table past 60 %
-    if ((((base - lo) / DO_THREADS) & 3u) == 3u) {
+    // every 8 batches (block-uniform): drain a table past 60 %
+    if ((((base - lo) / DO_THREADS) & 7u) == 7u) {
       __syncthreads();
       if (s_fill > DO_TS * 6 / 10) drain();
     }
