@@ -2475,6 +2475,7 @@ __global__ void __launch_bounds__(LF_THREADS) k_line_fold(const LineState* lcta,
 }
 
 ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
+  if (c->reset_ev) cudaStreamWaitEvent(s, c->reset_ev, 0);   // after the last (legacy-stream) reset
   AnalyzeParams P;
   P.recs = d;
   P.n = n;

@@ -125,6 +125,7 @@ __global__ void __launch_bounds__(256) k_touched(const uint32_t* __restrict__ W,
 
 ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask, ve_diff* out, cudaStream_t s) {
   const HostObject& o = c->objs[oi];
+  if (c->reset_ev) cudaStreamWaitEvent(s, c->reset_ev, 0);
   // counted loads set their L bits when flushed: flush first, so n_untouched does not
   // depend on whether ve_report ran before this call (idempotent; ve_report skips it then)
   if (!c->hist_merged) {

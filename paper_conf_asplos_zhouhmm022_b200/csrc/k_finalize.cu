@@ -472,21 +472,19 @@ __device__ __forceinline__ void block_chunk(uint64_t n, uint64_t& lo, uint64_t& 
   if (lo > hi) lo = hi;
 }
 
-__global__ void k_tagscan(const HSlot* hs, uint64_t cap, uint32_t* tags, unsigned long long* tcnt,
-                          unsigned long long* ovf, uint32_t* occ_idx, unsigned long long* n_occ) {
+// the distinct tags of the occupied slots (the table's occupancy list: O(entries), not O(capacity))
+// and their entry counts
+__global__ void k_tagscan(const HSlot* hs, const uint32_t* occ, const unsigned long long* n_occ, uint32_t* tags,
+                          unsigned long long* tcnt, unsigned long long* ovf) {
   __shared__ BlockKeys B;
-  __shared__ unsigned long long s_cur;
   bk_init(B);
-  if (threadIdx.x == 0) s_cur = 0;
   __syncthreads();
   uint64_t lo, hi;
-  block_chunk(cap, lo, hi);
-  unsigned long long my = 0;   // occupied slots seen by this thread
+  block_chunk(*n_occ, lo, hi);
   for (uint64_t b = lo; b < hi; b += blockDim.x) {
-    const uint64_t i = b + threadIdx.x;
-    const uint32_t tag = i < hi ? hs[i].tag : EMPTY_TAG;
+    const uint64_t j = b + threadIdx.x;
+    const uint32_t tag = j < hi ? hs[occ[j]].tag : EMPTY_TAG;
     const bool act = tag != EMPTY_TAG;
-    my += act ? 1u : 0u;
     const int sl = bk_add(B, act, tag);
     if (act && sl < 0) {   // shared table full: count this entry globally
       uint32_t h = (uint32_t)mix64(tag) & (TAG_CAP - 1);
@@ -515,28 +513,6 @@ __global__ void k_tagscan(const HSlot* hs, uint64_t cap, uint32_t* tags, unsigne
     }
     if (done) atomicAdd(&tcnt[h], B.cnt[j]);
     else atomicExch(ovf, 1ull);
-  }
-  // the chunk's occupied slots, compacted (one reservation per block; order within
-  // the block's range is irrelevant)
-  my = __reduce_add_sync(0xFFFFFFFFu, (unsigned)my);
-  if ((threadIdx.x & 31) == 0 && my) atomicAdd(&s_cur, my);
-  __syncthreads();
-  const unsigned long long nb = s_cur;
-  __syncthreads();
-  if (threadIdx.x == 0) s_cur = nb ? atomicAdd(n_occ, nb) : 0;
-  __syncthreads();
-  const unsigned long long base = s_cur;
-  __syncthreads();
-  if (threadIdx.x == 0) s_cur = 0;
-  __syncthreads();
-  for (uint64_t b = lo; b < hi && nb; b += blockDim.x) {
-    const uint64_t i = b + threadIdx.x;
-    const bool occ = i < hi && hs[i].tag != EMPTY_TAG;
-    const unsigned m = __ballot_sync(0xFFFFFFFFu, occ);
-    unsigned long long wb = 0;
-    if ((threadIdx.x & 31) == 0 && m) wb = atomicAdd(&s_cur, (unsigned long long)__popc(m));
-    wb = __shfl_sync(0xFFFFFFFFu, wb, 0);
-    if (occ) occ_idx[base + wb + __popc(m & ((1u << (threadIdx.x & 31)) - 1u))] = (uint32_t)i;
   }
 }
 
@@ -643,13 +619,13 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   unsigned long long* d_tcnt = nullptr;
   unsigned long long* d_small = nullptr;     // [0] overflow, [1] occupied slots
   unsigned long long* d_tl = nullptr;        // compacted tag list
-  uint32_t* d_occ = nullptr;                 // occupied slot indices
+  const uint32_t* d_occ = c->t.occ;          // occupied slot indices (maintained by every insert)
+  const unsigned long long* d_nocc = c->t.glob + G_NOCC;
   if (c->hcap > 0xFFFFFFFFull) return fail(c, VE_ERR_INVALID, "finalize: hist_capacity above 2^32");
   e = cudaMallocAsync((void**)&d_tags, TAG_CAP * 4, s);
   if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_tcnt, TAG_CAP * 8, s);
   if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_small, 16, s);
   if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_tl, (1 + 2 * TAGL_MAX) * 8, s);
-  if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_occ, c->hcap * 4, s);
   if (e != cudaSuccess) return cuda_fail(c, e, "finalize alloc");
   if (!c->pin) {
     e = cudaMallocHost(&c->pin, (1 + 2 * TAGL_MAX) * 8 + 64);
@@ -661,7 +637,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   cudaMemsetAsync(d_small, 0, 16, s);
   stage("start", s);
   count_launch();
-  k_tagscan<<<grid, 256, 0, s>>>(c->t.hslot, c->hcap, d_tags, d_tcnt, d_small, d_occ, d_small + 1);
+  k_tagscan<<<grid, 256, 0, s>>>(c->t.hslot, d_occ, d_nocc, d_tags, d_tcnt, d_small);
   count_launch();
   cudaMemsetAsync(d_tl, 0, 8, s);
   k_tag_compact<<<(TAG_CAP + 255) / 256, 256, 0, s>>>(d_tags, d_tcnt, d_tl);
@@ -689,7 +665,6 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   cudaFreeAsync(d_tl, s);
   stage("tagscan+d2h", s);
   if (ovf) {                                  // too many distinct tags: aggregate every key
-    cudaFreeAsync(d_occ, s);
     cudaFreeAsync(d_small, s);
     ViewTable V;
     ve_status st = build_views(c, s, V);
@@ -743,7 +718,7 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   stage("alloc", s);
   // 3. emit direct keys' entries, aggregate the others in the view table
   count_launch();
-  k_emit<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, d_occ, d_small + 1, npc, d_direct, d_off, d_off + nk, gb[0],
+  k_emit<<<grid, 256, 0, s>>>(c->t.hslot, c->t.hcount, d_occ, d_nocc, npc, d_direct, d_off, d_off + nk, gb[0],
                               gc[0], V.vs, V.vc, V.vcap ? V.vcap - 1 : 0, d_small);
   if (agg_in) {
     unsigned long long* d_nd = nullptr;
@@ -774,7 +749,6 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   unsigned long long h_ovf = 0;
   cudaMemcpyAsync(&h_ovf, d_small, 8, cudaMemcpyDeviceToHost, s);
   free_views(V, s);
-  cudaFreeAsync(d_occ, s);
   cudaFreeAsync(gbuf, s);
   cudaFreeAsync(d_direct, s);
   cudaFreeAsync(d_off, s);

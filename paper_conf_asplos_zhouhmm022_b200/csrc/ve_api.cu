@@ -40,6 +40,7 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->t.L);
   cudaFree(c->t.hslot);
   cudaFree(c->t.hcount);
+  cudaFree(c->t.occ);
   cudaFree(c->obj_block);
   cudaFree(c->scratch);
   if (c->pin) cudaFreeHost(c->pin);
@@ -52,6 +53,20 @@ static void free_dev(ve_ctx* c) {
     if (c->copied_ev[i]) cudaEventDestroy(c->copied_ev[i]);
   }
   if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
+  if (c->reset_ev) cudaEventDestroy(c->reset_ev);
+}
+
+// empty the occupied slots recorded in t.occ (the table's only non-empty slots), then their count
+__global__ void k_reset_occ(DevTables t) {
+  const unsigned long long n = t.glob[G_NOCC];
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const uint32_t h = t.occ[i];
+    t.hslot[h].bits = ~0ull;
+    t.hslot[h].tag = EMPTY_TAG;
+    t.hslot[h].pad = EMPTY_TAG;
+    t.hcount[h] = 0;
+  }
 }
 
 ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
@@ -69,19 +84,28 @@ ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
     if (used) cudaMemsetAsync(c->dense_pool, 0, used * 4, s);
     c->dense_dirty = false;
   }
+  // the value table: a fresh table is filled whole; afterwards only the slots claimed since the last
+  // reset (recorded in t.occ) are emptied -- O(entries), not O(hist_capacity), per epoch
+  const bool full = !c->table_clean;
+  if (!full) {
+    count_launch();
+    k_reset_occ<<<c->num_sms * 4, 256, 0, s>>>(c->t);
+  }
   cudaMemsetAsync(c->t.glob, 0, 8 * 8, s);
   if (c->bm_words) {
     cudaMemsetAsync(c->t.W, 0, c->bm_words * 4, s);
     cudaMemsetAsync(c->t.L, 0, c->bm_words * 4, s);
   }
-  cudaMemsetAsync(c->t.hslot, 0xFF, c->hcap * sizeof(HSlot), s);
+  if (full) cudaMemsetAsync(c->t.hslot, 0xFF, c->hcap * sizeof(HSlot), s);
   if (c->n_obj) {
     cudaMemcpyAsync(c->o.dense_pc, c->dense_pc_init.data(), 4ull * DENSE_PER_OBJ * c->n_obj, cudaMemcpyHostToDevice, s);
     cudaMemsetAsync(c->o.dense_off, 0xFF, 8ull * DENSE_PER_OBJ * c->n_obj, s);   // DENSE_NOT_READY
   }
   c->records_analyzed = 0;
-  cudaError_t e = cudaMemsetAsync(c->t.hcount, 0, c->hcap * 8, s);
+  cudaError_t e = full ? cudaMemsetAsync(c->t.hcount, 0, c->hcap * 8, s) : cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "reset");
+  c->table_clean = true;
+  if (c->reset_ev) cudaEventRecord(c->reset_ev, s);
   c->poisoned = false;
   c->hist_merged = false;
   c->merged_ndistinct.clear();
@@ -199,6 +223,7 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
   }
+  if (cfg->hist_capacity > (1ull << 32)) return VE_ERR_INVALID;   // (slot indices are 32-bit)
   uint64_t hcap = 1024;
   while (hcap < cfg->hist_capacity) hcap <<= 1;
   c->hcap = hcap;
@@ -211,7 +236,8 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
             cudaMalloc(&c->t.lcta, (size_t)c->num_sms * K1_NSK * sizeof(LineState)) == cudaSuccess &&
             cudaMalloc(&c->t.glob, 8 * 8) == cudaSuccess &&
             cudaMalloc(&c->t.hslot, hcap * sizeof(HSlot)) == cudaSuccess &&
-            cudaMalloc(&c->t.hcount, hcap * 8) == cudaSuccess;
+            cudaMalloc(&c->t.hcount, hcap * 8) == cudaSuccess &&
+            cudaMalloc(&c->t.occ, hcap * 4) == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
     free_dev(c);
@@ -220,6 +246,7 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
   }
   c->n_obj = 0;
   c->n_keys = cfg->n_pcs + 1;
+  if (cudaEventCreateWithFlags(&c->reset_ev, cudaEventDisableTiming) != cudaSuccess) c->reset_ev = nullptr;
   if (launch_reset(c, 0) != VE_OK || cudaDeviceSynchronize() != cudaSuccess) {
     free_dev(c);
     delete c;
@@ -324,9 +351,7 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     c->obj_block_bytes = 0;
     if (cudaMalloc(&c->obj_block, nb) != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "objects"); }
     c->obj_block_bytes = nb;
-  } else {
-    cudaDeviceSynchronize();
-  }
+  }   // (else: the block is reused -- the device was made idle above)
   std::vector<uint8_t> host(nb, 0);
   uint64_t* hb = (uint64_t*)host.data();
   uint64_t* he = hb + n;
@@ -362,11 +387,9 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   c->objs = v;
   c->n_obj = n;
   c->n_keys = c->cfg.n_pcs + n + 1;
-  ve_status st = launch_reset(c, 0);
-  if (st != VE_OK) return st;
-  cudaError_t e = cudaDeviceSynchronize();
-  if (e != cudaSuccess) return cuda_fail(c, e, "ve_set_objects");
-  return VE_OK;
+  // the reset runs on the legacy stream; the analysis / diff calls wait for its event on their
+  // stream (no host synchronisation per object set)
+  return launch_reset(c, 0);
 }
 
 ve_status ve_reset(ve_ctx* c) {

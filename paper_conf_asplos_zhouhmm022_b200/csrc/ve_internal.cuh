@@ -62,8 +62,10 @@ struct DevTables {
   HSlot* hslot;             // [hcap]
   unsigned long long* hcount;  // [hcap]
   uint64_t hmask;           // hcap - 1
+  uint32_t* occ;            // [hcap] indices of the occupied slots, in claim order (glob[G_NOCC] of them);
+                            // null for temporary tables: the report and the reset walk only these
 };
-enum : int { G_RECORDS = 0, G_INVALID = 1, G_UNMAPPED = 2, G_OVERFLOW = 3, G_WORK = 7 };  // 7: K1 chunk counter
+enum : int { G_RECORDS = 0, G_INVALID = 1, G_UNMAPPED = 2, G_OVERFLOW = 3, G_NOCC = 5, G_WORK = 7 };  // 7: K1 chunk counter
 
 struct DevObjects {          // sorted by base
   const uint64_t* base;
@@ -113,6 +115,8 @@ struct ve_ctx {
   std::string err;
   bool poisoned = false;
   bool hist_merged = false;  // set by an NCCL merge: top-k/n_distinct precomputed
+  bool table_clean = false;  // the value table holds only the slots recorded in t.occ (else: full clear)
+  cudaEvent_t reset_ev = nullptr;   // recorded after every reset (legacy stream); launches on s wait on it
   uint32_t n_obj = 0;
   uint32_t n_keys = 0;
   std::vector<ve::HostObject> objs;          // sorted by base
@@ -410,7 +414,12 @@ __device__ __forceinline__ bool hist_insert_global(const DevTables& t, uint32_t 
     HSlot* s = &t.hslot[h];
     uint64_t olo, ohi;
     cas128_global(s, ~0ull, ~0ull, bits, (uint64_t)tag, olo, ohi);
-    if ((olo == ~0ull && ohi == ~0ull) || (olo == bits && ohi == (uint64_t)tag)) {
+    if (olo == ~0ull && ohi == ~0ull) {          // claimed: record the slot
+      if (t.occ) t.occ[atomicAdd(&t.glob[G_NOCC], 1ull)] = (uint32_t)h;
+      atomicAdd(&t.hcount[h], cnt);
+      return true;
+    }
+    if (olo == bits && ohi == (uint64_t)tag) {
       atomicAdd(&t.hcount[h], cnt);
       return true;
     }
@@ -443,7 +452,12 @@ __device__ __forceinline__ bool hist_insert_global_rf(const DevTables& t, uint32
     if (lo == ~0ull || lo == bits) {
       uint64_t olo, ohi;
       cas128_global(s, ~0ull, ~0ull, bits, (uint64_t)tag, olo, ohi);
-      if ((olo == ~0ull && ohi == ~0ull) || (olo == bits && ohi == (uint64_t)tag)) {
+      if (olo == ~0ull && ohi == ~0ull) {        // claimed: record the slot
+        if (t.occ) t.occ[atomicAdd(&t.glob[G_NOCC], 1ull)] = (uint32_t)h;
+        atomicAdd(&t.hcount[h], cnt);
+        return true;
+      }
+      if (olo == bits && ohi == (uint64_t)tag) {
         atomicAdd(&t.hcount[h], cnt);
         return true;
       }
