@@ -240,6 +240,30 @@ ve_status ve_approx_topk(ve_ctx* ctx, uint64_t* h_ndistinct, ve_topk_entry* h_to
 typedef struct ve_dyadic { uint32_t state, scale; uint64_t px, qx; int64_t py, qy; } ve_dyadic;
 ve_status ve_dyadic_fit(ve_ctx* ctx, const ve_record* d_records, uint64_t n, ve_dyadic* h_out, cudaStream_t s);
 
+/* ---- approximate structured and structured with <= eps outliers ----
+ * The paper's approximate patterns cover "some fine-grained patterns" (Def 3.8,
+ * P:L191) without a definition, and Table 1 marks srad_v1 structured
+ * although its clamped boundary breaks an exact fit (Def 3.7).
+ *   ve_dyadic_fit_ex(flags = VE_FIT_TRUNC): C22 (R11) -- C21 over the
+ *     values every float record carries after Def 3.8's truncation to
+ *     cfg.mant_bits mantissa bits (toward zero); integers unchanged.  flags 0 is
+ *     ve_dyadic_fit.
+ *   ve_outlier_fit: C23 (R12) -- per key, points as in C21 (with
+ *     VE_FIT_TRUNC: truncated first); the line through the INTERIOR anchors A =
+ *     (second-smallest distinct address, smallest Y there) and B = (second-largest
+ *     distinct address, smallest Y there); n_off = records off it (exact 128-bit
+ *     check), n = records.  state FAIL (NaN / inf, |Y| >= 2^62), EMPTY, POINT
+ *     (fewer than 4 distinct addresses), LINE.  "Structured with <= eps outliers"
+ *     is LINE with ay != by and 100 n_off <= eps_pct n.
+ * Both: device records (8-byte aligned), h_out[n_keys] host; four (C23) or three
+ * streaming passes; synchronize s. */
+enum { VE_FIT_TRUNC = 1 };
+typedef struct ve_outlier { uint32_t state, scale; uint64_t ax, bx; int64_t ay, by; uint64_t n_off, n; } ve_outlier;
+ve_status ve_dyadic_fit_ex(ve_ctx* ctx, const ve_record* d_records, uint64_t n, uint32_t flags, ve_dyadic* h_out,
+                           cudaStream_t s);
+ve_status ve_outlier_fit(ve_ctx* ctx, const ve_record* d_records, uint64_t n, uint32_t flags, ve_outlier* h_out,
+                         cudaStream_t s);
+
 /* ---- accessed intervals and the adaptive copy plan --------
  * PAPER.md section 6.1: "We define an interval [start, end] as
  * the memory range accessed by each GPU instruction" and merge intervals "if

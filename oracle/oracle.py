@@ -233,6 +233,36 @@ def dyadic_fit(cfg, objs, recs):
     return out
 
 
+def dyadic_fit_trunc(cfg, objs, recs):
+    """C22 (f2): DYADIC_DTYPE[n_keys] -- C21 over the float values truncated to K mantissa bits."""
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    out = np.zeros(cfg.n_pcs + len(objs) + 1, dtype=DYADIC_DTYPE)
+    L = lib()
+    L.vo_dyadic_fit_trunc.argtypes = [ctypes.POINTER(VoConfig), ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+                                      ctypes.c_uint64, ctypes.c_void_p]
+    if L.vo_dyadic_fit_trunc(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), out.ctypes.data) != 0:
+        raise ValueError("vo_dyadic_fit_trunc rejected its arguments")
+    return out
+
+
+OUTLIER_DTYPE = np.dtype([("state", "<u4"), ("scale", "<u4"), ("ax", "<u8"), ("bx", "<u8"), ("ay", "<i8"),
+                          ("by", "<i8"), ("n_off", "<u8"), ("n", "<u8")])
+
+
+def outlier_fit(cfg, objs, recs, flags=0):
+    """C23 (f2): OUTLIER_DTYPE[n_keys] -- the interior-anchor line and the records off it."""
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    out = np.zeros(cfg.n_pcs + len(objs) + 1, dtype=OUTLIER_DTYPE)
+    L = lib()
+    L.vo_outlier_fit.argtypes = [ctypes.POINTER(VoConfig), ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+                                 ctypes.c_uint64, ctypes.c_uint32, ctypes.c_void_p]
+    if L.vo_outlier_fit(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), flags, out.ctypes.data) != 0:
+        raise ValueError("vo_outlier_fit rejected its arguments")
+    return out
+
+
 # ---- C18-C20: value flow graph (layouts of ve.h's ve_api_access / ve_vfg_edge / ve_vfg_vertex)
 HOST_VERTEX = 0xFFFFFFFF
 ACCESS_DTYPE = np.dtype([("seq", "<u8"), ("bytes", "<u8"), ("vertex", "<u4"), ("object", "<u4"), ("mode", "<u4"),

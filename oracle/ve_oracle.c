@@ -1040,3 +1040,188 @@ int vo_dyadic_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, c
   free(t.by_base);
   return 0;
 }
+
+/* ---- C22: approximate structured (f2; Def 3.7 over Def 3.8's truncated values) ----------------
+ * DESIGN.md reading R11 (SURVEY 8(f) f2 "approximate structured").  Exactly C21 (vo_dyadic_fit),
+ * step for step, over the values every float record carries after Def 3.8's truncation to K
+ * mantissa bits (C7: clear the low m-K mantissa bits, toward zero); integer records unchanged.
+ * A NaN or infinity in the record fails the key (truncation keeps a finite value finite). */
+static int trunc_exact_value(uint64_t b, uint32_t kind, uint32_t w, uint32_t K, int trunc, int64_t* M, int* E) {
+  if (trunc && kind >= 2) {
+    int64_t m0;
+    int e0;
+    if (!exact_value(b, kind, w, &m0, &e0)) return 0;      /* NaN / inf in the record itself */
+    b = vo_trunc(b, kind, w, K);
+  }
+  return exact_value(b, kind, w, M, E);
+}
+
+int vo_dyadic_fit_trunc(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                        uint64_t n, vo_dyadic* out) {
+  if (!cfg || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t n_keys = (uint64_t)cfg->n_pcs + n_obj + 1;
+  int* have = (int*)calloc(n_keys, sizeof(int));
+  int* fail = (int*)calloc(n_keys, sizeof(int));
+  int* T = (int*)calloc(n_keys, sizeof(int));
+  int* hp = (int*)calloc(n_keys, sizeof(int));
+  int* hq = (int*)calloc(n_keys, sizeof(int));
+  i128* py = (i128*)calloc(n_keys, sizeof(i128));
+  i128* qy = (i128*)calloc(n_keys, sizeof(i128));
+  memset(out, 0, sizeof(vo_dyadic) * n_keys);
+  for (int pass = 1; pass <= 3; ++pass) {
+    for (uint64_t i = 0; i < n; ++i) {
+      const vo_record* r = &recs[i];
+      dec_t d;
+      decode(cfg, &t, r, &d);
+      if (!d.valid) continue;
+      uint64_t kset[2];
+      int nk = 0;
+      kset[nk++] = r->pc;
+      if (d.shared) kset[nk++] = (uint64_t)cfg->n_pcs + n_obj;
+      else if (d.obj) kset[nk++] = (uint64_t)cfg->n_pcs + d.obj->id;
+      int64_t M = 0;
+      int E = 0;
+      const int finite = trunc_exact_value(r->value, d.kind, d.w, cfg->mant_bits, 1, &M, &E);
+      for (int j = 0; j < nk; ++j) {
+        const uint64_t k = kset[j];
+        vo_dyadic* o = &out[k];
+        if (pass == 1) {
+          if (!finite) { fail[k] = 1; continue; }
+          if (-E > T[k]) T[k] = -E;
+          if (!have[k] || r->addr < o->px) o->px = r->addr;
+          if (!have[k] || r->addr > o->qx) o->qx = r->addr;
+          have[k] = 1;
+          continue;
+        }
+        if (fail[k]) continue;
+        i128 Y;
+        if (!scaled_y(M, E + T[k], &Y)) { fail[k] = 1; continue; }
+        if (pass == 2) {
+          if (r->addr == o->px && (!hp[k] || Y < py[k])) { py[k] = Y; hp[k] = 1; }
+          if (r->addr == o->qx && (!hq[k] || Y < qy[k])) { qy[k] = Y; hq[k] = 1; }
+        } else if (!collinear((i128)o->px, py[k], (i128)o->qx, qy[k], (i128)r->addr, Y) ||
+                   (r->addr == o->px && Y != py[k]) || (r->addr == o->qx && Y != qy[k])) {
+          fail[k] = 1;
+        }
+      }
+    }
+  }
+  for (uint64_t k = 0; k < n_keys; ++k) {
+    vo_dyadic* o = &out[k];
+    if (fail[k] || !have[k]) {
+      memset(o, 0, sizeof(*o));
+      o->state = fail[k] ? VO_LINE_FAIL : VO_LINE_EMPTY;
+      continue;
+    }
+    o->state = (o->px == o->qx) ? VO_LINE_POINT : VO_LINE_LINE;
+    o->scale = (uint32_t)T[k];
+    o->py = (int64_t)py[k];
+    o->qy = (int64_t)qy[k];
+  }
+  free(hp); free(hq);
+  free(have); free(fail); free(T); free(py); free(qy);
+  free(t.by_base);
+  return 0;
+}
+
+/* ---- C23: structured with <= eps outliers (f2; Def 3.7, srad_v1's clamped boundary) -----------
+ * DESIGN.md reading R12.  Points as in C21 (x = addr, exact value y, Y = y 2^T; with flags & 1 the
+ * float values truncated as in C22).  Steps, in order:
+ *  1. NaN or infinity -> FAIL; T = max fractional bits; x1 = min x, xm = max x;
+ *  2. x2 = the smallest x above x1, x_(m-1) = the largest x below xm (distinct addresses);
+ *     |Y| >= 2^62 -> FAIL;
+ *  3. interior anchors A = (x2, smallest Y at x2), B = (x_(m-1), smallest Y at x_(m-1));
+ *  4. n_off = the records NOT collinear with A and B (exact 128-bit cross product), n = records.
+ * State: FAIL (steps 1-2), EMPTY (no record), POINT (fewer than 4 distinct x: no interior line),
+ * else LINE.  The flag "structured with <= eps outliers" is LINE with A.Y != B.Y and
+ * 100 n_off <= eps_pct n (the report's integer test; eps_pct a caller parameter). */
+/* (vo_outlier: ve_oracle.h) */
+
+int vo_outlier_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs, uint64_t n,
+                   uint32_t flags, vo_outlier* out) {
+  if (!cfg || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t n_keys = (uint64_t)cfg->n_pcs + n_obj + 1;
+  int* have = (int*)calloc(n_keys, sizeof(int));
+  int* fail = (int*)calloc(n_keys, sizeof(int));
+  int* T = (int*)calloc(n_keys, sizeof(int));
+  uint64_t* x1 = (uint64_t*)calloc(n_keys, sizeof(uint64_t));
+  uint64_t* xm = (uint64_t*)calloc(n_keys, sizeof(uint64_t));
+  uint64_t* x2 = (uint64_t*)calloc(n_keys, sizeof(uint64_t));
+  uint64_t* xl = (uint64_t*)calloc(n_keys, sizeof(uint64_t));
+  int* h2 = (int*)calloc(n_keys, sizeof(int));
+  int* hl = (int*)calloc(n_keys, sizeof(int));
+  int* ha = (int*)calloc(n_keys, sizeof(int));
+  int* hb = (int*)calloc(n_keys, sizeof(int));
+  i128* ay = (i128*)calloc(n_keys, sizeof(i128));
+  i128* by = (i128*)calloc(n_keys, sizeof(i128));
+  memset(out, 0, sizeof(vo_outlier) * n_keys);
+  for (int pass = 1; pass <= 4; ++pass) {
+    for (uint64_t i = 0; i < n; ++i) {
+      const vo_record* r = &recs[i];
+      dec_t d;
+      decode(cfg, &t, r, &d);
+      if (!d.valid) continue;
+      uint64_t kset[2];
+      int nk = 0;
+      kset[nk++] = r->pc;
+      if (d.shared) kset[nk++] = (uint64_t)cfg->n_pcs + n_obj;
+      else if (d.obj) kset[nk++] = (uint64_t)cfg->n_pcs + d.obj->id;
+      int64_t M = 0;
+      int E = 0;
+      const int finite = trunc_exact_value(r->value, d.kind, d.w, cfg->mant_bits, (int)(flags & 1u), &M, &E);
+      for (int j = 0; j < nk; ++j) {
+        const uint64_t k = kset[j];
+        if (pass == 1) {                                   /* step 1 */
+          if (!finite) { fail[k] = 1; continue; }
+          if (-E > T[k]) T[k] = -E;
+          if (!have[k] || r->addr < x1[k]) x1[k] = r->addr;
+          if (!have[k] || r->addr > xm[k]) xm[k] = r->addr;
+          have[k] = 1;
+          out[k].n++;
+          continue;
+        }
+        if (fail[k]) continue;
+        i128 Y;
+        if (!scaled_y(M, E + T[k], &Y)) { fail[k] = 1; continue; }
+        if (pass == 2) {                                   /* step 2 */
+          if (r->addr > x1[k] && (!h2[k] || r->addr < x2[k])) { x2[k] = r->addr; h2[k] = 1; }
+          if (r->addr < xm[k] && (!hl[k] || r->addr > xl[k])) { xl[k] = r->addr; hl[k] = 1; }
+        } else if (pass == 3) {                            /* step 3 */
+          if (h2[k] && r->addr == x2[k] && (!ha[k] || Y < ay[k])) { ay[k] = Y; ha[k] = 1; }
+          if (hl[k] && r->addr == xl[k] && (!hb[k] || Y < by[k])) { by[k] = Y; hb[k] = 1; }
+        } else if (h2[k] && hl[k] && x2[k] < xl[k]) {      /* step 4 */
+          if (!collinear((i128)x2[k], ay[k], (i128)xl[k], by[k], (i128)r->addr, Y)) out[k].n_off++;
+        }
+      }
+    }
+  }
+  for (uint64_t k = 0; k < n_keys; ++k) {
+    vo_outlier* o = &out[k];
+    if (fail[k] || !have[k]) {
+      memset(o, 0, sizeof(*o));
+      o->state = fail[k] ? VO_LINE_FAIL : VO_LINE_EMPTY;
+      continue;
+    }
+    o->scale = (uint32_t)T[k];
+    if (!(h2[k] && hl[k] && x2[k] < xl[k])) {
+      const uint64_t nn = o->n;
+      memset(o, 0, sizeof(*o));
+      o->state = VO_LINE_POINT;
+      o->n = nn;
+      continue;
+    }
+    o->state = VO_LINE_LINE;
+    o->ax = x2[k];
+    o->bx = xl[k];
+    o->ay = (int64_t)ay[k];
+    o->by = (int64_t)by[k];
+  }
+  free(have); free(fail); free(T); free(x1); free(xm); free(x2); free(xl); free(h2); free(hl); free(ha); free(hb);
+  free(ay); free(by);
+  free(t.by_base);
+  return 0;
+}

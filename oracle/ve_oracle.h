@@ -203,6 +203,17 @@ typedef struct vo_dyadic { uint32_t state, scale; uint64_t px, qx; int64_t py, q
 int vo_dyadic_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs, uint64_t n,
                   vo_dyadic* out);
 
+/* ---- approximate structured (C22) and structured with <= eps outliers (C23) ----
+ * C22: C21 over the float values truncated to K mantissa bits (Def 3.8 over Def 3.7; R11).
+ * C23: anchors at the second-smallest and second-largest distinct address (min Y there), n_off =
+ * records off that line, n = records (R12); flags & 1: the C22 truncation first.
+ * State FAIL on NaN / inf or |Y| >= 2^62, EMPTY, POINT (< 4 distinct addresses), LINE. */
+int vo_dyadic_fit_trunc(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                        uint64_t n, vo_dyadic* out);
+typedef struct vo_outlier { uint32_t state, scale; uint64_t ax, bx; int64_t ay, by; uint64_t n_off, n; } vo_outlier;
+int vo_outlier_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs, uint64_t n,
+                   uint32_t flags, vo_outlier* out);
+
 /* helpers exposed for pinning */
 uint64_t vo_ord(uint64_t b, uint32_t kind, uint32_t w);
 uint32_t vo_float_flags(uint64_t b, uint32_t kind, uint32_t w);   /* bit0 nan, 1 nonint, 2 not_f16, 3 not_bf16, 4 not_f32 */

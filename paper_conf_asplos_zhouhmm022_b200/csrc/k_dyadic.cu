@@ -27,11 +27,21 @@ constexpr uint32_t DY_T = 256;
 constexpr uint32_t DY_SK = 512;
 constexpr unsigned long long DY_NONE = ~0ull;
 
-struct DyKey {                  // global per-key state (32 B)
+struct DyKey {                  // global per-key state
   unsigned int T, fail;
   unsigned long long minx, maxx;
   unsigned long long py, qy;    // Y + 2^63 (order-preserving), DY_NONE = no anchor yet
+  unsigned long long x2, xl;    // C23: second-smallest / second-largest distinct address (DY_NONE / 0: none)
+  unsigned long long n, n_off;  // C23: records, records off the interior line
 };
+constexpr uint32_t DY_NOTRUNC = 0xFFFFFFFFu;
+
+// C22 / C23 with truncation: the value a float record carries after Def 3.8's truncation (C7);
+// a NaN / inf stays non-finite (its exponent is kept), so dy_exact still fails it
+__device__ __forceinline__ uint64_t dy_value(uint64_t b, uint32_t meta, uint32_t tr) {
+  const uint32_t kind = meta_kind(meta);
+  return (tr != DY_NOTRUNC && kind >= 2u) ? trunc_bits(b, kind, meta_lg(meta), tr) : b;
+}
 
 // exact value of the bits as M 2^E with M odd or zero; false for NaN / inf.  Unsigned values
 // >= 2^63 report M = 2^62 (they fail the |Y| < 2^62 bound for any T).
@@ -119,7 +129,7 @@ __device__ __forceinline__ bool dy_load(const ve_record* r, uint64_t i, const De
 }
 
 __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n, DevObjects o, uint32_t n_pcs,
-                                                  uint32_t nk, DyKey* K) {
+                                                  uint32_t nk, DyKey* K, uint32_t tr) {
   __shared__ unsigned int sT[DY_SK], sF[DY_SK];
   __shared__ unsigned long long sMin[DY_SK], sMax[DY_SK];
   const uint32_t ns = nk < DY_SK ? nk : DY_SK;
@@ -134,7 +144,7 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
     const bool act = i < n && dy_load(r, i, o, n_pcs, d, oc);
     long long M = 0;
     int E = 0;
-    const bool fin = act && dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E);
+    const bool fin = act && dy_exact(dy_value(d.v, d.meta, tr), meta_kind(d.meta), meta_lg(d.meta), M, E);
     unsigned int t = (fin && E < 0) ? (unsigned int)(-E) : 0u;
     for (uint32_t j = 0; j < 2; ++j) {
       const uint32_t k = j < d.nk ? d.k[j] : 0xFFFFFFFFu;
@@ -156,6 +166,7 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
         tt = __reduce_max_sync(0xFFFFFFFFu, tt);
         ff = __reduce_or_sync(0xFFFFFFFFu, ff);
         hv = __reduce_or_sync(0xFFFFFFFFu, hv);
+        if ((threadIdx.x & 31u) == 0u) atomicAdd(&K[k].n, 32ull);   // (C23's record count)
         if ((threadIdx.x & 31u) == 0u) {
           if (k < ns) {
             if (ff) sF[k] = 1u;
@@ -176,6 +187,7 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
         continue;
       }
       if (k == 0xFFFFFFFFu) continue;
+      atomicAdd(&K[k].n, 1ull);
       if (k < ns) {
         if (!fin) { sF[k] = 1u; continue; }
         if (t) atomicMax(&sT[k], t);
@@ -199,9 +211,11 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
   }
 }
 
-// D2 (anchors and the |Y| bound) when pass == 0, D3 (collinearity) when pass == 1
+// C21: D2 (anchors and the |Y| bound) when pass == 0, D3 (collinearity) when pass == 1;
+// C23: the second extreme addresses and the |Y| bound (2), the interior anchors (3), the records
+// off the interior line (4)
 __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t n, DevObjects o, uint32_t n_pcs,
-                                                   DyKey* K, int pass) {
+                                                   DyKey* K, int pass, uint32_t tr) {
   DyObjCache oc;
   for (uint64_t i = (uint64_t)blockIdx.x * DY_T + threadIdx.x; i < n; i += (uint64_t)gridDim.x * DY_T) {
     DyRec d;
@@ -213,14 +227,21 @@ __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t 
         any |= d.x == k.minx || d.x == k.maxx;
       }
       if (!any) continue;
-    } else {                               // D3: nothing left to check once every key of the record failed
+    } else if (pass == 3) {                // C23 anchors: only the records at the interior anchors
+      bool any = false;
+      for (uint32_t j = 0; j < d.nk; ++j) {
+        const DyKey& k = K[d.k[j]];
+        any |= d.x == k.x2 || d.x == k.xl;
+      }
+      if (!any) continue;
+    } else {                               // nothing left to check once every key of the record failed
       bool any = false;
       for (uint32_t j = 0; j < d.nk; ++j) any |= K[d.k[j]].fail == 0u;
       if (!any) continue;
     }
     long long M;
     int E;
-    if (!dy_exact(d.v, meta_kind(d.meta), meta_lg(d.meta), M, E)) continue;   // its keys failed in D1
+    if (!dy_exact(dy_value(d.v, d.meta, tr), meta_kind(d.meta), meta_lg(d.meta), M, E)) continue;   // failed in D1
     for (uint32_t j = 0; j < d.nk; ++j) {
       DyKey& k = K[d.k[j]];
       if (k.fail) continue;                  // a stale 0 only costs the check below
@@ -230,6 +251,23 @@ __global__ void __launch_bounds__(DY_T) k_dy_check(const ve_record* r, uint64_t 
       if (pass == 0) {
         if (d.x == k.minx) atomicMin(&k.py, yo);
         if (d.x == k.maxx) atomicMin(&k.qy, yo);
+        continue;
+      }
+      if (pass == 2) {                       // C23 step 2
+        if (d.x > k.minx) atomicMin(&k.x2, (unsigned long long)d.x);
+        if (d.x < k.maxx) atomicMax(&k.xl, (unsigned long long)d.x);
+        continue;
+      }
+      if (pass == 3) {                       // C23 step 3 (py / qy hold the interior anchors' Y)
+        if (d.x == k.x2) atomicMin(&k.py, yo);
+        if (d.x == k.xl) atomicMin(&k.qy, yo);
+        continue;
+      }
+      if (pass == 4) {                       // C23 step 4
+        if (!(k.x2 != DY_NONE && k.x2 < k.xl)) continue;
+        const long long ay = (long long)(k.py ^ (1ull << 63)), by = (long long)(k.qy ^ (1ull << 63));
+        const __int128 dx = (__int128)(long long)(d.x - k.x2), bxa = (__int128)(long long)(k.xl - k.x2);
+        if ((__int128)(Y - ay) * bxa != (__int128)(by - ay) * dx) atomicAdd(&k.n_off, 1ull);
         continue;
       }
       const long long py = (long long)(k.py ^ (1ull << 63)), qy = (long long)(k.qy ^ (1ull << 63));
@@ -246,6 +284,8 @@ __global__ void k_dy_init(DyKey* K, uint32_t nk) {
     K[k].T = 0; K[k].fail = 0;
     K[k].minx = DY_NONE; K[k].maxx = 0;
     K[k].py = DY_NONE; K[k].qy = DY_NONE;
+    K[k].x2 = DY_NONE; K[k].xl = 0;
+    K[k].n = 0; K[k].n_off = 0;
   }
 }
 
@@ -253,15 +293,14 @@ __global__ void k_dy_init(DyKey* K, uint32_t nk) {
 
 using namespace ve;
 
-extern "C" ve_status ve_dyadic_fit(ve_ctx* c, const ve_record* d_records, uint64_t n, ve_dyadic* h_out,
-                                   cudaStream_t s) {
-  if (!c || !h_out) return VE_ERR_INVALID;
+static ve_status dy_run(ve_ctx* c, const ve_record* d_records, uint64_t n, uint32_t tr, bool outlier,
+                        std::vector<DyKey>& hk, cudaStream_t s) {
   const uint32_t nk = c->n_keys;
-  if (n && (!d_records || ((uintptr_t)d_records & 7))) return fail(c, VE_ERR_INVALID, "ve_dyadic_fit: null or misaligned");
+  if (n && (!d_records || ((uintptr_t)d_records & 7))) return fail(c, VE_ERR_INVALID, "fit: null or misaligned records");
   cudaSetDevice(c->device);
   DyKey* K = nullptr;
   cudaError_t e = cudaMallocAsync((void**)&K, sizeof(DyKey) * (size_t)nk, s);
-  if (e != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "ve_dyadic_fit: workspace"); }
+  if (e != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "fit: workspace"); }
   count_launch();
   k_dy_init<<<(nk + 255) / 256, 256, 0, s>>>(K, nk);
   if (n) {
@@ -269,18 +308,29 @@ extern "C" ve_status ve_dyadic_fit(ve_ctx* c, const ve_record* d_records, uint64
     const uint64_t cap = (uint64_t)c->num_sms * 8;
     const unsigned grid = (unsigned)(b < cap ? b : cap);
     count_launch();
-    k_dy_scan<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, nk, K);
-    count_launch();
-    k_dy_check<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, K, 0);
-    count_launch();
-    k_dy_check<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, K, 1);
+    k_dy_scan<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, nk, K, tr);
+    const int passes[2][3] = {{0, 1, -1}, {2, 3, 4}};
+    for (int p : passes[outlier ? 1 : 0]) {
+      if (p < 0) continue;
+      count_launch();
+      k_dy_check<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, K, p, tr);
+    }
   }
-  std::vector<DyKey> hk(nk);
+  hk.resize(nk);
   e = cudaMemcpyAsync(hk.data(), K, sizeof(DyKey) * (size_t)nk, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   cudaFreeAsync(K, s);
-  if (e != cudaSuccess) return cuda_fail(c, e, "ve_dyadic_fit");
-  for (uint32_t k = 0; k < nk; ++k) {
+  if (e != cudaSuccess) return cuda_fail(c, e, "fit");
+  return VE_OK;
+}
+
+extern "C" ve_status ve_dyadic_fit_ex(ve_ctx* c, const ve_record* d_records, uint64_t n, uint32_t flags,
+                                      ve_dyadic* h_out, cudaStream_t s) {
+  if (!c || !h_out || (flags & ~VE_FIT_TRUNC)) return VE_ERR_INVALID;
+  std::vector<DyKey> hk;
+  ve_status st = dy_run(c, d_records, n, (flags & VE_FIT_TRUNC) ? c->cfg.mant_bits : DY_NOTRUNC, false, hk, s);
+  if (st != VE_OK) return st;
+  for (uint32_t k = 0; k < c->n_keys; ++k) {
     ve_dyadic& o = h_out[k];
     o = ve_dyadic{};
     if (hk[k].fail) { o.state = VE_LINE_FAIL; continue; }
@@ -291,6 +341,35 @@ extern "C" ve_status ve_dyadic_fit(ve_ctx* c, const ve_record* d_records, uint64
     o.qx = hk[k].maxx;
     o.py = (int64_t)(hk[k].py ^ (1ull << 63));
     o.qy = (int64_t)(hk[k].qy ^ (1ull << 63));
+  }
+  return VE_OK;
+}
+
+extern "C" ve_status ve_dyadic_fit(ve_ctx* c, const ve_record* d_records, uint64_t n, ve_dyadic* h_out,
+                                   cudaStream_t s) {
+  return ve_dyadic_fit_ex(c, d_records, n, 0u, h_out, s);
+}
+
+extern "C" ve_status ve_outlier_fit(ve_ctx* c, const ve_record* d_records, uint64_t n, uint32_t flags,
+                                    ve_outlier* h_out, cudaStream_t s) {
+  if (!c || !h_out || (flags & ~VE_FIT_TRUNC)) return VE_ERR_INVALID;
+  std::vector<DyKey> hk;
+  ve_status st = dy_run(c, d_records, n, (flags & VE_FIT_TRUNC) ? c->cfg.mant_bits : DY_NOTRUNC, true, hk, s);
+  if (st != VE_OK) return st;
+  for (uint32_t k = 0; k < c->n_keys; ++k) {
+    ve_outlier& o = h_out[k];
+    o = ve_outlier{};
+    if (hk[k].fail) { o.state = VE_LINE_FAIL; continue; }
+    if (hk[k].minx == DY_NONE) { o.state = VE_LINE_EMPTY; continue; }
+    o.n = hk[k].n;
+    o.scale = hk[k].T;
+    if (!(hk[k].x2 != DY_NONE && hk[k].x2 < hk[k].xl)) { o.state = VE_LINE_POINT; o.scale = 0; continue; }
+    o.state = VE_LINE_LINE;
+    o.ax = hk[k].x2;
+    o.bx = hk[k].xl;
+    o.ay = (int64_t)(hk[k].py ^ (1ull << 63));
+    o.by = (int64_t)(hk[k].qy ^ (1ull << 63));
+    o.n_off = hk[k].n_off;
   }
   return VE_OK;
 }

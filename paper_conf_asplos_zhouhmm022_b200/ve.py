@@ -53,6 +53,9 @@ DIFF_DTYPE = np.dtype([(f, "<u8") for f in ("n_elems", "n_masked", "n_unchanged"
 
 DYADIC_DTYPE = np.dtype([("state", "<u4"), ("scale", "<u4"), ("px", "<u8"), ("qx", "<u8"), ("py", "<i8"),
                          ("qy", "<i8")])
+OUTLIER_DTYPE = np.dtype([("state", "<u4"), ("scale", "<u4"), ("ax", "<u8"), ("bx", "<u8"), ("ay", "<i8"),
+                          ("by", "<i8"), ("n_off", "<u8"), ("n", "<u8")])
+FIT_TRUNC = 1
 
 
 class VeError(RuntimeError):
@@ -121,6 +124,8 @@ def lib():
             "ve_record_intervals": ([vp, vp, u64, vp, ctypes.POINTER(u64), vp], st),
             "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
             "ve_snapshot_diff_all": ([vp, u32, vp, vp, vp], st),
+            "ve_dyadic_fit_ex": ([vp, vp, u64, u32, vp, vp], st),
+            "ve_outlier_fit": ([vp, vp, u64, u32, vp, vp], st),
             "ve_object_dedup_comm": ([vp, vp, u32, vp, vp, vp], st),
             "ve_snapshot_diff_all_group": ([ctypes.POINTER(vp), u32, u32, vp, vp], st),
             "ve_object_dedup_group": ([ctypes.POINTER(vp), u32, vp, u32, vp, vp], st),
@@ -434,6 +439,22 @@ class Context:
         out = np.zeros(nk, dtype=DYADIC_DTYPE)
         self._check(lib().ve_dyadic_fit(self._h, _ptr(d_records), n, out.ctypes.data, _stream(stream)),
                     "ve_dyadic_fit")
+        return out
+
+    def dyadic_fit_trunc(self, d_records, n, stream=None):
+        """ve_dyadic_fit_ex(VE_FIT_TRUNC): C22, the fit over the K-bit truncated float values (f2)."""
+        nk = self.n_pcs + getattr(self, "n_objects", 0) + 1
+        out = np.zeros(nk, dtype=DYADIC_DTYPE)
+        self._check(lib().ve_dyadic_fit_ex(self._h, _ptr(d_records), n, FIT_TRUNC, out.ctypes.data, _stream(stream)),
+                    "ve_dyadic_fit_ex")
+        return out
+
+    def outlier_fit(self, d_records, n, flags=0, stream=None):
+        """ve_outlier_fit: C23, OUTLIER_DTYPE[n_keys] -- interior-anchor line and records off it (f2)."""
+        nk = self.n_pcs + getattr(self, "n_objects", 0) + 1
+        out = np.zeros(nk, dtype=OUTLIER_DTYPE)
+        self._check(lib().ve_outlier_fit(self._h, _ptr(d_records), n, flags, out.ctypes.data, _stream(stream)),
+                    "ve_outlier_fit")
         return out
 
     def temporal_loads(self, d_records, n, stream=None):
