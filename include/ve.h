@@ -209,6 +209,12 @@ ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
  * ctx's object table).  Order-dependent: one call covers one ordered trace.
  * n < 2^32.  Synchronizes s. */
 ve_status ve_temporal_loads(ve_ctx* ctx, const ve_record* d_records, uint64_t n, uint64_t* h_out, cudaStream_t s);
+/* The same, plus the per-(PC, object) table (Table 5's redundancy analysis P:L470 per
+ * instruction AND data object): h_pairs[2 (pc (n_objects + 1) + id)] = temporal, + 1 =
+ * redundant loads of PC pc whose first byte lies in object id (id = n_objects: in none).
+ * h_pairs NULL: ve_temporal_loads.  VE_ERR_INVALID if n_pcs x (n_objects + 1) > 2^24. */
+ve_status ve_temporal_loads_ex(ve_ctx* ctx, const ve_record* d_records, uint64_t n, uint64_t* h_out,
+                               uint64_t* h_pairs, cudaStream_t s);
 
 /* ---- approximate frequent values ---------------------------
  * Def 3.3 (frequent values) over the truncated values of Def 3.8

@@ -233,6 +233,19 @@ def dyadic_fit(cfg, objs, recs):
     return out
 
 
+def temporal_pairs(cfg, objs, recs):
+    """C17 per (PC, object): uint64[n_pcs, n_obj + 1, 2]; column n_obj = loads outside every object."""
+    recs = np.ascontiguousarray(recs)
+    arr, _keep = _objects(objs)
+    out = np.zeros((cfg.n_pcs, len(objs) + 1, 2), dtype=np.uint64)
+    L = lib()
+    L.vo_temporal_pairs.argtypes = [ctypes.POINTER(VoConfig), ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+                                    ctypes.c_uint64, ctypes.c_void_p]
+    if L.vo_temporal_pairs(ctypes.byref(cfg), arr, len(objs), recs.ctypes.data, len(recs), out.ctypes.data) != 0:
+        raise ValueError("vo_temporal_pairs rejected its arguments")
+    return out
+
+
 def dyadic_fit_trunc(cfg, objs, recs):
     """C22 (f2): DYADIC_DTYPE[n_keys] -- C21 over the float values truncated to K mantissa bits."""
     recs = np.ascontiguousarray(recs)

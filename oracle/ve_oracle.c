@@ -1225,3 +1225,40 @@ int vo_outlier_fit(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, 
   free(t.by_base);
   return 0;
 }
+
+/* ---- C17 per (PC, object) (f3; Table 5's redundancy analysis P:L470, LoadSpy ref [47] P:L658) ----
+ * DESIGN.md R6 split by the pair (pc, object of the load's first byte): out[(pc (n_obj + 1) + id) 2]
+ * = temporal loads of that pair, + 1 = temporally redundant ones; column id = n_obj collects the
+ * loads outside every object.  The same trace-order definition as vo_temporal_loads. */
+int vo_temporal_pairs(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                      uint64_t n, uint64_t* out) {
+  if (!cfg || cfg->n_pcs == 0) return -1;
+  objtab t;
+  if (objtab_build(&t, objs, n_obj) != 0) return -1;
+  const uint64_t cols = (uint64_t)n_obj + 1;
+  memset(out, 0, sizeof(uint64_t) * 2 * cfg->n_pcs * cols);
+  uint64_t cap = 16;
+  while (cap < 2 * n + 2) cap <<= 1;
+  lastload* tab = (lastload*)calloc(cap, sizeof(lastload));
+  for (uint64_t i = 0; i < n; ++i) {
+    const vo_record* r = &recs[i];
+    dec_t d;
+    decode(cfg, &t, r, &d);
+    if (!d.valid || d.shared || d.store) continue;
+    uint64_t h = (r->addr * 0x9E3779B97F4A7C15ull) >> 17 & (cap - 1);
+    while (tab[h].used && tab[h].addr != r->addr) h = (h + 1) & (cap - 1);
+    if (tab[h].used) {
+      const int red = tab[h].w == d.w && tab[h].value == r->value;
+      const uint64_t p = (uint64_t)r->pc * cols + (d.obj ? d.obj->id : n_obj);
+      out[2 * p]++;
+      out[2 * p + 1] += red;
+    }
+    tab[h].used = 1;
+    tab[h].addr = r->addr;
+    tab[h].value = r->value;
+    tab[h].w = d.w;
+  }
+  free(tab);
+  free(t.by_base);
+  return 0;
+}

@@ -180,6 +180,9 @@ int vo_vfg_important(const vo_vfg_edge* edges, uint64_t ne, const vo_vfg_vertex*
  * PC only): out[2 * key] = temporal, out[2 * key + 1] = redundant (C17). */
 int vo_temporal_loads(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
                       uint64_t n, uint64_t* out);
+/* the same per (PC, object): out[2 (pc (n_obj + 1) + id)], id = n_obj for loads outside every object */
+int vo_temporal_pairs(const vo_config* cfg, const vo_object* objs, uint32_t n_obj, const vo_record* recs,
+                      uint64_t n, uint64_t* out);
 
 /* ---- approximate frequent values -------------------------
  * Def 3.3 (frequent values) over the truncated values of Def 3.8

@@ -639,10 +639,22 @@ __global__ void __launch_bounds__(IV_T) k_tl_gather(const ve_record* r, const ui
   }
 }
 
+// pairs != null: also the (pc, object) table (f3 per pair): row pc, column = object id (nobj: none)
+__device__ __forceinline__ void tl_add_global(unsigned long long* out, bool act, uint64_t key, uint32_t red) {
+  const unsigned am = __ballot_sync(FULLM, act);
+  if (!act) return;
+  const unsigned g = __match_any_sync(am, key);
+  const uint32_t nr = __popc(__ballot_sync(g, red != 0u) & g);
+  if ((int)(threadIdx.x & 31) == __ffs(g) - 1) {
+    atomicAdd(&out[2 * key], (unsigned long long)__popc(g));
+    if (nr) atomicAdd(&out[2 * key + 1], (unsigned long long)nr);
+  }
+}
+
 __global__ void __launch_bounds__(IV_T) k_tl_judge(const uint64_t* S, const uint64_t* V, const uint64_t* PM,
                                                    uint64_t m, const uint64_t* ob, const uint64_t* oe,
                                                    const uint32_t* oid, uint32_t nobj, uint32_t n_pcs,
-                                                   unsigned long long* out) {
+                                                   unsigned long long* out, unsigned long long* pairs) {
   __shared__ uint32_t sc[2 * TL_SK];   // per-block counters of the first TL_SK keys (< 2^32 per block)
   for (uint32_t i = threadIdx.x; i < 2 * TL_SK; i += IV_T) sc[i] = 0;
   __syncthreads();
@@ -667,6 +679,10 @@ __global__ void __launch_bounds__(IV_T) k_tl_judge(const uint64_t* S, const uint
     }
     tl_add(sc, out, temporal, pc, red);
     tl_add(sc, out, has_obj, okey, red);
+    if (pairs) {                           // (block-uniform: every lane takes part)
+      const uint64_t pk = (uint64_t)pc * (nobj + 1) + (has_obj ? okey - n_pcs : nobj);
+      tl_add_global(pairs, temporal, pk, red);
+    }
   }
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < 2 * TL_SK; i += IV_T)
@@ -679,16 +695,21 @@ using namespace ve;
 
 extern "C" {
 
-ve_status ve_temporal_loads(ve_ctx* c, const ve_record* d_records, uint64_t n, uint64_t* h_out, cudaStream_t s) {
+ve_status ve_temporal_loads_ex(ve_ctx* c, const ve_record* d_records, uint64_t n, uint64_t* h_out,
+                               uint64_t* h_pairs, cudaStream_t s) {
   if (!c || !h_out) return VE_ERR_INVALID;
   const uint32_t nk = c->n_keys;
+  const uint64_t npairs = (uint64_t)c->cfg.n_pcs * (c->n_obj + 1);
+  if (h_pairs && npairs > (1ull << 24)) return fail(c, VE_ERR_INVALID, "ve_temporal_loads_ex: n_pcs x (objects + 1) > 2^24");
   memset(h_out, 0, sizeof(uint64_t) * 2 * nk);
+  if (h_pairs) memset(h_pairs, 0, sizeof(uint64_t) * 2 * npairs);
   if (n == 0) return VE_OK;
   if (!d_records || ((uintptr_t)d_records & 7)) return fail(c, VE_ERR_INVALID, "ve_temporal_loads: null or misaligned");
   if (n >= (1ull << 32)) return fail(c, VE_ERR_INVALID, "ve_temporal_loads: n >= 2^32");
   cudaSetDevice(c->device);
   const uint64_t ntile = (n + IV_TILE - 1) / IV_TILE;
-  const size_t need = 32 * n + sort_scratch_bytes(n) + 4 * ntile + 4 * (ntile / SC_TILE + 2) + 16 * (size_t)nk + 64;
+  const size_t need = 32 * n + sort_scratch_bytes(n) + 4 * ntile + 4 * (ntile / SC_TILE + 2) + 16 * (size_t)nk + 64 +
+                      (h_pairs ? 16 * npairs : 0);
   uint8_t* buf = nullptr;
   cudaError_t e = cudaMallocAsync((void**)&buf, need, s);
   if (e != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "ve_temporal_loads: workspace"); }
@@ -716,19 +737,25 @@ ve_status ve_temporal_loads(ve_ctx* c, const ve_record* d_records, uint64_t n, u
   if (m > 1) {
     st = sort_pairs(c, S, E, S2, E2, m, scr, s);
     if (st == VE_OK) {
-      cudaMemsetAsync(d_out, 0, 16 * (size_t)nk, s);
+      unsigned long long* d_pairs = h_pairs ? d_out + 2 * (size_t)nk : nullptr;
+      cudaMemsetAsync(d_out, 0, 16 * (size_t)nk + (h_pairs ? 16 * npairs : 0), s);
       count_launch();
       k_tl_gather<<<grid_for(c, IV_T, m), IV_T, 0, s>>>(d_records, E, m, S2, E2);   // the sort's spare buffers
       count_launch();
       k_tl_judge<<<grid_for(c, IV_T, m), IV_T, 0, s>>>(S, S2, E2, m, c->o.base, c->o.end, c->o.id, c->n_obj,
-                                                       c->cfg.n_pcs, d_out);
+                                                       c->cfg.n_pcs, d_out, d_pairs);
       e = cudaMemcpyAsync(h_out, d_out, 16 * (size_t)nk, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess && h_pairs) e = cudaMemcpyAsync(h_pairs, d_pairs, 16 * npairs, cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaStreamSynchronize(s);
       if (e != cudaSuccess) st = cuda_fail(c, e, "ve_temporal_loads");
     }
   }
   cudaFreeAsync(buf, s);
   return st;
+}
+
+ve_status ve_temporal_loads(ve_ctx* c, const ve_record* d_records, uint64_t n, uint64_t* h_out, cudaStream_t s) {
+  return ve_temporal_loads_ex(c, d_records, n, h_out, nullptr, s);
 }
 
 

@@ -125,6 +125,7 @@ def lib():
             "ve_plan_copies": ([vp, vp, u64, u32, u32, vp, vp], st),
             "ve_snapshot_diff_all": ([vp, u32, vp, vp, vp], st),
             "ve_dyadic_fit_ex": ([vp, vp, u64, u32, vp, vp], st),
+            "ve_temporal_loads_ex": ([vp, vp, u64, vp, vp, vp], st),
             "ve_outlier_fit": ([vp, vp, u64, u32, vp, vp], st),
             "ve_object_dedup_comm": ([vp, vp, u32, vp, vp, vp], st),
             "ve_snapshot_diff_all_group": ([ctypes.POINTER(vp), u32, u32, vp, vp], st),
@@ -464,6 +465,15 @@ class Context:
         self._check(lib().ve_temporal_loads(self._h, _ptr(d_records), n, out.ctypes.data, _stream(stream)),
                     "ve_temporal_loads")
         return out
+
+    def temporal_pairs(self, d_records, n, stream=None):
+        """ve_temporal_loads_ex: (uint64[n_keys, 2] per key, uint64[n_pcs, n_objects + 1, 2] per (PC, object))."""
+        nk = self.n_pcs + getattr(self, "n_objects", 0) + 1
+        out = np.zeros((nk, 2), dtype=np.uint64)
+        pairs = np.zeros((self.n_pcs, getattr(self, "n_objects", 0) + 1, 2), dtype=np.uint64)
+        self._check(lib().ve_temporal_loads_ex(self._h, _ptr(d_records), n, out.ctypes.data, pairs.ctypes.data,
+                                               _stream(stream)), "ve_temporal_loads_ex")
+        return out, pairs
 
     def interval_merge(self, d_in, n, d_out, stream=None):
         """ve_interval_merge: merge n device intervals (16 B each) into d_out; returns the merged count."""

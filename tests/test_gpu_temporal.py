@@ -74,3 +74,28 @@ def test_temporal_cfg2_full_size(torch_cuda):
     assert out[npc + 0].tolist() == [363 * wa, 363 * wa] and out[npc + 1].tolist() == [15 * wb, 15 * wb]
     assert out[npc + 2].tolist() == [0, 0]
     ctx.close()
+
+
+@pytest.mark.parametrize("cfg,epoch,seed,n", [(G.FUZZ, 0, 4, 300001), (G.scaled(G.CFG3, 6), 0, 3, None),
+                                              (G.scaled(G.CFG4, 4), 1, 4, None)])
+def test_temporal_pairs_parity(torch_cuda, cfg, epoch, seed, n):
+    """f3 per (PC, object) (ve_temporal_loads_ex) against the oracle's pair table, bit-exact"""
+    from paper_conf_asplos_zhouhmm022_b200 import ve
+    inf = G.info(cfg, epoch)
+    n = n or inf["n_records"]
+    hobjs = W.host_objects(cfg, epoch, seed)
+    recs = G.records_host(cfg, epoch, seed, 0, n)
+    if cfg == G.FUZZ:                                  # repeats: fold addresses onto a few lines
+        rng = np.random.default_rng(seed)
+        recs = recs.copy()
+        sel = rng.random(n) < 0.5
+        recs["addr"][sel] = (recs["addr"][sel] & ~np.uint64(0xFFF)) | (recs["addr"][sel] & np.uint64(0x3C))
+    ctx = ve.Context(n_pcs=inf["n_pcs"], max_objects=max(len(hobjs), 1))
+    ctx.set_objects(W.device_objects(hobjs))
+    keys, pairs = ctx.temporal_pairs(W.device_records(recs), n)
+    ocfg = O.make_config(inf["n_pcs"])
+    assert np.array_equal(keys, O.temporal_loads(ocfg, hobjs, recs))
+    want = O.temporal_pairs(ocfg, hobjs, recs)
+    assert np.array_equal(pairs, want)
+    assert int(want[..., 0].sum()) > 0
+    ctx.close()
