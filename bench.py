@@ -420,6 +420,7 @@ def main():
         torch.cuda.empty_cache()
         extra["cfg3"] = measure_cfg3(ve, torch.cuda.current_stream(), peak)
         extra["next_rows"] = f1
+        extra["f4_value_flow_graph"] = measure_vfg(ve)
     dd5 = r5 = None
     if single and not args.no_cfg5:
         stream = torch.cuda.current_stream()
@@ -559,6 +560,23 @@ def measure_cfg3(ve, stream, peak):
             "timed": "set_objects + analyze + report per iteration (no diff / dedup), second pass on a warm context"}
 
 
+def measure_vfg(ve):
+    """SURVEY 8(f) f4 on BASELINE configs[4]'s API-event log (tests/workloads.cfg5_api_log: 1000 objects,
+    4000 launches from 64 call paths): host-side graph build (Def 5.1) and important graph (Def 5.3,
+    edges >= 16 MiB, vertices invoked >= 70 times) -- libve's host code, wall time."""
+    from tests import workloads as W
+    lg = W.cfg5_api_log()
+    t = time.perf_counter()
+    g = ve.ValueFlowGraph.build(lg)
+    tb = time.perf_counter() - t
+    t = time.perf_counter()
+    gi = g.important(16 << 20, 70)
+    ti = time.perf_counter() - t
+    return {"events": len(lg), "vertices": len(g.vertices), "edges": len(g.edges),
+            "important_vertices": len(gi.vertices), "important_edges": len(gi.edges),
+            "build_ms": 1e3 * tb, "important_ms": 1e3 * ti, "where": "host (libve C++), not a GPU kernel"}
+
+
 def measure_cfg5_dedup(ve, stream, peak, reps=3):
     """BASELINE configs[4] (cfg5), duplicate-object half: ve_object_dedup over 1000 objects / ~19.7 GiB of
     post snapshots generated on the device (untimed); CUDA events around the (synchronizing) call.
@@ -593,8 +611,9 @@ def measure_cfg5_dedup(ve, stream, peak, reps=3):
     ctx.close()
     del dobjs
     torch.cuda.empty_cache()
-    return {"workload": "cfg5 duplicate-object scan: 1000 objects, 4 sizes (8-32 MiB), 30% zero / 10% copies / "
-                        "5% one-bit flips / 55% random", "objects": len(objs), "bytes": total, "ms": ms,
+    return {"workload": "cfg5 duplicate-object scan: 1000 objects, 50 log-uniform size classes over [64 KiB, 512 MiB] "
+                        "rescaled to 20 GiB, 30% zero / 10% copies / 5% one-bit flips / 55% random",
+            "objects": len(objs), "bytes": total, "ms": ms,
             "alg_bytes": alg, "alg_gbs": alg / (ms / 1e3) / 1e9, "frac_of_hbm_peak": alg / (ms / 1e3) / 1e9 / peak,
             "groups": len(set(want)), "parity_closed_form": [int(x) for x in g] == want}
 

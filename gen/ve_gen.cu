@@ -161,12 +161,27 @@ extern "C" int veg_snapshot_device(int cfg, int epoch, uint64_t seed, uint32_t o
 
 /* ---- dedup object sets --------------------------------------------------- */
 
+/* unit == 0 (the cfg5 recipe): the class sizes of objects 0..999 rescaled so that they total 20 GiB
+ * (4 KiB multiples, rounded down; the same factor for every object) */
+static uint64_t dedup_scaled(uint64_t seed, uint32_t i) {
+  static uint64_t cached_seed = ~0ull;
+  static double factor = 1.0;
+  if (cached_seed != seed) {
+    double tot = 0;
+    for (uint32_t j = 0; j < 1000; ++j) tot += (double)veg_dedup_size(seed, j, 0);
+    factor = (double)(20ull << 30) / tot;
+    cached_seed = seed;
+  }
+  const uint64_t v = (uint64_t)((double)veg_dedup_size(seed, i, 0) * factor) & ~4095ull;
+  return v ? v : 4096;
+}
+
 extern "C" int veg_dedup_object(uint64_t seed, uint32_t i, uint64_t unit, veg_object* out, uint32_t* cls,
                                 uint32_t* src) {
-  if (!out || unit == 0 || unit % 8) return -1;
+  if (!out || unit % 8) return -1;
   out->id = i;
   out->base = VEG_DD_BASE + (uint64_t)i * 0x100000000ull;
-  out->size = veg_dedup_size(seed, i, unit);
+  out->size = unit ? veg_dedup_size(seed, i, unit) : dedup_scaled(seed, i);
   out->elem_width = 8;
   out->has_pre = 1;
   out->has_post = 1;

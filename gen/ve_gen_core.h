@@ -14,6 +14,7 @@
  */
 #ifndef VE_GEN_CORE_H
 #define VE_GEN_CORE_H
+#include <math.h>
 #include <stdint.h>
 #include <string.h>
 
@@ -734,8 +735,17 @@ VEG_FN void veg_fuzz_record(uint64_t seed, uint64_t r, veg_record* out) {
  * ========================================================================= */
 #define VEG_DD_BASE 0x7d0000000000ull
 
+/* unit > 0: 4 distinct sizes unit .. 4 unit (the scaled test sets).  unit == 0: the cfg5 recipe
+ * (SURVEY 8(d) cfg5): 50 log-uniform size classes s = 0..49 over [64 KiB, 512 MiB] (64 KiB x 2^(13 s / 49),
+ * 4 KiB multiples); this returns the class size, whose EQUALITY is what the content classes use --
+ * veg_dedup_object rescales it so the 1000 objects total 20 GiB (ve_gen.cu). */
+VEG_FN uint64_t veg_dedup_class_size(uint32_t s) {
+  const double b = 65536.0 * exp2(13.0 * (double)s / 49.0);
+  return ((uint64_t)b + 4095ull) & ~4095ull;
+}
 VEG_FN uint64_t veg_dedup_size(uint64_t seed, uint32_t i, uint64_t unit) {
   uint64_t h = veg_h(seed, 4000, i);
+  if (unit == 0) return veg_dedup_class_size((uint32_t)(h % 50));
   return unit * (1 + h % 4);                                  /* 4 distinct sizes */
 }
 VEG_FN uint32_t veg_dedup_base_class(uint64_t seed, uint32_t i) {

@@ -12,7 +12,8 @@
  *        VEG_CFG4 (4)  f64 stencils; epoch 0 hotspot3D-like, epoch 1 Castro-like
  *                      (cfg3 / cfg4 | s << 8: tensors 2^s times smaller)
  *        VEG_FUZZ (100) adversarial mixed trace (unbounded record stream)
- *   Dedup sets: veg_dedup_* (object i of a set keyed by seed and size unit).
+ *   Dedup sets: veg_dedup_* (object i of a set keyed by seed and size unit; unit 0 = the cfg5
+ *   recipe: 50 log-uniform size classes over [64 KiB, 512 MiB], rescaled to 20 GiB per 1000 objects).
  *
  * Return 0 on success, -1 on bad arguments / launch failure.  Device calls are
  * asynchronous on stream s; d_out is caller-owned device memory (8-byte

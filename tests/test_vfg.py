@@ -111,3 +111,33 @@ def test_libve_figure3():
     assert E(g.slice(6).edges) == [(2, 4, B, W), (4, 6, B, W), (6, 7, B, W)]
     with pytest.raises(ve.VeError):
         ve.ValueFlowGraph.build(log([(2, 1, A, W, ALLOC, 4), (1, 2, A, R, DEV, 4)]))   # not in program order
+
+
+def test_cfg5_api_log_graph():
+    """f4 at the paper's scale (LAMMPS: 660 vertices pruned to 132, Def 5.3): the value flow graph
+    of cfg5's 4000-kernel API log (1000 objects, 64 kernel call paths) -- libve's builder, slice and
+    important graph against the oracle, and the invariants of the log's construction: one vertex per
+    call path, invocations = launches per path, every object's first edge leaves its allocation."""
+    from paper_conf_asplos_zhouhmm022_b200 import ve
+    from tests import workloads as WL
+    lg = WL.cfg5_api_log()
+    g = ve.ValueFlowGraph.build(lg)
+    oe, ov = O.vfg_build(lg)
+    assert g.edges.tobytes() == oe.tobytes() and g.vertices.tobytes() == ov.tobytes()
+    inv = {int(x["vertex"]): int(x["invocations"]) for x in ov}
+    launches = {}
+    for r in lg:
+        if int(r["kind"]) == DEV:
+            launches.setdefault(int(r["vertex"]), set()).add(int(r["seq"]))
+    for v, seqs in launches.items():
+        assert inv[v] == len(seqs)
+    assert sum(1 for v in inv if 100 <= v < 164) == 64
+    # Def 5.3: keep edges of >= 16 MiB and vertices invoked >= 70 times; the pruned graph is smaller
+    ie, iv = O.vfg_important(oe, ov, 16 << 20, 70)
+    gi = g.important(16 << 20, 70)
+    assert gi.edges.tobytes() == ie.tobytes() and gi.vertices.tobytes() == iv.tobytes()
+    assert 0 < len(ie) < len(oe) // 10 and len(iv) <= len(ov)
+    v0 = int(ov[len(ov) // 2]["vertex"])
+    se, sv = O.vfg_slice(oe, ov, v0)
+    s = g.slice(v0)
+    assert s.edges.tobytes() == se.tobytes() and s.vertices.tobytes() == sv.tobytes()
