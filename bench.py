@@ -423,9 +423,9 @@ def main():
         extra["f4_value_flow_graph"] = measure_vfg(ve)
     dd5 = r5 = None
     if single and not args.no_cfg5:
-        stream = torch.cuda.current_stream()
-        dd5 = measure_cfg5_dedup(ve, stream, peak)
-        r5 = measure_cfg5_records(ve, stream, peak)
+        dd5 = measure_cfg5_dedup(ve, torch.cuda.current_stream(), peak)
+    if not args.no_cfg5:          # every rank: its LPT share of the 4000 kernels (weak-style partition)
+        r5 = measure_cfg5_records(ve, torch.cuda.current_stream(), peak, rank, world, dev)
 
     cpu = None
     if not args.no_cpu and single:
@@ -618,7 +618,7 @@ def measure_cfg5_dedup(ve, stream, peak, reps=3):
             "groups": len(set(want)), "parity_closed_form": [int(x) for x in g] == want}
 
 
-def measure_cfg5_records(ve, stream, peak):
+def measure_cfg5_records(ve, stream, peak, rank=0, world=1, dev=None):
     """BASELINE configs[4] (cfg5), records half: 4000 independent kernels, 10^9 records in total (4..64 PCs,
     1..4 objects, 2,987 .. 1,676,166 records each; gen/ve_gen_core.h veg_cfg5_record).  All records and
     snapshots are generated on the device first (untimed, 24 GB + 2 x 4 GB); the timed region is the
@@ -632,13 +632,18 @@ def measure_cfg5_records(ve, stream, peak):
     sp = stream.cuda_stream
     cfg, seed, K = G.scaled(G.CFG5, 0), 5, 4000
     infos = [G.info(cfg, k) for k in range(K)]
-    n_tot = sum(i["n_records"] for i in infos)
+    n_all = sum(i["n_records"] for i in infos)
+    # N > 1: the kernels are independent units -- each rank takes its longest-processing-time-first
+    # share by record count (ve.lpt_assign: the same plan on every rank, no data-path collective)
+    owner = ve.lpt_assign([i["n_records"] for i in infos], world)
+    mine = [k for k in range(K) if owner[k] == rank]
+    n_tot = sum(infos[k]["n_records"] for k in mine)
     recs = torch.empty(n_tot * REC_BYTES, dtype=torch.uint8, device="cuda")
-    objs_of = [G.objects(cfg, k) for k in range(K)]
-    snap_tot = sum(o["size"] for objs in objs_of for o in objs)
+    objs_of = {k: G.objects(cfg, k) for k in mine}
+    snap_tot = sum(o["size"] for objs in objs_of.values() for o in objs)
     snaps = torch.empty(2 * snap_tot, dtype=torch.uint8, device="cuda")
     r0, s0, plan = 0, 0, []
-    for k in range(K):
+    for k in mine:
         n = infos[k]["n_records"]
         G.records_device(cfg, k, seed, 0, n, recs.data_ptr() + r0 * REC_BYTES, sp)
         dobjs = []
@@ -658,39 +663,47 @@ def measure_cfg5_records(ve, stream, peak):
         ctx.analyze_records(buf, n, stream=sp)
         ctx.report().close()
     torch.cuda.synchronize()
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in plan]
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    bad, checked = [], 0
+    bad, checked, got = [], 0, {}
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
     a.record(stream)
-    for k, (buf, n, dobjs) in enumerate(plan):
+    for j, (buf, n, dobjs) in enumerate(plan):
         ctx.set_objects(dobjs)
-        ev[k][0].record(stream)
+        ev[j][0].record(stream)
         ctx.analyze_records(buf, n, stream=sp)
-        ev[k][1].record(stream)
+        ev[j][1].record(stream)
         rep = ctx.report()
-        if k % 50 == 0:
-            keys = {f: rep.keys[f].copy() for f in ("n_ld", "n_st", "n_ld_eq_pre", "n_st_eq_pre", "raw_min",
-                                                     "raw_max", "single_zero", "single_value")}
-            plan[k] = (buf, n, dobjs, keys, int(rep.globals["n_records"]))
+        if mine[j] % 50 == 0:
+            got[mine[j]] = ({f: rep.keys[f].copy() for f in ("n_ld", "n_st", "n_ld_eq_pre", "n_st_eq_pre", "raw_min",
+                                                              "raw_max", "single_zero", "single_value")},
+                            int(rep.globals["n_records"]))
         rep.close()
     b.record(stream)
     torch.cuda.synchronize()
     ms = a.elapsed_time(b)
     an_ms = sum(x.elapsed_time(y) for x, y in ev)
-    for k in range(0, K, 50):
-        bad += cfg5k.check_cfg5_kernel(plan[k][3], plan[k][4], cfg, k)
+    if world > 1:
+        ms = max_over_ranks(ms, device=dev)
+    for k, (keys, nrec) in got.items():
+        bad += cfg5k.check_cfg5_kernel(keys, nrec, cfg, k)
         checked += 1
     ctx.close()
     del plan, recs, snaps
     torch.cuda.empty_cache()
-    gbs = n_tot * REC_BYTES / (ms / 1e3) / 1e9
+    gbs = n_all * REC_BYTES / (ms / 1e3) / 1e9
     return {"workload": "cfg5 records: 4000 kernels, 4-64 PCs with cfg1 roles, 1-4 objects, 10^9 records",
-            "kernels": K, "records": n_tot, "snapshot_bytes": 2 * snap_tot, "ms": ms,
-            "records_per_s": n_tot / (ms / 1e3), "trace_gbs": gbs, "trace_frac_of_hbm_peak": gbs / peak,
-            "analyze_ms": an_ms, "analyze_records_per_s": n_tot / (an_ms / 1e3),
-            "per_kernel_overhead_ms": (ms - an_ms) / K, "closed_forms_kernels_checked": checked,
+            "kernels": K, "records": n_all, "ranks": world, "partition": "longest-processing-time-first by records "
+            "(ve.lpt_assign), independent kernels, no data-path collective", "this_rank_kernels": len(mine),
+            "snapshot_bytes_this_rank": 2 * snap_tot, "ms": ms,
+            "records_per_s": n_all / (ms / 1e3), "trace_gbs": gbs, "trace_frac_of_hbm_peak": gbs / peak / world,
+            "analyze_ms_this_rank": an_ms, "analyze_records_per_s_this_rank": n_tot / (an_ms / 1e3),
+            "per_kernel_overhead_ms": (ms - an_ms) / max(len(mine), 1), "closed_forms_kernels_checked": checked,
             "closed_forms_ok": not bad, "closed_form_mismatches": bad[:5],
-            "timed": "set_objects + analyze + report per kernel on one context, CUDA events around the loop"}
+            "timed": "set_objects + analyze + report per kernel on one context per rank, CUDA events around the "
+                     "loop, max over ranks"}
 
 
 def measure_e2e(ve, ctx, wl, steps):

@@ -20,51 +20,52 @@ __device__ __forceinline__ uint64_t word_mix(uint64_t w, uint64_t j) {
   return mix64(w ^ (j * 0x9E3779B97F4A7C15ull) ^ 0x5851F42D4C957F2Dull) + j;
 }
 
-struct HashJob {
+struct HashJob {          // one chunk of one object: bytes [off, off + len) of p (size bytes in total)
   const uint8_t* p;
-  uint64_t size;
+  uint64_t size, off, len;
+  uint32_t pos, pad;     // the object's slot in the hash array
 };
 
-// K7: blockIdx.y = object, grid-stride over its 16-byte words; +tail bytes
+// K7: one CTA per chunk of <= DD_CH bytes; the hash is a sum over the object's 8-byte words of a
+// position-keyed mix, so the chunks' partial sums simply add (any order, any split)
+constexpr uint64_t DD_CH = 1ull << 20;
 __global__ void __launch_bounds__(256) k_hash(const HashJob* jobs, unsigned long long* hash) {
-  const HashJob jb = jobs[blockIdx.y];
+  const HashJob jb = jobs[blockIdx.x];
   unsigned long long acc = 0;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  if (((uintptr_t)jb.p & 15) == 0) {
-    const uint64_t nv = jb.size / 16;
+  const uint64_t w0 = jb.off / 8, w1 = (jb.off + jb.len + 7) / 8;    // the chunk's words (off is 8-aligned)
+  if (((uintptr_t)jb.p & 15) == 0 && (jb.off & 15) == 0) {
+    const uint64_t v0 = jb.off / 16, v1 = (jb.off + jb.len) / 16 < jb.size / 16 ? (jb.off + jb.len) / 16 : jb.size / 16;
     const uint4* v = (const uint4*)jb.p;
-    // four independent 16-byte loads in flight per thread per iteration
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    for (; i + 3 * stride < nv; i += 4 * stride) {
+    uint64_t i = v0 + threadIdx.x;
+    for (; i + 3 * 256 < v1; i += 4 * 256) {   // four independent 16-byte loads in flight per thread
       uint4 x[4];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) x[u] = __ldcs(v + i + u * stride);
+      for (int u = 0; u < 4; ++u) x[u] = __ldcs(v + i + u * 256);
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const uint64_t k = i + u * stride;
+        const uint64_t k = i + u * 256;
         acc += word_mix(((uint64_t)x[u].y << 32) | x[u].x, 2 * k) + word_mix(((uint64_t)x[u].w << 32) | x[u].z, 2 * k + 1);
       }
     }
-    for (; i < nv; i += stride) {
+    for (; i < v1; i += 256) {
       const uint4 x = __ldcs(v + i);
       acc += word_mix(((uint64_t)x.y << 32) | x.x, 2 * i) + word_mix(((uint64_t)x.w << 32) | x.z, 2 * i + 1);
     }
-    // tail: remaining words (incl. a zero-padded partial word)
-    const uint64_t done = nv * 16;
-    for (uint64_t j = done / 8 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j * 8 < jb.size; j += stride) {
+    // the chunk's words beyond its whole 16-byte blocks (the object's tail, incl. a partial word)
+    for (uint64_t j = 2 * v1 + threadIdx.x; j < w1 && j * 8 < jb.size; j += 256) {
       uint64_t w = 0;
       for (uint64_t b = 0; b < 8 && j * 8 + b < jb.size; ++b) w |= (uint64_t)jb.p[j * 8 + b] << (8 * b);
       acc += word_mix(w, j);
     }
   } else {
-    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j * 8 < jb.size; j += stride) {
+    for (uint64_t j = w0 + threadIdx.x; j < w1 && j * 8 < jb.size; j += 256) {
       uint64_t w = 0;
       for (uint64_t b = 0; b < 8 && j * 8 + b < jb.size; ++b) w |= (uint64_t)jb.p[j * 8 + b] << (8 * b);
       acc += word_mix(w, j);
     }
   }
   for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xFFFFFFFFu, acc, o);
-  if ((threadIdx.x & 31) == 0) atomicAdd(&hash[blockIdx.y], acc);
+  if ((threadIdx.x & 31) == 0 && acc) atomicAdd(&hash[jb.pos], acc);
 }
 
 struct CmpJob {
@@ -111,35 +112,29 @@ __global__ void __launch_bounds__(256) k_compare(const CmpJob* jobs, unsigned lo
   if (__syncthreads_or(diff) && threadIdx.x == 0) atomicOr(&differs[jb.pair], 1ull);
 }
 
-// K7 of the eligible objects k (positions in elig) with k mod G == rank into d_hash[k]
-static void hash_launch(ve_ctx* c, const ve_object* objs, const std::vector<uint32_t>& elig, int G, int rank,
-                        HashJob* d_jobs, std::vector<HashJob>& hj, unsigned long long* d_hash, cudaStream_t s) {
-  hj.clear();
-  std::vector<uint32_t> pos;
-  uint64_t maxsz = 0;
+// K7 of the eligible objects k (positions in elig) with k mod G == rank into d_hash[k]: every owned
+// object cut into DD_CH-byte chunk jobs, one CTA each (sizes from KiB to hundreds of MiB balance)
+static ve_status hash_launch(ve_ctx* c, const ve_object* objs, const std::vector<uint32_t>& elig, int G, int rank,
+                             unsigned long long* d_hash, cudaStream_t s) {
+  std::vector<HashJob> hj;
   for (size_t k = 0; k < elig.size(); ++k) {
     if ((int)(k % G) != rank) continue;
-    hj.push_back(HashJob{(const uint8_t*)objs[elig[k]].post, objs[elig[k]].size});
-    pos.push_back((uint32_t)k);
-    maxsz = std::max<uint64_t>(maxsz, objs[elig[k]].size);
+    const ve_object& o = objs[elig[k]];
+    for (uint64_t off = 0; off < o.size; off += DD_CH)
+      hj.push_back(HashJob{(const uint8_t*)o.post, o.size, off, std::min(DD_CH, o.size - off), (uint32_t)k, 0});
   }
-  if (hj.empty()) return;
-  // a rank's owned objects are not contiguous in elig: hash into a compact array, then scatter
+  if (hj.empty()) return VE_OK;
+  HashJob* d_jobs = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&d_jobs, hj.size() * sizeof(HashJob), s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "dedup hash jobs");
   cudaMemcpyAsync(d_jobs, hj.data(), hj.size() * sizeof(HashJob), cudaMemcpyHostToDevice, s);
-  unsigned long long* d_tmp = d_hash + elig.size();
-  cudaMemsetAsync(d_tmp, 0, hj.size() * 8, s);
-  // grid.x: ~256 KiB of the largest object per CTA (16 KiB per CTA-iteration, 4 loads deep),
-  // at least two CTAs per SM over the whole set
-  uint64_t gx = (maxsz + (256u << 10) - 1) / (256u << 10);
-  const uint64_t want = (2ull * c->num_sms + hj.size() - 1) / hj.size();
-  gx = std::min<uint64_t>(std::max<uint64_t>(std::max<uint64_t>(gx, want), 1), 1024);
-  for (size_t y0 = 0; y0 < hj.size(); y0 += 65535) {
-    const unsigned gy = (unsigned)std::min<size_t>(65535, hj.size() - y0);
+  for (size_t j0 = 0; j0 < hj.size(); j0 += (1u << 30)) {
     count_launch();
-    k_hash<<<dim3((unsigned)gx, gy), 256, 0, s>>>(d_jobs + y0, d_tmp + y0);
+    k_hash<<<(unsigned)std::min<size_t>(hj.size() - j0, 1u << 30), 256, 0, s>>>(d_jobs + j0, d_hash);
   }
-  for (size_t q = 0; q < pos.size(); ++q)      // (small: one 8-byte copy per owned object)
-    cudaMemcpyAsync(d_hash + pos[q], d_tmp + q, 8, cudaMemcpyDeviceToDevice, s);
+  cudaFreeAsync(d_jobs, s);
+  e = cudaStreamSynchronize(s);      // (hj is a host vector of this call)
+  return e == cudaSuccess ? VE_OK : cuda_fail(c, e, "dedup hash");
 }
 
 ve_status dedup_ranks(const std::vector<ve_ctx*>& cs, Comm& comm, const ve_object* objs, uint32_t n,
@@ -154,21 +149,17 @@ ve_status dedup_ranks(const std::vector<ve_ctx*>& cs, Comm& comm, const ve_objec
   const size_t ne = elig.size();
   // K7 on the owned objects, then a SUM allreduce: every rank holds every hash
   std::vector<void*> hb(cs.size());
-  std::vector<void*> jb(cs.size());
-  std::vector<HashJob> hj;
   for (size_t i = 0; i < cs.size(); ++i) {
-    cudaError_t e = cudaMallocAsync(&hb[i], 2 * ne * 8, s);
-    if (e == cudaSuccess) e = cudaMallocAsync(&jb[i], ne * sizeof(HashJob), s);
+    cudaError_t e = cudaMallocAsync(&hb[i], ne * 8, s);
     if (e != cudaSuccess) return cuda_fail(c0, e, "dedup alloc");
     cudaMemsetAsync(hb[i], 0, ne * 8, s);
-    hash_launch(cs[i], objs, elig, G, comm.local[i], (HashJob*)jb[i], hj, (unsigned long long*)hb[i], s);
-    // (hj is reused by the next rank only after this rank's H2D copy is ordered on s)
-    cudaStreamSynchronize(s);
+    ve_status st = hash_launch(cs[i], objs, elig, G, comm.local[i], (unsigned long long*)hb[i], s);
+    if (st != VE_OK) return st;
   }
   if (!comm.allreduce(hb, ne, OP_SUM, s)) return fail(c0, VE_ERR_NCCL, "dedup hash allreduce: " + comm.err);
   std::vector<unsigned long long> h(ne);
   cudaMemcpyAsync(h.data(), hb[0], ne * 8, cudaMemcpyDeviceToHost, s);
-  for (size_t i = 0; i < cs.size(); ++i) { cudaFreeAsync(hb[i], s); cudaFreeAsync(jb[i], s); }
+  for (size_t i = 0; i < cs.size(); ++i) cudaFreeAsync(hb[i], s);
   cudaError_t e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c0, e, "dedup hash");
 

@@ -129,7 +129,7 @@ __device__ __forceinline__ bool dy_load(const ve_record* r, uint64_t i, const De
 }
 
 __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n, DevObjects o, uint32_t n_pcs,
-                                                  uint32_t nk, DyKey* K, uint32_t tr) {
+                                                  uint32_t nk, DyKey* K, uint32_t tr, int count) {
   __shared__ unsigned int sT[DY_SK], sF[DY_SK];
   __shared__ unsigned long long sMin[DY_SK], sMax[DY_SK];
   const uint32_t ns = nk < DY_SK ? nk : DY_SK;
@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
         tt = __reduce_max_sync(0xFFFFFFFFu, tt);
         ff = __reduce_or_sync(0xFFFFFFFFu, ff);
         hv = __reduce_or_sync(0xFFFFFFFFu, hv);
-        if ((threadIdx.x & 31u) == 0u) atomicAdd(&K[k].n, 32ull);   // (C23's record count)
+        if (count && (threadIdx.x & 31u) == 0u) atomicAdd(&K[k].n, 32ull);   // (C23's record count)
         if ((threadIdx.x & 31u) == 0u) {
           if (k < ns) {
             if (ff) sF[k] = 1u;
@@ -187,7 +187,7 @@ __global__ void __launch_bounds__(DY_T) k_dy_scan(const ve_record* r, uint64_t n
         continue;
       }
       if (k == 0xFFFFFFFFu) continue;
-      atomicAdd(&K[k].n, 1ull);
+      if (count) atomicAdd(&K[k].n, 1ull);
       if (k < ns) {
         if (!fin) { sF[k] = 1u; continue; }
         if (t) atomicMax(&sT[k], t);
@@ -308,7 +308,7 @@ static ve_status dy_run(ve_ctx* c, const ve_record* d_records, uint64_t n, uint3
     const uint64_t cap = (uint64_t)c->num_sms * 8;
     const unsigned grid = (unsigned)(b < cap ? b : cap);
     count_launch();
-    k_dy_scan<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, nk, K, tr);
+    k_dy_scan<<<grid, DY_T, 0, s>>>(d_records, n, c->o, c->cfg.n_pcs, nk, K, tr, outlier ? 1 : 0);
     const int passes[2][3] = {{0, 1, -1}, {2, 3, 4}};
     for (int p : passes[outlier ? 1 : 0]) {
       if (p < 0) continue;
