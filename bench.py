@@ -355,12 +355,12 @@ def roofline_block(res, world, peak, peak_src, traffic):
 
 
 def traffic_of(name):
-    """dram__bytes_read.sum + dram__bytes_write.sum of the analyze launches, from the committed ncu capture
-    of the same command (profiles/r02_k_analyze_traffic.json, written by scripts/r2_bench_prof.sh)."""
+    """dram__bytes_read.sum + dram__bytes_write.sum per analyze launch (the step's epochs), from the committed
+    ncu --set full capture of the same command (profiles/r02_k_analyze_traffic.json, scripts/r2_bench_prof.sh):
+    a list per epoch, or None when no capture exists for the configuration."""
     prof = os.path.join(ROOT, "profiles", "r02_k_analyze_traffic.json")
     try:
-        d = json.load(open(prof))
-        return d.get(name)
+        return json.load(open(prof)).get(name)
     except Exception:
         return None
 
