@@ -60,6 +60,11 @@ typedef struct ve_config {
   uint32_t t_frequent_pct;  /* default 33 (Q2)                                            */
   uint64_t hist_capacity;   /* exact value-histogram slots (rounded up to 2^k); overflow  */
                             /* => VE_ERR_CAPACITY, never silently wrong stats              */
+  uint32_t min_windows_per_warp; /* 0 = every analysis launch spans all SMs; k > 0: a short */
+                            /* trace gets only the CTAs that give each warp >= k 32-record  */
+                            /* windows, so contexts analysing small traces on several        */
+                            /* streams run side by side (throughput over latency)            */
+  uint32_t reserved;        /* 0                                                         */
 } ve_config;
 
 typedef enum {
@@ -105,7 +110,9 @@ typedef struct ve_obj_stats {
 
 typedef struct ve_globals {
   uint64_t n_records, n_invalid, n_unmapped;
-  uint64_t hist_entries;        /* occupied (pc, object, value) histogram slots */
+  uint64_t hist_entries;        /* occupied slots of the device value table after the report's
+                                   dense flush (implementation statistic, not a parity field;
+                                   0 after a rank merge) */
 } ve_globals;
 
 /* ---- lifecycle ----------------------------------------------------------- */
@@ -196,7 +203,18 @@ ve_status ve_report_keys(const ve_rep* r, ve_key_stats* out);          /* n_keys
 ve_status ve_report_topk_entries(const ve_rep* r, ve_topk_entry* out); /* n_keys * topk entries  */
 ve_status ve_report_objects(const ve_rep* r, ve_obj_stats* out);       /* n_objects entries      */
 ve_status ve_report_globals(const ve_rep* r, ve_globals* out);
-/* format 0: binary (magic "VERP", header, then the arrays above); 1: JSON */
+/* S13 report dump (SURVEY 8(a) S13, 8(c) "full report == oracle").  format 0:
+ * binary, little-endian, no padding between parts:
+ *   u32 magic 0x50524556 ("VERP"), u32 version 1, u32 n_keys, u32 n_objects,
+ *   u32 topk, ve_globals (4 x u64), ve_key_stats[n_keys] (336 B each; p_* / q_*
+ *   are 0 unless line_state is POINT or LINE), ve_topk_entry[n_keys][topk]
+ *   (entries j >= n_top are {0, 0}), ve_obj_stats[n_objects] (indexed by id).
+ * format 1: JSON: {"n_records", "n_invalid", "n_unmapped", "keys": [{every raw
+ *   field, derived flag and n_type, "p"/"q": [x, y_hi, y_lo], "top": [[bits,
+ *   count] x n_top]}], "objects": [{"id", "n_elems", "n_written",
+ *   "n_loaded_eq", "n_ld_reload", "n_touched"}]}.
+ * Returns VE_ERR_INVALID for a null report / path, an unknown format or a file
+ * that cannot be opened. */
 ve_status ve_report_dump(const ve_rep* r, const char* path, int format);
 
 /* ---- LoadSpy temporal load redundancy in trace order --------

@@ -53,6 +53,7 @@ struct AnalyzeParams {
   uint32_t ring;            // records 16-byte aligned: stream windows with cp.async.bulk
   uint64_t nring;           // full windows (streamed through the per-warp rings)
   uint32_t chunk;           // windows per static chunk (VE_CLAIM 2): CHUNK, or one stage for short traces
+  uint32_t claim;           // 1: chunks claimed from the global counter *work (guided), 0: static interleave
   unsigned long long* work; // chunk claim counter (zeroed before the launch)
   // S8 insert staging: a private region of stage_rs 16-byte entries per warp for the
   // (tag, bits, count) groups the shared table cannot take; k_hist_drain inserts them
@@ -767,20 +768,23 @@ struct Ring {
 constexpr uint32_t CHUNK_TAIL = STAGE_WIN;
 __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
   uint64_t w0, len;
-#if VE_CLAIM == 2
-  // static interleave: chunk c goes to warp c mod (all warps); no atomics, and every
-  // warp sees the same mix of the trace
-  w0 = R.nextc * P.chunk;
-  len = P.chunk;
-  R.nextc += R.cstride;
-#else
-  unsigned long long c = 0;
-  if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
-  c = __shfl_sync(0xFFFFFFFFu, c, 0);
-  const uint64_t nbig = (P.nring - P.nring / 8) / CHUNK;
-  if (c < nbig) { w0 = (uint64_t)c * CHUNK; len = CHUNK; }
-  else { w0 = nbig * CHUNK + (uint64_t)(c - nbig) * CHUNK_TAIL; len = CHUNK_TAIL; }
-#endif
+  if (!P.claim) {
+    // static interleave: chunk c goes to warp c mod (all warps); no atomics, and every
+    // warp sees the same mix of the trace
+    w0 = R.nextc * P.chunk;
+    len = P.chunk;
+    R.nextc += R.cstride;
+  } else {
+    // dynamic (K1 v2): chunks from a global counter, the last 1/8 of the trace in one-stage
+    // chunks, so warps whose windows cost more (line keys, slot misses) do not set the end
+    // of the launch (cfg4: the exit barrier held 9.5% of v2's stall samples under the static split)
+    unsigned long long c = 0;
+    if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
+    c = __shfl_sync(0xFFFFFFFFu, c, 0);
+    const uint64_t nbig = (P.nring - P.nring / 8) / P.chunk;
+    if (c < nbig) { w0 = (uint64_t)c * P.chunk; len = P.chunk; }
+    else { w0 = nbig * P.chunk + (uint64_t)(c - nbig) * CHUNK_TAIL; len = CHUNK_TAIL; }
+  }
   if (w0 < P.nring) {
     R.src = P.recs + w0 * 32;
     R.iss = (uint32_t)(P.nring - w0 < len ? P.nring - w0 : len);
@@ -2125,6 +2129,9 @@ __device__ __noinline__ unsigned long long post_claim(const AnalyzeParams& P, in
 
 // K1 v2 runs K2_WARPS warps per CTA (168 registers: the slots and the object state stay in registers)
 // inside the 16-warp shared-memory layout of v1 (rings and staging regions of warps >= K2_WARPS unused)
+#ifndef VE_DIAG
+#define VE_DIAG 0
+#endif
 #ifndef VE_K2_THREADS
 #define VE_K2_THREADS 384
 #endif
@@ -2254,9 +2261,16 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   uint32_t kwm = 0, klg = 0;
   int s = 0, ls = -1;
 
+#if VE_DIAG == 2
+  uint64_t dsink = 0;
+#endif
   while (R.left) {
     uint64_t addr, val, pm;
     ring_next(P, R, addr, val, pm);
+#if VE_DIAG == 2   // diagnostic: the record stream alone (results wrong)
+    dsink += addr ^ val ^ pm;
+    continue;
+#endif
     const uint64_t pm0 = shfl64(FULL, pm, 0);
     const uint64_t a0 = shfl64(FULL, addr, 0);
     const unsigned hit = __ballot_sync(FULL, L.pmw == pm0 && a0 - L.ob <= L.olim);
@@ -2345,8 +2359,13 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
     // a fast window of slot s (its object in cb ..)
     const uint64_t o = addr - cb;
     uint64_t pv = 0, qv = 0;
+#if VE_DIAG == 1   // diagnostic: no snapshot gathers (results wrong)
+    if (cpre != 0ull) pv = val;
+    if (ldq != 0ull) qv = val;
+#else
     if (cpre != 0ull) pv = ld_pre<3>((cpre + o) & ~7ull) >> (8u * (uint32_t)((cpre + o) & 7ull));
     if (ldq != 0ull) qv = ld_pre<3>((cpost + o) & ~7ull) >> (8u * (uint32_t)((cpost + o) & 7ull));
+#endif
     const uint32_t meta0 = (uint32_t)(kkey >> 32), pc0 = (uint32_t)kkey & 0xFFFFu;
     bool wantq = false;
     switch (klg) {
@@ -2370,6 +2389,9 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
       }
     }
   }
+#if VE_DIAG == 2
+  if (dsink == 0x123456789ull) P.t.glob[G_WORK] = dsink;
+#endif
   // windows outside the ring: the partial last window, or (records not 16-byte aligned) a
   // static range of every warp
   const uint64_t nwin = (P.n + 31) / 32;
@@ -2475,7 +2497,7 @@ __global__ void __launch_bounds__(LF_THREADS) k_line_fold(const LineState* lcta,
 }
 
 ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
-  if (c->reset_ev) cudaStreamWaitEvent(s, c->reset_ev, 0);   // after the last (legacy-stream) reset
+  ctx_begin(c, s);   // after the ctx's earlier work (the last reset, a report), on any stream
   AnalyzeParams P;
   P.recs = d;
   P.n = n;
@@ -2486,8 +2508,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   // and only for a call with at least one record per pre-snapshot element: below that an element
   // is rarely loaded twice (cfg5's kernels touch each element once), and flushing per-element
   // counters costs more than the hash inserts they replace (measured: cfg5 report 0.7 -> 0.45 ms)
-  P.dense_ok = (c->dense_cap > 0 && c->records_analyzed + n < (1ull << 32) &&
-                (n >= c->pre_elems || getenv("VE_DENSE_ALWAYS"))) ? 1u : 0u;
+  P.dense_ok = (c->records_analyzed + n < (1ull << 32) && (n >= c->pre_elems || getenv("VE_DENSE_ALWAYS")) &&
+                dense_reserve(c)) ? 1u : 0u;
   if (P.dense_ok) c->dense_dirty = true;
   P.ring = ((uintptr_t)d % 16 == 0) ? 1u : 0u;
   P.nring = P.ring ? n / 32 : 0;
@@ -2524,15 +2546,26 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.hs = hs;
   carve_offsets(P, sp + so);
   const size_t sb = smem_bytes(sp + so, hs, P.objc);
-  cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sb);
+  // the attribute is per function, process-wide: set the device's maximum (every launch asks for
+  // sb <= it), so contexts launching from several host threads never undercut each other
+  cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       dev_smem - (int)fa.sharedSizeBytes);
   if (e != cudaSuccess) return cuda_fail(c, e, "cudaFuncSetAttribute(k_analyze)");
   if (n == 0) return VE_OK;
   uint64_t windows = (n + 31) / 32;
   uint64_t blocks = (windows + K1_WARPS - 1) / K1_WARPS;
+  if (c->cfg.min_windows_per_warp) {   // throughput mode (several contexts side by side): fewer, fuller CTAs
+    const uint64_t per = (uint64_t)c->cfg.min_windows_per_warp * (v2 ? K2_WARPS : K1_WARPS);
+    blocks = (windows + per - 1) / per;
+  }
   if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+  if (blocks == 0) blocks = 1;
   // a trace too short to give every warp a few CHUNK-window chunks (cfg5's kernels: a warp's
   // serial share of a 16-window chunk set a ~0.3 ms floor) is split into one-stage chunks
   P.chunk = P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? CHUNK : (uint32_t)STAGE_WIN;
+  // v2 claims its chunks dynamically (VE_CLAIM_MODE=0/1 forces the static / dynamic split)
+  const char* cm = getenv("VE_CLAIM_MODE");
+  P.claim = (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
   // staging regions: a warp stages at most one group per record of its static range
   {
     const uint64_t tw = blocks * K1_WARPS;
@@ -2551,10 +2584,10 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
     P.stage = (uint4*)c->hstage;
     P.stage_cnt = (uint32_t*)((uint8_t*)c->hstage + (size_t)tw * P.stage_rs * sizeof(uint4));
   }
-#if VE_CLAIM == 1
-  e = cudaMemsetAsync(P.work, 0, sizeof(unsigned long long), s);
-  if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze claim counter");
-#endif
+  if (P.claim) {
+    e = cudaMemsetAsync(P.work, 0, sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze claim counter");
+  }
   count_launch();
   kfn<<<(unsigned)blocks, v2 ? K2_THREADS : K1_THREADS, sb, s>>>(P);
   e = cudaGetLastError();
@@ -2568,6 +2601,7 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   k_line_fold<<<nsk, LF_THREADS, 0, s>>>(c->t.lcta, (uint32_t)blocks, nsk, sp, c->cfg.n_pcs, c->t.line);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_line_fold launch");
+  ctx_end(c, s);
   return VE_OK;
 }
 

@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(256) k_touched(const uint32_t* __restrict__ W,
 
 ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask, ve_diff* out, cudaStream_t s) {
   const HostObject& o = c->objs[oi];
-  if (c->reset_ev) cudaStreamWaitEvent(s, c->reset_ev, 0);
+  ctx_begin(c, s);
   // counted loads set their L bits when flushed: flush first, so n_untouched does not
   // depend on whether ve_report ran before this call (idempotent; ve_report skips it then)
   if (!c->hist_merged) {
@@ -178,6 +178,7 @@ ve_status run_diff(ve_ctx* c, uint32_t oi, uint32_t mode, const uint32_t* d_mask
   unsigned long long h[3];
   cudaMemcpyAsync(h, d_out, 24, cudaMemcpyDeviceToHost, s);
   cudaFreeAsync(d_out, s);
+  ctx_end(c, s);
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "ve_snapshot_diff");
   out->n_elems = o.n_elems;

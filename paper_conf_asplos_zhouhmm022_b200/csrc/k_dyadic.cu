@@ -328,6 +328,7 @@ extern "C" ve_status ve_dyadic_fit_ex(ve_ctx* c, const ve_record* d_records, uin
                                       ve_dyadic* h_out, cudaStream_t s) {
   if (!c || !h_out || (flags & ~VE_FIT_TRUNC)) return VE_ERR_INVALID;
   std::vector<DyKey> hk;
+  ctx_begin(c, s);
   ve_status st = dy_run(c, d_records, n, (flags & VE_FIT_TRUNC) ? c->cfg.mant_bits : DY_NOTRUNC, false, hk, s);
   if (st != VE_OK) return st;
   for (uint32_t k = 0; k < c->n_keys; ++k) {
@@ -354,6 +355,7 @@ extern "C" ve_status ve_outlier_fit(ve_ctx* c, const ve_record* d_records, uint6
                                     ve_outlier* h_out, cudaStream_t s) {
   if (!c || !h_out || (flags & ~VE_FIT_TRUNC)) return VE_ERR_INVALID;
   std::vector<DyKey> hk;
+  ctx_begin(c, s);
   ve_status st = dy_run(c, d_records, n, (flags & VE_FIT_TRUNC) ? c->cfg.mant_bits : DY_NOTRUNC, true, hk, s);
   if (st != VE_OK) return st;
   for (uint32_t k = 0; k < c->n_keys; ++k) {

@@ -858,7 +858,10 @@ template <int NT>
 __global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n_elems, const uint8_t* pre,
                                                            uint32_t ew, uint32_t tag, uint64_t bmoff, DevTables t,
                                                            uint32_t meta, uint32_t mant_bits, uint32_t kp, uint32_t ko,
-                                                           uint32_t ts, uint32_t csz, uint32_t setL) {
+                                                           uint32_t ts, uint32_t csz, uint32_t setL,
+                                                           const uint32_t* only_if = nullptr) {
+  // (only_if: the fallback of the per-object flush -- run only when its table overflowed)
+  if (only_if && *(volatile const uint32_t*)only_if == 0u) return;
   extern __shared__ unsigned long long df_smem[];
   unsigned long long* sbits = df_smem;
   uint32_t* scnt = reinterpret_cast<uint32_t*>(df_smem + ts);
@@ -1016,18 +1019,17 @@ __device__ void dense_sample_body(const uint32_t* cnt, uint64_t n_elems, const u
 // Every claim j of object o counts, per element e, the records of one (pc, access type) whose value
 // was e's PRE value (side 0, loads) or e's POST value (side 1, DENSE_POST): their histogram entries
 // are (tag_j, side value of e) with count c_j(e).  One pass over the object reads each snapshot side
-// once and every claim's counters, and aggregates in a block-local table:
-//   H0_side(v) = #elements of the pass with side value v (one insert per element and side), and
+// once and every claim's counters (k_dense_obj) and aggregates
+//   H0_side(v) = #elements with side value v (one insert per element and side), and
 //   D_j(v)    = sum of (c_j(e) - m_j) over the elements where c_j(e) != m_j,
-// m_j being a per-block base multiplicity (the mode of c_j over 32 sampled elements): stencils read
+// m_j being the claim's base multiplicity (the mode of c_j over 32 sampled elements): stencils read
 // every element once per PC, so H0 carries the whole count and corrections are few (clamped faces).
-// When the table is emptied, the local count of (j, v) is m_j * H0_side(v) + D_j(v) -- exactly the
-// number of counted records of claim j with value v among the elements of this table generation
-// (every D_j(v) of the generation has its H0_side(v) beside it); positive counts go to the HBM
-// table with their value statistics (C1 n_zero, C4-C7), so no zero-count entry is ever created.
+// Then (k_dense_emit) claim j's count of v over the object is m_j * H0_side(v) + D_j(v); positive
+// counts go to the HBM table with their value statistics (C1 n_zero, C4-C7), so no zero-count entry
+// is ever created.
 constexpr int DO_THREADS = 1024;
-// block table: 16-byte slots {value bits, cls << 56 | (count + 2^55)}: cls 0 / 1 = H0 of the pre / post
-// side, 2 + j = correction of claim j, 0xFF = empty; the biased 56-bit count takes signed adds
+// table slots (block and global): 16 bytes {value bits, cls << 56 | (count + 2^55)}: cls 0 / 1 = H0 of
+// the pre / post side, 2 + j = correction of claim j; the biased 56-bit count takes signed adds
 constexpr uint32_t DO_TS = 12288;                // 192 KiB of shared memory
 constexpr uint64_t DO_EMPTY = 0xFFull << 56;
 constexpr uint64_t DO_BIAS = 1ull << 55;
@@ -1182,165 +1184,192 @@ __global__ void k_dense_mode(const uint32_t* const* cnt, const uint64_t* ne, uin
   if (lane == 0) m[j] = mm;
 }
 
-__global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_constant__ DoArgs A, DevTables t) {
+// The object's (class, value) table in global memory: H0 of each side and the corrections D_j,
+// same slot format as the block table (empty = all ones).  Sized by the host from the sampled
+// cardinality; a full table sets *ovf and the claims take the per-array flush instead (exact).
+__device__ __forceinline__ bool gt_add(DoSlot* gt, uint32_t mask, uint32_t cls, uint64_t v, long long d, uint32_t* ovf) {
+  uint32_t h = (uint32_t)mix64(v ^ ((uint64_t)cls << 58)) & mask;
+  for (uint32_t probe = 0; probe <= mask && probe < 256u; ++probe) {
+    DoSlot* sl = &gt[h];
+    uint64_t lo, hi;
+    ld128_volatile(sl, lo, hi);
+    const uint32_t sc = (uint32_t)(hi >> 56);
+    // (an empty slot reads (~0, ~0): a match of value ~0 is confirmed by the CAS, never taken from the read)
+    if (sc == cls && lo == v && v != ~0ull) { atomicAdd((unsigned long long*)&sl->w, (unsigned long long)d); return true; }
+    if (sc == 0xFFu || (sc == cls && lo == v)) {
+      uint64_t olo, ohi;
+      cas128_global(sl, ~0ull, ~0ull, v, ((uint64_t)cls << 56) | DO_BIAS, olo, ohi);
+      if ((olo == ~0ull && ohi == ~0ull) || ((uint32_t)(ohi >> 56) == cls && olo == v)) {
+        atomicAdd((unsigned long long*)&sl->w, (unsigned long long)d);
+        return true;
+      }
+    }
+    h = (h + 1) & mask;
+  }
+  atomicExch(ovf, 1u);
+  return false;
+}
+__device__ __forceinline__ long long gt_get(const DoSlot* gt, uint32_t mask, uint32_t cls, uint64_t v) {
+  uint32_t h = (uint32_t)mix64(v ^ ((uint64_t)cls << 58)) & mask;
+  for (uint32_t probe = 0; probe <= mask && probe < 256u; ++probe) {
+    const DoSlot& sl = gt[h];
+    const uint32_t sc = (uint32_t)(sl.w >> 56);
+    if (sc == 0xFFu && sl.v == ~0ull) return 0;
+    if (sc == cls && sl.v == v) return do_cnt(sl.w);
+    h = (h + 1) & mask;
+  }
+  return 0;
+}
+
+// Pass 1 of the per-object flush: one read of every claim's counters and of each snapshot side.
+// H0 goes to the block table (one insert per element and side; values that do not fit go to the
+// global table), corrections (elements where c_j(e) != m_j: a stencil's clamped faces) straight to
+// the global table; at exit the block table is added into the global one.  No block barrier in the
+// loop and no per-claim emission here: the block table holds H0 only, so it never needs draining
+// (round 2's version drained it every few chunks -- 7 x 4096 contended HBM inserts per drain --
+// and checked its fill under a barrier every 8 batches: 20.6% of its stall samples).  The counters
+// are left as they are (zeroed by a memset after the emission, or by the fallback flush).
+__global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_constant__ DoArgs A, DevTables t, DoSlot* gt,
+                                                             uint32_t gmask, uint32_t* ovf) {
   extern __shared__ __align__(16) uint8_t do_smem[];
   DoSlot* ts = reinterpret_cast<DoSlot*>(do_smem);
-  __shared__ DoStat st[DO_MAXC];
   __shared__ uint32_t s_fill;
   const int tid = threadIdx.x, lane = tid & 31;
   for (uint32_t i = tid; i < DO_TS; i += blockDim.x) { ts[i].v = 0; ts[i].w = DO_EMPTY; }
-  if (tid < DO_MAXC * 6) st[tid / 6].s[tid % 6] = 0;
-  if (tid < DO_MAXC * 3) { st[tid / 3].mn[tid % 3] = ~0ull; st[tid / 3].mx[tid % 3] = 0; }
   if (tid == 0) s_fill = 0;
   uint32_t sides = 0;                                  // bit s: some claim reads side s
   for (uint32_t j = 0; j < A.nc; ++j) sides |= 1u << A.c[j].side;
   __syncthreads();
-  // empty the table: positive local counts of every (claim, value) -> HBM table + statistics
-  auto drain = [&]() {
-    __syncthreads();
-    for (uint32_t j = 0; j < A.nc; ++j) {
-      const uint32_t sd = A.c[j].side;
-      DoAcc acc;
-      do_acc_init(acc);
-      for (uint32_t i = tid; i < DO_TS; i += blockDim.x) {
-        const uint64_t w = ts[i].w;
-        if ((uint32_t)(w >> 56) != sd) continue;
-        const uint64_t v = ts[i].v;
-        const long long k = (long long)A.c[j].m * do_cnt(w) + do_get(ts, 2u + j, v);
-        if (k > 0) {
-          hist_insert_global_rf(t, A.c[j].tag, v, (unsigned long long)k);
-          do_acc(acc, v, (unsigned long long)k, A.c[j].meta, A.mant_bits);
-        }
-      }
-      do_acc_fold(st[j], acc);
-    }
-    __syncthreads();
-    for (uint32_t i = tid; i < DO_TS; i += blockDim.x) { ts[i].v = 0; ts[i].w = DO_EMPTY; }
-    if (tid == 0) s_fill = 0;
-    __syncthreads();
-  };
   const uint64_t nch = (A.ne + DO_CH - 1) / DO_CH;
   for (uint64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
-  const uint64_t lo = ch * DO_CH, hi = lo + DO_CH < A.ne ? lo + DO_CH : A.ne;
-  // the loads of a batch (the counters of all claims, the snapshot sides) are issued one batch
-  // ahead, so they are in flight while the previous batch is inserted
-  uint32_t ncj[DO_MAXC];
-  uint64_t nsv0 = 0, nsv1 = 0;
-  auto issue = [&](uint64_t b) {
-    const uint64_t e = b + tid;
-    const bool in = e < hi;
+    const uint64_t lo = ch * DO_CH, hi = lo + DO_CH < A.ne ? lo + DO_CH : A.ne;
+    // the loads of a batch (the counters of all claims, the snapshot sides) are issued one batch
+    // ahead, so they are in flight while the previous batch is inserted
+    uint32_t ncj[DO_MAXC];
+    uint64_t nsv0 = 0, nsv1 = 0;
+    auto issue = [&](uint64_t b) {
+      const uint64_t e = b + tid;
+      const bool in = e < hi;
 #pragma unroll
-    for (int j = 0; j < DO_MAXC; ++j) ncj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
-    nsv0 = (in && A.snap[0]) ? do_load(A.snap[0] + e * A.ew, A.ew) : 0ull;
-    nsv1 = (in && A.snap[1]) ? do_load(A.snap[1] + e * A.ew, A.ew) : 0ull;
-  };
-  issue(lo);
-  for (uint64_t base = lo; base < hi; base += DO_THREADS) {
-    const uint64_t e = base + tid;
-    const bool in = e < hi;
-    uint32_t cj[DO_MAXC];
+      for (int j = 0; j < DO_MAXC; ++j) ncj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
+      nsv0 = (in && A.snap[0]) ? do_load(A.snap[0] + e * A.ew, A.ew) : 0ull;
+      nsv1 = (in && A.snap[1]) ? do_load(A.snap[1] + e * A.ew, A.ew) : 0ull;
+    };
+    issue(lo);
+    for (uint64_t base = lo; base < hi; base += DO_THREADS) {
+      const uint64_t e = base + tid;
+      const bool in = e < hi;
+      uint32_t cj[DO_MAXC];
 #pragma unroll
-    for (int j = 0; j < DO_MAXC; ++j) cj[j] = ncj[j];
-    const uint64_t sv0 = nsv0, sv1 = nsv1;
-    if (base + DO_THREADS < hi) issue(base + DO_THREADS);
-    uint32_t corr = 0;                                 // claims whose count differs from their base
-    bool lbit = false;
-#pragma unroll
-    for (int j = 0; j < DO_MAXC; ++j) {
-      if ((uint32_t)j >= A.nc) break;
-      if (cj[j]) { __stcs(A.c[j].cnt + e, 0u); if (A.c[j].side == 0u) lbit = true; }
-      if (in && cj[j] != A.c[j].m) corr |= 1u << j;
-    }
-    // C3: a counted pre-value load started at element e (K1 leaves these L bits to the flush)
-    const unsigned lm = __ballot_sync(0xFFFFFFFFu, lbit);
-    if (lane == 0 && lm) atomicOr(&t.L[A.bmoff + (base + (uint64_t)(tid & ~31)) / 32], lm);
-    // the groups this lane leads: bit b (0, 1: H0 of a side; 2 + j: correction of claim j), sum gd[b]
-    uint32_t pend = 0;
-    long long gd[2 + DO_MAXC];
-#pragma unroll
-    for (int sd = 0; sd < 2; ++sd) {
-      gd[sd] = 0;
-      if (!((sides >> sd) & 1u)) continue;
-      const uint64_t v = sd ? sv1 : sv0;
-      const unsigned am = __ballot_sync(0xFFFFFFFFu, in);
-      if (in) {
-        const unsigned g = __match_any_sync(am, v);
-        if (lane == __ffs(g) - 1) { pend |= 1u << sd; gd[sd] = __popc(g); }
-      }
-    }
-#pragma unroll
-    for (int j = 0; j < DO_MAXC; ++j) gd[2 + j] = 0;
-    if (__any_sync(0xFFFFFFFFu, corr != 0u)) {         // (stencils: only at their faces)
+      for (int j = 0; j < DO_MAXC; ++j) cj[j] = ncj[j];
+      const uint64_t sv0 = nsv0, sv1 = nsv1;
+      if (base + DO_THREADS < hi) issue(base + DO_THREADS);
+      uint32_t corr = 0;                               // claims whose count differs from their base
+      bool lbit = false;
 #pragma unroll
       for (int j = 0; j < DO_MAXC; ++j) {
         if ((uint32_t)j >= A.nc) break;
-        const bool act = (corr >> j) & 1u;
-        const unsigned am = __ballot_sync(0xFFFFFFFFu, act);
-        if (act) {
-          const long long d = (long long)cj[j] - (long long)A.c[j].m;
-          const uint64_t v = A.c[j].side ? sv1 : sv0;
-          const unsigned g = __match_any_sync(am, v);
-          long long sum = d;
-          if (__popc(g) > 1) {                         // group sum: a shuffle from each member
-            sum = 0;
-            for (unsigned gg = g; gg; gg &= gg - 1) sum += __shfl_sync(g, d, __ffs(gg) - 1);
+        if (cj[j] && A.c[j].side == 0u) lbit = true;
+        if (in && cj[j] != A.c[j].m) corr |= 1u << j;
+      }
+      // C3: a counted pre-value load started at element e (K1 leaves these L bits to the flush)
+      const unsigned lm = __ballot_sync(0xFFFFFFFFu, lbit);
+      if (lane == 0 && lm) atomicOr(&t.L[A.bmoff + (base + (uint64_t)(tid & ~31)) / 32], lm);
+      // H0: no MATCH (it costs more than the shared atomics it would merge on a varied side)
+#pragma unroll
+      for (int sd = 0; sd < 2; ++sd) {
+        if (!((sides >> sd) & 1u)) continue;
+        const uint64_t v = sd ? sv1 : sv0;
+        const unsigned am = __ballot_sync(0xFFFFFFFFu, in);
+        if (!am) continue;
+        const int l0 = __ffs(am) - 1;
+        const uint64_t v0 = ((uint64_t)__shfl_sync(0xFFFFFFFFu, (uint32_t)(v >> 32), l0) << 32) |
+                            __shfl_sync(0xFFFFFFFFu, (uint32_t)v, l0);
+        // the lanes holding lane l0's value form one group (all of them for a = 1.0 or vol; most
+        // for a mostly-constant side), the others insert one element each
+        const unsigned eq0 = __ballot_sync(0xFFFFFFFFu, in && v == v0);
+        const unsigned rest = am & ~eq0;
+        unsigned eq1 = 0;
+        int l1 = 32;
+        if (rest) {                                  // a second group: the first other lane's value
+          l1 = __ffs(rest) - 1;
+          const uint64_t v1 = ((uint64_t)__shfl_sync(0xFFFFFFFFu, (uint32_t)(v >> 32), l1) << 32) |
+                              __shfl_sync(0xFFFFFFFFu, (uint32_t)v, l1);
+          eq1 = __ballot_sync(0xFFFFFFFFu, in && v == v1);
+        }
+        const bool g0 = (eq0 >> lane) & 1u, g1 = (eq1 >> lane) & 1u;
+        if (in && ((!g0 && !g1) || lane == l0 || lane == l1)) {
+          const long long c = g0 ? (long long)__popc(eq0) : g1 ? (long long)__popc(eq1) : 1ll;
+          if (!do_add(ts, (uint32_t)sd, v, c, &s_fill)) gt_add(gt, gmask, (uint32_t)sd, v, c, ovf);
+        }
+      }
+      if (__any_sync(0xFFFFFFFFu, corr != 0u)) {       // (stencils: only at their faces)
+#pragma unroll
+        for (int j = 0; j < DO_MAXC; ++j) {
+          if ((uint32_t)j >= A.nc) break;
+          const bool act = (corr >> j) & 1u;
+          const unsigned am = __ballot_sync(0xFFFFFFFFu, act);
+          if (act) {
+            const long long d = (long long)cj[j] - (long long)A.c[j].m;
+            const uint64_t v = A.c[j].side ? sv1 : sv0;
+            const unsigned g = __match_any_sync(am, v);
+            long long sum = d;
+            if (__popc(g) > 1) {                       // group sum: a shuffle from each member
+              sum = 0;
+              for (unsigned gg = g; gg; gg &= gg - 1) sum += __shfl_sync(g, d, __ffs(gg) - 1);
+            }
+            if (lane == __ffs(g) - 1 && sum != 0) gt_add(gt, gmask, 2u + (uint32_t)j, v, sum, ovf);
           }
-          if (lane == __ffs(g) - 1) { pend |= 1u << (2 + j); gd[2 + j] = sum; }
         }
       }
     }
-    // insert the warp's groups.  A table generation must hold all groups of the warp's 32 elements
-    // (H0 and corrections of the same elements), so should one not fit (64 probes full), the warp
-    // takes its inserted groups out again and sends its elements' counts to the HBM table one by one
-    // -- exact either way, and without a block barrier
-    uint32_t done = 0;
-#pragma unroll
-    for (int b = 0; b < 2 + DO_MAXC; ++b) {
-      if (!((pend >> b) & 1u)) continue;
-      const uint64_t v = (b == 1 || (b >= 2 && A.c[b - 2].side)) ? sv1 : sv0;
-      if (do_add(ts, (uint32_t)b, v, gd[b], &s_fill)) done |= 1u << b;
-    }
-    if (__any_sync(0xFFFFFFFFu, pend != done)) {
-#pragma unroll
-      for (int b = 0; b < 2 + DO_MAXC; ++b) {
-        if (!((done >> b) & 1u)) continue;
-        const uint64_t v = (b == 1 || (b >= 2 && A.c[b - 2].side)) ? sv1 : sv0;
-        do_add(ts, (uint32_t)b, v, -gd[b], &s_fill);    // present: always found
-      }
-      for (uint32_t j = 0; j < A.nc; ++j) {
-        DoAcc acc;
-        do_acc_init(acc);
-        const uint32_t c = cj[j];
-        if (c) {
-          const uint64_t v = A.c[j].side ? sv1 : sv0;
-          hist_insert_global_rf(t, A.c[j].tag, v, c);
-          do_acc(acc, v, c, A.c[j].meta, A.mant_bits);
-        }
-        do_acc_fold(st[j], acc);
-      }
-    }
-    // every 8 batches (block-uniform): drain a table past 60 %
-    if ((((base - lo) / DO_THREADS) & 7u) == 7u) {
-      __syncthreads();
-      if (s_fill > DO_TS * 6 / 10) drain();
-    }
   }
+  __syncthreads();
+  for (uint32_t i = tid; i < DO_TS; i += blockDim.x) {
+    const uint64_t w = ts[i].w;
+    if ((uint32_t)(w >> 56) != 0xFFu) gt_add(gt, gmask, (uint32_t)(w >> 56), ts[i].v, do_cnt(w), ovf);
   }
-  drain();
-  // statistics of every claim into its PC-key and object-key rows
-  if (tid < 2 * DO_MAXC) {
-    const uint32_t j = tid >> 1;
-    if (j < A.nc) {
-      const uint64_t key = (tid & 1) ? A.ko : A.c[j].kp;
-      const DoStat& S = st[j];
+}
+
+// Pass 2: the claims' histogram entries and value statistics.  For every H0 entry (side, v) and
+// every claim j of that side, claim j's count of v over the whole object is m_j * H0(v) + D_j(v)
+// (every corrected element's value is in H0); positive counts go to the HBM table, so no zero-count
+// entry is ever created.  Skipped when pass 1 overflowed the global table (the fallback runs).
+__global__ void __launch_bounds__(256) k_dense_emit(const __grid_constant__ DoArgs A, DevTables t, const DoSlot* gt,
+                                                    uint32_t gmask, const uint32_t* ovf) {
+  if (*(volatile const uint32_t*)ovf) return;
+  __shared__ DoStat st;
+  const int tid = threadIdx.x;
+  for (uint32_t j = 0; j < A.nc; ++j) {
+    if (tid < 6) st.s[tid] = 0;
+    if (tid < 3) { st.mn[tid] = ~0ull; st.mx[tid] = 0; }
+    __syncthreads();
+    const uint32_t sd = A.c[j].side;
+    DoAcc acc;
+    do_acc_init(acc);
+    for (uint32_t i = blockIdx.x * blockDim.x + tid; i <= gmask; i += gridDim.x * blockDim.x) {
+      const uint64_t w = gt[i].w;
+      if ((uint32_t)(w >> 56) != sd) continue;
+      const uint64_t v = gt[i].v;
+      const long long k = (long long)A.c[j].m * do_cnt(w) + gt_get(gt, gmask, 2u + j, v);
+      if (k > 0) {
+        hist_insert_global_rf(t, A.c[j].tag, v, (unsigned long long)k);
+        do_acc(acc, v, (unsigned long long)k, A.c[j].meta, A.mant_bits);
+      }
+    }
+    do_acc_fold(st, acc);
+    __syncthreads();
+    if (tid < 2) {
+      const uint64_t key = tid ? A.ko : A.c[j].kp;
       const int f[6] = {F_ZERO, F_NAN, F_NONINT, F_NF16, F_NBF16, F_NF32};
       for (int i = 0; i < 6; ++i)
-        if (S.s[i]) atomicAdd(&t.sum[key * NSUM + f[i]], S.s[i]);
+        if (st.s[i]) atomicAdd(&t.sum[key * NSUM + f[i]], st.s[i]);
       for (int i = 0; i < 3; ++i) {
-        if (S.mn[i] != ~0ull) atomicMin(&t.mn[key * NMM + i], S.mn[i]);
-        if (S.mx[i] != 0ull) atomicMax(&t.mx[key * NMM + i], S.mx[i]);
+        if (st.mn[i] != ~0ull) atomicMin(&t.mn[key * NMM + i], st.mn[i]);
+        if (st.mx[i] != 0ull) atomicMax(&t.mx[key * NMM + i], st.mx[i]);
       }
     }
+    __syncthreads();
   }
 }
 
@@ -1419,10 +1448,17 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   const size_t smem = (size_t)DO_TS * sizeof(DoSlot);
   cudaFuncSetAttribute(k_dense_obj, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_SLOTS * 12));
+  // per object: its claims for the fused flush (others: the per-array flush right away)
+  std::vector<DoArgs> objargs;
+  std::vector<std::vector<size_t>> objcl;        // claim indices (into cl) of each DoArgs
+  std::vector<uint32_t> objmask;                 // global table slots - 1
+  std::vector<uint32_t> objidx;
   for (uint32_t i = 0; i < c->n_obj; ++i) {
     const HostObject& o = c->objs[i];
     DoArgs A;
     memset(&A, 0, sizeof(A));
+    std::vector<size_t> mine;
+    uint32_t ndmax = 0;
     for (size_t k = 0; k < nc; ++k) {
       if (cl[k].i != i) continue;
       const uint32_t ck = cl[k].ck, pc = ck & 0xFFFFu, meta = (ck >> 16) & 0x3Fu;
@@ -1444,6 +1480,8 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
       d.kp = pc;
       d.m = mh[k];
       A.snap[d.side] = (const uint8_t*)(post ? o.post : o.pre);
+      mine.push_back(k);
+      ndmax = std::max(ndmax, nd[k]);
     }
     if (!A.nc) continue;
     A.ew = o.ew;
@@ -1451,11 +1489,55 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
     A.mant_bits = c->cfg.mant_bits;
     A.ne = o.size / o.ew;                  // whole elements (K1 counts only those)
     A.bmoff = o.bmoff;
-    uint64_t blocks = (A.ne + DO_CH - 1) / DO_CH;
-    if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
-    if (blocks == 0) blocks = 1;
-    count_launch();
-    k_dense_obj<<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t);
+    // global (class, value) table: H0 of <= 2 sides and <= nc correction classes over the sampled
+    // cardinality (<= 4096 here), at most half full
+    uint64_t want = 2ull * (2u + A.nc) * (uint64_t)std::max(ndmax + 64u, 1024u), cap = 1024;
+    while (cap < want) cap <<= 1;
+    objargs.push_back(A);
+    objcl.push_back(mine);
+    objmask.push_back((uint32_t)(cap - 1));
+    objidx.push_back(i);
+  }
+  if (!objargs.empty()) {
+    size_t tot = 0;
+    std::vector<size_t> toff(objargs.size());
+    for (size_t q = 0; q < objargs.size(); ++q) { toff[q] = tot; tot += ((size_t)objmask[q] + 1) * sizeof(DoSlot); }
+    const size_t fo = tot;
+    tot += 4 * objargs.size();
+    uint8_t* gbuf = nullptr;
+    e = cudaMallocAsync((void**)&gbuf, tot, s);
+    if (e != cudaSuccess) return cuda_fail(c, e, "dense_flush table alloc");
+    cudaMemsetAsync(gbuf, 0xFF, fo, s);
+    cudaMemsetAsync(gbuf + fo, 0, tot - fo, s);
+    for (size_t q = 0; q < objargs.size(); ++q) {
+      const DoArgs& A = objargs[q];
+      const HostObject& o = c->objs[objidx[q]];
+      DoSlot* gt = (DoSlot*)(gbuf + toff[q]);
+      uint32_t* ovf = (uint32_t*)(gbuf + fo) + q;
+      uint64_t blocks = (A.ne + DO_CH - 1) / DO_CH;
+      if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
+      if (blocks == 0) blocks = 1;
+      count_launch();
+      k_dense_obj<<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t, gt, objmask[q], ovf);
+      uint64_t eb = ((uint64_t)objmask[q] + 1) / 256;
+      eb = std::max<uint64_t>(1, std::min<uint64_t>(eb, 4ull * c->num_sms));
+      count_launch();
+      k_dense_emit<<<(unsigned)eb, 256, 0, s>>>(A, c->t, gt, objmask[q], ovf);
+      // fallback (only when the table overflowed: the kernels return at once otherwise): the
+      // per-array flush of every claim, exact at any cardinality
+      for (size_t k : objcl[q]) {
+        const uint32_t ck = cl[k].ck, pc = ck & 0xFFFFu, meta = (ck >> 16) & 0x3Fu;
+        const bool post = (ck & DENSE_POST) != 0u;
+        uint32_t* arr = (uint32_t*)c->dense_pool + cl[k].off;
+        const uint64_t fb = std::min<uint64_t>((o.n_elems + DF_CHUNK - 1) / DF_CHUNK, 2ull * c->num_sms);   // (grid-stride)
+        count_launch();
+        k_dense_flush<DF_THREADS><<<(unsigned)fb, DF_THREADS, DF_SLOTS * 12, s>>>(
+            arr, o.n_elems, (const uint8_t*)(post ? o.post : o.pre), o.ew, (pc << 16) | o.id, o.bmoff, c->t, meta,
+            c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id, (uint32_t)DF_SLOTS, (uint32_t)DF_CHUNK, post ? 0u : 1u, ovf);
+      }
+      for (uint32_t j = 0; j < A.nc; ++j) cudaMemsetAsync(A.c[j].cnt, 0, o.n_elems * 4, s);   // counters for the next epoch
+    }
+    cudaFreeAsync(gbuf, s);
   }
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "dense flush launch");

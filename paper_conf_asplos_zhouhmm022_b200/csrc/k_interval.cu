@@ -699,6 +699,7 @@ ve_status ve_temporal_loads_ex(ve_ctx* c, const ve_record* d_records, uint64_t n
                                uint64_t* h_pairs, cudaStream_t s) {
   if (!c || !h_out) return VE_ERR_INVALID;
   const uint32_t nk = c->n_keys;
+  ctx_begin(c, s);
   const uint64_t npairs = (uint64_t)c->cfg.n_pcs * (c->n_obj + 1);
   if (h_pairs && npairs > (1ull << 24)) return fail(c, VE_ERR_INVALID, "ve_temporal_loads_ex: n_pcs x (objects + 1) > 2^24");
   memset(h_out, 0, sizeof(uint64_t) * 2 * nk);
@@ -764,6 +765,7 @@ ve_status ve_interval_merge(ve_ctx* c, const ve_interval* d_in, uint64_t n, ve_i
   if (!c || !h_n_out) return VE_ERR_INVALID;
   *h_n_out = 0;
   if (n == 0) return VE_OK;
+  ctx_begin(c, s);
   if (!d_in || !d_out) return fail(c, VE_ERR_INVALID, "ve_interval_merge: null interval array");
   if (n >= (1ull << 32)) return fail(c, VE_ERR_INVALID, "ve_interval_merge: n >= 2^32");
   cudaSetDevice(c->device);
@@ -790,6 +792,7 @@ ve_status ve_record_intervals(ve_ctx* c, const ve_record* d_records, uint64_t n,
   if (!c || !h_n_out) return VE_ERR_INVALID;
   *h_n_out = 0;
   if (n == 0) return VE_OK;
+  ctx_begin(c, s);
   if (!d_records || !d_out || ((uintptr_t)d_records & 7))
     return fail(c, VE_ERR_INVALID, "ve_record_intervals: null or misaligned array");
   if (n >= (1ull << 32)) return fail(c, VE_ERR_INVALID, "ve_record_intervals: n >= 2^32");
@@ -817,6 +820,7 @@ ve_status ve_plan_copies(ve_ctx* c, const ve_interval* d_merged, uint64_t n, uin
   if (!c || (c->n_obj && !h_plan)) return VE_ERR_INVALID;
   if (n && !d_merged) return fail(c, VE_ERR_INVALID, "ve_plan_copies: null interval array");
   if (dense_pct > 100) return fail(c, VE_ERR_INVALID, "ve_plan_copies: dense_pct > 100");
+  ctx_begin(c, s);
   const uint32_t no = c->n_obj;
   if (no == 0) return VE_OK;
   cudaSetDevice(c->device);

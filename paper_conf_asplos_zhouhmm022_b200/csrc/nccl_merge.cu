@@ -416,7 +416,10 @@ ve_status ve_merge_group(ve_ctx** ctxs, uint32_t n, cudaStream_t s) {
   SimComm comm;
   comm.G = (int)n;
   for (uint32_t i = 0; i < n; ++i) comm.local.push_back((int)i);
-  return merge_ranks(cs, comm, s);
+  for (ve_ctx* c : cs) ctx_begin(c, s);
+  const ve_status st = merge_ranks(cs, comm, s);
+  for (ve_ctx* c : cs) ctx_end(c, s);
+  return st;
 }
 
 // S10 / S11 sharded by object: see diff_ranks / dedup_ranks
@@ -449,6 +452,7 @@ ve_status ve_object_dedup_comm(ve_ctx* ctx, const ve_object* objs, uint32_t n, v
   cudaSetDevice(ctx->device);
   NcclComm comm;
   ve_status st = comm_of(ctx, nccl_comm, comm);
+  ctx_begin(ctx, s);
   return st != VE_OK ? st : dedup_ranks({ctx}, comm, objs, n, h_group_of, s);
 }
 
@@ -474,6 +478,7 @@ ve_status ve_object_dedup_group(ve_ctx** ctxs, uint32_t n, const ve_object* objs
   SimComm comm;
   comm.G = (int)n;
   for (uint32_t i = 0; i < n; ++i) comm.local.push_back((int)i);
+  for (ve_ctx* c : cs) ctx_begin(c, s);
   return dedup_ranks(cs, comm, objs, n_objs, h_group_of, s);
 }
 

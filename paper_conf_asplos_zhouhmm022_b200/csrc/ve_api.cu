@@ -53,7 +53,43 @@ static void free_dev(ve_ctx* c) {
     if (c->copied_ev[i]) cudaEventDestroy(c->copied_ev[i]);
   }
   if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
-  if (c->reset_ev) cudaEventDestroy(c->reset_ev);
+  if (c->ord_ev) cudaEventDestroy(c->ord_ev);
+  if (c->cs) cudaStreamDestroy(c->cs);
+}
+
+// make the dense counter pool hold the current object set's claims (dense_want counters), allocated
+// on first need; false when there is no memory for it (the calls then count through the hash path)
+bool dense_reserve(ve_ctx* c) {
+  if (c->dense_want == 0) return false;
+  if (c->dense_pool && c->dense_cap >= c->dense_want) return true;
+  if (ctx_quiesce(c) != cudaSuccess) return false;   // (the old pool may still be read)
+  if (c->dense_pool) cudaFree(c->dense_pool);
+  c->dense_pool = nullptr;
+  c->dense_cap = 0;
+  c->dense_dirty = false;
+  if (cudaMalloc(&c->dense_pool, c->dense_want * 4) != cudaSuccess ||
+      cudaMemsetAsync(c->dense_pool, 0, c->dense_want * 4, c->cs) != cudaSuccess) {
+    cudaGetLastError();
+    if (c->dense_pool) cudaFree(c->dense_pool);
+    c->dense_pool = nullptr;
+    c->dense_want = 0;                                 // no memory: this object set uses the hash path
+    return false;
+  }
+  if (cudaStreamSynchronize(c->cs) != cudaSuccess) return false;   // (rare: the caller's launch follows)
+  c->dense_cap = c->dense_want;
+  c->o.dense_pool = (uint32_t*)c->dense_pool;
+  c->o.dense_cap = c->dense_cap;
+  return true;
+}
+
+void ctx_begin(ve_ctx* c, cudaStream_t s) {
+  if (c->ord_ev) cudaStreamWaitEvent(s, c->ord_ev, 0);
+}
+void ctx_end(ve_ctx* c, cudaStream_t s) {
+  if (c->ord_ev) cudaEventRecord(c->ord_ev, s);
+}
+cudaError_t ctx_quiesce(ve_ctx* c) {
+  return c->ord_ev ? cudaEventSynchronize(c->ord_ev) : cudaSuccess;
 }
 
 // empty the occupied slots recorded in t.occ (the table's only non-empty slots), then their count
@@ -70,6 +106,7 @@ __global__ void k_reset_occ(DevTables t) {
 }
 
 ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
+  ctx_begin(c, s);
   const uint64_t nk_max = (uint64_t)c->cfg.n_pcs + c->cfg.max_objects + 1;
   cudaMemsetAsync(c->t.sum, 0, nk_max * NSUM * 8, s);
   cudaMemsetAsync(c->t.mn, 0xFF, nk_max * NMM * 8, s);
@@ -105,7 +142,7 @@ ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
   cudaError_t e = full ? cudaMemsetAsync(c->t.hcount, 0, c->hcap * 8, s) : cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "reset");
   c->table_clean = true;
-  if (c->reset_ev) cudaEventRecord(c->reset_ev, s);
+  ctx_end(c, s);
   c->poisoned = false;
   c->hist_merged = false;
   c->merged_ndistinct.clear();
@@ -246,8 +283,14 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
   }
   c->n_obj = 0;
   c->n_keys = cfg->n_pcs + 1;
-  if (cudaEventCreateWithFlags(&c->reset_ev, cudaEventDisableTiming) != cudaSuccess) c->reset_ev = nullptr;
-  if (launch_reset(c, 0) != VE_OK || cudaDeviceSynchronize() != cudaSuccess) {
+  if (cudaEventCreateWithFlags(&c->ord_ev, cudaEventDisableTiming) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    free_dev(c);
+    delete c;
+    return VE_ERR_CUDA;
+  }
+  if (launch_reset(c, c->cs) != VE_OK || cudaStreamSynchronize(c->cs) != cudaSuccess) {
     free_dev(c);
     delete c;
     return VE_ERR_CUDA;
@@ -259,7 +302,8 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
 ve_status ve_destroy(ve_ctx* c) {
   if (!c) return VE_ERR_INVALID;
   cudaSetDevice(c->device);
-  cudaDeviceSynchronize();
+  ctx_quiesce(c);
+  if (c->cs) cudaStreamSynchronize(c->cs);
   free_dev(c);
   delete c;
   return VE_OK;
@@ -293,7 +337,10 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     words += o.bmwords;
   }
   cudaSetDevice(c->device);
-  cudaDeviceSynchronize();
+  // the buffers below are reused or replaced: the ctx's queued work (any stream) must be done
+  // (a wait on this ctx's work only -- other contexts and the application keep running)
+  cudaError_t qe = ctx_quiesce(c);
+  if (qe != cudaSuccess) return cuda_fail(c, qe, "ve_set_objects (pending work)");
   if (words > c->bm_words || !c->t.W) {
     cudaFree(c->t.W);
     cudaFree(c->t.L);
@@ -323,24 +370,9 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   }
   c->pre_elems = pre_elems;
   if (want > DENSE_BUDGET) want = DENSE_BUDGET;
-  if (want > c->dense_cap) {
-    if (c->dense_pool) {
-      cudaDeviceSynchronize();
-      cudaFree(c->dense_pool);
-    }
-    c->dense_pool = nullptr;
-    c->dense_cap = 0;
-    if (cudaMalloc(&c->dense_pool, want * 4) != cudaSuccess ||
-        cudaMemset(c->dense_pool, 0, want * 4) != cudaSuccess) {
-      cudaGetLastError();
-      if (c->dense_pool) cudaFree(c->dense_pool);
-      c->dense_pool = nullptr;                         // no memory: everything goes to the hash path
-      std::fill(c->dense_pc_init.begin(), c->dense_pc_init.end(), DENSE_OFF);
-    } else {
-      c->dense_cap = want;
-    }
-    c->dense_dirty = false;
-  }
+  // the pool itself is allocated by the first analysis call that may count densely (dense_reserve):
+  // a ctx whose calls never carry a record per pre element (cfg5's kernels) holds no pool
+  c->dense_want = want;
   // device object table (SoA, sorted by base); the block is reused when it is large
   // enough (after the device is idle: earlier launches may still read the old table)
   const size_t nn = n ? n : 1;
@@ -369,7 +401,7 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     c->sorted_of_id[v[i].id] = i;
   }
   for (size_t k = 0; k < (size_t)DENSE_PER_OBJ * n; ++k) { hdo[k] = DENSE_NOT_READY; hdp[k] = c->dense_pc_init[k]; }
-  cudaMemcpy(c->obj_block, host.data(), nb, cudaMemcpyHostToDevice);
+  cudaMemcpyAsync(c->obj_block, host.data(), nb, cudaMemcpyHostToDevice, c->cs);   // (pageable: staged before return)
   uint64_t* db = (uint64_t*)c->obj_block;
   c->o.base = db;
   c->o.end = db + n;
@@ -381,27 +413,24 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   c->o.ew = c->o.id + n;
   c->o.dense_pc = const_cast<uint32_t*>(c->o.ew + n);
   c->o.dense_pool = (uint32_t*)c->dense_pool;
-  c->o.dense_cap = c->dense_cap;
+  c->o.dense_cap = c->dense_pool ? std::min(c->dense_cap, c->dense_want) : 0;
   c->o.dense_next = c->t.glob + G_DENSE_NEXT;
   c->o.n = n;
   c->objs = v;
   c->n_obj = n;
   c->n_keys = c->cfg.n_pcs + n + 1;
-  // the reset runs on the legacy stream; the analysis / diff calls wait for its event on their
-  // stream (no host synchronisation per object set)
-  return launch_reset(c, 0);
+  // the reset runs on the ctx stream; the analysis / diff calls wait for it on their stream
+  // (no host synchronisation per object set)
+  return launch_reset(c, c->cs);
 }
 
 ve_status ve_reset(ve_ctx* c) {
   if (!ctx_ok(c)) return VE_ERR_INVALID;
   cudaSetDevice(c->device);
-  // work still queued on other (non-blocking) streams may write the tables: let it finish
-  // before the reset memsets, which run on the legacy stream
-  cudaError_t e = cudaDeviceSynchronize();
-  if (e != cudaSuccess) return cuda_fail(c, e, "ve_reset (pending work)");
-  ve_status st = launch_reset(c, 0);
+  // the reset is ordered after the ctx's queued work on any stream (ctx_begin in launch_reset)
+  ve_status st = launch_reset(c, c->cs);
   if (st != VE_OK) return st;
-  e = cudaDeviceSynchronize();
+  cudaError_t e = cudaStreamSynchronize(c->cs);
   return e == cudaSuccess ? VE_OK : cuda_fail(c, e, "ve_reset");
 }
 
@@ -488,26 +517,34 @@ ve_status ve_snapshot_diff(ve_ctx* c, uint32_t obj_id, uint32_t mode, const uint
 
 ve_status ve_object_dedup(ve_ctx* c, const ve_object* objs, uint32_t n, uint32_t* h_group_of, cudaStream_t s) {
   if (!ctx_ok(c) || (n && (!objs || !h_group_of))) return VE_ERR_INVALID;
-  return run_dedup(c, objs, n, h_group_of, s);
+  ctx_begin(c, s);
+  const ve_status st = run_dedup(c, objs, n, h_group_of, s);
+  ctx_end(c, s);
+  return st;
 }
 
 ve_status ve_merge_stats(ve_ctx* dst, const ve_ctx* src, void* comm, cudaStream_t s) {
   if (!ctx_ok(dst) || (!src && !comm) || (src && comm)) return VE_ERR_INVALID;
   if (dst->hist_merged) return fail(dst, VE_ERR_STATE, "ve_merge_stats: ctx already merged over ranks");
   cudaSetDevice(dst->device);
-  if (src) return merge_local(dst, src, s);
-  return merge_nccl(dst, comm, s);
+  ctx_begin(dst, s);
+  if (src) ctx_begin(const_cast<ve_ctx*>(src), s);   // (waits for src's queued work; src's order is unchanged)
+  const ve_status st = src ? merge_local(dst, src, s) : merge_nccl(dst, comm, s);
+  ctx_end(dst, s);
+  return st;
 }
 
 ve_status ve_report(ve_ctx* c, ve_rep** out) {
   if (!ctx_ok(c) || !out) return VE_ERR_INVALID;
   *out = nullptr;
   cudaSetDevice(c->device);
-  cudaError_t e = cudaDeviceSynchronize();
+  cudaStream_t cs = c->cs;
+  ctx_begin(c, cs);                 // after the ctx's analyses, on whatever stream they ran
+  unsigned long long glob[8];
+  cudaError_t e = cudaMemcpyAsync(glob, c->t.glob, sizeof(glob), cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
   if (e != cudaSuccess) return cuda_fail(c, e, "ve_report (pending work)");
   if (c->poisoned) return fail(c, VE_ERR_STATE, "ve_report: ctx poisoned by histogram overflow; ve_reset");
-  unsigned long long glob[8];
-  cudaMemcpy(glob, c->t.glob, sizeof(glob), cudaMemcpyDeviceToHost);
   if (glob[G_OVERFLOW]) {
     c->poisoned = true;
     return fail(c, VE_ERR_CAPACITY, "value histogram capacity exceeded (hist_capacity)");
@@ -517,10 +554,10 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
   const bool tm = getenv("VE_TIMING") != nullptr;
   auto t0 = std::chrono::steady_clock::now();
   if (!c->hist_merged) {
-    ve_status st = dense_flush(c, 0);
+    ve_status st = dense_flush(c, cs);
     if (st != VE_OK) return st;
     if (tm) {
-      cudaDeviceSynchronize();
+      cudaStreamSynchronize(cs);
       fprintf(stderr, "[ve] dense_flush %.3f ms\n",
               std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
       t0 = std::chrono::steady_clock::now();
@@ -541,11 +578,11 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
       c->rpin_bytes = need;
     }
     uint8_t* hp = (uint8_t*)c->rpin;
-    cudaMemcpyAsync(hp, c->t.sum, bs, cudaMemcpyDeviceToHost, 0);
-    cudaMemcpyAsync(hp + bs, c->t.mn, bm, cudaMemcpyDeviceToHost, 0);
-    cudaMemcpyAsync(hp + bs + bm, c->t.mx, bm, cudaMemcpyDeviceToHost, 0);
-    cudaMemcpyAsync(hp + bs + 2 * bm, c->t.line, bl, cudaMemcpyDeviceToHost, 0);
-    e = cudaStreamSynchronize(0);
+    cudaMemcpyAsync(hp, c->t.sum, bs, cudaMemcpyDeviceToHost, cs);
+    cudaMemcpyAsync(hp + bs, c->t.mn, bm, cudaMemcpyDeviceToHost, cs);
+    cudaMemcpyAsync(hp + bs + bm, c->t.mx, bm, cudaMemcpyDeviceToHost, cs);
+    cudaMemcpyAsync(hp + bs + 2 * bm, c->t.line, bl, cudaMemcpyDeviceToHost, cs);
+    e = cudaStreamSynchronize(cs);
     if (e != cudaSuccess) return cuda_fail(c, e, "ve_report copy");
     memcpy(sum.data(), hp, bs);
     memcpy(mn.data(), hp + bs, bm);
@@ -563,15 +600,15 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
     nd = c->merged_ndistinct;
     r->top = c->merged_topk;
   } else {
-    st = finalize_hist(c, 0, nd, r->top);
+    st = finalize_hist(c, cs, nd, r->top);
     if (tm) {
-      cudaDeviceSynchronize();
+      cudaStreamSynchronize(cs);
       fprintf(stderr, "[ve] finalize_hist %.3f ms\n",
               std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
     }
     if (st != VE_OK) { delete r; return st; }
   }
-  st = bitmap_counts(c, 0, r->objs);
+  st = bitmap_counts(c, cs, r->objs);
   if (st != VE_OK) { delete r; return st; }
   r->keys.assign(nk, ve_key_stats{});
   for (uint32_t k = 0; k < nk; ++k) {
@@ -606,6 +643,13 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
   r->glob.n_invalid = glob[G_INVALID];
   r->glob.n_unmapped = glob[G_UNMAPPED];
   r->glob.hist_entries = 0;
+  if (!c->hist_merged) {   // occupied value-table slots after the dense flush (implementation statistic)
+    unsigned long long nocc = 0;
+    if (cudaMemcpyAsync(&nocc, c->t.glob + G_NOCC, 8, cudaMemcpyDeviceToHost, cs) == cudaSuccess &&
+        cudaStreamSynchronize(cs) == cudaSuccess)
+      r->glob.hist_entries = nocc;
+  }
+  ctx_end(c, cs);
   *out = r;
   return VE_OK;
 }
@@ -617,6 +661,7 @@ ve_status ve_approx_topk(ve_ctx* c, uint64_t* h_ndistinct, ve_topk_entry* h_top,
   if (c->poisoned) return fail(c, VE_ERR_STATE, "ve_approx_topk: ctx poisoned by histogram overflow; ve_reset");
   if (c->hist_merged)
     return fail(c, VE_ERR_STATE, "ve_approx_topk: the histogram of a rank-merged ctx is partitioned over ranks");
+  ctx_begin(c, s);
   ve_status st = dense_flush(c, s);   // counted loads -> exact histogram (idempotent)
   if (st != VE_OK) return st;
   const uint32_t nk = c->n_keys, K = c->cfg.topk;
@@ -688,14 +733,27 @@ ve_status ve_report_dump(const ve_rep* r, const char* path, int format) {
             (unsigned long long)r->glob.n_unmapped);
     for (uint32_t k = 0; k < r->n_keys; ++k) {
       const ve_key_stats& s = r->keys[k];
+      typedef unsigned long long ull;
       fprintf(f,
               "  {\"key\": %u, \"n_ld\": %llu, \"n_st\": %llu, \"n_zero\": %llu, \"n_ld_eq_pre\": %llu, "
-              "\"n_st_eq_pre\": %llu, \"n_distinct\": %llu, \"single_value\": %u, \"single_zero\": %u, "
-              "\"frequent\": %u, \"structured\": %u, \"approx\": %u, \"dict8\": %u, \"heavy\": \"%s\", \"top\": [",
-              k, (unsigned long long)s.n_ld, (unsigned long long)s.n_st, (unsigned long long)s.n_zero,
-              (unsigned long long)s.n_ld_eq_pre, (unsigned long long)s.n_st_eq_pre,
-              (unsigned long long)s.n_distinct, s.single_value, s.single_zero, s.frequent, s.structured, s.approx,
-              s.dict8, s.heavy < 12 ? tn[s.heavy] : "none");
+              "\"n_st_eq_pre\": %llu, \"n_nosnap\": %llu, \"n_distinct\": %llu, \"single_value\": %u, "
+              "\"single_zero\": %u, \"frequent\": %u, \"structured\": %u, \"approx\": %u, \"dict8\": %u, "
+              "\"heavy\": \"%s\", \"single_type\": %u, ",
+              k, (ull)s.n_ld, (ull)s.n_st, (ull)s.n_zero, (ull)s.n_ld_eq_pre, (ull)s.n_st_eq_pre, (ull)s.n_nosnap,
+              (ull)s.n_distinct, s.single_value, s.single_zero, s.frequent, s.structured, s.approx, s.dict8,
+              s.heavy < 12 ? tn[s.heavy] : "none", s.single_type);
+      // C5 float flags, C4 / C5 / C7 ranges, C8 line (y as signed 128-bit: hi, lo words), n_type
+      fprintf(f,
+              "\"n_nan\": %llu, \"n_nonint\": %llu, \"n_not_f16\": %llu, \"n_not_bf16\": %llu, \"n_not_f32\": %llu, "
+              "\"raw_min\": %llu, \"raw_max\": %llu, \"ord_min\": %llu, \"ord_max\": %llu, \"trunc_min\": %llu, "
+              "\"trunc_max\": %llu, \"line_state\": %llu, \"p\": [%llu, %lld, %llu], \"q\": [%llu, %lld, %llu], "
+              "\"n_type\": [",
+              (ull)s.n_nan, (ull)s.n_nonint, (ull)s.n_not_f16, (ull)s.n_not_bf16, (ull)s.n_not_f32, (ull)s.raw_min,
+              (ull)s.raw_max, (ull)s.ord_min, (ull)s.ord_max, (ull)s.trunc_min, (ull)s.trunc_max,
+              (ull)s.line_state, (ull)s.p_x, (long long)s.p_yhi, (ull)s.p_ylo, (ull)s.q_x, (long long)s.q_yhi,
+              (ull)s.q_ylo);
+      for (int t = 0; t < 12; ++t) fprintf(f, "%s%llu", t ? ", " : "", (ull)s.n_type[t]);
+      fprintf(f, "], \"top\": [");
       for (uint64_t j = 0; j < s.n_top; ++j)
         fprintf(f, "%s[%llu, %llu]", j ? ", " : "", (unsigned long long)r->top[(size_t)k * r->topk + j].bits,
                 (unsigned long long)r->top[(size_t)k * r->topk + j].count);
@@ -704,9 +762,11 @@ ve_status ve_report_dump(const ve_rep* r, const char* path, int format) {
     fprintf(f, "], \"objects\": [\n");
     for (uint32_t i = 0; i < r->n_obj; ++i) {
       const ve_obj_stats& o = r->objs[i];
-      fprintf(f, "  {\"id\": %u, \"n_elems\": %llu, \"n_written\": %llu, \"n_ld_reload\": %llu, \"n_touched\": %llu}%s\n",
-              i, (unsigned long long)o.n_elems, (unsigned long long)o.n_written, (unsigned long long)o.n_ld_reload,
-              (unsigned long long)o.n_touched, i + 1 < r->n_obj ? "," : "");
+      fprintf(f,
+              "  {\"id\": %u, \"n_elems\": %llu, \"n_written\": %llu, \"n_loaded_eq\": %llu, \"n_ld_reload\": %llu, "
+              "\"n_touched\": %llu}%s\n",
+              i, (unsigned long long)o.n_elems, (unsigned long long)o.n_written, (unsigned long long)o.n_loaded_eq,
+              (unsigned long long)o.n_ld_reload, (unsigned long long)o.n_touched, i + 1 < r->n_obj ? "," : "");
     }
     fprintf(f, "]}\n");
   }

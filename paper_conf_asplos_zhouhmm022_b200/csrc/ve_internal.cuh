@@ -116,7 +116,12 @@ struct ve_ctx {
   bool poisoned = false;
   bool hist_merged = false;  // set by an NCCL merge: top-k/n_distinct precomputed
   bool table_clean = false;  // the value table holds only the slots recorded in t.occ (else: full clear)
-  cudaEvent_t reset_ev = nullptr;   // recorded after every reset (legacy stream); launches on s wait on it
+  // Stream order of the ctx's work (no device-wide synchronisation anywhere): every call that
+  // touches the ctx's device state waits for ord_ev on its stream first and records ord_ev there
+  // after its last launch (ctx_begin / ctx_end), so the ctx's calls run in call order whatever
+  // streams they use; ctx-internal work (resets, the report) runs on the ctx's own stream cs.
+  cudaEvent_t ord_ev = nullptr;
+  cudaStream_t cs = nullptr;
   uint32_t n_obj = 0;
   uint32_t n_keys = 0;
   std::vector<ve::HostObject> objs;          // sorted by base
@@ -131,6 +136,7 @@ struct ve_ctx {
   // dense counters (see DevObjects); disabled once 2^32 records could overflow a u32 counter
   void* dense_pool = nullptr;
   uint64_t dense_cap = 0;                    // counters allocated
+  uint64_t dense_want = 0;                   // counters the current object set may claim (0: none)
   bool dense_dirty = false;                  // pool may hold counts not yet flushed
   std::vector<uint32_t> dense_pc_init;       // [DENSE_PER_OBJ*n_obj]: DENSE_FREE or DENSE_OFF
   uint64_t records_analyzed = 0;
@@ -169,6 +175,10 @@ ve_status fail(ve_ctx* c, ve_status s, const std::string& msg);
 ve_status cuda_fail(ve_ctx* c, cudaError_t e, const char* where);
 ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s);
 ve_status launch_reset(ve_ctx* c, cudaStream_t s);
+void ctx_begin(ve_ctx* c, cudaStream_t s);      // order s after the ctx's earlier work
+void ctx_end(ve_ctx* c, cudaStream_t s);        // the ctx's work so far ends with s's queued work
+cudaError_t ctx_quiesce(ve_ctx* c);             // host wait for the ctx's queued work (not the device's)
+bool dense_reserve(ve_ctx* c);                  // the dense counter pool for the current object set
 ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
                         std::vector<ve_topk_entry>& top);
 ve_status bitmap_counts(ve_ctx* c, cudaStream_t s, std::vector<ve_obj_stats>& out);

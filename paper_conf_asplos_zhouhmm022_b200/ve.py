@@ -67,7 +67,8 @@ class VeError(RuntimeError):
 class _Config(ctypes.Structure):
     _fields_ = [("n_pcs", ctypes.c_uint32), ("max_objects", ctypes.c_uint32), ("topk", ctypes.c_uint32),
                 ("mant_bits", ctypes.c_uint32), ("t_redundant_pct", ctypes.c_uint32),
-                ("t_frequent_pct", ctypes.c_uint32), ("hist_capacity", ctypes.c_uint64)]
+                ("t_frequent_pct", ctypes.c_uint32), ("hist_capacity", ctypes.c_uint64),
+                ("min_windows_per_warp", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
 
 class _Object(ctypes.Structure):
@@ -341,13 +342,14 @@ class Context:
     """A ve_ctx bound to one CUDA device."""
 
     def __init__(self, n_pcs, max_objects=64, topk=8, mant_bits=7, t_redundant_pct=33, t_frequent_pct=33,
-                 hist_capacity=1 << 22, device=None):
+                 hist_capacity=1 << 22, device=None, min_windows_per_warp=0):
         L = lib()
         if device is None:
             import torch
             device = torch.cuda.current_device()
         self.device = device
-        cfg = _Config(n_pcs, max_objects, topk, mant_bits, t_redundant_pct, t_frequent_pct, hist_capacity)
+        cfg = _Config(n_pcs, max_objects, topk, mant_bits, t_redundant_pct, t_frequent_pct, hist_capacity,
+                      min_windows_per_warp, 0)
         h = ctypes.c_void_p()
         rc = L.ve_create(ctypes.byref(cfg), device, ctypes.byref(h))
         if rc != OK:

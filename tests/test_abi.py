@@ -65,3 +65,28 @@ def test_record_layout():
     from gen import vegen
     assert ve.RECORD_DTYPE.itemsize == 24 and vegen.REC_DTYPE == ve.RECORD_DTYPE
     assert ve.KEY_DTYPE.itemsize == 8 * (6 + 12 + 5 + 6 + 7 + 2) + 4 * 8
+
+
+def test_dump_spec_layout_matches_header_struct():
+    """tests/dump_spec.py packs ve_key_stats field by field in include/ve.h's order: the same values placed
+    in the binding's struct mirror give the same 336 bytes (a pin of the S13 dump layout, no GPU)."""
+    import numpy as np
+    from paper_conf_asplos_zhouhmm022_b200 import ve
+    from oracle import oracle as O
+    from tests import dump_spec as D
+    rng = np.random.default_rng(7)
+    ok = np.zeros(1, dtype=O.KEY_DTYPE)[0]
+    gk = np.zeros(1, dtype=ve.KEY_DTYPE)
+    for f in ve.KEY_DTYPE.names:
+        shape = ve.KEY_DTYPE[f].shape
+        v = rng.integers(0, 1 << 62, size=shape if shape else None, dtype=np.int64)
+        if f == "line_state":
+            v = O.LINE_LINE
+        if ve.KEY_DTYPE[f].base == np.dtype("<u4"):
+            v = int(v) & 0xFFFFFFFF
+        ok[f] = v
+        gk[0][f] = v
+    assert D.key_bytes(ok) == gk.tobytes() and len(gk.tobytes()) == D.KEY_BYTES
+    ok["line_state"] = O.LINE_FAIL       # endpoints of a FAILed line are written as 0
+    b = D.key_bytes(ok)
+    assert b[30 * 8:36 * 8] == bytes(48)
