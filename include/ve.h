@@ -16,7 +16,13 @@
  *     ve_last_error(ctx) describes the last failure (cudaGetErrorString for
  *     CUDA errors).  Asynchronous kernel faults surface at the next
  *     synchronising call (ve_snapshot_diff, ve_object_dedup, ve_report).
- *   - A ctx is bound to one CUDA device and is not thread-safe.
+ *   - A ctx is bound to one CUDA device and is not thread-safe; different
+ *     contexts may be driven from different host threads at once.
+ *   - Stream order, no device-wide synchronisation: a ctx's calls run in call
+ *     order whatever streams they are given (each waits for the ctx's previous
+ *     work through a per-ctx event); calls that return host results wait only
+ *     for that ctx's work (its event / its own internal stream), never for the
+ *     device, so other contexts and application streams keep running.
  */
 #ifndef VE_H
 #define VE_H

@@ -2574,10 +2574,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
     P.stage_rs = (uint32_t)(per < STAGE_RS_MAX ? per : STAGE_RS_MAX);
     const size_t need = (size_t)tw * P.stage_rs * sizeof(uint4) + tw * sizeof(uint32_t);
     if (c->hstage_bytes < need) {
-      if (c->hstage) cudaFree(c->hstage);
-      c->hstage = nullptr;
       c->hstage_bytes = 0;
-      e = cudaMalloc(&c->hstage, need);
+      e = ctx_realloc(c, &c->hstage, need);
       if (e != cudaSuccess) return cuda_fail(c, e, "k_analyze staging");
       c->hstage_bytes = need;
     }

@@ -31,10 +31,8 @@ static void stage(const char* name, cudaStream_t s) {
 // ---- scratch management ------------------------------------------------------
 static cudaError_t scratch_need(ve_ctx* c, size_t bytes) {
   if (c->scratch_bytes >= bytes) return cudaSuccess;
-  if (c->scratch) cudaFree(c->scratch);
-  c->scratch = nullptr;
   c->scratch_bytes = 0;
-  cudaError_t e = cudaMalloc(&c->scratch, bytes);
+  cudaError_t e = ctx_realloc(c, &c->scratch, bytes);
   if (e == cudaSuccess) c->scratch_bytes = bytes;
   return e;
 }

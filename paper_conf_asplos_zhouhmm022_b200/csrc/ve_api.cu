@@ -57,20 +57,33 @@ static void free_dev(ve_ctx* c) {
   if (c->cs) cudaStreamDestroy(c->cs);
 }
 
+// grow-only device buffers: freed and allocated stream-ordered on the ctx stream after the ctx's queued
+// work (cudaFree / cudaMalloc would synchronise the whole device and stall every other context), then
+// one wait on the ctx stream so the new block is valid for whatever stream the caller uses next
+cudaError_t ctx_realloc(ve_ctx* c, void** p, size_t bytes) {
+  ctx_begin(c, c->cs);
+  if (*p) cudaFreeAsync(*p, c->cs);
+  *p = nullptr;
+  cudaError_t e = cudaMallocAsync(p, bytes, c->cs);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->cs);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    *p = nullptr;
+  }
+  return e;
+}
+
 // make the dense counter pool hold the current object set's claims (dense_want counters), allocated
 // on first need; false when there is no memory for it (the calls then count through the hash path)
 bool dense_reserve(ve_ctx* c) {
   if (c->dense_want == 0) return false;
   if (c->dense_pool && c->dense_cap >= c->dense_want) return true;
-  if (ctx_quiesce(c) != cudaSuccess) return false;   // (the old pool may still be read)
-  if (c->dense_pool) cudaFree(c->dense_pool);
-  c->dense_pool = nullptr;
   c->dense_cap = 0;
   c->dense_dirty = false;
-  if (cudaMalloc(&c->dense_pool, c->dense_want * 4) != cudaSuccess ||
+  if (ctx_realloc(c, &c->dense_pool, c->dense_want * 4) != cudaSuccess ||
       cudaMemsetAsync(c->dense_pool, 0, c->dense_want * 4, c->cs) != cudaSuccess) {
     cudaGetLastError();
-    if (c->dense_pool) cudaFree(c->dense_pool);
+    if (c->dense_pool) cudaFreeAsync(c->dense_pool, c->cs);
     c->dense_pool = nullptr;
     c->dense_want = 0;                                 // no memory: this object set uses the hash path
     return false;
@@ -341,15 +354,13 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   // (a wait on this ctx's work only -- other contexts and the application keep running)
   cudaError_t qe = ctx_quiesce(c);
   if (qe != cudaSuccess) return cuda_fail(c, qe, "ve_set_objects (pending work)");
-  if (words > c->bm_words || !c->t.W) {
-    cudaFree(c->t.W);
-    cudaFree(c->t.L);
-    c->t.W = c->t.L = nullptr;
+  if (words > c->bm_cap || !c->t.W) {
     const uint64_t alloc = words ? words : 1;
-    if (cudaMalloc(&c->t.W, alloc * 4) != cudaSuccess || cudaMalloc(&c->t.L, alloc * 4) != cudaSuccess) {
-      cudaGetLastError();
+    c->bm_cap = 0;
+    if (ctx_realloc(c, (void**)&c->t.W, alloc * 4) != cudaSuccess ||
+        ctx_realloc(c, (void**)&c->t.L, alloc * 4) != cudaSuccess)
       return fail(c, VE_ERR_NOMEM, "ve_set_objects: bitmaps");
-    }
+    c->bm_cap = alloc;
   }
   c->bm_words = words;
   // dense per-element counters: up to DENSE_PER_OBJ arrays per object with a pre
@@ -378,12 +389,10 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   const size_t nn = n ? n : 1;
   const size_t nb = nn * (8 * 5 + 8 * DENSE_PER_OBJ + 4 * 2 + 4 * DENSE_PER_OBJ) + 64;
   if (nb > c->obj_block_bytes) {
-    cudaFree(c->obj_block);
-    c->obj_block = nullptr;
     c->obj_block_bytes = 0;
-    if (cudaMalloc(&c->obj_block, nb) != cudaSuccess) { cudaGetLastError(); return fail(c, VE_ERR_NOMEM, "objects"); }
+    if (ctx_realloc(c, &c->obj_block, nb) != cudaSuccess) return fail(c, VE_ERR_NOMEM, "objects");
     c->obj_block_bytes = nb;
-  }   // (else: the block is reused -- the device was made idle above)
+  }   // (else: the block is reused -- the ctx's work was waited for above)
   std::vector<uint8_t> host(nb, 0);
   uint64_t* hb = (uint64_t*)host.data();
   uint64_t* he = hb + n;

@@ -132,6 +132,7 @@ struct ve_ctx {
   void* obj_block = nullptr;                 // backing store of DevObjects arrays
   size_t obj_block_bytes = 0;
   uint64_t bm_words = 0;
+  uint64_t bm_cap = 0;                       // words allocated for W and L
   uint64_t hcap = 0;
   // dense counters (see DevObjects); disabled once 2^32 records could overflow a u32 counter
   void* dense_pool = nullptr;
@@ -179,6 +180,7 @@ void ctx_begin(ve_ctx* c, cudaStream_t s);      // order s after the ctx's earli
 void ctx_end(ve_ctx* c, cudaStream_t s);        // the ctx's work so far ends with s's queued work
 cudaError_t ctx_quiesce(ve_ctx* c);             // host wait for the ctx's queued work (not the device's)
 bool dense_reserve(ve_ctx* c);                  // the dense counter pool for the current object set
+cudaError_t ctx_realloc(ve_ctx* c, void** p, size_t bytes);   // grow a ctx buffer without a device sync
 ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndistinct,
                         std::vector<ve_topk_entry>& top);
 ve_status bitmap_counts(ve_ctx* c, cudaStream_t s, std::vector<ve_obj_stats>& out);
