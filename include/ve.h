@@ -138,6 +138,32 @@ ve_status   ve_reset(ve_ctx* ctx);              /* zero all statistics, clear po
  * on s.  VE_ERR_STATE if the ctx is poisoned (histogram overflow). */
 ve_status ve_analyze_records(ve_ctx* ctx, const ve_record* d_records, uint64_t n, cudaStream_t s);
 
+/* Several independent traces in one launch (units): cfg5's thousands of small
+ * kernels (the paper's whole-application runs, P:L105,
+ * Table 5) pay one launch and one report instead of one each.  ve_set_units
+ * takes the objects of n_units units, unit u being the next unit_nobj[u]
+ * entries of objs (ids 0..n-1 over the whole set, so each unit's objects have
+ * their own keys n_pcs + id); objects may overlap across units, not within one
+ * (the units' address spaces are separate).  Errors as ve_set_objects, plus
+ * VE_ERR_INVALID when the counts do not sum to n or n_units is 0 or > 65535. */
+ve_status ve_set_units(ve_ctx* ctx, const ve_object* objs, uint32_t n, const uint32_t* unit_nobj, uint32_t n_units);
+
+/* Unit u's device records (16-byte aligned); its record pc p < n_pcs is key
+ * pc_base + p of the ctx (pc_base + n_pcs <= cfg.n_pcs), p >= n_pcs is invalid;
+ * its addresses map to its own objects only (an address outside them is
+ * unmapped).  The result equals analysing each unit alone with its PCs shifted
+ * to pc_base (C12); the SHARED key and the globals add over the units. */
+typedef struct ve_unit {
+  const ve_record* d_records;
+  uint64_t n;
+  uint32_t pc_base, n_pcs;
+} ve_unit;
+/* All units in one launch (K1 v2), accumulating into the ctx like
+ * ve_analyze_records.  n_units must equal the last ve_set_units' (or 1 after
+ * ve_set_objects).  VE_ERR_INVALID on misaligned records, a PC range outside
+ * the ctx or a batch of >= 2^31 records per SM (split it).  Asynchronous on s. */
+ve_status ve_analyze_units(ve_ctx* ctx, const ve_unit* units, uint32_t n_units, cudaStream_t s);
+
 /* End-to-end variant: records in HOST memory (pinned or pageable), streamed to
  * the device in chunks through a double-buffered staging area and analyzed
  * (the paper's collector->analyzer buffer path).  Returns after the

@@ -54,6 +54,13 @@ struct AnalyzeParams {
   uint64_t nring;           // full windows (streamed through the per-warp rings)
   uint32_t chunk;           // windows per static chunk (VE_CLAIM 2): CHUNK, or one stage for short traces
   uint32_t claim;           // 1: chunks claimed from the global counter *work (guided), 0: static interleave
+  // units mode (ve_analyze_units, K1 v2 only): independent traces in one launch.  Unit u's records
+  // are units[u].recs (16-byte aligned); its PCs are keys pcb .. pcb + npc - 1 (a record's pc is
+  // local: pc >= npc is invalid) and its objects the sorted table entries [olo, ohi).  Chunk c of
+  // the launch is chunk c - ucb[u] of the unit u with ucb[u] <= c < ucb[u + 1].
+  const struct UnitDesc* units;
+  const uint32_t* ucb;      // [n_units + 1] chunk prefix
+  uint32_t n_units;
   unsigned long long* work; // chunk claim counter (zeroed before the launch)
   // S8 insert staging: a private region of stage_rs 16-byte entries per warp for the
   // (tag, bits, count) groups the shared table cannot take; k_hist_drain inserts them
@@ -66,6 +73,13 @@ struct AnalyzeParams {
   uint32_t o_ssum, o_smin, o_smax, o_sline, o_shs, o_shc, o_sob, o_soe, o_sctr, o_ring, o_bars;
   DevObjects o;
   DevTables t;
+};
+
+struct UnitDesc {
+  const ve_record* recs;
+  uint64_t n;
+  uint32_t pcb, npc;        // key base and count of the unit's PCs
+  uint32_t olo, ohi;        // the unit's objects in the sorted table
 };
 
 struct Smem {
@@ -344,6 +358,7 @@ __device__ __noinline__ void merge_lines(const AnalyzeParams& P, WarpCache& C, b
 }
 
 __shared__ uint32_t s_stage_n[K1_WARPS];   // entries claimed in the warp's staging region
+__shared__ uint32_t s_urange[K1_WARPS][2];  // units mode: the object range [lo, hi) of the warp's current unit
 
 // Stage a (tag, bits, c) group for k_hist_drain; the HBM table directly once the
 // warp's region is full.  A plain store: the warp does not wait on it.
@@ -430,11 +445,16 @@ __device__ __noinline__ int find_object(const AnalyzeParams& P, uint64_t addr) {
   const Smem S = smem_of(P);
   const uint64_t* base = P.objc ? S.sob : P.o.base;
   int lo = 0, hi = (int)P.o.n;  // first object with base > addr
+  if (P.units) {                // units mode: only the current unit's objects
+    lo = (int)s_urange[threadIdx.x >> 5][0];
+    hi = (int)s_urange[threadIdx.x >> 5][1];
+  }
+  const int lo0 = lo;
   while (lo < hi) {
     int mid = (lo + hi) >> 1;
     if (base[mid] <= addr) lo = mid + 1; else hi = mid;
   }
-  if (lo == 0) return -1;
+  if (lo == lo0) return -1;
   const uint64_t e = P.objc ? S.soe[lo - 1] : P.o.end[lo - 1];
   return addr < e ? lo - 1 : -1;
 }
@@ -760,6 +780,9 @@ struct Ring {
   uint32_t pend;          // stage + 1 to refill at the next read, 0 = none
   uint64_t nextc;         // VE_CLAIM == 2: the warp's next static chunk (gw, gw + warps, ...)
   uint32_t cstride;       // warps of the grid (the static interleave's stride)
+  uint32_t cu;            // units mode: unit of the chunk being issued
+  uint32_t su;            // units mode: unit of the windows in stage d: bits [16d, 16d + 16)
+  uint32_t snw;           // windows issued into stage d: bits [4d, 4d + 4) (< STAGE_WIN only for a chunk's end)
 };
 
 // claim the next chunk of full windows (all lanes; lane 0 does the atomic).  Guided:
@@ -768,6 +791,25 @@ struct Ring {
 constexpr uint32_t CHUNK_TAIL = STAGE_WIN;
 __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
   uint64_t w0, len;
+  if (P.units) {
+    // a dynamic claim; its unit by binary search over the chunk prefix (warp-uniform)
+    unsigned long long c = 0;
+    if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
+    c = __shfl_sync(0xFFFFFFFFu, c, 0);
+    if (c >= P.ucb[P.n_units]) { R.iss = 0; return; }
+    uint32_t lo = 0, hi = P.n_units;          // last u with ucb[u] <= c
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (P.ucb[mid] <= c) lo = mid; else hi = mid;
+    }
+    const UnitDesc& U = P.units[lo];
+    const uint64_t fw = U.n / 32;
+    w0 = (c - P.ucb[lo]) * (uint64_t)P.chunk;
+    R.src = U.recs + w0 * 32;
+    R.iss = (uint32_t)(fw - w0 < P.chunk ? fw - w0 : P.chunk);
+    R.cu = lo;
+    return;
+  }
   if (!P.claim) {
     // static interleave: chunk c goes to warp c mod (all warps); no atomics, and every
     // warp sees the same mix of the trace
@@ -797,6 +839,8 @@ __device__ __forceinline__ void ring_issue_stage(const AnalyzeParams& P, Ring& R
   const uint32_t nw = R.iss < (uint32_t)STAGE_WIN ? R.iss : (uint32_t)STAGE_WIN;
   if (nw == 0u) return;
   ring_issue_pred((threadIdx.x & 31) == 0, R.dst0 + d * STAGE_BYTES, R.src, nw * WIN_BYTES, R.bar0 + d * 8u);
+  R.su = (R.su & ~(0xFFFFu << (16u * d))) | (R.cu << (16u * d));
+  R.snw = (R.snw & ~(0xFu << (4u * d))) | (nw << (4u * d));
   R.src += nw * 32;
   R.iss -= nw;
   R.left += nw;
@@ -821,10 +865,11 @@ __device__ __forceinline__ void ring_next(const AnalyzeParams& P, Ring& R, uint6
                : "memory");
   --R.left;
   R.o += WIN_BYTES;
-  if (++R.sw == (uint32_t)STAGE_WIN) {   // stage consumed: refill it at the next read
+  if (++R.sw == ((R.snw >> (4u * d)) & 0xFu)) {   // stage consumed (whole, or a chunk's short last stage)
     R.sw = 0;
     R.pend = R.iss ? d + 1u : 0u;
-    if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.o = R.o0; R.ph ^= 1u; }
+    if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.ph ^= 1u; }
+    R.o = R.o0 + R.d * STAGE_BYTES;
   }
 }
 
@@ -1639,6 +1684,7 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
   R.bar0 = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
   R.d = R.sw = R.ph = R.pend = 0;
   R.left = 0;
+  R.cu = R.su = R.snw = 0;
   if (lane == 0 && P.nring) {
     for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar0 + d * 8u, 1);
     fence_mbar_init();
@@ -2139,6 +2185,7 @@ constexpr int K2_THREADS = VE_K2_THREADS;
 constexpr int K2_WARPS = K2_THREADS / 32;
 static_assert(K2_WARPS <= K1_WARPS, "v2 uses the v1 shared-memory layout");
 
+template <bool UNITS>
 __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constant__ AnalyzeParams P) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const unsigned FULL = 0xFFFFFFFFu;
@@ -2190,6 +2237,7 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   R.bar0 = smem_u32(ve_smem + P.o_bars + (uint32_t)warp * RING * 8u);
   R.d = R.sw = R.ph = R.pend = 0;
   R.left = 0;
+  R.cu = R.su = R.snw = 0;
   if (lane == 0 && P.nring) {
     for (int d = 0; d < NSTAGE; ++d) mbar_init(R.bar0 + d * 8u, 1);
     fence_mbar_init();
@@ -2210,6 +2258,9 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   bool lpt = false;          // the post array of the current slot was claimed (or tried)
   uint32_t llf = 3;
   uint32_t n_inv = 0, n_unm = 0;
+  // units mode: the current unit's PC base / count and object range (registers; the range also in
+  // s_urange for find_object)
+  uint32_t cu = ~0u, upcb = 0, unpc = ~0u, ulo = 0, uhi = P.o.n;
 
   // make sorted object oi (-1: none) the current object
   auto obj_set = [&](int oi) {
@@ -2244,7 +2295,8 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
     if (a0 - cb <= clim && coi >= 0) return;
     int oi;
     if (ob32) {
-      const unsigned m = __ballot_sync(FULL, (uint32_t)lane < P.o.n && s_ob[lane] <= a0 && a0 < s_oe[lane]);
+      const unsigned m = __ballot_sync(FULL, (UNITS ? (uint32_t)lane >= ulo && (uint32_t)lane < uhi
+                                                    : (uint32_t)lane < P.o.n) && s_ob[lane] <= a0 && a0 < s_oe[lane]);
       oi = m ? __ffs(m) - 1 : -1;
     } else {
       oi = find_object(P, a0);
@@ -2264,9 +2316,23 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
 #if VE_DIAG == 2
   uint64_t dsink = 0;
 #endif
+  auto unit_enter = [&](uint32_t u) {
+    cu = u;
+    const UnitDesc& U = P.units[u];
+    upcb = U.pcb; unpc = U.npc; ulo = U.olo; uhi = U.ohi;
+    if (lane == 0) { s_urange[warp][0] = ulo; s_urange[warp][1] = uhi; }
+    __syncwarp();
+    coi = -1; cb = 1; clim = 0; clg = 0xFFu; ls = -1;   // the object registers belong to the last unit
+  };
   while (R.left) {
     uint64_t addr, val, pm;
+    const uint32_t wd = R.d;
     ring_next(P, R, addr, val, pm);
+    if constexpr (UNITS) {                     // a local pc -> the unit's key; out of range -> invalid
+      const uint32_t u = (R.su >> (16u * wd)) & 0xFFFFu;
+      if (u != cu) unit_enter(u);
+      pm = (uint32_t)pm < unpc ? pm + upcb : (pm | 0xFFFFFFFFull);
+    }
 #if VE_DIAG == 2   // diagnostic: the record stream alone (results wrong)
     dsink += addr ^ val ^ pm;
     continue;
@@ -2398,6 +2464,26 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   const uint64_t tw = (uint64_t)gridDim.x * K2_WARPS, gw = (uint64_t)blockIdx.x * K2_WARPS + warp;
   uint64_t wbeg = P.nring, wend = gw == 0 ? nwin : P.nring;
   if (!P.nring) { wbeg = gw * nwin / tw; wend = (gw + 1) * nwin / tw; }
+  if constexpr (UNITS) {                       // units mode: every unit's partial last window
+    wbeg = wend = 0;
+    for (uint64_t u = gw; u < P.n_units; u += tw) {
+      const uint64_t un = P.units[u].n;
+      const uint32_t rem = (uint32_t)(un & 31u);
+      if (!rem) continue;
+      unit_enter((uint32_t)u);
+      uint64_t addr = 0, val = 0, pm = 0;
+      if ((uint32_t)lane < rem) {
+        const unsigned long long* q = reinterpret_cast<const unsigned long long*>(&P.units[u].recs[(un & ~31ull) + lane]);
+        addr = __ldcs(q);
+        val = __ldcs(q + 1);
+        pm = __ldcs(q + 2);
+        pm = (uint32_t)pm < unpc ? pm + upcb : (pm | 0xFFFFFFFFull);
+      }
+      const uint32_t cnt = slow_window(P, wc, addr, val, pm, (uint32_t)lane < rem);
+      n_inv += cnt & 0xFFFFu;
+      n_unm += cnt >> 16;
+    }
+  }
   for (uint64_t w = wbeg; w < wend; ++w) {
     const Rec cur = load_rec(P, w, wend, lane);
     const uint32_t cnt = slow_window(P, wc, cur.addr, cur.val, cur.pm, w * 32 + lane < P.n);
@@ -2496,11 +2582,21 @@ __global__ void __launch_bounds__(LF_THREADS) k_line_fold(const LineState* lcta,
   }
 }
 
-ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
-  ctx_begin(c, s);   // after the ctx's earlier work (the last reset, a report), on any stream
+struct UnitLaunch {           // units mode of one launch (ve_analyze_units)
+  const UnitDesc* d_units;
+  const uint32_t* d_ucb;
+  uint32_t n_units;
+  uint64_t nring;             // full windows of all units
+};
+
+static ve_status launch_analyze_impl(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s,
+                                     const UnitLaunch* ul) {
   AnalyzeParams P;
   P.recs = d;
   P.n = n;
+  P.units = ul ? ul->d_units : nullptr;
+  P.ucb = ul ? ul->d_ucb : nullptr;
+  P.n_units = ul ? ul->n_units : 0u;
   P.n_pcs = c->cfg.n_pcs;
   P.n_obj = c->n_obj;
   P.mant_bits = c->cfg.mant_bits;
@@ -2511,8 +2607,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   P.dense_ok = (c->records_analyzed + n < (1ull << 32) && (n >= c->pre_elems || getenv("VE_DENSE_ALWAYS")) &&
                 dense_reserve(c)) ? 1u : 0u;
   if (P.dense_ok) c->dense_dirty = true;
-  P.ring = ((uintptr_t)d % 16 == 0) ? 1u : 0u;
-  P.nring = P.ring ? n / 32 : 0;
+  P.ring = (ul || (uintptr_t)d % 16 == 0) ? 1u : 0u;
+  P.nring = ul ? ul->nring : P.ring ? n / 32 : 0;
   P.work = c->t.glob + G_WORK;
   c->records_analyzed += n;
   // shared stat rows: up to 256 keys, PCs first then object keys (incl. SHARED)
@@ -2536,8 +2632,8 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   // K1 v2 (register key slots, post-value counting) for traces of many PCs, whose windows alternate
   // keys; v1 (single-key runs, stage-batched dense gathers) for few PCs.  VE_K1=1 / 2 forces one.
   const char* kv = getenv("VE_K1");
-  const bool v2 = (kv && *kv) ? *kv == '2' : c->cfg.n_pcs >= VE_MULTI_MIN_PCS;
-  auto kfn = v2 ? k_analyze2 : multi ? k_analyze<true> : k_analyze<false>;
+  const bool v2 = ul || ((kv && *kv) ? *kv == '2' : c->cfg.n_pcs >= VE_MULTI_MIN_PCS);   // (units: v2 only)
+  auto kfn = ul ? k_analyze2<true> : v2 ? k_analyze2<false> : multi ? k_analyze<true> : k_analyze<false>;
   cudaFuncGetAttributes(&fa, kfn);
   const size_t budget = (size_t)dev_smem - fa.sharedSizeBytes - 1024;   // dynamic smem left after the TMA ring
   // 2048 slots measured best on cfg2 / cfg3 / cfg4 (the HBM table behind it stays L2-resident)
@@ -2562,10 +2658,10 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   if (blocks == 0) blocks = 1;
   // a trace too short to give every warp a few CHUNK-window chunks (cfg5's kernels: a warp's
   // serial share of a 16-window chunk set a ~0.3 ms floor) is split into one-stage chunks
-  P.chunk = P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? CHUNK : (uint32_t)STAGE_WIN;
+  P.chunk = (ul || P.nring >= 4ull * blocks * K1_WARPS * CHUNK) ? CHUNK : (uint32_t)STAGE_WIN;
   // v2 claims its chunks dynamically (VE_CLAIM_MODE=0/1 forces the static / dynamic split)
   const char* cm = getenv("VE_CLAIM_MODE");
-  P.claim = (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
+  P.claim = ul ? 1u : (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
   // staging regions: a warp stages at most one group per record of its static range
   {
     const uint64_t tw = blocks * K1_WARPS;
@@ -2599,8 +2695,61 @@ ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t
   k_line_fold<<<nsk, LF_THREADS, 0, s>>>(c->t.lcta, (uint32_t)blocks, nsk, sp, c->cfg.n_pcs, c->t.line);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "k_line_fold launch");
-  ctx_end(c, s);
   return VE_OK;
 }
 
+ve_status launch_analyze(ve_ctx* c, const ve_record* d, uint64_t n, cudaStream_t s) {
+  ctx_begin(c, s);   // after the ctx's earlier work (the last reset, a report), on any stream
+  const ve_status st = launch_analyze_impl(c, d, n, s, nullptr);
+  if (st == VE_OK) ctx_end(c, s);
+  return st;
+}
+
 }  // namespace ve
+
+using namespace ve;
+
+// ve_analyze_units (include/ve.h): independent traces of the units set by ve_set_units in one launch
+extern "C" ve_status ve_analyze_units(ve_ctx* c, const ve_unit* units, uint32_t n_units, cudaStream_t s) {
+  if (!c || (n_units && !units)) return VE_ERR_INVALID;
+  if (c->poisoned || c->hist_merged) return fail(c, VE_ERR_STATE, "ve_analyze_units: ctx poisoned or merged; ve_reset first");
+  if (n_units != c->n_units || c->unit_obj.size() != (size_t)n_units + 1)
+    return fail(c, VE_ERR_INVALID, "ve_analyze_units: n_units differs from the last ve_set_units");
+  if (n_units == 0) return VE_OK;
+  if (n_units > 65535) return fail(c, VE_ERR_INVALID, "ve_analyze_units: more than 65535 units");
+  std::vector<UnitDesc> ud(n_units);
+  std::vector<uint32_t> ucb(n_units + 1, 0);
+  uint64_t ntot = 0, nring = 0;
+  for (uint32_t u = 0; u < n_units; ++u) {
+    const ve_unit& U = units[u];
+    if (U.n && (!U.d_records || ((uintptr_t)U.d_records & 15)))
+      return fail(c, VE_ERR_INVALID, "ve_analyze_units: unit records null or not 16-byte aligned");
+    if ((uint64_t)U.pc_base + U.n_pcs > c->cfg.n_pcs)
+      return fail(c, VE_ERR_INVALID, "ve_analyze_units: pc_base + n_pcs above the ctx's n_pcs");
+    ud[u] = UnitDesc{U.d_records, U.n, U.pc_base, U.n_pcs, c->unit_obj[u], c->unit_obj[u + 1]};
+    const uint64_t fw = U.n / 32, ch = (fw + CHUNK - 1) / CHUNK;
+    if ((uint64_t)ucb[u] + ch > 0xFFFFFFFFull) return fail(c, VE_ERR_INVALID, "ve_analyze_units: batch too large");
+    ucb[u + 1] = ucb[u] + (uint32_t)ch;
+    ntot += U.n;
+    nring += fw;
+  }
+  if (ntot == 0) return VE_OK;
+  // per-CTA shared counters are 32-bit (see ve_analyze_records)
+  if (ntot >= ((uint64_t)(c->num_sms > 0 ? c->num_sms : 1) << 31))
+    return fail(c, VE_ERR_INVALID, "ve_analyze_units: batch above the per-launch record limit; split it");
+  cudaSetDevice(c->device);
+  ctx_begin(c, s);
+  const size_t bytes = ud.size() * sizeof(UnitDesc) + ucb.size() * 4;
+  void* d = nullptr;
+  cudaError_t e = cudaMallocAsync(&d, bytes, s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "ve_analyze_units alloc");
+  std::vector<uint8_t> h(bytes);
+  memcpy(h.data(), ud.data(), ud.size() * sizeof(UnitDesc));
+  memcpy(h.data() + ud.size() * sizeof(UnitDesc), ucb.data(), ucb.size() * 4);
+  cudaMemcpyAsync(d, h.data(), bytes, cudaMemcpyHostToDevice, s);   // (pageable: staged before return)
+  UnitLaunch ul{(const UnitDesc*)d, (const uint32_t*)((uint8_t*)d + ud.size() * sizeof(UnitDesc)), n_units, nring};
+  const ve_status st = launch_analyze_impl(c, nullptr, ntot, s, &ul);
+  cudaFreeAsync(d, s);
+  if (st == VE_OK) ctx_end(c, s);
+  return st;
+}

@@ -470,6 +470,36 @@ __device__ __forceinline__ void block_chunk(uint64_t n, uint64_t& lo, uint64_t& 
   if (lo > hi) lo = hi;
 }
 
+__global__ void __launch_bounds__(256) k_occ_count(const uint32_t* bm, uint64_t nw, unsigned long long* total) {
+  unsigned long long n = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x)
+    n += __popc(bm[i]);
+  for (int o = 16; o; o >>= 1) n += __shfl_xor_sync(0xFFFFFFFFu, n, o);
+  if ((threadIdx.x & 31) == 0 && n) atomicAdd(total, n);
+}
+
+// the occupied slots of the value table, listed from its occupancy bitmap (order-free: every consumer
+// aggregates); *total = their number (one warp-aggregated atomic per 32 bitmap words)
+__global__ void __launch_bounds__(256) k_occ_list(const uint32_t* bm, uint64_t nw, uint32_t* flat,
+                                                  unsigned long long* total) {
+  const int lane = threadIdx.x & 31;
+  for (uint64_t b = blockIdx.x * (uint64_t)blockDim.x; b < nw; b += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    uint32_t w = i < nw ? bm[i] : 0u;
+    const uint32_t k = __popc(w);
+    uint32_t x = k;                                    // inclusive warp scan of the counts
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+      if (lane >= o) x += y;
+    }
+    const uint32_t wsum = __shfl_sync(0xFFFFFFFFu, x, 31);
+    unsigned long long base = 0;
+    if (lane == 31 && wsum) base = atomicAdd(total, (unsigned long long)wsum);
+    base = __shfl_sync(0xFFFFFFFFu, base, 31) + (x - k);
+    for (; w; w &= w - 1) flat[base++] = (uint32_t)((i << 5) + (uint32_t)(__ffs(w) - 1));
+  }
+}
+
 // the distinct tags of the occupied slots (the table's occupancy list: O(entries), not O(capacity))
 // and their entry counts
 __global__ void k_tagscan(const HSlot* hs, const uint32_t* occ, const unsigned long long* n_occ, uint32_t* tags,
@@ -617,8 +647,41 @@ ve_status finalize_hist(ve_ctx* c, cudaStream_t s, std::vector<uint64_t>& ndisti
   unsigned long long* d_tcnt = nullptr;
   unsigned long long* d_small = nullptr;     // [0] overflow, [1] occupied slots
   unsigned long long* d_tl = nullptr;        // compacted tag list
-  const uint32_t* d_occ = c->t.occ;          // occupied slot indices (maintained by every insert)
-  const unsigned long long* d_nocc = c->t.glob + G_NOCC;
+  // occupied slot indices, listed from the occupancy bitmap (the count read back to size the list)
+  const uint64_t nbw = c->hcap >> 5;
+  {
+    const size_t need = 16;
+    if (c->occ_flat_bytes < need || !c->occ_flat) {
+      c->occ_flat_bytes = 0;
+      e = ctx_realloc(c, &c->occ_flat, 1 << 16);
+      if (e != cudaSuccess) return cuda_fail(c, e, "finalize occupancy alloc");
+      c->occ_flat_bytes = 1 << 16;
+    }
+  }
+  // pass 1: count (the list is written in pass 2 once it fits)
+  unsigned long long* d_cnt = (unsigned long long*)c->occ_flat;
+  cudaMemsetAsync(d_cnt, 0, 8, s);
+  count_launch();
+  k_occ_count<<<c->num_sms * 4, 256, 0, s>>>(c->t.occ_bm, nbw, d_cnt);
+  unsigned long long tot = 0;
+  cudaMemcpyAsync(&tot, d_cnt, 8, cudaMemcpyDeviceToHost, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "finalize occupancy");
+  c->last_nocc = tot;
+  {
+    const size_t need = (size_t)tot * 4 + 16;
+    if (c->occ_flat_bytes < need) {      // grow-only (ctx_realloc: no device sync)
+      c->occ_flat_bytes = 0;
+      e = ctx_realloc(c, &c->occ_flat, need + need / 4);
+      if (e != cudaSuccess) return cuda_fail(c, e, "finalize occupancy alloc");
+      c->occ_flat_bytes = need + need / 4;
+    }
+  }
+  unsigned long long* d_nocc = (unsigned long long*)c->occ_flat;
+  uint32_t* d_occ = (uint32_t*)((uint8_t*)c->occ_flat + 16);
+  cudaMemsetAsync(d_nocc, 0, 8, s);
+  count_launch();
+  k_occ_list<<<c->num_sms * 4, 256, 0, s>>>(c->t.occ_bm, nbw, d_occ, d_nocc);
   if (c->hcap > 0xFFFFFFFFull) return fail(c, VE_ERR_INVALID, "finalize: hist_capacity above 2^32");
   e = cudaMallocAsync((void**)&d_tags, TAG_CAP * 4, s);
   if (e == cudaSuccess) e = cudaMallocAsync((void**)&d_tcnt, TAG_CAP * 8, s);

@@ -40,9 +40,10 @@ static void free_dev(ve_ctx* c) {
   cudaFree(c->t.L);
   cudaFree(c->t.hslot);
   cudaFree(c->t.hcount);
-  cudaFree(c->t.occ);
+  cudaFree(c->t.occ_bm);
   cudaFree(c->obj_block);
   cudaFree(c->scratch);
+  cudaFree(c->occ_flat);
   if (c->pin) cudaFreeHost(c->pin);
   if (c->rpin) cudaFreeHost(c->rpin);
   cudaFree(c->dense_pool);
@@ -105,16 +106,20 @@ cudaError_t ctx_quiesce(ve_ctx* c) {
   return c->ord_ev ? cudaEventSynchronize(c->ord_ev) : cudaSuccess;
 }
 
-// empty the occupied slots recorded in t.occ (the table's only non-empty slots), then their count
+// empty the slots marked in the occupancy bitmap (the table's only non-empty slots), and the bitmap
 __global__ void k_reset_occ(DevTables t) {
-  const unsigned long long n = t.glob[G_NOCC];
-  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
-       i += (unsigned long long)gridDim.x * blockDim.x) {
-    const uint32_t h = t.occ[i];
-    t.hslot[h].bits = ~0ull;
-    t.hslot[h].tag = EMPTY_TAG;
-    t.hslot[h].pad = EMPTY_TAG;
-    t.hcount[h] = 0;
+  const uint64_t nw = (t.hmask + 1) >> 5;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t w = t.occ_bm[i];
+    if (!w) continue;
+    t.occ_bm[i] = 0;
+    for (; w; w &= w - 1) {
+      const uint64_t h = (i << 5) + (uint32_t)(__ffs(w) - 1);
+      t.hslot[h].bits = ~0ull;
+      t.hslot[h].tag = EMPTY_TAG;
+      t.hslot[h].pad = EMPTY_TAG;
+      t.hcount[h] = 0;
+    }
   }
 }
 
@@ -135,11 +140,13 @@ ve_status launch_reset(ve_ctx* c, cudaStream_t s) {
     c->dense_dirty = false;
   }
   // the value table: a fresh table is filled whole; afterwards only the slots claimed since the last
-  // reset (recorded in t.occ) are emptied -- O(entries), not O(hist_capacity), per epoch
+  // reset (marked in t.occ_bm) are emptied -- O(entries + hist_capacity / 32), per epoch
   const bool full = !c->table_clean;
   if (!full) {
     count_launch();
     k_reset_occ<<<c->num_sms * 4, 256, 0, s>>>(c->t);
+  } else {
+    cudaMemsetAsync(c->t.occ_bm, 0, c->hcap / 8, s);
   }
   cudaMemsetAsync(c->t.glob, 0, 8 * 8, s);
   if (c->bm_words) {
@@ -287,7 +294,7 @@ ve_status ve_create(const ve_config* cfg, int cuda_device, ve_ctx** out) {
             cudaMalloc(&c->t.glob, 8 * 8) == cudaSuccess &&
             cudaMalloc(&c->t.hslot, hcap * sizeof(HSlot)) == cudaSuccess &&
             cudaMalloc(&c->t.hcount, hcap * 8) == cudaSuccess &&
-            cudaMalloc(&c->t.occ, hcap * 4) == cudaSuccess;
+            cudaMalloc(&c->t.occ_bm, hcap / 8) == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
     free_dev(c);
@@ -324,11 +331,28 @@ ve_status ve_destroy(ve_ctx* c) {
 
 const char* ve_last_error(const ve_ctx* c) { return c ? c->err.c_str() : "null context"; }
 
-ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
+// the object table of n objects in units (unit u = the next unit_nobj[u] entries of objs; one unit
+// holding all of them for ve_set_objects): sorted by (unit, base), overlaps rejected within a unit
+static ve_status set_objects_units(ve_ctx* c, const ve_object* objs, uint32_t n, const uint32_t* unit_nobj,
+                                   uint32_t n_units) {
   if (!ctx_ok(c)) return VE_ERR_INVALID;
   if (n > c->cfg.max_objects) return fail(c, VE_ERR_INVALID, "ve_set_objects: n > max_objects");
   if (n && !objs) return fail(c, VE_ERR_INVALID, "ve_set_objects: null objects");
+  std::vector<uint32_t> unit_of(n, 0), ustart(n_units + 1, 0);
+  if (unit_nobj) {
+    uint64_t tot = 0;
+    for (uint32_t u = 0; u < n_units; ++u) {
+      ustart[u] = (uint32_t)std::min<uint64_t>(tot, n);
+      for (uint64_t i = tot; i < tot + unit_nobj[u] && i < n; ++i) unit_of[i] = u;
+      tot += unit_nobj[u];
+    }
+    if (tot != n) return fail(c, VE_ERR_INVALID, "ve_set_units: unit object counts do not sum to n");
+    ustart[n_units] = n;
+  } else {
+    ustart[n_units] = n;       // one unit of every object
+  }
   std::vector<HostObject> v(n);
+  std::vector<uint32_t> vu(n);
   std::vector<char> seen(n, 0);
   for (uint32_t i = 0; i < n; ++i) {
     const ve_object& o = objs[i];
@@ -340,9 +364,19 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
     v[i] = HostObject{o.base, o.size, (uint64_t)(uintptr_t)o.pre, (uint64_t)(uintptr_t)o.post, o.id, ew,
                       (o.size + ew - 1) / ew, 0, 0};
   }
-  std::sort(v.begin(), v.end(), [](const HostObject& a, const HostObject& b) { return a.base < b.base; });
+  {
+    std::vector<uint32_t> ord(n);
+    for (uint32_t i = 0; i < n; ++i) ord[i] = i;
+    std::sort(ord.begin(), ord.end(), [&](uint32_t a, uint32_t b) {
+      return unit_of[a] != unit_of[b] ? unit_of[a] < unit_of[b] : v[a].base < v[b].base;
+    });
+    std::vector<HostObject> w(n);
+    for (uint32_t i = 0; i < n; ++i) { w[i] = v[ord[i]]; vu[i] = unit_of[ord[i]]; }
+    v.swap(w);
+  }
   for (uint32_t i = 1; i < n; ++i)
-    if (v[i - 1].base + v[i - 1].size > v[i].base) return fail(c, VE_ERR_INVALID, "ve_set_objects: overlap");
+    if (vu[i - 1] == vu[i] && v[i - 1].base + v[i - 1].size > v[i].base)
+      return fail(c, VE_ERR_INVALID, "ve_set_objects: overlap");
   uint64_t words = 0;
   for (auto& o : v) {
     o.bmoff = words;
@@ -428,9 +462,21 @@ ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
   c->objs = v;
   c->n_obj = n;
   c->n_keys = c->cfg.n_pcs + n + 1;
+  c->n_units = n_units;
+  c->unit_obj = ustart;
   // the reset runs on the ctx stream; the analysis / diff calls wait for it on their stream
   // (no host synchronisation per object set)
   return launch_reset(c, c->cs);
+}
+
+ve_status ve_set_objects(ve_ctx* c, const ve_object* objs, uint32_t n) {
+  return set_objects_units(c, objs, n, nullptr, 1u);
+}
+
+ve_status ve_set_units(ve_ctx* c, const ve_object* objs, uint32_t n, const uint32_t* unit_nobj, uint32_t n_units) {
+  if (!ctx_ok(c)) return VE_ERR_INVALID;
+  if (n_units == 0 || n_units > 65535 || !unit_nobj) return fail(c, VE_ERR_INVALID, "ve_set_units: 1..65535 units");
+  return set_objects_units(c, objs, n, unit_nobj, n_units);
 }
 
 ve_status ve_reset(ve_ctx* c) {
@@ -653,10 +699,7 @@ ve_status ve_report(ve_ctx* c, ve_rep** out) {
   r->glob.n_unmapped = glob[G_UNMAPPED];
   r->glob.hist_entries = 0;
   if (!c->hist_merged) {   // occupied value-table slots after the dense flush (implementation statistic)
-    unsigned long long nocc = 0;
-    if (cudaMemcpyAsync(&nocc, c->t.glob + G_NOCC, 8, cudaMemcpyDeviceToHost, cs) == cudaSuccess &&
-        cudaStreamSynchronize(cs) == cudaSuccess)
-      r->glob.hist_entries = nocc;
+    r->glob.hist_entries = c->last_nocc;   // (counted by finalize_hist's occupancy compaction)
   }
   ctx_end(c, cs);
   *out = r;

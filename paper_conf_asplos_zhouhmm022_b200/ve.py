@@ -71,6 +71,11 @@ class _Config(ctypes.Structure):
                 ("min_windows_per_warp", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
 
+class _Unit(ctypes.Structure):
+    _fields_ = [("d_records", ctypes.c_void_p), ("n", ctypes.c_uint64), ("pc_base", ctypes.c_uint32),
+                ("n_pcs", ctypes.c_uint32)]
+
+
 class _Object(ctypes.Structure):
     _fields_ = [("base", ctypes.c_uint64), ("size", ctypes.c_uint64), ("pre", ctypes.c_void_p),
                 ("post", ctypes.c_void_p), ("id", ctypes.c_uint32), ("elem_width", ctypes.c_uint32)]
@@ -131,6 +136,8 @@ def lib():
             "ve_object_dedup_comm": ([vp, vp, u32, vp, vp, vp], st),
             "ve_snapshot_diff_all_group": ([ctypes.POINTER(vp), u32, u32, vp, vp], st),
             "ve_object_dedup_group": ([ctypes.POINTER(vp), u32, vp, u32, vp, vp], st),
+            "ve_set_units": ([vp, vp, u32, vp, u32], st),
+            "ve_analyze_units": ([vp, vp, u32, vp], st),
         }
         for name, (args, res) in sig.items():
             if os.environ.get("VE_LIB_PATH") and not hasattr(L, name):
@@ -380,6 +387,27 @@ class Context:
         self._keep = keep
         self._check(lib().ve_set_objects(self._h, arr, len(objs)), "ve_set_objects")
         self.n_objects = len(objs)
+
+    def set_units(self, units_objs):
+        """units_objs: one list of object dicts per unit (ids unique over the whole set)."""
+        flat = [o for objs in units_objs for o in objs]
+        arr = (_Object * max(len(flat), 1))()
+        keep = []
+        for i, o in enumerate(flat):
+            arr[i] = _Object(o["base"], o["size"], _ptr(o.get("pre")), _ptr(o.get("post")), o["id"],
+                             o["elem_width"])
+            keep += [o.get("pre"), o.get("post")]
+        cnt = (ctypes.c_uint32 * max(len(units_objs), 1))(*[len(objs) for objs in units_objs])
+        self._keep = keep
+        self._check(lib().ve_set_units(self._h, arr, len(flat), cnt, len(units_objs)), "ve_set_units")
+        self.n_objects = len(flat)
+
+    def analyze_units(self, units, stream=None):
+        """units: (d_records, n, pc_base, n_pcs) per unit, in ve_set_units' order."""
+        arr = (_Unit * max(len(units), 1))()
+        for i, (d, n, pcb, npc) in enumerate(units):
+            arr[i] = _Unit(_ptr(d), n, pcb, npc)
+        self._check(lib().ve_analyze_units(self._h, arr, len(units), _stream(stream)), "ve_analyze_units")
 
     def reset(self):
         self._check(lib().ve_reset(self._h), "ve_reset")
