@@ -746,6 +746,142 @@ def measure_cfg5_records(ve, stream, peak, rank=0, world=1, dev=None, workers=8,
                      "(longest kernel first from a shared queue), CUDA events around the whole, max over ranks"}
 
 
+def measure_cfg5_units(ve, stream, peak, rank=0, world=1, dev=None, batch=250, workers=2):
+    """BASELINE configs[4] (cfg5), records half, batched: the same 4000 independent kernels (10^9 records)
+    analysed `batch` kernels per launch through ve_set_units + ve_analyze_units + one ve_report per batch
+    (each kernel a unit: its own PC keys and objects, exactly as if analysed alone -- tests/test_gpu_units.py),
+    `workers` contexts in host threads on their own streams taking batches from a shared queue.  Records
+    and snapshots are generated on the device first (untimed; every kernel's records 16-byte aligned);
+    the timed region is bracketed by CUDA events (start event waited on by every worker stream, end event
+    after each worker's last work), max over ranks.  Closed forms (tests/cfg5k.py) on every 50th kernel,
+    from its key slice of the batch report."""
+    import threading
+    import torch
+    from gen import vegen as G
+    from tests import cfg5k
+    sp = stream.cuda_stream
+    cfg, seed, K = G.scaled(G.CFG5, 0), 5, 4000
+    infos = [G.info(cfg, k) for k in range(K)]
+    n_all = sum(i["n_records"] for i in infos)
+    owner = ve.lpt_assign([i["n_records"] for i in infos], world)
+    mine = [k for k in range(K) if owner[k] == rank]
+    roff, tot = {}, 0
+    for k in mine:                                  # 16-byte aligned records: even record offsets
+        roff[k] = tot
+        tot += infos[k]["n_records"] + (infos[k]["n_records"] & 1)
+    recs = torch.empty(max(tot, 2) * REC_BYTES, dtype=torch.uint8, device="cuda")
+    objs_of = {k: G.objects(cfg, k) for k in mine}
+    snap_tot = sum(o["size"] for objs in objs_of.values() for o in objs)
+    snaps = torch.empty(2 * snap_tot, dtype=torch.uint8, device="cuda")
+    s0, plan = 0, {}
+    for k in mine:
+        n = infos[k]["n_records"]
+        G.records_device(cfg, k, seed, 0, n, recs.data_ptr() + roff[k] * REC_BYTES, sp)
+        dobjs = []
+        for i, o in enumerate(objs_of[k]):
+            d = {f: o[f] for f in ("base", "size", "id", "elem_width")}
+            for side in ("pre", "post"):
+                t = snaps[s0:s0 + o["size"]]
+                s0 += o["size"]
+                G.snapshot_device(cfg, k, seed, i, side == "post", t.data_ptr(), sp)
+                d[side] = t
+            dobjs.append(d)
+        plan[k] = (recs.data_ptr() + roff[k] * REC_BYTES, n, infos[k]["n_pcs"], dobjs)
+    batches = [mine[i:i + batch] for i in range(0, len(mine), batch)]
+    prep = []
+    for b in batches:                               # per batch: the units' objects (ids shifted) and PC bases
+        uobjs, units, pcb, ob, slices = [], [], 0, 0, {}
+        for k in b:
+            ptr, n, npc, dobjs = plan[k]
+            uobjs.append([dict(d, id=d["id"] + ob) for d in dobjs])
+            units.append((ptr, n, pcb, npc))
+            slices[k] = (pcb, npc, n)
+            pcb += npc
+            ob += len(dobjs)
+        prep.append((uobjs, units, pcb, ob, slices))
+    W = max(1, min(workers, len(prep)))
+    max_pcs = max(p[2] for p in prep)
+    max_obj = max(p[3] for p in prep)
+    streams = [torch.cuda.Stream() for _ in range(W)]
+    ctxs = [ve.Context(n_pcs=max_pcs, max_objects=max_obj, hist_capacity=1 << 25) for _ in range(W)]
+    for w in range(W):                              # warm every context on the last batch (untimed)
+        uobjs, units, _, _, _ = prep[-1]
+        ctxs[w].set_units(uobjs)
+        ctxs[w].analyze_units(units, stream=streams[w].cuda_stream)
+        ctxs[w].report().close()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ends = [torch.cuda.Event() for _ in range(W)]
+    got, errors, nxt, lock = {}, [], [0], threading.Lock()
+    nrec_seen = [0]
+
+    def work(w):
+        ctx, st = ctxs[w], streams[w]
+        try:
+            st.wait_event(a)
+            while True:
+                with lock:
+                    if nxt[0] >= len(prep):
+                        break
+                    j = nxt[0]
+                    nxt[0] += 1
+                uobjs, units, _, _, slices = prep[j]
+                ctx.set_units(uobjs)
+                ctx.analyze_units(units, stream=st.cuda_stream)
+                rep = ctx.report()
+                with lock:
+                    nrec_seen[0] += int(rep.globals["n_records"])
+                for k, (pcb, npc, n) in slices.items():
+                    if k % 50 == 0:
+                        got[k] = ({f: rep.keys[f][pcb:pcb + npc].copy() for f in
+                                   ("n_ld", "n_st", "n_ld_eq_pre", "n_st_eq_pre", "raw_min", "raw_max", "single_zero",
+                                    "single_value")}, n)
+                rep.close()
+            ends[w].record(st)
+        except Exception as e:      # noqa: BLE001  (reported below)
+            errors.append(repr(e))
+            ends[w].record(st)
+
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    a.record(stream)
+    th = [threading.Thread(target=work, args=(w,)) for w in range(W)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    for e in ends:
+        stream.wait_event(e)
+    b.record(stream)
+    torch.cuda.synchronize()
+    if errors:
+        raise RuntimeError("cfg5 units worker failed: " + errors[0])
+    ms = a.elapsed_time(b)
+    if world > 1:
+        ms = max_over_ranks(ms, device=dev)
+    bad, checked = [], 0
+    for k, (keys, nrec) in got.items():
+        bad += cfg5k.check_cfg5_kernel(keys, nrec, cfg, k)
+        checked += 1
+    n_mine = sum(infos[k]["n_records"] for k in mine)
+    if nrec_seen[0] != n_mine:
+        bad.append(f"batch reports counted {nrec_seen[0]} records, expected {n_mine}")
+    for c in ctxs:
+        c.close()
+    del plan, recs, snaps, prep
+    torch.cuda.empty_cache()
+    gbs = n_all * REC_BYTES / (ms / 1e3) / 1e9
+    return {"workload": "cfg5 records: 4000 kernels, 4-64 PCs with cfg1 roles, 1-4 objects, 10^9 records",
+            "kernels": K, "records": n_all, "ranks": world, "this_rank_kernels": len(mine),
+            "partition": "longest-processing-time-first by records (ve.lpt_assign), independent kernels",
+            "mode": f"units: {batch} kernels per ve_analyze_units launch and per report, {W} contexts in host "
+                    "threads on their own streams", "batches": len(prep), "ms": ms,
+            "records_per_s": n_all / (ms / 1e3), "trace_gbs": gbs, "trace_frac_of_hbm_peak": gbs / peak / world,
+            "closed_forms_kernels_checked": checked, "closed_forms_ok": not bad, "closed_form_mismatches": bad[:5],
+            "timed": "set_units + analyze_units + report per batch, CUDA events around the whole, max over ranks"}
+
+
 def measure_e2e(ve, ctx, wl, steps):
     """Same metric through the public API from pinned HOST buffers: every step copies each epoch's records
     (ve_analyze_records_host: two device staging buffers, H2D on a side stream overlapped with the
