@@ -375,6 +375,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-f1", action="store_true")
     ap.add_argument("--no-cfg5", action="store_true")
+    ap.add_argument("--cfg5-mode", default="units", choices=["units", "contexts"],
+                    help="cfg5 records: batched units per launch (default) or one context per kernel x 8 threads")
     ap.add_argument("--no-extra", action="store_true", help="skip the cfg2 / cfg3 lines")
     args = ap.parse_args()
 
@@ -425,7 +427,10 @@ def main():
     if single and not args.no_cfg5:
         dd5 = measure_cfg5_dedup(ve, torch.cuda.current_stream(), peak)
     if not args.no_cfg5:          # every rank: its LPT share of the 4000 kernels (weak-style partition)
-        r5 = measure_cfg5_records(ve, torch.cuda.current_stream(), peak, rank, world, dev)
+        if args.cfg5_mode == "units":
+            r5 = measure_cfg5_units(ve, torch.cuda.current_stream(), peak, rank, world, dev)
+        else:
+            r5 = measure_cfg5_records(ve, torch.cuda.current_stream(), peak, rank, world, dev)
 
     cpu = None
     if not args.no_cpu and single:
@@ -869,6 +874,7 @@ def measure_cfg5_units(ve, stream, peak, rank=0, world=1, dev=None, batch=250, w
         bad.append(f"batch reports counted {nrec_seen[0]} records, expected {n_mine}")
     for c in ctxs:
         c.close()
+    n_batches = len(prep)
     del plan, recs, snaps, prep
     torch.cuda.empty_cache()
     gbs = n_all * REC_BYTES / (ms / 1e3) / 1e9
@@ -876,7 +882,7 @@ def measure_cfg5_units(ve, stream, peak, rank=0, world=1, dev=None, batch=250, w
             "kernels": K, "records": n_all, "ranks": world, "this_rank_kernels": len(mine),
             "partition": "longest-processing-time-first by records (ve.lpt_assign), independent kernels",
             "mode": f"units: {batch} kernels per ve_analyze_units launch and per report, {W} contexts in host "
-                    "threads on their own streams", "batches": len(prep), "ms": ms,
+                    "threads on their own streams", "batches": n_batches, "ms": ms,
             "records_per_s": n_all / (ms / 1e3), "trace_gbs": gbs, "trace_frac_of_hbm_peak": gbs / peak / world,
             "closed_forms_kernels_checked": checked, "closed_forms_ok": not bad, "closed_form_mismatches": bad[:5],
             "timed": "set_units + analyze_units + report per batch, CUDA events around the whole, max over ranks"}
