@@ -294,7 +294,10 @@ __device__ __noinline__ void apply_group(const AnalyzeParams& P, unsigned gm, in
 // lock per window serialises warps on keys that stay collinear.  Each warp keeps
 // the last WC keys' states privately and folds them into the CTA state only on
 // eviction, on the first FAIL (so other warps skip the key early) and at exit.
-constexpr int WC = 4;
+#ifndef VE_WC
+#define VE_WC 4
+#endif
+constexpr int WC = VE_WC;
 struct WarpCache {
   uint32_t key1[WC];   // key + 1, 0 = empty
   int32_t slot[WC];
@@ -2582,6 +2585,16 @@ __global__ void __launch_bounds__(LF_THREADS) k_line_fold(const LineState* lcta,
   }
 }
 
+// Units mode claims UNIT_CHUNK windows at a time: a warp stays on one unit's keys for a while, so
+// its key slots and line-state cache stay warm and few warps merge into one unit's line states at
+// once (16-window chunks spread every unit over every warp: the line-state locks then held 55% of
+// the issued instructions on a 250-kernel cfg5 batch)
+#ifndef VE_UNIT_CHUNK
+#define VE_UNIT_CHUNK 256
+#endif
+constexpr uint32_t UNIT_CHUNK = VE_UNIT_CHUNK;
+static_assert(UNIT_CHUNK % STAGE_WIN == 0, "whole stages");
+
 struct UnitLaunch {           // units mode of one launch (ve_analyze_units)
   const UnitDesc* d_units;
   const uint32_t* d_ucb;
@@ -2658,7 +2671,7 @@ static ve_status launch_analyze_impl(ve_ctx* c, const ve_record* d, uint64_t n, 
   if (blocks == 0) blocks = 1;
   // a trace too short to give every warp a few CHUNK-window chunks (cfg5's kernels: a warp's
   // serial share of a 16-window chunk set a ~0.3 ms floor) is split into one-stage chunks
-  P.chunk = (ul || P.nring >= 4ull * blocks * K1_WARPS * CHUNK) ? CHUNK : (uint32_t)STAGE_WIN;
+  P.chunk = ul ? UNIT_CHUNK : P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? CHUNK : (uint32_t)STAGE_WIN;
   // v2 claims its chunks dynamically (VE_CLAIM_MODE=0/1 forces the static / dynamic split)
   const char* cm = getenv("VE_CLAIM_MODE");
   P.claim = ul ? 1u : (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
@@ -2727,7 +2740,7 @@ extern "C" ve_status ve_analyze_units(ve_ctx* c, const ve_unit* units, uint32_t 
     if ((uint64_t)U.pc_base + U.n_pcs > c->cfg.n_pcs)
       return fail(c, VE_ERR_INVALID, "ve_analyze_units: pc_base + n_pcs above the ctx's n_pcs");
     ud[u] = UnitDesc{U.d_records, U.n, U.pc_base, U.n_pcs, c->unit_obj[u], c->unit_obj[u + 1]};
-    const uint64_t fw = U.n / 32, ch = (fw + CHUNK - 1) / CHUNK;
+    const uint64_t fw = U.n / 32, ch = (fw + UNIT_CHUNK - 1) / UNIT_CHUNK;
     if ((uint64_t)ucb[u] + ch > 0xFFFFFFFFull) return fail(c, VE_ERR_INVALID, "ve_analyze_units: batch too large");
     ucb[u + 1] = ucb[u] + (uint32_t)ch;
     ntot += U.n;
