@@ -970,7 +970,7 @@ __global__ void __launch_bounds__(NT, 1) k_dense_flush(uint32_t* cnt, uint64_t n
         // only an 8-byte element can hold: such values go straight to the global table)
         uint32_t h = (uint32_t)hist_hash(tag, bits) & (ts - 1);
         bool done = false;
-        for (int probe = 0; probe < 8 && !done && bits != ~0ull; ++probe) {
+        for (int probe = 0; probe < 8 && !done && ts && bits != ~0ull; ++probe) {   // (ts 0: direct)
           // look first (a warm table mostly holds the value already), claim only empty slots
           unsigned long long cur = *(volatile unsigned long long*)&sbits[h];
           if (cur == ~0ull) {
@@ -1526,11 +1526,14 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
       const bool post = (ck & DENSE_POST) != 0u;
       uint32_t* arr = (uint32_t*)c->dense_pool + cl[k].off;
       if (mh[k] == 0u || nd[k] > 4096u) {   // mostly unread elements, or many values: per-array flush
+        // (many values: no block table -- it would fill at once and every element would probe it in
+        // vain before its global insert; cfg3's 21 such arrays: see DESIGN 5 "dense flush")
+        const uint32_t ts = nd[k] > 4096u ? 0u : (uint32_t)DF_SLOTS;
         const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
         count_launch();
-        k_dense_flush<DF_THREADS><<<(unsigned)blocks, DF_THREADS, DF_SLOTS * 12, s>>>(
+        k_dense_flush<DF_THREADS><<<(unsigned)blocks, DF_THREADS, ts * 12, s>>>(
             arr, o.n_elems, (const uint8_t*)(post ? o.post : o.pre), o.ew, (pc << 16) | o.id, o.bmoff, c->t, meta,
-            c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id, (uint32_t)DF_SLOTS, (uint32_t)DF_CHUNK, post ? 0u : 1u);
+            c->cfg.mant_bits, pc, c->cfg.n_pcs + o.id, ts, (uint32_t)DF_CHUNK, post ? 0u : 1u);
         continue;
       }
       DoClaim& d = A.c[A.nc++];
