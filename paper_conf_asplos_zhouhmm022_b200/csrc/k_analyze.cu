@@ -54,6 +54,7 @@ struct AnalyzeParams {
   uint64_t nring;           // full windows (streamed through the per-warp rings)
   uint32_t chunk;           // windows per static chunk (VE_CLAIM 2): CHUNK, or one stage for short traces
   uint32_t claim;           // 1: chunks claimed from the global counter *work (guided), 0: static interleave
+  uint64_t nbig;            // claim mode: chunks of P.chunk windows before the one-stage tail chunks
   // units mode (ve_analyze_units, K1 v2 only): independent traces in one launch.  Unit u's records
   // are units[u].recs (16-byte aligned); its PCs are keys pcb .. pcb + npc - 1 (a record's pc is
   // local: pc >= npc is invalid) and its objects the sorted table entries [olo, ohi).  Chunk c of
@@ -703,6 +704,9 @@ __device__ __forceinline__ bool mbar_test(uint32_t bar, uint32_t phase) {
       : "=r"(r) : "r"(bar), "r"(phase) : "memory");
   return r != 0u;
 }
+#ifndef VE_APFAST
+#define VE_APFAST 1           // K1 v2: structured windows that are arithmetic progressions held per slot
+#endif
 #ifndef VE_PF_NEXT
 #define VE_PF_NEXT 0
 #endif
@@ -826,8 +830,12 @@ __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
     unsigned long long c = 0;
     if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
     c = __shfl_sync(0xFFFFFFFFu, c, 0);
+#if VE_NBIG_DEV
     const uint64_t nbig = (P.nring - P.nring / 8) / P.chunk;
-    if (c < nbig) { w0 = (uint64_t)c * P.chunk; len = P.chunk; }
+#else
+    const uint64_t nbig = P.nbig;           // (host-computed: a 64-bit division per claim cost ~12
+#endif
+    if (c < nbig) { w0 = (uint64_t)c * P.chunk; len = P.chunk; }   //  instructions per window on cfg4)
     else { w0 = nbig * P.chunk + (uint64_t)(c - nbig) * CHUNK_TAIL; len = CHUNK_TAIL; }
   }
   if (w0 < P.nring) {
@@ -1911,9 +1919,16 @@ __global__ void __launch_bounds__(K1_THREADS, 1) k_analyze(const __grid_constant
 // else (slow windows, S8 inserts, line states, dense counters) is shared with v1.
 // ============================================================================
 constexpr int NS2 = 32;
-struct SlotLine {            // deferred C8 constant segment of slot s (see SlotE::cy)
+// deferred C8 state of slot s, merged into the key's line states on eviction / FAIL / exit (the (+)
+// monoid is associative and commutative, so this equals merging every window): cpend 1: a run of one
+// value (raw bits cy) between addresses cx0 and cx1 (SlotE::cy); cpend 2: a POINT / LINE segment
+// st from (cx0, (int64) cy) to (cx1, y1), |y| < 2^62 -- the windows of a structured key whose 32
+// points are an arithmetic progression in address and value (cfg4's xc[x]: ~960 instructions per
+// window through the generic fit and two cache merges)
+struct SlotLine {
   uint64_t cy, cx0, cx1;
-  uint32_t cpend, pad;
+  int64_t y1;
+  uint32_t cpend, st;
 };
 struct SlotRec {             // slot s's object and arrays (per warp, shared memory; read by every lane)
   uint64_t cb, clim, cpre, cpost, cbm;
@@ -1989,9 +2004,18 @@ __device__ __noinline__ void lslot_fold(const AnalyzeParams& P, const SlotSave* 
 // merge slot v's deferred constant segment into the line states (all lanes); returns the new FAIL bits
 __device__ __noinline__ uint32_t sl_flush(const AnalyzeParams& P, WarpCache& wc, SlotLine* sl, int v, uint64_t key,
                                           uint32_t lf) {
-  if (!sl[v].cpend) return lf;
-  const uint32_t nlf = const_line(P, wc, sl[v].cx0, sl[v].cx1, sl[v].cy, (uint32_t)(key >> 32), (uint32_t)key & 0xFFFFu,
-                                  (uint32_t)(key >> 16) & 0xFFFFu, lf);
+  const uint32_t cp = sl[v].cpend;
+  if (!cp) return lf;
+  uint32_t nlf;
+  if (cp == 1u) {
+    nlf = const_line(P, wc, sl[v].cx0, sl[v].cx1, sl[v].cy, (uint32_t)(key >> 32), (uint32_t)key & 0xFFFFu,
+                     (uint32_t)(key >> 16) & 0xFFFFu, lf);
+  } else {
+    LinePts g;
+    g.state = sl[v].st; g.px = sl[v].cx0; g.qx = sl[v].cx1;
+    g.py = (__int128)(int64_t)sl[v].cy; g.qy = (__int128)sl[v].y1;
+    nlf = line_apply(P, wc, g, (uint32_t)key & 0xFFFFu, (uint32_t)(key >> 16) & 0xFFFFu, lf);
+  }
   __syncwarp();
   if ((threadIdx.x & 31) == 0) sl[v].cpend = 0;
   __syncwarp();
@@ -2022,14 +2046,70 @@ __device__ __noinline__ unsigned long long lslot_prepare(const AnalyzeParams& P,
 __device__ __noinline__ uint32_t win_line(const AnalyzeParams& P, WarpCache& wc, SlotLine* sl, int s, uint64_t key,
                                           uint32_t lf, uint64_t addr, uint64_t val) {
   const unsigned FULL = 0xFFFFFFFFu;
+  const int lane = threadIdx.x & 31;
   const uint32_t pc0 = (uint32_t)key & 0xFFFFu, koi0 = (uint32_t)(key >> 16) & 0xFFFFu, meta0 = (uint32_t)(key >> 32);
   const uint64_t cy = shfl64(FULL, val, 0);
+  SlotLine& e = sl[s];
+#if !VE_APFAST
   if (!__all_sync(FULL, val == cy)) return fast_line(P, wc, addr, val, meta0, pc0, koi0, lf);
+#endif
+  if (!__all_sync(FULL, val == cy)) {
+    // an arithmetic-progression window (lane i at a0 + i*w with value y0 + i*dy, exact integers
+    // |y| < 2^62) is the segment of its end points; merged into the held segment by lane 0
+    const uint32_t kind = (meta0 >> 2) & 3u, lg = meta0 & 3u;
+    int64_t y = 0;
+    bool ok = false;
+    if (kind == 0u) { y = (int64_t)val; ok = val < (1ull << 62); }
+    else if (kind == 1u) {
+      const uint32_t sh64 = 64u - (8u << lg);
+      y = (int64_t)(val << sh64) >> sh64;
+      ok = y > -(1ll << 62) && y < (1ll << 62);
+    } else if (kind == 2u && lg >= 2u) {
+      const double d = lg == 3u ? __longlong_as_double((long long)val) : (double)__uint_as_float((uint32_t)val);
+      // an exact integer below 2^62 (NaN, inf and fractions fail) and not -0.0, which the line fit
+      // does not admit (DESIGN 3, Q11-Q13; float_flags): such windows take the generic path
+      const bool negz = val == (lg == 3u ? 0x8000000000000000ull : 0x80000000ull);
+      ok = !negz && d == trunc(d) && fabs(d) < 4611686018427387904.0;
+      y = ok ? (int64_t)d : 0;
+    }
+    const uint64_t a0 = shfl64(FULL, addr, 0);
+    const int64_t y0 = (int64_t)shfl64(FULL, (uint64_t)y, 0), dy = (int64_t)shfl64(FULL, (uint64_t)y, 1) - y0;
+    const bool dok = dy > -(1ll << 56) && dy < (1ll << 56);
+    if (!__all_sync(FULL, ok && dok && addr == a0 + ((uint64_t)lane << lg) && y == y0 + (int64_t)lane * dy))
+      return fast_line(P, wc, addr, val, meta0, pc0, koi0, lf);
+    LinePts g;
+    g.state = VE_LINE_LINE;
+    g.px = a0; g.py = (__int128)y0;
+    g.qx = a0 + (31ull << lg); g.qy = (__int128)(y0 + 31 * dy);
+    if (e.cpend == 1u) lf = sl_flush(P, wc, sl, s, key, lf);   // (a held run of one value goes first)
+    uint32_t st = 0;
+    __syncwarp();
+    if (lane == 0) {
+      LinePts r = g;
+      if (e.cpend == 2u) {
+        LinePts a;
+        a.state = e.st; a.px = e.cx0; a.qx = e.cx1; a.py = (__int128)(int64_t)e.cy; a.qy = (__int128)e.y1;
+        r = line_merge(a, g);
+      }
+      st = r.state;
+      if (st != VE_LINE_FAIL) {
+        e.st = r.state; e.cx0 = r.px; e.cx1 = r.qx; e.cy = (uint64_t)(int64_t)r.py; e.y1 = (int64_t)r.qy; e.cpend = 2u;
+      } else {
+        e.cpend = 0u;
+      }
+    }
+    st = __shfl_sync(FULL, st, 0);
+    __syncwarp();
+    if (st == VE_LINE_FAIL) {            // the slot's points are not collinear: publish the FAIL now
+      g.state = VE_LINE_FAIL;
+      return line_apply(P, wc, g, pc0, koi0, lf);
+    }
+    return lf;
+  }
   // a window of one value: its points lie on y = cy between its extreme addresses; consecutive
   // windows of one value only widen a held segment (the (+) monoid keeps the extreme points)
   const uint64_t xmin = redmin64(FULL, addr), xmax = redmax64(FULL, addr);
-  SlotLine& e = sl[s];
-  if (e.cpend && e.cy == cy) {
+  if (e.cpend == 1u && e.cy == cy) {
     __syncwarp();
     if ((threadIdx.x & 31) == 0) {
       e.cx0 = xmin < e.cx0 ? xmin : e.cx0;
@@ -2181,6 +2261,7 @@ __device__ __noinline__ unsigned long long post_claim(const AnalyzeParams& P, in
 #ifndef VE_DIAG
 #define VE_DIAG 0
 #endif
+
 #ifndef VE_K2_THREADS
 #define VE_K2_THREADS 384
 #endif
@@ -2675,6 +2756,7 @@ static ve_status launch_analyze_impl(ve_ctx* c, const ve_record* d, uint64_t n, 
   // v2 claims its chunks dynamically (VE_CLAIM_MODE=0/1 forces the static / dynamic split)
   const char* cm = getenv("VE_CLAIM_MODE");
   P.claim = ul ? 1u : (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
+  P.nbig = (P.nring - P.nring / 8) / P.chunk;
   // staging regions: a warp stages at most one group per record of its static range
   {
     const uint64_t tw = blocks * K1_WARPS;

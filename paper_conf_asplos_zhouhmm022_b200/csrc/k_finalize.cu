@@ -1528,7 +1528,10 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
       if (mh[k] == 0u || nd[k] > 4096u) {   // mostly unread elements, or many values: per-array flush
         // (many values: no block table -- it would fill at once and every element would probe it in
         // vain before its global insert; cfg3's 21 such arrays: see DESIGN 5 "dense flush")
-        const uint32_t ts = nd[k] > 4096u ? 0u : (uint32_t)DF_SLOTS;
+#ifndef VE_DF_DIRECT
+#define VE_DF_DIRECT 1
+#endif
+        const uint32_t ts = (VE_DF_DIRECT && nd[k] > 4096u) ? 0u : (uint32_t)DF_SLOTS;
         const uint64_t blocks = (o.n_elems + DF_CHUNK - 1) / DF_CHUNK;
         count_launch();
         k_dense_flush<DF_THREADS><<<(unsigned)blocks, DF_THREADS, ts * 12, s>>>(
