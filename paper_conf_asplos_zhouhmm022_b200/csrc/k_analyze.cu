@@ -1925,11 +1925,24 @@ constexpr int NS2 = 32;
 // st from (cx0, (int64) cy) to (cx1, y1), |y| < 2^62 -- the windows of a structured key whose 32
 // points are an arithmetic progression in address and value (cfg4's xc[x]: ~960 instructions per
 // window through the generic fit and two cache merges)
+// (32 bytes: the flags ride in the top bits of the < 2^48 addresses -- a 40-byte record cost epoch 0
+// of cfg4 over a millisecond)
+constexpr uint64_t SL_XM = (1ull << 48) - 1ull;
 struct SlotLine {
-  uint64_t cy, cx0, cx1;
+  uint64_t cy;            // cpend 1: the run's raw bits; cpend 2: (int64) y of the first end point
+  uint64_t w0, w1;        // bits 0-47: cx0 / cx1; bits 62-63 of w0: cpend, of w1: the segment's state
   int64_t y1;
-  uint32_t cpend, st;
+  __device__ __forceinline__ uint32_t cpend() const { return (uint32_t)(w0 >> 62); }
+  __device__ __forceinline__ uint32_t st() const { return (uint32_t)(w1 >> 62); }
+  __device__ __forceinline__ uint64_t cx0() const { return w0 & SL_XM; }
+  __device__ __forceinline__ uint64_t cx1() const { return w1 & SL_XM; }
+  __device__ __forceinline__ void set(uint32_t pend, uint32_t state, uint64_t x0, uint64_t x1) {
+    w0 = x0 | ((uint64_t)pend << 62);
+    w1 = x1 | ((uint64_t)state << 62);
+  }
+  __device__ __forceinline__ void clear() { w0 &= SL_XM; }
 };
+static_assert(sizeof(SlotLine) == 32, "SlotLine layout");
 struct SlotRec {             // slot s's object and arrays (per warp, shared memory; read by every lane)
   uint64_t cb, clim, cpre, cpost, cbm;
   unsigned long long dn, dq;
@@ -2004,20 +2017,20 @@ __device__ __noinline__ void lslot_fold(const AnalyzeParams& P, const SlotSave* 
 // merge slot v's deferred constant segment into the line states (all lanes); returns the new FAIL bits
 __device__ __noinline__ uint32_t sl_flush(const AnalyzeParams& P, WarpCache& wc, SlotLine* sl, int v, uint64_t key,
                                           uint32_t lf) {
-  const uint32_t cp = sl[v].cpend;
+  const uint32_t cp = sl[v].cpend();
   if (!cp) return lf;
   uint32_t nlf;
   if (cp == 1u) {
-    nlf = const_line(P, wc, sl[v].cx0, sl[v].cx1, sl[v].cy, (uint32_t)(key >> 32), (uint32_t)key & 0xFFFFu,
+    nlf = const_line(P, wc, sl[v].cx0(), sl[v].cx1(), sl[v].cy, (uint32_t)(key >> 32), (uint32_t)key & 0xFFFFu,
                      (uint32_t)(key >> 16) & 0xFFFFu, lf);
   } else {
     LinePts g;
-    g.state = sl[v].st; g.px = sl[v].cx0; g.qx = sl[v].cx1;
+    g.state = sl[v].st(); g.px = sl[v].cx0(); g.qx = sl[v].cx1();
     g.py = (__int128)(int64_t)sl[v].cy; g.qy = (__int128)sl[v].y1;
     nlf = line_apply(P, wc, g, (uint32_t)key & 0xFFFFu, (uint32_t)(key >> 16) & 0xFFFFu, lf);
   }
   __syncwarp();
-  if ((threadIdx.x & 31) == 0) sl[v].cpend = 0;
+  if ((threadIdx.x & 31) == 0) sl[v].clear();
   __syncwarp();
   return nlf;
 }
@@ -2037,7 +2050,7 @@ __device__ __noinline__ unsigned long long lslot_prepare(const AnalyzeParams& P,
   (void)postok;
   *dq = 0ull;   // a post array is claimed on demand (win_fast), so keys counted against pre use no slot
   __syncwarp();
-  if ((threadIdx.x & 31) == 0) sl[v].cpend = 0;
+  if ((threadIdx.x & 31) == 0) sl[v].clear();
   __syncwarp();
   return dn;
 }
@@ -2081,21 +2094,21 @@ __device__ __noinline__ uint32_t win_line(const AnalyzeParams& P, WarpCache& wc,
     g.state = VE_LINE_LINE;
     g.px = a0; g.py = (__int128)y0;
     g.qx = a0 + (31ull << lg); g.qy = (__int128)(y0 + 31 * dy);
-    if (e.cpend == 1u) lf = sl_flush(P, wc, sl, s, key, lf);   // (a held run of one value goes first)
+    if (e.cpend() == 1u) lf = sl_flush(P, wc, sl, s, key, lf);   // (a held run of one value goes first)
     uint32_t st = 0;
     __syncwarp();
     if (lane == 0) {
       LinePts r = g;
-      if (e.cpend == 2u) {
+      if (e.cpend() == 2u) {
         LinePts a;
-        a.state = e.st; a.px = e.cx0; a.qx = e.cx1; a.py = (__int128)(int64_t)e.cy; a.qy = (__int128)e.y1;
+        a.state = e.st(); a.px = e.cx0(); a.qx = e.cx1(); a.py = (__int128)(int64_t)e.cy; a.qy = (__int128)e.y1;
         r = line_merge(a, g);
       }
       st = r.state;
       if (st != VE_LINE_FAIL) {
-        e.st = r.state; e.cx0 = r.px; e.cx1 = r.qx; e.cy = (uint64_t)(int64_t)r.py; e.y1 = (int64_t)r.qy; e.cpend = 2u;
+        e.set(2u, r.state, r.px, r.qx); e.cy = (uint64_t)(int64_t)r.py; e.y1 = (int64_t)r.qy;
       } else {
-        e.cpend = 0u;
+        e.clear();
       }
     }
     st = __shfl_sync(FULL, st, 0);
@@ -2109,17 +2122,17 @@ __device__ __noinline__ uint32_t win_line(const AnalyzeParams& P, WarpCache& wc,
   // a window of one value: its points lie on y = cy between its extreme addresses; consecutive
   // windows of one value only widen a held segment (the (+) monoid keeps the extreme points)
   const uint64_t xmin = redmin64(FULL, addr), xmax = redmax64(FULL, addr);
-  if (e.cpend == 1u && e.cy == cy) {
+  if (e.cpend() == 1u && e.cy == cy) {
     __syncwarp();
     if ((threadIdx.x & 31) == 0) {
-      e.cx0 = xmin < e.cx0 ? xmin : e.cx0;
-      e.cx1 = xmax > e.cx1 ? xmax : e.cx1;
+      const uint64_t x0 = e.cx0(), x1 = e.cx1();
+      e.set(1u, 0u, xmin < x0 ? xmin : x0, xmax > x1 ? xmax : x1);
     }
     __syncwarp();
     return lf;
   }
   lf = sl_flush(P, wc, sl, s, key, lf);
-  if (lf != 3u && (threadIdx.x & 31) == 0) { e.cpend = 1; e.cy = cy; e.cx0 = xmin; e.cx1 = xmax; }
+  if (lf != 3u && (threadIdx.x & 31) == 0) { e.set(1u, 0u, xmin, xmax); e.cy = cy; }
   __syncwarp();
   return lf;
 }
@@ -2292,7 +2305,7 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   WarpCache& wc = s_wc[warp];
   SlotLine* sl = s_sl[warp];
   if (lane < WC) wc.key1[lane] = 0;
-  sl[lane].cpend = 0;
+  sl[lane].w0 = 0;
   if (lane == 0) { wc.next = 0; s_stage_n[warp] = 0; }
   LaneSlot L;
   L.key = ~0ull; L.pmw = ~0ull; L.ob = 1; L.olim = 0; L.dn = 0; L.dq = 0; L.info = 0;
