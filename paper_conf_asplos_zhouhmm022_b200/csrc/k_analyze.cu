@@ -2689,6 +2689,13 @@ __global__ void __launch_bounds__(LF_THREADS) k_line_fold(const LineState* lcta,
 constexpr uint32_t UNIT_CHUNK = VE_UNIT_CHUNK;
 static_assert(UNIT_CHUNK % STAGE_WIN == 0, "whole stages");
 
+// v2's claims on long traces (a claim is one atomic on one global counter from every warp)
+#ifndef VE_V2_CHUNK
+#define VE_V2_CHUNK 64
+#endif
+constexpr uint32_t V2_CHUNK = VE_V2_CHUNK;
+static_assert(V2_CHUNK % STAGE_WIN == 0, "whole stages");
+
 struct UnitLaunch {           // units mode of one launch (ve_analyze_units)
   const UnitDesc* d_units;
   const uint32_t* d_ucb;
@@ -2765,7 +2772,7 @@ static ve_status launch_analyze_impl(ve_ctx* c, const ve_record* d, uint64_t n, 
   if (blocks == 0) blocks = 1;
   // a trace too short to give every warp a few CHUNK-window chunks (cfg5's kernels: a warp's
   // serial share of a 16-window chunk set a ~0.3 ms floor) is split into one-stage chunks
-  P.chunk = ul ? UNIT_CHUNK : P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? CHUNK : (uint32_t)STAGE_WIN;
+  P.chunk = ul ? UNIT_CHUNK : P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? (v2 ? V2_CHUNK : CHUNK) : (uint32_t)STAGE_WIN;
   // v2 claims its chunks dynamically (VE_CLAIM_MODE=0/1 forces the static / dynamic split)
   const char* cm = getenv("VE_CLAIM_MODE");
   P.claim = ul ? 1u : (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
