@@ -1290,6 +1290,9 @@ __device__ __forceinline__ long long gt_get(const DoSlot* gt, uint32_t mask, uin
 // (round 2's version drained it every few chunks -- 7 x 4096 contended HBM inserts per drain --
 // and checked its fill under a barrier every 8 batches: 20.6% of its stall samples).  The counters
 // are left as they are (zeroed by a memset after the emission, or by the fallback flush).
+// NC: the claims' loops run NC iterations (an instantiation per bound: a single-claim object -- T_out's
+// post values, vol, a -- does not pay for eight predicated iterations per element)
+template <int NC>
 __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_constant__ DoArgs A, DevTables t, DoSlot* gt,
                                                              uint32_t gmask, uint32_t* ovf) {
   extern __shared__ __align__(16) uint8_t do_smem[];
@@ -1306,13 +1309,13 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
     const uint64_t lo = ch * DO_CH, hi = lo + DO_CH < A.ne ? lo + DO_CH : A.ne;
     // the loads of a batch (the counters of all claims, the snapshot sides) are issued one batch
     // ahead, so they are in flight while the previous batch is inserted
-    uint32_t ncj[DO_MAXC];
+    uint32_t ncj[NC];
     uint64_t nsv0 = 0, nsv1 = 0;
     auto issue = [&](uint64_t b) {
       const uint64_t e = b + tid;
       const bool in = e < hi;
 #pragma unroll
-      for (int j = 0; j < DO_MAXC; ++j) ncj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
+      for (int j = 0; j < NC; ++j) ncj[j] = ((uint32_t)j < A.nc && in) ? __ldcs(A.c[j].cnt + e) : 0u;
       nsv0 = (in && A.snap[0]) ? do_load(A.snap[0] + e * A.ew, A.ew) : 0ull;
       nsv1 = (in && A.snap[1]) ? do_load(A.snap[1] + e * A.ew, A.ew) : 0ull;
     };
@@ -1320,15 +1323,15 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
     for (uint64_t base = lo; base < hi; base += DO_THREADS) {
       const uint64_t e = base + tid;
       const bool in = e < hi;
-      uint32_t cj[DO_MAXC];
+      uint32_t cj[NC];
 #pragma unroll
-      for (int j = 0; j < DO_MAXC; ++j) cj[j] = ncj[j];
+      for (int j = 0; j < NC; ++j) cj[j] = ncj[j];
       const uint64_t sv0 = nsv0, sv1 = nsv1;
       if (base + DO_THREADS < hi) issue(base + DO_THREADS);
       uint32_t corr = 0;                               // claims whose count differs from their base
       bool lbit = false;
 #pragma unroll
-      for (int j = 0; j < DO_MAXC; ++j) {
+      for (int j = 0; j < NC; ++j) {
         if ((uint32_t)j >= A.nc) break;
         if (cj[j] && A.c[j].side == 0u) lbit = true;
         if (in && cj[j] != A.c[j].m) corr |= 1u << j;
@@ -1366,7 +1369,7 @@ __global__ void __launch_bounds__(DO_THREADS, 1) k_dense_obj(const __grid_consta
       }
       if (__any_sync(0xFFFFFFFFu, corr != 0u)) {       // (stencils: only at their faces)
 #pragma unroll
-        for (int j = 0; j < DO_MAXC; ++j) {
+        for (int j = 0; j < NC; ++j) {
           if ((uint32_t)j >= A.nc) break;
           const bool act = (corr >> j) & 1u;
           const unsigned am = __ballot_sync(0xFFFFFFFFu, act);
@@ -1507,7 +1510,9 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(c, e, "k_dense_mode");
   const size_t smem = (size_t)DO_TS * sizeof(DoSlot);
-  cudaFuncSetAttribute(k_dense_obj, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(k_dense_obj<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(k_dense_obj<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(k_dense_obj<DO_MAXC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   cudaFuncSetAttribute(k_dense_flush<DF_THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(DF_SLOTS * 12));
   // per object: its claims for the fused flush (others: the per-array flush right away)
   std::vector<DoArgs> objargs;
@@ -1585,7 +1590,9 @@ ve_status dense_flush(ve_ctx* c, cudaStream_t s) {
       if (blocks > (uint64_t)c->num_sms) blocks = (uint64_t)c->num_sms;
       if (blocks == 0) blocks = 1;
       count_launch();
-      k_dense_obj<<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t, gt, objmask[q], ovf);
+      if (A.nc <= 1) k_dense_obj<1><<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t, gt, objmask[q], ovf);
+      else if (A.nc <= 4) k_dense_obj<4><<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t, gt, objmask[q], ovf);
+      else k_dense_obj<DO_MAXC><<<(unsigned)blocks, DO_THREADS, smem, s>>>(A, c->t, gt, objmask[q], ovf);
       uint64_t eb = ((uint64_t)objmask[q] + 1) / 256;
       eb = std::max<uint64_t>(1, std::min<uint64_t>(eb, 4ull * c->num_sms));
       count_launch();
