@@ -2443,8 +2443,13 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
       if (s != ls) {
         ls = s;
         const SlotRec& r = sr[s];
-        cb = r.cb; clim = r.clim; cpre = r.cpre; cpost = r.cpost; cbm = r.cbm; ldn = r.dn; ldq = r.dq;
-        cid = r.cidlg & 0xFFFFu; coi = (int)r.coi; clg = r.cidlg >> 16;
+        // the object registers are reloaded only when the slot's object differs (a stencil's PCs
+        // alternate over one object: their slots differ in their arrays alone)
+        if ((int)r.coi != coi) {
+          cb = r.cb; clim = r.clim; cpre = r.cpre; cpost = r.cpost; cbm = r.cbm;
+          cid = r.cidlg & 0xFFFFu; coi = (int)r.coi; clg = r.cidlg >> 16;
+        }
+        ldn = r.dn; ldq = r.dq;
         kkey = ((uint64_t)(uint32_t)(pm0 >> 32) << 32) | ((uint64_t)cid << 16) | (uint32_t)pm0;
         klg = (uint32_t)(pm0 >> 32) & 3u;
         kwm = (1u << klg) - 1u;
