@@ -348,7 +348,10 @@ def roofline_block(res, world, peak, peak_src, traffic):
     t = sum(res["an_ms"]) / 1e3
     achieved = alg / t / 1e9
     return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": traffic, "kernel": "k_analyze2 / k_analyze (every epoch's ve_analyze_records)",
+            "traffic": traffic,
+            "traffic_source": ("ncu --set full capture of this command's timed step (scripts/r2_final.sh), "
+                               "profiles/r02_k_analyze_traffic.json; per launch, bytes moved" if traffic else None),
+            "kernel": "k_analyze2 / k_analyze (every epoch's ve_analyze_records)",
             "peak_source": peak_src, "ms_per_launch": [round(x, 4) for x in res["an_ms"]],
             "alg_bytes_per_launch": [b / world for b in wl.alg_bytes_epoch],
             "alg_bytes_rule": "24 B per record + element width x U (distinct pre-snapshot elements referenced)"}
@@ -356,7 +359,7 @@ def roofline_block(res, world, peak, peak_src, traffic):
 
 def traffic_of(name):
     """dram__bytes_read.sum + dram__bytes_write.sum per analyze launch (the step's epochs), from the committed
-    ncu --set full capture of the same command (profiles/r02_k_analyze_traffic.json, scripts/r2_bench_prof.sh):
+    ncu --set full capture of the same command (profiles/r02_k_analyze_traffic.json, scripts/r2_final.sh):
     a list per epoch, or None when no capture exists for the configuration."""
     prof = os.path.join(ROOT, "profiles", "r02_k_analyze_traffic.json")
     try:
