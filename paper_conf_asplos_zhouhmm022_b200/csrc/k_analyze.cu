@@ -2421,10 +2421,24 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
     __syncwarp();
     coi = -1; cb = 1; clim = 0; clg = 0xFFu; ls = -1;   // the object registers belong to the last unit
   };
+  // the ring is consumed a stage at a time: one refill and one barrier wait per stage, then its
+  // windows in a loop (ring_next's per-window bookkeeping cost ~40 instructions per window)
   while (R.left) {
-    uint64_t addr, val, pm;
+    if (R.pend) {
+      __syncwarp();
+      ring_issue_stage(P, R, R.pend - 1u);
+      R.pend = 0;
+    }
     const uint32_t wd = R.d;
-    ring_next(P, R, addr, val, pm);
+    ring_wait(R.bar0 + wd * 8u, R.ph);
+    const uint32_t nws = (R.snw >> (4u * wd)) & 0xFu;
+    const uint32_t sbase = R.o0 + wd * STAGE_BYTES;
+    for (uint32_t wj = 0; wj < nws; ++wj) {
+    uint64_t addr, val, pm;
+    asm volatile("ld.shared.u64 %0, [%3];\n\tld.shared.u64 %1, [%3+8];\n\tld.shared.u64 %2, [%3+16];"
+                 : "=l"(addr), "=l"(val), "=l"(pm)
+                 : "r"(sbase + wj * WIN_BYTES)
+                 : "memory");
     if constexpr (UNITS) {                     // a local pc -> the unit's key; out of range -> invalid
       const uint32_t u = (R.su >> (16u * wd)) & 0xFFFFu;
       if (u != cu) unit_enter(u);
@@ -2556,6 +2570,12 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
         if (lane == s) L.info = (L.info & ~3u) | nlf;
       }
     }
+    }   // the stage's windows
+    R.left -= nws;
+    R.pend = R.iss ? wd + 1u : 0u;     // refilled at the next stage's start (its windows are all done)
+    if (++R.d == (uint32_t)NSTAGE) { R.d = 0; R.ph ^= 1u; }
+    R.o = R.o0 + R.d * STAGE_BYTES;
+    R.sw = 0;
   }
 #if VE_DIAG == 2
   if (dsink == 0x123456789ull) P.t.glob[G_WORK] = dsink;
