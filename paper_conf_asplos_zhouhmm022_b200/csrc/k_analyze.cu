@@ -796,9 +796,12 @@ struct Ring {
 // CHUNK-window chunks cover the first 7/8 of the trace, then chunks of one stage, so
 // the warps finish together even where windows differ much in cost.
 constexpr uint32_t CHUNK_TAIL = STAGE_WIN;
+// MODE: 0 any split (v1: P.claim / P.units at run time), 1 dynamic claims only (v2), 2 units only
+// (v2 units mode) -- the v2 instantiations carry no code or registers of the splits they never use
+template <int MODE = 0>
 __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
   uint64_t w0, len;
-  if (P.units) {
+  if (MODE == 2 || (MODE == 0 && P.units)) {
     // a dynamic claim; its unit by binary search over the chunk prefix (warp-uniform)
     unsigned long long c = 0;
     if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
@@ -817,7 +820,7 @@ __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
     R.cu = lo;
     return;
   }
-  if (!P.claim) {
+  if (MODE == 0 && !P.claim) {
     // static interleave: chunk c goes to warp c mod (all warps); no atomics, and every
     // warp sees the same mix of the trace
     w0 = R.nextc * P.chunk;
@@ -846,6 +849,7 @@ __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
   }
 }
 
+template <int MODE = 0>
 __device__ __forceinline__ void ring_issue_stage(const AnalyzeParams& P, Ring& R, uint32_t d) {
   const uint32_t nw = R.iss < (uint32_t)STAGE_WIN ? R.iss : (uint32_t)STAGE_WIN;
   if (nw == 0u) return;
@@ -856,7 +860,7 @@ __device__ __forceinline__ void ring_issue_stage(const AnalyzeParams& P, Ring& R
   R.iss -= nw;
   R.left += nw;
 #if VE_CLAIM
-  if (R.iss == 0u) ring_claim(P, R);
+  if (R.iss == 0u) ring_claim<MODE>(P, R);
 #endif
 }
 
@@ -2342,8 +2346,8 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   __syncwarp();
   R.nextc = P.chunk == CHUNK ? (uint64_t)blockIdx.x * K2_WARPS + warp : (uint64_t)warp * gridDim.x + blockIdx.x;
   R.cstride = gridDim.x * K2_WARPS;
-  ring_claim(P, R);
-  for (int d = 0; d < NSTAGE; ++d) ring_issue_stage(P, R, (uint32_t)d);
+  ring_claim<UNITS ? 2 : 1>(P, R);
+  for (int d = 0; d < NSTAGE; ++d) ring_issue_stage<UNITS ? 2 : 1>(P, R, (uint32_t)d);
   __syncthreads();
 
   // the current object (warp-uniform): offsets [0, clim] hold a whole element
@@ -2426,7 +2430,7 @@ __global__ void __launch_bounds__(K2_THREADS, 1) k_analyze2(const __grid_constan
   while (R.left) {
     if (R.pend) {
       __syncwarp();
-      ring_issue_stage(P, R, R.pend - 1u);
+      ring_issue_stage<UNITS ? 2 : 1>(P, R, R.pend - 1u);
       R.pend = 0;
     }
     const uint32_t wd = R.d;
@@ -2798,9 +2802,9 @@ static ve_status launch_analyze_impl(ve_ctx* c, const ve_record* d, uint64_t n, 
   // a trace too short to give every warp a few CHUNK-window chunks (cfg5's kernels: a warp's
   // serial share of a 16-window chunk set a ~0.3 ms floor) is split into one-stage chunks
   P.chunk = ul ? UNIT_CHUNK : P.nring >= 4ull * blocks * K1_WARPS * CHUNK ? (v2 ? V2_CHUNK : CHUNK) : (uint32_t)STAGE_WIN;
-  // v2 claims its chunks dynamically (VE_CLAIM_MODE=0/1 forces the static / dynamic split)
+  // v2 claims its chunks dynamically; v1 splits statically (VE_CLAIM_MODE=1: dynamic claims for v1)
   const char* cm = getenv("VE_CLAIM_MODE");
-  P.claim = ul ? 1u : (cm && *cm) ? (*cm == '1' ? 1u : 0u) : (v2 ? 1u : 0u);
+  P.claim = (ul || v2) ? 1u : (cm && *cm && *cm == '1') ? 1u : 0u;   // (v2: always dynamic)
   P.nbig = (P.nring - P.nring / 8) / P.chunk;
   // staging regions: a warp stages at most one group per record of its static range
   {
