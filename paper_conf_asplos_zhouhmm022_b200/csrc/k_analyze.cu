@@ -833,11 +833,7 @@ __device__ __forceinline__ void ring_claim(const AnalyzeParams& P, Ring& R) {
     unsigned long long c = 0;
     if ((threadIdx.x & 31) == 0) c = atomicAdd(P.work, 1ull);
     c = __shfl_sync(0xFFFFFFFFu, c, 0);
-#if VE_NBIG_DEV
-    const uint64_t nbig = (P.nring - P.nring / 8) / P.chunk;
-#else
     const uint64_t nbig = P.nbig;           // (host-computed: a 64-bit division per claim cost ~12
-#endif
     if (c < nbig) { w0 = (uint64_t)c * P.chunk; len = P.chunk; }   //  instructions per window on cfg4)
     else { w0 = nbig * P.chunk + (uint64_t)(c - nbig) * CHUNK_TAIL; len = CHUNK_TAIL; }
   }
